@@ -1,0 +1,154 @@
+"""Cost-model oracle pinned to the paper's printed tables (CPU only).
+
+Golden fixtures (tests/golden/) are transcriptions of PAPER.md Table IV
+(L230–249) and Table VI (L272–283).
+"""
+import os
+import random
+import re
+
+import pytest
+
+from oracle import cost_model as cm
+from oracle import redistribution as rd
+
+GOLD = os.path.join(os.path.dirname(__file__), "golden")
+_VAR = {"f_in": "fin", "f_h": "fh", "f_out": "fout", "min(f_in,f_h)": "m1", "min(f_h,f_out)": "m2"}
+
+
+def _parse(expr):
+    co = dict(fin=0, fh=0, fout=0, m1=0, m2=0)
+    for t in expr.split("+"):
+        m = re.fullmatch(r"(\d*)(f_in|f_h|f_out|min\(f_in,f_h\)|min\(f_h,f_out\))", t.replace(" ", ""))
+        assert m, t
+        co[_VAR[m.group(2)]] += int(m.group(1) or 1)
+    return co
+
+
+def _eval(co, fin, fh, fout):
+    return (co["fin"] * fin + co["fh"] * fh + co["fout"] * fout + co["m1"] * min(fin, fh)
+            + co["m2"] * min(fh, fout))
+
+
+def _table_iv():
+    rows = {}
+    for line in open(os.path.join(GOLD, "table_iv.txt")):
+        if line.startswith("#") or not line.strip():
+            continue
+        i, c, s = [x.strip() for x in line.split("|")]
+        rows[int(i)] = (_parse(c), _parse(s))
+    return rows
+
+
+def _table_vi():
+    out = []
+    for line in open(os.path.join(GOLD, "table_vi.txt")):
+        if line.startswith("#") or not line.strip():
+            continue
+        d, a, b, c, ids = [x.strip() for x in line.split("|")]
+        out.append((d, (int(a), int(b), int(c)), sorted(int(x) for x in ids.split())))
+    return out
+
+
+def test_table_iv_printed_rows():
+    """All 14 consistent printed rows agree with the simulator on 2,000 random triples."""
+    rows = _table_iv()
+    rnd = random.Random(0)
+    mismatched = set()
+    for _ in range(2000):
+        fin, fh, fout = (rnd.randint(1, 3000) for _ in range(3))
+        for i in range(16):
+            printed = (_eval(rows[i][0], fin, fh, fout), _eval(rows[i][1], fin, fh, fout))
+            if cm.simulate(i, (fin, fh, fout)) != printed:
+                mismatched.add(i)
+    assert mismatched == {13, 15}  # reading R19: the two inconsistent printed rows
+
+
+def test_table_iv_typo_rows_derived():
+    """Row 13's printed comm is a copy of row 9's; row 15 matches no configuration (R19)."""
+    rows = _table_iv()
+    assert rows[13][0] == rows[9][0]
+    rnd = random.Random(1)
+    for _ in range(500):
+        f = tuple(rnd.randint(1, 3000) for _ in range(3))
+        assert cm.simulate(13, f) == cm.table_iv_symbolic(13, *f)
+        assert cm.simulate(15, f) == cm.table_iv_symbolic(15, *f)
+        # row 13's printed sparse column is right; only its comm entry is wrong
+        assert cm.simulate(13, f)[1] == _eval(rows[13][1], *f)
+    f = (602, 128, 41)
+    printed15 = (_eval(rows[15][0], *f), _eval(rows[15][1], *f))
+    assert printed15 not in set(cm.all_costs(f).values())
+
+
+@pytest.mark.parametrize("name,f,ids", _table_vi())
+def test_table_vi_pareto_sets(name, f, ids):
+    assert cm.pareto_front(f) == ids
+
+
+def test_fig4_id10_is_dense_sparse_dense_sparse():
+    """Fig. 4 (L132–134): ID 10 = D,S forward and D,S backward; cost (4f_h, 4f_h)."""
+    fwd, bwd = cm.decode(10, 2)
+    assert (fwd[1], fwd[2], bwd[2], bwd[1]) == (1, 0, 1, 0)
+    assert cm.name(10, 2) == "FDS/BDS"
+    for f in [(602, 128, 41), (1, 7, 3000), (128, 256, 47)]:
+        assert cm.simulate(10, f) == (4 * f[1], 4 * f[1])
+        assert cm.simulate(5, f) == (2 * f[0] + 4 * f[2], 2 * f[0] + 2 * f[2])
+
+
+def test_encode_decode_roundtrip():
+    for L in (1, 2, 3, 4):
+        for i in range(4 ** L):
+            fwd, bwd = cm.decode(i, L)
+            assert cm.encode(fwd, bwd, L) == i
+
+
+def test_three_layer_products_front():
+    """products-shaped 3L h256: SURVEY App. A front incl. the 3-way tie (reading R23)."""
+    f = (100, 256, 256, 47)
+    costs = cm.all_costs(f)
+    front = cm.pareto(costs)
+    names = {cm.name(i, 3): costs[i] for i in front}
+    assert names["FDSD/BSDS"] == (1212, 1118)
+    assert names["FSSD/BSDS"] == (1312, 962)
+    assert names["FSDD/BSSD"] == names["FSSD/BSDD"] == names["FSSD/BSSD"] == (1412, 806)
+    assert len(front) == 5
+
+
+def test_sparse_units_equal_spmm_widths():
+    """Sparse units are SpMM widths: every config does ≥ one SpMM per layer per pass."""
+    f = (602, 128, 41)
+    for i, (c, s) in cm.all_costs(f).items():
+        assert s >= 2 * min(f[1:]) and c >= 0
+
+
+def test_redistribution_volume_constant_in_P():
+    """(P−1)/P·N·f elements per redistribution (L142): exact partition counts."""
+    n, f = 232965, 128
+    for P in (2, 4, 8):
+        tot = rd.total_elements(n, f, P)
+        approx = (P - 1) / P * n * f
+        assert abs(tot - approx) / approx < 1e-3
+    assert rd.total_elements(n, f, 1) == 0
+
+
+def test_partition_covers():
+    for n, f, P in [(10, 7, 8), (2708, 1433, 8), (5, 3, 8), (100, 41, 3)]:
+        rows = [rd.row_range(n, P, p) for p in range(P)]
+        cols = [rd.col_range(f, P, p) for p in range(P)]
+        assert rows[0][0] == 0 and rows[-1][1] == n
+        assert cols[0][0] == 0 and cols[-1][1] == f
+        for p in range(P - 1):
+            assert rows[p][1] == rows[p + 1][0]
+            assert cols[p][1] == cols[p + 1][0]
+            assert cols[p][0] % 4 == 0 and (cols[p][1] - cols[p][0]) % 4 == 0
+
+
+def test_fig7_two_process_roundtrip():
+    import numpy as np
+    M = np.arange(6 * 8, dtype=np.float32).reshape(6, 8)
+    rows = rd.row_slices(M, 2)
+    cols = rd.redistribute_row2col(rows, 2)
+    assert cols[0].shape == (6, 4) and np.array_equal(cols[1], M[:, 4:])
+    back = rd.redistribute_col2row(cols, 2)
+    for a, b in zip(rows, back):
+        assert np.array_equal(a.view(np.uint32), b.view(np.uint32))
