@@ -1,0 +1,349 @@
+/* rdm.h — C ABI of the B200-native GNN-RDM hot path.
+ *
+ * GNN-RDM (Kurt, Yan, Sukumaran-Rajam, Pandey, Sadayappan, IPDPS'23,
+ * "Communication Optimization for Distributed Execution of Graph Neural
+ * Networks"); citations are PAPER.md line numbers "L<n>" with the section,
+ * equation or table they fall in.
+ *
+ * The method: a full-batch GCN layer Z^l = Aᵀ H^{l-1} W^l, H^l = σ(Z^l)
+ * (eq. 1-2) and its backward (eq. 3-4) distributed over P
+ * processes with NO communication inside the products:
+ *   - SpMM  Out = A·In    with A replicated, In/Out column ("vertically")
+ *     sliced  (§III-A, Fig. 2a);
+ *   - GEMM  Out = In·W    with W replicated, In/Out row ("horizontally")
+ *     sliced  (Fig. 2b);
+ *   - an all-to-all personalized redistribution between the two layouts is
+ *     the only bulk communication (§III-D; Fig. 7);
+ *   - the order (AᵀH)W vs Aᵀ(HW) is chosen per layer, forward and backward,
+ *     by a redistribution-volume / SpMM-op-count model (§IV, Tables II-IV,
+ *     Pareto set Table VI).
+ *
+ * Conventions for every entry point
+ * ---------------------------------
+ *  * Return value: an rdm_status.  Nothing is thrown across the ABI.  On a
+ *    non-RDM_OK status, rdm_last_error(ctx) returns a human-readable reason
+ *    (thread-unsafe; one ctx per thread).  Arguments are validated
+ *    synchronously (RDM_ERR_ARG).  Kernel-launch errors are reported
+ *    immediately (RDM_ERR_CUDA); asynchronous device faults surface at
+ *    rdm_sync() or the next call.  After an NCCL failure the communicator is
+ *    aborted and every later call on the ctx returns RDM_ERR_STATE.
+ *  * Asynchrony: every call that takes a ctx enqueues its work on the ctx's
+ *    CUDA stream and returns without synchronising, except rdm_set_graph,
+ *    rdm_gcn_create/set_input (setup, synchronous) and the pure host
+ *    functions (rdm_partition, rdm_config_*, rdm_select_config).
+ *  * Memory: all float / index buffers passed to compute entry points are
+ *    CUDA device memory on the ctx's device unless a parameter says
+ *    otherwise (`on_host`).  The caller owns every buffer it passes; the
+ *    library owns the device CSR copy, the row bins, the pack/recv
+ *    workspace, the NCCL communicator and the activation workspace of an
+ *    rdm_gcn.  Nothing the caller passed is freed by the library.
+ *  * Dense layout: row-major fp32 with a leading dimension `ld` (elements)
+ *    that is a multiple of 4 and 16-byte aligned base pointers; columns
+ *    [width, ld) are padding and must hold zeros on input (outputs keep them
+ *    zero).  rdm_partition() returns the ld the library expects.
+ *  * Ranks: a ctx is either ONE rank of a P-process NCCL job (one process per
+ *    GPU) or, with rank == RDM_ALL_RANKS, a "virtual group" holding all P
+ *    ranks in this process on one device, whose all-to-all is a device copy
+ *    (used to exercise the P>1 partitions, pack/unpack and executor on a
+ *    single GPU).  Collective entry points take one pointer per LOCAL rank
+ *    (1 for an NCCL rank, P for a virtual group, local slot i = rank i).
+ *  * Collective entry points (rdm_redistribute, rdm_allreduce_sum,
+ *    rdm_gcn_forward, rdm_gcn_backward, rdm_gcn_set_input) must be called
+ *    by every rank in the same order.
+ */
+#ifndef RDM_H
+#define RDM_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define RDM_ABI_VERSION 1
+#define RDM_ALL_RANKS (-1)
+#define RDM_MAX_LAYERS 8
+#define RDM_UNIQUE_ID_BYTES 128
+
+typedef struct rdm_ctx rdm_ctx; /* one per process (= one per GPU), or one virtual group */
+typedef struct rdm_gcn rdm_gcn; /* a GCN model instance: config + activation workspace */
+
+typedef enum {
+  RDM_OK = 0,
+  RDM_ERR_ARG = 1,         /* invalid argument / size / layout; nothing enqueued            */
+  RDM_ERR_CUDA = 2,        /* CUDA runtime or launch error                                  */
+  RDM_ERR_NCCL = 3,        /* NCCL error; the communicator has been aborted                 */
+  RDM_ERR_OOM = 4,         /* device allocation failed (e.g. A does not fit: R_A < P, L148) */
+  RDM_ERR_UNSUPPORTED = 5, /* valid request this build does not implement                   */
+  RDM_ERR_STATE = 6        /* ctx poisoned by an earlier NCCL/CUDA fault, or call order     */
+} rdm_status;
+
+/* Row-sliced ("horizontal", Fig. 2b) or column-sliced ("vertical", Fig. 2a). */
+typedef enum { RDM_ROW = 0, RDM_COL = 1 } rdm_layout;
+
+/* Fused epilogues (bit set).  BIAS: out[:, c] += bias[c] (reading R8);
+ * RELU: σ = ReLU (reading R4); MASK: out ⊙= 1[mask > 0], the Hadamard with
+ * σ'(Z^{l-1}) of eq. (3), given H^{l-1} = ReLU(Z^{l-1}) in the same layout. */
+enum { RDM_EPI_NONE = 0, RDM_EPI_BIAS = 1, RDM_EPI_RELU = 2, RDM_EPI_MASK = 4 };
+
+/* GEMM forms (eq. 1, 3, 4).  rows = local row count, W is k x m:
+ *   NN: C[rows x m] = X[rows x k] · W          (forward, Z = T W or T = H W)
+ *   NT: C[rows x k] = X[rows x m] · Wᵀ         (backward data, A G Wᵀ)
+ *   TN: C[k x m]    = X[rows x k]ᵀ · U[rows x m] (weight gradient, eq. 4) */
+enum { RDM_GEMM_NN = 0, RDM_GEMM_NT = 1, RDM_GEMM_TN = 2 };
+
+/* One configuration (Table IV): for each layer l = 1..L (index
+ * l-1), 1 = GEMM first ("D", dense first), 0 = SpMM first ("S").  The
+ * integer ID of a config puts bits MSB→LSB as [bwd L … bwd 1, fwd 1 … fwd L]
+ * (for L = 2: ID = 8·bwdL2 + 4·bwdL1 + 2·fwdL1 + fwdL2; ID 10 = the
+ * dense-sparse-dense-sparse path of Fig. 4). */
+typedef struct {
+  int L;
+  uint8_t fwd_D[RDM_MAX_LAYERS];
+  uint8_t bwd_D[RDM_MAX_LAYERS];
+} rdm_config;
+
+/* Flags for rdm_gcn_create. */
+enum {
+  RDM_GCN_INPUT_GRAD = 1, /* also compute G^0 = A G^1 (W^1)ᵀ (Fig. 4 output; reading R2) —
+                             required for costs to match Table IV                       */
+  RDM_GCN_BIAS = 2        /* Z = Â H W + 1 bᵀ (reading R8); not implemented: UNSUPPORTED */
+};
+
+/* Tensors exposed by rdm_gcn_tensor (for parity tests / inspection). */
+enum {
+  RDM_T_H = 0,    /* H^l, l = 0..L-1                                   */
+  RDM_T_Z = 1,    /* logits Z^L (layer argument ignored)               */
+  RDM_T_G = 2,    /* G^l = ∂ℓ/∂Z^l, l = 0..L (G^0 = ∂ℓ/∂H^0)           */
+  RDM_T_MEMO = 3, /* T_l = Aᵀ H^{l-1}, row-sliced, S-first layers (L134) */
+  RDM_T_DWP = 4   /* this rank's partial Y^l before the all-reduce     */
+};
+
+/* Per-phase timers (Fig. 12 analogue: communication vs computation). */
+enum {
+  RDM_PH_SPMM = 0,
+  RDM_PH_GEMM = 1,
+  RDM_PH_PACK = 2,      /* pack + unpack kernels of the redistribution  */
+  RDM_PH_A2A = 3,       /* NCCL grouped send/recv (or virtual copies)    */
+  RDM_PH_LOSS = 4,
+  RDM_PH_ALLREDUCE = 5, /* Y^l / loss all-reduce                         */
+  RDM_PH_ADAM = 6,
+  RDM_PH_OTHER = 7,
+  RDM_PH_COUNT = 8
+};
+
+typedef struct {
+  int64_t a2a_calls;          /* redistributions executed                                    */
+  int64_t a2a_elems_payload;  /* elements crossing ranks (exact partition, no padding)       */
+  int64_t a2a_bytes_wire;     /* bytes handed to the transport for other ranks (incl. pad)   */
+  int64_t a2a_width_units;    /* Σ widths f of redistributions = the model's comm units      */
+  int64_t spmm_calls;
+  int64_t spmm_nnz_cols;      /* Σ nnz · w over SpMM calls (sparse ops, L142)                 */
+  int64_t spmm_width_units;   /* Σ full widths f of SpMM steps = the model's sparse units    */
+  int64_t gemm_calls;
+  int64_t gemm_flops;
+  int64_t allreduce_bytes;
+  int64_t kernel_launches;    /* kernels this library launched                               */
+} rdm_counters;
+
+/* ---------------------------------------------------------------- context */
+
+/* ncclGetUniqueId into id[RDM_UNIQUE_ID_BYTES]; rank 0 calls it and the caller
+ * broadcasts the bytes (e.g. with torch.distributed). */
+rdm_status rdm_get_unique_id(void* id);
+
+/* Create a context on CUDA device `device`, enqueuing on `cuda_stream`
+ * (cudaStream_t; NULL = the legacy default stream).
+ *   world == 1                  : single process, no NCCL.
+ *   0 <= rank < world, world > 1: one rank of an NCCL job; `nccl_unique_id`
+ *                                 (RDM_UNIQUE_ID_BYTES) from rdm_get_unique_id.
+ *   rank == RDM_ALL_RANKS       : virtual group of `world` ranks in-process.
+ * Errors: RDM_ERR_ARG (bad rank/world/device), RDM_ERR_CUDA, RDM_ERR_NCCL. */
+rdm_status rdm_init(rdm_ctx** ctx, int rank, int world, const void* nccl_unique_id, int device,
+                    void* cuda_stream);
+rdm_status rdm_finalize(rdm_ctx* ctx);
+const char* rdm_last_error(const rdm_ctx* ctx);
+/* Block until the ctx's stream is idle; surfaces asynchronous CUDA/NCCL faults. */
+rdm_status rdm_sync(rdm_ctx* ctx);
+rdm_status rdm_set_stream(rdm_ctx* ctx, void* cuda_stream);
+int rdm_world(const rdm_ctx* ctx);
+int rdm_num_local(const rdm_ctx* ctx);            /* local rank slots (1 or world)  */
+int rdm_local_rank(const rdm_ctx* ctx, int slot); /* global rank of local slot      */
+
+/* Partition (reading R11; the paper draws even halves, Fig. 5/7):
+ *   RDM_ROW: rows [lo, hi) of n, lo = ⌊rank·n/world⌋; ld = roundup(f, 4)
+ *   RDM_COL: cols [lo, hi) of f in 4-float granules g = ⌈f/4⌉,
+ *            lo = min(f, 4·⌊rank·g/world⌋); ld = roundup(hi − lo, 4)
+ * Pure host function. */
+rdm_status rdm_partition(int world, rdm_layout layout, int64_t n, int64_t f, int rank,
+                         int64_t* lo, int64_t* hi, int64_t* ld);
+
+/* ------------------------------------------------------------------ graph */
+
+/* Install the replicated sparse adjacency A (N x N CSR: int64 rowptr[n+1],
+ * int32 col[nnz], fp32 val[nnz]) on every local rank — R_A = P full
+ * replication (§III-E).  Values are used as given (the GCN
+ * normalization is the caller's, L255).  `symmetric` != 0 promises A = Aᵀ
+ * (one CSR serves eq. 1's Aᵀ and eq. 3-4's A, reading R3); otherwise the
+ * transpose is built.  `on_host` != 0: pointers are host memory.  Validates
+ * rowptr monotonicity and column range (RDM_ERR_ARG) and builds the row
+ * bins (light rows warp-per-row, heavy rows split into fixed nnz segments).
+ * RDM_ERR_OOM if A does not fit (R_A < P is not supported).  Synchronous. */
+rdm_status rdm_set_graph(rdm_ctx* ctx, int64_t n, int64_t nnz, const int64_t* rowptr,
+                         const int32_t* col, const float* val, int symmetric, int on_host);
+
+/* --------------------------------------------------- communication-free ops */
+
+/* Communication-free SpMM on one column slice (Fig. 2a):
+ *   out[N x w] = op(A) · in[N x w],  op(A) = Aᵀ if transpose (eq. 1) else A
+ * (eq. 3-4).  in/out: row-major, leading dims ld_in/ld_out (multiples of 4,
+ * ≥ w).  Epilogue bits RDM_EPI_*: bias[w] (device) added, then ReLU, then
+ * ⊙ 1[mask > 0] with mask[N x w] at leading dim ld_mask.  Local: no
+ * communication.  Deterministic (fixed summation order, no float atomics). */
+rdm_status rdm_spmm(rdm_ctx* ctx, int transpose, const float* in, int64_t ld_in, float* out,
+                    int64_t ld_out, int64_t w, int epilogue, const float* bias, const float* mask,
+                    int64_t ld_mask);
+
+/* Communication-free GEMM on row slices (Fig. 2b), fp32-accurate.
+ * op = RDM_GEMM_NN / NT / TN (see above); X at leading dim ldx, W k x m
+ * contiguous (ldw = m) for NN/NT; for TN the second operand U is rows x m at
+ * leading dim ldw.  C at leading dim ldc.  Epilogue (NN/NT only): BIAS, RELU,
+ * MASK (mask at leading dim ldc).  Local: no communication. */
+rdm_status rdm_gemm(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, int64_t ldw,
+                    float* C, int64_t ldc, int64_t rows, int64_t k, int64_t m, int epilogue,
+                    const float* bias, const float* mask);
+
+/* ------------------------------------------------------------- collectives */
+
+/* All-to-all personalized redistribution of an N x f matrix between the
+ * row-sliced and column-sliced layouts (§III-D, Fig. 7: divide
+ * into P chunks → exchange → merge).  from = RDM_ROW: src[i] is local slot
+ * i's row slice (rows_p x ld_row), dst[i] its column slice (N x ld_col_p);
+ * from = RDM_COL the reverse.  Pure data movement: bit-exact.  Moves
+ * Σ_{p≠q} rows·cols ≈ (P−1)/P·N·f elements in total (L142).  P = 1: copies
+ * src to dst if they differ (the two layouts coincide). */
+rdm_status rdm_redistribute(rdm_ctx* ctx, rdm_layout from, const float* const* src,
+                            float* const* dst, int64_t n, int64_t f);
+
+/* Exchange plan of one redistribution for `rank` (pure host function), per
+ * peer q (arrays of `world` entries, element units): the rank sends
+ * send_elems[q] floats starting at send_off[q] and receives recv_elems[q]
+ * floats at recv_off[q].  from = RDM_ROW: sends from the packed staging
+ * buffer (blocks rows_p x ld_q in q order), receives straight into its
+ * column slice; from = RDM_COL: sends straight from its column slice,
+ * receives into the staging buffer (then merged).  Self entries are 0 (the
+ * self block is copied on-device).  Wire blocks are ld-padded (rdm.h). */
+rdm_status rdm_redist_plan(int world, int rank, rdm_layout from, int64_t n, int64_t f,
+                           int64_t* send_off, int64_t* send_elems, int64_t* recv_off,
+                           int64_t* recv_elems);
+
+/* In-place sum over all ranks of count floats per local slot (weight-gradient
+ * reduction, reading R16).  Virtual group: every slot receives the sum. */
+rdm_status rdm_allreduce_sum(rdm_ctx* ctx, float* const* bufs, int64_t count);
+
+/* ----------------------------------------------------- cost model / selector */
+
+/* Decode / encode a configuration ID (see rdm_config). */
+rdm_status rdm_config_from_id(int L, int64_t id, rdm_config* out);
+int64_t rdm_config_to_id(const rdm_config* cfg);
+
+/* The paper's model cost of one configuration (§IV-A/B, Tables II-IV):
+ * comm_units = Σ redistribution widths (units of (P−1)/P·N elements),
+ * sparse_units = Σ SpMM widths (units of nnz FMAs).  f has L+1 entries.
+ * need_input_grad must be 1 for Table IV's costs (G^0 is an output, Fig. 4).
+ * Pure host function. */
+rdm_status rdm_config_costs(int L, const int64_t* f, int need_input_grad, int64_t id,
+                            int64_t* comm_units, int64_t* sparse_units);
+
+/* Enumerate the 4^L configurations, keep the Pareto-optimal ones in
+ * (comm, sparse) (L31, L224; ties kept, reading R23) into pareto_ids
+ * (*n_pareto: capacity in, count out), and pick one (reading R23): the
+ * minimum of a B200-calibrated time model t = comm·(P−1)/P·N·4 B / B_link +
+ * Σ_spmm (8·nnz + 8·N·w/P) / B_hbm, ties → fewer SpMM width → lower ID.
+ * P = 1: comm is free, so the pick is the minimum sparse cost (reading R24).
+ * Pure host function. */
+rdm_status rdm_select_config(int L, const int64_t* f, int64_t n, int64_t nnz, int P,
+                             int need_input_grad, int64_t* pareto_ids, int* n_pareto,
+                             int64_t* chosen_id, int64_t* comm_units, int64_t* sparse_units);
+
+/* -------------------------------------------------------------------- GCN */
+
+/* Create a GCN instance with L layers of widths f[0..L] using configuration
+ * cfg, and allocate its activation workspace on every local rank.  Requires
+ * rdm_set_graph.  flags: RDM_GCN_*.  Synchronous. */
+rdm_status rdm_gcn_create(rdm_ctx* ctx, int L, const int64_t* f, const rdm_config* cfg, int flags,
+                          rdm_gcn** out);
+rdm_status rdm_gcn_destroy(rdm_gcn* g);
+
+/* Per local slot i: H0_row[i] = the rank's row slice of H^0 (rows_p x f0,
+ * dense, ld = f0), labels_row[i] (int32, rows_p), mask_row[i] (uint8 train
+ * mask, rows_p; NULL = all rows).  `on_host` != 0: host pointers (pinned for
+ * async copies).  Builds H^0 in every layout the config reads (the model
+ * charges nothing for H^0's layout, reading R12) and n_train (global).
+ * Collective. */
+rdm_status rdm_gcn_set_input(rdm_gcn* g, const float* const* H0_row,
+                             const int32_t* const* labels_row, const uint8_t* const* mask_row,
+                             int on_host);
+
+/* Forward pass of all layers + loss (eq. 1-2; loss L206, reading R5).  W[l]
+ * (l = 0..L-1) = W^{l+1}, f_l x f_{l+1} row-major, replicated (one copy per
+ * process).  loss_dev: device double, receives the global mean loss.
+ * Collective. */
+rdm_status rdm_gcn_forward(rdm_gcn* g, const float* const* W, const float* const* b,
+                           double* loss_dev);
+
+/* Backward pass (eq. 3-4) with fwd→bwd memo reuse (§III-C):
+ * dW[l] receives Y^{l+1}, all-reduced over ranks (one copy per process);
+ * db ignored (bias unsupported).  Collective. */
+rdm_status rdm_gcn_backward(rdm_gcn* g, const float* const* W, float* const* dW, float* const* db);
+
+/* What the executor will run for this instance (per epoch, per rank):
+ *   model_*  : the paper's cost of the config (rdm_config_costs);
+ *   plan_*   : the units the executor actually issues — redistribution widths
+ *              (incl. `plan_hidden_comm_units`, transfers the paper's model
+ *              does not charge, e.g. the Hadamard operand of IDs 6/9,
+ *              reading R15) and SpMM widths; at P = 1 no redistribution runs.
+ *   a2a_elems: exact elements crossing ranks per epoch summed over all ranks
+ *              (Σ over redistributions of Σ_{p≠q} rows·cols, no padding). */
+typedef struct {
+  int64_t model_comm_units, model_sparse_units;
+  int64_t plan_comm_units, plan_hidden_comm_units, plan_sparse_units;
+  int64_t a2a_elems;
+  int n_fwd_steps, n_bwd_steps;
+  int64_t workspace_bytes; /* activation workspace per process */
+} rdm_gcn_info;
+rdm_status rdm_gcn_get_info(const rdm_gcn* g, rdm_gcn_info* out);
+/* Human-readable step list (forward then backward) into buf[cap]. */
+rdm_status rdm_gcn_describe(const rdm_gcn* g, char* buf, size_t cap);
+/* The same plan for a hypothetical instance (pure host function, no ctx):
+ * L layers, widths f[0..L], config cfg, P ranks, N vertices, RDM_GCN_* flags.
+ * `desc` (may be NULL) receives the step list. */
+rdm_status rdm_plan_info(int L, const int64_t* f, const rdm_config* cfg, int P, int64_t n,
+                         int flags, rdm_gcn_info* out, char* desc, size_t cap);
+
+/* Device pointer + shape of an internal tensor of local slot `slot` in
+ * `layout` (RDM_ERR_ARG if that layout is not resident). */
+rdm_status rdm_gcn_tensor(rdm_gcn* g, int which, int layer, int slot, rdm_layout layout,
+                          const float** ptr, int64_t* rows, int64_t* cols, int64_t* ld);
+
+/* Adam (PyTorch semantics, no weight decay; L297 lr = 0.01) on `count`
+ * replicated parameter arrays of sizes[i] floats; step ≥ 1. */
+rdm_status rdm_adam_step(rdm_ctx* ctx, int count, float* const* params, const float* const* grads,
+                         float* const* m, float* const* v, const int64_t* sizes, float lr,
+                         float beta1, float beta2, float eps, int step);
+
+/* -------------------------------------------------------- instrumentation */
+rdm_status rdm_get_counters(const rdm_ctx* ctx, rdm_counters* out);
+rdm_status rdm_reset_counters(rdm_ctx* ctx);
+/* Enable per-phase CUDA-event timing on the ctx stream (small overhead). */
+rdm_status rdm_set_timing(rdm_ctx* ctx, int enable);
+/* Accumulated ms per RDM_PH_* phase and launches per phase since the last
+ * reset (synchronises the stream). */
+rdm_status rdm_get_phase_times(rdm_ctx* ctx, double* ms, int64_t* launches);
+rdm_status rdm_reset_phase_times(rdm_ctx* ctx);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* RDM_H */

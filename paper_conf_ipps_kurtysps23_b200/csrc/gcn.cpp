@@ -1,0 +1,762 @@
+// gcn.cpp — planner + executor of the per-layer GNN-RDM sequence.
+//
+// PAPER.md §III (L85-167) and §IV (L175-224):
+//  * forward layer l, SpMM first (S):  T = Aᵀ H^{l-1} on column slices,
+//    redistribute T col→row (kept as the memo T_l, Fig. 4 "T_d saved",
+//    L134), Z^l = T W^l on row slices;
+//  * forward layer l, GEMM first (D): T = H^{l-1} W^l on row slices,
+//    redistribute row→col, Z^l = Aᵀ T on column slices;
+//  * H^l = ReLU(Z^l) fused into the producing kernel's epilogue;
+//  * the loss needs Z^L row-sliced (L206);
+//  * backward layer l, S:  U = A G^l (col), U col→row, Y^l = H^{l-1}ᵀ U,
+//    G^{l-1} = U W^{lᵀ} ⊙ σ'(Z^{l-1});  D: V = G^l W^{lᵀ} (row), V row→col,
+//    G^{l-1} = (A V) ⊙ σ'(Z^{l-1}), Y^l = T_lᵀ G^l (memo, L120) — or, without
+//    the memo, one extra SpMM of width min(f_{l-1}, f_l) (L208, Table III);
+//  * every operand is redistributed only when it is not resident in the
+//    layout its consumer needs (L210), exactly as the cost model charges.
+// The Hadamard σ'(Z^{l-1}) = 1[H^{l-1} > 0] is applied wherever H^{l-1} is
+// resident in G^{l-1}'s layout (it commutes with redistribution, reading
+// R15); only configurations 6 and 9 (L = 2) must move H^{l-1} for it, which
+// the plan reports as hidden communication.
+#include <algorithm>
+#include <cstdio>
+#include <cstring>
+#include <map>
+#include <set>
+#include <sstream>
+
+#include "internal.h"
+
+rdm_status rdm_guarded_call(rdm_ctx* ctx, void (*fn)(void*), void* arg);
+
+namespace rdm {
+namespace {
+
+enum Kind { K_H = 0, K_Z, K_T, K_G, K_U, K_V, K_X };
+const char* kKindName[] = {"H", "Z", "T", "G", "U", "V", "X"};
+struct Key {
+  int kind = 0, layer = 0;
+  int id() const { return kind * 64 + layer; }
+};
+enum Op { S_SPMM = 0, S_GEMM, S_TN, S_REDIST, S_MASK, S_LOSS };
+
+struct Step {
+  int op = 0;
+  int trans = 0, gop = 0, epi = 0, wl = 0;
+  Key in, in2, out, mask;
+  int lin = 0, lin2 = 0, lout = 0, lmask = 0;
+  int64_t width = 0;
+  bool hidden = false;
+};
+
+struct Planner {
+  int L = 0, P = 1;
+  std::vector<int64_t> f;
+  rdm_config cfg{};
+  bool igrad = true;
+  std::set<std::pair<int, int>> res, masked;
+  std::map<int, int64_t> width;
+  std::set<int> pending;
+  std::vector<bool> memo;
+  std::vector<Step>* cur = nullptr;
+
+  int lay(int l) const { return P == 1 ? 0 : l; }
+  bool has(Key k, int l) const {
+    return res.count({k.id(), lay(l)}) || (P == 1 && res.count({k.id(), 1}));
+  }
+  void produce(Key k, int l, int64_t w) {
+    res.insert({k.id(), lay(l)});
+    width[k.id()] = w;
+  }
+  void need(Key k, int l, bool hidden) {
+    if (has(k, l)) return;
+    const int other = 1 - l;
+    if (!has(k, other)) throw Error(RDM_ERR_STATE, "planner: operand never produced");
+    Step s;
+    s.op = S_REDIST;
+    s.in = k;
+    s.lin = other;
+    s.out = k;
+    s.lout = l;
+    s.width = width[k.id()];
+    s.hidden = hidden;
+    cur->push_back(s);
+    res.insert({k.id(), lay(l)});
+    if (masked.count({k.id(), lay(other)})) masked.insert({k.id(), lay(l)});
+  }
+  void needG(int l, int ly) {
+    Key g{K_G, l};
+    need(g, ly, false);
+    if (l < L && pending.count(g.id()) && !masked.count({g.id(), lay(ly)})) {
+      Key h{K_H, l};
+      if (!has(h, ly)) need(h, ly, true);
+      Step s;
+      s.op = S_MASK;
+      s.out = g;
+      s.lout = ly;
+      s.mask = h;
+      s.lmask = ly;
+      s.width = f[l];
+      cur->push_back(s);
+      masked.insert({g.id(), lay(ly)});
+    }
+  }
+  void spmm(int trans, Key in, Key out, int64_t w, int epi = 0, Key mask = Key{}) {
+    Step s;
+    s.op = S_SPMM;
+    s.trans = trans;
+    s.in = in;
+    s.lin = RDM_COL;
+    s.out = out;
+    s.lout = RDM_COL;
+    s.width = w;
+    s.epi = epi;
+    s.mask = mask;
+    s.lmask = RDM_COL;
+    cur->push_back(s);
+    produce(out, RDM_COL, w);
+    if (epi & RDM_EPI_MASK) masked.insert({out.id(), lay(RDM_COL)});
+  }
+  void gemm(int gop, Key in, int wl, Key out, int64_t w, int epi = 0, Key mask = Key{}) {
+    Step s;
+    s.op = S_GEMM;
+    s.gop = gop;
+    s.in = in;
+    s.lin = RDM_ROW;
+    s.wl = wl;
+    s.out = out;
+    s.lout = RDM_ROW;
+    s.epi = epi;
+    s.mask = mask;
+    s.lmask = RDM_ROW;
+    s.width = w;
+    cur->push_back(s);
+    produce(out, RDM_ROW, w);
+    if (epi & RDM_EPI_MASK) masked.insert({out.id(), lay(RDM_ROW)});
+  }
+  void tn(Key x, Key u, int wl) {
+    Step s;
+    s.op = S_TN;
+    s.in = x;
+    s.lin = RDM_ROW;
+    s.in2 = u;
+    s.lin2 = RDM_ROW;
+    s.wl = wl;
+    cur->push_back(s);
+  }
+
+  void plan(std::vector<Step>& fwd, std::vector<Step>& bwd) {
+    memo.assign(L + 1, false);
+    produce({K_H, 0}, RDM_ROW, f[0]);
+    produce({K_H, 0}, RDM_COL, f[0]);
+    cur = &fwd;
+    for (int l = 1; l <= L; ++l) {
+      Key hin{K_H, l - 1}, hout = l < L ? Key{K_H, l} : Key{K_Z, 0}, t{K_T, l};
+      const int epi = l < L ? RDM_EPI_RELU : 0;
+      if (!cfg.fwd_D[l - 1]) {
+        need(hin, RDM_COL, false);
+        spmm(1, hin, t, f[l - 1]);
+        need(t, RDM_ROW, false);
+        gemm(RDM_GEMM_NN, t, l, hout, f[l], epi);
+        memo[l] = true;
+      } else {
+        need(hin, RDM_ROW, false);
+        gemm(RDM_GEMM_NN, hin, l, t, f[l]);
+        need(t, RDM_COL, false);
+        spmm(1, t, hout, f[l], epi);
+      }
+    }
+    need({K_Z, 0}, RDM_ROW, false);
+    {
+      Step s;
+      s.op = S_LOSS;
+      s.in = {K_Z, 0};
+      s.lin = RDM_ROW;
+      s.out = {K_G, L};
+      s.lout = RDM_ROW;
+      s.width = f[L];
+      fwd.push_back(s);
+      produce({K_G, L}, RDM_ROW, f[L]);
+    }
+    cur = &bwd;
+    for (int l = L; l >= 1; --l) {
+      Key g{K_G, l}, gout{K_G, l - 1}, hprev{K_H, l - 1}, t{K_T, l};
+      const bool out = l > 1 || igrad;
+      if (!cfg.bwd_D[l - 1]) {
+        needG(l, RDM_COL);
+        Key u{K_U, l};
+        spmm(0, g, u, f[l]);
+        need(u, RDM_ROW, false);
+        if (has(hprev, RDM_ROW)) {
+          tn(hprev, u, l);
+        } else if (memo[l] && has(g, RDM_ROW) && (l == L || masked.count({g.id(), lay(RDM_ROW)}))) {
+          tn(t, g, l);
+        } else {
+          need(hprev, RDM_ROW, true);
+          tn(hprev, u, l);
+        }
+        if (out) {
+          int epi = 0;
+          if (l > 1) {
+            if (has(hprev, RDM_ROW)) epi = RDM_EPI_MASK;
+            else pending.insert(gout.id());
+          }
+          gemm(RDM_GEMM_NT, u, l, gout, f[l - 1], epi, hprev);
+        }
+      } else {
+        needG(l, RDM_ROW);
+        Key v{K_V, l};
+        gemm(RDM_GEMM_NT, g, l, v, f[l - 1]);
+        if (memo[l]) tn(t, g, l);
+        if (out) {
+          need(v, RDM_COL, false);
+          int epi = 0;
+          if (l > 1) {
+            if (has(hprev, RDM_COL)) epi = RDM_EPI_MASK;
+            else pending.insert(gout.id());
+          }
+          spmm(0, v, gout, f[l - 1], epi, hprev);
+        }
+        if (!memo[l]) {
+          Key x{K_X, l};
+          if (f[l - 1] < f[l]) {
+            need(hprev, RDM_COL, false);
+            spmm(1, hprev, x, f[l - 1]);
+            need(x, RDM_ROW, false);
+            tn(x, g, l);
+          } else {
+            needG(l, RDM_COL);
+            spmm(0, g, x, f[l]);
+            need(x, RDM_ROW, false);
+            need(hprev, RDM_ROW, false);
+            tn(hprev, x, l);
+          }
+        }
+      }
+    }
+  }
+};
+
+struct Buf {
+  float* p = nullptr;
+  int64_t rows = 0, cols = 0, ld = 0;
+};
+
+}  // namespace
+}  // namespace rdm
+
+using namespace rdm;
+
+struct rdm_gcn {
+  rdm_ctx* ctx = nullptr;
+  int L = 0, flags = 0;
+  std::vector<int64_t> f;
+  rdm_config cfg{};
+  std::vector<Step> fwd, bwd;
+  Planner pl;
+  std::vector<std::unique_ptr<DevBuf>> mem;
+  // per slot: (key id, layout) → buffer
+  std::vector<std::map<std::pair<int, int>, Buf>> bufs;
+  std::vector<std::vector<float*>> dwp;     // per slot per layer partial Y (virtual group)
+  std::vector<int32_t*> labels;
+  std::vector<uint8_t*> mask;
+  std::vector<double*> scal;                // per slot: [0] n_train, [1] loss partial
+  bool input_set = false;
+  int64_t ws_bytes = 0;
+  rdm_gcn_info info{};
+};
+
+namespace rdm {
+namespace {
+
+int norm_lay(const rdm_gcn* g, int l) { return g->ctx->world == 1 ? 0 : l; }
+
+Buf& buf(rdm_gcn* g, int slot, Key k, int l) {
+  auto it = g->bufs[slot].find({k.id(), norm_lay(g, l)});
+  if (it == g->bufs[slot].end())
+    throw Error(RDM_ERR_STATE, std::string("executor: missing buffer ") + kKindName[k.kind] +
+                                   std::to_string(k.layer));
+  return it->second;
+}
+
+void alloc_buf(rdm_gcn* g, Key k, int l, int64_t width) {
+  rdm_ctx* ctx = g->ctx;
+  const int P = ctx->world;
+  const int64_t n = ctx->graph.n;
+  for (int s = 0; s < ctx->nlocal(); ++s) {
+    auto key = std::make_pair(k.id(), norm_lay(g, l));
+    if (g->bufs[s].count(key)) continue;
+    const int p = ctx->local[s];
+    Buf b;
+    if (norm_lay(g, l) == RDM_ROW) {
+      b.rows = row_range(n, P, p).size();
+      b.cols = width;
+      b.ld = roundup4(width);
+    } else {
+      b.rows = n;
+      b.cols = col_range(width, P, p).size();
+      b.ld = roundup4(b.cols);
+    }
+    const size_t bytes = (size_t)std::max<int64_t>(1, b.rows * b.ld) * sizeof(float);
+    g->mem.emplace_back(new DevBuf(bytes));
+    RDM_CUDA(cudaMemset(g->mem.back()->ptr, 0, bytes));
+    b.p = g->mem.back()->as<float>();
+    g->ws_bytes += bytes;
+    g->bufs[s][key] = b;
+  }
+}
+
+void plan_info(const Planner& pl, const std::vector<Step>& fwd, const std::vector<Step>& bwd,
+               int64_t n, rdm_gcn_info* out) {
+  rdm_gcn_info in{};
+  const int P = pl.P;
+  model_costs(pl.L, pl.f.data(), pl.igrad ? 1 : 0, pl.cfg, &in.model_comm_units,
+              &in.model_sparse_units);
+  auto tot_elems = [&](int64_t w) {
+    int64_t t = 0;
+    if (P == 1) return t;
+    for (int p = 0; p < P; ++p)
+      for (int q = 0; q < P; ++q)
+        if (p != q) t += row_range(n, P, p).size() * col_range(w, P, q).size();
+    return t;
+  };
+  for (auto* v : {&fwd, &bwd})
+    for (auto& s : *v) {
+      if (s.op == S_REDIST) {
+        in.plan_comm_units += s.width;
+        if (s.hidden) in.plan_hidden_comm_units += s.width;
+        in.a2a_elems += tot_elems(s.width);
+      }
+      if (s.op == S_SPMM) in.plan_sparse_units += s.width;
+    }
+  in.n_fwd_steps = (int)fwd.size();
+  in.n_bwd_steps = (int)bwd.size();
+  *out = in;
+}
+
+std::string describe_steps(const std::vector<Step>& fwd, const std::vector<Step>& bwd);
+
+void create(rdm_gcn* g) {
+  rdm_ctx* ctx = g->ctx;
+  Planner& pl = g->pl;
+  pl.L = g->L;
+  pl.P = ctx->world;
+  pl.f = g->f;
+  pl.cfg = g->cfg;
+  pl.igrad = (g->flags & RDM_GCN_INPUT_GRAD) != 0;
+  pl.plan(g->fwd, g->bwd);
+  g->bufs.assign(ctx->nlocal(), {});
+  auto touch = [&](const Step& s) {
+    auto w = [&](Key k) { return pl.width.at(k.id()); };
+    switch (s.op) {
+      case S_SPMM:
+      case S_GEMM:
+        alloc_buf(g, s.in, s.lin, w(s.in));
+        alloc_buf(g, s.out, s.lout, w(s.out));
+        if (s.epi & RDM_EPI_MASK) alloc_buf(g, s.mask, s.lmask, w(s.mask));
+        break;
+      case S_TN:
+        alloc_buf(g, s.in, s.lin, w(s.in));
+        alloc_buf(g, s.in2, s.lin2, w(s.in2));
+        break;
+      case S_REDIST:
+        alloc_buf(g, s.in, s.lin, w(s.in));
+        alloc_buf(g, s.out, s.lout, w(s.out));
+        break;
+      case S_MASK:
+        alloc_buf(g, s.out, s.lout, w(s.out));
+        alloc_buf(g, s.mask, s.lmask, w(s.mask));
+        break;
+      case S_LOSS:
+        alloc_buf(g, s.in, s.lin, w(s.in));
+        alloc_buf(g, s.out, s.lout, w(s.out));
+        break;
+    }
+  };
+  // H^0 lives in both layouts
+  alloc_buf(g, {K_H, 0}, RDM_ROW, g->f[0]);
+  alloc_buf(g, {K_H, 0}, RDM_COL, g->f[0]);
+  for (auto& s : g->fwd) touch(s);
+  for (auto& s : g->bwd) touch(s);
+  const int P = ctx->world;
+  const int64_t n = ctx->graph.n;
+  g->dwp.assign(ctx->nlocal(), std::vector<float*>(g->L + 1, nullptr));
+  g->labels.assign(ctx->nlocal(), nullptr);
+  g->mask.assign(ctx->nlocal(), nullptr);
+  g->scal.assign(ctx->nlocal(), nullptr);
+  for (int s = 0; s < ctx->nlocal(); ++s) {
+    const int64_t r = row_range(n, P, ctx->local[s]).size();
+    if (ctx->virtual_group()) {
+      for (int l = 1; l <= g->L; ++l) {
+        g->mem.emplace_back(new DevBuf((size_t)g->f[l - 1] * g->f[l] * sizeof(float)));
+        g->dwp[s][l] = g->mem.back()->as<float>();
+      }
+    }
+    g->mem.emplace_back(new DevBuf(std::max<int64_t>(r, 1) * sizeof(int32_t)));
+    g->labels[s] = g->mem.back()->as<int32_t>();
+    g->mem.emplace_back(new DevBuf(std::max<int64_t>(r, 1)));
+    g->mask[s] = reinterpret_cast<uint8_t*>(g->mem.back()->ptr);
+    g->mem.emplace_back(new DevBuf(4 * sizeof(double)));
+    g->scal[s] = reinterpret_cast<double*>(g->mem.back()->ptr);
+    RDM_CUDA(cudaMemset(g->scal[s], 0, 4 * sizeof(double)));
+  }
+  plan_info(pl, g->fwd, g->bwd, n, &g->info);
+  g->info.workspace_bytes = g->ws_bytes;
+}
+
+void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
+  rdm_ctx* ctx = g->ctx;
+  const int nl = ctx->nlocal();
+  const int P = ctx->world;
+  switch (s.op) {
+    case S_SPMM: {
+      Phase ph(ctx, RDM_PH_SPMM);
+      const Csr& A = s.trans ? ctx->graph.fwd() : ctx->graph.bwd();
+      for (int i = 0; i < nl; ++i) {
+        Buf& in = buf(g, i, s.in, s.lin);
+        Buf& out = buf(g, i, s.out, s.lout);
+        const float* mk = nullptr;
+        int64_t ldm = 0;
+        if (s.epi & RDM_EPI_MASK) {
+          Buf& m = buf(g, i, s.mask, s.lmask);
+          mk = m.p;
+          ldm = m.ld;
+        }
+        const int64_t w = P == 1 ? s.width : col_range(s.width, P, ctx->local[i]).size();
+        spmm(ctx, A, in.p, in.ld, out.p, out.ld, w, s.epi, nullptr, mk, ldm);
+      }
+      ctx->counters.spmm_width_units += s.width;
+      break;
+    }
+    case S_GEMM: {
+      Phase ph(ctx, RDM_PH_GEMM);
+      const int64_t fin = g->f[s.wl - 1], fout = g->f[s.wl];
+      for (int i = 0; i < nl; ++i) {
+        Buf& in = buf(g, i, s.in, s.lin);
+        Buf& out = buf(g, i, s.out, s.lout);
+        const float* mk = (s.epi & RDM_EPI_MASK) ? buf(g, i, s.mask, s.lmask).p : nullptr;
+        gemm(ctx, s.gop, in.p, in.ld, W[s.wl - 1], fout, out.p, out.ld, in.rows, fin, fout, s.epi,
+             nullptr, mk);
+      }
+      break;
+    }
+    case S_TN: {
+      Phase ph(ctx, RDM_PH_GEMM);
+      const int64_t fin = g->f[s.wl - 1], fout = g->f[s.wl];
+      for (int i = 0; i < nl; ++i) {
+        Buf& x = buf(g, i, s.in, s.lin);
+        Buf& u = buf(g, i, s.in2, s.lin2);
+        float* dst = g->dwp[i][s.wl];  // per-slot partial, or the caller's dW (set in backward)
+        gemm(ctx, RDM_GEMM_TN, x.p, x.ld, u.p, u.ld, dst, fout, x.rows, fin, fout, 0, nullptr,
+             nullptr);
+      }
+      break;
+    }
+    case S_REDIST: {
+      std::vector<const float*> src(nl);
+      std::vector<float*> dst(nl);
+      for (int i = 0; i < nl; ++i) {
+        src[i] = buf(g, i, s.in, s.lin).p;
+        dst[i] = buf(g, i, s.out, s.lout).p;
+      }
+      redistribute(ctx, (rdm_layout)s.lin, src.data(), dst.data(), ctx->graph.n, s.width);
+      break;
+    }
+    case S_MASK: {
+      Phase ph(ctx, RDM_PH_OTHER);
+      for (int i = 0; i < nl; ++i) {
+        Buf& x = buf(g, i, s.out, s.lout);
+        Buf& h = buf(g, i, s.mask, s.lmask);
+        apply_mask(ctx, x.p, x.ld, h.p, h.ld, x.rows, x.cols);
+      }
+      break;
+    }
+    case S_LOSS: {
+      Phase ph(ctx, RDM_PH_LOSS);
+      for (int i = 0; i < nl; ++i) {
+        Buf& z = buf(g, i, s.in, s.lin);
+        Buf& gl = buf(g, i, s.out, s.lout);
+        softmax_xent(ctx, z.p, z.ld, g->labels[i], g->mask[i], z.rows, s.width, g->scal[i] + 0,
+                     gl.p, gl.ld, g->scal[i] + 1);
+      }
+      break;
+    }
+  }
+}
+
+std::string step_str(const Step& s) {
+  auto k = [](Key x, int l) {
+    return std::string(kKindName[x.kind]) + std::to_string(x.layer) + (l == RDM_ROW ? ".row" : ".col");
+  };
+  std::ostringstream o;
+  switch (s.op) {
+    case S_SPMM:
+      o << "SPMM  " << (s.trans ? "A^T" : "A  ") << " " << k(s.in, s.lin) << " -> " << k(s.out, s.lout)
+        << " w=" << s.width << (s.epi & RDM_EPI_RELU ? " +relu" : "")
+        << (s.epi & RDM_EPI_MASK ? " *mask(" + k(s.mask, s.lmask) + ")" : "");
+      break;
+    case S_GEMM:
+      o << "GEMM  " << (s.gop == RDM_GEMM_NN ? "NN " : "NT ") << k(s.in, s.lin) << " W" << s.wl << " -> "
+        << k(s.out, s.lout) << (s.epi & RDM_EPI_RELU ? " +relu" : "")
+        << (s.epi & RDM_EPI_MASK ? " *mask(" + k(s.mask, s.lmask) + ")" : "");
+      break;
+    case S_TN:
+      o << "GEMM  TN " << k(s.in, s.lin) << "^T " << k(s.in2, s.lin2) << " -> Y" << s.wl;
+      break;
+    case S_REDIST:
+      o << "A2A   " << k(s.in, s.lin) << " -> " << k(s.out, s.lout) << " f=" << s.width
+        << (s.hidden ? " (hidden)" : "");
+      break;
+    case S_MASK:
+      o << "MASK  " << k(s.out, s.lout) << " *= 1[" << k(s.mask, s.lmask) << " > 0]";
+      break;
+    case S_LOSS:
+      o << "LOSS  " << k(s.in, s.lin) << " -> " << k(s.out, s.lout);
+      break;
+  }
+  return o.str();
+}
+
+std::string describe_steps(const std::vector<Step>& fwd, const std::vector<Step>& bwd) {
+  std::string s = "forward:\n";
+  for (auto& st : fwd) s += "  " + step_str(st) + "\n";
+  s += "backward:\n";
+  for (auto& st : bwd) s += "  " + step_str(st) + "\n";
+  return s;
+}
+
+struct FwdArgs {
+  rdm_gcn* g;
+  const float* const* W;
+  double* loss;
+};
+struct BwdArgs {
+  rdm_gcn* g;
+  const float* const* W;
+  float* const* dW;
+};
+
+void do_forward(void* a_) {
+  auto* a = static_cast<FwdArgs*>(a_);
+  rdm_gcn* g = a->g;
+  rdm_ctx* ctx = g->ctx;
+  if (!g->input_set) throw Error(RDM_ERR_STATE, "rdm_gcn_forward: call rdm_gcn_set_input first");
+  RDM_CHECK_ARG(a->W && a->loss, "rdm_gcn_forward: W and loss_dev required");
+  for (int l = 0; l < g->L; ++l) RDM_CHECK_ARG(a->W[l], "rdm_gcn_forward: null W");
+  for (auto& s : g->fwd) run_step(g, s, a->W);
+  const int nl = ctx->nlocal();
+  std::vector<double*> parts(nl);
+  for (int i = 0; i < nl; ++i) parts[i] = g->scal[i] + 1;
+  allreduce_d(ctx, parts.data(), 1);
+  Phase ph(ctx, RDM_PH_LOSS);
+  finish_loss(ctx, g->scal[0] + 1, g->scal[0] + 0, a->loss);
+}
+
+void do_backward(void* a_) {
+  auto* a = static_cast<BwdArgs*>(a_);
+  rdm_gcn* g = a->g;
+  rdm_ctx* ctx = g->ctx;
+  RDM_CHECK_ARG(a->W && a->dW, "rdm_gcn_backward: W and dW required");
+  for (int l = 0; l < g->L; ++l) RDM_CHECK_ARG(a->W[l] && a->dW[l], "rdm_gcn_backward: null W/dW");
+  if (!ctx->virtual_group())
+    for (int l = 1; l <= g->L; ++l) g->dwp[0][l] = a->dW[l - 1];
+  for (auto& s : g->bwd) run_step(g, s, a->W);
+  const int nl = ctx->nlocal();
+  for (int l = 1; l <= g->L; ++l) {
+    const int64_t cnt = g->f[l - 1] * g->f[l];
+    if (ctx->virtual_group()) {
+      Phase ph(ctx, RDM_PH_ALLREDUCE);
+      std::vector<const float*> parts(nl);
+      for (int i = 0; i < nl; ++i) parts[i] = g->dwp[i][l];
+      sum_slots(ctx, a->dW[l - 1], parts.data(), nl, cnt);
+      ctx->counters.allreduce_bytes += cnt * 4;
+    } else {
+      float* b = a->dW[l - 1];
+      allreduce(ctx, &b, cnt);
+    }
+  }
+}
+
+struct InputArgs {
+  rdm_gcn* g;
+  const float* const* H0;
+  const int32_t* const* labels;
+  const uint8_t* const* mask;
+  int on_host;
+};
+
+void do_set_input(void* a_) {
+  auto* a = static_cast<InputArgs*>(a_);
+  rdm_gcn* g = a->g;
+  rdm_ctx* ctx = g->ctx;
+  const int nl = ctx->nlocal(), P = ctx->world;
+  const int64_t n = ctx->graph.n, f0 = g->f[0];
+  RDM_CHECK_ARG(a->H0 && a->labels, "set_input: H0 and labels required");
+  const cudaMemcpyKind kind = a->on_host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
+  const rdm_counters saved = ctx->counters;
+  std::vector<const float*> src(nl);
+  std::vector<float*> dst(nl);
+  for (int i = 0; i < nl; ++i) {
+    const int64_t r = row_range(n, P, ctx->local[i]).size();
+    Buf& h = buf(g, i, {K_H, 0}, RDM_ROW);
+    if (r && f0)
+      RDM_CUDA(cudaMemcpy2DAsync(h.p, h.ld * sizeof(float), a->H0[i], f0 * sizeof(float),
+                                 f0 * sizeof(float), r, kind, ctx->stream));
+    if (r) {
+      RDM_CUDA(cudaMemcpyAsync(g->labels[i], a->labels[i], r * sizeof(int32_t), kind, ctx->stream));
+      if (a->mask && a->mask[i])
+        RDM_CUDA(cudaMemcpyAsync(g->mask[i], a->mask[i], r, kind, ctx->stream));
+      else
+        RDM_CUDA(cudaMemsetAsync(g->mask[i], 1, r, ctx->stream));
+    }
+    src[i] = h.p;
+    dst[i] = buf(g, i, {K_H, 0}, RDM_COL).p;
+  }
+  if (P > 1) redistribute(ctx, RDM_ROW, src.data(), dst.data(), n, f0);
+  std::vector<double*> nt(nl);
+  for (int i = 0; i < nl; ++i) {
+    const int64_t r = row_range(n, P, ctx->local[i]).size();
+    count_mask(ctx, g->mask[i], r, g->scal[i] + 0);
+    nt[i] = g->scal[i] + 0;
+  }
+  allreduce_d(ctx, nt.data(), 1);
+  ctx->counters = saved;
+  g->input_set = true;
+}
+
+void do_create(void* a_) { create(static_cast<rdm_gcn*>(a_)); }
+
+}  // namespace
+}  // namespace rdm
+
+extern "C" {
+
+rdm_status rdm_gcn_create(rdm_ctx* ctx, int L, const int64_t* f, const rdm_config* cfg, int flags,
+                          rdm_gcn** out) {
+  if (!ctx || !out || !f || !cfg || L < 1 || L > RDM_MAX_LAYERS || cfg->L != L) return RDM_ERR_ARG;
+  for (int l = 0; l <= L; ++l)
+    if (f[l] < 1) return RDM_ERR_ARG;
+  if (flags & RDM_GCN_BIAS) {
+    ctx->err = "rdm_gcn_create: RDM_GCN_BIAS is not implemented";
+    return RDM_ERR_UNSUPPORTED;
+  }
+  if (!ctx->has_graph) {
+    ctx->err = "rdm_gcn_create: no graph (call rdm_set_graph)";
+    return RDM_ERR_STATE;
+  }
+  auto* g = new rdm_gcn();
+  g->ctx = ctx;
+  g->L = L;
+  g->flags = flags;
+  g->f.assign(f, f + L + 1);
+  g->cfg = *cfg;
+  rdm_status st = rdm_guarded_call(ctx, do_create, g);
+  if (st != RDM_OK) {
+    delete g;
+    return st;
+  }
+  *out = g;
+  return RDM_OK;
+}
+
+rdm_status rdm_gcn_destroy(rdm_gcn* g) {
+  if (!g) return RDM_ERR_ARG;
+  cudaSetDevice(g->ctx->device);
+  cudaStreamSynchronize(g->ctx->stream);
+  delete g;
+  return RDM_OK;
+}
+
+rdm_status rdm_gcn_set_input(rdm_gcn* g, const float* const* H0_row, const int32_t* const* labels_row,
+                             const uint8_t* const* mask_row, int on_host) {
+  if (!g) return RDM_ERR_ARG;
+  InputArgs a{g, H0_row, labels_row, mask_row, on_host};
+  return rdm_guarded_call(g->ctx, do_set_input, &a);
+}
+
+rdm_status rdm_gcn_forward(rdm_gcn* g, const float* const* W, const float* const* b,
+                           double* loss_dev) {
+  (void)b;
+  if (!g) return RDM_ERR_ARG;
+  FwdArgs a{g, W, loss_dev};
+  return rdm_guarded_call(g->ctx, do_forward, &a);
+}
+
+rdm_status rdm_gcn_backward(rdm_gcn* g, const float* const* W, float* const* dW, float* const* db) {
+  (void)db;
+  if (!g) return RDM_ERR_ARG;
+  BwdArgs a{g, W, dW};
+  return rdm_guarded_call(g->ctx, do_backward, &a);
+}
+
+rdm_status rdm_gcn_tensor(rdm_gcn* g, int which, int layer, int slot, rdm_layout layout,
+                          const float** ptr, int64_t* rows, int64_t* cols, int64_t* ld) {
+  if (!g || slot < 0 || slot >= g->ctx->nlocal()) return RDM_ERR_ARG;
+  Key k;
+  switch (which) {
+    case RDM_T_H: k = {K_H, layer}; break;
+    case RDM_T_Z: k = {K_Z, 0}; break;
+    case RDM_T_G: k = {K_G, layer}; break;
+    case RDM_T_MEMO: k = {K_T, layer}; break;
+    case RDM_T_DWP: {
+      if (layer < 1 || layer > g->L || !g->dwp[slot][layer]) return RDM_ERR_ARG;
+      if (ptr) *ptr = g->dwp[slot][layer];
+      if (rows) *rows = g->f[layer - 1];
+      if (cols) *cols = g->f[layer];
+      if (ld) *ld = g->f[layer];
+      return RDM_OK;
+    }
+    default: return RDM_ERR_ARG;
+  }
+  if (which == RDM_T_MEMO && (layer < 1 || layer > g->L || g->cfg.fwd_D[layer - 1])) return RDM_ERR_ARG;
+  auto it = g->bufs[slot].find({k.id(), norm_lay(g, layout)});
+  if (it == g->bufs[slot].end()) {
+    g->ctx->err = "rdm_gcn_tensor: tensor not resident in that layout";
+    return RDM_ERR_ARG;
+  }
+  const Buf& b = it->second;
+  if (ptr) *ptr = b.p;
+  if (rows) *rows = b.rows;
+  if (cols) *cols = b.cols;
+  if (ld) *ld = b.ld;
+  return RDM_OK;
+}
+
+rdm_status rdm_gcn_get_info(const rdm_gcn* g, rdm_gcn_info* out) {
+  if (!g || !out) return RDM_ERR_ARG;
+  *out = g->info;
+  return RDM_OK;
+}
+
+rdm_status rdm_gcn_describe(const rdm_gcn* g, char* buf, size_t cap) {
+  if (!g || !buf || !cap) return RDM_ERR_ARG;
+  const std::string s = describe_steps(g->fwd, g->bwd);
+  std::snprintf(buf, cap, "%s", s.c_str());
+  return s.size() < cap ? RDM_OK : RDM_ERR_ARG;
+}
+
+}  // extern "C"
+
+extern "C" rdm_status rdm_plan_info(int L, const int64_t* f, const rdm_config* cfg, int P, int64_t n,
+                                    int flags, rdm_gcn_info* out, char* desc, size_t cap) {
+  if (L < 1 || L > RDM_MAX_LAYERS || !f || !cfg || cfg->L != L || P < 1 || n < 0) return RDM_ERR_ARG;
+  try {
+    Planner pl;
+    pl.L = L;
+    pl.P = P;
+    pl.f.assign(f, f + L + 1);
+    pl.cfg = *cfg;
+    pl.igrad = (flags & RDM_GCN_INPUT_GRAD) != 0;
+    std::vector<Step> fwd, bwd;
+    pl.plan(fwd, bwd);
+    if (out) plan_info(pl, fwd, bwd, n, out);
+    if (desc && cap) {
+      const std::string s = describe_steps(fwd, bwd);
+      std::snprintf(desc, cap, "%s", s.c_str());
+      if (s.size() >= cap) return RDM_ERR_ARG;
+    }
+    return RDM_OK;
+  } catch (const std::exception&) {
+    return RDM_ERR_STATE;
+  }
+}

@@ -1,0 +1,209 @@
+// internal.h — shared declarations of the rdm library (not part of the ABI).
+#pragma once
+
+#include <cuda_runtime.h>
+#include <nccl.h>
+
+#include <cstdint>
+#include <map>
+#include <memory>
+#include <stdexcept>
+#include <string>
+#include <vector>
+
+#include "../../include/rdm.h"
+
+namespace rdm {
+
+// ------------------------------------------------------------------ errors
+struct Error : std::runtime_error {
+  rdm_status status;
+  Error(rdm_status s, const std::string& m) : std::runtime_error(m), status(s) {}
+};
+
+#define RDM_CHECK_ARG(cond, msg)                                      \
+  do {                                                                \
+    if (!(cond)) throw ::rdm::Error(RDM_ERR_ARG, std::string(msg));   \
+  } while (0)
+
+#define RDM_CUDA(call)                                                                     \
+  do {                                                                                     \
+    cudaError_t e_ = (call);                                                               \
+    if (e_ != cudaSuccess)                                                                 \
+      throw ::rdm::Error(e_ == cudaErrorMemoryAllocation ? RDM_ERR_OOM : RDM_ERR_CUDA,     \
+                         std::string(#call) + ": " + cudaGetErrorString(e_) + " @" +       \
+                             __FILE__ + ":" + std::to_string(__LINE__));                   \
+  } while (0)
+
+#define RDM_LAUNCHED(ctx)                                                                  \
+  do {                                                                                     \
+    cudaError_t e_ = cudaGetLastError();                                                   \
+    if (e_ != cudaSuccess)                                                                 \
+      throw ::rdm::Error(RDM_ERR_CUDA, std::string("kernel launch: ") +                    \
+                                           cudaGetErrorString(e_) + " @" + __FILE__ + ":" + \
+                                           std::to_string(__LINE__));                      \
+    (ctx)->counters.kernel_launches++;                                                     \
+    (ctx)->phase_launches[(ctx)->cur_phase]++;                                             \
+  } while (0)
+
+inline int64_t roundup4(int64_t x) { return (x + 3) & ~int64_t(3); }
+inline int64_t ceil_div(int64_t a, int64_t b) { return (a + b - 1) / b; }
+
+// --------------------------------------------------------------- partition
+struct Range {
+  int64_t lo, hi;
+  int64_t size() const { return hi - lo; }
+};
+Range row_range(int64_t n, int P, int p);
+Range col_range(int64_t f, int P, int p);
+
+// ------------------------------------------------------------ device memory
+struct DevBuf {
+  void* ptr = nullptr;
+  size_t bytes = 0;
+  DevBuf() = default;
+  explicit DevBuf(size_t b);
+  ~DevBuf();
+  DevBuf(const DevBuf&) = delete;
+  DevBuf& operator=(const DevBuf&) = delete;
+  template <class T>
+  T* as() const { return static_cast<T*>(ptr); }
+};
+
+// ------------------------------------------------------------------- graph
+struct Csr {
+  int64_t n = 0, nnz = 0;
+  std::unique_ptr<DevBuf> rowptr, col, val;
+  // row bins (see spmm.cu): light rows processed warp-per-row, heavy rows
+  // split into fixed-size nnz segments reduced deterministically.
+  int64_t n_light = 0, n_seg = 0, n_heavy = 0;
+  std::unique_ptr<DevBuf> light_rows;   // int32[n_light], longest rows first
+  std::unique_ptr<DevBuf> seg_start;    // int64[n_seg]: first nnz of each segment
+  std::unique_ptr<DevBuf> heavy_rows;   // int32[n_heavy]
+  std::unique_ptr<DevBuf> heavy_seg;    // int32[n_heavy+1]: segment range of heavy row
+  int64_t max_deg = 0;
+};
+
+struct Graph {
+  int64_t n = 0, nnz = 0;
+  bool symmetric = true;
+  Csr A;    // rows of A: used for A·X (eq. 3-4)
+  Csr AT;   // rows of Aᵀ: used for Aᵀ·X (eq. 1); empty if symmetric
+  const Csr& fwd() const { return symmetric ? A : AT; }
+  const Csr& bwd() const { return A; }
+};
+
+}  // namespace rdm
+
+// --------------------------------------------------------------- context
+struct rdm_ctx {
+  int world = 1;
+  int rank = 0;                  // RDM_ALL_RANKS for a virtual group
+  std::vector<int> local;        // global ranks held in this process
+  int device = 0;
+  int num_sms = 148;
+  cudaStream_t stream = nullptr;
+  ncclComm_t comm = nullptr;
+  bool poisoned = false;
+  std::string err;
+  rdm::Graph graph;
+  bool has_graph = false;
+  rdm_counters counters{};
+  // workspace (grown on demand, never shrunk)
+  std::vector<std::unique_ptr<rdm::DevBuf>> ws_send, ws_recv;  // per local slot
+  std::unique_ptr<rdm::DevBuf> ws_seg;                         // SpMM heavy-row partials
+  std::unique_ptr<rdm::DevBuf> ws_gemm;                        // GEMM split-K partials
+  std::unique_ptr<rdm::DevBuf> ws_scratch;
+  // phase timing
+  bool timing = false;
+  int cur_phase = RDM_PH_OTHER;
+  struct Ev {
+    int phase;
+    cudaEvent_t a, b;
+  };
+  std::vector<Ev> events;
+  std::vector<cudaEvent_t> event_pool;
+  double phase_ms[RDM_PH_COUNT] = {};
+  int64_t phase_launches[RDM_PH_COUNT] = {};
+  bool virtual_group() const { return rank == RDM_ALL_RANKS && world > 1; }
+  int nlocal() const { return (int)local.size(); }
+};
+
+namespace rdm {
+
+float* ensure_ws(std::unique_ptr<DevBuf>& b, size_t bytes);
+
+// Scoped phase timer: records CUDA events on the ctx stream around a phase.
+struct Phase {
+  rdm_ctx* ctx;
+  int prev;
+  cudaEvent_t a = nullptr;
+  Phase(rdm_ctx* c, int ph);
+  ~Phase();
+};
+
+// ------------------------------------------------------------------ kernels
+// spmm.cu
+void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
+          int64_t w, int epi, const float* bias, const float* mask, int64_t ld_mask);
+void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host);
+
+// gemm.cu
+void gemm(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, int64_t ldw, float* C,
+          int64_t ldc, int64_t rows, int64_t k, int64_t m, int epi, const float* bias,
+          const float* mask);
+
+// redist.cu — pack (row slice → P contiguous blocks, each r x ld_q) and
+// unpack (P blocks r x ld_q → row slice).  `blocks[q]` points to block q.
+struct BlockTable {
+  static constexpr int kMax = 64;
+  const float* src[kMax];
+  float* dst[kMax];
+  int64_t col_lo[kMax];
+  int64_t width[kMax];
+  int64_t ld[kMax];
+};
+void pack_rows(rdm_ctx* ctx, const float* row_slice, int64_t ld_row, int64_t rows, int P,
+               const BlockTable& t);
+void unpack_rows(rdm_ctx* ctx, float* row_slice, int64_t ld_row, int64_t rows, int P,
+                 const BlockTable& t);
+
+// misc.cu
+void softmax_xent(rdm_ctx* ctx, const float* Z, int64_t ldz, const int32_t* labels,
+                  const uint8_t* mask, int64_t rows, int64_t C, const double* n_train, float* G,
+                  int64_t ldg, double* loss_partial);
+void count_mask(rdm_ctx* ctx, const uint8_t* mask, int64_t rows, double* out);
+void apply_mask(rdm_ctx* ctx, float* X, int64_t ldx, const float* H, int64_t ldh, int64_t rows,
+                int64_t cols);
+void sum_slots(rdm_ctx* ctx, float* out, const float* const* parts, int nparts, int64_t count);
+void sum_doubles(rdm_ctx* ctx, double* out, const double* const* parts, int nparts);
+void finish_loss(rdm_ctx* ctx, const double* sum, const double* n_train, double* loss);
+void adam(rdm_ctx* ctx, float* p, const float* g, float* m, float* v, int64_t n, float lr,
+          float b1, float b2, float eps, float bc1, float bc2);
+void copy_2d(rdm_ctx* ctx, float* dst, int64_t ldd, const float* src, int64_t lds, int64_t rows,
+             int64_t cols);
+
+// ---------------------------------------------------------------- transport
+// Exchange of the redistribution: for every local slot i and peer q != p,
+// send[i][q] (bytes) → slot of q, recv[i][q].
+struct Xfer {
+  const void* send[BlockTable::kMax];
+  void* recv[BlockTable::kMax];
+  size_t send_bytes[BlockTable::kMax];
+  size_t recv_bytes[BlockTable::kMax];
+};
+void exchange(rdm_ctx* ctx, std::vector<Xfer>& x);   // x[i] for local slot i
+void allreduce(rdm_ctx* ctx, float* const* bufs, int64_t count);
+void allreduce_d(rdm_ctx* ctx, double* const* bufs, int64_t count);
+
+// redistribution on all local slots (used by rdm_redistribute and the executor)
+void redistribute(rdm_ctx* ctx, rdm_layout from, const float* const* src, float* const* dst,
+                  int64_t n, int64_t f);
+
+// ------------------------------------------------------------------- plan
+int64_t config_to_id(const rdm_config& c);
+rdm_config config_from_id(int L, int64_t id);
+void model_costs(int L, const int64_t* f, int need_input_grad, const rdm_config& c, int64_t* comm,
+                 int64_t* sparse);
+
+}  // namespace rdm

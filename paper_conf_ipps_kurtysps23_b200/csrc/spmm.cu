@@ -1,0 +1,270 @@
+// spmm.cu — communication-free CSR SpMM on a feature-column slice (sm_100a).
+//
+// PAPER.md §III-A (L102-104, Fig. 2a): Out = M·In needs no communication when
+// M (here the adjacency A) is replicated and In/Out are column ("vertically")
+// sliced.  The GCN aggregation of eq. (1) is Aᵀ·H (L69-71) and the backward
+// products of eq. (3)(4) are A·G (L77-79).  Each GPU multiplies the WHOLE
+// replicated CSR by its N x w column slice.
+//
+// Design (B200):
+//  * Work items are (light row) or (fixed-size nnz segment of a heavy row).
+//    Light rows (deg <= kSeg) are processed warp-per-row in descending-degree
+//    order (LPT), heavy rows are cut into kSeg-nnz segments processed
+//    warp-per-segment, whose partial rows are summed in segment order by a
+//    second tiny kernel: deterministic, no float atomics (the "CTA per heavy
+//    row" variant generalised to any degree).
+//  * Inside a warp, G lanes cover one nnz × (4G) columns with 128-bit gathers
+//    of the H row; 32/G nnz are in flight per warp step, so narrow slices
+//    (w = 16 at P = 8) still issue full-warp gathers.  Columns beyond 128 are
+//    handled by blockIdx.y chunks.
+//  * CSR col/val are streamed with evict-first loads (__ldcs) so the gathered
+//    H slice keeps L2; gathers use the read-only path (__ldg).
+//  * Fused epilogue: bias, ReLU, Hadamard mask 1[mask > 0] (eq. 3's σ').
+#include <algorithm>
+#include <vector>
+
+#include "internal.h"
+
+namespace rdm {
+namespace {
+
+constexpr int kWarps = 8;            // warps per CTA
+constexpr int64_t kSeg = 2048;       // nnz per heavy-row segment / light-row cap
+constexpr unsigned kFull = 0xffffffffu;
+
+struct Epi {
+  int flags;
+  const float* bias;
+  const float* mask;
+  int64_t ld_mask;
+  int64_t w;
+};
+
+__device__ __forceinline__ float4 apply_epi(float4 a, const Epi& e, int64_t row, int64_t c) {
+  if (e.flags & RDM_EPI_BIAS) {
+    if (c + 0 < e.w) a.x += e.bias[c + 0];
+    if (c + 1 < e.w) a.y += e.bias[c + 1];
+    if (c + 2 < e.w) a.z += e.bias[c + 2];
+    if (c + 3 < e.w) a.w += e.bias[c + 3];
+  }
+  if (e.flags & RDM_EPI_RELU) {
+    a.x = fmaxf(a.x, 0.f); a.y = fmaxf(a.y, 0.f); a.z = fmaxf(a.z, 0.f); a.w = fmaxf(a.w, 0.f);
+  }
+  if (e.flags & RDM_EPI_MASK) {
+    const float4 m = __ldg(reinterpret_cast<const float4*>(e.mask + row * e.ld_mask + c));
+    a.x = m.x > 0.f ? a.x : 0.f;
+    a.y = m.y > 0.f ? a.y : 0.f;
+    a.z = m.z > 0.f ? a.z : 0.f;
+    a.w = m.w > 0.f ? a.w : 0.f;
+  }
+  return a;
+}
+
+// Warp computes Σ_{j in [beg,end)} val[j] · X[col[j], c0 + sub*4 .. +4];
+// result valid in every lane of group 0 (lanes 0..G-1) after the reduction.
+template <int G>
+__device__ __forceinline__ float4 warp_nnz_range(const int32_t* __restrict__ col,
+                                                 const float* __restrict__ val,
+                                                 const float* __restrict__ X, int64_t ldx,
+                                                 int64_t beg, int64_t end, int lane, bool col_ok,
+                                                 int64_t cbase) {
+  constexpr int NG = 32 / G;
+  const int g = lane / G;
+  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+  const float* xb = X + cbase;
+  for (int64_t base = beg; base < end; base += 32) {
+    const int64_t j = base + lane;
+    int c = 0;
+    float v = 0.f;
+    if (j < end) {
+      c = __ldcs(col + j);
+      v = __ldcs(val + j);
+    }
+    const int cnt = (end - base) < 32 ? (int)(end - base) : 32;
+#pragma unroll
+    for (int t = 0; t < G; ++t) {
+      const int k = t * NG + g;
+      const int cc = __shfl_sync(kFull, c, k);
+      const float vv = __shfl_sync(kFull, v, k);
+      if (k < cnt && col_ok) {
+        const float4 x = __ldg(reinterpret_cast<const float4*>(xb + (int64_t)cc * ldx));
+        acc.x = fmaf(vv, x.x, acc.x);
+        acc.y = fmaf(vv, x.y, acc.y);
+        acc.z = fmaf(vv, x.z, acc.z);
+        acc.w = fmaf(vv, x.w, acc.w);
+      }
+    }
+  }
+#pragma unroll
+  for (int off = G; off < 32; off <<= 1) {
+    acc.x += __shfl_xor_sync(kFull, acc.x, off);
+    acc.y += __shfl_xor_sync(kFull, acc.y, off);
+    acc.z += __shfl_xor_sync(kFull, acc.z, off);
+    acc.w += __shfl_xor_sync(kFull, acc.w, off);
+  }
+  return acc;
+}
+
+// One warp per work item: items [0, n_seg) are heavy-row segments (partial
+// rows to `part`), items [n_seg, n_seg + n_light) are light rows (to out).
+template <int G>
+__global__ void __launch_bounds__(kWarps * 32)
+spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
+            const float* __restrict__ val, const int32_t* __restrict__ light_rows,
+            const int64_t* __restrict__ seg_start, const int32_t* __restrict__ seg_row,
+            int64_t n_light, int64_t n_seg, const float* __restrict__ X, int64_t ldx,
+            float* __restrict__ out, int64_t ld_out, float* __restrict__ part, int64_t ld_part,
+            int64_t w4, Epi epi) {
+  const int lane = threadIdx.x & 31;
+  const int64_t item = (int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5);
+  if (item >= n_seg + n_light) return;
+  const int64_t c = (int64_t)blockIdx.y * (4 * G) + (lane % G) * 4;  // this lane's first column
+  const bool col_ok = c < w4;
+  if (item < n_seg) {
+    const int32_t r = seg_row[item];
+    const int64_t beg = seg_start[item];
+    const int64_t end = min(beg + kSeg, rowptr[r + 1]);
+    const float4 acc = warp_nnz_range<G>(col, val, X, ldx, beg, end, lane, col_ok, c);
+    if (lane < G && col_ok) *reinterpret_cast<float4*>(part + item * ld_part + c) = acc;
+  } else {
+    const int32_t r = light_rows[item - n_seg];
+    const float4 acc = warp_nnz_range<G>(col, val, X, ldx, rowptr[r], rowptr[r + 1], lane, col_ok, c);
+    if (lane < G && col_ok)
+      *reinterpret_cast<float4*>(out + (int64_t)r * ld_out + c) = apply_epi(acc, epi, r, c);
+  }
+}
+
+// Heavy rows: sum the partial rows of their segments in segment order.
+__global__ void spmm_heavy_reduce(const int32_t* __restrict__ heavy_rows,
+                                  const int32_t* __restrict__ heavy_seg,
+                                  const float* __restrict__ part, int64_t ld_part,
+                                  float* __restrict__ out, int64_t ld_out, int64_t w4, Epi epi) {
+  const int64_t h = blockIdx.x;
+  const int32_t r = heavy_rows[h];
+  const int s0 = heavy_seg[h], s1 = heavy_seg[h + 1];
+  for (int64_t c = (int64_t)threadIdx.x * 4; c < w4; c += (int64_t)blockDim.x * 4) {
+    float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
+    for (int s = s0; s < s1; ++s) {
+      const float4 p = *reinterpret_cast<const float4*>(part + (int64_t)s * ld_part + c);
+      acc.x += p.x; acc.y += p.y; acc.z += p.z; acc.w += p.w;
+    }
+    *reinterpret_cast<float4*>(out + (int64_t)r * ld_out + c) = apply_epi(acc, epi, r, c);
+  }
+}
+
+template <int G>
+void launch_spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out,
+                 int64_t ld_out, float* part, int64_t ld_part, int64_t w4, const Epi& epi) {
+  const int64_t items = A.n_seg + A.n_light;
+  if (items == 0) return;
+  const int64_t chunks = ceil_div(w4, 4 * G);
+  dim3 grid((unsigned)ceil_div(items, kWarps), (unsigned)chunks);
+  spmm_kernel<G><<<grid, kWarps * 32, 0, ctx->stream>>>(
+      A.rowptr->as<int64_t>(), A.col->as<int32_t>(), A.val->as<float>(),
+      A.light_rows ? A.light_rows->as<int32_t>() : nullptr,
+      A.seg_start ? A.seg_start->as<int64_t>() : nullptr,
+      A.heavy_rows ? reinterpret_cast<const int32_t*>(A.seg_start->as<int64_t>() + A.n_seg) : nullptr,
+      A.n_light, A.n_seg, in, ld_in, out, ld_out, part, ld_part, w4, epi);
+  RDM_LAUNCHED(ctx);
+}
+
+}  // namespace
+
+void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
+          int64_t w, int epi_flags, const float* bias, const float* mask, int64_t ld_mask) {
+  RDM_CHECK_ARG(w >= 0, "spmm: negative width");
+  if (w == 0 || A.n == 0) return;
+  const int64_t w4 = roundup4(w);
+  RDM_CHECK_ARG(ld_in >= w4 && ld_out >= w4 && ld_in % 4 == 0 && ld_out % 4 == 0,
+                "spmm: leading dims must be multiples of 4 and >= roundup4(w)");
+  RDM_CHECK_ARG(((uintptr_t)in & 15) == 0 && ((uintptr_t)out & 15) == 0,
+                "spmm: in/out must be 16-byte aligned");
+  RDM_CHECK_ARG(!(epi_flags & RDM_EPI_MASK) || (mask && ld_mask >= w4 && ld_mask % 4 == 0 &&
+                                                ((uintptr_t)mask & 15) == 0),
+                "spmm: mask requires a 16-byte aligned N x w buffer with ld % 4 == 0");
+  RDM_CHECK_ARG(!(epi_flags & RDM_EPI_BIAS) || bias, "spmm: bias pointer missing");
+  Epi epi{epi_flags, bias, mask, ld_mask, w};
+  float* part = nullptr;
+  if (A.n_seg) part = ensure_ws(ctx->ws_seg, (size_t)A.n_seg * w4 * sizeof(float));
+  const int64_t w4c = w4;
+  const int64_t g_need = std::min<int64_t>(w4 / 4, 32);
+  if (g_need <= 1)       launch_spmm<1>(ctx, A, in, ld_in, out, ld_out, part, w4, w4c, epi);
+  else if (g_need <= 2)  launch_spmm<2>(ctx, A, in, ld_in, out, ld_out, part, w4, w4c, epi);
+  else if (g_need <= 4)  launch_spmm<4>(ctx, A, in, ld_in, out, ld_out, part, w4, w4c, epi);
+  else if (g_need <= 8)  launch_spmm<8>(ctx, A, in, ld_in, out, ld_out, part, w4, w4c, epi);
+  else if (g_need <= 16) launch_spmm<16>(ctx, A, in, ld_in, out, ld_out, part, w4, w4c, epi);
+  else                   launch_spmm<32>(ctx, A, in, ld_in, out, ld_out, part, w4, w4c, epi);
+  if (A.n_heavy) {
+    spmm_heavy_reduce<<<(unsigned)A.n_heavy, 128, 0, ctx->stream>>>(
+        A.heavy_rows->as<int32_t>(), A.heavy_seg->as<int32_t>(), part, w4, out, ld_out, w4c, epi);
+    RDM_LAUNCHED(ctx);
+  }
+  ctx->counters.spmm_calls++;
+  ctx->counters.spmm_nnz_cols += A.nnz * w;
+}
+
+// Row bins (host, one-time at rdm_set_graph; pure indexing of rowptr).
+void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rp) {
+  (void)ctx;
+  const int64_t n = A.n;
+  std::vector<int64_t> cnt(kSeg + 2, 0);
+  int64_t n_heavy = 0, n_seg = 0, max_deg = 0;
+  for (int64_t i = 0; i < n; ++i) {
+    const int64_t d = rp[i + 1] - rp[i];
+    max_deg = std::max(max_deg, d);
+    if (d > kSeg) {
+      ++n_heavy;
+      n_seg += ceil_div(d, kSeg);
+    } else {
+      cnt[kSeg - d]++;  // descending degree
+    }
+  }
+  const int64_t n_light = n - n_heavy;
+  std::vector<int64_t> pos(kSeg + 2, 0);
+  for (int64_t b = 1; b < kSeg + 2; ++b) pos[b] = pos[b - 1] + cnt[b - 1];
+  std::vector<int32_t> light(n_light);
+  std::vector<int64_t> seg_start(n_seg);
+  std::vector<int32_t> seg_row(n_seg), heavy(n_heavy), heavy_seg(n_heavy + 1);
+  int64_t s = 0, h = 0;
+  for (int64_t i = 0; i < n; ++i) {
+    const int64_t d = rp[i + 1] - rp[i];
+    if (d > kSeg) {
+      heavy[h] = (int32_t)i;
+      heavy_seg[h] = (int32_t)s;
+      ++h;
+      for (int64_t b = rp[i]; b < rp[i + 1]; b += kSeg) {
+        seg_start[s] = b;
+        seg_row[s] = (int32_t)i;
+        ++s;
+      }
+    } else {
+      light[pos[kSeg - d]++] = (int32_t)i;
+    }
+  }
+  heavy_seg[n_heavy] = (int32_t)s;
+  A.n_light = n_light;
+  A.n_seg = n_seg;
+  A.n_heavy = n_heavy;
+  A.max_deg = max_deg;
+  A.light_rows.reset(new DevBuf(std::max<int64_t>(1, n_light) * sizeof(int32_t)));
+  // seg_start (int64) followed by seg_row (int32) in one allocation
+  A.seg_start.reset(new DevBuf(std::max<int64_t>(1, n_seg) * (sizeof(int64_t) + sizeof(int32_t))));
+  A.heavy_rows.reset(new DevBuf(std::max<int64_t>(1, n_heavy) * sizeof(int32_t)));
+  A.heavy_seg.reset(new DevBuf((n_heavy + 1) * sizeof(int32_t)));
+  if (n_light)
+    RDM_CUDA(cudaMemcpy(A.light_rows->ptr, light.data(), n_light * sizeof(int32_t),
+                        cudaMemcpyHostToDevice));
+  if (n_seg) {
+    RDM_CUDA(cudaMemcpy(A.seg_start->ptr, seg_start.data(), n_seg * sizeof(int64_t),
+                        cudaMemcpyHostToDevice));
+    RDM_CUDA(cudaMemcpy(A.seg_start->as<int64_t>() + n_seg, seg_row.data(),
+                        n_seg * sizeof(int32_t), cudaMemcpyHostToDevice));
+  }
+  if (n_heavy)
+    RDM_CUDA(cudaMemcpy(A.heavy_rows->ptr, heavy.data(), n_heavy * sizeof(int32_t),
+                        cudaMemcpyHostToDevice));
+  RDM_CUDA(cudaMemcpy(A.heavy_seg->ptr, heavy_seg.data(), (n_heavy + 1) * sizeof(int32_t),
+                      cudaMemcpyHostToDevice));
+}
+
+}  // namespace rdm
