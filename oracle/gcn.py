@@ -129,8 +129,14 @@ def forward(A, H0, Ws, labels, mask, bs=None, orders=None) -> Result:
     return res
 
 
-def backward(A, res: Result, Ws) -> Result:
-    """eqs. (3)(4) with G^l = ∂ℓ/∂Z^l (reading R1), G^0 without Hadamard (R2)."""
+def backward(A, res: Result, Ws, relu_masks=None) -> Result:
+    """eqs. (3)(4) with G^l = ∂ℓ/∂Z^l (reading R1), G^0 without Hadamard (R2).
+
+    `relu_masks[l-1]` (optional, l = 1..L-1) replaces the decision 1[Z^l > 0]
+    of σ'(Z^l): where floating point decides a discrete value both sides must
+    take that decision in the same precision (reading R30), so the
+    parity tests pass the fp32 kernel's own sign pattern; the arithmetic stays
+    fp64 and unchanged."""
     L = len(Ws)
     G = [None] * (L + 1)
     Y = [None] * (L + 1)
@@ -142,16 +148,17 @@ def backward(A, res: Result, Ws) -> Result:
         db[l] = G[l].sum(axis=0)
         D = S @ np.asarray(Ws[l - 1], np.float64).T   # A G^l (W^l)ᵀ
         if l > 1:
-            G[l - 1] = D * (res.Z[l - 1] > 0)   # eq. (3), σ'(Z) = 1[Z > 0]
+            sig = (res.Z[l - 1] > 0) if relu_masks is None else np.asarray(relu_masks[l - 2], bool)
+            G[l - 1] = D * sig                  # eq. (3), σ'(Z) = 1[Z > 0]
         else:
             G[0] = D
     res.G, res.Y, res.db = G, Y, db
     return res
 
 
-def epoch(A, H0, Ws, labels, mask, bs=None):
+def epoch(A, H0, Ws, labels, mask, bs=None, relu_masks=None):
     res = forward(A, H0, Ws, labels, mask, bs)
-    return backward(A, res, Ws)
+    return backward(A, res, Ws, relu_masks)
 
 
 def adam(p, g, m, v, step, lr=0.01, b1=0.9, b2=0.999, eps=1e-8):

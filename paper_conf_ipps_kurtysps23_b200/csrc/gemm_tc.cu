@@ -1,10 +1,490 @@
-// gemm_tc.cu — tcgen05 (5th-gen tensor core) 3xTF32 GEMM for sm_100a.
-// Placeholder dispatcher: returns false (shape not taken) until the kernel lands.
+// gemm_tc.cu — fp32-accurate GEMM on the 5th-generation tensor cores (sm_100a).
+//
+// The communication-free dense products of the GCN layer (Fig. 2b,
+// L112: W replicated, row-sliced operands) — eq. (1) Z = T·W, eq. (3) A·G·Wᵀ,
+// eq. (4) Y = Hᵀ·(A·G) — run as tcgen05.mma kind::tf32 with the 3xTF32 split
+// (x = hi + lo, hi = x with the 13 low mantissa bits cleared, lo = x − hi
+// exactly; C = A_hi·B_hi + A_hi·B_lo + A_lo·B_hi), which keeps fp32-class
+// accuracy (the 1e-4 parity gate excludes 1xTF32's 2^-11 unit roundoff).
+//
+// Per CTA: one 128 x BN output tile accumulated in TMEM (fp32).  Warp roles:
+//   warp 0  TMA producer (cp.async.bulk.tensor, 128B swizzle, mbarrier tx)
+//   warp 1  MMA issuer (one thread issues tcgen05.mma; tcgen05.commit frees
+//           the smem stage and finally signals the epilogue)
+//   warp 2  TMEM allocator
+//   warps 4-7  split converter (in-place hi, lo into a twin buffer, then
+//           fence.proxy.async so the tensor core sees it) and afterwards the
+//           epilogue (tcgen05.ld 32x32b → fused ReLU / Hadamard mask / bias →
+//           global), one TMEM lane quadrant per warp.
+// Modes:
+//   NN / NT  A = X (K-major, TMA box 32 x 128); B = W or Wᵀ pre-split into
+//            hi/lo K-major panels by a tiny prep kernel (W is ≤ 1433 x 256).
+//   TN       A = Xᵀ and B = U are MN-major in memory (rows of X / U are the
+//            contraction): both loaded MN-major (box 32 x 32 per 128-byte
+//            chunk) with MN-major UMMA descriptors, both split in smem;
+//            split-K over rows with an ordered (deterministic) reduction.
+#include <cuda.h>
+#include <cudaTypedefs.h>
+
+#include <algorithm>
+#include <cstdlib>
+#include <cstring>
+
 #include "internal.h"
 
 namespace rdm {
-bool gemm_tc(rdm_ctx*, int, const float*, int64_t, const float*, int64_t, float*, int64_t, int64_t,
-             int64_t, int64_t, int, const float*, const float*) {
-  return false;
+namespace {
+
+constexpr int BM = 128;        // UMMA M (cta_group::1)
+constexpr int BK = 32;         // fp32 elements per 128-byte swizzle row
+constexpr int UK = 8;          // UMMA K for kind::tf32
+constexpr int kThreads = 256;
+
+// ------------------------------------------------------------ PTX wrappers
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return (uint32_t)__cvta_generic_to_shared(p);
 }
+__device__ __forceinline__ void mbar_init(uint64_t* b, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;" ::"r"(smem_u32(b)), "r"(count));
+}
+__device__ __forceinline__ void mbar_expect_tx(uint64_t* b, uint32_t bytes) {
+  asm volatile("mbarrier.arrive.expect_tx.shared::cta.b64 _, [%0], %1;" ::"r"(smem_u32(b)), "r"(bytes)
+               : "memory");
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* b) {
+  asm volatile("mbarrier.arrive.shared::cta.b64 _, [%0];" ::"r"(smem_u32(b)) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
+  uint32_t done;
+  do {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.b32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(smem_u32(b)), "r"(parity)
+        : "memory");
+  } while (!done);
+}
+__device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, uint64_t* bar, int c0,
+                                            int c1) {
+  asm volatile(
+      "cp.async.bulk.tensor.2d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4}], [%2];" ::"r"(
+          smem_u32(dst)),
+      "l"((uint64_t)map), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
+      : "memory");
+}
+__device__ __forceinline__ void fence_proxy_async() {
+  asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
+}
+__device__ __forceinline__ void tc_fence_after() {
+  asm volatile("tcgen05.fence::after_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tc_fence_before() {
+  asm volatile("tcgen05.fence::before_thread_sync;" ::: "memory");
+}
+__device__ __forceinline__ void tc_commit(uint64_t* b) {
+  asm volatile("tcgen05.commit.cta_group::1.mbarrier::arrive::one.shared::cluster.b64 [%0];" ::"r"(
+                   smem_u32(b))
+               : "memory");
+}
+__device__ __forceinline__ void tc_mma(uint32_t tmem_d, uint64_t da, uint64_t db, uint32_t idesc,
+                                       uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "l"(da), "l"(db), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+__device__ __forceinline__ void tmem_ld16(uint32_t addr, uint32_t (&r)[16]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x16.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15}, [%16];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]),
+        "=r"(r[14]), "=r"(r[15])
+      : "r"(addr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
+// UMMA shared-memory descriptor, 128-byte swizzle (layout type 2), version 1.
+__device__ __forceinline__ uint64_t sdesc(uint32_t saddr, uint32_t lbo_bytes, uint32_t sbo_bytes,
+                                          uint32_t layout = 2) {
+  uint64_t d = 0;
+  d |= (uint64_t)((saddr >> 4) & 0x3FFF);
+  d |= (uint64_t)((lbo_bytes >> 4) & 0x3FFF) << 16;
+  d |= (uint64_t)((sbo_bytes >> 4) & 0x3FFF) << 32;
+  d |= (uint64_t)1 << 46;  // version (sm_100)
+  d |= (uint64_t)layout << 61;  // 2 = SWIZZLE_128B, 1 = SWIZZLE_128B_BASE32B (MN-major tf32)
+  return d;
+}
+
+// kind::tf32 instruction descriptor: D f32, A/B tf32, M = 128, N, majors.
+__host__ __device__ constexpr uint32_t idesc_tf32(int N, int a_mn, int b_mn) {
+  return (1u << 4) | (2u << 7) | (2u << 10) | ((uint32_t)a_mn << 15) | ((uint32_t)b_mn << 16) |
+         ((uint32_t)(N >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+}
+
+// Round-to-nearest fp32 → tf32 (ties away from zero; finite inputs).  Both
+// halves of the split are rounded, so neither the split nor the tensor core's
+// own treatment of the 13 dropped bits biases the products: truncation made
+// every product err toward zero and the error then accumulated coherently
+// through the heavy cancellation of the weight-gradient sums (softmax-gradient
+// rows sum to zero), costing 3 decimal digits.
+__device__ __forceinline__ float tf32_rn(float x) {
+  return __uint_as_float((__float_as_uint(x) + 0x1000u) & 0xFFFFE000u);
+}
+
+__device__ __forceinline__ void split_inplace(float4* hi, float4* lo, int n4, int t, int nt) {
+  for (int i = t; i < n4; i += nt) {
+    float4 x = hi[i];
+    float4 h, l;
+    h.x = tf32_rn(x.x); l.x = tf32_rn(x.x - h.x);
+    h.y = tf32_rn(x.y); l.y = tf32_rn(x.y - h.y);
+    h.z = tf32_rn(x.z); l.z = tf32_rn(x.z - h.z);
+    h.w = tf32_rn(x.w); l.w = tf32_rn(x.w - h.w);
+    hi[i] = h;
+    lo[i] = l;
+  }
+}
+
+struct TcEpi {
+  int flags;
+  const float* bias;
+  const float* mask;
+  int64_t ld_mask;
+  int dbg;
+};
+
+template <int BN>
+struct Cfg {
+  static constexpr int kABytes = BM * BK * 4;   // 16 KB
+  static constexpr int kBBytes = BN * BK * 4;
+  static constexpr int kStageBytes = 2 * kABytes + 2 * kBBytes;
+  static constexpr int kStages = (200 * 1024) / kStageBytes >= 4 ? 4 : (200 * 1024) / kStageBytes;
+  static constexpr int kSmem = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/;
+  static constexpr int kTmemCols = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
+};
+
+// MODE 0: NN/NT (A K-major + converter, B pre-split K-major).
+// MODE 1: TN (A, B MN-major, both split in smem), split-K over blockIdx.z.
+template <int BN, int MODE>
+__global__ void __launch_bounds__(kThreads, 1)
+gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
+               const __grid_constant__ CUtensorMap tmBlo, float* __restrict__ C, int64_t ldc,
+               int64_t M, int64_t N, int64_t K, int64_t k_per_split, int n_mma, TcEpi epi) {
+  using CF = Cfg<BN>;
+  constexpr int S = CF::kStages;
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  uint8_t* stage_base = smem;
+  uint64_t* full = (uint64_t*)(smem + S * CF::kStageBytes);
+  uint64_t* conv = full + S;
+  uint64_t* empty = conv + S;
+  uint64_t* tmem_full = empty + S;
+  uint32_t* tmem_slot = (uint32_t*)(tmem_full + 1);
+
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int64_t m0 = (int64_t)blockIdx.x * BM, n0 = (int64_t)blockIdx.y * BN;
+  const int64_t kbeg = (int64_t)blockIdx.z * k_per_split;
+  const int64_t kend = min(K, kbeg + k_per_split);
+  const int nkb = (int)((kend - kbeg + BK - 1) / BK);
+
+  auto A_hi = [&](int s) { return stage_base + s * CF::kStageBytes; };
+  auto A_lo = [&](int s) { return stage_base + s * CF::kStageBytes + CF::kABytes; };
+  auto B_hi = [&](int s) { return stage_base + s * CF::kStageBytes + 2 * CF::kABytes; };
+  auto B_lo = [&](int s) { return stage_base + s * CF::kStageBytes + 2 * CF::kABytes + CF::kBBytes; };
+
+  if (threadIdx.x == 0) {
+    for (int s = 0; s < S; ++s) {
+      mbar_init(&full[s], 1);
+      mbar_init(&conv[s], 128);
+      mbar_init(&empty[s], 1);
+    }
+    mbar_init(tmem_full, 1);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 2) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(tmem_slot)),
+                 "n"(CF::kTmemCols));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+
+  if (warp == 0) {
+    if (lane == 0 && nkb > 0) {
+      const uint32_t bytes = MODE == 0 ? (CF::kABytes + 2 * CF::kBBytes) : (CF::kABytes + CF::kBBytes);
+      for (int kb = 0; kb < nkb; ++kb) {
+        const int s = kb % S;
+        if (kb >= S) mbar_wait(&empty[s], ((kb / S) - 1) & 1);
+        mbar_expect_tx(&full[s], bytes);
+        const int kc = (int)(kbeg + (int64_t)kb * BK);
+        if (MODE == 0) {
+          tma_load_2d(A_hi(s), &tmA, &full[s], kc, (int)m0);
+          tma_load_2d(B_hi(s), &tmB, &full[s], kc, (int)n0);
+          tma_load_2d(B_lo(s), &tmBlo, &full[s], kc, (int)n0);
+        } else {
+          for (int c = 0; c < BM / 32; ++c)
+            tma_load_2d(A_hi(s) + c * 4096, &tmA, &full[s], (int)m0 + 32 * c, kc);
+          for (int c = 0; c < BN / 32; ++c)
+            tma_load_2d(B_hi(s) + c * 4096, &tmB, &full[s], (int)n0 + 32 * c, kc);
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0 && nkb > 0) {
+      const uint32_t idesc = (epi.dbg & 1) ? idesc_tf32(n_mma, 0, 0) : idesc_tf32(n_mma, MODE, MODE);
+      for (int kb = 0; kb < nkb; ++kb) {
+        const int s = kb % S;
+        mbar_wait(&conv[s], (kb / S) & 1);
+        tc_fence_after();
+        const uint32_t ah = smem_u32(A_hi(s)), al = smem_u32(A_lo(s));
+        const uint32_t bh = smem_u32(B_hi(s)), bl = smem_u32(B_lo(s));
+#pragma unroll
+        for (int j = 0; j < BK / UK; ++j) {
+          uint64_t dah, dal, dbh, dbl;
+          if (MODE == 0) {  // K-major: advance 32 B along the swizzled row
+            dah = sdesc(ah + j * 32, 16, 1024);
+            dal = sdesc(al + j * 32, 16, 1024);
+            dbh = sdesc(bh + j * 32, 16, 1024);
+            dbl = sdesc(bl + j * 32, 16, 1024);
+          } else {
+            // MN-major tf32 needs the 128B swizzle with 32-byte atoms: K rows are
+            // 128-byte lines, 4-row groups 512 B apart (SBO), 32-wide MN chunks
+            // 4 KB apart (LBO); one K = 8 step spans two groups (1 KB).
+            dah = sdesc(ah + j * 1024, 4096, 512, 1);
+            dal = sdesc(al + j * 1024, 4096, 512, 1);
+            dbh = sdesc(bh + j * 1024, 4096, 512, 1);
+            dbl = sdesc(bl + j * 1024, 4096, 512, 1);
+          }
+          const uint32_t acc0 = (kb > 0 || j > 0) ? 1u : 0u;
+          tc_mma(tmem_base, dah, dbh, idesc, acc0);
+          tc_mma(tmem_base, dah, dbl, idesc, 1u);
+          tc_mma(tmem_base, dal, dbh, idesc, 1u);
+        }
+        tc_commit(&empty[s]);
+      }
+      tc_commit(tmem_full);
+    }
+  } else if (warp >= 4) {
+    const int t = threadIdx.x - 128;
+    for (int kb = 0; kb < nkb; ++kb) {
+      const int s = kb % S;
+      mbar_wait(&full[s], (kb / S) & 1);
+      if (epi.dbg & 4) { if (kb == 0) for (int i = t; i < 16 * 128; i += 128) C[i] = ((float*)A_hi(s))[i]; }
+      if (!(epi.dbg & 2)) split_inplace((float4*)A_hi(s), (float4*)A_lo(s), CF::kABytes / 16, t, 128);
+      if (MODE == 1 && !(epi.dbg & 2)) split_inplace((float4*)B_hi(s), (float4*)B_lo(s), CF::kBBytes / 16, t, 128);
+      fence_proxy_async();
+      mbar_arrive(&conv[s]);
+    }
+    // ---------------- epilogue: TMEM → registers → global
+    const int q = warp - 4;                 // TMEM lane quadrant
+    const int64_t row = m0 + q * 32 + lane;
+    if (nkb > 0) {
+      mbar_wait(tmem_full, 0);
+      tc_fence_after();
+    }
+    float* Cz = C + (int64_t)blockIdx.z * M * ldc;
+#pragma unroll 1
+    for (int c0 = 0; c0 < BN; c0 += 16) {
+      if (n0 + c0 >= N) break;
+      uint32_t r[16];
+      if (nkb > 0) {
+        tmem_ld16(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)c0, r);
+      } else {
+#pragma unroll
+        for (int i = 0; i < 16; ++i) r[i] = 0;
+      }
+      if (row < M && !(epi.dbg & 4)) {
+        float v[16];
+#pragma unroll
+        for (int i = 0; i < 16; ++i) {
+          const int64_t col = n0 + c0 + i;
+          float x = __uint_as_float(r[i]);
+          if (MODE == 0 && col < N) {
+            if (epi.flags & RDM_EPI_BIAS) x += epi.bias[col];
+            if (epi.flags & RDM_EPI_RELU) x = fmaxf(x, 0.f);
+            if ((epi.flags & RDM_EPI_MASK) && !(epi.mask[row * epi.ld_mask + col] > 0.f)) x = 0.f;
+          }
+          v[i] = x;
+        }
+        float* dst = Cz + row * ldc + n0 + c0;
+        if (n0 + c0 + 16 <= N && ((ldc & 3) == 0)) {
+#pragma unroll
+          for (int i = 0; i < 16; i += 4)
+            *reinterpret_cast<float4*>(dst + i) = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
+        } else {
+          for (int i = 0; i < 16 && n0 + c0 + i < N; ++i) dst[i] = v[i];
+        }
+      }
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
+                 "n"(CF::kTmemCols));
+  }
+}
+
+// B panels for NN / NT: Bt[n][kk] (K-major, row length ldb4) as hi and lo.
+//  NN: B[kk][n] = W[kk][n]  → Bt[n][kk] = W[kk*ldw + n]   (W is K x N)
+//  NT: B[kk][n] = W[n][kk]  → Bt[n][kk] = W[n*ldw + kk]   (W is N x K)
+__global__ void prep_b_kernel(const float* __restrict__ W, int64_t ldw, int64_t K, int64_t N,
+                              int transpose, float* __restrict__ hi, float* __restrict__ lo,
+                              int64_t ldb) {
+  const int64_t total = N * ldb;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t n = i / ldb, kk = i % ldb;
+    float x = 0.f;
+    if (kk < K) x = transpose ? W[kk * ldw + n] : W[n * ldw + kk];
+    const float h = tf32_rn(x);
+    hi[i] = h;
+    lo[i] = tf32_rn(x - h);
+  }
+}
+
+__global__ void splitk_sum(const float* __restrict__ part, int splits, int64_t M, int64_t N,
+                           int64_t ldp, float* __restrict__ C, int64_t ldc) {
+  const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (idx >= M * N) return;
+  const int64_t i = idx / N, n = idx % N;
+  float s = 0.f;
+  for (int z = 0; z < splits; ++z) s += part[(int64_t)z * M * ldp + i * ldp + n];
+  C[i * ldc + n] = s;
+}
+
+// ------------------------------------------------------------ host side
+PFN_cuTensorMapEncodeTiled_v12000 encode_fn() {
+  static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
+  if (!fn) {
+    cudaDriverEntryPointQueryResult q;
+    void* p = nullptr;
+    RDM_CUDA(cudaGetDriverEntryPoint("cuTensorMapEncodeTiled", &p, cudaEnableDefault, &q));
+    if (q != cudaDriverEntryPointSuccess || !p)
+      throw Error(RDM_ERR_CUDA, "cuTensorMapEncodeTiled unavailable");
+    fn = (PFN_cuTensorMapEncodeTiled_v12000)p;
+  }
+  return fn;
+}
+
+// 2-D fp32 tensor map: inner dim (contiguous) x outer dim, row stride ld
+// elements, box {box_inner, box_outer}, 128-byte swizzle, OOB → zeros.
+CUtensorMap make_map(const float* base, int64_t inner, int64_t outer, int64_t ld, int box_inner,
+                     int box_outer, CUtensorMapSwizzle swz = CU_TENSOR_MAP_SWIZZLE_128B) {
+  CUtensorMap m;
+  cuuint64_t dims[2] = {(cuuint64_t)inner, (cuuint64_t)outer};
+  cuuint64_t strides[1] = {(cuuint64_t)(ld * 4)};
+  cuuint32_t box[2] = {(cuuint32_t)box_inner, (cuuint32_t)box_outer};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = encode_fn()(&m, CU_TENSOR_MAP_DATA_TYPE_FLOAT32, 2, (void*)base, dims, strides, box,
+                           es, CU_TENSOR_MAP_INTERLEAVE_NONE, swz,
+                           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS)
+    throw Error(RDM_ERR_CUDA, "cuTensorMapEncodeTiled failed (" + std::to_string((int)r) + ")");
+  return m;
+}
+
+template <int BN, int MODE>
+void launch_tc(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& blo,
+               float* C, int64_t ldc, int64_t M, int64_t N, int64_t K, int splits, int n_mma,
+               const TcEpi& e) {
+  using CF = Cfg<BN>;
+  RDM_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<BN, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                                CF::kSmem));
+  const int64_t kps = ceil_div(ceil_div(K, splits), BK) * BK;
+  dim3 grid((unsigned)ceil_div(M, BM), (unsigned)ceil_div(N, BN), (unsigned)splits);
+  gemm_tc_kernel<BN, MODE><<<grid, kThreads, CF::kSmem, ctx->stream>>>(a, b, blo, C, ldc, M, N, K,
+                                                                        kps, n_mma, e);
+  RDM_LAUNCHED(ctx);
+}
+
+int pick_bn(int64_t N) {
+  if (N <= 16) return 16;
+  if (N <= 32) return 32;
+  if (N <= 64) return 64;
+  if (N <= 128) return 128;
+  return 256;
+}
+
+}  // namespace
+
+static bool g_tc_disabled = false;
+
+bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, int64_t ldw,
+             float* C, int64_t ldc, int64_t rows, int64_t k, int64_t m, int epi, const float* bias,
+             const float* mask) {
+  if (g_tc_disabled) return false;
+  // TMA: global base 16-byte aligned, row strides multiples of 16 bytes
+  if (((uintptr_t)X & 15) || (ldx & 3)) return false;
+  const char* dbgs = getenv("RDM_TC_DBG");
+  const int dbg = dbgs ? atoi(dbgs) : 0;
+  TcEpi e{epi, bias, mask, ldc, dbg};
+  if (op == RDM_GEMM_NN || op == RDM_GEMM_NT) {
+    const int64_t M = rows;
+    const int64_t N = op == RDM_GEMM_NN ? m : k;   // output columns
+    const int64_t K = op == RDM_GEMM_NN ? k : m;   // contraction
+    const int64_t ldb = roundup4(K);
+    float* bws = ensure_ws(ctx->ws_tcb, (size_t)2 * N * ldb * sizeof(float));
+    float* bhi = bws;
+    float* blo = bws + N * ldb;
+    prep_b_kernel<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(N * ldb, 256), 4096)), 256, 0,
+                    ctx->stream>>>(W, ldw, K, N, op == RDM_GEMM_NN ? 1 : 0, bhi, blo, ldb);
+    RDM_LAUNCHED(ctx);
+    const int BN = pick_bn(N);
+    // one MMA width for every tile: BN when N spans several tiles, else N rounded to 16
+    const int nm = N > BN ? BN : (int)(((N + 15) / 16) * 16);
+    const CUtensorMap ta = make_map(X, K, M, ldx, BK, BM);
+    const CUtensorMap tb = make_map(bhi, K, N, ldb, BK, BN);
+    const CUtensorMap tbl = make_map(blo, K, N, ldb, BK, BN);
+    switch (BN) {
+      case 16: launch_tc<16, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
+      case 32: launch_tc<32, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
+      case 64: launch_tc<64, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
+      case 128: launch_tc<128, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
+      default: launch_tc<256, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
+    }
+    return true;
+  }
+  // TN: C[k x m] = Xᵀ U  (X rows x k at ldx, U rows x m at ldw)
+  if (((uintptr_t)W & 15) || (ldw & 3)) return false;
+  const int64_t M = k, N = m, K = rows;
+  const int BN = N <= 32 ? 32 : N <= 64 ? 64 : N <= 128 ? 128 : 256;
+  const int n_mma = (int)std::min<int64_t>(BN, ((N + 31) / 32) * 32);
+  const int64_t tiles = ceil_div(M, BM) * ceil_div(N, BN);
+  int64_t splits = std::max<int64_t>(1, ctx->num_sms / std::max<int64_t>(1, tiles));
+  splits = std::min<int64_t>(splits, std::max<int64_t>(1, K / (8 * BK)));
+  const CUtensorMap ta = make_map(X, M, K, ldx, 32, BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B);  // inner = k
+  const CUtensorMap tb = make_map(W, N, K, ldw, 32, BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B);  // inner = m
+  float* out = C;
+  int64_t ldo = ldc;
+  if (splits > 1) {
+    ldo = roundup4(N);
+    out = ensure_ws(ctx->ws_gemm, (size_t)splits * M * ldo * sizeof(float));
+  }
+  TcEpi none{0, nullptr, nullptr, 0, dbg};
+  switch (BN) {
+    case 32: launch_tc<32, 1>(ctx, ta, tb, tb, out, ldo, M, N, K, (int)splits, n_mma, none); break;
+    case 64: launch_tc<64, 1>(ctx, ta, tb, tb, out, ldo, M, N, K, (int)splits, n_mma, none); break;
+    case 128: launch_tc<128, 1>(ctx, ta, tb, tb, out, ldo, M, N, K, (int)splits, n_mma, none); break;
+    default: launch_tc<256, 1>(ctx, ta, tb, tb, out, ldo, M, N, K, (int)splits, n_mma, none); break;
+  }
+  if (splits > 1) {
+    splitk_sum<<<(unsigned)ceil_div(M * N, 256), 256, 0, ctx->stream>>>(out, (int)splits, M, N, ldo, C,
+                                                                          ldc);
+    RDM_LAUNCHED(ctx);
+  }
+  return true;
+}
+
 }  // namespace rdm
+
+extern "C" int rdm_debug_disable_tc(int disable) {
+  rdm::g_tc_disabled = disable != 0;
+  return 0;
+}

@@ -72,38 +72,52 @@ def cora():
     return g, H0, Ws, y, m, ref
 
 
-def _check(ref, loss, dW, model, rdm, P=1, check_g0=True):
+def _gather(model, rdm, which, layer, n, width, P):
+    """Full n x width matrix of an internal tensor from whichever layout is resident."""
+    full = np.zeros((n, width))
+    for layout in (rdm.ROW, rdm.COL):
+        try:
+            parts = [model.tensor_torch(which, layer, p, layout).cpu().numpy() for p in range(P)]
+        except rdm.RdmError:
+            continue
+        for p, t in enumerate(parts):
+            if P == 1:
+                full[:] = t
+            elif layout == rdm.ROW:
+                lo, hi, _ = rdm.partition(P, rdm.ROW, n, width, p)
+                full[lo:hi] = t
+            else:
+                lo, hi, _ = rdm.partition(P, rdm.COL, n, width, p)
+                full[:, lo:hi] = t
+        return full
+    raise AssertionError(f"tensor {which}/{layer} not resident")
+
+
+def _check(prob, loss, dW, model, rdm, P=1, check_g0=True):
+    """Compare with the fp64 oracle.  The ReLU decisions 1[Z^l > 0] are taken from
+    the kernel's own fp32 forward (reading R30: a float-decided discrete value is
+    decided in the kernel's precision on both sides); everything else is fp64.
+    The forward itself (H^l, logits, loss) is compared independently."""
+    g, H0, Ws, y, m = prob
+    L = len(Ws)
+    f = [H0.shape[1]] + [w.shape[1] for w in Ws]
+    n = g.n
+    Hs = [_gather(model, rdm, rdm.T_H, l, n, f[l], P) for l in range(1, L)]
+    ref = og.epoch(g, H0, Ws, y, m, relu_masks=[h > 0 for h in Hs])
+    # forward parity (independent of the masks)
+    for l in range(1, L):
+        assert og.max_rel_err(Hs[l - 1], og.relu(ref.Z[l])) < 1e-4, ("H", l)
+    flips = sum(int(((h > 0) != (ref.Z[l + 1] > 0)).sum()) for l, h in enumerate(Hs))
+    assert flips <= max(2, 1e-4 * n * max(f)), flips
     assert abs(loss - ref.loss) <= 1e-5 * abs(ref.loss), (loss, ref.loss)
-    for l in range(len(dW)):
+    for l in range(L):
         err = og.max_rel_err(dW[l], ref.Y[l + 1])
         assert err < 1e-4, (l + 1, err)
-    L = len(dW)
-    # logits and G^0, gathered from whichever layout they live in
-    import torch
-    n = ref.Z[L].shape[0]
-    for which, layer, refm in [(rdm.T_Z, 0, ref.Z[L])] + ([(rdm.T_G, 0, ref.G[0])] if check_g0 else []):
-        full = np.zeros_like(refm)
-        for layout in (rdm.ROW, rdm.COL):
-            ok = True
-            for p in range(P):
-                try:
-                    t = model.tensor_torch(which, layer, p, layout).cpu().numpy()
-                except rdm.RdmError:
-                    ok = False
-                    break
-                if layout == rdm.ROW and P > 1:
-                    lo, hi, _ = rdm.partition(P, rdm.ROW, n, refm.shape[1], p)
-                    full[lo:hi] = t
-                elif layout == rdm.COL and P > 1:
-                    lo, hi, _ = rdm.partition(P, rdm.COL, n, refm.shape[1], p)
-                    full[:, lo:hi] = t
-                else:
-                    full[:] = t
-            if ok:
-                break
-        assert ok
-        err = og.max_rel_err(full, refm)
-        assert err < 1e-4, (which, err)
+    Z = _gather(model, rdm, rdm.T_Z, 0, n, f[L], P)
+    assert og.max_rel_err(Z, ref.Z[L]) < 1e-4
+    if check_g0:
+        G0 = _gather(model, rdm, rdm.T_G, 0, n, f[0], P)
+        assert og.max_rel_err(G0, ref.G[0]) < 1e-4
 
 
 @pytest.mark.parametrize("cfg", list(range(16)))
@@ -111,7 +125,7 @@ def test_every_config_p1(rdm, cora, cfg):
     """All 16 Table IV configurations on one GPU agree with the oracle (L323)."""
     g, H0, Ws, y, m, ref = cora
     loss, dW, model, ctx, _ = _run(rdm, g, H0, Ws, y, m, cfg)
-    _check(ref, loss, dW, model, rdm)
+    _check((g, H0, Ws, y, m), loss, dW, model, rdm)
 
 
 @pytest.mark.parametrize("P", [2, 3, 4, 8])
@@ -120,7 +134,7 @@ def test_virtual_group_configs(rdm, cora, P, cfg):
     """P ranks in one process: partitions, pack/unpack, executor and counters."""
     g, H0, Ws, y, m, ref = cora
     loss, dW, model, ctx, _ = _run(rdm, g, H0, Ws, y, m, cfg, P=P)
-    _check(ref, loss, dW, model, rdm, P=P)
+    _check((g, H0, Ws, y, m), loss, dW, model, rdm, P=P)
     info = model.info()
     c = ctx.counters()
     f = [H0.shape[1]] + [w.shape[1] for w in Ws]
@@ -142,7 +156,7 @@ def test_three_layer_products_shaped(rdm):
     for cfg in front + [0, 63]:
         for P in (1, 4):
             loss, dW, model, ctx, _ = _run(rdm, g, H0, Ws, y, m, cfg, P=P)
-            _check(ref, loss, dW, model, rdm, P=P)
+            _check((g, H0, Ws, y, m), loss, dW, model, rdm, P=P)
 
 
 def test_adam_epochs_track_oracle(rdm, cora):
@@ -155,10 +169,7 @@ def test_adam_epochs_track_oracle(rdm, cora):
     loss, dW, model, ctx, Wd = _run(rdm, g, H0, Ws, y, m, 10, P=2, epochs=3)
     Wr = [w.cpu().numpy().astype(np.float64) for w in Wd]
     assert any(not np.array_equal(Wr[l], Ws[l]) for l in range(2))
-    r = og.epoch(g, H0, Wr, y, m)
-    assert abs(loss - r.loss) <= 1e-5 * abs(r.loss)
-    for l in range(2):
-        assert og.max_rel_err(dW[l], r.Y[l + 1]) < 1e-4
+    _check((g, H0, Wr, y, m), loss, dW, model, rdm, P=2)
 
 
 def test_epoch_deterministic(rdm, cora):

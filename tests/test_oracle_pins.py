@@ -239,3 +239,18 @@ def test_symmetric_rmat_properties():
     assert abs(A - A.T).max() == 0
     assert np.all(A.diagonal() > 0)
     assert np.all(np.diff(g.col[g.rowptr[0]:g.rowptr[1]]) > 0)
+
+
+def test_relu_masks_default_equivalence():
+    """Passing the oracle's own decisions 1[Z^l > 0] as relu_masks changes nothing."""
+    n, f = 50, (6, 5, 4, 3)
+    g = synth.rmat(n, 150, seed=2)
+    H0 = synth.features(n, f[0])
+    Ws = synth.weights(f)
+    y = synth.labels(n, f[-1])
+    m = synth.train_mask(n)
+    a = gcn.epoch(g, H0, Ws, y, m)
+    b = gcn.epoch(g, H0, Ws, y, m, relu_masks=[a.Z[1] > 0, a.Z[2] > 0])
+    for l in (1, 2, 3):
+        assert np.array_equal(a.Y[l], b.Y[l])
+    assert np.array_equal(a.G[0], b.G[0])
