@@ -599,9 +599,16 @@ void do_set_input(void* a_) {
   for (int i = 0; i < nl; ++i) {
     const int64_t r = row_range(n, P, ctx->local[i]).size();
     Buf& h = buf(g, i, {K_H, 0}, RDM_ROW);
-    if (r && f0)
-      RDM_CUDA(cudaMemcpy2DAsync(h.p, h.ld * sizeof(float), a->H0[i], f0 * sizeof(float),
-                                 f0 * sizeof(float), r, kind, ctx->stream));
+    if (r && f0) {
+      if (h.ld == f0) {
+        RDM_CUDA(cudaMemcpyAsync(h.p, a->H0[i], r * f0 * sizeof(float), kind, ctx->stream));
+      } else {
+        // one contiguous (DMA-friendly) copy, then re-pitch to ld on the device
+        float* stage = ensure_ws(ctx->ws_stage, (size_t)r * f0 * sizeof(float));
+        RDM_CUDA(cudaMemcpyAsync(stage, a->H0[i], r * f0 * sizeof(float), kind, ctx->stream));
+        copy_2d(ctx, h.p, h.ld, stage, f0, r, f0);
+      }
+    }
     if (r) {
       RDM_CUDA(cudaMemcpyAsync(g->labels[i], a->labels[i], r * sizeof(int32_t), kind, ctx->stream));
       if (a->mask && a->mask[i])

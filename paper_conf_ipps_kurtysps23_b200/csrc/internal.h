@@ -114,6 +114,7 @@ struct rdm_ctx {
   std::unique_ptr<rdm::DevBuf> ws_seg;                         // SpMM heavy-row partials
   std::unique_ptr<rdm::DevBuf> ws_gemm;                        // GEMM split-K partials
   std::unique_ptr<rdm::DevBuf> ws_tcb;                         // tcgen05 B panels (hi | lo)
+  std::unique_ptr<rdm::DevBuf> ws_stage;                       // host-input staging
   std::unique_ptr<rdm::DevBuf> ws_scratch;
   // phase timing
   bool timing = false;

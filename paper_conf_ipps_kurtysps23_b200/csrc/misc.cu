@@ -243,6 +243,25 @@ void adam(rdm_ctx* ctx, float* p, const float* g, float* m, float* v, int64_t n,
   RDM_LAUNCHED(ctx);
 }
 
+__global__ void copy_2d_kernel(float* __restrict__ dst, int64_t ldd, const float* __restrict__ src,
+                               int64_t lds, int64_t rows, int64_t cols) {
+  const int64_t total = rows * cols;
+  for (int64_t g = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; g < total;
+       g += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = g / cols, c = g % cols;
+    dst[r * ldd + c] = src[r * lds + c];
+  }
+}
+
+void copy_2d(rdm_ctx* ctx, float* dst, int64_t ldd, const float* src, int64_t lds, int64_t rows,
+             int64_t cols) {
+  if (rows * cols == 0) return;
+  const int64_t want = ceil_div(rows * cols, 256);
+  const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(want, (int64_t)ctx->num_sms * 16));
+  copy_2d_kernel<<<grid, 256, 0, ctx->stream>>>(dst, ldd, src, lds, rows, cols);
+  RDM_LAUNCHED(ctx);
+}
+
 int validate_csr(rdm_ctx* ctx, const int64_t* rowptr, const int32_t* col, int64_t n, int64_t nnz) {
   int* flag = reinterpret_cast<int*>(ensure_ws(ctx->ws_scratch, 64));
   RDM_CUDA(cudaMemsetAsync(flag, 0, sizeof(int), ctx->stream));

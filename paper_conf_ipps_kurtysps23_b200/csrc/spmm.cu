@@ -60,54 +60,71 @@ __device__ __forceinline__ float4 apply_epi(float4 a, const Epi& e, int64_t row,
   return a;
 }
 
-// Warp computes Σ_{j in [beg,end)} val[j] · X[col[j], c0 + sub*4 .. +4];
-// result valid in every lane of group 0 (lanes 0..G-1) after the reduction.
-template <int G>
-__device__ __forceinline__ float4 warp_nnz_range(const int32_t* __restrict__ col,
-                                                 const float* __restrict__ val,
-                                                 const float* __restrict__ X, int64_t ldx,
-                                                 int64_t beg, int64_t end, int lane, bool col_ok,
-                                                 int64_t cbase) {
+// Warp computes Σ_{j in [beg,end)} val[j] · X[col[j], chunk columns].  A group
+// of G lanes owns one nnz at a time; lane `sub` of the group loads float4
+// chunks sub, sub+G, …, sub+(V-1)G of the row chunk (each warp-level load is a
+// contiguous 16·G-byte run per group), so 32/G nnz are in flight per step and
+// every lane issues V independent 128-bit gathers per nnz.  (col, val) of 32
+// nnz are loaded once per batch, coalesced, and broadcast with shuffles (none
+// when G = 1).  Result: lanes of group 0 hold the row-chunk sum.
+template <int G, int V>
+__device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
+                                               const float* __restrict__ val,
+                                               const float* __restrict__ xb, int64_t ldx,
+                                               int64_t beg, int64_t end, int lane, int c4n,
+                                               float4 (&acc)[V]) {
   constexpr int NG = 32 / G;
-  const int g = lane / G;
-  float4 acc = make_float4(0.f, 0.f, 0.f, 0.f);
-  const float* xb = X + cbase;
+  const int g = lane / G, sub = lane % G;
+#pragma unroll
+  for (int v = 0; v < V; ++v) acc[v] = make_float4(0.f, 0.f, 0.f, 0.f);
   for (int64_t base = beg; base < end; base += 32) {
     const int64_t j = base + lane;
     int c = 0;
-    float v = 0.f;
+    float a = 0.f;
     if (j < end) {
       c = __ldcs(col + j);
-      v = __ldcs(val + j);
+      a = __ldcs(val + j);
     }
     const int cnt = (end - base) < 32 ? (int)(end - base) : 32;
 #pragma unroll
     for (int t = 0; t < G; ++t) {
       const int k = t * NG + g;
-      const int cc = __shfl_sync(kFull, c, k);
-      const float vv = __shfl_sync(kFull, v, k);
-      if (k < cnt && col_ok) {
-        const float4 x = __ldg(reinterpret_cast<const float4*>(xb + (int64_t)cc * ldx));
-        acc.x = fmaf(vv, x.x, acc.x);
-        acc.y = fmaf(vv, x.y, acc.y);
-        acc.z = fmaf(vv, x.z, acc.z);
-        acc.w = fmaf(vv, x.w, acc.w);
+      const int cc = (G == 1) ? c : __shfl_sync(kFull, c, k);
+      const float vv = (G == 1) ? a : __shfl_sync(kFull, a, k);
+      if (k < cnt) {
+        const float4* xr = reinterpret_cast<const float4*>(xb + (int64_t)cc * ldx);
+        float4 x[V];
+#pragma unroll
+        for (int v = 0; v < V; ++v)
+          if (v * G + sub < c4n) x[v] = __ldg(xr + v * G + sub);
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          if (v * G + sub < c4n) {
+            acc[v].x = fmaf(vv, x[v].x, acc[v].x);
+            acc[v].y = fmaf(vv, x[v].y, acc[v].y);
+            acc[v].z = fmaf(vv, x[v].z, acc[v].z);
+            acc[v].w = fmaf(vv, x[v].w, acc[v].w);
+          }
+        }
       }
     }
   }
 #pragma unroll
   for (int off = G; off < 32; off <<= 1) {
-    acc.x += __shfl_xor_sync(kFull, acc.x, off);
-    acc.y += __shfl_xor_sync(kFull, acc.y, off);
-    acc.z += __shfl_xor_sync(kFull, acc.z, off);
-    acc.w += __shfl_xor_sync(kFull, acc.w, off);
+#pragma unroll
+    for (int v = 0; v < V; ++v) {
+      acc[v].x += __shfl_xor_sync(kFull, acc[v].x, off);
+      acc[v].y += __shfl_xor_sync(kFull, acc[v].y, off);
+      acc[v].z += __shfl_xor_sync(kFull, acc[v].z, off);
+      acc[v].w += __shfl_xor_sync(kFull, acc[v].w, off);
+    }
   }
-  return acc;
 }
 
 // One warp per work item: items [0, n_seg) are heavy-row segments (partial
 // rows to `part`), items [n_seg, n_seg + n_light) are light rows (to out).
-template <int G>
+// blockIdx.y selects a 128-column chunk of the slice.
+template <int G, int V>
 __global__ void __launch_bounds__(kWarps * 32)
 spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
             const float* __restrict__ val, const int32_t* __restrict__ light_rows,
@@ -118,19 +135,35 @@ spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
   const int lane = threadIdx.x & 31;
   const int64_t item = (int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5);
   if (item >= n_seg + n_light) return;
-  const int64_t c = (int64_t)blockIdx.y * (4 * G) + (lane % G) * 4;  // this lane's first column
-  const bool col_ok = c < w4;
+  const int64_t cbase = (int64_t)blockIdx.y * 128;             // first column of the chunk
+  const int64_t rem4 = (w4 - cbase) / 4;
+  const int c4n = rem4 < 32 ? (int)rem4 : 32;                  // float4 chunks in this chunk
+  const int sub = lane % G;
+  float4 acc[V];
+  int32_t r;
   if (item < n_seg) {
-    const int32_t r = seg_row[item];
+    r = seg_row[item];
     const int64_t beg = seg_start[item];
     const int64_t end = min(beg + kSeg, rowptr[r + 1]);
-    const float4 acc = warp_nnz_range<G>(col, val, X, ldx, beg, end, lane, col_ok, c);
-    if (lane < G && col_ok) *reinterpret_cast<float4*>(part + item * ld_part + c) = acc;
+    warp_nnz_range<G, V>(col, val, X + cbase, ldx, beg, end, lane, c4n, acc);
+    if (lane < G) {
+      float* dst = part + item * ld_part + cbase;
+#pragma unroll
+      for (int v = 0; v < V; ++v)
+        if (v * G + sub < c4n) reinterpret_cast<float4*>(dst)[v * G + sub] = acc[v];
+    }
   } else {
-    const int32_t r = light_rows[item - n_seg];
-    const float4 acc = warp_nnz_range<G>(col, val, X, ldx, rowptr[r], rowptr[r + 1], lane, col_ok, c);
-    if (lane < G && col_ok)
-      *reinterpret_cast<float4*>(out + (int64_t)r * ld_out + c) = apply_epi(acc, epi, r, c);
+    r = light_rows[item - n_seg];
+    warp_nnz_range<G, V>(col, val, X + cbase, ldx, rowptr[r], rowptr[r + 1], lane, c4n, acc);
+    if (lane < G) {
+      float* dst = out + (int64_t)r * ld_out + cbase;
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        const int ch = v * G + sub;
+        if (ch < c4n)
+          reinterpret_cast<float4*>(dst)[ch] = apply_epi(acc[v], epi, r, cbase + 4 * ch);
+      }
+    }
   }
 }
 
@@ -152,20 +185,39 @@ __global__ void spmm_heavy_reduce(const int32_t* __restrict__ heavy_rows,
   }
 }
 
-template <int G>
+template <int G, int V>
 void launch_spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out,
                  int64_t ld_out, float* part, int64_t ld_part, int64_t w4, const Epi& epi) {
   const int64_t items = A.n_seg + A.n_light;
   if (items == 0) return;
-  const int64_t chunks = ceil_div(w4, 4 * G);
+  const int64_t chunks = ceil_div(w4, 128);
   dim3 grid((unsigned)ceil_div(items, kWarps), (unsigned)chunks);
-  spmm_kernel<G><<<grid, kWarps * 32, 0, ctx->stream>>>(
+  spmm_kernel<G, V><<<grid, kWarps * 32, 0, ctx->stream>>>(
       A.rowptr->as<int64_t>(), A.col->as<int32_t>(), A.val->as<float>(),
-      A.light_rows ? A.light_rows->as<int32_t>() : nullptr,
-      A.seg_start ? A.seg_start->as<int64_t>() : nullptr,
-      A.heavy_rows ? reinterpret_cast<const int32_t*>(A.seg_start->as<int64_t>() + A.n_seg) : nullptr,
-      A.n_light, A.n_seg, in, ld_in, out, ld_out, part, ld_part, w4, epi);
+      A.light_rows->as<int32_t>(), A.seg_start->as<int64_t>(),
+      reinterpret_cast<const int32_t*>(A.seg_start->as<int64_t>() + A.n_seg), A.n_light, A.n_seg,
+      in, ld_in, out, ld_out, part, ld_part, w4, epi);
   RDM_LAUNCHED(ctx);
+}
+
+// (G, V) for a chunk of c4 float4 columns: fewest lane slots G·V ≥ c4, ties to
+// the G closest to 8 (short reductions, several nnz in flight).
+void pick_gv(int c4, int* G, int* V) {
+  int best_s = 1 << 30, bg = 32, bv = 1;
+  for (int v = 1; v <= 4; ++v) {
+    int g = 1;
+    while (g * v < c4) g <<= 1;
+    if (g > 32) continue;
+    const int s = g * v;
+    const int d = g > 8 ? g / 8 : 8 / g, bd = bg > 8 ? bg / 8 : 8 / bg;
+    if (s < best_s || (s == best_s && d < bd)) {
+      best_s = s;
+      bg = g;
+      bv = v;
+    }
+  }
+  *G = bg;
+  *V = bv;
 }
 
 }  // namespace
@@ -186,17 +238,21 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
   Epi epi{epi_flags, bias, mask, ld_mask, w};
   float* part = nullptr;
   if (A.n_seg) part = ensure_ws(ctx->ws_seg, (size_t)A.n_seg * w4 * sizeof(float));
-  const int64_t w4c = w4;
-  const int64_t g_need = std::min<int64_t>(w4 / 4, 32);
-  if (g_need <= 1)       launch_spmm<1>(ctx, A, in, ld_in, out, ld_out, part, w4, w4c, epi);
-  else if (g_need <= 2)  launch_spmm<2>(ctx, A, in, ld_in, out, ld_out, part, w4, w4c, epi);
-  else if (g_need <= 4)  launch_spmm<4>(ctx, A, in, ld_in, out, ld_out, part, w4, w4c, epi);
-  else if (g_need <= 8)  launch_spmm<8>(ctx, A, in, ld_in, out, ld_out, part, w4, w4c, epi);
-  else if (g_need <= 16) launch_spmm<16>(ctx, A, in, ld_in, out, ld_out, part, w4, w4c, epi);
-  else                   launch_spmm<32>(ctx, A, in, ld_in, out, ld_out, part, w4, w4c, epi);
+  int G, V;
+  pick_gv((int)std::min<int64_t>(32, w4 / 4), &G, &V);
+#define RDM_SPMM_CASE(g_, v_) \
+  if (G == g_ && V == v_) launch_spmm<g_, v_>(ctx, A, in, ld_in, out, ld_out, part, w4, w4, epi); else
+  RDM_SPMM_CASE(1, 1) RDM_SPMM_CASE(1, 2) RDM_SPMM_CASE(1, 3) RDM_SPMM_CASE(1, 4)
+  RDM_SPMM_CASE(2, 1) RDM_SPMM_CASE(2, 2) RDM_SPMM_CASE(2, 3) RDM_SPMM_CASE(2, 4)
+  RDM_SPMM_CASE(4, 1) RDM_SPMM_CASE(4, 2) RDM_SPMM_CASE(4, 3) RDM_SPMM_CASE(4, 4)
+  RDM_SPMM_CASE(8, 1) RDM_SPMM_CASE(8, 2) RDM_SPMM_CASE(8, 3) RDM_SPMM_CASE(8, 4)
+  RDM_SPMM_CASE(16, 1) RDM_SPMM_CASE(16, 2) RDM_SPMM_CASE(16, 3) RDM_SPMM_CASE(16, 4)
+  RDM_SPMM_CASE(32, 1)
+  throw Error(RDM_ERR_STATE, "spmm: no kernel for G/V");
+#undef RDM_SPMM_CASE
   if (A.n_heavy) {
     spmm_heavy_reduce<<<(unsigned)A.n_heavy, 128, 0, ctx->stream>>>(
-        A.heavy_rows->as<int32_t>(), A.heavy_seg->as<int32_t>(), part, w4, out, ld_out, w4c, epi);
+        A.heavy_rows->as<int32_t>(), A.heavy_seg->as<int32_t>(), part, w4, out, ld_out, w4, epi);
     RDM_LAUNCHED(ctx);
   }
   ctx->counters.spmm_calls++;
