@@ -38,7 +38,6 @@ namespace {
 constexpr int BM = 128;        // UMMA M (cta_group::1)
 constexpr int BK = 32;         // fp32 elements per 128-byte swizzle row
 constexpr int UK = 8;          // UMMA K for kind::tf32
-constexpr int kThreads = 256;
 
 // ------------------------------------------------------------ PTX wrappers
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -148,12 +147,29 @@ __device__ __forceinline__ void split_inplace(float4* hi, float4* lo, int n4, in
   }
 }
 
+__device__ __forceinline__ void tmem_ld32(uint32_t addr, uint32_t (&r)[32]) {
+  asm volatile(
+      "tcgen05.ld.sync.aligned.32x32b.x32.b32 {%0,%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,"
+      "%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31}, [%32];"
+      : "=r"(r[0]), "=r"(r[1]), "=r"(r[2]), "=r"(r[3]), "=r"(r[4]), "=r"(r[5]), "=r"(r[6]),
+        "=r"(r[7]), "=r"(r[8]), "=r"(r[9]), "=r"(r[10]), "=r"(r[11]), "=r"(r[12]), "=r"(r[13]),
+        "=r"(r[14]), "=r"(r[15]), "=r"(r[16]), "=r"(r[17]), "=r"(r[18]), "=r"(r[19]), "=r"(r[20]),
+        "=r"(r[21]), "=r"(r[22]), "=r"(r[23]), "=r"(r[24]), "=r"(r[25]), "=r"(r[26]), "=r"(r[27]),
+        "=r"(r[28]), "=r"(r[29]), "=r"(r[30]), "=r"(r[31])
+      : "r"(addr));
+  asm volatile("tcgen05.wait::ld.sync.aligned;" ::: "memory");
+}
+
 struct TcEpi {
   int flags;
   const float* bias;
   const float* mask;
   int64_t ld_mask;
-  int dbg;
+};
+
+struct TcShape {
+  int64_t M, N, K, k_per_split;
+  int tiles_m, tiles_n, splits, n_mma;
 };
 
 template <int BN>
@@ -161,39 +177,57 @@ struct Cfg {
   static constexpr int kABytes = BM * BK * 4;   // 16 KB
   static constexpr int kBBytes = BN * BK * 4;
   static constexpr int kStageBytes = 2 * kABytes + 2 * kBBytes;
-  static constexpr int kStages = (200 * 1024) / kStageBytes >= 4 ? 4 : (200 * 1024) / kStageBytes;
-  static constexpr int kSmem = kStages * kStageBytes + 1024 /*align*/ + 256 /*barriers*/;
-  static constexpr int kTmemCols = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
+  static constexpr int kEpiBytes = 4 * 32 * 33 * 4;   // per-warp 32 x 32 transpose tiles (+1 pad)
+  static constexpr int kBudget = 224 * 1024 - kEpiBytes - 1024 - 256;
+  static constexpr int kStages = kBudget / kStageBytes >= 4 ? 4 : kBudget / kStageBytes;
+  static constexpr int kSmem = kStages * kStageBytes + kEpiBytes + 1024 /*align*/ + 256 /*barriers*/;
+  static constexpr int kAccCols = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
+  static constexpr int kTmemCols = 2 * kAccCols;      // double-buffered accumulator
 };
 
+// Persistent, warp-specialised tcgen05 GEMM.  384 threads:
+//   warp 0      TMA producer           warp 1  MMA issuer (one thread)
+//   warp 2      TMEM allocator         warp 3  idle
+//   warps 4-7   3xTF32 split converter (in-place hi, lo twin buffer)
+//   warps 8-11  epilogue: TMEM → registers → smem transpose → coalesced
+//               global stores with fused bias / ReLU / Hadamard mask
+// Tiles (m, n, split) are strided over the grid; the smem ring runs across
+// tiles and the TMEM accumulator is double-buffered, so the epilogue of tile i
+// overlaps the mainloop of tile i + 1.
 // MODE 0: NN/NT (A K-major + converter, B pre-split K-major).
-// MODE 1: TN (A, B MN-major, both split in smem), split-K over blockIdx.z.
+// MODE 1: TN (A, B MN-major, both split in smem), split-K slabs.
 template <int BN, int MODE>
-__global__ void __launch_bounds__(kThreads, 1)
+__global__ void __launch_bounds__(384, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const __grid_constant__ CUtensorMap tmBlo, float* __restrict__ C, int64_t ldc,
-               int64_t M, int64_t N, int64_t K, int64_t k_per_split, int n_mma, TcEpi epi) {
+               TcShape sh, TcEpi epi) {
   using CF = Cfg<BN>;
   constexpr int S = CF::kStages;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint8_t* stage_base = smem;
-  uint64_t* full = (uint64_t*)(smem + S * CF::kStageBytes);
+  float* epi_smem = (float*)(smem + S * CF::kStageBytes);
+  uint64_t* full = (uint64_t*)(smem + S * CF::kStageBytes + CF::kEpiBytes);
   uint64_t* conv = full + S;
   uint64_t* empty = conv + S;
-  uint64_t* tmem_full = empty + S;
-  uint32_t* tmem_slot = (uint32_t*)(tmem_full + 1);
+  uint64_t* tfull = empty + S;   // [2]
+  uint64_t* tempty = tfull + 2;  // [2]
+  uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int64_t m0 = (int64_t)blockIdx.x * BM, n0 = (int64_t)blockIdx.y * BN;
-  const int64_t kbeg = (int64_t)blockIdx.z * k_per_split;
-  const int64_t kend = min(K, kbeg + k_per_split);
-  const int nkb = (int)((kend - kbeg + BK - 1) / BK);
+  const int tiles_mn = sh.tiles_m * sh.tiles_n;
+  const int total = tiles_mn * sh.splits;
 
   auto A_hi = [&](int s) { return stage_base + s * CF::kStageBytes; };
   auto A_lo = [&](int s) { return stage_base + s * CF::kStageBytes + CF::kABytes; };
   auto B_hi = [&](int s) { return stage_base + s * CF::kStageBytes + 2 * CF::kABytes; };
   auto B_lo = [&](int s) { return stage_base + s * CF::kStageBytes + 2 * CF::kABytes + CF::kBBytes; };
+  auto tile_kb = [&](int t, int64_t& kbeg) {
+    const int z = t / tiles_mn;
+    kbeg = (int64_t)z * sh.k_per_split;
+    const int64_t kend = min(sh.K, kbeg + sh.k_per_split);
+    return kend > kbeg ? (int)((kend - kbeg + BK - 1) / BK) : 0;
+  };
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
@@ -201,7 +235,10 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       mbar_init(&conv[s], 128);
       mbar_init(&empty[s], 1);
     }
-    mbar_init(tmem_full, 1);
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&tfull[b], 1);
+      mbar_init(&tempty[b], 128);
+    }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 2) {
@@ -216,111 +253,162 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   const uint32_t tmem_base = *tmem_slot;
 
   if (warp == 0) {
-    if (lane == 0 && nkb > 0) {
+    if (lane == 0) {
       const uint32_t bytes = MODE == 0 ? (CF::kABytes + 2 * CF::kBBytes) : (CF::kABytes + CF::kBBytes);
-      for (int kb = 0; kb < nkb; ++kb) {
-        const int s = kb % S;
-        if (kb >= S) mbar_wait(&empty[s], ((kb / S) - 1) & 1);
-        mbar_expect_tx(&full[s], bytes);
-        const int kc = (int)(kbeg + (int64_t)kb * BK);
-        if (MODE == 0) {
-          tma_load_2d(A_hi(s), &tmA, &full[s], kc, (int)m0);
-          tma_load_2d(B_hi(s), &tmB, &full[s], kc, (int)n0);
-          tma_load_2d(B_lo(s), &tmBlo, &full[s], kc, (int)n0);
-        } else {
-          for (int c = 0; c < BM / 32; ++c)
-            tma_load_2d(A_hi(s) + c * 4096, &tmA, &full[s], (int)m0 + 32 * c, kc);
-          for (int c = 0; c < BN / 32; ++c)
-            tma_load_2d(B_hi(s) + c * 4096, &tmB, &full[s], (int)n0 + 32 * c, kc);
+      uint32_t kc = 0;
+      for (int t = blockIdx.x; t < total; t += gridDim.x) {
+        int64_t kbeg;
+        const int nkb = tile_kb(t, kbeg);
+        const int rem = t % tiles_mn;
+        const int m0 = (rem / sh.tiles_n) * BM, n0 = (rem % sh.tiles_n) * BN;
+        for (int kb = 0; kb < nkb; ++kb, ++kc) {
+          const int s = kc % S;
+          if (kc >= (uint32_t)S) mbar_wait(&empty[s], ((kc / S) - 1) & 1);
+          mbar_expect_tx(&full[s], bytes);
+          const int kk = (int)(kbeg + (int64_t)kb * BK);
+          if (MODE == 0) {
+            tma_load_2d(A_hi(s), &tmA, &full[s], kk, m0);
+            tma_load_2d(B_hi(s), &tmB, &full[s], kk, n0);
+            tma_load_2d(B_lo(s), &tmBlo, &full[s], kk, n0);
+          } else {
+            for (int c = 0; c < BM / 32; ++c) tma_load_2d(A_hi(s) + c * 4096, &tmA, &full[s], m0 + 32 * c, kk);
+            for (int c = 0; c < BN / 32; ++c) tma_load_2d(B_hi(s) + c * 4096, &tmB, &full[s], n0 + 32 * c, kk);
+          }
         }
       }
     }
   } else if (warp == 1) {
-    if (lane == 0 && nkb > 0) {
-      const uint32_t idesc = (epi.dbg & 1) ? idesc_tf32(n_mma, 0, 0) : idesc_tf32(n_mma, MODE, MODE);
-      for (int kb = 0; kb < nkb; ++kb) {
-        const int s = kb % S;
-        mbar_wait(&conv[s], (kb / S) & 1);
+    if (lane == 0) {
+      const uint32_t idesc = idesc_tf32(sh.n_mma, MODE, MODE);
+      uint32_t kc = 0;
+      int it = 0;
+      for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
+        int64_t kbeg;
+        const int nkb = tile_kb(t, kbeg);
+        const int acc = it & 1;
+        if (it >= 2) mbar_wait(&tempty[acc], ((it >> 1) - 1) & 1);
         tc_fence_after();
-        const uint32_t ah = smem_u32(A_hi(s)), al = smem_u32(A_lo(s));
-        const uint32_t bh = smem_u32(B_hi(s)), bl = smem_u32(B_lo(s));
+        const uint32_t d_tmem = tmem_base + acc * CF::kAccCols;
+        for (int kb = 0; kb < nkb; ++kb, ++kc) {
+          const int s = kc % S;
+          mbar_wait(&conv[s], (kc / S) & 1);
+          tc_fence_after();
+          const uint32_t ah = smem_u32(A_hi(s)), al = smem_u32(A_lo(s));
+          const uint32_t bh = smem_u32(B_hi(s)), bl = smem_u32(B_lo(s));
 #pragma unroll
-        for (int j = 0; j < BK / UK; ++j) {
-          uint64_t dah, dal, dbh, dbl;
-          if (MODE == 0) {  // K-major: advance 32 B along the swizzled row
-            dah = sdesc(ah + j * 32, 16, 1024);
-            dal = sdesc(al + j * 32, 16, 1024);
-            dbh = sdesc(bh + j * 32, 16, 1024);
-            dbl = sdesc(bl + j * 32, 16, 1024);
-          } else {
-            // MN-major tf32 needs the 128B swizzle with 32-byte atoms: K rows are
-            // 128-byte lines, 4-row groups 512 B apart (SBO), 32-wide MN chunks
-            // 4 KB apart (LBO); one K = 8 step spans two groups (1 KB).
-            dah = sdesc(ah + j * 1024, 4096, 512, 1);
-            dal = sdesc(al + j * 1024, 4096, 512, 1);
-            dbh = sdesc(bh + j * 1024, 4096, 512, 1);
-            dbl = sdesc(bl + j * 1024, 4096, 512, 1);
+          for (int j = 0; j < BK / UK; ++j) {
+            uint64_t dah, dal, dbh, dbl;
+            if (MODE == 0) {  // K-major: advance 32 B along the swizzled row
+              dah = sdesc(ah + j * 32, 16, 1024);
+              dal = sdesc(al + j * 32, 16, 1024);
+              dbh = sdesc(bh + j * 32, 16, 1024);
+              dbl = sdesc(bl + j * 32, 16, 1024);
+            } else {
+              // MN-major tf32 needs the 128B swizzle with 32-byte atoms: K rows are
+              // 128-byte lines, 4-row groups 512 B apart (SBO), 32-wide MN chunks
+              // 4 KB apart (LBO); one K = 8 step spans two groups (1 KB).
+              dah = sdesc(ah + j * 1024, 4096, 512, 1);
+              dal = sdesc(al + j * 1024, 4096, 512, 1);
+              dbh = sdesc(bh + j * 1024, 4096, 512, 1);
+              dbl = sdesc(bl + j * 1024, 4096, 512, 1);
+            }
+            const uint32_t acc0 = (kb > 0 || j > 0) ? 1u : 0u;
+            tc_mma(d_tmem, dah, dbh, idesc, acc0);
+            tc_mma(d_tmem, dah, dbl, idesc, 1u);
+            tc_mma(d_tmem, dal, dbh, idesc, 1u);
           }
-          const uint32_t acc0 = (kb > 0 || j > 0) ? 1u : 0u;
-          tc_mma(tmem_base, dah, dbh, idesc, acc0);
-          tc_mma(tmem_base, dah, dbl, idesc, 1u);
-          tc_mma(tmem_base, dal, dbh, idesc, 1u);
+          tc_commit(&empty[s]);
         }
-        tc_commit(&empty[s]);
+        tc_commit(&tfull[acc]);   // fires when this tile's MMAs (if any) are done
       }
-      tc_commit(tmem_full);
     }
-  } else if (warp >= 4) {
-    const int t = threadIdx.x - 128;
-    for (int kb = 0; kb < nkb; ++kb) {
-      const int s = kb % S;
-      mbar_wait(&full[s], (kb / S) & 1);
-      if (epi.dbg & 4) { if (kb == 0) for (int i = t; i < 16 * 128; i += 128) C[i] = ((float*)A_hi(s))[i]; }
-      if (!(epi.dbg & 2)) split_inplace((float4*)A_hi(s), (float4*)A_lo(s), CF::kABytes / 16, t, 128);
-      if (MODE == 1 && !(epi.dbg & 2)) split_inplace((float4*)B_hi(s), (float4*)B_lo(s), CF::kBBytes / 16, t, 128);
-      fence_proxy_async();
-      mbar_arrive(&conv[s]);
+  } else if (warp >= 4 && warp < 8) {
+    const int t128 = threadIdx.x - 128;
+    uint32_t kc = 0;
+    for (int t = blockIdx.x; t < total; t += gridDim.x) {
+      int64_t kbeg;
+      const int nkb = tile_kb(t, kbeg);
+      for (int kb = 0; kb < nkb; ++kb, ++kc) {
+        const int s = kc % S;
+        mbar_wait(&full[s], (kc / S) & 1);
+        split_inplace((float4*)A_hi(s), (float4*)A_lo(s), CF::kABytes / 16, t128, 128);
+        if (MODE == 1) split_inplace((float4*)B_hi(s), (float4*)B_lo(s), CF::kBBytes / 16, t128, 128);
+        fence_proxy_async();
+        mbar_arrive(&conv[s]);
+      }
     }
-    // ---------------- epilogue: TMEM → registers → global
-    const int q = warp - 4;                 // TMEM lane quadrant
-    const int64_t row = m0 + q * 32 + lane;
-    if (nkb > 0) {
-      mbar_wait(tmem_full, 0);
+  } else if (warp >= 8) {
+    const int q = warp - 8;                    // TMEM lane quadrant of this warp
+    float* tb = epi_smem + q * 32 * 33;        // 32 x 32 transpose tile
+    int it = 0;
+    for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
+      int64_t kbeg;
+      const int nkb = tile_kb(t, kbeg);
+      const int z = t / tiles_mn, rem = t % tiles_mn;
+      const int64_t m0 = (int64_t)(rem / sh.tiles_n) * BM, n0 = (int64_t)(rem % sh.tiles_n) * BN;
+      const int acc = it & 1;
+      mbar_wait(&tfull[acc], (it >> 1) & 1);
       tc_fence_after();
-    }
-    float* Cz = C + (int64_t)blockIdx.z * M * ldc;
+      float* Cz = C + (int64_t)z * sh.M * ldc;
+      const int64_t row0 = m0 + q * 32;
 #pragma unroll 1
-    for (int c0 = 0; c0 < BN; c0 += 16) {
-      if (n0 + c0 >= N) break;
-      uint32_t r[16];
-      if (nkb > 0) {
-        tmem_ld16(tmem_base + ((uint32_t)(q * 32) << 16) + (uint32_t)c0, r);
-      } else {
-#pragma unroll
-        for (int i = 0; i < 16; ++i) r[i] = 0;
-      }
-      if (row < M && !(epi.dbg & 4)) {
-        float v[16];
-#pragma unroll
-        for (int i = 0; i < 16; ++i) {
-          const int64_t col = n0 + c0 + i;
-          float x = __uint_as_float(r[i]);
-          if (MODE == 0 && col < N) {
-            if (epi.flags & RDM_EPI_BIAS) x += epi.bias[col];
-            if (epi.flags & RDM_EPI_RELU) x = fmaxf(x, 0.f);
-            if ((epi.flags & RDM_EPI_MASK) && !(epi.mask[row * epi.ld_mask + col] > 0.f)) x = 0.f;
-          }
-          v[i] = x;
-        }
-        float* dst = Cz + row * ldc + n0 + c0;
-        if (n0 + c0 + 16 <= N && ((ldc & 3) == 0)) {
-#pragma unroll
-          for (int i = 0; i < 16; i += 4)
-            *reinterpret_cast<float4*>(dst + i) = make_float4(v[i], v[i + 1], v[i + 2], v[i + 3]);
+      for (int c0 = 0; c0 < BN; c0 += 32) {
+        if (n0 + c0 >= sh.N) break;
+        uint32_t r[32];
+        if (nkb > 0) {
+          tmem_ld32(tmem_base + acc * CF::kAccCols + ((uint32_t)(q * 32) << 16) + (uint32_t)c0, r);
         } else {
-          for (int i = 0; i < 16 && n0 + c0 + i < N; ++i) dst[i] = v[i];
+#pragma unroll
+          for (int i = 0; i < 32; ++i) r[i] = 0;
         }
+        // lane owns row (row0 + lane): epilogue in registers — the mask row
+        // segment is read as 8 independent 128-bit loads per lane — then
+        // transpose through smem and write column-coalesced.
+        if (MODE == 0 && epi.flags) {
+          const int64_t row = row0 + lane;
+          float v[32];
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
+          if (epi.flags & RDM_EPI_BIAS) {
+#pragma unroll
+            for (int i = 0; i < 32; ++i)
+              if (n0 + c0 + i < sh.N) v[i] += __ldg(epi.bias + n0 + c0 + i);
+          }
+          if (epi.flags & RDM_EPI_RELU) {
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] = fmaxf(v[i], 0.f);
+          }
+          if ((epi.flags & RDM_EPI_MASK) && row < sh.M) {
+            const float4* mrow = reinterpret_cast<const float4*>(epi.mask + row * epi.ld_mask + n0 + c0);
+            float4 mk[8];
+#pragma unroll
+            for (int j = 0; j < 8; ++j)
+              mk[j] = (n0 + c0 + 4 * j < sh.N) ? __ldg(mrow + j) : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+            for (int j = 0; j < 8; ++j) {
+              v[4 * j + 0] = mk[j].x > 0.f ? v[4 * j + 0] : 0.f;
+              v[4 * j + 1] = mk[j].y > 0.f ? v[4 * j + 1] : 0.f;
+              v[4 * j + 2] = mk[j].z > 0.f ? v[4 * j + 2] : 0.f;
+              v[4 * j + 3] = mk[j].w > 0.f ? v[4 * j + 3] : 0.f;
+            }
+          }
+#pragma unroll
+          for (int i = 0; i < 32; ++i) tb[lane * 33 + i] = v[i];
+        } else {
+#pragma unroll
+          for (int i = 0; i < 32; ++i) tb[lane * 33 + i] = __uint_as_float(r[i]);
+        }
+        __syncwarp();
+        const int64_t col = n0 + c0 + lane;
+        if (col < sh.N) {
+          const int nrows = (sh.M - row0) < 32 ? (int)(sh.M - row0) : 32;
+#pragma unroll 8
+          for (int rr = 0; rr < nrows; ++rr) Cz[(row0 + rr) * ldc + col] = tb[rr * 33 + lane];
+        }
+        __syncwarp();
       }
+      tc_fence_before();
+      mbar_arrive(&tempty[acc]);
     }
   }
   tc_fence_before();
@@ -397,10 +485,18 @@ void launch_tc(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, const C
   using CF = Cfg<BN>;
   RDM_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<BN, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 CF::kSmem));
-  const int64_t kps = ceil_div(ceil_div(K, splits), BK) * BK;
-  dim3 grid((unsigned)ceil_div(M, BM), (unsigned)ceil_div(N, BN), (unsigned)splits);
-  gemm_tc_kernel<BN, MODE><<<grid, kThreads, CF::kSmem, ctx->stream>>>(a, b, blo, C, ldc, M, N, K,
-                                                                        kps, n_mma, e);
+  TcShape sh;
+  sh.M = M;
+  sh.N = N;
+  sh.K = K;
+  sh.k_per_split = ceil_div(ceil_div(K, splits), BK) * BK;
+  sh.tiles_m = (int)ceil_div(M, BM);
+  sh.tiles_n = (int)ceil_div(N, BN);
+  sh.splits = splits;
+  sh.n_mma = n_mma;
+  const int64_t total = (int64_t)sh.tiles_m * sh.tiles_n * splits;
+  const unsigned grid = (unsigned)std::min<int64_t>(total, ctx->num_sms);
+  gemm_tc_kernel<BN, MODE><<<grid, 384, CF::kSmem, ctx->stream>>>(a, b, blo, C, ldc, sh, e);
   RDM_LAUNCHED(ctx);
 }
 
@@ -422,9 +518,9 @@ bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, 
   if (g_tc_disabled) return false;
   // TMA: global base 16-byte aligned, row strides multiples of 16 bytes
   if (((uintptr_t)X & 15) || (ldx & 3)) return false;
-  const char* dbgs = getenv("RDM_TC_DBG");
-  const int dbg = dbgs ? atoi(dbgs) : 0;
-  TcEpi e{epi, bias, mask, ldc, dbg};
+  // the epilogue reads mask rows as float4: 16-byte aligned rows required
+  if ((epi & RDM_EPI_MASK) && (((uintptr_t)mask & 15) || (ldc & 3))) return false;
+  TcEpi e{epi, bias, mask, ldc};
   if (op == RDM_GEMM_NN || op == RDM_GEMM_NT) {
     const int64_t M = rows;
     const int64_t N = op == RDM_GEMM_NN ? m : k;   // output columns
@@ -467,7 +563,7 @@ bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, 
     ldo = roundup4(N);
     out = ensure_ws(ctx->ws_gemm, (size_t)splits * M * ldo * sizeof(float));
   }
-  TcEpi none{0, nullptr, nullptr, 0, dbg};
+  TcEpi none{0, nullptr, nullptr, 0};
   switch (BN) {
     case 32: launch_tc<32, 1>(ctx, ta, tb, tb, out, ldo, M, N, K, (int)splits, n_mma, none); break;
     case 64: launch_tc<64, 1>(ctx, ta, tb, tb, out, ldo, M, N, K, (int)splits, n_mma, none); break;
