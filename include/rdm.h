@@ -193,6 +193,19 @@ rdm_status rdm_partition(int world, rdm_layout layout, int64_t n, int64_t f, int
 rdm_status rdm_set_graph(rdm_ctx* ctx, int64_t n, int64_t nnz, const int64_t* rowptr,
                          const int32_t* col, const float* val, int symmetric, int on_host);
 
+/* What rdm_set_graph built: row bins (light rows warp-per-row, heavy rows in
+ * 2048-nnz segments) and, for symmetric graphs with a dense block of
+ * high-degree vertices, the "hub core": the K x K block A[hubs, hubs] (K a
+ * multiple of 128, core_nnz entries) held dense and multiplied on the tensor
+ * cores, the other entries in a residual CSR (core_K = 0: no core). */
+typedef struct {
+  int64_t n, nnz;
+  int64_t n_light_rows, n_heavy_rows, n_segments, max_degree;
+  int64_t core_K, core_nnz;
+  int symmetric;
+} rdm_graph_info;
+rdm_status rdm_get_graph_info(const rdm_ctx* ctx, rdm_graph_info* out);
+
 /* --------------------------------------------------- communication-free ops */
 
 /* Communication-free SpMM on one column slice (Fig. 2a):

@@ -405,3 +405,26 @@ class GCN:
 
         view = torch.as_tensor(_View(), device=f"cuda:{self.ctx.device}")
         return view[:, :c].clone()
+
+
+class RdmGraphInfo(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_int64) for n in ("n", "nnz", "n_light_rows", "n_heavy_rows",
+                                               "n_segments", "max_degree", "core_K", "core_nnz")] + \
+               [("symmetric", ctypes.c_int)]
+
+    def as_dict(self):
+        return {n: getattr(self, n) for n, _ in self._fields_}
+
+
+_lib.rdm_get_graph_info.argtypes = [_vp, ctypes.POINTER(RdmGraphInfo)]
+_lib.rdm_get_graph_info.restype = _int
+EXPORTS.append("rdm_get_graph_info")
+
+
+def _graph_info(self) -> dict:
+    gi = RdmGraphInfo()
+    self._c(_lib.rdm_get_graph_info(self.h, ctypes.byref(gi)))
+    return gi.as_dict()
+
+
+Context.graph_info = _graph_info

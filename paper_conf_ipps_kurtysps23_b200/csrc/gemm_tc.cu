@@ -130,10 +130,6 @@ __host__ __device__ constexpr uint32_t idesc_tf32(int N, int a_mn, int b_mn) {
 // every product err toward zero and the error then accumulated coherently
 // through the heavy cancellation of the weight-gradient sums (softmax-gradient
 // rows sum to zero), costing 3 decimal digits.
-__device__ __forceinline__ float tf32_rn(float x) {
-  return __uint_as_float((__float_as_uint(x) + 0x1000u) & 0xFFFFE000u);
-}
-
 __device__ __forceinline__ void split_inplace(float4* hi, float4* lo, int n4, int t, int nt) {
   for (int i = t; i < n4; i += nt) {
     float4 x = hi[i];
@@ -510,6 +506,34 @@ int pick_bn(int64_t N) {
 
 }  // namespace
 
+namespace {
+void launch_nn_panels(rdm_ctx* ctx, const float* X, int64_t ldx, const float* bhi, const float* blo,
+                      int64_t ldb, float* C, int64_t ldc, int64_t M, int64_t N, int64_t K,
+                      const TcEpi& e) {
+  const int BN = pick_bn(N);
+  // one MMA width for every tile: BN when N spans several tiles, else N rounded to 16
+  const int nm = N > BN ? BN : (int)(((N + 15) / 16) * 16);
+  const CUtensorMap ta = make_map(X, K, M, ldx, BK, BM);
+  const CUtensorMap tb = make_map(bhi, K, N, ldb, BK, BN);
+  const CUtensorMap tbl = make_map(blo, K, N, ldb, BK, BN);
+  switch (BN) {
+    case 16: launch_tc<16, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
+    case 32: launch_tc<32, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
+    case 64: launch_tc<64, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
+    case 128: launch_tc<128, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
+    default: launch_tc<256, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
+  }
+}
+}  // namespace
+
+void gemm_tc_panels(rdm_ctx* ctx, const float* A, int64_t lda, const float* bhi, const float* blo,
+                    int64_t ldb, float* C, int64_t ldc, int64_t M, int64_t N, int64_t K) {
+  RDM_CHECK_ARG(!((uintptr_t)A & 15) && !(lda & 3) && !((uintptr_t)bhi & 15) &&
+                    !((uintptr_t)blo & 15) && !(ldb & 3),
+                "gemm_tc_panels: 16-byte aligned operands with ld % 4 == 0 required");
+  launch_nn_panels(ctx, A, lda, bhi, blo, ldb, C, ldc, M, N, K, TcEpi{0, nullptr, nullptr, 0});
+}
+
 static bool g_tc_disabled = false;
 
 bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, int64_t ldw,
@@ -532,19 +556,7 @@ bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, 
     prep_b_kernel<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(N * ldb, 256), 4096)), 256, 0,
                     ctx->stream>>>(W, ldw, K, N, op == RDM_GEMM_NN ? 1 : 0, bhi, blo, ldb);
     RDM_LAUNCHED(ctx);
-    const int BN = pick_bn(N);
-    // one MMA width for every tile: BN when N spans several tiles, else N rounded to 16
-    const int nm = N > BN ? BN : (int)(((N + 15) / 16) * 16);
-    const CUtensorMap ta = make_map(X, K, M, ldx, BK, BM);
-    const CUtensorMap tb = make_map(bhi, K, N, ldb, BK, BN);
-    const CUtensorMap tbl = make_map(blo, K, N, ldb, BK, BN);
-    switch (BN) {
-      case 16: launch_tc<16, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
-      case 32: launch_tc<32, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
-      case 64: launch_tc<64, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
-      case 128: launch_tc<128, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
-      default: launch_tc<256, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
-    }
+    launch_nn_panels(ctx, X, ldx, bhi, blo, ldb, C, ldc, M, N, K, e);
     return true;
   }
   // TN: C[k x m] = Xᵀ U  (X rows x k at ldx, U rows x m at ldw)

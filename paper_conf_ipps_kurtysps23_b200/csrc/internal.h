@@ -71,9 +71,26 @@ struct DevBuf {
 };
 
 // ------------------------------------------------------------------- graph
+struct Csr;
+
+// Dense "hub core" of a symmetric adjacency: the K highest-degree vertices'
+// mutual block A[hubs, hubs], stored dense (K x K fp32, hub slots in degree
+// order) and multiplied on the tensor cores; the CSR `resid` holds every other
+// entry.  A·X = resid·X + scatter_hub_rows(Acore · X[hubs]).
+struct Core {
+  int64_t K = 0;                       // hub count (multiple of 128), 0 = no core
+  int64_t nnz = 0;                     // entries moved into the dense block
+  bool forced = false;                 // RDM_CORE_K override: use at every width
+  std::unique_ptr<DevBuf> A;           // K x K fp32, row-major
+  std::unique_ptr<DevBuf> hub_ids;     // int32[K]: vertex of slot k
+  std::unique_ptr<DevBuf> hub_slot;    // int32[N]: slot of vertex v, -1 if not a hub
+  std::unique_ptr<Csr> resid;          // A minus the core entries (with its own bins)
+};
+
 struct Csr {
   int64_t n = 0, nnz = 0;
   std::unique_ptr<DevBuf> rowptr, col, val;
+  Core core;
   // row bins (see spmm.cu): light rows processed warp-per-row, heavy rows
   // split into fixed-size nnz segments reduced deterministically.
   int64_t n_light = 0, n_seg = 0, n_heavy = 0;
@@ -115,6 +132,7 @@ struct rdm_ctx {
   std::unique_ptr<rdm::DevBuf> ws_gemm;                        // GEMM split-K partials
   std::unique_ptr<rdm::DevBuf> ws_tcb;                         // tcgen05 B panels (hi | lo)
   std::unique_ptr<rdm::DevBuf> ws_stage;                       // host-input staging
+  std::unique_ptr<rdm::DevBuf> ws_core_b, ws_core_c;           // hub-core panels / product
   std::unique_ptr<rdm::DevBuf> ws_scratch;
   // phase timing
   bool timing = false;
@@ -154,6 +172,18 @@ void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host);
 void gemm(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, int64_t ldw, float* C,
           int64_t ldc, int64_t rows, int64_t k, int64_t m, int epi, const float* bias,
           const float* mask);
+// C[M x N] = A[M x K] · B with B given as pre-split tf32 hi / lo panels
+// Bt[N][K] (K-major, row length ldb; 16-byte aligned), on the tensor cores.
+void gemm_tc_panels(rdm_ctx* ctx, const float* A, int64_t lda, const float* bhi, const float* blo,
+                    int64_t ldb, float* C, int64_t ldc, int64_t M, int64_t N, int64_t K);
+// dense hub core (spmm.cu)
+void build_core(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, const int32_t* col_host,
+                const float* val_host);
+
+// Round-to-nearest fp32 → tf32 (ties away from zero), used by every 3xTF32 split.
+__device__ __forceinline__ float tf32_rn(float x) {
+  return __uint_as_float((__float_as_uint(x) + 0x1000u) & 0xFFFFE000u);
+}
 
 // redist.cu — pack (row slice → P contiguous blocks, each r x ld_q) and
 // unpack (P blocks r x ld_q → row slice).  `blocks[q]` points to block q.

@@ -276,6 +276,13 @@ static void set_graph(rdm_ctx* ctx, int64_t n, int64_t nnz, const int64_t* rowpt
   std::vector<int64_t> rp(n + 1);
   RDM_CUDA(cudaMemcpy(rp.data(), g.A.rowptr->ptr, (n + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost));
   build_bins(ctx, g.A, rp.data());
+  if (g.symmetric && n >= 4096 && nnz > 0) {
+    std::vector<int32_t> hc(nnz);
+    std::vector<float> hv(nnz);
+    RDM_CUDA(cudaMemcpy(hc.data(), g.A.col->ptr, nnz * sizeof(int32_t), cudaMemcpyDeviceToHost));
+    RDM_CUDA(cudaMemcpy(hv.data(), g.A.val->ptr, nnz * sizeof(float), cudaMemcpyDeviceToHost));
+    build_core(ctx, g.A, rp.data(), hc.data(), hv.data());
+  }
   if (!g.symmetric) {
     // Aᵀ as CSR: stable counting sort of (col, row) — one-time setup.
     std::vector<int32_t> c(nnz);
@@ -438,6 +445,23 @@ rdm_status rdm_partition(int world, rdm_layout layout, int64_t n, int64_t f, int
 rdm_status rdm_set_graph(rdm_ctx* ctx, int64_t n, int64_t nnz, const int64_t* rowptr,
                          const int32_t* col, const float* val, int symmetric, int on_host) {
   return guarded(ctx, [&] { set_graph(ctx, n, nnz, rowptr, col, val, symmetric, on_host); });
+}
+
+rdm_status rdm_get_graph_info(const rdm_ctx* ctx, rdm_graph_info* out) {
+  if (!ctx || !out) return RDM_ERR_ARG;
+  if (!ctx->has_graph) return RDM_ERR_STATE;
+  const Csr& A = ctx->graph.A;
+  *out = rdm_graph_info{};
+  out->n = A.n;
+  out->nnz = A.nnz;
+  out->n_light_rows = A.n_light;
+  out->n_heavy_rows = A.n_heavy;
+  out->n_segments = A.n_seg;
+  out->max_degree = A.max_deg;
+  out->core_K = A.core.K;
+  out->core_nnz = A.core.nnz;
+  out->symmetric = ctx->graph.symmetric ? 1 : 0;
+  return RDM_OK;
 }
 
 rdm_status rdm_spmm(rdm_ctx* ctx, int transpose, const float* in, int64_t ld_in, float* out,

@@ -21,6 +21,8 @@
 //    H slice keeps L2; gathers use the read-only path (__ldg).
 //  * Fused epilogue: bias, ReLU, Hadamard mask 1[mask > 0] (eq. 3's σ').
 #include <algorithm>
+#include <cmath>
+#include <cstdlib>
 #include <vector>
 
 #include "internal.h"
@@ -38,9 +40,19 @@ struct Epi {
   const float* mask;
   int64_t ld_mask;
   int64_t w;
+  const float* core;        // hub-core product (K x ld_core) or null
+  int64_t ld_core;
+  const int32_t* hub_slot;  // int32[N], -1 for non-hubs
 };
 
 __device__ __forceinline__ float4 apply_epi(float4 a, const Epi& e, int64_t row, int64_t c) {
+  if (e.core) {  // add the dense hub-core contribution of this row (fixed order: after the CSR sum)
+    const int s = __ldg(e.hub_slot + row);
+    if (s >= 0) {
+      const float4 k = __ldg(reinterpret_cast<const float4*>(e.core + (int64_t)s * e.ld_core + c));
+      a.x += k.x; a.y += k.y; a.z += k.z; a.w += k.w;
+    }
+  }
   if (e.flags & RDM_EPI_BIAS) {
     if (c + 0 < e.w) a.x += e.bias[c + 0];
     if (c + 1 < e.w) a.y += e.bias[c + 1];
@@ -220,6 +232,43 @@ void pick_gv(int c4, int* G, int* V) {
   *V = bv;
 }
 
+void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
+             int64_t w4, const Epi& epi);
+
+// Hub-core cost model (B200-calibrated, profiles/r1_core_experiment.md): the
+// CSR SpMM spends ≈ 24 ps · (w/128)^0.55 per nnz (L2-gather bound), the core
+// GEMM ≈ 1.25 ps per K² element (A-operand stream + 3xTF32 MMA), both per call.
+double core_saving_s(int64_t core_nnz, int64_t w) {
+  return (double)core_nnz * 24e-12 * std::pow((double)w / 128.0, 0.55);
+}
+double core_cost_s(int64_t K, int64_t w) { return (double)K * K * 1.25e-12 * (1.0 + w / 600.0) + 20e-6; }
+bool core_pays(const Core& c, int64_t w) {
+  return c.forced || core_saving_s(c.nnz, w) > core_cost_s(c.K, w);
+}
+
+// Panels of X[hubs] for the core GEMM: Bt_hi/lo[n][k] = tf32 split of X[hub_ids[k]][n]
+// (transposed through shared memory: coalesced reads along n, writes along k).
+__global__ void core_panels_kernel(const float* __restrict__ X, int64_t ldx,
+                                   const int32_t* __restrict__ hub_ids, int64_t K, int64_t w,
+                                   float* __restrict__ bhi, float* __restrict__ blo) {
+  __shared__ float t[32][33];
+  const int64_t k0 = (int64_t)blockIdx.x * 32, n0 = (int64_t)blockIdx.y * 32;
+  for (int i = threadIdx.y; i < 32; i += 8) {
+    const int64_t k = k0 + i, n = n0 + threadIdx.x;
+    t[i][threadIdx.x] = (n < w) ? X[(int64_t)hub_ids[k] * ldx + n] : 0.f;
+  }
+  __syncthreads();
+  for (int i = threadIdx.y; i < 32; i += 8) {
+    const int64_t n = n0 + i, k = k0 + threadIdx.x;
+    if (n < w) {
+      const float x = t[threadIdx.x][i];
+      const float h = tf32_rn(x);
+      bhi[n * K + k] = h;
+      blo[n * K + k] = tf32_rn(x - h);
+    }
+  }
+}
+
 }  // namespace
 
 void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
@@ -235,7 +284,32 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
                                                 ((uintptr_t)mask & 15) == 0),
                 "spmm: mask requires a 16-byte aligned N x w buffer with ld % 4 == 0");
   RDM_CHECK_ARG(!(epi_flags & RDM_EPI_BIAS) || bias, "spmm: bias pointer missing");
-  Epi epi{epi_flags, bias, mask, ld_mask, w};
+  Epi epi{epi_flags, bias, mask, ld_mask, w, nullptr, 0, nullptr};
+  if (A.core.K && core_pays(A.core, w)) {
+    // hub core on the tensor cores: panels Bt[n][k] = split(X[hub_k][n]), then
+    // C_core = Acore · X[hubs]; the residual CSR's epilogue adds C_core rows.
+    const int64_t K = A.core.K;
+    float* bp = ensure_ws(ctx->ws_core_b, (size_t)2 * w * K * sizeof(float));
+    float* cc = ensure_ws(ctx->ws_core_c, (size_t)K * w4 * sizeof(float));
+    dim3 grid((unsigned)(K / 32), (unsigned)ceil_div(w, 32));
+    core_panels_kernel<<<grid, dim3(32, 8), 0, ctx->stream>>>(in, ld_in, A.core.hub_ids->as<int32_t>(),
+                                                              K, w, bp, bp + w * K);
+    RDM_LAUNCHED(ctx);
+    gemm_tc_panels(ctx, A.core.A->as<float>(), K, bp, bp + w * K, K, cc, w4, K, w, K);
+    epi.core = cc;
+    epi.ld_core = w4;
+    epi.hub_slot = A.core.hub_slot->as<int32_t>();
+    run_csr(ctx, *A.core.resid, in, ld_in, out, ld_out, w4, epi);
+  } else {
+    run_csr(ctx, A, in, ld_in, out, ld_out, w4, epi);
+  }
+  ctx->counters.spmm_calls++;
+  ctx->counters.spmm_nnz_cols += A.nnz * w;
+}
+
+namespace {
+void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
+             int64_t w4, const Epi& epi) {
   float* part = nullptr;
   if (A.n_seg) part = ensure_ws(ctx->ws_seg, (size_t)A.n_seg * w4 * sizeof(float));
   int G, V;
@@ -255,9 +329,8 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
         A.heavy_rows->as<int32_t>(), A.heavy_seg->as<int32_t>(), part, w4, out, ld_out, w4, epi);
     RDM_LAUNCHED(ctx);
   }
-  ctx->counters.spmm_calls++;
-  ctx->counters.spmm_nnz_cols += A.nnz * w;
 }
+}  // namespace
 
 // Row bins (host, one-time at rdm_set_graph; pure indexing of rowptr).
 void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rp) {
@@ -321,6 +394,106 @@ void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rp) {
                         cudaMemcpyHostToDevice));
   RDM_CUDA(cudaMemcpy(A.heavy_seg->ptr, heavy_seg.data(), (n_heavy + 1) * sizeof(int32_t),
                       cudaMemcpyHostToDevice));
+}
+
+// Dense hub core (one-time, host side, at rdm_set_graph for symmetric A):
+// rank vertices by degree, take the K (multiple of 128) highest-degree ones
+// whose mutual block pays for itself on the tensor cores (core_pays at the
+// reference width 128), move A[hubs, hubs] into a dense K x K matrix and keep
+// every other entry in a residual CSR.  K = 0 (no core) for graphs without a
+// dense hub block.  Set RDM_NO_CORE=1 to disable.
+void build_core(rdm_ctx* ctx, Csr& A, const int64_t* rp, const int32_t* col, const float* val) {
+  (void)ctx;
+  const int64_t n = A.n, nnz = A.nnz;
+  const char* off = getenv("RDM_NO_CORE");
+  if ((off && atoi(off)) || n < 4096 || nnz == 0) return;
+  std::vector<int32_t> order(n);
+  for (int64_t i = 0; i < n; ++i) order[i] = (int32_t)i;
+  std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {
+    return rp[a + 1] - rp[a] > rp[b + 1] - rp[b];
+  });
+  std::vector<int32_t> rank(n);
+  for (int64_t i = 0; i < n; ++i) rank[order[i]] = (int32_t)i;
+  const int64_t kmax = std::min<int64_t>((n / 2) / 128 * 128, 20480);
+  if (kmax < 1024) return;
+  std::vector<int64_t> hist(kmax + 1, 0);  // entries whose max(rank_r, rank_c) falls in bucket
+  for (int64_t i = 0; i < n; ++i) {
+    const int32_t ri = rank[i];
+    for (int64_t j = rp[i]; j < rp[i + 1]; ++j) {
+      const int32_t m = std::max(ri, rank[col[j]]);
+      hist[m < kmax ? m : kmax]++;
+    }
+  }
+  int64_t best_K = 0, best_nnz = 0;
+  double best_gain = 1e-4;  // must save at least 0.1 ms per width-128 call
+  int64_t acc = 0, b = 0;
+  for (int64_t K = 128; K <= kmax; K += 128) {
+    for (; b < K; ++b) acc += hist[b];
+    const double gain = core_saving_s(acc, 128) - core_cost_s(K, 128);
+    if (gain > best_gain) {
+      best_gain = gain;
+      best_K = K;
+      best_nnz = acc;
+    }
+  }
+  const char* force = getenv("RDM_CORE_K");  // tests: force a core of this size
+  bool forced = false;
+  if (force && atoi(force) > 0) {
+    best_K = std::min<int64_t>(kmax, std::max<int64_t>(128, (int64_t)atoi(force) / 128 * 128));
+    forced = true;
+  }
+  if (!best_K) return;
+  const int64_t K = best_K;
+  A.core.forced = forced;
+  std::vector<float> dense((size_t)K * K, 0.f);
+  std::vector<int64_t> rrp(n + 1, 0);
+  for (int64_t i = 0; i < n; ++i) {
+    int64_t keep = 0;
+    for (int64_t j = rp[i]; j < rp[i + 1]; ++j)
+      keep += !(rank[i] < K && rank[col[j]] < K);
+    rrp[i + 1] = rrp[i] + keep;
+  }
+  const int64_t rnnz = rrp[n];
+  std::vector<int32_t> rcol(std::max<int64_t>(rnnz, 1));
+  std::vector<float> rval(std::max<int64_t>(rnnz, 1));
+  for (int64_t i = 0; i < n; ++i) {
+    int64_t o = rrp[i];
+    for (int64_t j = rp[i]; j < rp[i + 1]; ++j) {
+      const int32_t c = col[j];
+      if (rank[i] < K && rank[c] < K) {
+        dense[(size_t)rank[i] * K + rank[c]] += val[j];
+      } else {
+        rcol[o] = c;
+        rval[o] = val[j];
+        ++o;
+      }
+    }
+  }
+  std::vector<int32_t> slot(n);
+  for (int64_t v = 0; v < n; ++v) slot[v] = rank[v] < K ? rank[v] : -1;
+  Core& c = A.core;
+  c.K = K;
+  c.nnz = nnz - rnnz;
+  (void)best_nnz;
+  c.A.reset(new DevBuf((size_t)K * K * sizeof(float)));
+  RDM_CUDA(cudaMemcpy(c.A->ptr, dense.data(), (size_t)K * K * sizeof(float), cudaMemcpyHostToDevice));
+  c.hub_ids.reset(new DevBuf(K * sizeof(int32_t)));
+  RDM_CUDA(cudaMemcpy(c.hub_ids->ptr, order.data(), K * sizeof(int32_t), cudaMemcpyHostToDevice));
+  c.hub_slot.reset(new DevBuf(n * sizeof(int32_t)));
+  RDM_CUDA(cudaMemcpy(c.hub_slot->ptr, slot.data(), n * sizeof(int32_t), cudaMemcpyHostToDevice));
+  c.resid.reset(new Csr());
+  Csr& R = *c.resid;
+  R.n = n;
+  R.nnz = rnnz;
+  R.rowptr.reset(new DevBuf((n + 1) * sizeof(int64_t)));
+  R.col.reset(new DevBuf(std::max<int64_t>(rnnz, 1) * sizeof(int32_t)));
+  R.val.reset(new DevBuf(std::max<int64_t>(rnnz, 1) * sizeof(float)));
+  RDM_CUDA(cudaMemcpy(R.rowptr->ptr, rrp.data(), (n + 1) * sizeof(int64_t), cudaMemcpyHostToDevice));
+  if (rnnz) {
+    RDM_CUDA(cudaMemcpy(R.col->ptr, rcol.data(), rnnz * sizeof(int32_t), cudaMemcpyHostToDevice));
+    RDM_CUDA(cudaMemcpy(R.val->ptr, rval.data(), rnnz * sizeof(float), cudaMemcpyHostToDevice));
+  }
+  build_bins(ctx, R, rrp.data());
 }
 
 }  // namespace rdm

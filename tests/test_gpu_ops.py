@@ -209,3 +209,28 @@ def test_adam_matches_oracle(torch_dev, rdm):
         rp, rm, rv = og.adam(rp, gr, rm, rv, t)
     ctx.sync()
     assert og.max_rel_err(p.cpu().numpy(), rp) < 1e-6
+
+
+@pytest.mark.parametrize("w", [4, 16, 41, 128, 130])
+@pytest.mark.parametrize("K", [128, 1024])
+def test_spmm_hub_core_matches_oracle(torch_dev, w, K, monkeypatch):
+    """Dense hub core (tensor cores) + residual CSR == the plain product, with
+    epilogues; forced core sizes (RDM_CORE_K) so small graphs exercise it."""
+    torch, dev = torch_dev
+    import paper_conf_ipps_kurtysps23_b200 as rdm
+    monkeypatch.setenv("RDM_CORE_K", str(K))
+    g = synth.rmat(6000, 150000, seed=13)
+    ctx = rdm.Context(device=0)
+    ctx.set_graph(g.rowptr, g.col, g.val)
+    gi = ctx.graph_info()
+    assert gi["core_K"] == K and gi["core_nnz"] > 0
+    rng = np.random.default_rng(w)
+    X = rng.standard_normal((g.n, w)).astype(np.float32)
+    M = rng.standard_normal((g.n, w)).astype(np.float32)
+    xd, md = _padded(torch, dev, X), _padded(torch, dev, M)
+    out = torch.zeros_like(xd)
+    ctx.spmm(0, xd, out, w, rdm.EPI_RELU | rdm.EPI_MASK, mask=md)
+    ctx.sync()
+    ref = np.maximum(og.spmm(g, X), 0) * (M > 0)
+    assert og.max_rel_err(out[:, :w].cpu().numpy(), ref) < TOL
+    assert np.all(out[:, w:].cpu().numpy() == 0)
