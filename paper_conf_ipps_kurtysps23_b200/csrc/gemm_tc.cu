@@ -73,6 +73,11 @@ __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, u
       "l"((uint64_t)map), "r"(smem_u32(bar)), "r"(c0), "r"(c1)
       : "memory");
 }
+__device__ __forceinline__ void tma_prefetch_2d(const CUtensorMap* map, int c0, int c1) {
+  asm volatile("cp.async.bulk.prefetch.tensor.2d.L2.global [%0, {%1, %2}];" ::"l"((uint64_t)map),
+               "r"(c0), "r"(c1)
+               : "memory");
+}
 __device__ __forceinline__ void fence_proxy_async() {
   asm volatile("fence.proxy.async.shared::cta;" ::: "memory");
 }
@@ -166,20 +171,81 @@ struct TcEpi {
 struct TcShape {
   int64_t M, N, K, k_per_split;
   int tiles_m, tiles_n, splits, n_mma;
+  int pf;   // issue L2 prefetches of A through tmApf
+  int dbg;  // timing experiments only (RDM_TC_DBG): 1 = skip split, 2 = skip MMA
 };
 
+// A operand placement.  For BN ≤ 128 the converter writes A's hi / lo split
+// straight into TMEM (tcgen05.st) and the MMA reads A from TMEM: the smem
+// stage then only carries the raw A tile and the B panels, which removes the
+// smem-bandwidth bound of the converter (write hi + lo) plus three MMA reads
+// of A per k-block.  BN = 256 needs all 512 TMEM columns for the two
+// accumulators and keeps A in shared memory.
 template <int BN>
 struct Cfg {
+  static constexpr int kAccCols = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
+  static constexpr bool kTmemA = BN <= 128;
+  static constexpr int kNAcc = !kTmemA ? 1 : BN <= 32 ? 4 : BN <= 64 ? 2 : 1;  // partial accumulators
   static constexpr int kABytes = BM * BK * 4;   // 16 KB
   static constexpr int kBBytes = BN * BK * 4;
-  static constexpr int kStageBytes = 2 * kABytes + 2 * kBBytes;
+  static constexpr int kStageBytes = (kTmemA ? 1 : 2) * kABytes + 2 * kBBytes;
   static constexpr int kEpiBytes = 4 * 32 * 33 * 4;   // per-warp 32 x 32 transpose tiles (+1 pad)
   static constexpr int kBudget = 224 * 1024 - kEpiBytes - 1024 - 256;
-  static constexpr int kStages = kBudget / kStageBytes >= 4 ? 4 : kBudget / kStageBytes;
+  // deep rings hide TMA latency; with A in TMEM each stage also takes 64 columns
+  static constexpr int kMaxStages = kTmemA ? (512 - 2 * kNAcc * kAccCols) / (2 * BK) : 4;
+  static constexpr int kFitStages = kBudget / kStageBytes < 8 ? kBudget / kStageBytes : 8;
+  static constexpr int kStages = kFitStages < kMaxStages ? kFitStages : kMaxStages;
   static constexpr int kSmem = kStages * kStageBytes + kEpiBytes + 1024 /*align*/ + 256 /*barriers*/;
-  static constexpr int kAccCols = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
-  static constexpr int kTmemCols = 2 * kAccCols;      // double-buffered accumulator
+  static constexpr int kACol0 = 2 * kNAcc * kAccCols;  // first TMEM column of the A stages
+  static constexpr int kUsedCols = kACol0 + (kTmemA ? kStages * 2 * BK : 0);
+  static constexpr int kTmemCols = kUsedCols <= 32 ? 32 : kUsedCols <= 64 ? 64 : kUsedCols <= 128 ? 128
+                                   : kUsedCols <= 256 ? 256 : 512;
+  static_assert(kUsedCols <= 512, "TMEM overflow");
 };
+
+__device__ __forceinline__ void tc_mma_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db,
+                                          uint32_t idesc, uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "r"(tmem_a), "l"(db), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+
+__device__ __forceinline__ void tmem_st32(uint32_t addr, const float (&v)[32]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,"
+      "%15,%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(addr),
+      "f"(v[0]), "f"(v[1]), "f"(v[2]), "f"(v[3]), "f"(v[4]), "f"(v[5]), "f"(v[6]), "f"(v[7]),
+      "f"(v[8]), "f"(v[9]), "f"(v[10]), "f"(v[11]), "f"(v[12]), "f"(v[13]), "f"(v[14]), "f"(v[15]),
+      "f"(v[16]), "f"(v[17]), "f"(v[18]), "f"(v[19]), "f"(v[20]), "f"(v[21]), "f"(v[22]), "f"(v[23]),
+      "f"(v[24]), "f"(v[25]), "f"(v[26]), "f"(v[27]), "f"(v[28]), "f"(v[29]), "f"(v[30]), "f"(v[31])
+      : "memory");
+}
+
+// Row m (0..127) of the raw A tile, 32 K values, from the swizzled smem stage.
+//  MODE 0 (K-major, 128B swizzle): row m is the 128-byte line m, 16-byte chunk c
+//          stored at chunk c ^ (m & 7).
+//  MODE 1 (MN-major, 128B swizzle with 32-byte atoms): element (k, m) lives in
+//          MN chunk m/32 (4 KB), line k, 32-byte atom ((m%32)/8) ^ (k & 3).
+template <int MODE>
+__device__ __forceinline__ void load_a_row(const uint8_t* tile, int m, float (&v)[32]) {
+  if (MODE == 0) {
+    const float4* line = reinterpret_cast<const float4*>(tile + m * 128);
+#pragma unroll
+    for (int c = 0; c < 8; ++c) {
+      const float4 x = line[c ^ (m & 7)];
+      v[4 * c + 0] = x.x; v[4 * c + 1] = x.y; v[4 * c + 2] = x.z; v[4 * c + 3] = x.w;
+    }
+  } else {
+    const uint8_t* chunk = tile + (m >> 5) * 4096;
+    const int mm = m & 31;
+#pragma unroll
+    for (int k = 0; k < 32; ++k)
+      v[k] = *reinterpret_cast<const float*>(chunk + k * 128 + ((((mm >> 3) ^ (k & 3)) << 5) | ((mm & 7) << 2)));
+  }
+}
 
 // Persistent, warp-specialised tcgen05 GEMM.  384 threads:
 //   warp 0      TMA producer           warp 1  MMA issuer (one thread)
@@ -195,7 +261,8 @@ struct Cfg {
 template <int BN, int MODE>
 __global__ void __launch_bounds__(384, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
-               const __grid_constant__ CUtensorMap tmBlo, float* __restrict__ C, int64_t ldc,
+               const __grid_constant__ CUtensorMap tmBlo, const __grid_constant__ CUtensorMap tmApf,
+               float* __restrict__ C, int64_t ldc,
                TcShape sh, TcEpi epi) {
   using CF = Cfg<BN>;
   constexpr int S = CF::kStages;
@@ -214,10 +281,11 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   const int tiles_mn = sh.tiles_m * sh.tiles_n;
   const int total = tiles_mn * sh.splits;
 
+  constexpr int kAB = (CF::kTmemA ? 1 : 2) * CF::kABytes;   // A bytes per stage in smem
   auto A_hi = [&](int s) { return stage_base + s * CF::kStageBytes; };
-  auto A_lo = [&](int s) { return stage_base + s * CF::kStageBytes + CF::kABytes; };
-  auto B_hi = [&](int s) { return stage_base + s * CF::kStageBytes + 2 * CF::kABytes; };
-  auto B_lo = [&](int s) { return stage_base + s * CF::kStageBytes + 2 * CF::kABytes + CF::kBBytes; };
+  auto A_lo = [&](int s) { return stage_base + s * CF::kStageBytes + CF::kABytes; };  // !kTmemA only
+  auto B_hi = [&](int s) { return stage_base + s * CF::kStageBytes + kAB; };
+  auto B_lo = [&](int s) { return stage_base + s * CF::kStageBytes + kAB + CF::kBBytes; };
   auto tile_kb = [&](int t, int64_t& kbeg) {
     const int z = t / tiles_mn;
     kbeg = (int64_t)z * sh.k_per_split;
@@ -263,6 +331,16 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           mbar_expect_tx(&full[s], bytes);
           const int kk = (int)(kbeg + (int64_t)kb * BK);
           if (MODE == 0) {
+            // L2 prefetch of A in 512-byte row segments, one group (4 k-blocks)
+            // ahead: the 128-byte swizzled boxes alone touch each DRAM page once
+            // per k-block across thousands of concurrent rows.
+            if (sh.pf) {
+              const int g = kb >> 2;
+              if ((kb & 3) == 0) {
+                if (kb == 0) tma_prefetch_2d(&tmApf, kk, m0);
+                if ((int64_t)(g + 1) * 4 < nkb) tma_prefetch_2d(&tmApf, kk + 4 * BK, m0);
+              }
+            }
             tma_load_2d(A_hi(s), &tmA, &full[s], kk, m0);
             tma_load_2d(B_hi(s), &tmB, &full[s], kk, n0);
             tma_load_2d(B_lo(s), &tmBlo, &full[s], kk, n0);
@@ -275,7 +353,8 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     }
   } else if (warp == 1) {
     if (lane == 0) {
-      const uint32_t idesc = idesc_tf32(sh.n_mma, MODE, MODE);
+      // A read from TMEM is K-major by construction (the converter writes rows)
+      const uint32_t idesc = idesc_tf32(sh.n_mma, CF::kTmemA ? 0 : MODE, MODE);
       uint32_t kc = 0;
       int it = 0;
       for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
@@ -284,34 +363,53 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         const int acc = it & 1;
         if (it >= 2) mbar_wait(&tempty[acc], ((it >> 1) - 1) & 1);
         tc_fence_after();
-        const uint32_t d_tmem = tmem_base + acc * CF::kAccCols;
+        const uint32_t d_tmem = tmem_base + acc * (CF::kNAcc * CF::kAccCols);
         for (int kb = 0; kb < nkb; ++kb, ++kc) {
           const int s = kc % S;
           mbar_wait(&conv[s], (kc / S) & 1);
           tc_fence_after();
-          const uint32_t ah = smem_u32(A_hi(s)), al = smem_u32(A_lo(s));
           const uint32_t bh = smem_u32(B_hi(s)), bl = smem_u32(B_lo(s));
 #pragma unroll
           for (int j = 0; j < BK / UK; ++j) {
-            uint64_t dah, dal, dbh, dbl;
+            uint64_t dbh, dbl;
             if (MODE == 0) {  // K-major: advance 32 B along the swizzled row
-              dah = sdesc(ah + j * 32, 16, 1024);
-              dal = sdesc(al + j * 32, 16, 1024);
               dbh = sdesc(bh + j * 32, 16, 1024);
               dbl = sdesc(bl + j * 32, 16, 1024);
             } else {
               // MN-major tf32 needs the 128B swizzle with 32-byte atoms: K rows are
               // 128-byte lines, 4-row groups 512 B apart (SBO), 32-wide MN chunks
               // 4 KB apart (LBO); one K = 8 step spans two groups (1 KB).
-              dah = sdesc(ah + j * 1024, 4096, 512, 1);
-              dal = sdesc(al + j * 1024, 4096, 512, 1);
               dbh = sdesc(bh + j * 1024, 4096, 512, 1);
               dbl = sdesc(bl + j * 1024, 4096, 512, 1);
             }
             const uint32_t acc0 = (kb > 0 || j > 0) ? 1u : 0u;
-            tc_mma(d_tmem, dah, dbh, idesc, acc0);
-            tc_mma(d_tmem, dah, dbl, idesc, 1u);
-            tc_mma(d_tmem, dal, dbh, idesc, 1u);
+            if (sh.dbg & 2) {
+            } else if (CF::kTmemA) {
+              // A stage s: hi in columns [kACol0 + 64 s, +32), lo in the next 32.
+              // Narrow tiles rotate over kNAcc independent accumulators so that
+              // consecutive MMAs do not serialise on one accumulator.
+              const uint32_t ta = tmem_base + CF::kACol0 + s * 2 * BK + j * UK;
+              const uint32_t tab[3] = {ta, ta, ta + BK};
+#pragma unroll
+              for (int p = 0; p < 3; ++p) {
+                const int i = j * 3 + p;
+                const uint32_t d = d_tmem + (uint32_t)((i % CF::kNAcc) * CF::kAccCols);
+                tc_mma_ts(d, tab[p], p == 1 ? dbl : dbh, idesc, (kb > 0 || i >= CF::kNAcc) ? 1u : 0u);
+              }
+            } else {
+              const uint32_t ah = smem_u32(A_hi(s)), al = smem_u32(A_lo(s));
+              uint64_t dah, dal;
+              if (MODE == 0) {
+                dah = sdesc(ah + j * 32, 16, 1024);
+                dal = sdesc(al + j * 32, 16, 1024);
+              } else {
+                dah = sdesc(ah + j * 1024, 4096, 512, 1);
+                dal = sdesc(al + j * 1024, 4096, 512, 1);
+              }
+              tc_mma(d_tmem, dah, dbh, idesc, acc0);
+              tc_mma(d_tmem, dah, dbl, idesc, 1u);
+              tc_mma(d_tmem, dal, dbh, idesc, 1u);
+            }
           }
           tc_commit(&empty[s]);
         }
@@ -327,9 +425,26 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       for (int kb = 0; kb < nkb; ++kb, ++kc) {
         const int s = kc % S;
         mbar_wait(&full[s], (kc / S) & 1);
-        split_inplace((float4*)A_hi(s), (float4*)A_lo(s), CF::kABytes / 16, t128, 128);
+        if (sh.dbg & 1) {
+        } else if (CF::kTmemA) {
+          // thread t128 owns A row t128 = TMEM lane (quadrant warp % 4)
+          float v[32], h[32];
+          load_a_row<MODE>(A_hi(s), t128, v);
+#pragma unroll
+          for (int i = 0; i < 32; ++i) {
+            h[i] = tf32_rn(v[i]);
+            v[i] = tf32_rn(v[i] - h[i]);
+          }
+          const uint32_t ta = tmem_base + ((uint32_t)((warp & 3) * 32) << 16) + CF::kACol0 + s * 2 * BK;
+          tmem_st32(ta, h);
+          tmem_st32(ta + BK, v);
+          asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+        } else {
+          split_inplace((float4*)A_hi(s), (float4*)A_lo(s), CF::kABytes / 16, t128, 128);
+        }
         if (MODE == 1) split_inplace((float4*)B_hi(s), (float4*)B_lo(s), CF::kBBytes / 16, t128, 128);
         fence_proxy_async();
+        tc_fence_before();
         mbar_arrive(&conv[s]);
       }
     }
@@ -352,7 +467,16 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         if (n0 + c0 >= sh.N) break;
         uint32_t r[32];
         if (nkb > 0) {
-          tmem_ld32(tmem_base + acc * CF::kAccCols + ((uint32_t)(q * 32) << 16) + (uint32_t)c0, r);
+          const uint32_t a0 = tmem_base + acc * (CF::kNAcc * CF::kAccCols) + ((uint32_t)(q * 32) << 16) +
+                              (uint32_t)c0;
+          tmem_ld32(a0, r);
+#pragma unroll
+          for (int pa = 1; pa < CF::kNAcc; ++pa) {   // fixed-order sum of the partial accumulators
+            uint32_t r2[32];
+            tmem_ld32(a0 + pa * CF::kAccCols, r2);
+#pragma unroll
+            for (int i = 0; i < 32; ++i) r[i] = __float_as_uint(__uint_as_float(r[i]) + __uint_as_float(r2[i]));
+          }
         } else {
 #pragma unroll
           for (int i = 0; i < 32; ++i) r[i] = 0;
@@ -477,7 +601,7 @@ CUtensorMap make_map(const float* base, int64_t inner, int64_t outer, int64_t ld
 template <int BN, int MODE>
 void launch_tc(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& blo,
                float* C, int64_t ldc, int64_t M, int64_t N, int64_t K, int splits, int n_mma,
-               const TcEpi& e) {
+               const TcEpi& e, const CUtensorMap* apf = nullptr) {
   using CF = Cfg<BN>;
   RDM_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<BN, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 CF::kSmem));
@@ -490,9 +614,13 @@ void launch_tc(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, const C
   sh.tiles_n = (int)ceil_div(N, BN);
   sh.splits = splits;
   sh.n_mma = n_mma;
+  sh.pf = apf != nullptr;
+  const char* dbg = getenv("RDM_TC_DBG");
+  sh.dbg = dbg ? atoi(dbg) : 0;
   const int64_t total = (int64_t)sh.tiles_m * sh.tiles_n * splits;
   const unsigned grid = (unsigned)std::min<int64_t>(total, ctx->num_sms);
-  gemm_tc_kernel<BN, MODE><<<grid, 384, CF::kSmem, ctx->stream>>>(a, b, blo, C, ldc, sh, e);
+  gemm_tc_kernel<BN, MODE><<<grid, 384, CF::kSmem, ctx->stream>>>(a, b, blo, apf ? *apf : a, C, ldc,
+                                                                  sh, e);
   RDM_LAUNCHED(ctx);
 }
 
@@ -516,12 +644,16 @@ void launch_nn_panels(rdm_ctx* ctx, const float* X, int64_t ldx, const float* bh
   const CUtensorMap ta = make_map(X, K, M, ldx, BK, BM);
   const CUtensorMap tb = make_map(bhi, K, N, ldb, BK, BN);
   const CUtensorMap tbl = make_map(blo, K, N, ldb, BK, BN);
+  // L2-prefetch map: 128 x 128 fp32 boxes (512-byte row segments), no swizzle
+  const bool pf = K > 4 * BK && !getenv("RDM_NO_PF");
+  const CUtensorMap tpf = pf ? make_map(X, K, M, ldx, 4 * BK, BM, CU_TENSOR_MAP_SWIZZLE_NONE) : ta;
+  const CUtensorMap* p = pf ? &tpf : nullptr;
   switch (BN) {
-    case 16: launch_tc<16, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
-    case 32: launch_tc<32, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
-    case 64: launch_tc<64, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
-    case 128: launch_tc<128, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
-    default: launch_tc<256, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e); break;
+    case 16: launch_tc<16, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e, p); break;
+    case 32: launch_tc<32, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e, p); break;
+    case 64: launch_tc<64, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e, p); break;
+    case 128: launch_tc<128, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e, p); break;
+    default: launch_tc<256, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e, p); break;
   }
 }
 }  // namespace

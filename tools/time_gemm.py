@@ -19,3 +19,8 @@ for (op, k, m, epi) in [(rdm.GEMM_NT, 128, 41, 0), (rdm.GEMM_NT, 128, 41, rdm.EP
         X = torch.randn(rows, ldk, device=dev); U = torch.randn(rows, ldm, device=dev); C = torch.zeros(k, m, device=dev)
         f = lambda: ctx.gemm(op, X, U, C, rows, k, m)
     print(['NN','NT','TN'][op], k, m, 'epi', epi, f'{t(f):.1f} us')
+# hub-core shaped GEMMs: K x K dense times K x w
+for K in (8192, 16384):
+    for w in (16, 48, 128):
+        A = torch.randn(K, K, device=dev); B = torch.randn(K, w, device=dev); C = torch.zeros(K, w, device=dev)
+        print('core', K, w, f'{t(lambda: ctx.gemm(rdm.GEMM_NN, A, B, C, K, K, w), 5):.1f} us')
