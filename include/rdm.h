@@ -291,10 +291,16 @@ rdm_status rdm_gcn_destroy(rdm_gcn* g);
 
 /* Per local slot i: H0_row[i] = the rank's row slice of H^0 (rows_p x f0,
  * dense, ld = f0), labels_row[i] (int32, rows_p), mask_row[i] (uint8 train
- * mask, rows_p; NULL = all rows).  `on_host` != 0: host pointers (pinned for
- * async copies).  Builds H^0 in every layout the config reads (the model
- * charges nothing for H^0's layout, reading R12) and n_train (global).
- * Collective. */
+ * mask, rows_p; NULL = all rows).  Builds H^0 in every layout the config
+ * reads (the model charges nothing for H^0's layout, reading R12) and n_train
+ * (global).  Collective.
+ * `on_host` == 0: device pointers, applied on the ctx stream immediately.
+ * `on_host` != 0: host pointers (pinned): ASYNCHRONOUS and double-buffered —
+ * the H2D copy is enqueued on a private copy stream into staging buffers
+ * (after the previously staged input was consumed) and the next
+ * rdm_gcn_forward consumes it, so the copy of step i+1's input overlaps step
+ * i's compute.  The host buffers must stay unmodified until that forward has
+ * completed (rdm_sync). */
 rdm_status rdm_gcn_set_input(rdm_gcn* g, const float* const* H0_row,
                              const int32_t* const* labels_row, const uint8_t* const* mask_row,
                              int on_host);

@@ -262,6 +262,13 @@ struct rdm_gcn {
   std::vector<uint8_t*> mask;
   std::vector<double*> scal;                // per slot: [0] n_train, [1] loss partial
   bool input_set = false;
+  // double-buffered host input (see stage_host_input)
+  cudaStream_t cs = nullptr;
+  cudaEvent_t ev_ready = nullptr, ev_free = nullptr;
+  std::vector<float*> st_h0;
+  std::vector<int32_t*> st_lab;
+  std::vector<uint8_t*> st_mask;
+  bool staged = false;
   int64_t ws_bytes = 0;
   rdm_gcn_info info{};
 };
@@ -536,6 +543,8 @@ struct BwdArgs {
   float* const* dW;
 };
 
+void consume_staged(rdm_gcn* g);
+
 void do_forward(void* a_) {
   auto* a = static_cast<FwdArgs*>(a_);
   rdm_gcn* g = a->g;
@@ -543,6 +552,10 @@ void do_forward(void* a_) {
   if (!g->input_set) throw Error(RDM_ERR_STATE, "rdm_gcn_forward: call rdm_gcn_set_input first");
   RDM_CHECK_ARG(a->W && a->loss, "rdm_gcn_forward: W and loss_dev required");
   for (int l = 0; l < g->L; ++l) RDM_CHECK_ARG(a->W[l], "rdm_gcn_forward: null W");
+  if (g->staged) {
+    Phase ph(ctx, RDM_PH_OTHER);
+    consume_staged(g);
+  }
   for (auto& s : g->fwd) run_step(g, s, a->W);
   const int nl = ctx->nlocal();
   std::vector<double*> parts(nl);
@@ -585,13 +598,84 @@ struct InputArgs {
   int on_host;
 };
 
-void do_set_input(void* a_) {
-  auto* a = static_cast<InputArgs*>(a_);
-  rdm_gcn* g = a->g;
+// Host inputs are double-buffered: rdm_gcn_set_input(on_host) only enqueues
+// the H2D copy into device staging buffers on a private copy stream (after the
+// previous input has been consumed) and returns; the next rdm_gcn_forward
+// makes the compute stream wait for it and moves the staged input into place
+// (D2D).  The next step's 0.5 GB input copy therefore overlaps the current
+// step's compute instead of serialising with it.
+void stage_host_input(rdm_gcn* g, const InputArgs* a) {
   rdm_ctx* ctx = g->ctx;
   const int nl = ctx->nlocal(), P = ctx->world;
   const int64_t n = ctx->graph.n, f0 = g->f[0];
+  if (!g->cs) {
+    RDM_CUDA(cudaStreamCreateWithFlags(&g->cs, cudaStreamNonBlocking));
+    RDM_CUDA(cudaEventCreateWithFlags(&g->ev_ready, cudaEventDisableTiming));
+    RDM_CUDA(cudaEventCreateWithFlags(&g->ev_free, cudaEventDisableTiming));
+    g->st_h0.assign(nl, nullptr);
+    g->st_lab.assign(nl, nullptr);
+    g->st_mask.assign(nl, nullptr);
+    for (int i = 0; i < nl; ++i) {
+      const int64_t r = row_range(n, P, ctx->local[i]).size();
+      g->mem.emplace_back(new DevBuf((size_t)std::max<int64_t>(1, r * f0) * sizeof(float)));
+      g->st_h0[i] = g->mem.back()->as<float>();
+      g->mem.emplace_back(new DevBuf((size_t)std::max<int64_t>(1, r) * sizeof(int32_t)));
+      g->st_lab[i] = g->mem.back()->as<int32_t>();
+      g->mem.emplace_back(new DevBuf((size_t)std::max<int64_t>(1, r)));
+      g->st_mask[i] = reinterpret_cast<uint8_t*>(g->mem.back()->ptr);
+    }
+  }
+  RDM_CUDA(cudaStreamWaitEvent(g->cs, g->ev_free, 0));   // previous staged input consumed
+  for (int i = 0; i < nl; ++i) {
+    const int64_t r = row_range(n, P, ctx->local[i]).size();
+    if (!r) continue;
+    if (f0)
+      RDM_CUDA(cudaMemcpyAsync(g->st_h0[i], a->H0[i], r * f0 * sizeof(float), cudaMemcpyHostToDevice, g->cs));
+    RDM_CUDA(cudaMemcpyAsync(g->st_lab[i], a->labels[i], r * sizeof(int32_t), cudaMemcpyHostToDevice, g->cs));
+    if (a->mask && a->mask[i])
+      RDM_CUDA(cudaMemcpyAsync(g->st_mask[i], a->mask[i], r, cudaMemcpyHostToDevice, g->cs));
+    else
+      RDM_CUDA(cudaMemsetAsync(g->st_mask[i], 1, r, g->cs));
+  }
+  RDM_CUDA(cudaEventRecord(g->ev_ready, g->cs));
+  g->staged = true;
+  g->input_set = true;
+}
+
+void apply_input(rdm_gcn* g, const InputArgs* a);
+
+// Called at the start of forward: consume a staged host input on the compute stream.
+void consume_staged(rdm_gcn* g) {
+  if (!g->staged) return;
+  rdm_ctx* ctx = g->ctx;
+  RDM_CUDA(cudaStreamWaitEvent(ctx->stream, g->ev_ready, 0));
+  const int nl = ctx->nlocal();
+  std::vector<const float*> h(g->st_h0.begin(), g->st_h0.end());
+  std::vector<const int32_t*> l(g->st_lab.begin(), g->st_lab.end());
+  std::vector<const uint8_t*> m(g->st_mask.begin(), g->st_mask.end());
+  (void)nl;
+  InputArgs a{g, h.data(), l.data(), m.data(), 0};
+  apply_input(g, &a);           // device-to-device into the working buffers
+  RDM_CUDA(cudaEventRecord(g->ev_free, ctx->stream));
+  g->staged = false;
+}
+
+void do_set_input(void* a_) {
+  auto* a = static_cast<InputArgs*>(a_);
+  rdm_gcn* g = a->g;
   RDM_CHECK_ARG(a->H0 && a->labels, "set_input: H0 and labels required");
+  if (a->on_host) {
+    stage_host_input(g, a);
+  } else {
+    g->staged = false;
+    apply_input(g, a);
+  }
+}
+
+void apply_input(rdm_gcn* g, const InputArgs* a) {
+  rdm_ctx* ctx = g->ctx;
+  const int nl = ctx->nlocal(), P = ctx->world;
+  const int64_t n = ctx->graph.n, f0 = g->f[0];
   const cudaMemcpyKind kind = a->on_host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
   const rdm_counters saved = ctx->counters;
   std::vector<const float*> src(nl);
@@ -602,6 +686,8 @@ void do_set_input(void* a_) {
     if (r && f0) {
       if (h.ld == f0) {
         RDM_CUDA(cudaMemcpyAsync(h.p, a->H0[i], r * f0 * sizeof(float), kind, ctx->stream));
+      } else if (!a->on_host) {
+        copy_2d(ctx, h.p, h.ld, a->H0[i], f0, r, f0);   // device source: re-pitch directly
       } else {
         // one contiguous (DMA-friendly) copy, then re-pitch to ld on the device
         float* stage = ensure_ws(ctx->ws_stage, (size_t)r * f0 * sizeof(float));
@@ -630,6 +716,7 @@ void do_set_input(void* a_) {
   ctx->counters = saved;
   g->input_set = true;
 }
+
 
 void do_create(void* a_) { create(static_cast<rdm_gcn*>(a_)); }
 
@@ -670,6 +757,12 @@ rdm_status rdm_gcn_destroy(rdm_gcn* g) {
   if (!g) return RDM_ERR_ARG;
   cudaSetDevice(g->ctx->device);
   cudaStreamSynchronize(g->ctx->stream);
+  if (g->cs) {
+    cudaStreamSynchronize(g->cs);
+    cudaStreamDestroy(g->cs);
+    cudaEventDestroy(g->ev_ready);
+    cudaEventDestroy(g->ev_free);
+  }
   delete g;
   return RDM_OK;
 }

@@ -45,25 +45,52 @@ xent_kernel(const float* __restrict__ Z, int64_t ldz, const int32_t* __restrict_
   const double nt = *n_train;
   const float inv_n = nt > 0 ? (float)(1.0 / nt) : 0.f;
   double local = 0.0;
+  constexpr int NV = 8;  // logits held in registers for C <= 256
   for (int64_t i = (int64_t)blockIdx.x * kLossWarps + wid; i < rows;
        i += (int64_t)gridDim.x * kLossWarps) {
     const float* z = Z + i * ldz;
-    float mx = -FLT_MAX;
-    for (int64_t c = lane; c < C; c += 32) mx = fmaxf(mx, z[c]);
-    mx = warp_max(mx);
-    float s = 0.f;
-    for (int64_t c = lane; c < C; c += 32) s += expf(z[c] - mx);
-    s = warp_sum(s);
     const int y = labels[i];
     const bool m = mask ? mask[i] != 0 : true;
     const float scale = m ? inv_n : 0.f;
-    const float inv_s = 1.f / s;
     float* g = G + i * ldg;
-    for (int64_t c = lane; c < C; c += 32) {
-      const float p = expf(z[c] - mx) * inv_s;
-      g[c] = (p - (c == y ? 1.f : 0.f)) * scale;
+    float mx = -FLT_MAX, s = 0.f, zy = 0.f;
+    if (C <= 32 * NV) {
+      float v[NV];
+#pragma unroll
+      for (int t = 0; t < NV; ++t) {
+        const int64_t c = lane + 32 * t;
+        v[t] = c < C ? z[c] : -FLT_MAX;
+        mx = fmaxf(mx, v[t]);
+      }
+      mx = warp_max(mx);
+#pragma unroll
+      for (int t = 0; t < NV; ++t) {
+        const int64_t c = lane + 32 * t;
+        v[t] = c < C ? expf(v[t] - mx) : 0.f;
+        s += v[t];
+      }
+      s = warp_sum(s);
+      const float inv_s = 1.f / s;
+#pragma unroll
+      for (int t = 0; t < NV; ++t) {
+        const int64_t c = lane + 32 * t;
+        if (c < C) g[c] = (v[t] * inv_s - (c == y ? 1.f : 0.f)) * scale;
+      }
+    } else {
+      for (int64_t c = lane; c < C; c += 32) mx = fmaxf(mx, z[c]);
+      mx = warp_max(mx);
+      for (int64_t c = lane; c < C; c += 32) s += expf(z[c] - mx);
+      s = warp_sum(s);
+      const float inv_s = 1.f / s;
+      for (int64_t c = lane; c < C; c += 32) {
+        const float p = expf(z[c] - mx) * inv_s;
+        g[c] = (p - (c == y ? 1.f : 0.f)) * scale;
+      }
     }
-    if (lane == 0 && m) local += (double)mx + log((double)s) - (double)z[y];
+    if (lane == 0 && m) {
+      zy = z[y];
+      local += (double)mx + log((double)s) - (double)zy;
+    }
   }
   if (lane == 0) red[wid] = local;
   __syncthreads();
@@ -192,11 +219,14 @@ unsigned grid_for(rdm_ctx* ctx, int64_t total, int per = 256) {
 void softmax_xent(rdm_ctx* ctx, const float* Z, int64_t ldz, const int32_t* labels,
                   const uint8_t* mask, int64_t rows, int64_t C, const double* n_train, float* G,
                   int64_t ldg, double* loss_partial) {
-  double* part = reinterpret_cast<double*>(ensure_ws(ctx->ws_scratch, kLossBlocks * sizeof(double)));
-  xent_kernel<<<kLossBlocks, kLossWarps * 32, 0, ctx->stream>>>(Z, ldz, labels, mask, rows, C,
-                                                                n_train, G, ldg, part);
+  // ≈2 rows per warp; the grid depends only on `rows`, so the partials and
+  // their ordered sum are deterministic
+  const int nb = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(rows, kLossWarps * 2), 16384));
+  double* part = reinterpret_cast<double*>(ensure_ws(ctx->ws_scratch, (size_t)nb * sizeof(double)));
+  xent_kernel<<<nb, kLossWarps * 32, 0, ctx->stream>>>(Z, ldz, labels, mask, rows, C, n_train, G,
+                                                       ldg, part);
   RDM_LAUNCHED(ctx);
-  sum_partials<<<1, 1024, 0, ctx->stream>>>(part, kLossBlocks, loss_partial);
+  sum_partials<<<1, 1024, 0, ctx->stream>>>(part, nb, loss_partial);
   RDM_LAUNCHED(ctx);
 }
 

@@ -172,6 +172,42 @@ def test_adam_epochs_track_oracle(rdm, cora):
     _check((g, H0, Wr, y, m), loss, dW, model, rdm, P=2)
 
 
+def test_host_input_double_buffered(rdm, cora):
+    """set_input(on_host) is staged on a copy stream and consumed by the next
+    forward: results equal the device-input path bit for bit, also when a
+    different input is staged while the previous epoch runs."""
+    import torch
+    g, H0, Ws, y, m, _ = cora
+    dev = torch.device("cuda:0")
+    ctx = rdm.Context(device=0)
+    ctx.set_graph(g.rowptr, g.col, g.val)
+    model = rdm.GCN(ctx, [H0.shape[1]] + [w.shape[1] for w in Ws], 10)
+    Wd = [torch.from_numpy(w).to(dev) for w in Ws]
+    dW = [torch.zeros_like(w) for w in Wd]
+    loss = torch.zeros(1, dtype=torch.float64, device=dev)
+    H1 = np.ascontiguousarray(H0[:, ::-1])   # a second, different input
+    results = {}
+    for name, src in (("a", H0), ("b", H1)):
+        model.set_input([torch.from_numpy(src).to(dev)], [torch.from_numpy(y).to(dev)],
+                        [torch.from_numpy(m).to(dev)])
+        model.forward(Wd, loss)
+        model.backward(Wd, dW)
+        ctx.sync()
+        results[name] = (float(loss.item()), [d.cpu().numpy().copy() for d in dW])
+    pins = [torch.from_numpy(x).pin_memory() for x in (H0, H1)]
+    yp, mp = torch.from_numpy(y).pin_memory(), torch.from_numpy(m).pin_memory()
+    for it, name in enumerate(["a", "b", "a", "b"]):
+        model.set_input([pins[0] if name == "a" else pins[1]], [yp], [mp], on_host=True)
+        model.forward(Wd, loss)
+        model.backward(Wd, dW)
+        if it % 2:
+            ctx.sync()
+        ctx.sync()
+        assert float(loss.item()) == results[name][0]
+        for a_, b_ in zip(dW, results[name][1]):
+            assert np.array_equal(a_.cpu().numpy(), b_)
+
+
 def test_epoch_deterministic(rdm, cora):
     g, H0, Ws, y, m, _ = cora
     a = _run(rdm, g, H0, Ws, y, m, 10, P=4)
