@@ -42,6 +42,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--sweep", action="store_true",
+                    help="also time every configuration (Table VIII analogue) into config.sweep_ms")
     return ap.parse_args()
 
 
@@ -218,26 +220,70 @@ def main():
                       unique_id=uid)
     ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
     pareto, chosen, comm_u, sparse_u = rdm.select_config(list(wl.f), wl.n, wl.nnz, world)
-    cfg_id = chosen if a.config == "auto" else int(a.config)
-    model = rdm.GCN(ctx, wl.f, cfg_id)
     lo, hi, _ = rdm.partition(world, rdm.ROW, wl.n, wl.f[0], rank if world > 1 else 0)
     H0_pin = torch.from_numpy(H0[lo:hi]).pin_memory()
     y_pin = torch.from_numpy(y[lo:hi]).pin_memory()
     m_pin = torch.from_numpy(msk[lo:hi]).pin_memory()
     H0_d, y_d, m_d = H0_pin.to(dev), y_pin.to(dev), m_pin.to(dev)
-    model.set_input([H0_d], [y_d], [m_d])
     Wd = [torch.from_numpy(w).to(dev) for w in Ws_h]
     dW = [torch.zeros_like(w) for w in Wd]
     mom = [torch.zeros_like(w) for w in Wd]
     vel = [torch.zeros_like(w) for w in Wd]
     loss = torch.zeros(1, dtype=torch.float64, device=dev)
     step = [0]
+    cur = {}
+
+    def build(cfg):
+        if "model" in cur:
+            cur["model"].close()
+        m = rdm.GCN(ctx, wl.f, cfg)
+        m.set_input([H0_d], [y_d], [m_d])
+        cur["model"] = m
+        return m
 
     def epoch():
-        model.forward(Wd, loss)
-        model.backward(Wd, dW)
+        cur["model"].forward(Wd, loss)
+        cur["model"].backward(Wd, dW)
         step[0] += 1
         ctx.adam_step(Wd, dW, mom, vel, step[0], lr=0.01)
+
+    def time_epochs(k):
+        """ms per epoch over k epochs: CUDA events on the library stream, max over ranks."""
+        if world > 1:
+            dist.barrier()
+        torch.cuda.synchronize(dev)
+        s0 = torch.cuda.Event(enable_timing=True)
+        s1 = torch.cuda.Event(enable_timing=True)
+        s0.record(stream)
+        for _ in range(k):
+            epoch()
+        s1.record(stream)
+        torch.cuda.synchronize(dev)
+        ms = s0.elapsed_time(s1) / k
+        if world > 1:
+            t = torch.tensor([ms], device=dev)
+            dist.all_reduce(t, op=dist.ReduceOp.MAX)
+            ms = float(t.item())
+        return ms
+
+    sweep = None
+    if a.sweep or a.config == "trial":
+        # NEXT-1 / PAPER.md L224: "after trying out each pareto-optimal configuration in
+        # the first few epochs, we can dynamically determine the fastest configuration".
+        cand = list(range(4 ** wl.L)) if a.sweep else list(pareto)
+        sweep = {}
+        for cid in cand:
+            build(cid)
+            time_epochs(2)
+            sweep[cid] = time_epochs(3)
+        trial_pick = min(pareto, key=lambda c: sweep[c])
+    if a.config == "auto":
+        cfg_id = chosen
+    elif a.config == "trial":
+        cfg_id = trial_pick
+    else:
+        cfg_id = int(a.config)
+    model = build(cfg_id)
 
     for _ in range(max(3, a.warmup)):
         epoch()
@@ -340,7 +386,9 @@ def main():
                 "self loops, D^-1/2 (A+I) D^-1/2", "global_batch": n, "seq_len": None,
                 "parallelism": f"rdm{world} (A replicated, H row/col redistributed)",
                 "config_id": cfg_id, "config_name": rdm.config_name(model.cfg),
-                "pareto": pareto, "model_comm_units": info["model_comm_units"],
+                "pareto": pareto, "pick": a.config,
+                "sweep_ms": ({str(k): round(v, 4) for k, v in sweep.items()} if sweep else None),
+                "model_comm_units": info["model_comm_units"],
                 "model_sparse_units": info["model_sparse_units"],
                 "l2": "inputs larger than L2 (CSR 0.92 GB streamed per SpMM; H0 561 MB)",
                 "gen_s": round(t_gen, 1)},

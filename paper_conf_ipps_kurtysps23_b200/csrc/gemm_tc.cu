@@ -637,7 +637,7 @@ int pick_bn(int64_t N) {
 namespace {
 void launch_nn_panels(rdm_ctx* ctx, const float* X, int64_t ldx, const float* bhi, const float* blo,
                       int64_t ldb, float* C, int64_t ldc, int64_t M, int64_t N, int64_t K,
-                      const TcEpi& e) {
+                      const TcEpi& e, int splits = 1) {
   const int BN = pick_bn(N);
   // one MMA width for every tile: BN when N spans several tiles, else N rounded to 16
   const int nm = N > BN ? BN : (int)(((N + 15) / 16) * 16);
@@ -649,11 +649,11 @@ void launch_nn_panels(rdm_ctx* ctx, const float* X, int64_t ldx, const float* bh
   const CUtensorMap tpf = pf ? make_map(X, K, M, ldx, 4 * BK, BM, CU_TENSOR_MAP_SWIZZLE_NONE) : ta;
   const CUtensorMap* p = pf ? &tpf : nullptr;
   switch (BN) {
-    case 16: launch_tc<16, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e, p); break;
-    case 32: launch_tc<32, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e, p); break;
-    case 64: launch_tc<64, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e, p); break;
-    case 128: launch_tc<128, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e, p); break;
-    default: launch_tc<256, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, 1, nm, e, p); break;
+    case 16: launch_tc<16, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, splits, nm, e, p); break;
+    case 32: launch_tc<32, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, splits, nm, e, p); break;
+    case 64: launch_tc<64, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, splits, nm, e, p); break;
+    case 128: launch_tc<128, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, splits, nm, e, p); break;
+    default: launch_tc<256, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, splits, nm, e, p); break;
   }
 }
 }  // namespace
@@ -663,7 +663,29 @@ void gemm_tc_panels(rdm_ctx* ctx, const float* A, int64_t lda, const float* bhi,
   RDM_CHECK_ARG(!((uintptr_t)A & 15) && !(lda & 3) && !((uintptr_t)bhi & 15) &&
                     !((uintptr_t)blo & 15) && !(ldb & 3),
                 "gemm_tc_panels: 16-byte aligned operands with ld % 4 == 0 required");
-  launch_nn_panels(ctx, A, lda, bhi, blo, ldb, C, ldc, M, N, K, TcEpi{0, nullptr, nullptr, 0});
+  // Split K so that the persistent grid has no idle SMs (the hub-core GEMM has
+  // only ~110 M-tiles for 148 SMs); partial slabs are summed in split order.
+  const int64_t tiles = ceil_div(M, BM) * ceil_div(N, pick_bn(N));
+  int best_s = 1;
+  double best_eff = 0;
+  for (int s = 1; s <= 8; ++s) {
+    if (s > 1 && K / s < 16 * BK) break;
+    const int64_t t = tiles * s;
+    const double eff = (double)t / (double)(ctx->num_sms * ceil_div(t, ctx->num_sms));
+    if (eff > best_eff + 0.02) {
+      best_eff = eff;
+      best_s = s;
+    }
+  }
+  if (best_s == 1) {
+    launch_nn_panels(ctx, A, lda, bhi, blo, ldb, C, ldc, M, N, K, TcEpi{0, nullptr, nullptr, 0});
+    return;
+  }
+  const int64_t ldo = roundup4(N);
+  float* part = ensure_ws(ctx->ws_gemm, (size_t)best_s * M * ldo * sizeof(float));
+  launch_nn_panels(ctx, A, lda, bhi, blo, ldb, part, ldo, M, N, K, TcEpi{0, nullptr, nullptr, 0}, best_s);
+  splitk_sum<<<(unsigned)ceil_div(M * N, 256), 256, 0, ctx->stream>>>(part, best_s, M, N, ldo, C, ldc);
+  RDM_LAUNCHED(ctx);
 }
 
 static bool g_tc_disabled = false;
