@@ -628,7 +628,7 @@ int pick_bn(int64_t N) {
   if (N <= 16) return 16;
   if (N <= 32) return 32;
   if (N <= 64) return 64;
-  if (N <= 128) return 128;
+  if (N <= 128 || !getenv("RDM_BN256")) return 128;   // wider N: several 128-wide tiles (TMEM-A path)
   return 256;
 }
 
@@ -716,7 +716,7 @@ bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, 
   // TN: C[k x m] = Xᵀ U  (X rows x k at ldx, U rows x m at ldw)
   if (((uintptr_t)W & 15) || (ldw & 3)) return false;
   const int64_t M = k, N = m, K = rows;
-  const int BN = N <= 32 ? 32 : N <= 64 ? 64 : N <= 128 ? 128 : 256;
+  const int BN = N <= 32 ? 32 : N <= 64 ? 64 : (N <= 128 || !getenv("RDM_BN256")) ? 128 : 256;
   const int n_mma = (int)std::min<int64_t>(BN, ((N + 31) / 32) * 32);
   const int64_t tiles = ceil_div(M, BM) * ceil_div(N, BN);
   int64_t splits = std::max<int64_t>(1, ctx->num_sms / std::max<int64_t>(1, tiles));

@@ -143,13 +143,13 @@ spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
             const int64_t* __restrict__ seg_start, const int32_t* __restrict__ seg_row,
             int64_t n_light, int64_t n_seg, const float* __restrict__ X, int64_t ldx,
             float* __restrict__ out, int64_t ld_out, float* __restrict__ part, int64_t ld_part,
-            int64_t w4, Epi epi) {
+            int64_t w4, int chunk4, Epi epi) {
   const int lane = threadIdx.x & 31;
   const int64_t item = (int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5);
   if (item >= n_seg + n_light) return;
-  const int64_t cbase = (int64_t)blockIdx.y * 128;             // first column of the chunk
+  const int64_t cbase = (int64_t)blockIdx.y * chunk4 * 4;      // first column of the chunk
   const int64_t rem4 = (w4 - cbase) / 4;
-  const int c4n = rem4 < 32 ? (int)rem4 : 32;                  // float4 chunks in this chunk
+  const int c4n = rem4 < chunk4 ? (int)rem4 : chunk4;          // float4 chunks in this chunk
   const int sub = lane % G;
   float4 acc[V];
   int32_t r;
@@ -199,16 +199,17 @@ __global__ void spmm_heavy_reduce(const int32_t* __restrict__ heavy_rows,
 
 template <int G, int V>
 void launch_spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out,
-                 int64_t ld_out, float* part, int64_t ld_part, int64_t w4, const Epi& epi) {
+                 int64_t ld_out, float* part, int64_t ld_part, int64_t w4, int chunk4,
+                 const Epi& epi) {
   const int64_t items = A.n_seg + A.n_light;
   if (items == 0) return;
-  const int64_t chunks = ceil_div(w4, 128);
+  const int64_t chunks = ceil_div(w4, 4 * chunk4);
   dim3 grid((unsigned)ceil_div(items, kWarps), (unsigned)chunks);
   spmm_kernel<G, V><<<grid, kWarps * 32, 0, ctx->stream>>>(
       A.rowptr->as<int64_t>(), A.col->as<int32_t>(), A.val->as<float>(),
       A.light_rows->as<int32_t>(), A.seg_start->as<int64_t>(),
       reinterpret_cast<const int32_t*>(A.seg_start->as<int64_t>() + A.n_seg), A.n_light, A.n_seg,
-      in, ld_in, out, ld_out, part, ld_part, w4, epi);
+      in, ld_in, out, ld_out, part, ld_part, w4, chunk4, epi);
   RDM_LAUNCHED(ctx);
 }
 
@@ -313,9 +314,17 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
   float* part = nullptr;
   if (A.n_seg) part = ensure_ws(ctx->ws_seg, (size_t)A.n_seg * w4 * sizeof(float));
   int G, V;
-  pick_gv((int)std::min<int64_t>(32, w4 / 4), &G, &V);
+  // Column chunks (blockIdx.y, scheduled chunk after chunk): narrower chunks
+  // keep the gathered slice L2-resident at the price of re-streaming the CSR.
+  // Measured (profiles/r1_summary.md): one 256-wide chunk beats two 128-wide
+  // ones for 128 < w <= 256 (the CSR is streamed once); wider slices use
+  // 128-wide chunks; narrower chunks lose more to CSR re-streaming than they
+  // gain in L2 residency.
+  int chunk4 = (w4 > 128 && w4 <= 256) ? 64 : 32;
+  if (const char* e = getenv("RDM_SPMM_CHUNK4")) chunk4 = std::max(1, std::min(64, atoi(e)));
+  pick_gv((int)std::min<int64_t>(chunk4, w4 / 4), &G, &V);
 #define RDM_SPMM_CASE(g_, v_) \
-  if (G == g_ && V == v_) launch_spmm<g_, v_>(ctx, A, in, ld_in, out, ld_out, part, w4, w4, epi); else
+  if (G == g_ && V == v_) launch_spmm<g_, v_>(ctx, A, in, ld_in, out, ld_out, part, w4, w4, chunk4, epi); else
   RDM_SPMM_CASE(1, 1) RDM_SPMM_CASE(1, 2) RDM_SPMM_CASE(1, 3) RDM_SPMM_CASE(1, 4)
   RDM_SPMM_CASE(2, 1) RDM_SPMM_CASE(2, 2) RDM_SPMM_CASE(2, 3) RDM_SPMM_CASE(2, 4)
   RDM_SPMM_CASE(4, 1) RDM_SPMM_CASE(4, 2) RDM_SPMM_CASE(4, 3) RDM_SPMM_CASE(4, 4)

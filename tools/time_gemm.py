@@ -24,3 +24,18 @@ for K in (8192, 16384):
     for w in (16, 48, 128):
         A = torch.randn(K, K, device=dev); B = torch.randn(K, w, device=dev); C = torch.zeros(K, w, device=dev)
         print('core', K, w, f'{t(lambda: ctx.gemm(rdm.GEMM_NN, A, B, C, K, K, w), 5):.1f} us')
+# products-shaped
+rows = 2449029
+for (op, k, m) in [(rdm.GEMM_NN, 256, 256), (rdm.GEMM_NT, 256, 256), (rdm.GEMM_TN, 256, 256), (rdm.GEMM_NN, 100, 256), (rdm.GEMM_TN, 100, 256)]:
+    ldk, ldm = (k + 3) // 4 * 4, (m + 3) // 4 * 4
+    if op == rdm.GEMM_NN:
+        X = torch.randn(rows, ldk, device=dev); C = torch.zeros(rows, ldm, device=dev); W = torch.randn(k, m, device=dev)
+        f = lambda: ctx.gemm(op, X, W, C, rows, k, m)
+    elif op == rdm.GEMM_NT:
+        X = torch.randn(rows, ldm, device=dev); C = torch.zeros(rows, ldk, device=dev); W = torch.randn(k, m, device=dev)
+        f = lambda: ctx.gemm(op, X, W, C, rows, k, m)
+    else:
+        X = torch.randn(rows, ldk, device=dev); U = torch.randn(rows, ldm, device=dev); C = torch.zeros(k, m, device=dev)
+        f = lambda: ctx.gemm(op, X, U, C, rows, k, m)
+    print('products', ['NN','NT','TN'][op], k, m, f'{t(f, 5):.1f} us')
+    del X, C
