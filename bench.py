@@ -361,8 +361,21 @@ def main():
     alg_bytes = spmm_calls * (8 * nnz + 8 * (n + 1)) + 8 * n * sum_w
     spmm_s = ph_ms["spmm"] / 1e3
     achieved = alg_bytes / spmm_s / 1e9 if spmm_s > 0 else 0.0
+    # traffic: DRAM bytes per SpMM launch from the committed ncu --set full capture
+    traffic, traffic_src = None, None
+    try:
+        tj = _json.load(open(os.path.join(ROOT, "profiles", "r1_spmm_traffic.json")))
+        if a.workload == "reddit" and world == 1:
+            ls = tj["spmm_launches"]
+            traffic = sum(x["dram_bytes"] for x in ls) / len(ls) / 1e9
+            traffic_src = tj["source"]
+    except Exception:
+        pass
     roofline = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
-                "frac": achieved / hbm_peak, "traffic": None,
+                "frac": achieved / hbm_peak, "traffic": traffic, "traffic_unit": "GB per launch",
+                "traffic_source": traffic_src,
+                "algorithmic_gb_per_call": alg_bytes / max(1, spmm_calls) / 1e9,
+                "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)",
                 "kernel": "spmm (rdm::spmm_kernel + heavy-row reduce)",
                 "spmm_share_of_step": ph_ms["spmm"] / max(1e-9, ms_total),
                 "avg_call_ms": ph_ms["spmm"] / max(1, spmm_calls),
