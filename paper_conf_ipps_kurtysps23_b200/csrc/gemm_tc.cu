@@ -65,6 +65,29 @@ __device__ __forceinline__ void mbar_wait(uint64_t* b, uint32_t parity) {
         : "memory");
   } while (!done);
 }
+// Wait with back-off, for warps whose wait is long and off the critical path
+// (epilogue warps idle through a whole mainloop): keeps their polling from
+// stealing issue slots from the converter warps on the same SM sub-partition.
+__device__ __forceinline__ void mbar_wait_sleep(uint64_t* b, uint32_t parity) {
+  uint32_t done;
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+      "selp.b32 %0, 1, 0, p;\n\t}"
+      : "=r"(done)
+      : "r"(smem_u32(b)), "r"(parity)
+      : "memory");
+  while (!done) {
+    __nanosleep(256);
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "mbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\n\t"
+        "selp.b32 %0, 1, 0, p;\n\t}"
+        : "=r"(done)
+        : "r"(smem_u32(b)), "r"(parity)
+        : "memory");
+  }
+}
 __device__ __forceinline__ void tma_load_2d(void* dst, const CUtensorMap* map, uint64_t* bar, int c0,
                                             int c1) {
   asm volatile(
@@ -181,15 +204,20 @@ struct TcShape {
 // smem-bandwidth bound of the converter (write hi + lo) plus three MMA reads
 // of A per k-block.  BN = 256 needs all 512 TMEM columns for the two
 // accumulators and keeps A in shared memory.
-template <int BN>
+// EW = epilogue warps: 4 (one per TMEM lane quadrant) for mainloop-bound
+// calls, 8 (two per quadrant, column halves) for epilogue-bound ones (short
+// K, wide outputs) — 8 warps cost one smem stage of transpose buffers.
+template <int BN, int EW>
 struct Cfg {
+  static constexpr int kEpiWarps = EW;
+  static constexpr int kThreads = 256 + 32 * EW;
   static constexpr int kAccCols = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
   static constexpr bool kTmemA = BN <= 128;
   static constexpr int kNAcc = !kTmemA ? 1 : BN <= 32 ? 4 : BN <= 64 ? 2 : 1;  // partial accumulators
   static constexpr int kABytes = BM * BK * 4;   // 16 KB
   static constexpr int kBBytes = BN * BK * 4;
   static constexpr int kStageBytes = (kTmemA ? 1 : 2) * kABytes + 2 * kBBytes;
-  static constexpr int kEpiBytes = 4 * 32 * 33 * 4;   // per-warp 32 x 32 transpose tiles (+1 pad)
+  static constexpr int kEpiBytes = EW * 32 * 33 * 4;  // per-warp 32 x 32 transpose tiles (+1 pad)
   static constexpr int kBudget = 224 * 1024 - kEpiBytes - 1024 - 256;
   // deep rings hide TMA latency; with A in TMEM each stage also takes 64 columns
   static constexpr int kMaxStages = kTmemA ? (512 - 2 * kNAcc * kAccCols) / (2 * BK) : 4;
@@ -258,13 +286,13 @@ __device__ __forceinline__ void load_a_row(const uint8_t* tile, int m, float (&v
 // overlaps the mainloop of tile i + 1.
 // MODE 0: NN/NT (A K-major + converter, B pre-split K-major).
 // MODE 1: TN (A, B MN-major, both split in smem), split-K slabs.
-template <int BN, int MODE>
-__global__ void __launch_bounds__(384, 1)
+template <int BN, int MODE, int EW>
+__global__ void __launch_bounds__(256 + 32 * EW, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const __grid_constant__ CUtensorMap tmBlo, const __grid_constant__ CUtensorMap tmApf,
                float* __restrict__ C, int64_t ldc,
                TcShape sh, TcEpi epi) {
-  using CF = Cfg<BN>;
+  using CF = Cfg<BN, EW>;
   constexpr int S = CF::kStages;
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
@@ -301,7 +329,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&tfull[b], 1);
-      mbar_init(&tempty[b], 128);
+      mbar_init(&tempty[b], 32 * EW);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
@@ -449,8 +477,9 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       }
     }
   } else if (warp >= 8) {
-    const int q = warp - 8;                    // TMEM lane quadrant of this warp
-    float* tb = epi_smem + q * 32 * 33;        // 32 x 32 transpose tile
+    const int q = warp & 3;                    // TMEM lane quadrant of this warp
+    const int half = (warp - 8) >> 2;          // column half (chunks 32 apart)
+    float* tb = epi_smem + (warp - 8) * 32 * 33;  // 32 x 32 transpose tile
     int it = 0;
     for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
       int64_t kbeg;
@@ -458,12 +487,12 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       const int z = t / tiles_mn, rem = t % tiles_mn;
       const int64_t m0 = (int64_t)(rem / sh.tiles_n) * BM, n0 = (int64_t)(rem % sh.tiles_n) * BN;
       const int acc = it & 1;
-      mbar_wait(&tfull[acc], (it >> 1) & 1);
+      mbar_wait_sleep(&tfull[acc], (it >> 1) & 1);
       tc_fence_after();
       float* Cz = C + (int64_t)z * sh.M * ldc;
       const int64_t row0 = m0 + q * 32;
 #pragma unroll 1
-      for (int c0 = 0; c0 < BN; c0 += 32) {
+      for (int c0 = 32 * half; c0 < BN; c0 += 32 * (EW / 4)) {
         if (n0 + c0 >= sh.N) break;
         uint32_t r[32];
         if (nkb > 0) {
@@ -598,12 +627,12 @@ CUtensorMap make_map(const float* base, int64_t inner, int64_t outer, int64_t ld
   return m;
 }
 
-template <int BN, int MODE>
-void launch_tc(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& blo,
+template <int BN, int MODE, int EW>
+void launch_tc_ew(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& blo,
                float* C, int64_t ldc, int64_t M, int64_t N, int64_t K, int splits, int n_mma,
                const TcEpi& e, const CUtensorMap* apf = nullptr) {
-  using CF = Cfg<BN>;
-  RDM_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<BN, MODE>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+  using CF = Cfg<BN, EW>;
+  RDM_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<BN, MODE, EW>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                 CF::kSmem));
   TcShape sh;
   sh.M = M;
@@ -619,9 +648,20 @@ void launch_tc(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, const C
   sh.dbg = dbg ? atoi(dbg) : 0;
   const int64_t total = (int64_t)sh.tiles_m * sh.tiles_n * splits;
   const unsigned grid = (unsigned)std::min<int64_t>(total, ctx->num_sms);
-  gemm_tc_kernel<BN, MODE><<<grid, 384, CF::kSmem, ctx->stream>>>(a, b, blo, apf ? *apf : a, C, ldc,
+  gemm_tc_kernel<BN, MODE, EW><<<grid, CF::kThreads, CF::kSmem, ctx->stream>>>(a, b, blo, apf ? *apf : a, C, ldc,
                                                                   sh, e);
   RDM_LAUNCHED(ctx);
+}
+
+template <int BN, int MODE>
+void launch_tc(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& blo,
+               float* C, int64_t ldc, int64_t M, int64_t N, int64_t K, int splits, int n_mma,
+               const TcEpi& e, const CUtensorMap* apf = nullptr) {
+  // short contractions produce a wide output per k-block: epilogue-bound
+  if (BN <= 128 && K <= 256)
+    launch_tc_ew<BN, MODE, 8>(ctx, a, b, blo, C, ldc, M, N, K, splits, n_mma, e, apf);
+  else
+    launch_tc_ew<BN, MODE, 4>(ctx, a, b, blo, C, ldc, M, N, K, splits, n_mma, e, apf);
 }
 
 int pick_bn(int64_t N) {
