@@ -42,6 +42,8 @@ def parse():
     ap.add_argument("--no-cpu-baseline", action="store_true")
     ap.add_argument("--cpu-seconds", type=float, default=12.0)
     ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p"],
+                    help="redistribution transport for N > 1 (rdm.h rdm_set_transport)")
     ap.add_argument("--sweep", action="store_true",
                     help="also time every configuration (Table VIII analogue) into config.sweep_ms")
     return ap.parse_args()
@@ -218,6 +220,7 @@ def main():
 
     ctx = rdm.Context(rank=rank if world > 1 else 0, world=world, device=local_rank, stream=stream,
                       unique_id=uid)
+    ctx.set_transport(a.transport)
     ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
     pareto, chosen, comm_u, sparse_u = rdm.select_config(list(wl.f), wl.n, wl.nnz, world)
     lo, hi, _ = rdm.partition(world, rdm.ROW, wl.n, wl.f[0], rank if world > 1 else 0)
@@ -398,6 +401,7 @@ def main():
                 "n": n, "nnz": nnz, "graph": "R-MAT (0.57,0.19,0.19,0.05), permuted, symmetric, "
                 "self loops, D^-1/2 (A+I) D^-1/2", "global_batch": n, "seq_len": None,
                 "parallelism": f"rdm{world} (A replicated, H row/col redistributed)",
+                "transport": a.transport,
                 "config_id": cfg_id, "config_name": rdm.config_name(model.cfg),
                 "pareto": pareto, "pick": a.config,
                 "sweep_ms": ({str(k): round(v, 4) for k, v in sweep.items()} if sweep else None),

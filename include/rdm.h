@@ -167,6 +167,24 @@ const char* rdm_last_error(const rdm_ctx* ctx);
 /* Block until the ctx's stream is idle; surfaces asynchronous CUDA/NCCL faults. */
 rdm_status rdm_sync(rdm_ctx* ctx);
 rdm_status rdm_set_stream(rdm_ctx* ctx, void* cuda_stream);
+
+/* Transport of the GCN executor's redistributions (§III-D; SURVEY
+ * §8(e) "Phase 2"):
+ *   RDM_TRANSPORT_NCCL (default): pack → NCCL grouped send/recv → unpack.
+ *   RDM_TRANSPORT_P2P: a redistribution whose source was produced by the
+ *     step right before it is fused into that producer: the GEMM (row → col)
+ *     or SpMM (col → row) epilogue stores every output element straight into
+ *     its owner's destination slice — the other slots' buffers in a virtual
+ *     group, CUDA-IPC-mapped peer memory over NVLink for NCCL ranks (fenced
+ *     by two one-word NCCL all-reduces around the producer).  Unfused
+ *     redistributions keep the NCCL path.  Results are bit-identical to the
+ *     default (pure data movement); counters count the same logical traffic.
+ * Takes effect for GCN instances created afterwards.  The environment
+ * variable RDM_P2P=1 selects P2P at rdm_init.  Errors: RDM_ERR_ARG. */
+enum { RDM_TRANSPORT_NCCL = 0, RDM_TRANSPORT_P2P = 1 };
+rdm_status rdm_set_transport(rdm_ctx* ctx, int transport);
+int rdm_get_transport(const rdm_ctx* ctx);
+
 int rdm_world(const rdm_ctx* ctx);
 int rdm_num_local(const rdm_ctx* ctx);            /* local rank slots (1 or world)  */
 int rdm_local_rank(const rdm_ctx* ctx, int slot); /* global rank of local slot      */
@@ -361,6 +379,11 @@ rdm_status rdm_set_timing(rdm_ctx* ctx, int enable);
  * reset (synchronises the stream). */
 rdm_status rdm_get_phase_times(rdm_ctx* ctx, double* ms, int64_t* launches);
 rdm_status rdm_reset_phase_times(rdm_ctx* ctx);
+
+/* Debug: route every NN/NT/TN GEMM to the SIMT fp32 kernel (disable != 0)
+ * instead of the tcgen05 3xTF32 kernel (0, default).  Process-wide; for
+ * cross-checking the two GEMM paths.  Returns 0. */
+int rdm_debug_disable_tc(int disable);
 
 #ifdef __cplusplus
 }

@@ -35,6 +35,8 @@ PHASES = ["spmm", "gemm", "pack", "a2a", "loss", "allreduce", "adam", "other"]
 _STATUS = {0: "OK", 1: "ERR_ARG", 2: "ERR_CUDA", 3: "ERR_NCCL", 4: "ERR_OOM",
            5: "ERR_UNSUPPORTED", 6: "ERR_STATE"}
 
+TRANSPORTS = {"nccl": 0, "p2p": 1}
+
 # C symbols declared in include/rdm.h (checked by tests/test_abi.py)
 EXPORTS = [
     "rdm_get_unique_id", "rdm_init", "rdm_finalize", "rdm_last_error", "rdm_sync",
@@ -45,6 +47,7 @@ EXPORTS = [
     "rdm_gcn_backward", "rdm_gcn_get_info", "rdm_gcn_describe", "rdm_gcn_tensor",
     "rdm_adam_step", "rdm_get_counters", "rdm_reset_counters", "rdm_set_timing",
     "rdm_get_phase_times", "rdm_reset_phase_times", "rdm_redist_plan", "rdm_plan_info",
+    "rdm_set_transport", "rdm_get_transport", "rdm_debug_disable_tc",
 ]
 
 
@@ -106,6 +109,7 @@ _sig = {
     "rdm_get_counters": [_vp, ctypes.POINTER(RdmCounters)],
     "rdm_reset_counters": [_vp],
     "rdm_set_timing": [_vp, _int],
+    "rdm_set_transport": [_vp, _int],
     "rdm_get_phase_times": [_vp, ctypes.POINTER(ctypes.c_double), _pi64],
     "rdm_reset_phase_times": [_vp],
     "rdm_redist_plan": [_int, _int, _int, _i64, _i64, _pi64, _pi64, _pi64, _pi64],
@@ -119,9 +123,11 @@ _lib.rdm_last_error.argtypes = [_vp]
 _lib.rdm_last_error.restype = ctypes.c_char_p
 _lib.rdm_config_to_id.argtypes = [ctypes.POINTER(RdmConfig)]
 _lib.rdm_config_to_id.restype = _i64
-for _n in ("rdm_world", "rdm_num_local"):
+for _n in ("rdm_world", "rdm_num_local", "rdm_get_transport"):
     getattr(_lib, _n).argtypes = [_vp]
     getattr(_lib, _n).restype = _int
+_lib.rdm_debug_disable_tc.argtypes = [_int]
+_lib.rdm_debug_disable_tc.restype = _int
 _lib.rdm_local_rank.argtypes = [_vp, _int]
 _lib.rdm_local_rank.restype = _int
 
@@ -168,6 +174,11 @@ def get_unique_id() -> bytes:
     buf = ctypes.create_string_buffer(UNIQUE_ID_BYTES)
     _check(_lib.rdm_get_unique_id(buf), what="rdm_get_unique_id")
     return buf.raw
+
+
+def debug_disable_tc(disable=True):
+    """Route GEMMs to the SIMT kernel instead of tcgen05 (rdm.h rdm_debug_disable_tc)."""
+    _lib.rdm_debug_disable_tc(int(bool(disable)))
 
 
 def partition(world, layout, n, f, rank):
@@ -315,6 +326,16 @@ class Context:
 
     def set_timing(self, on=True):
         self._c(_lib.rdm_set_timing(self.h, int(on)))
+
+    def set_transport(self, transport):
+        """"nccl" (pack + all-to-all + unpack) or "p2p" (redistributions fused
+        into their producing kernel's epilogue, rdm.h rdm_set_transport);
+        applies to GCN instances created afterwards."""
+        self._c(_lib.rdm_set_transport(self.h, TRANSPORTS[transport]))
+
+    @property
+    def transport(self):
+        return {v: k for k, v in TRANSPORTS.items()}[_lib.rdm_get_transport(self.h)]
 
     def phase_times(self):
         ms = (ctypes.c_double * len(PHASES))()

@@ -47,6 +47,7 @@ struct Step {
   int lin = 0, lin2 = 0, lout = 0, lmask = 0;
   int64_t width = 0;
   bool hidden = false;
+  int fuse = 0;   // RDM_TRANSPORT_P2P: 1 = producer also scatters (next step), 2 = redist done by producer
 };
 
 struct Planner {
@@ -271,6 +272,11 @@ struct rdm_gcn {
   bool staged = false;
   int64_t ws_bytes = 0;
   rdm_gcn_info info{};
+  // fused redistribution (RDM_TRANSPORT_P2P): destination base per rank of
+  // every fused (tensor, layout), and the IPC mappings to close at destroy
+  bool p2p = false;
+  std::map<std::pair<int, int>, std::vector<float*>> peers;
+  std::vector<void*> ipc_opened;
 };
 
 namespace rdm {
@@ -343,6 +349,71 @@ void plan_info(const Planner& pl, const std::vector<Step>& fwd, const std::vecto
 
 std::string describe_steps(const std::vector<Step>& fwd, const std::vector<Step>& bwd);
 
+// Fused redistribution (§III-D's all-to-all folded into the producing kernel;
+// SURVEY §8(e)): a REDIST whose source the step right before it produced, in
+// the producer's own layout (GEMM → row slice → column slices; SpMM → column
+// slice → row slices), is replaced by the producer storing each element into
+// its owner's destination slice as well.
+void setup_fusion(rdm_gcn* g) {
+  rdm_ctx* ctx = g->ctx;
+  g->p2p = true;
+  for (auto* v : {&g->fwd, &g->bwd}) {
+    auto& st = *v;
+    for (size_t i = 0; i + 1 < st.size(); ++i) {
+      Step& a = st[i];
+      Step& r = st[i + 1];
+      if (r.op != S_REDIST || r.in.id() != a.out.id() || r.lin != a.lout) continue;
+      if (!((a.op == S_GEMM && a.lout == RDM_ROW) || (a.op == S_SPMM && a.lout == RDM_COL))) continue;
+      a.fuse = 1;
+      r.fuse = 2;
+      const auto key = std::make_pair(r.out.id(), norm_lay(g, r.lout));
+      if (g->peers.count(key)) continue;
+      std::vector<float*> ptr(ctx->world, nullptr);
+      if (ctx->virtual_group()) {
+        for (int q = 0; q < ctx->world; ++q) ptr[q] = buf(g, q, r.out, r.lout).p;
+      } else {
+        ptr = p2p_open(ctx, buf(g, 0, r.out, r.lout).p, g->ipc_opened);
+      }
+      g->peers[key] = ptr;
+    }
+  }
+}
+
+// Scatter descriptor of fused producer step `s` for local slot i.
+Scatter make_scatter(rdm_gcn* g, const Step& s, int i) {
+  rdm_ctx* ctx = g->ctx;
+  const int P = ctx->world;
+  const int p = ctx->local[i];
+  const int64_t n = ctx->graph.n, w = s.width;
+  const int dl = s.lout == RDM_ROW ? RDM_COL : RDM_ROW;
+  const std::vector<float*>& ptr = g->peers.at({s.out.id(), norm_lay(g, dl)});
+  Scatter sc;
+  sc.P = P;
+  if (s.op == S_GEMM) {   // row slice → column slices
+    sc.mode = 1;
+    for (int q = 0; q < P; ++q) {
+      const Range c = col_range(w, P, q);
+      sc.lo[q] = c.lo;
+      sc.ld[q] = roundup4(c.size());
+      sc.ptr[q] = ptr[q];
+    }
+    sc.lo[P] = w;
+    sc.my_off = row_range(n, P, p).lo;
+  } else {                // column slice → row slices
+    sc.mode = 2;
+    for (int q = 0; q < P; ++q) {
+      sc.lo[q] = row_range(n, P, q).lo;
+      sc.ld[q] = roundup4(w);
+      sc.ptr[q] = ptr[q];
+    }
+    sc.lo[P] = n;
+    const Range c = col_range(w, P, p);
+    sc.my_off = c.lo;
+    sc.my_w = c.size();
+  }
+  return sc;
+}
+
 void create(rdm_gcn* g) {
   rdm_ctx* ctx = g->ctx;
   Planner& pl = g->pl;
@@ -409,12 +480,16 @@ void create(rdm_gcn* g) {
   }
   plan_info(pl, g->fwd, g->bwd, n, &g->info);
   g->info.workspace_bytes = g->ws_bytes;
+  if (ctx->transport == RDM_TRANSPORT_P2P && P > 1) setup_fusion(g);
 }
 
 void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
   rdm_ctx* ctx = g->ctx;
   const int nl = ctx->nlocal();
   const int P = ctx->world;
+  // a fused producer overwrites peers' destination slices: every rank must be
+  // done reading their previous contents
+  if (s.fuse == 1) p2p_barrier(ctx);
   switch (s.op) {
     case S_SPMM: {
       Phase ph(ctx, RDM_PH_SPMM);
@@ -430,7 +505,12 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
           ldm = m.ld;
         }
         const int64_t w = P == 1 ? s.width : col_range(s.width, P, ctx->local[i]).size();
-        spmm(ctx, A, in.p, in.ld, out.p, out.ld, w, s.epi, nullptr, mk, ldm);
+        if (s.fuse == 1) {
+          const Scatter sc = make_scatter(g, s, i);
+          spmm(ctx, A, in.p, in.ld, out.p, out.ld, w, s.epi, nullptr, mk, ldm, &sc);
+        } else {
+          spmm(ctx, A, in.p, in.ld, out.p, out.ld, w, s.epi, nullptr, mk, ldm);
+        }
       }
       ctx->counters.spmm_width_units += s.width;
       break;
@@ -442,8 +522,10 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
         Buf& in = buf(g, i, s.in, s.lin);
         Buf& out = buf(g, i, s.out, s.lout);
         const float* mk = (s.epi & RDM_EPI_MASK) ? buf(g, i, s.mask, s.lmask).p : nullptr;
+        Scatter sc;
+        if (s.fuse == 1) sc = make_scatter(g, s, i);
         gemm(ctx, s.gop, in.p, in.ld, W[s.wl - 1], fout, out.p, out.ld, in.rows, fin, fout, s.epi,
-             nullptr, mk);
+             nullptr, mk, s.fuse == 1 ? &sc : nullptr);
       }
       break;
     }
@@ -460,6 +542,11 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
       break;
     }
     case S_REDIST: {
+      if (s.fuse == 2) {   // the producer already stored it; fence peers before the consumer
+        p2p_barrier(ctx);
+        count_fused_redist(ctx, (rdm_layout)s.lin, ctx->graph.n, s.width);
+        break;
+      }
       std::vector<const float*> src(nl);
       std::vector<float*> dst(nl);
       for (int i = 0; i < nl; ++i) {
@@ -512,7 +599,7 @@ std::string step_str(const Step& s) {
       break;
     case S_REDIST:
       o << "A2A   " << k(s.in, s.lin) << " -> " << k(s.out, s.lout) << " f=" << s.width
-        << (s.hidden ? " (hidden)" : "");
+        << (s.hidden ? " (hidden)" : "") << (s.fuse == 2 ? " [fused into producer]" : "");
       break;
     case S_MASK:
       o << "MASK  " << k(s.out, s.lout) << " *= 1[" << k(s.mask, s.lmask) << " > 0]";
@@ -762,6 +849,12 @@ rdm_status rdm_gcn_destroy(rdm_gcn* g) {
     cudaStreamDestroy(g->cs);
     cudaEventDestroy(g->ev_ready);
     cudaEventDestroy(g->ev_free);
+  }
+  if (!g->ipc_opened.empty()) {
+    // no rank may free a slice a peer still maps: close, then fence, then free
+    for (void* p : g->ipc_opened) cudaIpcCloseMemHandle(p);
+    rdm_guarded_call(g->ctx, [](void* c) { p2p_barrier(static_cast<rdm_ctx*>(c)); }, g->ctx);
+    cudaStreamSynchronize(g->ctx->stream);
   }
   delete g;
   return RDM_OK;

@@ -189,6 +189,7 @@ struct TcEpi {
   const float* bias;
   const float* mask;
   int64_t ld_mask;
+  Scatter scat;   // fused row→column redistribution (MODE 0, no split-K); scat.P == 0: off
 };
 
 struct TcShape {
@@ -553,6 +554,17 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           const int nrows = (sh.M - row0) < 32 ? (int)(sh.M - row0) : 32;
 #pragma unroll 8
           for (int rr = 0; rr < nrows; ++rr) Cz[(row0 + rr) * ldc + col] = tb[rr * 33 + lane];
+          if (MODE == 0 && epi.scat.P) {
+            // the same coalesced rows, stored into the owner of column `col`
+            // (its column slice keeps global rows: my_off + row)
+            const Scatter& s = epi.scat;
+            int q = 0;
+            while (q + 1 < s.P && s.lo[q + 1] <= col) ++q;
+            const int64_t ldq = s.ld[q];
+            float* d = s.ptr[q] + (s.my_off + row0) * ldq + (col - s.lo[q]);
+#pragma unroll 8
+            for (int rr = 0; rr < nrows; ++rr) d[rr * ldq] = tb[rr * 33 + lane];
+          }
         }
         __syncwarp();
       }
@@ -732,14 +744,15 @@ static bool g_tc_disabled = false;
 
 bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, int64_t ldw,
              float* C, int64_t ldc, int64_t rows, int64_t k, int64_t m, int epi, const float* bias,
-             const float* mask) {
+             const float* mask, const Scatter* scat) {
   if (g_tc_disabled) return false;
   // TMA: global base 16-byte aligned, row strides multiples of 16 bytes
   if (((uintptr_t)X & 15) || (ldx & 3)) return false;
   // the epilogue reads mask rows as float4: 16-byte aligned rows required
   if ((epi & RDM_EPI_MASK) && (((uintptr_t)mask & 15) || (ldc & 3))) return false;
-  TcEpi e{epi, bias, mask, ldc};
+  TcEpi e{epi, bias, mask, ldc, Scatter{}};
   if (op == RDM_GEMM_NN || op == RDM_GEMM_NT) {
+    if (scat) e.scat = *scat;
     const int64_t M = rows;
     const int64_t N = op == RDM_GEMM_NN ? m : k;   // output columns
     const int64_t K = op == RDM_GEMM_NN ? k : m;   // contraction
@@ -754,6 +767,7 @@ bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, 
     return true;
   }
   // TN: C[k x m] = Xᵀ U  (X rows x k at ldx, U rows x m at ldw)
+  if (scat) return false;   // weight gradients are never redistributed
   if (((uintptr_t)W & 15) || (ldw & 3)) return false;
   const int64_t M = k, N = m, K = rows;
   const int BN = N <= 32 ? 32 : N <= 64 ? 64 : (N <= 128 || !getenv("RDM_BN256")) ? 128 : 256;

@@ -122,6 +122,7 @@ struct rdm_ctx {
   cudaStream_t stream = nullptr;
   ncclComm_t comm = nullptr;
   bool poisoned = false;
+  int transport = 0;             // RDM_TRANSPORT_NCCL / RDM_TRANSPORT_P2P
   std::string err;
   rdm::Graph graph;
   bool has_graph = false;
@@ -162,16 +163,32 @@ struct Phase {
   ~Phase();
 };
 
+// Fused redistribution ("p2p" transport): the producing kernel of a tensor
+// that is redistributed next also stores every element straight into its
+// owner's destination layout (peer memory over NVLink for NCCL ranks, the
+// other slots' buffers in a virtual group), replacing pack + all-to-all.
+struct Scatter {
+  static constexpr int kMax = 64;
+  int P = 0;                 // 0 = no scatter
+  int mode = 0;              // 1: row slice → column slices (GEMM), 2: column slice → row slices (SpMM)
+  int64_t lo[kMax + 1] = {}; // destination partition: columns (mode 1) / rows (mode 2)
+  int64_t ld[kMax] = {};     // destination leading dim per rank
+  float* ptr[kMax] = {};     // destination base per rank
+  int64_t my_off = 0;        // mode 1: my first global row; mode 2: my first global column
+  int64_t my_w = 0;          // mode 2: real width of my column slice
+};
+
 // ------------------------------------------------------------------ kernels
 // spmm.cu
 void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
-          int64_t w, int epi, const float* bias, const float* mask, int64_t ld_mask);
+          int64_t w, int epi, const float* bias, const float* mask, int64_t ld_mask,
+          const Scatter* scat = nullptr);
 void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host);
 
 // gemm.cu
 void gemm(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, int64_t ldw, float* C,
           int64_t ldc, int64_t rows, int64_t k, int64_t m, int epi, const float* bias,
-          const float* mask);
+          const float* mask, const Scatter* scat = nullptr);
 // C[M x N] = A[M x K] · B with B given as pre-split tf32 hi / lo panels
 // Bt[N][K] (K-major, row length ldb; 16-byte aligned), on the tensor cores.
 void gemm_tc_panels(rdm_ctx* ctx, const float* A, int64_t lda, const float* bhi, const float* blo,
@@ -179,6 +196,11 @@ void gemm_tc_panels(rdm_ctx* ctx, const float* A, int64_t lda, const float* bhi,
 // dense hub core (spmm.cu)
 void build_core(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, const int32_t* col_host,
                 const float* val_host);
+
+// runtime.cpp — fused ("p2p") redistribution support
+void count_fused_redist(rdm_ctx* ctx, rdm_layout from, int64_t n, int64_t f);
+void p2p_barrier(rdm_ctx* ctx);
+std::vector<float*> p2p_open(rdm_ctx* ctx, float* mine, std::vector<void*>& opened);
 
 // Round-to-nearest fp32 → tf32 (ties away from zero), used by every 3xTF32 split.
 __device__ __forceinline__ float tf32_rn(float x) {
@@ -199,6 +221,10 @@ void pack_rows(rdm_ctx* ctx, const float* row_slice, int64_t ld_row, int64_t row
                const BlockTable& t);
 void unpack_rows(rdm_ctx* ctx, float* row_slice, int64_t ld_row, int64_t rows, int P,
                  const BlockTable& t);
+// Unfused form of a Scatter (producers without a fused epilogue): copies the
+// rows x cols slice `src` into the destinations the descriptor names.
+void scatter_slice(rdm_ctx* ctx, const float* src, int64_t lds, int64_t rows, int64_t cols,
+                   const Scatter& s);
 
 // misc.cu
 void softmax_xent(rdm_ctx* ctx, const float* Z, int64_t ldz, const int32_t* labels,

@@ -101,4 +101,32 @@ void unpack_rows(rdm_ctx* ctx, float* row_slice, int64_t ld_row, int64_t rows, i
   RDM_LAUNCHED(ctx);
 }
 
+namespace {
+__global__ void scatter_kernel(const float* __restrict__ src, int64_t lds, int64_t rows, int64_t cols,
+                               Scatter s) {
+  const int64_t total = rows * cols;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / cols, c = i % cols;
+    const float x = src[r * lds + c];
+    if (s.mode == 1) {   // row slice → column slices (global rows my_off + r)
+      int q = 0;
+      while (q + 1 < s.P && s.lo[q + 1] <= c) ++q;
+      s.ptr[q][(s.my_off + r) * s.ld[q] + (c - s.lo[q])] = x;
+    } else if (c < s.my_w) {   // column slice → row slices (global columns my_off + c)
+      int q = 0;
+      while (q + 1 < s.P && s.lo[q + 1] <= r) ++q;
+      s.ptr[q][(r - s.lo[q]) * s.ld[q] + s.my_off + c] = x;
+    }
+  }
+}
+}  // namespace
+
+void scatter_slice(rdm_ctx* ctx, const float* src, int64_t lds, int64_t rows, int64_t cols,
+                   const Scatter& s) {
+  if (rows == 0 || cols == 0) return;
+  scatter_kernel<<<grid_for(ctx, rows * cols), 256, 0, ctx->stream>>>(src, lds, rows, cols, s);
+  RDM_LAUNCHED(ctx);
+}
+
 }  // namespace rdm

@@ -16,7 +16,7 @@ void gemm_simt(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W
                const float* bias, const float* mask);
 bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, int64_t ldw,
              float* C, int64_t ldc, int64_t rows, int64_t k, int64_t m, int epi, const float* bias,
-             const float* mask);
+             const float* mask, const Scatter* scat);
 
 #define RDM_NCCL(call)                                                                     \
   do {                                                                                     \
@@ -242,6 +242,62 @@ void redistribute(rdm_ctx* ctx, rdm_layout from, const float* const* src, float*
   ctx->counters.a2a_width_units += f;
 }
 
+// A redistribution fused into its producer (RDM_TRANSPORT_P2P): the data
+// already moved; count the same logical traffic as redistribute() — payload
+// elements and the wire bytes the producer stored into peer memory (real
+// elements only: no ld padding crosses the link).
+void count_fused_redist(rdm_ctx* ctx, rdm_layout from, int64_t n, int64_t f) {
+  const int P = ctx->world;
+  int64_t payload = 0;
+  for (int i = 0; i < ctx->nlocal(); ++i) {
+    const int p = ctx->local[i];
+    for (int q = 0; q < P; ++q) {
+      if (q == p) continue;
+      payload += from == RDM_ROW ? row_range(n, P, p).size() * col_range(f, P, q).size()
+                                 : row_range(n, P, q).size() * col_range(f, P, p).size();
+    }
+  }
+  ctx->counters.a2a_calls++;
+  ctx->counters.a2a_elems_payload += payload;
+  ctx->counters.a2a_bytes_wire += payload * (int64_t)sizeof(float);
+  ctx->counters.a2a_width_units += f;
+}
+
+// Stream-ordered barrier across NCCL ranks (one-word all-reduce): when it
+// completes on my stream, every rank's stream has reached the same point.
+// Virtual group / P = 1: stream order already is the barrier.
+void p2p_barrier(rdm_ctx* ctx) {
+  if (ctx->world == 1 || ctx->virtual_group()) return;
+  Phase ph(ctx, RDM_PH_A2A);
+  float* w = ensure_ws(ctx->ws_scratch, 4096);
+  RDM_NCCL(ncclAllReduce(w, w, 1, ncclFloat, ncclSum, ctx->comm, ctx->stream));
+}
+
+// Peer base addresses of one device allocation per rank (CUDA IPC, handles
+// all-gathered over NCCL).  Virtual group: not used (slots share a process).
+std::vector<float*> p2p_open(rdm_ctx* ctx, float* mine, std::vector<void*>& opened) {
+  const int P = ctx->world;
+  std::vector<float*> out(P, nullptr);
+  out[ctx->rank] = mine;
+  cudaIpcMemHandle_t h;
+  RDM_CUDA(cudaIpcGetMemHandle(&h, mine));
+  constexpr size_t hb = sizeof(cudaIpcMemHandle_t);
+  uint8_t* d = reinterpret_cast<uint8_t*>(ensure_ws(ctx->ws_scratch, 4096 + P * hb));
+  RDM_CUDA(cudaMemcpyAsync(d + 1024, &h, hb, cudaMemcpyHostToDevice, ctx->stream));
+  RDM_NCCL(ncclAllGather(d + 1024, d + 1024 + hb, hb, ncclUint8, ctx->comm, ctx->stream));
+  std::vector<cudaIpcMemHandle_t> all(P);
+  RDM_CUDA(cudaMemcpyAsync(all.data(), d + 1024 + hb, P * hb, cudaMemcpyDeviceToHost, ctx->stream));
+  RDM_CUDA(cudaStreamSynchronize(ctx->stream));
+  for (int q = 0; q < P; ++q) {
+    if (q == ctx->rank) continue;
+    void* ptr = nullptr;
+    RDM_CUDA(cudaIpcOpenMemHandle(&ptr, all[q], cudaIpcMemLazyEnablePeerAccess));
+    opened.push_back(ptr);
+    out[q] = static_cast<float*>(ptr);
+  }
+  return out;
+}
+
 // ------------------------------------------------------------------ graph
 static void upload_csr(rdm_ctx* ctx, Csr& A, int64_t n, int64_t nnz, const int64_t* rowptr,
                        const int32_t* col, const float* val, bool on_host) {
@@ -366,6 +422,7 @@ rdm_status rdm_init(rdm_ctx** out, int rank, int world, const void* uid, int dev
     return RDM_ERR_CUDA;
   }
   rdm_ctx* ctx = new rdm_ctx();
+  if (const char* e = getenv("RDM_P2P")) ctx->transport = atoi(e) ? RDM_TRANSPORT_P2P : RDM_TRANSPORT_NCCL;
   ctx->world = world;
   ctx->rank = (world == 1) ? 0 : rank;
   ctx->device = device;
@@ -426,6 +483,14 @@ rdm_status rdm_set_stream(rdm_ctx* ctx, void* stream) {
   return RDM_OK;
 }
 
+rdm_status rdm_set_transport(rdm_ctx* ctx, int transport) {
+  if (!ctx || (transport != RDM_TRANSPORT_NCCL && transport != RDM_TRANSPORT_P2P)) return RDM_ERR_ARG;
+  ctx->transport = transport;
+  return RDM_OK;
+}
+
+int rdm_get_transport(const rdm_ctx* ctx) { return ctx ? ctx->transport : -1; }
+
 int rdm_world(const rdm_ctx* ctx) { return ctx ? ctx->world : -1; }
 int rdm_num_local(const rdm_ctx* ctx) { return ctx ? ctx->nlocal() : -1; }
 int rdm_local_rank(const rdm_ctx* ctx, int slot) {
@@ -480,8 +545,11 @@ rdm_status rdm_spmm(rdm_ctx* ctx, int transpose, const float* in, int64_t ld_in,
 namespace rdm {
 void gemm(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, int64_t ldw, float* C,
           int64_t ldc, int64_t rows, int64_t k, int64_t m, int epi, const float* bias,
-          const float* mask) {
+          const float* mask, const Scatter* scat) {
   RDM_CHECK_ARG(op >= 0 && op <= 2 && rows >= 0 && k >= 0 && m >= 0, "gemm: bad op/shape");
+  RDM_CHECK_ARG(!scat || (op != RDM_GEMM_TN && scat->mode == 1 && scat->P >= 1 &&
+                          scat->P <= Scatter::kMax),
+                "gemm: bad scatter descriptor");
   RDM_CHECK_ARG(!(epi & RDM_EPI_BIAS) || bias, "gemm: bias pointer missing");
   RDM_CHECK_ARG(!(epi & RDM_EPI_MASK) || mask, "gemm: mask pointer missing");
   RDM_CHECK_ARG(op != RDM_GEMM_TN || epi == 0, "gemm: TN takes no epilogue");
@@ -492,8 +560,9 @@ void gemm(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, int
       RDM_CUDA(cudaMemset2DAsync(C, ldc * 4, 0, m * 4, k, ctx->stream));
     return;
   }
-  if (gemm_tc(ctx, op, X, ldx, W, ldw, C, ldc, rows, k, m, epi, bias, mask)) return;
+  if (gemm_tc(ctx, op, X, ldx, W, ldw, C, ldc, rows, k, m, epi, bias, mask, scat)) return;
   gemm_simt(ctx, op, X, ldx, W, ldw, C, ldc, rows, k, m, epi, bias, mask);
+  if (scat) scatter_slice(ctx, C, ldc, rows, op == RDM_GEMM_NN ? m : k, *scat);
 }
 }  // namespace rdm
 

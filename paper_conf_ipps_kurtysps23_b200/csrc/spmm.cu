@@ -43,7 +43,24 @@ struct Epi {
   const float* core;        // hub-core product (K x ld_core) or null
   int64_t ld_core;
   const int32_t* hub_slot;  // int32[N], -1 for non-hubs
+  Scatter scat;             // fused col→row redistribution (scat.P == 0: off)
 };
+
+// Fused col→row redistribution: row r of my column slice (columns c..c+3 of
+// it) goes to the row-slice buffer of r's owner, at my global column offset.
+__device__ __forceinline__ void scatter_row_store(const Scatter& s, int64_t r, int64_t c, float4 v) {
+  if (c >= s.my_w) return;  // slice padding is not part of the row layout
+  int q = 0;
+  while (q + 1 < s.P && s.lo[q + 1] <= r) ++q;
+  float* d = s.ptr[q] + (r - s.lo[q]) * s.ld[q] + s.my_off + c;
+  if (c + 4 <= s.my_w) {
+    *reinterpret_cast<float4*>(d) = v;
+  } else {
+    d[0] = v.x;
+    if (c + 1 < s.my_w) d[1] = v.y;
+    if (c + 2 < s.my_w) d[2] = v.z;
+  }
+}
 
 __device__ __forceinline__ float4 apply_epi(float4 a, const Epi& e, int64_t row, int64_t c) {
   if (e.core) {  // add the dense hub-core contribution of this row (fixed order: after the CSR sum)
@@ -172,8 +189,11 @@ spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
 #pragma unroll
       for (int v = 0; v < V; ++v) {
         const int ch = v * G + sub;
-        if (ch < c4n)
-          reinterpret_cast<float4*>(dst)[ch] = apply_epi(acc[v], epi, r, cbase + 4 * ch);
+        if (ch < c4n) {
+          const float4 o = apply_epi(acc[v], epi, r, cbase + 4 * ch);
+          reinterpret_cast<float4*>(dst)[ch] = o;
+          if (epi.scat.P) scatter_row_store(epi.scat, r, cbase + 4 * ch, o);
+        }
       }
     }
   }
@@ -193,7 +213,9 @@ __global__ void spmm_heavy_reduce(const int32_t* __restrict__ heavy_rows,
       const float4 p = *reinterpret_cast<const float4*>(part + (int64_t)s * ld_part + c);
       acc.x += p.x; acc.y += p.y; acc.z += p.z; acc.w += p.w;
     }
-    *reinterpret_cast<float4*>(out + (int64_t)r * ld_out + c) = apply_epi(acc, epi, r, c);
+    const float4 o = apply_epi(acc, epi, r, c);
+    *reinterpret_cast<float4*>(out + (int64_t)r * ld_out + c) = o;
+    if (epi.scat.P) scatter_row_store(epi.scat, r, c, o);
   }
 }
 
@@ -273,7 +295,8 @@ __global__ void core_panels_kernel(const float* __restrict__ X, int64_t ldx,
 }  // namespace
 
 void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
-          int64_t w, int epi_flags, const float* bias, const float* mask, int64_t ld_mask) {
+          int64_t w, int epi_flags, const float* bias, const float* mask, int64_t ld_mask,
+          const Scatter* scat) {
   RDM_CHECK_ARG(w >= 0, "spmm: negative width");
   if (w == 0 || A.n == 0) return;
   const int64_t w4 = roundup4(w);
@@ -285,7 +308,12 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
                                                 ((uintptr_t)mask & 15) == 0),
                 "spmm: mask requires a 16-byte aligned N x w buffer with ld % 4 == 0");
   RDM_CHECK_ARG(!(epi_flags & RDM_EPI_BIAS) || bias, "spmm: bias pointer missing");
-  Epi epi{epi_flags, bias, mask, ld_mask, w, nullptr, 0, nullptr};
+  Epi epi{epi_flags, bias, mask, ld_mask, w, nullptr, 0, nullptr, Scatter{}};
+  if (scat) {
+    RDM_CHECK_ARG(scat->mode == 2 && scat->P >= 1 && scat->P <= Scatter::kMax && scat->my_w <= w,
+                  "spmm: bad scatter descriptor");
+    epi.scat = *scat;
+  }
   if (A.core.K && core_pays(A.core, w)) {
     // hub core on the tensor cores: panels Bt[n][k] = split(X[hub_k][n]), then
     // C_core = Acore · X[hubs]; the residual CSR's epilogue adds C_core rows.

@@ -22,7 +22,7 @@ def rdm():
     return r
 
 
-def _run(rdm, g, H0, Ws, y, m, cfg, P=1, epochs=1):
+def _run(rdm, g, H0, Ws, y, m, cfg, P=1, epochs=1, transport="nccl"):
     """Run `epochs` epochs (fwd, bwd, Adam) on P ranks (virtual group if P > 1);
     returns loss, dW (of the last epoch), model, ctx and the weights."""
     import torch
@@ -32,6 +32,7 @@ def _run(rdm, g, H0, Ws, y, m, cfg, P=1, epochs=1):
         ctx = rdm.Context(device=0)
     else:
         ctx = rdm.Context(rank=rdm.ALL_RANKS, world=P, device=0)
+    ctx.set_transport(transport)
     ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
     model = rdm.GCN(ctx, f, cfg)
     Hs, ys, ms = [], [], []
@@ -146,6 +147,70 @@ def test_virtual_group_configs(rdm, cora, P, cfg):
     assert info["plan_comm_units"] - info["plan_hidden_comm_units"] >= 0
     if cfg not in (6, 9):
         assert info["plan_hidden_comm_units"] == 0
+
+
+def _resident(model, rdm, which, layer, P):
+    out = []
+    for layout in (rdm.ROW, rdm.COL):
+        for p in range(P):
+            try:
+                out.append(model.tensor_torch(which, layer, p, layout).cpu().numpy())
+            except rdm.RdmError:
+                pass
+    return out
+
+
+@pytest.mark.parametrize("P", [2, 3, 4, 8])
+@pytest.mark.parametrize("cfg", [2, 3, 5, 6, 9, 10, 15])
+def test_p2p_fused_redistribution_bitwise(rdm, cora, P, cfg):
+    """RDM_TRANSPORT_P2P (redistribution fused into the producing GEMM / SpMM
+    epilogue, rdm.h) moves the same data as pack + all-to-all + unpack: every
+    resident tensor, the loss and dW are bit-identical; counters are equal."""
+    g, H0, Ws, y, m, ref = cora
+    la, dWa, ma, ca, _ = _run(rdm, g, H0, Ws, y, m, cfg, P=P, transport="nccl")
+    lb, dWb, mb, cb, _ = _run(rdm, g, H0, Ws, y, m, cfg, P=P, transport="p2p")
+    assert cb.transport == "p2p"
+    assert "[fused into producer]" in mb.describe()
+    assert "[fused into producer]" not in ma.describe()
+    assert la == lb
+    for a, b in zip(dWa, dWb):
+        assert np.array_equal(a, b)
+    L = len(Ws)
+    for which, layers in ((rdm.T_H, range(1, L)), (rdm.T_Z, [0]), (rdm.T_G, range(L + 1)),
+                          (rdm.T_MEMO, range(1, L + 1))):
+        for layer in layers:
+            ra, rb = _resident(ma, rdm, which, layer, P), _resident(mb, rdm, which, layer, P)
+            assert len(ra) == len(rb)
+            for a, b in zip(ra, rb):
+                assert np.array_equal(a, b), (which, layer)
+    x, yy = ca.counters(), cb.counters()
+    for k in ("a2a_calls", "a2a_elems_payload", "a2a_width_units", "spmm_width_units",
+              "gemm_flops"):
+        assert x[k] == yy[k], k
+
+
+def test_p2p_products_shaped_oracle(rdm):
+    """Fused redistribution on a 3-layer products-shaped model: oracle parity."""
+    f = (100, 256, 256, 47)
+    g, H0, Ws, y, m = _problem(n=6000, E=60000, f=f, seed=4)
+    for cfg in ocm.pareto_front(f)[:3] + [63]:
+        loss, dW, model, ctx, _ = _run(rdm, g, H0, Ws, y, m, cfg, P=4, transport="p2p")
+        _check((g, H0, Ws, y, m), loss, dW, model, rdm, P=4)
+
+
+def test_p2p_simt_fallback_scatter(rdm, cora):
+    """With the tensor-core GEMM disabled the fused GEMM falls back to SIMT +
+    the unfused scatter kernel: still bit-identical to the NCCL transport."""
+    g, H0, Ws, y, m, ref = cora
+    rdm.debug_disable_tc(True)
+    try:
+        la, dWa, *_ = _run(rdm, g, H0, Ws, y, m, 10, P=3, transport="nccl")
+        lb, dWb, *_ = _run(rdm, g, H0, Ws, y, m, 10, P=3, transport="p2p")
+    finally:
+        rdm.debug_disable_tc(False)
+    assert la == lb
+    for a, b in zip(dWa, dWb):
+        assert np.array_equal(a, b)
 
 
 def test_three_layer_products_shaped(rdm):
