@@ -130,7 +130,8 @@ enum {
   RDM_PH_ALLREDUCE = 5, /* Y^l / loss all-reduce                         */
   RDM_PH_ADAM = 6,
   RDM_PH_OTHER = 7,
-  RDM_PH_COUNT = 8
+  RDM_PH_SAMPLE = 8,    /* GraphSAINT sampler + induced-subgraph build    */
+  RDM_PH_COUNT = 9
 };
 
 typedef struct {
@@ -363,6 +364,55 @@ rdm_status rdm_plan_info(int L, const int64_t* f, const rdm_config* cfg, int P, 
  * `layout` (RDM_ERR_ARG if that layout is not resident). */
 rdm_status rdm_gcn_tensor(rdm_gcn* g, int which, int layer, int slot, rdm_layout layout,
                           const float** ptr, int64_t* rows, int64_t* cols, int64_t* ld);
+
+/* ------------------------------------------------------ GraphSAINT-RDM */
+
+/* Sampling-based training (§III-F, §V-C): "graph-sampling
+ * to create independently processed subgraphs" (GraphSAINT [17]); "each
+ * subgraph is parallelized using our RDM scheme" (L388) and the weights are
+ * updated after each subgraph (L390).  "A random generated seed can be
+ * passed to all processes and each process can generate its sparse mask
+ * individually" (L173): every rank samples the SAME subgraph from the shared
+ * seed — no communication.
+ *
+ * Sampler (readings R31-R34): GraphSAINT random-walk sampler on
+ * the installed graph (rdm_set_graph; walks follow its stored CSR entries,
+ * self loops included).  For subgraph `it`, with key = splitmix64(seed +
+ * it·0x9E3779B97F4A7C15) and u(i, j) = splitmix64(key ^ (i << 8 | j)):
+ * root i (0 ≤ i < roots) is u(i, 0) mod N; step j = 1..walk_len moves from v
+ * to col[rowptr[v] + u(i, j) mod deg(v)].  The node set is the sorted set of
+ * visited vertices (new id = rank in that order).  The subgraph is the
+ * induced one, Â_s[i][j] = 1/sqrt(d_i·d_j) for every stored entry (v_i, v_j)
+ * with both ends sampled, d_i = entries of row i kept (GCN normalisation of
+ * the induced graph, entries in the original row order), computed as
+ * (float)(1.0 / sqrt((double)d_i·d_j)).
+ * Requires a symmetric graph.  walk_len ≤ 255.  The sampler's GCN instances
+ * hold capacity for n_cap = min(N, roots·(walk_len + 1)) vertices. */
+typedef struct rdm_saint rdm_saint;
+rdm_status rdm_saint_create(rdm_ctx* ctx, int64_t roots, int walk_len, uint64_t seed,
+                            rdm_saint** out);
+rdm_status rdm_saint_destroy(rdm_saint* s);
+/* Sample subgraph number `iteration` and build its CSR on the device (GPU
+ * random walks, vertex compaction, induced-subgraph extraction, row bins).
+ * Returns its vertex and entry counts.  Synchronises the ctx stream (the
+ * host needs the sizes for the executor's launch shapes). */
+rdm_status rdm_saint_sample(rdm_saint* s, int64_t iteration, int64_t* n_sub, int64_t* nnz_sub);
+/* Device pointers to the current subgraph: nodes[n] (int32 original ids,
+ * ascending), rowptr[n+1] (int64), col[nnz] (int32 new ids), val[nnz]. */
+rdm_status rdm_saint_subgraph(const rdm_saint* s, const int32_t** nodes, const int64_t** rowptr,
+                              const int32_t** col, const float** val, int64_t* n, int64_t* nnz);
+/* A GCN instance (as rdm_gcn_create) whose graph is the sampler's current
+ * subgraph; forward/backward/adam as for any rdm_gcn.  Destroy the GCN
+ * before the sampler. */
+rdm_status rdm_saint_gcn_create(rdm_saint* s, int L, const int64_t* f, const rdm_config* cfg,
+                                int flags, rdm_gcn** out);
+/* Input of the current subgraph for every local slot, gathered on the device
+ * from the FULL-graph arrays every rank holds (H0_full N x f0 at leading
+ * dim ld_h, labels_full[N], mask_full[N] or NULL = all): H^0 row and column
+ * slices, labels, mask and the subgraph's training count.  No communication.
+ * Call after each rdm_saint_sample, before rdm_gcn_forward. */
+rdm_status rdm_saint_set_input(rdm_gcn* g, const float* H0_full, int64_t ld_h,
+                               const int32_t* labels_full, const uint8_t* mask_full);
 
 /* Adam (PyTorch semantics, no weight decay; L297 lr = 0.01) on `count`
  * replicated parameter arrays of sizes[i] floats; step ≥ 1. */

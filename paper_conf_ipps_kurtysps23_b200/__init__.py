@@ -31,7 +31,7 @@ MAX_LAYERS = 8
 UNIQUE_ID_BYTES = 128
 GCN_INPUT_GRAD, GCN_BIAS = 1, 2
 T_H, T_Z, T_G, T_MEMO, T_DWP = range(5)
-PHASES = ["spmm", "gemm", "pack", "a2a", "loss", "allreduce", "adam", "other"]
+PHASES = ["spmm", "gemm", "pack", "a2a", "loss", "allreduce", "adam", "other", "sample"]
 _STATUS = {0: "OK", 1: "ERR_ARG", 2: "ERR_CUDA", 3: "ERR_NCCL", 4: "ERR_OOM",
            5: "ERR_UNSUPPORTED", 6: "ERR_STATE"}
 
@@ -350,7 +350,7 @@ class Context:
 class GCN:
     """A GCN instance (L layers, widths f) running configuration `cfg` (ID or RdmConfig)."""
 
-    def __init__(self, ctx: Context, f, cfg, input_grad=True):
+    def __init__(self, ctx: Context, f, cfg, input_grad=True, saint=None):
         self.ctx = ctx
         self.f = list(f)
         self.L = len(f) - 1
@@ -358,8 +358,13 @@ class GCN:
         fa = (ctypes.c_int64 * len(f))(*f)
         h = ctypes.c_void_p()
         flags = GCN_INPUT_GRAD if input_grad else 0
-        ctx._c(_lib.rdm_gcn_create(ctx.h, self.L, fa, ctypes.byref(self.cfg), flags,
-                                   ctypes.byref(h)))
+        self.saint = saint   # keeps the sampler alive while this instance exists
+        if saint is None:
+            ctx._c(_lib.rdm_gcn_create(ctx.h, self.L, fa, ctypes.byref(self.cfg), flags,
+                                       ctypes.byref(h)))
+        else:
+            ctx._c(_lib.rdm_saint_gcn_create(saint.h, self.L, fa, ctypes.byref(self.cfg), flags,
+                                             ctypes.byref(h)))
         self.h = h
 
     def close(self):
@@ -385,6 +390,13 @@ class GCN:
         else:
             mp, _c2 = _parr(mask_rows)
         self.ctx._c(_lib.rdm_gcn_set_input(self.h, hp, lp, mp, int(on_host)))
+
+    def saint_input(self, H0_full, labels_full, mask_full=None):
+        """GraphSAINT: gather the current subgraph's input from full-graph device
+        tensors (rdm.h rdm_saint_set_input)."""
+        self.ctx._c(_lib.rdm_saint_set_input(self.h, _ptr(H0_full), H0_full.stride(0),
+                                             _ptr(labels_full),
+                                             None if mask_full is None else _ptr(mask_full)))
 
     def forward(self, Ws, loss_dev):
         wp, _a = _parr(Ws)
@@ -426,6 +438,77 @@ class GCN:
 
         view = torch.as_tensor(_View(), device=f"cuda:{self.ctx.device}")
         return view[:, :c].clone()
+
+
+def _dev_view(ptr, shape, typestr, device):
+    """Zero-copy torch view of library device memory (via __cuda_array_interface__)."""
+    import torch
+
+    class _View:
+        __cuda_array_interface__ = {"shape": tuple(shape), "typestr": typestr, "data": (ptr, False),
+                                    "version": 3, "strides": None}
+
+    return torch.as_tensor(_View(), device=device)
+
+
+class Saint:
+    """GraphSAINT-RDM random-walk sampler (rdm.h rdm_saint_*): `roots` walks of
+    `walk_len` steps from the shared `seed`; every rank samples the same subgraph."""
+
+    def __init__(self, ctx: Context, roots, walk_len=4, seed=1):
+        self.ctx = ctx
+        h = ctypes.c_void_p()
+        ctx._c(_lib.rdm_saint_create(ctx.h, int(roots), int(walk_len), ctypes.c_uint64(seed),
+                                     ctypes.byref(h)))
+        self.h = h
+
+    def sample(self, iteration):
+        n, nnz = _i64(), _i64()
+        self.ctx._c(_lib.rdm_saint_sample(self.h, int(iteration), ctypes.byref(n), ctypes.byref(nnz)))
+        return n.value, nnz.value
+
+    def subgraph(self):
+        """Copies of the current subgraph: nodes, rowptr, col, val (torch, on the device)."""
+        ps = [ctypes.c_void_p() for _ in range(4)]
+        n, nnz = _i64(), _i64()
+        self.ctx._c(_lib.rdm_saint_subgraph(self.h, *[ctypes.byref(p) for p in ps],
+                                            ctypes.byref(n), ctypes.byref(nnz)))
+        self.ctx.sync()
+        dev = f"cuda:{self.ctx.device}"
+        shapes = [(n.value,), (n.value + 1,), (nnz.value,), (nnz.value,)]
+        types = ["<i4", "<i8", "<i4", "<f4"]
+        import torch
+        tt = {"<i4": torch.int32, "<i8": torch.int64, "<f4": torch.float32}
+        return tuple(_dev_view(p.value, s, t, dev).clone() if s[0] else
+                     torch.zeros(s, dtype=tt[t], device=dev)
+                     for p, s, t in zip(ps, shapes, types))
+
+    def gcn(self, f, cfg, input_grad=True):
+        return GCN(self.ctx, f, cfg, input_grad=input_grad, saint=self)
+
+    def close(self):
+        if getattr(self, "h", None):
+            _lib.rdm_saint_destroy(self.h)
+            self.h = None
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+_lib.rdm_saint_create.argtypes = [_vp, _i64, _int, ctypes.c_uint64, ctypes.POINTER(_vp)]
+_lib.rdm_saint_destroy.argtypes = [_vp]
+_lib.rdm_saint_sample.argtypes = [_vp, _i64, _pi64, _pi64]
+_lib.rdm_saint_subgraph.argtypes = [_vp, _pp, _pp, _pp, _pp, _pi64, _pi64]
+_lib.rdm_saint_gcn_create.argtypes = [_vp, _int, _pi64, ctypes.POINTER(RdmConfig), _int,
+                                      ctypes.POINTER(_vp)]
+_lib.rdm_saint_set_input.argtypes = [_vp, _vp, _i64, _vp, _vp]
+for _n in ("rdm_saint_create", "rdm_saint_destroy", "rdm_saint_sample", "rdm_saint_subgraph",
+           "rdm_saint_gcn_create", "rdm_saint_set_input"):
+    getattr(_lib, _n).restype = _int
+    EXPORTS.append(_n)
 
 
 class RdmGraphInfo(ctypes.Structure):

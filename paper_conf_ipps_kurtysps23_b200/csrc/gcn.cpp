@@ -277,12 +277,43 @@ struct rdm_gcn {
   bool p2p = false;
   std::map<std::pair<int, int>, std::vector<float*>> peers;
   std::vector<void*> ipc_opened;
+  // the graph this instance runs on: the ctx's full graph, or a GraphSAINT
+  // sampler's current subgraph (buffers sized for n_cap vertices, row counts
+  // refreshed whenever the sampler's version changes)
+  const rdm::Graph* graph = nullptr;
+  rdm_saint* saint = nullptr;
+  int64_t n_cap = 0;
+  int64_t gver = -1;
 };
 
 namespace rdm {
 namespace {
 
 int norm_lay(const rdm_gcn* g, int l) { return g->ctx->world == 1 ? 0 : l; }
+
+int64_t gn(const rdm_gcn* g) { return g->graph->n; }
+
+// rows a row slice of rank p is allocated for: its share of n_cap, or, for a
+// sampler's instance (any n <= n_cap), the largest share ceil(n_cap / P)
+int64_t cap_rows(const rdm_gcn* g, int p) {
+  const int P = g->ctx->world;
+  if (g->saint) return ceil_div(g->n_cap, P);
+  return row_range(g->n_cap, P, p).size();
+}
+
+// A sampler's instance: after a new subgraph, every buffer's row count
+// follows the new vertex count (capacity and leading dims are unchanged).
+void sync_graph(rdm_gcn* g) {
+  if (!g->saint || g->gver == g->saint->version) return;
+  if (g->saint->iteration < 0) throw Error(RDM_ERR_STATE, "GraphSAINT: call rdm_saint_sample first");
+  rdm_ctx* ctx = g->ctx;
+  const int64_t n = gn(g);
+  for (int s = 0; s < ctx->nlocal(); ++s)
+    for (auto& kv : g->bufs[s])
+      kv.second.rows = kv.first.second == RDM_ROW ? row_range(n, ctx->world, ctx->local[s]).size() : n;
+  g->gver = g->saint->version;
+  g->input_set = false;
+}
 
 Buf& buf(rdm_gcn* g, int slot, Key k, int l) {
   auto it = g->bufs[slot].find({k.id(), norm_lay(g, l)});
@@ -295,14 +326,14 @@ Buf& buf(rdm_gcn* g, int slot, Key k, int l) {
 void alloc_buf(rdm_gcn* g, Key k, int l, int64_t width) {
   rdm_ctx* ctx = g->ctx;
   const int P = ctx->world;
-  const int64_t n = ctx->graph.n;
+  const int64_t n = g->n_cap;
   for (int s = 0; s < ctx->nlocal(); ++s) {
     auto key = std::make_pair(k.id(), norm_lay(g, l));
     if (g->bufs[s].count(key)) continue;
     const int p = ctx->local[s];
     Buf b;
     if (norm_lay(g, l) == RDM_ROW) {
-      b.rows = row_range(n, P, p).size();
+      b.rows = cap_rows(g, p);
       b.cols = width;
       b.ld = roundup4(width);
     } else {
@@ -384,7 +415,7 @@ Scatter make_scatter(rdm_gcn* g, const Step& s, int i) {
   rdm_ctx* ctx = g->ctx;
   const int P = ctx->world;
   const int p = ctx->local[i];
-  const int64_t n = ctx->graph.n, w = s.width;
+  const int64_t n = gn(g), w = s.width;
   const int dl = s.lout == RDM_ROW ? RDM_COL : RDM_ROW;
   const std::vector<float*>& ptr = g->peers.at({s.out.id(), norm_lay(g, dl)});
   Scatter sc;
@@ -457,13 +488,13 @@ void create(rdm_gcn* g) {
   for (auto& s : g->fwd) touch(s);
   for (auto& s : g->bwd) touch(s);
   const int P = ctx->world;
-  const int64_t n = ctx->graph.n;
+  const int64_t n = g->n_cap;
   g->dwp.assign(ctx->nlocal(), std::vector<float*>(g->L + 1, nullptr));
   g->labels.assign(ctx->nlocal(), nullptr);
   g->mask.assign(ctx->nlocal(), nullptr);
   g->scal.assign(ctx->nlocal(), nullptr);
   for (int s = 0; s < ctx->nlocal(); ++s) {
-    const int64_t r = row_range(n, P, ctx->local[s]).size();
+    const int64_t r = cap_rows(g, ctx->local[s]);
     if (ctx->virtual_group()) {
       for (int l = 1; l <= g->L; ++l) {
         g->mem.emplace_back(new DevBuf((size_t)g->f[l - 1] * g->f[l] * sizeof(float)));
@@ -493,7 +524,7 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
   switch (s.op) {
     case S_SPMM: {
       Phase ph(ctx, RDM_PH_SPMM);
-      const Csr& A = s.trans ? ctx->graph.fwd() : ctx->graph.bwd();
+      const Csr& A = s.trans ? g->graph->fwd() : g->graph->bwd();
       for (int i = 0; i < nl; ++i) {
         Buf& in = buf(g, i, s.in, s.lin);
         Buf& out = buf(g, i, s.out, s.lout);
@@ -544,7 +575,7 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
     case S_REDIST: {
       if (s.fuse == 2) {   // the producer already stored it; fence peers before the consumer
         p2p_barrier(ctx);
-        count_fused_redist(ctx, (rdm_layout)s.lin, ctx->graph.n, s.width);
+        count_fused_redist(ctx, (rdm_layout)s.lin, gn(g), s.width);
         break;
       }
       std::vector<const float*> src(nl);
@@ -553,7 +584,7 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
         src[i] = buf(g, i, s.in, s.lin).p;
         dst[i] = buf(g, i, s.out, s.lout).p;
       }
-      redistribute(ctx, (rdm_layout)s.lin, src.data(), dst.data(), ctx->graph.n, s.width);
+      redistribute(ctx, (rdm_layout)s.lin, src.data(), dst.data(), gn(g), s.width);
       break;
     }
     case S_MASK: {
@@ -636,6 +667,7 @@ void do_forward(void* a_) {
   auto* a = static_cast<FwdArgs*>(a_);
   rdm_gcn* g = a->g;
   rdm_ctx* ctx = g->ctx;
+  sync_graph(g);
   if (!g->input_set) throw Error(RDM_ERR_STATE, "rdm_gcn_forward: call rdm_gcn_set_input first");
   RDM_CHECK_ARG(a->W && a->loss, "rdm_gcn_forward: W and loss_dev required");
   for (int l = 0; l < g->L; ++l) RDM_CHECK_ARG(a->W[l], "rdm_gcn_forward: null W");
@@ -657,6 +689,8 @@ void do_backward(void* a_) {
   rdm_gcn* g = a->g;
   rdm_ctx* ctx = g->ctx;
   RDM_CHECK_ARG(a->W && a->dW, "rdm_gcn_backward: W and dW required");
+  if (g->saint && g->gver != g->saint->version)
+    throw Error(RDM_ERR_STATE, "rdm_gcn_backward: the subgraph changed since the forward pass");
   for (int l = 0; l < g->L; ++l) RDM_CHECK_ARG(a->W[l] && a->dW[l], "rdm_gcn_backward: null W/dW");
   if (!ctx->virtual_group())
     for (int l = 1; l <= g->L; ++l) g->dwp[0][l] = a->dW[l - 1];
@@ -694,7 +728,8 @@ struct InputArgs {
 void stage_host_input(rdm_gcn* g, const InputArgs* a) {
   rdm_ctx* ctx = g->ctx;
   const int nl = ctx->nlocal(), P = ctx->world;
-  const int64_t n = ctx->graph.n, f0 = g->f[0];
+  const int64_t n = gn(g), f0 = g->f[0];
+  RDM_CHECK_ARG(!g->saint, "set_input: a sampler's GCN takes rdm_saint_set_input");
   if (!g->cs) {
     RDM_CUDA(cudaStreamCreateWithFlags(&g->cs, cudaStreamNonBlocking));
     RDM_CUDA(cudaEventCreateWithFlags(&g->ev_ready, cudaEventDisableTiming));
@@ -762,7 +797,8 @@ void do_set_input(void* a_) {
 void apply_input(rdm_gcn* g, const InputArgs* a) {
   rdm_ctx* ctx = g->ctx;
   const int nl = ctx->nlocal(), P = ctx->world;
-  const int64_t n = ctx->graph.n, f0 = g->f[0];
+  const int64_t n = gn(g), f0 = g->f[0];
+  RDM_CHECK_ARG(!g->saint, "set_input: a sampler's GCN takes rdm_saint_set_input");
   const cudaMemcpyKind kind = a->on_host ? cudaMemcpyHostToDevice : cudaMemcpyDeviceToDevice;
   const rdm_counters saved = ctx->counters;
   std::vector<const float*> src(nl);
@@ -805,6 +841,47 @@ void apply_input(rdm_gcn* g, const InputArgs* a) {
 }
 
 
+struct SaintInputArgs {
+  rdm_gcn* g;
+  const float* H;
+  int64_t ldh;
+  const int32_t* labels;
+  const uint8_t* mask;
+};
+
+// GraphSAINT input: gathered on the device from the full-graph arrays every
+// rank holds — H^0 straight into both layouts, so no redistribution.
+void do_saint_input(void* a_) {
+  auto* a = static_cast<SaintInputArgs*>(a_);
+  rdm_gcn* g = a->g;
+  rdm_ctx* ctx = g->ctx;
+  RDM_CHECK_ARG(g->saint, "rdm_saint_set_input: not a sampler's GCN (rdm_saint_gcn_create)");
+  RDM_CHECK_ARG(a->H && a->labels && a->ldh >= g->f[0], "rdm_saint_set_input: bad arguments");
+  sync_graph(g);
+  Phase ph(ctx, RDM_PH_SAMPLE);
+  const int P = ctx->world;
+  const int64_t n = gn(g), f0 = g->f[0];
+  const int32_t* nodes = g->saint->nodes->as<int32_t>();
+  for (int i = 0; i < ctx->nlocal(); ++i) {
+    const int p = ctx->local[i];
+    const Range r = row_range(n, P, p);
+    Buf& hr = buf(g, i, {K_H, 0}, RDM_ROW);
+    saint_gather(ctx, a->H, a->ldh, nodes, r.lo, r.size(), 0, f0, hr.p, hr.ld);
+    if (P > 1) {
+      Buf& hc = buf(g, i, {K_H, 0}, RDM_COL);
+      const Range c = col_range(f0, P, p);
+      saint_gather(ctx, a->H, a->ldh, nodes, 0, n, c.lo, c.size(), hc.p, hc.ld);
+    }
+    saint_gather_labels(ctx, a->labels, a->mask, nodes, r.lo, r.size(), g->labels[i], g->mask[i]);
+  }
+  // the subgraph's training count from the whole node list (no communication)
+  uint8_t* ms = reinterpret_cast<uint8_t*>(ensure_ws(g->saint->mask_s, std::max<int64_t>(n, 1)));
+  saint_gather_labels(ctx, a->labels, a->mask, nodes, 0, n, nullptr, ms);
+  for (int i = 0; i < ctx->nlocal(); ++i) count_mask(ctx, ms, n, g->scal[i] + 0);
+  g->staged = false;
+  g->input_set = true;
+}
+
 void do_create(void* a_) { create(static_cast<rdm_gcn*>(a_)); }
 
 }  // namespace
@@ -827,6 +904,8 @@ rdm_status rdm_gcn_create(rdm_ctx* ctx, int L, const int64_t* f, const rdm_confi
   }
   auto* g = new rdm_gcn();
   g->ctx = ctx;
+  g->graph = &ctx->graph;
+  g->n_cap = ctx->graph.n;
   g->L = L;
   g->flags = flags;
   g->f.assign(f, f + L + 1);
@@ -838,6 +917,41 @@ rdm_status rdm_gcn_create(rdm_ctx* ctx, int L, const int64_t* f, const rdm_confi
   }
   *out = g;
   return RDM_OK;
+}
+
+rdm_status rdm_saint_gcn_create(rdm_saint* s, int L, const int64_t* f, const rdm_config* cfg,
+                                int flags, rdm_gcn** out) {
+  if (!s || !out || !f || !cfg || L < 1 || L > RDM_MAX_LAYERS || cfg->L != L) return RDM_ERR_ARG;
+  rdm_ctx* ctx = s->ctx;
+  for (int l = 0; l <= L; ++l)
+    if (f[l] < 1) return RDM_ERR_ARG;
+  if (flags & RDM_GCN_BIAS) {
+    ctx->err = "rdm_saint_gcn_create: RDM_GCN_BIAS is not implemented";
+    return RDM_ERR_UNSUPPORTED;
+  }
+  auto* g = new rdm_gcn();
+  g->ctx = ctx;
+  g->graph = &s->graph;
+  g->saint = s;
+  g->n_cap = s->n_cap;
+  g->L = L;
+  g->flags = flags;
+  g->f.assign(f, f + L + 1);
+  g->cfg = *cfg;
+  rdm_status st = rdm_guarded_call(ctx, do_create, g);
+  if (st != RDM_OK) {
+    delete g;
+    return st;
+  }
+  *out = g;
+  return RDM_OK;
+}
+
+rdm_status rdm_saint_set_input(rdm_gcn* g, const float* H0_full, int64_t ld_h,
+                               const int32_t* labels_full, const uint8_t* mask_full) {
+  if (!g) return RDM_ERR_ARG;
+  SaintInputArgs a{g, H0_full, ld_h, labels_full, mask_full};
+  return rdm_guarded_call(g->ctx, do_saint_input, &a);
 }
 
 rdm_status rdm_gcn_destroy(rdm_gcn* g) {

@@ -150,6 +150,20 @@ struct rdm_ctx {
   int nlocal() const { return (int)local.size(); }
 };
 
+// GraphSAINT-RDM sampler (saint.cu): the current subgraph and the device
+// workspace that builds it.
+struct rdm_saint {
+  rdm_ctx* ctx = nullptr;
+  int64_t roots = 0;
+  int walk_len = 0;
+  uint64_t seed = 0;
+  int64_t n_cap = 0;
+  rdm::Graph graph;       // current subgraph (symmetric: A only)
+  int64_t version = 0;    // bumped by every rdm_saint_sample
+  int64_t iteration = -1;
+  std::unique_ptr<rdm::DevBuf> visits, flag, map, nodes, deg, seg, rps, scal, tmp, mask_s;
+};
+
 namespace rdm {
 
 float* ensure_ws(std::unique_ptr<DevBuf>& b, size_t bytes);
@@ -196,6 +210,13 @@ void gemm_tc_panels(rdm_ctx* ctx, const float* A, int64_t lda, const float* bhi,
 // dense hub core (spmm.cu)
 void build_core(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, const int32_t* col_host,
                 const float* val_host);
+
+// saint.cu — gathers of the full-graph input into a subgraph's slices
+void saint_gather(rdm_ctx* ctx, const float* H, int64_t ldh, const int32_t* nodes, int64_t row_lo,
+                  int64_t rows, int64_t col_lo, int64_t cols, float* out, int64_t ldo);
+void saint_gather_labels(rdm_ctx* ctx, const int32_t* labels, const uint8_t* mask,
+                         const int32_t* nodes, int64_t row_lo, int64_t rows, int32_t* lab_out,
+                         uint8_t* mask_out);
 
 // runtime.cpp — fused ("p2p") redistribution support
 void count_fused_redist(rdm_ctx* ctx, rdm_layout from, int64_t n, int64_t f);

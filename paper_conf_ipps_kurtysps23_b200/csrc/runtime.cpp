@@ -52,8 +52,11 @@ DevBuf::~DevBuf() {
 
 float* ensure_ws(std::unique_ptr<DevBuf>& b, size_t bytes) {
   if (!b || b->bytes < bytes) {
+    // regrowth (sizes that vary per call, e.g. GraphSAINT subgraphs) gets 25 %
+    // headroom so that cudaFree / cudaMalloc — both synchronising — stay rare
+    const size_t want = b ? bytes + bytes / 4 : bytes;
     b.reset();
-    b.reset(new DevBuf(std::max<size_t>(bytes, 256)));
+    b.reset(new DevBuf(std::max<size_t>(want, 256)));
   }
   return b->as<float>();
 }

@@ -412,11 +412,12 @@ void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rp) {
   A.n_seg = n_seg;
   A.n_heavy = n_heavy;
   A.max_deg = max_deg;
-  A.light_rows.reset(new DevBuf(std::max<int64_t>(1, n_light) * sizeof(int32_t)));
+  // capacity is reused across calls (a GraphSAINT sampler rebuilds bins per subgraph)
+  ensure_ws(A.light_rows, std::max<int64_t>(1, n_light) * sizeof(int32_t));
   // seg_start (int64) followed by seg_row (int32) in one allocation
-  A.seg_start.reset(new DevBuf(std::max<int64_t>(1, n_seg) * (sizeof(int64_t) + sizeof(int32_t))));
-  A.heavy_rows.reset(new DevBuf(std::max<int64_t>(1, n_heavy) * sizeof(int32_t)));
-  A.heavy_seg.reset(new DevBuf((n_heavy + 1) * sizeof(int32_t)));
+  ensure_ws(A.seg_start, std::max<int64_t>(1, n_seg) * (sizeof(int64_t) + sizeof(int32_t)));
+  ensure_ws(A.heavy_rows, std::max<int64_t>(1, n_heavy) * sizeof(int32_t));
+  ensure_ws(A.heavy_seg, (n_heavy + 1) * sizeof(int32_t));
   if (n_light)
     RDM_CUDA(cudaMemcpy(A.light_rows->ptr, light.data(), n_light * sizeof(int32_t),
                         cudaMemcpyHostToDevice));

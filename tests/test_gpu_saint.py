@@ -1,0 +1,146 @@
+"""GraphSAINT-RDM on the GPU (rdm.h rdm_saint_*) against the oracle.
+
+Sampler + induced-subgraph build: bit-exact (indices, counts and the fp32
+values, which both sides compute as (float)(1/sqrt((double) d_i d_j))).
+Training on the subgraph: the GCN epoch gates of tests/test_gpu_gcn.py
+against oracle.gcn.epoch on the oracle's own subgraph, one Adam step per
+subgraph (L390), P = 1 and virtual P = 2, 4."""
+import numpy as np
+import pytest
+
+import synth
+from oracle import gcn as og
+from oracle import saint as osaint
+
+pytestmark = pytest.mark.gpu
+
+
+@pytest.fixture(scope="module")
+def rdm():
+    import paper_conf_ipps_kurtysps23_b200 as r
+    return r
+
+
+def _sub_np(s):
+    return [t.cpu().numpy() for t in s.subgraph()]
+
+
+@pytest.mark.parametrize("n,E,roots,h", [(2708, 5278, 300, 4), (20000, 200000, 1500, 4),
+                                         (500, 4000, 40, 0), (300, 3000, 400, 7)])
+def test_sampler_bit_exact(rdm, n, E, roots, h):
+    g = synth.rmat(n, E, seed=2)
+    ctx = rdm.Context(device=0)
+    ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
+    s = rdm.Saint(ctx, roots, walk_len=h, seed=17)
+    for it in (0, 1, 5):
+        n_s, nnz_s = s.sample(it)
+        nodes, rp, cs, vs = osaint.sample(g, roots, h, 17, it)
+        assert (n_s, nnz_s) == (len(nodes), len(cs))
+        gn, grp, gcs, gvs = _sub_np(s)
+        assert np.array_equal(gn, nodes)
+        assert np.array_equal(grp, rp)
+        assert np.array_equal(gcs, cs)
+        assert np.array_equal(gvs.view(np.uint32), vs.view(np.uint32))
+
+
+def test_sampler_whole_graph_capacity(rdm):
+    """roots·(h+1) ≥ N: capacity = N; a subgraph may contain every vertex."""
+    g = synth.complete_graph(12)
+    ctx = rdm.Context(device=0)
+    ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
+    s = rdm.Saint(ctx, 200, walk_len=2, seed=3)
+    n_s, nnz_s = s.sample(0)
+    nodes, rp, cs, vs = osaint.sample(g, 200, 2, 3, 0)
+    assert n_s == len(nodes) == 12 and nnz_s == 144
+    gn, grp, gcs, gvs = _sub_np(s)
+    assert np.array_equal(gvs.view(np.uint32), vs.view(np.uint32))
+
+
+def _saint_run(rdm, g, H0, Ws, y, m, cfg, P, roots, h, seed, iters):
+    import torch
+    dev = torch.device("cuda:0")
+    f = [Ws[0].shape[0]] + [w.shape[1] for w in Ws]
+    ctx = rdm.Context(device=0) if P == 1 else rdm.Context(rank=rdm.ALL_RANKS, world=P, device=0)
+    ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
+    s = rdm.Saint(ctx, roots, walk_len=h, seed=seed)
+    model = s.gcn(f, cfg)
+    Hd = torch.from_numpy(H0).to(dev)
+    yd = torch.from_numpy(y).to(dev)
+    md = torch.from_numpy(m.astype(np.uint8)).to(dev)
+    Wd = [torch.from_numpy(w.copy()).to(dev) for w in Ws]
+    dW = [torch.zeros_like(w) for w in Wd]
+    mo = [torch.zeros_like(w) for w in Wd]
+    ve = [torch.zeros_like(w) for w in Wd]
+    loss = torch.zeros(1, dtype=torch.float64, device=dev)
+    out = []
+    for it in range(iters):
+        s.sample(it)
+        model.saint_input(Hd, yd, md)
+        W_now = [w.cpu().numpy().copy() for w in Wd]
+        model.forward(Wd, loss)
+        model.backward(Wd, dW)
+        ctx.sync()
+        out.append((it, float(loss.item()), [d.cpu().numpy() for d in dW], W_now, model))
+        # per-subgraph parity is checked by the caller before the update
+        yield out[-1]
+        ctx.adam_step(Wd, dW, mo, ve, it + 1)
+    model.close()
+    s.close()
+
+
+@pytest.mark.parametrize("P,cfg", [(1, 3), (1, 10), (2, 3), (4, 10), (4, 2)])
+def test_saint_gcn_matches_oracle(rdm, P, cfg):
+    n, f = 4000, (300, 64, 11)
+    g = synth.rmat(n, 40000, seed=6)
+    H0 = synth.features(n, f[0])
+    Ws = synth.weights(f)
+    y = synth.labels(n, f[-1])
+    m = synth.train_mask(n, 0.7, seed=2)
+    roots, h, seed = 250, 4, 99
+    for it, loss, dW, W_now, model in _saint_run(rdm, g, H0, Ws, y, m, cfg, P, roots, h, seed, 3):
+        nodes, rp, cs, vs = osaint.sample(g, roots, h, seed, it)
+        sub = synth.CSR(len(nodes), rp, cs, vs)
+        # ReLU decisions from the kernel's own forward (reading R30)
+        Hs = []
+        for l in range(1, len(Ws)):
+            full = np.zeros((len(nodes), f[l]))
+            for layout in (rdm.ROW, rdm.COL):
+                try:
+                    parts = [model.tensor_torch(rdm.T_H, l, p, layout).cpu().numpy() for p in range(P)]
+                except rdm.RdmError:
+                    continue
+                for p, t in enumerate(parts):
+                    lo, hi, _ = rdm.partition(P, layout, len(nodes), f[l], p)
+                    if P == 1:
+                        full[:] = t
+                    elif layout == rdm.ROW:
+                        full[lo:hi] = t
+                    else:
+                        full[:, lo:hi] = t
+                break
+            Hs.append(full)
+        ref = og.epoch(sub, H0[nodes], W_now, y[nodes], m[nodes], relu_masks=[x > 0 for x in Hs])
+        assert abs(loss - ref.loss) <= 1e-5 * abs(ref.loss), (it, loss, ref.loss)
+        for l in range(len(Ws)):
+            assert og.max_rel_err(dW[l], ref.Y[l + 1]) < 1e-4, (it, l)
+
+
+def test_saint_requires_sample_and_input(rdm):
+    import torch
+    g = synth.rmat(500, 3000, seed=1)
+    ctx = rdm.Context(device=0)
+    ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
+    s = rdm.Saint(ctx, 50, walk_len=2, seed=1)
+    model = s.gcn([16, 8, 3], 3)
+    W = [torch.zeros(16, 8, device="cuda:0"), torch.zeros(8, 3, device="cuda:0")]
+    loss = torch.zeros(1, dtype=torch.float64, device="cuda:0")
+    with pytest.raises(rdm.RdmError):
+        model.forward(W, loss)           # no subgraph yet
+    s.sample(0)
+    with pytest.raises(rdm.RdmError):
+        model.forward(W, loss)           # subgraph without its input
+    with pytest.raises(rdm.RdmError):
+        model.set_input([torch.zeros(1, 16, device="cuda:0")], [torch.zeros(1, dtype=torch.int32,
+                                                                             device="cuda:0")])
+    model.close()
+    s.close()
