@@ -65,18 +65,21 @@ def induced(rowptr, col, nodes: np.ndarray):
     """Induced, re-normalised subgraph (R32): returns rowptr_s (int64),
     col_s (int32, new ids, original row order), val_s (float32)."""
     n = len(nodes)
-    new_id = {int(v): i for i, v in enumerate(nodes)}
-    rows = []
-    for v in nodes:
-        b, e = int(rowptr[v]), int(rowptr[v + 1])
-        rows.append([new_id[int(u)] for u in col[b:e] if int(u) in new_id])
-    deg = np.array([len(r) for r in rows], dtype=np.int64)
+    nodes = np.asarray(nodes, dtype=np.int64)
+    new_id = np.full(len(rowptr) - 1, -1, dtype=np.int64)   # new id of every vertex, -1 = not sampled
+    new_id[nodes] = np.arange(n)
+    # every stored entry of every sampled row, in row order then original entry order
+    starts, ends = rowptr[nodes], rowptr[nodes + 1]
+    row_of = np.repeat(np.arange(n), ends - starts)
+    entry = np.concatenate([np.arange(b, e) for b, e in zip(starts, ends)]) if n else np.zeros(0, np.int64)
+    j = new_id[col[entry]]
+    keep = j >= 0                                            # both ends sampled
+    row_of, j = row_of[keep], j[keep]
+    deg = np.bincount(row_of, minlength=n).astype(np.int64)  # d_i = kept entries of row i
     rp = np.zeros(n + 1, dtype=np.int64)
     rp[1:] = np.cumsum(deg)
-    cs = np.array([j for r in rows for j in r], dtype=np.int32)
-    vals = np.array([1.0 / np.sqrt(float(deg[i]) * float(deg[j])) for i, r in enumerate(rows) for j in r],
-                    dtype=np.float64).astype(np.float32)
-    return rp, cs, vals
+    vals = (1.0 / np.sqrt(deg[row_of].astype(np.float64) * deg[j].astype(np.float64))).astype(np.float32)
+    return rp, j.astype(np.int32), vals
 
 
 def sample(g, roots: int, walk_len: int, seed: int, it: int):
