@@ -162,6 +162,7 @@ struct rdm_saint {
   int64_t version = 0;    // bumped by every rdm_saint_sample
   int64_t iteration = -1;
   std::unique_ptr<rdm::DevBuf> visits, flag, map, nodes, deg, seg, rps, scal, tmp, mask_s;
+  std::unique_ptr<rdm::DevBuf> core_tmp, core_rank, core_seg, core_cnt, core_bucket, tmp2;
 };
 
 namespace rdm {
@@ -210,6 +211,9 @@ void gemm_tc_panels(rdm_ctx* ctx, const float* A, int64_t lda, const float* bhi,
 // dense hub core (spmm.cu)
 void build_core(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, const int32_t* col_host,
                 const float* val_host);
+
+// hub-core size rule shared by the host (full graph) and device (subgraph) builders
+int64_t choose_core_K(const int64_t* bucket, int64_t kmax, const char* force, bool* forced);
 
 // saint.cu — gathers of the full-graph input into a subgraph's slices
 void saint_gather(rdm_ctx* ctx, const float* H, int64_t ldh, const int32_t* nodes, int64_t row_lo,

@@ -73,21 +73,30 @@ __global__ void compact_kernel(const int32_t* __restrict__ flag, const int32_t* 
   }
 }
 
-// Induced-subgraph extraction is entry-parallel: each sampled row's ORIGINAL
-// adjacency list (random walks favour hubs: rows of 10^4-10^5 entries) is cut
-// into kSeg-entry segments, one warp per segment, so a hub row does not
-// serialise on one warp.
+// Every pass over adjacency entries is entry-parallel: each row's list (of
+// the full graph for the sampled rows — random walks favour hubs, rows of
+// 10^4-10^5 entries — or of the subgraph) is cut into kSeg-entry segments,
+// one warp per segment, so a hub row does not serialise on one warp.
 constexpr int kSeg = 1024;
+constexpr int kMaxBuckets = 160;   // hub-core histogram: kmax <= 20480 in 128-buckets
 
-// nseg[i] = segments of sampled row i (0 for i >= n_sub)
+// Row lengths for the segment tables: rows i < n of `rowptr`, through
+// `nodes` (rows of the full graph) when given.  n from the device (scal[0])
+// when `scal` is given, else n_host.
+__device__ __forceinline__ int64_t seg_n(const unsigned long long* scal, int64_t n_host) {
+  return scal ? (int64_t)scal[0] : n_host;
+}
+
+// nseg[i] = segments of row i, for i <= n_cap (0 beyond n)
 __global__ void rowseg_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ nodes,
-                              int64_t n_cap, const unsigned long long* scal, int32_t* __restrict__ nseg) {
-  const int64_t n = (int64_t)scal[0];
+                              int64_t n_cap, const unsigned long long* scal, int64_t n_host,
+                              int32_t* __restrict__ nseg) {
+  const int64_t n = seg_n(scal, n_host);
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i <= n_cap;
        i += (int64_t)gridDim.x * blockDim.x) {
     int32_t c = 0;
     if (i < n) {
-      const int32_t v = nodes[i];
+      const int64_t v = nodes ? nodes[i] : i;
       c = (int32_t)((rowptr[v + 1] - rowptr[v] + kSeg - 1) / kSeg);
     }
     nseg[i] = c;
@@ -95,11 +104,27 @@ __global__ void rowseg_kernel(const int64_t* __restrict__ rowptr, const int32_t*
 }
 
 __global__ void segrow_kernel(const int32_t* __restrict__ nseg, const int32_t* __restrict__ segoff,
-                              const unsigned long long* scal, int32_t* __restrict__ seg_row) {
-  const int64_t n = (int64_t)scal[0];
+                              const unsigned long long* scal, int64_t n_host,
+                              int32_t* __restrict__ seg_row) {
+  const int64_t n = seg_n(scal, n_host);
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
        i += (int64_t)gridDim.x * blockDim.x)
     for (int32_t k = 0; k < nseg[i]; ++k) seg_row[segoff[i] + k] = (int32_t)i;
+}
+
+struct Seg {     // segment sg of row i covers entries [b, end) of the row list
+  int32_t i;
+  int64_t b, end;
+};
+__device__ __forceinline__ Seg seg_of(int64_t sg, const int32_t* seg_row, const int32_t* segoff,
+                                      const int64_t* rowptr, const int32_t* nodes) {
+  Seg s;
+  s.i = seg_row[sg];
+  const int64_t v = nodes ? nodes[s.i] : s.i;
+  const int64_t e = rowptr[v + 1];
+  s.b = rowptr[v] + (sg - segoff[s.i]) * kSeg;
+  s.end = s.b + kSeg < e ? s.b + kSeg : e;
+  return s;
 }
 
 // warp per segment: kept entries c_s; d_i += c_s; scal[1] += c_s
@@ -112,23 +137,30 @@ __global__ void count_kernel(const int64_t* __restrict__ rowptr, const int32_t* 
   const int64_t nsegs = segoff[n_cap];
   for (int64_t sg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; sg < nsegs;
        sg += ((int64_t)gridDim.x * blockDim.x) >> 5) {
-    const int32_t i = seg_row[sg];
-    const int32_t v = nodes[i];
-    const int64_t e = rowptr[v + 1];
-    const int64_t b = rowptr[v] + (sg - segoff[i]) * kSeg;
-    const int64_t end = b + kSeg < e ? b + kSeg : e;
+    const Seg q = seg_of(sg, seg_row, segoff, rowptr, nodes);
     int c = 0;
-    for (int64_t k = b + lane; k < end; k += 32) c += flag[__ldg(col + k)] ? 1 : 0;
+    for (int64_t k = q.b + lane; k < q.end; k += 32) c += flag[__ldg(col + k)] ? 1 : 0;
 #pragma unroll
     for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
     if (lane == 0) {
       cnt[sg] = c;
       if (c) {
-        atomicAdd(deg + i, (unsigned long long)c);
+        atomicAdd(deg + q.i, (unsigned long long)c);
         atomicAdd(scal + 1, (unsigned long long)c);
       }
     }
   }
+}
+
+// Per-warp-step histogram update: one shared atomic per distinct bucket.
+__device__ __forceinline__ void bucket_add(unsigned* sb, int b, int lane) {
+  const unsigned same = __match_any_sync(0xffffffffu, b);
+  if (b >= 0 && lane == __ffs(same) - 1) atomicAdd(&sb[b], (unsigned)__popc(same));
+}
+__device__ __forceinline__ void bucket_flush(unsigned* sb, unsigned long long* bucket) {
+  __syncthreads();
+  for (int b = threadIdx.x; b < kMaxBuckets; b += blockDim.x)
+    if (sb[b]) atomicAdd(bucket + b, (unsigned long long)sb[b]);
 }
 
 // warp per segment: kept entries in the original order at pos[s] onwards
@@ -142,17 +174,13 @@ __global__ void fill_kernel(const int64_t* __restrict__ rowptr, const int32_t* _
   const int64_t nsegs = segoff[n_cap];
   for (int64_t sg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; sg < nsegs;
        sg += ((int64_t)gridDim.x * blockDim.x) >> 5) {
-    const int32_t i = seg_row[sg];
-    const int32_t v = nodes[i];
-    const int64_t e = rowptr[v + 1];
-    const int64_t b = rowptr[v] + (sg - segoff[i]) * kSeg;
-    const int64_t end = b + kSeg < e ? b + kSeg : e;
+    const Seg q = seg_of(sg, seg_row, segoff, rowptr, nodes);
     int64_t at0 = pos[sg];
-    const double di = (double)deg[i];
-    for (int64_t k0 = b; k0 < end; k0 += 32) {
+    const double di = (double)deg[q.i];
+    for (int64_t k0 = q.b; k0 < q.end; k0 += 32) {
       const int64_t k = k0 + lane;
-      const int32_t u = k < end ? __ldg(col + k) : 0;
-      const bool keep = k < end && flag[u];
+      const int32_t u = k < q.end ? __ldg(col + k) : 0;
+      const bool keep = k < q.end && flag[u];
       const unsigned m = __ballot_sync(0xffffffffu, keep);
       if (keep) {
         const int64_t at = at0 + __popc(m & ((1u << lane) - 1u));
@@ -161,6 +189,147 @@ __global__ void fill_kernel(const int64_t* __restrict__ rowptr, const int32_t* _
         val_s[at] = (float)(1.0 / sqrt(di * (double)deg[j]));
       }
       at0 += __popc(m);
+    }
+  }
+}
+
+// ---- dense hub core of a subgraph (device-side twin of spmm.cu build_core):
+// degree-rank the vertices (stable, descending), histogram the entries by
+// max(rank_i, rank_j) (fused into fill_kernel), pick K with the shared rule
+// (choose_core_K), move the K x K block of the top-K vertices into a dense
+// matrix and keep the rest as a residual CSR in the original order.
+// Random-walk subgraphs are hub-heavy: for the Reddit-shaped config the top
+// 12k of ~25k vertices hold ~88 % of the entries at ~20 % density.
+__global__ void deg_key_kernel(const unsigned long long* __restrict__ deg, int64_t n,
+                               int32_t* __restrict__ key, int32_t* __restrict__ iota) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    key[i] = (int32_t)deg[i];
+    iota[i] = (int32_t)i;
+  }
+}
+
+__global__ void rank_kernel(const int32_t* __restrict__ order, int64_t n, int32_t* __restrict__ rank) {
+  for (int64_t k = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; k < n;
+       k += (int64_t)gridDim.x * blockDim.x)
+    rank[order[k]] = (int32_t)k;
+}
+
+// Histogram for the core size: entries by max(rank_i, rank_j) in 128-buckets
+// below kmax, over the rows i ≡ 0 (mod 8) (a deterministic 1/8 sample; the
+// size is a cost heuristic, the product is exact for any K).
+__global__ void hist_kernel(const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
+                            const int32_t* __restrict__ rank, const int32_t* __restrict__ seg_row,
+                            const int32_t* __restrict__ segoff, int64_t n, int64_t kmax,
+                            unsigned long long* __restrict__ bucket) {
+  __shared__ unsigned sb[kMaxBuckets];
+  for (int b = threadIdx.x; b < kMaxBuckets; b += blockDim.x) sb[b] = 0;
+  __syncthreads();
+  const int lane = threadIdx.x & 31;
+  const int64_t nsegs = segoff[n];
+  for (int64_t sg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; sg < nsegs;
+       sg += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+    const int32_t i = seg_row[sg];
+    if (i & 7) continue;                       // warp-uniform
+    const Seg q = seg_of(sg, seg_row, segoff, rp, nullptr);
+    const int32_t ri = rank[i];
+    for (int64_t k0 = q.b; k0 < q.end; k0 += 32) {
+      const int64_t k = k0 + lane;
+      int bk = -1;
+      if (k < q.end) {
+        const int32_t mx = max(ri, rank[__ldg(col + k)]);
+        if (mx < kmax) bk = mx >> 7;
+      }
+      bucket_add(sb, bk, lane);
+    }
+  }
+  bucket_flush(sb, bucket);
+}
+
+// CTA per hub (rank r < K): its dense row built in shared memory, then
+// written whole (coalesced; zeros included, so no separate memset).
+__global__ void core_rows_kernel(const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                 const float* __restrict__ val, const int32_t* __restrict__ rank,
+                                 const int32_t* __restrict__ order, int64_t K, float* __restrict__ dense) {
+  extern __shared__ float row[];
+  for (int64_t r = blockIdx.x; r < K; r += gridDim.x) {
+    for (int64_t c = threadIdx.x; c < K; c += blockDim.x) row[c] = 0.f;
+    __syncthreads();
+    const int32_t i = order[r];
+    for (int64_t k = rp[i] + threadIdx.x; k < rp[i + 1]; k += blockDim.x) {
+      const int32_t rj = rank[__ldg(col + k)];
+      if (rj < K) row[rj] = __ldg(val + k);   // CSR entries are distinct
+    }
+    __syncthreads();
+    float4* out = reinterpret_cast<float4*>(dense + r * K);
+    const float4* in = reinterpret_cast<const float4*>(row);
+    for (int64_t c = threadIdx.x; c < K / 4; c += blockDim.x) out[c] = in[c];
+    __syncthreads();
+  }
+}
+
+// warp per subgraph segment: residual (non-core) entries counted
+__global__ void resid_count_kernel(const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
+                                   const int32_t* __restrict__ rank, const int32_t* __restrict__ seg_row,
+                                   const int32_t* __restrict__ segoff, int64_t n, int64_t K,
+                                   int64_t* __restrict__ cnt) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nsegs = segoff[n];
+  for (int64_t sg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; sg < nsegs;
+       sg += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+    const Seg q = seg_of(sg, seg_row, segoff, rp, nullptr);
+    int c = 0;
+    if (rank[q.i] >= K) {
+      c = (int)(q.end - q.b);
+    } else {
+      for (int64_t k = q.b + lane; k < q.end; k += 32) c += rank[__ldg(col + k)] >= K ? 1 : 0;
+#pragma unroll
+      for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
+    }
+    if (lane == 0) cnt[sg] = c;
+  }
+}
+
+__global__ void resid_kernel(const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
+                             const float* __restrict__ val, const int32_t* __restrict__ rank,
+                             const int32_t* __restrict__ seg_row, const int32_t* __restrict__ segoff,
+                             int64_t n, int64_t K, const int64_t* __restrict__ pos,
+                             int32_t* __restrict__ rcol, float* __restrict__ rval) {
+  const int lane = threadIdx.x & 31;
+  const int64_t nsegs = segoff[n];
+  for (int64_t sg = ((int64_t)blockIdx.x * blockDim.x + threadIdx.x) >> 5; sg < nsegs;
+       sg += ((int64_t)gridDim.x * blockDim.x) >> 5) {
+    const Seg q = seg_of(sg, seg_row, segoff, rp, nullptr);
+    const bool hub_i = rank[q.i] < K;
+    int64_t at0 = pos[sg];
+    for (int64_t k0 = q.b; k0 < q.end; k0 += 32) {
+      const int64_t k = k0 + lane;
+      const bool in = k < q.end;
+      const int32_t c = in ? __ldg(col + k) : 0;
+      const bool keep = in && !(hub_i && rank[c] < K);
+      const unsigned m = __ballot_sync(0xffffffffu, keep);
+      if (keep) {
+        const int64_t at = at0 + __popc(m & ((1u << lane) - 1u));
+        rcol[at] = c;
+        rval[at] = __ldg(val + k);
+      }
+      at0 += __popc(m);
+    }
+  }
+}
+
+// residual rowptr from the segment offsets; hub ids / slots
+__global__ void resid_rp_kernel(const int32_t* __restrict__ segoff, const int64_t* __restrict__ pos,
+                                int64_t n, int64_t rnnz, const int32_t* __restrict__ order,
+                                const int32_t* __restrict__ rank, int64_t K, int64_t* __restrict__ rrp,
+                                int32_t* __restrict__ hub_ids, int32_t* __restrict__ hub_slot) {
+  const int64_t nsegs = segoff[n];
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i <= n;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    rrp[i] = segoff[i] < nsegs ? pos[segoff[i]] : rnnz;
+    if (i < n) {
+      if (i < K) hub_ids[i] = order[i];
+      hub_slot[i] = rank[i] < K ? rank[i] : -1;
     }
   }
 }
@@ -192,6 +361,118 @@ unsigned grid_of(rdm_ctx* ctx, int64_t work, int per_block) {
   return (unsigned)std::min<int64_t>(b, (int64_t)ctx->num_sms * 16);
 }
 
+template <class In, class Out>
+void scan(rdm_ctx* ctx, std::unique_ptr<DevBuf>& tmp, In* in, Out* out, int64_t count) {
+  size_t t = 0;
+  RDM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, t, in, out, (int)count, ctx->stream));
+  void* w = ensure_ws(tmp, std::max<size_t>(t, 256));
+  RDM_CUDA(cub::DeviceScan::ExclusiveSum(w, t, in, out, (int)count, ctx->stream));
+}
+
+// Core size bound for a subgraph of n vertices: 0 = no core considered.
+// RDM_NO_CORE=1 disables; RDM_SAINT_CORE_K forces a size (tests).
+int64_t core_kmax(int64_t n, int64_t nnz) {
+  const char* off = getenv("RDM_NO_CORE");
+  const char* force = getenv("RDM_SAINT_CORE_K");
+  const bool forced = force && atoi(force) > 0;
+  if ((off && atoi(off)) || nnz == 0 || (n < 4096 && !forced)) return 0;
+  const int64_t kmax = std::min<int64_t>((forced ? n : n / 2) / 128 * 128, 128 * kMaxBuckets);
+  return kmax >= (forced ? 128 : 1024) ? kmax : 0;
+}
+
+// Hub core of the current subgraph S (bins of S already built): ranks,
+// sampled histogram, K, dense rows, residual CSR (+ its bins).
+void build_core_sub(rdm_saint* s, Csr& S, int64_t kmax, const unsigned long long* deg) {
+  rdm_ctx* ctx = s->ctx;
+  const int64_t n = S.n, nnz = S.nnz;
+  Core& c = S.core;
+  const int64_t* rp = S.rowptr->as<int64_t>();
+  const int32_t* col = S.col->as<int32_t>();
+  const float* val = S.val->as<float>();
+  // degree order (stable, descending) and ranks
+  int32_t* keys = reinterpret_cast<int32_t*>(ensure_ws(s->core_tmp, (size_t)4 * n * sizeof(int32_t) + 256));
+  int32_t* iota = keys + n;
+  int32_t* keys_sorted = iota + n;
+  int32_t* order = keys_sorted + n;
+  int32_t* rank = reinterpret_cast<int32_t*>(ensure_ws(s->core_rank, n * sizeof(int32_t)));
+  deg_key_kernel<<<grid_of(ctx, n, 256), 256, 0, ctx->stream>>>(deg, n, keys, iota);
+  RDM_LAUNCHED(ctx);
+  size_t tb = 0;
+  RDM_CUDA(cub::DeviceRadixSort::SortPairsDescending(nullptr, tb, keys, keys_sorted, iota, order, (int)n, 0,
+                                                      32, ctx->stream));
+  void* tmp = ensure_ws(s->tmp2, std::max<size_t>(tb, 256));
+  RDM_CUDA(cub::DeviceRadixSort::SortPairsDescending(tmp, tb, keys, keys_sorted, iota, order, (int)n, 0, 32,
+                                                      ctx->stream));
+  rank_kernel<<<grid_of(ctx, n, 256), 256, 0, ctx->stream>>>(order, n, rank);
+  RDM_LAUNCHED(ctx);
+  // segment tables of S
+  const int64_t seg_cap = n + nnz / kSeg + 1;
+  int32_t* nseg = reinterpret_cast<int32_t*>(ensure_ws(s->core_seg, (2 * (n + 1) + seg_cap) * 4 + 16));
+  int32_t* segoff = nseg + (n + 1);
+  int32_t* seg_row = segoff + (n + 1);
+  int64_t* cnt = reinterpret_cast<int64_t*>(ensure_ws(s->core_cnt, 2 * seg_cap * sizeof(int64_t)));
+  int64_t* pos = cnt + seg_cap;
+  unsigned long long* bucket = reinterpret_cast<unsigned long long*>(ensure_ws(s->core_bucket, kMaxBuckets * 8));
+  rowseg_kernel<<<grid_of(ctx, n + 1, 256), 256, 0, ctx->stream>>>(rp, nullptr, n, nullptr, n, nseg);
+  RDM_LAUNCHED(ctx);
+  scan(ctx, s->tmp, nseg, segoff, n + 1);
+  segrow_kernel<<<grid_of(ctx, n, 256), 256, 0, ctx->stream>>>(nseg, segoff, nullptr, n, seg_row);
+  RDM_LAUNCHED(ctx);
+  RDM_CUDA(cudaMemsetAsync(bucket, 0, kMaxBuckets * 8, ctx->stream));
+  hist_kernel<<<grid_of(ctx, seg_cap * 32, 256), 256, 0, ctx->stream>>>(rp, col, rank, seg_row, segoff, n, kmax,
+                                                                         bucket);
+  RDM_LAUNCHED(ctx);
+  std::vector<unsigned long long> hb(kMaxBuckets);
+  RDM_CUDA(cudaMemcpyAsync(hb.data(), bucket, kMaxBuckets * 8, cudaMemcpyDeviceToHost, ctx->stream));
+  RDM_CUDA(cudaStreamSynchronize(ctx->stream));
+  std::vector<int64_t> b64(kMaxBuckets);
+  for (int b = 0; b < kMaxBuckets; ++b) b64[b] = (int64_t)hb[b] * 8;   // 1/8 row sample
+  bool forced = false;
+  const int64_t K = choose_core_K(b64.data(), kmax, getenv("RDM_SAINT_CORE_K"), &forced);
+  if (!K) return;
+  // dense rows of the hubs
+  float* dense = ensure_ws(c.A, (size_t)K * K * sizeof(float));
+  const int smem = (int)(K * sizeof(float));
+  RDM_CUDA(cudaFuncSetAttribute(core_rows_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  core_rows_kernel<<<(unsigned)std::min<int64_t>(K, (int64_t)ctx->num_sms * 4), 256, smem, ctx->stream>>>(
+      rp, col, val, rank, order, K, dense);
+  RDM_LAUNCHED(ctx);
+  // residual CSR: count, scan, fill in the original order
+  RDM_CUDA(cudaMemsetAsync(cnt, 0, seg_cap * sizeof(int64_t), ctx->stream));
+  resid_count_kernel<<<grid_of(ctx, seg_cap * 32, 256), 256, 0, ctx->stream>>>(rp, col, rank, seg_row, segoff,
+                                                                                 n, K, cnt);
+  RDM_LAUNCHED(ctx);
+  scan(ctx, s->tmp, cnt, pos, seg_cap);
+  if (!c.resid) c.resid.reset(new Csr());
+  Csr& R = *c.resid;
+  int64_t* rrp = reinterpret_cast<int64_t*>(ensure_ws(R.rowptr, (n + 1) * sizeof(int64_t)));
+  // exact residual size: one more small D2H (the scan's last prefix + count)
+  int64_t tail[2];
+  RDM_CUDA(cudaMemcpyAsync(tail, pos + seg_cap - 1, 8, cudaMemcpyDeviceToHost, ctx->stream));
+  RDM_CUDA(cudaMemcpyAsync(tail + 1, cnt + seg_cap - 1, 8, cudaMemcpyDeviceToHost, ctx->stream));
+  RDM_CUDA(cudaStreamSynchronize(ctx->stream));
+  const int64_t rnnz = tail[0] + tail[1];
+  int32_t* rcol = reinterpret_cast<int32_t*>(ensure_ws(R.col, std::max<int64_t>(rnnz, 1) * sizeof(int32_t)));
+  float* rval = ensure_ws(R.val, std::max<int64_t>(rnnz, 1) * sizeof(float));
+  resid_kernel<<<grid_of(ctx, seg_cap * 32, 256), 256, 0, ctx->stream>>>(rp, col, val, rank, seg_row, segoff,
+                                                                          n, K, pos, rcol, rval);
+  RDM_LAUNCHED(ctx);
+  int32_t* hub_ids = reinterpret_cast<int32_t*>(ensure_ws(c.hub_ids, K * sizeof(int32_t)));
+  int32_t* hub_slot = reinterpret_cast<int32_t*>(ensure_ws(c.hub_slot, n * sizeof(int32_t)));
+  resid_rp_kernel<<<grid_of(ctx, n + 1, 256), 256, 0, ctx->stream>>>(segoff, pos, n, rnnz, order, rank, K,
+                                                                       rrp, hub_ids, hub_slot);
+  RDM_LAUNCHED(ctx);
+  std::vector<int64_t> rrph(n + 1);
+  RDM_CUDA(cudaMemcpyAsync(rrph.data(), rrp, (n + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, ctx->stream));
+  RDM_CUDA(cudaStreamSynchronize(ctx->stream));
+  R.n = n;
+  R.nnz = rnnz;
+  build_bins(ctx, R, rrph.data());
+  c.K = K;
+  c.nnz = nnz - rnnz;
+  c.forced = forced;
+}
+
 void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
   rdm_ctx* ctx = s->ctx;
   Phase ph(ctx, RDM_PH_SAMPLE);
@@ -213,18 +494,6 @@ void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
   int64_t* cnt = reinterpret_cast<int64_t*>(ensure_ws(s->rps, 2 * seg_cap * sizeof(int64_t)));
   int64_t* pos = cnt + seg_cap;
   unsigned long long* scal = reinterpret_cast<unsigned long long*>(ensure_ws(s->scal, 64));
-  size_t tb[4] = {0, 0, 0, 0};
-  RDM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb[0], flag, map, (int)N, ctx->stream));
-  RDM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb[1], nseg, segoff, (int)(cap + 1), ctx->stream));
-  RDM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb[2], cnt, pos, (int)seg_cap, ctx->stream));
-  int64_t* rp_dummy = nullptr;
-  RDM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, tb[3], deg, rp_dummy, (int)(cap + 1), ctx->stream));
-  const size_t tbm = std::max(std::max(tb[0], tb[1]), std::max(tb[2], tb[3]));
-  void* tmp = ensure_ws(s->tmp, tbm);
-  auto scan = [&](auto* in, auto* out, int64_t count) {
-    size_t t = tbm;
-    RDM_CUDA(cub::DeviceScan::ExclusiveSum(tmp, t, in, out, (int)count, ctx->stream));
-  };
 
   const uint64_t key = splitmix64_host(s->seed + (uint64_t)it * 0x9E3779B97F4A7C15ull);
   RDM_CUDA(cudaMemsetAsync(flag, 0, N * sizeof(int32_t), ctx->stream));
@@ -236,14 +505,14 @@ void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
   RDM_LAUNCHED(ctx);
   mark_kernel<<<grid_of(ctx, nv, 256), 256, 0, ctx->stream>>>(visits, nv, flag);
   RDM_LAUNCHED(ctx);
-  scan(flag, map, N);
+  scan(ctx, s->tmp, flag, map, N);
   compact_kernel<<<grid_of(ctx, N, 256), 256, 0, ctx->stream>>>(flag, map, N, nodes, scal);
   RDM_LAUNCHED(ctx);
-  rowseg_kernel<<<grid_of(ctx, cap + 1, 256), 256, 0, ctx->stream>>>(A.rowptr->as<int64_t>(), nodes,
-                                                                       cap, scal, nseg);
+  rowseg_kernel<<<grid_of(ctx, cap + 1, 256), 256, 0, ctx->stream>>>(A.rowptr->as<int64_t>(), nodes, cap,
+                                                                       scal, 0, nseg);
   RDM_LAUNCHED(ctx);
-  scan(nseg, segoff, cap + 1);
-  segrow_kernel<<<grid_of(ctx, cap, 256), 256, 0, ctx->stream>>>(nseg, segoff, scal, seg_row);
+  scan(ctx, s->tmp, nseg, segoff, cap + 1);
+  segrow_kernel<<<grid_of(ctx, cap, 256), 256, 0, ctx->stream>>>(nseg, segoff, scal, 0, seg_row);
   RDM_LAUNCHED(ctx);
   count_kernel<<<grid_of(ctx, seg_cap * 32, 256), 256, 0, ctx->stream>>>(
       A.rowptr->as<int64_t>(), A.col->as<int32_t>(), flag, nodes, seg_row, segoff, cap, cnt, deg, scal);
@@ -256,12 +525,14 @@ void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
 
   Graph& G = s->graph;
   Csr& S = G.A;
+  S.core.K = 0;
+  S.core.nnz = 0;
   int64_t* rp = reinterpret_cast<int64_t*>(ensure_ws(S.rowptr, (cap + 1) * sizeof(int64_t)));
   int32_t* cs = reinterpret_cast<int32_t*>(ensure_ws(S.col, std::max<int64_t>(nnz, 1) * sizeof(int32_t)));
   float* vs = ensure_ws(S.val, std::max<int64_t>(nnz, 1) * sizeof(float));
   // rowptr_s: prefix of d (zero beyond n); segment output offsets: prefix of c
-  scan(deg, rp, cap + 1);
-  scan(cnt, pos, seg_cap);
+  scan(ctx, s->tmp, deg, rp, cap + 1);
+  scan(ctx, s->tmp, cnt, pos, seg_cap);
   fill_kernel<<<grid_of(ctx, seg_cap * 32, 256), 256, 0, ctx->stream>>>(
       A.rowptr->as<int64_t>(), A.col->as<int32_t>(), flag, map, nodes, seg_row, segoff, cap, deg, pos,
       cs, vs);
@@ -272,6 +543,7 @@ void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
   S.n = n;
   S.nnz = nnz;
   build_bins(ctx, S, rph.data());
+  if (const int64_t kmax = core_kmax(n, nnz)) build_core_sub(s, S, kmax, deg);
   G.n = n;
   G.nnz = nnz;
   G.symmetric = true;

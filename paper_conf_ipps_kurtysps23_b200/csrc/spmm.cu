@@ -269,6 +269,33 @@ bool core_pays(const Core& c, int64_t w) {
   return c.forced || core_saving_s(c.nnz, w) > core_cost_s(c.K, w);
 }
 
+}  // namespace
+
+// Core size (multiple of 128, <= kmax) with the largest modelled saving at the
+// reference width 128, at least 0.1 ms per call; bucket[b] = entries whose
+// larger endpoint degree-rank lies in [128 b, 128 b + 128).  `force` (an env
+// value, tests): use that size.  0 = no core.
+int64_t choose_core_K(const int64_t* bucket, int64_t kmax, const char* force, bool* forced) {
+  int64_t best_K = 0;
+  double best_gain = 1e-4;
+  int64_t acc = 0;
+  for (int64_t K = 128; K <= kmax; K += 128) {
+    acc += bucket[K / 128 - 1];
+    const double gain = core_saving_s(acc, 128) - core_cost_s(K, 128);
+    if (gain > best_gain) {
+      best_gain = gain;
+      best_K = K;
+    }
+  }
+  *forced = false;
+  if (force && atoi(force) > 0 && kmax >= 128) {
+    best_K = std::min<int64_t>(kmax, std::max<int64_t>(128, (int64_t)atoi(force) / 128 * 128));
+    *forced = true;
+  }
+  return best_K;
+}
+
+namespace {
 // Panels of X[hubs] for the core GEMM: Bt_hi/lo[n][k] = tf32 split of X[hub_ids[k]][n]
 // (transposed through shared memory: coalesced reads along n, writes along k).
 __global__ void core_panels_kernel(const float* __restrict__ X, int64_t ldx,
@@ -462,24 +489,10 @@ void build_core(rdm_ctx* ctx, Csr& A, const int64_t* rp, const int32_t* col, con
       hist[m < kmax ? m : kmax]++;
     }
   }
-  int64_t best_K = 0, best_nnz = 0;
-  double best_gain = 1e-4;  // must save at least 0.1 ms per width-128 call
-  int64_t acc = 0, b = 0;
-  for (int64_t K = 128; K <= kmax; K += 128) {
-    for (; b < K; ++b) acc += hist[b];
-    const double gain = core_saving_s(acc, 128) - core_cost_s(K, 128);
-    if (gain > best_gain) {
-      best_gain = gain;
-      best_K = K;
-      best_nnz = acc;
-    }
-  }
-  const char* force = getenv("RDM_CORE_K");  // tests: force a core of this size
+  std::vector<int64_t> bucket(kmax / 128, 0);
+  for (int64_t m = 0; m < kmax; ++m) bucket[m / 128] += hist[m];
   bool forced = false;
-  if (force && atoi(force) > 0) {
-    best_K = std::min<int64_t>(kmax, std::max<int64_t>(128, (int64_t)atoi(force) / 128 * 128));
-    forced = true;
-  }
+  const int64_t best_K = choose_core_K(bucket.data(), kmax, getenv("RDM_CORE_K"), &forced);
   if (!best_K) return;
   const int64_t K = best_K;
   A.core.forced = forced;
@@ -512,7 +525,6 @@ void build_core(rdm_ctx* ctx, Csr& A, const int64_t* rp, const int32_t* col, con
   Core& c = A.core;
   c.K = K;
   c.nnz = nnz - rnnz;
-  (void)best_nnz;
   c.A.reset(new DevBuf((size_t)K * K * sizeof(float)));
   RDM_CUDA(cudaMemcpy(c.A->ptr, dense.data(), (size_t)K * K * sizeof(float), cudaMemcpyHostToDevice));
   c.hub_ids.reset(new DevBuf(K * sizeof(int32_t)));

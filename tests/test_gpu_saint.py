@@ -88,8 +88,13 @@ def _saint_run(rdm, g, H0, Ws, y, m, cfg, P, roots, h, seed, iters):
     s.close()
 
 
-@pytest.mark.parametrize("P,cfg", [(1, 3), (1, 10), (2, 3), (4, 10), (4, 2)])
-def test_saint_gcn_matches_oracle(rdm, P, cfg):
+@pytest.mark.parametrize("P,cfg,core", [(1, 3, 0), (1, 10, 0), (2, 3, 0), (4, 10, 0), (4, 2, 0),
+                                        (1, 3, 256), (2, 10, 384)])
+def test_saint_gcn_matches_oracle(rdm, P, cfg, core, monkeypatch):
+    """core > 0 forces a dense hub core of that size on every subgraph
+    (RDM_SAINT_CORE_K): the device-built core + residual CSR path."""
+    if core:
+        monkeypatch.setenv("RDM_SAINT_CORE_K", str(core))
     n, f = 4000, (300, 64, 11)
     g = synth.rmat(n, 40000, seed=6)
     H0 = synth.features(n, f[0])
@@ -142,5 +147,36 @@ def test_saint_requires_sample_and_input(rdm):
     with pytest.raises(rdm.RdmError):
         model.set_input([torch.zeros(1, 16, device="cuda:0")], [torch.zeros(1, dtype=torch.int32,
                                                                              device="cuda:0")])
+    model.close()
+    s.close()
+
+
+def test_saint_core_spmm_matches_oracle(rdm, monkeypatch):
+    """Device-built hub core of a subgraph: A_s·X through rdm's SpMM on the
+    sampler's graph equals the oracle product on the oracle's subgraph."""
+    import torch
+    monkeypatch.setenv("RDM_SAINT_CORE_K", "512")
+    g = synth.rmat(6000, 90000, seed=8)
+    ctx = rdm.Context(device=0)
+    ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
+    s = rdm.Saint(ctx, 600, walk_len=4, seed=5)
+    f = [48, 40, 5]
+    model = s.gcn(f, 10)          # D-first forward: SpMM of width 40 and 5
+    for it in range(2):
+        s.sample(it)
+        nodes, rp, cs, vs = osaint.sample(g, 600, 4, 5, it)
+        sub = synth.CSR(len(nodes), rp, cs, vs)
+        H0 = synth.features(g.n, f[0])
+        Ws = synth.weights(f)
+        y = synth.labels(g.n, f[-1])
+        dev = "cuda:0"
+        model.saint_input(torch.from_numpy(H0).to(dev), torch.from_numpy(y).to(dev))
+        Wd = [torch.from_numpy(w).to(dev) for w in Ws]
+        loss = torch.zeros(1, dtype=torch.float64, device=dev)
+        model.forward(Wd, loss)
+        ctx.sync()
+        Z = model.tensor_torch(rdm.T_Z, 0).cpu().numpy()
+        ref = og.forward(sub, H0[nodes], Ws, y[nodes], np.ones(len(nodes), dtype=bool))
+        assert og.max_rel_err(Z, ref.Z[len(Ws)]) < 1e-4
     model.close()
     s.close()
