@@ -19,11 +19,11 @@ LIB       := $(PKG)/lib/librdm.so
 
 all: $(LIB) synth/libsynth.so oracle/liboracle.so
 
-$(OBJDIR)/%.o: $(SRC)/%.cu $(SRC)/internal.h include/rdm.h
+$(OBJDIR)/%.o: $(SRC)/%.cu $(wildcard $(SRC)/*.h) include/rdm.h
 	@mkdir -p $(OBJDIR)
 	$(NVCC) $(NVFLAGS) -c $< -o $@ 2> $@.log || (cat $@.log; false)
 
-$(OBJDIR)/%.o: $(SRC)/%.cpp $(SRC)/internal.h include/rdm.h
+$(OBJDIR)/%.o: $(SRC)/%.cpp $(wildcard $(SRC)/*.h) include/rdm.h
 	@mkdir -p $(OBJDIR)
 	$(NVCC) $(NVFLAGS) -x cu -c $< -o $@ 2> $@.log || (cat $@.log; false)
 

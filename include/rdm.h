@@ -216,12 +216,19 @@ rdm_status rdm_set_graph(rdm_ctx* ctx, int64_t n, int64_t nnz, const int64_t* ro
  * 2048-nnz segments) and, for symmetric graphs with a dense block of
  * high-degree vertices, the "hub core": the K x K block A[hubs, hubs] (K a
  * multiple of 128, core_nnz entries) held dense and multiplied on the tensor
- * cores, the other entries in a residual CSR (core_K = 0: no core). */
+ * cores, the other entries in a residual CSR (core_K = 0: no core).
+ * When every value of the hub region factors as a_ij = s_i s_j (the GCN
+ * normalization D^-1/2 (A+I) D^-1/2, or all ones; checked entry by entry to
+ * 2^-21 relative) the core is instead a set of "binary hub tiles": the
+ * tile_ranks highest-degree vertices' block cut into 128 x 128 rank blocks,
+ * the n_tiles blocks dense enough to pay stored as 0/1 and multiplied on the
+ * tensor cores against s ⊙ X (core_K = 0, core_nnz = entries moved). */
 typedef struct {
   int64_t n, nnz;
   int64_t n_light_rows, n_heavy_rows, n_segments, max_degree;
   int64_t core_K, core_nnz;
   int symmetric;
+  int64_t tile_ranks, n_tiles, n_tile_items;
 } rdm_graph_info;
 rdm_status rdm_get_graph_info(const rdm_ctx* ctx, rdm_graph_info* out);
 

@@ -514,7 +514,8 @@ for _n in ("rdm_saint_create", "rdm_saint_destroy", "rdm_saint_sample", "rdm_sai
 class RdmGraphInfo(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int64) for n in ("n", "nnz", "n_light_rows", "n_heavy_rows",
                                                "n_segments", "max_degree", "core_K", "core_nnz")] + \
-               [("symmetric", ctypes.c_int)]
+               [("symmetric", ctypes.c_int)] + \
+               [(k, ctypes.c_int64) for k in ("tile_ranks", "n_tiles", "n_tile_items")]
 
     def as_dict(self):
         return {n: getattr(self, n) for n, _ in self._fields_}

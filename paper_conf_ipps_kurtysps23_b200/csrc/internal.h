@@ -85,6 +85,19 @@ struct Core {
   std::unique_ptr<DevBuf> hub_ids;     // int32[K]: vertex of slot k
   std::unique_ptr<DevBuf> hub_slot;    // int32[N]: slot of vertex v, -1 if not a hub
   std::unique_ptr<Csr> resid;          // A minus the core entries (with its own bins)
+  // Binary hub tiles (hubtiles.cu) — used instead of the dense block (K = 0)
+  // when every value of the hub region factors as a_ij = s_i·s_j (the GCN
+  // symmetric normalisation D^-1/2 (A+I) D^-1/2, or all ones): the region of
+  // the K2 highest-degree vertices is cut into 128 x 128 rank blocks, blocks
+  // dense enough to pay are stored as 0/1 bf16 tiles and multiplied on the
+  // kind::f16 tensor cores against s_j·X_j split into three bf16 pieces.
+  int64_t K2 = 0;                      // rank range covered (multiple of 128), 0 = none
+  int64_t n_tiles = 0, n_items = 0, n_rb = 0;
+  std::unique_ptr<DevBuf> tiles;       // bf16 [n_tiles][128][128], 0/1 (row = rank in block)
+  std::unique_ptr<DevBuf> tile_cb;     // int32[n_tiles]: column block of each tile
+  std::unique_ptr<DevBuf> item_tb;     // int32[n_items+1]: tile range of each work item
+  std::unique_ptr<DevBuf> rb_item;     // int32[n_rb+1]: item range of each row block
+  std::unique_ptr<DevBuf> scale;       // fp32[K2]: s of the vertex of slot k
 };
 
 struct Csr {
@@ -211,6 +224,16 @@ void gemm_tc_panels(rdm_ctx* ctx, const float* A, int64_t lda, const float* bhi,
 // dense hub core (spmm.cu)
 void build_core(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, const int32_t* col_host,
                 const float* val_host);
+
+// binary hub tiles (hubtiles.cu): host builder (false = values do not factor
+// or no tile pays; nothing built) and the per-call product
+//   part[item][r][c] = Σ_{tiles of item} T01 · (s ⊙ X[hubs]) (columns < w),
+// summed per row block and scaled by s_i in the SpMM epilogue.
+bool build_hub_tiles(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, const int32_t* col_host,
+                     const float* val_host);
+bool hub_tiles_pay(const Core& c, int64_t w);
+void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx, int64_t w,
+                       float* part, int64_t ldp);
 
 // hub-core size rule shared by the host (full graph) and device (subgraph) builders
 int64_t choose_core_K(const int64_t* bucket, int64_t kmax, const char* force, bool* forced);

@@ -529,6 +529,9 @@ rdm_status rdm_get_graph_info(const rdm_ctx* ctx, rdm_graph_info* out) {
   out->core_K = A.core.K;
   out->core_nnz = A.core.nnz;
   out->symmetric = ctx->graph.symmetric ? 1 : 0;
+  out->tile_ranks = A.core.K2;
+  out->n_tiles = A.core.n_tiles;
+  out->n_tile_items = A.core.n_items;
   return RDM_OK;
 }
 

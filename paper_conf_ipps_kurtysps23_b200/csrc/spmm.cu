@@ -43,6 +43,10 @@ struct Epi {
   const float* core;        // hub-core product (K x ld_core) or null
   int64_t ld_core;
   const int32_t* hub_slot;  // int32[N], -1 for non-hubs
+  const float* tpart;       // binary hub tiles: per-item partials (n_items x 128 x ld_tpart) or null
+  int64_t ld_tpart;
+  const int32_t* rb_item;   // item range of each 128-row rank block
+  const float* tscale;      // s_i of slot i
   Scatter scat;             // fused col→row redistribution (scat.P == 0: off)
 };
 
@@ -68,6 +72,20 @@ __device__ __forceinline__ float4 apply_epi(float4 a, const Epi& e, int64_t row,
     if (s >= 0) {
       const float4 k = __ldg(reinterpret_cast<const float4*>(e.core + (int64_t)s * e.ld_core + c));
       a.x += k.x; a.y += k.y; a.z += k.z; a.w += k.w;
+    }
+  }
+  if (e.tpart) {  // binary hub tiles: s_i · Σ_items partial (item order; after the CSR sum)
+    const int s = __ldg(e.hub_slot + row);
+    if (s >= 0) {
+      const int i0 = __ldg(e.rb_item + (s >> 7)), i1 = __ldg(e.rb_item + (s >> 7) + 1);
+      float4 t = make_float4(0.f, 0.f, 0.f, 0.f);
+      for (int it = i0; it < i1; ++it) {
+        const float4 k =
+            __ldg(reinterpret_cast<const float4*>(e.tpart + ((int64_t)it * 128 + (s & 127)) * e.ld_tpart + c));
+        t.x += k.x; t.y += k.y; t.z += k.z; t.w += k.w;
+      }
+      const float sc = __ldg(e.tscale + s);
+      a.x = fmaf(sc, t.x, a.x); a.y = fmaf(sc, t.y, a.y); a.z = fmaf(sc, t.z, a.z); a.w = fmaf(sc, t.w, a.w);
     }
   }
   if (e.flags & RDM_EPI_BIAS) {
@@ -335,13 +353,25 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
                                                 ((uintptr_t)mask & 15) == 0),
                 "spmm: mask requires a 16-byte aligned N x w buffer with ld % 4 == 0");
   RDM_CHECK_ARG(!(epi_flags & RDM_EPI_BIAS) || bias, "spmm: bias pointer missing");
-  Epi epi{epi_flags, bias, mask, ld_mask, w, nullptr, 0, nullptr, Scatter{}};
+  Epi epi{epi_flags, bias, mask, ld_mask, w, nullptr, 0, nullptr, nullptr, 0, nullptr, nullptr, Scatter{}};
   if (scat) {
     RDM_CHECK_ARG(scat->mode == 2 && scat->P >= 1 && scat->P <= Scatter::kMax && scat->my_w <= w,
                   "spmm: bad scatter descriptor");
     epi.scat = *scat;
   }
-  if (A.core.K && core_pays(A.core, w)) {
+  if (A.core.n_tiles && hub_tiles_pay(A.core, w)) {
+    // binary hub tiles on the kind::f16 tensor cores (hubtiles.cu); the
+    // residual CSR's epilogue adds s_i · Σ_items partial for hub rows.
+    const int64_t ldp = w4;
+    float* part = ensure_ws(ctx->ws_core_c, (size_t)A.core.n_items * 128 * ldp * sizeof(float));
+    hub_tiles_product(ctx, A.core, in, ld_in, w, part, ldp);
+    epi.tpart = part;
+    epi.ld_tpart = ldp;
+    epi.rb_item = A.core.rb_item->as<int32_t>();
+    epi.tscale = A.core.scale->as<float>();
+    epi.hub_slot = A.core.hub_slot->as<int32_t>();
+    run_csr(ctx, *A.core.resid, in, ld_in, out, ld_out, w4, epi);
+  } else if (A.core.K && core_pays(A.core, w)) {
     // hub core on the tensor cores: panels Bt[n][k] = split(X[hub_k][n]), then
     // C_core = Acore · X[hubs]; the residual CSR's epilogue adds C_core rows.
     const int64_t K = A.core.K;
@@ -471,7 +501,9 @@ void build_core(rdm_ctx* ctx, Csr& A, const int64_t* rp, const int32_t* col, con
   (void)ctx;
   const int64_t n = A.n, nnz = A.nnz;
   const char* off = getenv("RDM_NO_CORE");
-  if ((off && atoi(off)) || n < 4096 || nnz == 0) return;
+  if ((off && atoi(off)) || nnz == 0) return;
+  if (build_hub_tiles(ctx, A, rp, col, val)) return;   // values factor: binary tiles
+  if (n < 4096) return;
   std::vector<int32_t> order(n);
   for (int64_t i = 0; i < n; ++i) order[i] = (int32_t)i;
   std::stable_sort(order.begin(), order.end(), [&](int32_t a, int32_t b) {

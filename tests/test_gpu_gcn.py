@@ -290,6 +290,17 @@ def test_zero_last_layer_loss_is_ln_C(rdm):
     assert abs(loss - np.log(41)) < 1e-6
 
 
+@pytest.mark.parametrize("P,cfg", [(1, 3), (1, 10), (2, 3), (4, 10), (2, 6), (3, 9)])
+def test_hub_tiles_gcn(rdm, P, cfg, monkeypatch):
+    """Full epoch with the SpMMs on binary hub tiles (forced selection) + the
+    residual CSR, single GPU and virtual groups, against the oracle."""
+    monkeypatch.setenv("RDM_TILE_MIN_NNZ", "20")
+    prob = _problem(n=6000, E=150000, f=(64, 48, 41), seed=13)
+    loss, dW, model, ctx, _ = _run(rdm, *prob, cfg, P=P)
+    assert ctx.graph_info()["n_tiles"] > 0
+    _check(prob, loss, dW, model, rdm, P=P)
+
+
 @pytest.mark.slow
 def test_reddit_full_size_sampled(rdm):
     """BASELINE configs[1] at full size, in bench.py's launch configuration (P=1,

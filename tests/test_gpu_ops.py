@@ -219,6 +219,7 @@ def test_spmm_hub_core_matches_oracle(torch_dev, w, K, monkeypatch):
     torch, dev = torch_dev
     import paper_conf_ipps_kurtysps23_b200 as rdm
     monkeypatch.setenv("RDM_CORE_K", str(K))
+    monkeypatch.setenv("RDM_NO_TILES", "1")   # the fp32 dense core, not the binary tiles
     g = synth.rmat(6000, 150000, seed=13)
     ctx = rdm.Context(device=0)
     ctx.set_graph(g.rowptr, g.col, g.val)
@@ -234,3 +235,82 @@ def test_spmm_hub_core_matches_oracle(torch_dev, w, K, monkeypatch):
     ref = np.maximum(og.spmm(g, X), 0) * (M > 0)
     assert og.max_rel_err(out[:, :w].cpu().numpy(), ref) < TOL
     assert np.all(out[:, w:].cpu().numpy() == 0)
+
+
+@pytest.mark.parametrize("w", [1, 4, 16, 41, 128, 130, 256, 301])
+@pytest.mark.parametrize("min_nnz,k2", [(1, 0), (40, 0), (1, 1024)])
+def test_spmm_hub_tiles_matches_oracle(torch_dev, w, min_nnz, k2, monkeypatch):
+    """Binary hub tiles (kind::f16 tensor cores on 0/1 tiles against the
+    3-piece bf16 split of s ⊙ X) + residual CSR == the plain product, with
+    epilogues.  min_nnz forces the tile selection (every block with at least
+    that many entries), k2 limits the rank range (0 = all)."""
+    torch, dev = torch_dev
+    import paper_conf_ipps_kurtysps23_b200 as rdm
+    monkeypatch.setenv("RDM_TILE_MIN_NNZ", str(min_nnz))
+    if k2:
+        monkeypatch.setenv("RDM_TILE_K2", str(k2))
+    g = synth.rmat(6000, 150000, seed=13)
+    ctx = rdm.Context(device=0)
+    ctx.set_graph(g.rowptr, g.col, g.val)
+    gi = ctx.graph_info()
+    assert gi["n_tiles"] > 0 and gi["core_K"] == 0 and gi["core_nnz"] > 0
+    assert gi["tile_ranks"] % 128 == 0 and gi["tile_ranks"] <= (k2 or g.n)
+    rng = np.random.default_rng(w)
+    X = rng.standard_normal((g.n, w)).astype(np.float32)
+    M = rng.standard_normal((g.n, w)).astype(np.float32)
+    xd, md = _padded(torch, dev, X), _padded(torch, dev, M)
+    out = torch.zeros_like(xd)
+    ctx.spmm(0, xd, out, w)
+    ctx.sync()
+    assert og.max_rel_err(out[:, :w].cpu().numpy(), og.spmm(g, X)) < TOL
+    out.zero_()
+    ctx.spmm(0, xd, out, w, rdm.EPI_RELU | rdm.EPI_MASK, mask=md)
+    ctx.sync()
+    ref = np.maximum(og.spmm(g, X), 0) * (M > 0)
+    assert og.max_rel_err(out[:, :w].cpu().numpy(), ref) < TOL
+    assert np.all(out[:, w:].cpu().numpy() == 0)
+
+
+def test_spmm_hub_tiles_wide_range_values(torch_dev, monkeypatch):
+    """Inputs spanning 2^±30 and exact zeros: the three bf16 pieces keep
+    fp32-class relative accuracy per row (no flush of the small pieces)."""
+    torch, dev = torch_dev
+    import paper_conf_ipps_kurtysps23_b200 as rdm
+    monkeypatch.setenv("RDM_TILE_MIN_NNZ", "1")
+    g = synth.rmat(6000, 150000, seed=14)
+    ctx = rdm.Context(device=0)
+    ctx.set_graph(g.rowptr, g.col, g.val)
+    assert ctx.graph_info()["n_tiles"] > 0
+    rng = np.random.default_rng(0)
+    w = 64
+    X = (rng.standard_normal((g.n, w)) * np.exp2(rng.integers(-30, 30, (g.n, 1)))).astype(np.float32)
+    X[rng.random((g.n, w)) < 0.1] = 0
+    xd = _padded(torch, dev, X)
+    out = torch.zeros_like(xd)
+    ctx.spmm(0, xd, out, w)
+    ctx.sync()
+    assert og.max_rel_err(out[:, :w].cpu().numpy(), og.spmm(g, X)) < TOL
+
+
+def test_spmm_hub_tiles_need_factorised_values(torch_dev, monkeypatch):
+    """Values that are not s_i·s_j (here: perturbed by 1e-3 relative) build no
+    binary tiles (the fp32 dense core or plain CSR instead); unit values do."""
+    torch, dev = torch_dev
+    import paper_conf_ipps_kurtysps23_b200 as rdm
+    monkeypatch.setenv("RDM_TILE_MIN_NNZ", "1")
+    g = synth.rmat(6000, 150000, seed=15)
+    rng = np.random.default_rng(1)
+    bad = (g.val * (1 + 1e-3 * rng.standard_normal(g.nnz))).astype(np.float32)
+    ones = np.ones_like(g.val)
+    w = 41
+    X = rng.standard_normal((g.n, w)).astype(np.float32)
+    xd = _padded(torch, dev, X)
+    for vals, tiled in ((bad, False), (ones, True)):
+        ctx = rdm.Context(device=0)
+        ctx.set_graph(g.rowptr, g.col, vals)
+        assert (ctx.graph_info()["n_tiles"] > 0) == tiled
+        out = torch.zeros_like(xd)
+        ctx.spmm(0, xd, out, w)
+        ctx.sync()
+        g2 = synth.CSR(g.n, g.rowptr, g.col, vals)
+        assert og.max_rel_err(out[:, :w].cpu().numpy(), og.spmm(g2, X)) < TOL
