@@ -13,6 +13,8 @@ import os
 
 _HERE = os.path.dirname(os.path.abspath(__file__))
 LIB_PATH = os.path.join(_HERE, "lib", "librdm.so")
+if os.environ.get("RDM_LIB_VARIANT"):   # timing experiments only (tools/build_variant.sh)
+    LIB_PATH = os.path.join(_HERE, "lib", f"librdm_{os.environ['RDM_LIB_VARIANT']}.so")
 
 if not os.path.exists(LIB_PATH):
     raise ImportError(

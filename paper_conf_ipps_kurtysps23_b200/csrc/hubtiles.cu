@@ -15,8 +15,9 @@
 //
 //   (Â X)_i = s_i · Σ_j b_ij · (s_j X_j)        b_ij ∈ {0, 1}
 //
-// * b is exact in bf16 → the A operand of a kind::f16 MMA is exact, and a
-//   tile costs 32 KB (vs 64 KB fp32) of HBM;
+// * b is exact in bf16 → the A operand of a kind::f16 MMA is exact; tiles are
+//   stored as bits (2 KB per 128 x 128 tile, vs 64 KB fp32) and expanded to
+//   bf16 in shared memory;
 // * X'_j = s_j X_j (fp32) is split into three bf16 pieces hi + mid + lo
 //   (8 + 8 + 8 significant bits = fp32's 24), so b·X' = b·hi + b·mid + b·lo
 //   with exact products and fp32 accumulation: fp32-class accuracy at 1.5x the
@@ -30,12 +31,13 @@
 // (spmm.cu build_core) or none.
 //
 // Kernel (persistent, one CTA per SM, warp-specialised like gemm_tc.cu):
-//   warp 0 TMA producer: per 64-wide k stage the A tile half (128 x 64 bf16,
-//          16 KB) and the three B pieces (n_mma x 64 bf16 each), 128B swizzle
+//   warp 0 TMA producer: per 64-wide k stage the tile half's bits (1 KB, bulk
+//          copy) and the three B pieces (n_mma x 64 bf16 each, 128B swizzle)
 //   warp 1 MMA issuer: 4 k16 steps x 3 pieces of tcgen05.mma kind::f16 per
 //          stage into a double-buffered TMEM accumulator (128 x n_mma fp32)
 //   warp 2 TMEM allocator
-//   warps 4-7 epilogue: tcgen05.ld → partial rows of the work item → global
+//   warps 4-7 expander: bits → 0/1 bf16 A half-tile (128 x 64, swizzled smem)
+//   warps 8-11 epilogue: tcgen05.ld → partial rows of the work item → global
 // A work item is a run of ≤ `chunk` tiles of one 128-row block; its 128 x w
 // partial goes to part[item] and the SpMM epilogue sums the items of the row's
 // block in item order.
@@ -66,28 +68,74 @@ __host__ __device__ constexpr uint32_t idesc_bf16(int N) {
   return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
 }
 
-__global__ void __launch_bounds__(256, 1)
-hub_tile_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB0,
-                const __grid_constant__ CUtensorMap tmB1, const __grid_constant__ CUtensorMap tmB2,
+__device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile(
+      "cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];" ::"r"(
+          smem_u32(dst)),
+      "l"((uint64_t)src), "r"(bytes), "r"(smem_u32(bar))
+      : "memory");
+}
+
+// kind::f16 MMA with A from TMEM (bf16 pairs packed in 32-bit columns).
+__device__ __forceinline__ void tc_mma_f16_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t idesc,
+                                              uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "r"(tmem_a), "l"(db), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+__device__ __forceinline__ void tmem_st32u(uint32_t addr, const uint32_t (&v)[32]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x32.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,"
+      "%15,%16,%17,%18,%19,%20,%21,%22,%23,%24,%25,%26,%27,%28,%29,%30,%31,%32};" ::"r"(addr),
+      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]),
+      "r"(v[8]), "r"(v[9]), "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15]),
+      "r"(v[16]), "r"(v[17]), "r"(v[18]), "r"(v[19]), "r"(v[20]), "r"(v[21]), "r"(v[22]), "r"(v[23]),
+      "r"(v[24]), "r"(v[25]), "r"(v[26]), "r"(v[27]), "r"(v[28]), "r"(v[29]), "r"(v[30]), "r"(v[31])
+      : "memory");
+}
+
+// Two bits → two bf16 (0 or 1.0 = 0x3F80) packed in one 32-bit word.
+__device__ __forceinline__ uint32_t bits2_bf16(uint32_t b) {
+  return ((b & 1u) * 0x3F80u) | (((b >> 1) & 1u) * 0x3F800000u);
+}
+
+__global__ void __launch_bounds__(384, 1)
+hub_tile_kernel(const __grid_constant__ CUtensorMap tmB0, const __grid_constant__ CUtensorMap tmB1,
+                const __grid_constant__ CUtensorMap tmB2, const uint64_t* __restrict__ bits,
                 const int32_t* __restrict__ tile_cb, const int32_t* __restrict__ item_tb, int n_items,
                 int tiles_n, int n_mma, int64_t w, float* __restrict__ part, int64_t ldp, int S,
-                int stage_bytes) {
+                int stage_bytes, int R, int acc_cols, int dbg) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint64_t* full = (uint64_t*)(smem + S * stage_bytes);
-  uint64_t* empty = full + S;
+  uint64_t* conv = full + S;
+  uint64_t* empty = conv + S;
   uint64_t* tfull = empty + S;   // [2]
   uint64_t* tempty = tfull + 2;  // [2]
   uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
+  uint4* lut = (uint4*)(smem + S * stage_bytes + 1024);   // byte → 8 bf16 (0 / 1)
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int total = n_items * tiles_n;
+  for (int i = threadIdx.x; i < 256; i += blockDim.x)
+    lut[i] = make_uint4(bits2_bf16(i), bits2_bf16(i >> 2), bits2_bf16(i >> 4), bits2_bf16(i >> 6));
   const int bpiece = n_mma * 128;                 // bytes of one B piece per stage
-  auto A_st = [&](int s) { return smem + s * stage_bytes; };
-  auto B_st = [&](int s, int p) { return smem + s * stage_bytes + 16384 + p * bpiece; };
+  // stage: three B pieces | the half-tile's bits.  TMEM: two accumulator
+  // buffers of acc_cols columns, then the A ring (stage s at kAcol + 32 s, 64
+  // bf16 per row packed in pairs).  R > 0 ("concatenated" mode, n_mma ≤ 64):
+  // one MMA of N = 3 n_mma covers the three pieces (adjacent in smem) and
+  // k16 steps rotate over R accumulator sets [rho][piece][n_mma]; R = 0: three
+  // MMAs of N = n_mma into one accumulator.
+  const uint32_t kAcol = 2 * acc_cols;
+  auto B_st = [&](int s, int p) { return smem + s * stage_bytes + p * bpiece; };
+  auto bits_st = [&](int s) { return smem + s * stage_bytes + 3 * bpiece; };
 
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
       mbar_init(&full[s], 1);
+      mbar_init(&conv[s], 128);
       mbar_init(&empty[s], 1);
     }
     for (int b = 0; b < 2; ++b) {
@@ -99,7 +147,7 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
   if (warp == 2) {
     asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
                      smem_u32(tmem_slot)),
-                 "n"(256));
+                 "n"(512));
     asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
   }
   tc_fence_before();
@@ -107,32 +155,50 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
 
+  // Every role walks the same stage sequence with (s, ph) counters (no
+  // divisions on the single-thread issue paths).
   if (warp == 0) {
     if (lane == 0) {
-      const uint32_t bytes = 16384 + 3 * bpiece;
-      uint32_t kc = 0;
+      int s = 0;
+      uint32_t ph = 0, kc = 0;
       for (int t = blockIdx.x; t < total; t += gridDim.x) {
         const int item = t / tiles_n;
         const int n0 = (t % tiles_n) * 128;
-        const int tb = item_tb[item], te = item_tb[item + 1];
-        for (int tile = tb; tile < te; ++tile) {
+        const int tb = item_tb[item], T = item_tb[item + 1] - tb;
+        // items start at a per-item rotation of their tile run, so that the
+        // CTAs working on neighbouring row blocks (whose tiles share column
+        // blocks) do not all read the same B panel lines at once
+        int ti = (int)(((unsigned)item * 2654435761u) % (unsigned)max(T, 1));
+        for (int i = 0; i < T; ++i) {
+          const int tile = tb + ti;
+          if (++ti == T) ti = 0;
           const int kcol = tile_cb[tile] * TK;
-          for (int h = 0; h < TK / SK; ++h, ++kc) {
-            const int s = kc % S;
-            if (kc >= (uint32_t)S) mbar_wait(&empty[s], ((kc / S) - 1) & 1);
-            mbar_expect_tx(&full[s], bytes);
-            tma_load_2d(A_st(s), &tmA, &full[s], h * SK, tile * TK);
-            tma_load_2d(B_st(s, 0), &tmB0, &full[s], kcol + h * SK, n0);
-            tma_load_2d(B_st(s, 1), &tmB1, &full[s], kcol + h * SK, n0);
-            tma_load_2d(B_st(s, 2), &tmB2, &full[s], kcol + h * SK, n0);
+#pragma unroll
+          for (int h = 0; h < TK / SK; ++h) {
+            if (kc >= (uint32_t)S) mbar_wait(&empty[s], ph ^ 1);
+            mbar_expect_tx(&full[s], (dbg & 4 ? 0 : 3 * bpiece) + (dbg & 8 ? 0 : 1024));
+            if (!(dbg & 8)) bulk_load(bits_st(s), bits + ((int64_t)tile * 2 + h) * TK, 1024, &full[s]);
+            if (!(dbg & 4)) {
+              tma_load_2d(B_st(s, 0), &tmB0, &full[s], kcol + h * SK, n0);
+              tma_load_2d(B_st(s, 1), &tmB1, &full[s], kcol + h * SK, n0);
+              tma_load_2d(B_st(s, 2), &tmB2, &full[s], kcol + h * SK, n0);
+            }
+            ++kc;
+            if (++s == S) { s = 0; ph ^= 1; }
           }
         }
       }
     }
   } else if (warp == 1) {
     if (lane == 0) {
-      const uint32_t idesc = idesc_bf16(n_mma);
-      uint32_t kc = 0;
+      const uint32_t idesc = idesc_bf16(R ? 3 * n_mma : n_mma);
+      // descriptors advance linearly: +stage_bytes per stage, +bpiece per
+      // piece, +32 B per k16 step (start address field in 16-byte units)
+      const uint64_t bd0 = sdesc(smem_u32(B_st(0, 0)), 16, 1024);
+      const uint32_t st16 = (uint32_t)stage_bytes >> 4, pc16 = (uint32_t)bpiece >> 4;
+      const uint32_t rho_step = 3u * n_mma, rho_end = (uint32_t)R * rho_step;
+      int s = 0;
+      uint32_t ph = 0;
       int it = 0;
       for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
         const int item = t / tiles_n;
@@ -140,26 +206,67 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
         const int acc = it & 1;
         if (it >= 2) mbar_wait(&tempty[acc], ((it >> 1) - 1) & 1);
         tc_fence_after();
-        const uint32_t d_tmem = tmem_base + acc * 128;
-        for (int st = 0; st < nst; ++st, ++kc) {
-          const int s = kc % S;
-          mbar_wait(&full[s], (kc / S) & 1);
+        const uint32_t d_tmem = tmem_base + acc * acc_cols;
+        uint32_t rho = 0;      // rotating accumulator set offset (R > 0)
+        int g = 0;             // k16 steps issued for this item
+        for (int st = 0; st < nst; ++st) {
+          mbar_wait(&conv[s], ph);
           tc_fence_after();
-          const uint32_t a = smem_u32(A_st(s));
-          const uint32_t b0 = smem_u32(B_st(s, 0)), b1 = smem_u32(B_st(s, 1)), b2 = smem_u32(B_st(s, 2));
+          const uint32_t ta = tmem_base + kAcol + s * 32;
+          const uint64_t bd = bd0 + (uint64_t)(s * st16);
+          if (!(dbg & 1)) {
+            if (R) {
 #pragma unroll
-          for (int j = 0; j < SK / 16; ++j) {   // k16 steps: 32 bytes along the swizzled row
-            const uint64_t da = sdesc(a + j * 32, 16, 1024);
-            tc_mma_f16(d_tmem, da, sdesc(b0 + j * 32, 16, 1024), idesc, (st > 0 || j > 0) ? 1u : 0u);
-            tc_mma_f16(d_tmem, da, sdesc(b1 + j * 32, 16, 1024), idesc, 1u);
-            tc_mma_f16(d_tmem, da, sdesc(b2 + j * 32, 16, 1024), idesc, 1u);
+              for (int j = 0; j < SK / 16; ++j, ++g) {
+                tc_mma_f16_ts(d_tmem + rho, ta + j * 8, bd + 2 * j, idesc, g >= R ? 1u : 0u);
+                rho += rho_step;
+                if (rho == rho_end) rho = 0;
+              }
+            } else {
+#pragma unroll
+              for (int j = 0; j < SK / 16; ++j) {   // 16 bf16 = 8 packed A columns, 32 B of B rows
+                tc_mma_f16_ts(d_tmem, ta + j * 8, bd + 2 * j, idesc, (st > 0 || j > 0) ? 1u : 0u);
+                tc_mma_f16_ts(d_tmem, ta + j * 8, bd + pc16 + 2 * j, idesc, 1u);
+                tc_mma_f16_ts(d_tmem, ta + j * 8, bd + 2 * pc16 + 2 * j, idesc, 1u);
+              }
+            }
           }
           tc_commit(&empty[s]);
+          if (++s == S) { s = 0; ph ^= 1; }
         }
         tc_commit(&tfull[acc]);
       }
     }
-  } else if (warp >= 4) {
+  } else if (warp >= 4 && warp < 8) {
+    // expander: row r of the stage's A half-tile from its 64 bits → 64 bf16
+    // (0 / 1), two per 32-bit TMEM column, stored to TMEM lane r (the warp's
+    // lane quadrant), so the MMAs read A from TMEM and only B from smem.
+    const int r = threadIdx.x - 128;
+    const uint32_t lane_off = (uint32_t)((warp & 3) * 32) << 16;
+    int s = 0;
+    uint32_t ph = 0;
+    for (int t = blockIdx.x; t < total; t += gridDim.x) {
+      const int item = t / tiles_n;
+      const int nst = (item_tb[item + 1] - item_tb[item]) * (TK / SK);
+      for (int st = 0; st < nst; ++st) {
+        mbar_wait(&full[s], ph);
+        const uint2 b = reinterpret_cast<const uint2*>(bits_st(s))[r];
+        uint32_t v[32];
+#pragma unroll
+        for (int i = 0; i < 8; ++i) {   // one table lookup per byte of the row's bits
+          const uint4 e = lut[((i < 4 ? b.x : b.y) >> (8 * (i & 3))) & 0xFFu];
+          v[4 * i] = e.x; v[4 * i + 1] = e.y; v[4 * i + 2] = e.z; v[4 * i + 3] = e.w;
+        }
+        if (!(dbg & 2)) {
+          tmem_st32u(tmem_base + lane_off + kAcol + s * 32, v);
+          asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+        }
+        tc_fence_before();
+        mbar_arrive(&conv[s]);
+        if (++s == S) { s = 0; ph ^= 1; }
+      }
+    }
+  } else if (warp >= 8) {
     const int q = warp & 3;
     int it = 0;
     for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
@@ -171,14 +278,29 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
       float* prow = part + ((int64_t)item * TK + q * 32 + lane) * ldp + n0;
       for (int c0 = 0; c0 < n_mma; c0 += 32) {
         if (n0 + c0 >= w) break;
-        uint32_t r[32];
-        tmem_ld32(tmem_base + acc * 128 + ((uint32_t)(q * 32) << 16) + (uint32_t)c0, r);
+        uint32_t rr[32];
+        const uint32_t a0 = tmem_base + acc * acc_cols + ((uint32_t)(q * 32) << 16) + (uint32_t)c0;
+        if (R) {   // fixed order: lo, mid, hi pieces, each over its rotations
+          float sum[32];
+#pragma unroll
+          for (int i = 0; i < 32; ++i) sum[i] = 0.f;
+          for (int pc = 2; pc >= 0; --pc)
+            for (int rho = 0; rho < R; ++rho) {
+              tmem_ld32(a0 + (uint32_t)((rho * 3 + pc) * n_mma), rr);
+#pragma unroll
+              for (int i = 0; i < 32; ++i) sum[i] += __uint_as_float(rr[i]);
+            }
+#pragma unroll
+          for (int i = 0; i < 32; ++i) rr[i] = __float_as_uint(sum[i]);
+        } else {
+          tmem_ld32(a0, rr);
+        }
 #pragma unroll
         for (int i = 0; i < 32; i += 4)
           if (n0 + c0 + i < w)
             *reinterpret_cast<float4*>(prow + c0 + i) =
-                make_float4(__uint_as_float(r[i]), __uint_as_float(r[i + 1]), __uint_as_float(r[i + 2]),
-                            __uint_as_float(r[i + 3]));
+                make_float4(__uint_as_float(rr[i]), __uint_as_float(rr[i + 1]), __uint_as_float(rr[i + 2]),
+                            __uint_as_float(rr[i + 3]));
       }
       tc_fence_before();
       mbar_arrive(&tempty[acc]);
@@ -187,7 +309,7 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__
   tc_fence_before();
   __syncthreads();
   if (warp == 2) {
-    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "n"(256));
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "n"(512));
   }
 }
 
@@ -251,13 +373,13 @@ CUtensorMap bf16_map(const void* base, int64_t inner, int64_t outer, int64_t ld,
   return m;
 }
 
-// Per-call cost model (B200, calibrated against profiles/r1_core_experiment.md
-// and the hub-tile timings): a CSR entry costs ≈ 24 ps·(w/128)^0.55 (L2-gather
-// bound), a tile ≈ ceil(w/128)·(4 + 6·min(w,128)/128) ns (A-tile stream +
-// 3 bf16 MMAs), plus ≈ 20 µs of fixed per-call cost.
+// Per-call cost model (B200, calibrated on the Reddit-shaped graph,
+// profiles/r1_hub_tiles_reddit.txt): a CSR entry costs ≈ 24 ps·(w/128)^0.55
+// (L2-gather bound), a tile ≈ ceil(w/128)·(4.5 + 5.2·min(w,128)/128) ns (bit
+// expansion + 3 bf16 MMA pieces per 128-wide chunk), plus ≈ 20 µs per call.
 double csr_entry_s(int64_t w) { return 24e-12 * std::pow((double)w / 128.0, 0.55); }
 double tile_s(int64_t w) {
-  return (double)ceil_div(w, 128) * (4e-9 + 6e-9 * (double)std::min<int64_t>(w, 128) / 128.0);
+  return (double)ceil_div(w, 128) * (4.5e-9 + 5.2e-9 * (double)std::min<int64_t>(w, 128) / 128.0);
 }
 }  // namespace
 
@@ -277,18 +399,23 @@ void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx,
   RDM_LAUNCHED(ctx);
   const int n_mma = (int)std::min<int64_t>(128, ((w + 15) / 16) * 16);
   const int tiles_n = (int)ceil_div(w, 128);
-  const CUtensorMap ta = bf16_map(c.tiles->ptr, TK, c.n_tiles * TK, TK, TK);
   const CUtensorMap b0 = bf16_map(pan, K2, w, K2, n_mma);
   const CUtensorMap b1 = bf16_map(pan + w * K2, K2, w, K2, n_mma);
   const CUtensorMap b2 = bf16_map(pan + 2 * w * K2, K2, w, K2, n_mma);
-  const int stage_bytes = 16384 + 3 * n_mma * 128;
-  const int S = std::min(8, (kSmemBudget - 1024 - 256) / stage_bytes);
-  const int smem = S * stage_bytes + 1024 + 256;
+  const int stage_bytes = 3 * n_mma * 128 + 1024;
+  int R = n_mma <= 64 ? (n_mma <= 16 ? 2 : 1) : 0;
+  if (const char* e = getenv("RDM_TILE_R")) R = n_mma <= 64 ? std::max(0, std::min(4, atoi(e))) : 0;
+  const int acc_cols = (int)((R ? R * 3 * n_mma : n_mma) + 31) / 32 * 32;
+  const int S = std::min({8, (kSmemBudget - 1024 - 1024 - 4096) / stage_bytes, (512 - 2 * acc_cols) / 32});
+  RDM_CHECK_ARG(S >= 2, "hub tiles: TMEM/smem budget");
+  const int smem = S * stage_bytes + 1024 + 1024 + 4096;   // stages, align, barriers, LUT
   RDM_CUDA(cudaFuncSetAttribute(hub_tile_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
   const int64_t total = c.n_items * tiles_n;
   const unsigned grid = (unsigned)std::min<int64_t>(total, ctx->num_sms);
-  hub_tile_kernel<<<grid, 256, smem, ctx->stream>>>(ta, b0, b1, b2, c.tile_cb->as<int32_t>(), c.item_tb->as<int32_t>(),
-                                                   (int)c.n_items, tiles_n, n_mma, w, part, ldp, S, stage_bytes);
+  hub_tile_kernel<<<grid, 384, smem, ctx->stream>>>(b0, b1, b2, c.tiles->as<uint64_t>(), c.tile_cb->as<int32_t>(),
+                                                   c.item_tb->as<int32_t>(),
+                                                   (int)c.n_items, tiles_n, n_mma, w, part, ldp, S, stage_bytes, R, acc_cols,
+                                                   getenv("RDM_TILE_DBG") ? atoi(getenv("RDM_TILE_DBG")) : 0);
   RDM_LAUNCHED(ctx);
 }
 
@@ -384,50 +511,48 @@ bool build_hub_tiles(rdm_ctx* ctx, Csr& A, const int64_t* rp, const int32_t* col
   rb_item[c.n_rb] = (int32_t)item_tb.size();
   c.n_items = (int64_t)item_tb.size();
   item_tb.push_back((int32_t)n_tiles);
-  // tiles (bf16 0/1, filled one row block at a time) and the residual CSR
-  c.tiles.reset(new DevBuf((size_t)n_tiles * TK * TK * 2));
-  std::vector<int64_t> rrp(n + 1, 0);
-  auto in_tile = [&](int64_t ri, int64_t rj) {
-    return ri < K2 && rj < K2 && tile_id[(size_t)(ri / TK) * nrb + rj / TK] >= 0;
-  };
-  std::vector<uint16_t> buf;
+  // tiles as bits (bits[tile][half][row] = u64, bit kk = column half·64 + kk),
+  // filled one row block at a time; an entry whose cell is already set (a
+  // duplicate (i, j) in the CSR) stays in the residual CSR.
+  c.tiles.reset(new DevBuf((size_t)n_tiles * TK * TK / 8));
+  std::vector<uint8_t> tin(nnz, 0);
+  std::vector<uint64_t> buf;
   for (int64_t rb = 0; rb < c.n_rb; ++rb) {
     const int64_t t0 = rb_first[rb], T = rb_first[rb + 1] - t0;
     if (!T) continue;
-    buf.assign((size_t)T * TK * TK, 0);
+    buf.assign((size_t)T * 2 * TK, 0);
     for (int64_t r = 0; r < TK; ++r) {
       const int64_t v = order[rb * TK + r];
       for (int64_t j = rp[v]; j < rp[v + 1]; ++j) {
         const int64_t rj = rank[col[j]];
-        if (!in_tile(rb * TK + r, rj)) continue;
-        const int64_t t = tile_id[(size_t)rb * nrb + rj / TK] - t0;
-        uint16_t& e = buf[(size_t)t * TK * TK + r * TK + (rj % TK)];
-        float f = 0.f;
-        if (e) {
-          uint32_t u = (uint32_t)e << 16;
-          std::memcpy(&f, &u, 4);
-        }
-        f += 1.f;   // duplicate entries add up (small integers are exact in bf16)
-        uint32_t u;
-        std::memcpy(&u, &f, 4);
-        e = (uint16_t)(u >> 16);
+        if (rj >= K2) continue;
+        const int64_t id = tile_id[(size_t)rb * nrb + rj / TK];
+        if (id < 0) continue;
+        const int64_t cc = rj % TK;
+        uint64_t& word = buf[(size_t)(id - t0) * 2 * TK + (cc / SK) * TK + r];
+        const uint64_t bit = 1ull << (cc % SK);
+        if (word & bit) continue;
+        word |= bit;
+        tin[j] = 1;
       }
     }
-    RDM_CUDA(cudaMemcpy(c.tiles->as<uint8_t>() + (size_t)t0 * TK * TK * 2, buf.data(), buf.size() * 2,
+    RDM_CUDA(cudaMemcpy(c.tiles->as<uint64_t>() + (size_t)t0 * 2 * TK, buf.data(), buf.size() * 8,
                         cudaMemcpyHostToDevice));
   }
+  std::vector<int64_t> rrp(n + 1, 0);
   for (int64_t i = 0; i < n; ++i) {
     int64_t keep = 0;
-    for (int64_t j = rp[i]; j < rp[i + 1]; ++j) keep += !in_tile(rank[i], rank[col[j]]);
+    for (int64_t j = rp[i]; j < rp[i + 1]; ++j) keep += !tin[j];
     rrp[i + 1] = rrp[i] + keep;
   }
   const int64_t rnnz = rrp[n];
+  c.nnz = nnz - rnnz;
   std::vector<int32_t> rcol(std::max<int64_t>(rnnz, 1));
   std::vector<float> rval(std::max<int64_t>(rnnz, 1));
   for (int64_t i = 0; i < n; ++i) {
     int64_t o = rrp[i];
     for (int64_t j = rp[i]; j < rp[i + 1]; ++j)
-      if (!in_tile(rank[i], rank[col[j]])) {
+      if (!tin[j]) {
         rcol[o] = col[j];
         rval[o] = val[j];
         ++o;

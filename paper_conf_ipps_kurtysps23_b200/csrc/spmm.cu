@@ -171,8 +171,12 @@ __device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
 // One warp per work item: items [0, n_seg) are heavy-row segments (partial
 // rows to `part`), items [n_seg, n_seg + n_light) are light rows (to out).
 // blockIdx.y selects a 128-column chunk of the slice.
+// Resident CTAs per SM: the gathers are latency-bound, so occupancy is capped
+// by registers only as far as the V accumulators need (measured on the
+// Reddit-shaped residual CSR: V = 4 best at 4 CTAs, V = 3 at 5, V ≤ 2 at 6).
+constexpr int spmm_minb(int V) { return V >= 4 ? 4 : V == 3 ? 5 : 6; }
 template <int G, int V>
-__global__ void __launch_bounds__(kWarps * 32)
+__global__ void __launch_bounds__(kWarps * 32, spmm_minb(V))
 spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
             const float* __restrict__ val, const int32_t* __restrict__ light_rows,
             const int64_t* __restrict__ seg_start, const int32_t* __restrict__ seg_row,
