@@ -76,6 +76,15 @@ __device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t b
       : "memory");
 }
 
+__device__ __forceinline__ void tma_load_4d(void* dst, const CUtensorMap* map, uint64_t* bar, int c0, int c1,
+                                            int c2, int c3) {
+  asm volatile(
+      "cp.async.bulk.tensor.4d.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1, {%3, %4, %5, %6}], [%2];" ::"r"(
+          smem_u32(dst)),
+      "l"((uint64_t)map), "r"(smem_u32(bar)), "r"(c0), "r"(c1), "r"(c2), "r"(c3)
+      : "memory");
+}
+
 // kind::f16 MMA with A from TMEM (bf16 pairs packed in 32-bit columns).
 __device__ __forceinline__ void tc_mma_f16_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t idesc,
                                               uint32_t accumulate) {
@@ -102,41 +111,58 @@ __device__ __forceinline__ uint32_t bits2_bf16(uint32_t b) {
   return ((b & 1u) * 0x3F80u) | (((b >> 1) & 1u) * 0x3F800000u);
 }
 
+// Launch shape of one product (host-computed).
+struct TileShape {
+  int n_items, tiles_n, n_mma;
+  int64_t w, ldp;
+  int S, SA;          // shared-memory stages, TMEM A slots
+  int HS;             // 64-wide k halves per stage (1 or 2)
+  int stage_bytes;    // HS · (3 · n_mma · 128 + 1024)
+  int R;              // > 0: concatenated-piece MMAs with R rotating accumulator sets
+  int acc_cols;       // TMEM columns per accumulator buffer
+  int dbg;            // timing experiments (RDM_TILE_DBG): 1 = skip the MMAs
+};
+
+template <int HS>
 __global__ void __launch_bounds__(384, 1)
-hub_tile_kernel(const __grid_constant__ CUtensorMap tmB0, const __grid_constant__ CUtensorMap tmB1,
-                const __grid_constant__ CUtensorMap tmB2, const uint64_t* __restrict__ bits,
-                const int32_t* __restrict__ tile_cb, const int32_t* __restrict__ item_tb, int n_items,
-                int tiles_n, int n_mma, int64_t w, float* __restrict__ part, int64_t ldp, int S,
-                int stage_bytes, int R, int acc_cols, int dbg) {
+hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__ CUtensorMap tmB2d,
+                const uint64_t* __restrict__ bits,
+                const int32_t* __restrict__ tile_cb, const int32_t* __restrict__ item_tb,
+                float* __restrict__ part, const TileShape sh) {
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
-  uint64_t* full = (uint64_t*)(smem + S * stage_bytes);
-  uint64_t* conv = full + S;
-  uint64_t* empty = conv + S;
-  uint64_t* tfull = empty + S;   // [2]
+  const int S = sh.S, SA = sh.SA, R = sh.R, n_mma = sh.n_mma;
+  uint64_t* full = (uint64_t*)(smem + S * sh.stage_bytes);
+  uint64_t* empty = full + S;
+  uint64_t* conv = empty + S;    // [SA] TMEM A slot expanded
+  uint64_t* aempty = conv + SA;  // [SA] TMEM A slot consumed by its MMAs
+  uint64_t* tfull = aempty + SA; // [2]
   uint64_t* tempty = tfull + 2;  // [2]
   uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
-  uint4* lut = (uint4*)(smem + S * stage_bytes + 1024);   // byte → 8 bf16 (0 / 1)
+  uint4* lut = (uint4*)(smem + S * sh.stage_bytes + 1024);   // byte → 8 bf16 (0 / 1)
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
-  const int total = n_items * tiles_n;
+  const int total = sh.n_items * sh.tiles_n;
   for (int i = threadIdx.x; i < 256; i += blockDim.x)
     lut[i] = make_uint4(bits2_bf16(i), bits2_bf16(i >> 2), bits2_bf16(i >> 4), bits2_bf16(i >> 6));
-  const int bpiece = n_mma * 128;                 // bytes of one B piece per stage
-  // stage: three B pieces | the half-tile's bits.  TMEM: two accumulator
-  // buffers of acc_cols columns, then the A ring (stage s at kAcol + 32 s, 64
-  // bf16 per row packed in pairs).  R > 0 ("concatenated" mode, n_mma ≤ 64):
-  // one MMA of N = 3 n_mma covers the three pieces (adjacent in smem) and
-  // k16 steps rotate over R accumulator sets [rho][piece][n_mma]; R = 0: three
-  // MMAs of N = n_mma into one accumulator.
-  const uint32_t kAcol = 2 * acc_cols;
-  auto B_st = [&](int s, int p) { return smem + s * stage_bytes + p * bpiece; };
-  auto bits_st = [&](int s) { return smem + s * stage_bytes + 3 * bpiece; };
+  // Two rings.  Shared-memory stage s: the B pieces of HS k-halves as
+  // [half][piece][n_mma][64 bf16] (one 4-D TMA; pieces of a half adjacent, so
+  // a concatenated MMA of N = 3 n_mma reads all three), then the halves' bits
+  // [half][128 rows] u64.  TMEM: two accumulator buffers of acc_cols columns,
+  // then SA A slots of 32·HS columns (64·HS bf16 per row, packed in pairs).
+  const int bpiece = n_mma * 128;                 // bytes of one piece of one half
+  const int bbytes = HS * 3 * bpiece;
+  const uint32_t kAcol = 2 * sh.acc_cols;
+  auto B_st = [&](int s) { return smem + s * sh.stage_bytes; };
+  auto bits_st = [&](int s) { return smem + s * sh.stage_bytes + bbytes; };
 
   if (threadIdx.x == 0) {
-    for (int s = 0; s < S; ++s) {
-      mbar_init(&full[s], 1);
-      mbar_init(&conv[s], 128);
-      mbar_init(&empty[s], 1);
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&empty[i], 1);
+    }
+    for (int i = 0; i < SA; ++i) {
+      mbar_init(&conv[i], 128);
+      mbar_init(&aempty[i], 1);
     }
     for (int b = 0; b < 2; ++b) {
       mbar_init(&tfull[b], 1);
@@ -154,16 +180,18 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB0, const __grid_constant_
   __syncthreads();
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
+  const int spt = (TK / SK) / HS;                 // stages per tile
 
-  // Every role walks the same stage sequence with (s, ph) counters (no
+  // Every role walks the same stage sequence with (slot, phase) counters (no
   // divisions on the single-thread issue paths).
   if (warp == 0) {
     if (lane == 0) {
       int s = 0;
       uint32_t ph = 0, kc = 0;
+      const uint32_t bytes = (uint32_t)bbytes + HS * 1024;
       for (int t = blockIdx.x; t < total; t += gridDim.x) {
-        const int item = t / tiles_n;
-        const int n0 = (t % tiles_n) * 128;
+        const int item = t / sh.tiles_n;
+        const int n0 = (t % sh.tiles_n) * 128;
         const int tb = item_tb[item], T = item_tb[item + 1] - tb;
         // items start at a per-item rotation of their tile run, so that the
         // CTAs working on neighbouring row blocks (whose tiles share column
@@ -172,16 +200,16 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB0, const __grid_constant_
         for (int i = 0; i < T; ++i) {
           const int tile = tb + ti;
           if (++ti == T) ti = 0;
-          const int kcol = tile_cb[tile] * TK;
-#pragma unroll
-          for (int h = 0; h < TK / SK; ++h) {
+          const int kb = tile_cb[tile] * (TK / SK);   // first 64-wide k block of the tile
+          for (int h = 0; h < spt; ++h) {
             if (kc >= (uint32_t)S) mbar_wait(&empty[s], ph ^ 1);
-            mbar_expect_tx(&full[s], (dbg & 4 ? 0 : 3 * bpiece) + (dbg & 8 ? 0 : 1024));
-            if (!(dbg & 8)) bulk_load(bits_st(s), bits + ((int64_t)tile * 2 + h) * TK, 1024, &full[s]);
-            if (!(dbg & 4)) {
-              tma_load_2d(B_st(s, 0), &tmB0, &full[s], kcol + h * SK, n0);
-              tma_load_2d(B_st(s, 1), &tmB1, &full[s], kcol + h * SK, n0);
-              tma_load_2d(B_st(s, 2), &tmB2, &full[s], kcol + h * SK, n0);
+            mbar_expect_tx(&full[s], bytes);
+            bulk_load(bits_st(s), bits + ((int64_t)tile * 2 + h * HS) * TK, HS * 1024, &full[s]);
+            if (HS == 2) {
+              tma_load_4d(B_st(s), &tmB, &full[s], 0, n0, 0, kb);
+            } else {   // three 2-D boxes from the stacked panels (measured faster for one half)
+              for (int pc = 0; pc < 3; ++pc)
+                tma_load_2d(B_st(s) + pc * bpiece, &tmB2d, &full[s], (kb + h) * SK, pc * (int)sh.w + n0);
             }
             ++kc;
             if (++s == S) { s = 0; ph ^= 1; }
@@ -192,94 +220,107 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB0, const __grid_constant_
   } else if (warp == 1) {
     if (lane == 0) {
       const uint32_t idesc = idesc_bf16(R ? 3 * n_mma : n_mma);
-      // descriptors advance linearly: +stage_bytes per stage, +bpiece per
-      // piece, +32 B per k16 step (start address field in 16-byte units)
-      const uint64_t bd0 = sdesc(smem_u32(B_st(0, 0)), 16, 1024);
-      const uint32_t st16 = (uint32_t)stage_bytes >> 4, pc16 = (uint32_t)bpiece >> 4;
+      // descriptors advance linearly: +stage_bytes per stage, +3·bpiece per
+      // k half, +bpiece per piece, +32 B per k16 step (16-byte units)
+      const uint64_t bd0 = sdesc(smem_u32(B_st(0)), 16, 1024);
+      const uint32_t st16 = (uint32_t)sh.stage_bytes >> 4, pc16 = (uint32_t)bpiece >> 4;
       const uint32_t rho_step = 3u * n_mma, rho_end = (uint32_t)R * rho_step;
-      int s = 0;
-      uint32_t ph = 0;
+      int s = 0, a = 0;
+      uint32_t ph = 0, aph = 0;
       int it = 0;
       for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
-        const int item = t / tiles_n;
-        const int nst = (item_tb[item + 1] - item_tb[item]) * (TK / SK);
+        const int item = t / sh.tiles_n;
+        const int nst = (item_tb[item + 1] - item_tb[item]) * spt;
         const int acc = it & 1;
         if (it >= 2) mbar_wait(&tempty[acc], ((it >> 1) - 1) & 1);
         tc_fence_after();
-        const uint32_t d_tmem = tmem_base + acc * acc_cols;
+        const uint32_t d_tmem = tmem_base + acc * sh.acc_cols;
         uint32_t rho = 0;      // rotating accumulator set offset (R > 0)
         int g = 0;             // k16 steps issued for this item
         for (int st = 0; st < nst; ++st) {
-          mbar_wait(&conv[s], ph);
+          mbar_wait(&conv[a], aph);
           tc_fence_after();
-          const uint32_t ta = tmem_base + kAcol + s * 32;
+          const uint32_t ta = tmem_base + kAcol + a * 32 * HS;
           const uint64_t bd = bd0 + (uint64_t)(s * st16);
-          if (!(dbg & 1)) {
-            if (R) {
+          if (!(sh.dbg & 1)) {
 #pragma unroll
-              for (int j = 0; j < SK / 16; ++j, ++g) {
-                tc_mma_f16_ts(d_tmem + rho, ta + j * 8, bd + 2 * j, idesc, g >= R ? 1u : 0u);
-                rho += rho_step;
-                if (rho == rho_end) rho = 0;
-              }
-            } else {
+            for (int h = 0; h < HS; ++h) {
+              const uint64_t bh = bd + (uint64_t)(h * 3 * pc16);
+              const uint32_t th = ta + h * 32;
+              if (R) {
 #pragma unroll
-              for (int j = 0; j < SK / 16; ++j) {   // 16 bf16 = 8 packed A columns, 32 B of B rows
-                tc_mma_f16_ts(d_tmem, ta + j * 8, bd + 2 * j, idesc, (st > 0 || j > 0) ? 1u : 0u);
-                tc_mma_f16_ts(d_tmem, ta + j * 8, bd + pc16 + 2 * j, idesc, 1u);
-                tc_mma_f16_ts(d_tmem, ta + j * 8, bd + 2 * pc16 + 2 * j, idesc, 1u);
+                for (int j = 0; j < SK / 16; ++j, ++g) {
+                  tc_mma_f16_ts(d_tmem + rho, th + j * 8, bh + 2 * j, idesc, g >= R ? 1u : 0u);
+                  rho += rho_step;
+                  if (rho == rho_end) rho = 0;
+                }
+              } else {
+#pragma unroll
+                for (int j = 0; j < SK / 16; ++j, ++g) {   // 8 packed A columns, 32 B of B rows per k16
+                  tc_mma_f16_ts(d_tmem, th + j * 8, bh + 2 * j, idesc, g > 0 ? 1u : 0u);
+                  tc_mma_f16_ts(d_tmem, th + j * 8, bh + pc16 + 2 * j, idesc, 1u);
+                  tc_mma_f16_ts(d_tmem, th + j * 8, bh + 2 * pc16 + 2 * j, idesc, 1u);
+                }
               }
             }
           }
           tc_commit(&empty[s]);
+          tc_commit(&aempty[a]);
           if (++s == S) { s = 0; ph ^= 1; }
+          if (++a == SA) { a = 0; aph ^= 1; }
         }
         tc_commit(&tfull[acc]);
       }
     }
   } else if (warp >= 4 && warp < 8) {
-    // expander: row r of the stage's A half-tile from its 64 bits → 64 bf16
-    // (0 / 1), two per 32-bit TMEM column, stored to TMEM lane r (the warp's
-    // lane quadrant), so the MMAs read A from TMEM and only B from smem.
+    // expander: row r of the stage's A tile part from its bits → bf16 0 / 1
+    // (one table lookup per byte), two per 32-bit TMEM column, stored to TMEM
+    // lane r (the warp's lane quadrant): the MMAs read A from TMEM.
     const int r = threadIdx.x - 128;
     const uint32_t lane_off = (uint32_t)((warp & 3) * 32) << 16;
-    int s = 0;
-    uint32_t ph = 0;
+    int s = 0, a = 0;
+    uint32_t ph = 0, aph = 0, kc = 0;
     for (int t = blockIdx.x; t < total; t += gridDim.x) {
-      const int item = t / tiles_n;
-      const int nst = (item_tb[item + 1] - item_tb[item]) * (TK / SK);
-      for (int st = 0; st < nst; ++st) {
+      const int item = t / sh.tiles_n;
+      const int nst = (item_tb[item + 1] - item_tb[item]) * spt;
+      for (int st = 0; st < nst; ++st, ++kc) {
         mbar_wait(&full[s], ph);
-        const uint2 b = reinterpret_cast<const uint2*>(bits_st(s))[r];
-        uint32_t v[32];
+        if (kc >= (uint32_t)SA) {
+          mbar_wait(&aempty[a], aph ^ 1);
+          tc_fence_after();
+        }
 #pragma unroll
-        for (int i = 0; i < 8; ++i) {   // one table lookup per byte of the row's bits
-          const uint4 e = lut[((i < 4 ? b.x : b.y) >> (8 * (i & 3))) & 0xFFu];
-          v[4 * i] = e.x; v[4 * i + 1] = e.y; v[4 * i + 2] = e.z; v[4 * i + 3] = e.w;
+        for (int h = 0; h < HS; ++h) {
+          const uint2 b = reinterpret_cast<const uint2*>(bits_st(s) + h * 1024)[r];
+          uint32_t v[32];
+#pragma unroll
+          for (int i = 0; i < 8; ++i) {
+            const uint4 e = lut[((i < 4 ? b.x : b.y) >> (8 * (i & 3))) & 0xFFu];
+            v[4 * i] = e.x; v[4 * i + 1] = e.y; v[4 * i + 2] = e.z; v[4 * i + 3] = e.w;
+          }
+          tmem_st32u(tmem_base + lane_off + kAcol + a * 32 * HS + h * 32, v);
         }
-        if (!(dbg & 2)) {
-          tmem_st32u(tmem_base + lane_off + kAcol + s * 32, v);
-          asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
-        }
+        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
         tc_fence_before();
-        mbar_arrive(&conv[s]);
+        mbar_arrive(&conv[a]);
         if (++s == S) { s = 0; ph ^= 1; }
+        if (++a == SA) { a = 0; aph ^= 1; }
       }
     }
   } else if (warp >= 8) {
     const int q = warp & 3;
     int it = 0;
     for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
-      const int item = t / tiles_n;
-      const int64_t n0 = (int64_t)(t % tiles_n) * 128;
+      const int item = t / sh.tiles_n;
+      const int64_t n0 = (int64_t)(t % sh.tiles_n) * 128;
       const int acc = it & 1;
       mbar_wait_sleep(&tfull[acc], (it >> 1) & 1);
       tc_fence_after();
-      float* prow = part + ((int64_t)item * TK + q * 32 + lane) * ldp + n0;
+      float* prow = part + ((int64_t)item * TK + q * 32 + lane) * sh.ldp + n0;
       for (int c0 = 0; c0 < n_mma; c0 += 32) {
-        if (n0 + c0 >= w) break;
+        if (n0 + c0 >= sh.w) break;
         uint32_t rr[32];
-        const uint32_t a0 = tmem_base + acc * acc_cols + ((uint32_t)(q * 32) << 16) + (uint32_t)c0;
+        const uint32_t a0 = tmem_base + acc * sh.acc_cols + ((uint32_t)(q * 32) << 16) + (uint32_t)c0;
         if (R) {   // fixed order: lo, mid, hi pieces, each over its rotations
           float sum[32];
 #pragma unroll
@@ -297,7 +338,7 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB0, const __grid_constant_
         }
 #pragma unroll
         for (int i = 0; i < 32; i += 4)
-          if (n0 + c0 + i < w)
+          if (n0 + c0 + i < sh.w)
             *reinterpret_cast<float4*>(prow + c0 + i) =
                 make_float4(__uint_as_float(rr[i]), __uint_as_float(rr[i + 1]), __uint_as_float(rr[i + 2]),
                             __uint_as_float(rr[i + 3]));
@@ -358,18 +399,33 @@ PFN_cuTensorMapEncodeTiled_v12000 encode() {
   return fn;
 }
 
-// 2-D bf16 map: inner (contiguous) x outer, row stride ld elements, box
-// {64, box_outer}, 128-byte swizzle, out-of-bounds rows read as zeros.
-CUtensorMap bf16_map(const void* base, int64_t inner, int64_t outer, int64_t ld, int box_outer) {
+// 4-D bf16 map over the three B panels P_p[n][k] (row length K2, panel p at
+// p·w·K2): dims {64 (k within a 128-byte swizzle row), n, piece, k / 64}, box
+// {64, n_mma, 3, HS}, so that one TMA lands [half][piece][n_mma][64] in smem
+// with the 128-byte swizzle; rows n ≥ w read as zeros.
+CUtensorMap panel_map(const void* base, int64_t K2, int64_t w, int n_mma, int HS) {
   CUtensorMap m;
-  cuuint64_t dims[2] = {(cuuint64_t)inner, (cuuint64_t)outer};
-  cuuint64_t strides[1] = {(cuuint64_t)(ld * 2)};
-  cuuint32_t box[2] = {(cuuint32_t)SK, (cuuint32_t)box_outer};
+  cuuint64_t dims[4] = {(cuuint64_t)SK, (cuuint64_t)w, 3, (cuuint64_t)(K2 / SK)};
+  cuuint64_t strides[3] = {(cuuint64_t)(K2 * 2), (cuuint64_t)(w * K2 * 2), (cuuint64_t)(SK * 2)};
+  cuuint32_t box[4] = {(cuuint32_t)SK, (cuuint32_t)n_mma, 3, (cuuint32_t)HS};
+  cuuint32_t es[4] = {1, 1, 1, 1};
+  CUresult r = encode()(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(base), dims, strides, box, es,
+                        CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                        CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) throw Error(RDM_ERR_CUDA, "cuTensorMapEncodeTiled (panels) failed (" + std::to_string((int)r) + ")");
+  return m;
+}
+
+CUtensorMap stacked_map(const void* base, int64_t K2, int64_t rows, int n_mma) {
+  CUtensorMap m;
+  cuuint64_t dims[2] = {(cuuint64_t)K2, (cuuint64_t)rows};
+  cuuint64_t strides[1] = {(cuuint64_t)(K2 * 2)};
+  cuuint32_t box[2] = {(cuuint32_t)SK, (cuuint32_t)n_mma};
   cuuint32_t es[2] = {1, 1};
   CUresult r = encode()(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, const_cast<void*>(base), dims, strides, box, es,
                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
                         CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
-  if (r != CUDA_SUCCESS) throw Error(RDM_ERR_CUDA, "cuTensorMapEncodeTiled (bf16) failed (" + std::to_string((int)r) + ")");
+  if (r != CUDA_SUCCESS) throw Error(RDM_ERR_CUDA, "cuTensorMapEncodeTiled (stacked) failed (" + std::to_string((int)r) + ")");
   return m;
 }
 
@@ -397,25 +453,36 @@ void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx,
   tile_panels_kernel<<<pg, dim3(32, 8), 0, ctx->stream>>>(X, ldx, c.hub_ids->as<int32_t>(), c.scale->as<float>(), K2,
                                                         w, pan, pan + w * K2, pan + 2 * w * K2);
   RDM_LAUNCHED(ctx);
-  const int n_mma = (int)std::min<int64_t>(128, ((w + 15) / 16) * 16);
-  const int tiles_n = (int)ceil_div(w, 128);
-  const CUtensorMap b0 = bf16_map(pan, K2, w, K2, n_mma);
-  const CUtensorMap b1 = bf16_map(pan + w * K2, K2, w, K2, n_mma);
-  const CUtensorMap b2 = bf16_map(pan + 2 * w * K2, K2, w, K2, n_mma);
-  const int stage_bytes = 3 * n_mma * 128 + 1024;
-  int R = n_mma <= 64 ? (n_mma <= 16 ? 2 : 1) : 0;
-  if (const char* e = getenv("RDM_TILE_R")) R = n_mma <= 64 ? std::max(0, std::min(4, atoi(e))) : 0;
-  const int acc_cols = (int)((R ? R * 3 * n_mma : n_mma) + 31) / 32 * 32;
-  const int S = std::min({8, (kSmemBudget - 1024 - 1024 - 4096) / stage_bytes, (512 - 2 * acc_cols) / 32});
-  RDM_CHECK_ARG(S >= 2, "hub tiles: TMEM/smem budget");
-  const int smem = S * stage_bytes + 1024 + 1024 + 4096;   // stages, align, barriers, LUT
-  RDM_CUDA(cudaFuncSetAttribute(hub_tile_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-  const int64_t total = c.n_items * tiles_n;
+  TileShape sh;
+  sh.n_mma = (int)std::min<int64_t>(128, ((w + 15) / 16) * 16);
+  sh.tiles_n = (int)ceil_div(w, 128);
+  sh.n_items = (int)c.n_items;
+  sh.w = w;
+  sh.ldp = ldp;
+  sh.R = sh.n_mma <= 64 ? (sh.n_mma <= 16 ? 2 : 1) : 0;
+  if (const char* e = getenv("RDM_TILE_R")) sh.R = sh.n_mma <= 64 ? std::max(0, std::min(4, atoi(e))) : 0;
+  sh.acc_cols = (int)((sh.R ? sh.R * 3 * sh.n_mma : sh.n_mma) + 31) / 32 * 32;
+  // whole tiles per stage when the stage stays small (narrow slices: halves
+  // the per-stage fixed cost), else 64-wide k halves
+  sh.HS = 3 * sh.n_mma * 256 + 2048 <= 50 * 1024 ? 2 : 1;
+  if (const char* e = getenv("RDM_TILE_HS")) sh.HS = atoi(e) == 2 ? 2 : 1;
+  sh.stage_bytes = sh.HS * (3 * sh.n_mma * 128 + 1024);
+  const int avail = kSmemBudget - 1024 - 1024 - 4096;   // align, barriers, LUT
+  sh.S = std::min(32, avail / sh.stage_bytes);
+  sh.SA = std::min(8, (512 - 2 * sh.acc_cols) / (32 * sh.HS));
+  sh.dbg = getenv("RDM_TILE_DBG") ? atoi(getenv("RDM_TILE_DBG")) : 0;
+  RDM_CHECK_ARG(sh.S >= 2 && sh.SA >= 2, "hub tiles: TMEM/smem budget");
+  const CUtensorMap tb = panel_map(pan, K2, w, sh.n_mma, sh.HS);
+  // the three panels stacked as one 3w x K2 matrix: rows past a panel's w
+  // only feed accumulator columns ≥ w, which are never stored
+  const CUtensorMap tb2 = stacked_map(pan, K2, 3 * w, sh.n_mma);
+  const int smem = sh.S * sh.stage_bytes + 1024 + 1024 + 4096;
+  const int64_t total = c.n_items * sh.tiles_n;
   const unsigned grid = (unsigned)std::min<int64_t>(total, ctx->num_sms);
-  hub_tile_kernel<<<grid, 384, smem, ctx->stream>>>(b0, b1, b2, c.tiles->as<uint64_t>(), c.tile_cb->as<int32_t>(),
-                                                   c.item_tb->as<int32_t>(),
-                                                   (int)c.n_items, tiles_n, n_mma, w, part, ldp, S, stage_bytes, R, acc_cols,
-                                                   getenv("RDM_TILE_DBG") ? atoi(getenv("RDM_TILE_DBG")) : 0);
+  auto kern = sh.HS == 2 ? hub_tile_kernel<2> : hub_tile_kernel<1>;
+  RDM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  kern<<<grid, 384, smem, ctx->stream>>>(tb, tb2, c.tiles->as<uint64_t>(), c.tile_cb->as<int32_t>(),
+                                         c.item_tb->as<int32_t>(), part, sh);
   RDM_LAUNCHED(ctx);
 }
 
