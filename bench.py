@@ -29,6 +29,8 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "full-batch GCN epoch ms at 1/2/4/8 B200; SpMM HBM GB/s; all-to-all bus GB/s"
+DTYPES = {"fp32": "f32", "fast": "bf16 SpMM operand + tf32 GEMM, f32 accumulate"}
+GATES = {"fp32": 1e-4, "fast": 2e-2}
 
 
 def parse():
@@ -44,6 +46,11 @@ def parse():
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--transport", default="nccl", choices=["nccl", "p2p"],
                     help="redistribution transport for N > 1 (rdm.h rdm_set_transport)")
+    ap.add_argument("--precision", default="fp32", choices=["fp32", "fast"],
+                    help="operator arithmetic (rdm.h rdm_set_precision): fp32 (1e-4 gate) or fast "
+                         "(bf16 SpMM operand + 1xTF32 GEMM, 2e-2 gate)")
+    ap.add_argument("--no-variants", action="store_true",
+                    help="skip the extra timing of the fast-precision variant")
     ap.add_argument("--saint", action="store_true",
                     help="GraphSAINT-RDM (BASELINE configs[3]): step = one sampled subgraph")
     ap.add_argument("--roots", type=int, default=8000)
@@ -414,6 +421,7 @@ def main():
     ctx = rdm.Context(rank=rank if world > 1 else 0, world=world, device=local_rank, stream=stream,
                       unique_id=uid)
     ctx.set_transport(a.transport)
+    ctx.set_precision(a.precision)
     ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
     pareto, chosen, comm_u, sparse_u = rdm.select_config(list(wl.f), wl.n, wl.nnz, world)
     lo, hi, _ = rdm.partition(world, rdm.ROW, wl.n, wl.f[0], rank if world > 1 else 0)
@@ -540,6 +548,20 @@ def main():
         e2e = {"value": e_ms / k2, "unit": "ms", "h2d_bytes_per_step": int(h2d),
                "d2h_bytes_per_step": 8}
 
+    loss_main = float(loss.item())
+
+    # ---------------- the other precision variant, same model and inputs (NEXT-3)
+    variants = None
+    if not a.no_variants:
+        other = "fast" if a.precision == "fp32" else "fp32"
+        ctx.set_precision(other)
+        for _ in range(3):
+            epoch()
+        v_ms = time_epochs(a.steps)
+        ctx.set_precision(a.precision)
+        variants = {other: {"ms_per_step": v_ms, "dtype": DTYPES[other],
+                            "parity_gate": GATES[other]}}
+
     # ---------------- roofline of the dominant kernel (SpMM)
     import json as _json
     peaks = {}
@@ -588,9 +610,11 @@ def main():
         line = {
             "metric": METRIC, "value": ms_epoch, "unit": "ms", "n_gpus": world, "steps": a.steps,
             "warmup": max(3, a.warmup), "ms_per_step": ms_epoch, "higher_is_better": False,
-            "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
+            "scaling": "strong", "vs_baseline": None, "dtype": DTYPES[a.precision],
+            "data": "synthetic",
             "config": {
                 "workload": wl.name, "model": f"GCN {wl.L}L f={'/'.join(map(str, wl.f))}",
+                "precision": a.precision, "parity_gate": GATES[a.precision],
                 "n": n, "nnz": nnz, "graph": "R-MAT (0.57,0.19,0.19,0.05), permuted, symmetric, "
                 "self loops, D^-1/2 (A+I) D^-1/2", "global_batch": n, "seq_len": None,
                 "parallelism": f"rdm{world} (A replicated, H row/col redistributed)",
@@ -600,14 +624,15 @@ def main():
                 "sweep_ms": ({str(k): round(v, 4) for k, v in sweep.items()} if sweep else None),
                 "model_comm_units": info["model_comm_units"],
                 "model_sparse_units": info["model_sparse_units"],
-                "l2": "inputs larger than L2 (CSR 0.92 GB streamed per SpMM; H0 561 MB)",
+                "l2": (f"inputs larger than L2 (CSR {(8 * nnz + 8 * (n + 1)) / 1e9:.2f} GB streamed "
+                       f"per SpMM; H0 {n * wl.f[0] * 4 / 1e6:.0f} MB)"),
                 "gen_s": round(t_gen, 1)},
             "clocks": clocks, "e2e": e2e, "gpu_launches": cnt["kernel_launches"],
             "roofline": roofline, "cpu_baseline": cpu,
             "phases_ms_per_step": {k: v / a.steps for k, v in ph_ms.items()},
             "spmm_hbm_gbs": achieved, "a2a_bus_gbs": a2a_bus,
             "a2a_bytes_per_step": cnt["a2a_bytes_wire"] / a.steps,
-            "loss": float(loss.item()),
+            "loss": loss_main, "variants": variants,
         }
         print(json.dumps(line), flush=True)
     ctx.sync()

@@ -146,6 +146,7 @@ typedef struct {
   int64_t gemm_flops;
   int64_t allreduce_bytes;
   int64_t kernel_launches;    /* kernels this library launched                               */
+  int64_t bcast_elems;        /* R_A < P: elements of input tiles broadcast to other ranks   */
 } rdm_counters;
 
 /* ---------------------------------------------------------------- context */
@@ -185,6 +186,24 @@ rdm_status rdm_set_stream(rdm_ctx* ctx, void* cuda_stream);
 enum { RDM_TRANSPORT_NCCL = 0, RDM_TRANSPORT_P2P = 1 };
 rdm_status rdm_set_transport(rdm_ctx* ctx, int transport);
 int rdm_get_transport(const rdm_ctx* ctx);
+
+/* Arithmetic variant of the operators (BASELINE
+ * north_star: "2e-2 if a bf16 GEMM variant is enabled"):
+ *   RDM_PREC_FP32 (default): fp32 storage and accumulation, GEMMs in 3xTF32
+ *     on the tensor cores — the 1e-4 parity gate.
+ *   RDM_PREC_FAST: every rdm_spmm rounds its input column slice to bf16
+ *     (round-to-nearest-even) once per call and gathers the bf16 rows
+ *     (half the L2/HBM gather bytes), accumulating in fp32; the binary hub
+ *     tiles multiply one bf16 piece of s⊙X instead of three; every rdm_gemm
+ *     (NN / NT / TN) issues one tf32 MMA per k step instead of 3xTF32 (the
+ *     tensor core reads fp32 operands as tf32).  Outputs, gradients and the
+ *     loss stay fp32 in the caller's buffers; redistribution stays bit-exact.
+ *     Parity gate 2e-2 (max relative error per tensor, reading R26).
+ * Applies to every later call on the ctx (the executor included).
+ * Errors: RDM_ERR_ARG (unknown value). */
+enum { RDM_PREC_FP32 = 0, RDM_PREC_FAST = 1 };
+rdm_status rdm_set_precision(rdm_ctx* ctx, int precision);
+int rdm_get_precision(const rdm_ctx* ctx);
 
 int rdm_world(const rdm_ctx* ctx);
 int rdm_num_local(const rdm_ctx* ctx);            /* local rank slots (1 or world)  */
@@ -276,6 +295,46 @@ rdm_status rdm_redistribute(rdm_ctx* ctx, rdm_layout from, const float* const* s
 rdm_status rdm_redist_plan(int world, int rank, rdm_layout from, int64_t n, int64_t f,
                            int64_t* send_off, int64_t* send_elems, int64_t* recv_off,
                            int64_t* recv_elems);
+
+/* -------------------------------------------- partial replication, R_A < P */
+/* §III-E (L146-167, Fig. 6), Tables II/III "Comm. (R_A < P)" rows, §IV-A.4
+ * (L214-216); SURVEY §8(f) NEXT-4.  The P ranks form a grid of P/R_A row
+ * panels x R_A column groups, rank p = i·R_A + j.  Row panel i of the
+ * adjacency (rows row_range(N, P/R_A, i) — ⌊i·N·R_A/P⌋ … — all N columns) is
+ * stored on the R_A ranks of panel group i: R_A copies of A in total instead
+ * of P.  Dense SpMM operands use the TILE layout: rank (i, j) holds panel i's
+ * rows x the column range of RDM_COL partitioned over R_A (rdm_partition_tile).
+ *
+ * rdm_set_graph_panels: install the panels this process needs (1 for an NCCL
+ *   rank, P/R_A for a virtual group).  The matrix is used as given (pass Aᵀ
+ *   for eq. 1 on a directed graph).  R_A must divide P.  Synchronous.  Errors:
+ *   RDM_ERR_ARG (R_A, CSR), RDM_ERR_OOM.  Independent of rdm_set_graph.
+ * rdm_partition_tile: rank's tile (pure host function): rows [row_lo, row_hi),
+ *   columns [col_lo, col_hi), leading dim ld = roundup4(col_hi − col_lo).
+ * rdm_redistribute_panels: row slices (rdm_partition RDM_ROW) ↔ tiles, an
+ *   all-to-all inside every panel group: (R_A−1)/R_A·N·f elements in total
+ *   (L214).  from = RDM_ROW: src row slices → dst tiles; RDM_COL: tiles →
+ *   row slices.  Collective, bit-exact.
+ * rdm_spmm_panels: out_tile = A[panel rows, :] · In[:, tile columns] (Fig. 6):
+ *   each rank broadcasts its input tile to the other P/R_A − 1 ranks of its
+ *   column group ((P/R_A − 1)·N·f elements per call, L152/L216, counted in
+ *   rdm_counters.bcast_elems), then multiplies its row panel by the
+ *   assembled N x w_j slice (the rdm_spmm kernels, honouring
+ *   rdm_set_precision).  Epilogue bits as rdm_spmm; bias: f floats (device,
+ *   replicated) or NULL; mask: one tile per local slot or NULL.  Collective.
+ * rdm_max_replication: L160-167 R_A = P·(M − H_all)/G capped at P; the
+ *   largest divisor of P not above it (reading R36); 0 if A does not fit in
+ *   the aggregate memory.  Pure host function. */
+rdm_status rdm_set_graph_panels(rdm_ctx* ctx, int R_A, int64_t n, int64_t nnz, const int64_t* rowptr,
+                                const int32_t* col, const float* vals, int on_host);
+rdm_status rdm_partition_tile(int world, int R_A, int64_t n, int64_t f, int rank, int64_t* row_lo,
+                              int64_t* row_hi, int64_t* col_lo, int64_t* col_hi, int64_t* ld);
+rdm_status rdm_redistribute_panels(rdm_ctx* ctx, rdm_layout from, const float* const* src,
+                                   float* const* dst, int64_t n, int64_t f);
+rdm_status rdm_spmm_panels(rdm_ctx* ctx, const float* const* in_tiles, float* const* out_tiles,
+                           int64_t f, int epilogue, const float* bias, const float* const* mask_tiles);
+int rdm_max_replication(int world, double mem_bytes_per_gpu, double h_all_bytes_per_gpu,
+                        double graph_bytes);
 
 /* In-place sum over all ranks of count floats per local slot (weight-gradient
  * reduction, reading R16).  Virtual group: every slot receives the sum. */

@@ -153,3 +153,48 @@ def table_iv_symbolic(cfg_id: int, fin, fh, fout) -> tuple:
         15: (fin + 4 * fh + 2 * fout + 2 * mn1 + 2 * mn2, fin + 2 * fh + fout + mn1 + mn2),
     }
     return t[cfg_id]
+
+
+# ---------------------------------------------------------------- R_A < P
+# §III-E (Fig. 6) and the "Comm. (R_A < P)" rows of
+# Tables II/III (L185-202), §IV-A.4 (L214-216).  P GPUs form a grid of
+# P/R_A row panels x R_A column groups; A's row panel i is held by the R_A GPUs
+# of panel group i (R_A copies of A in total).  Dense operands of the SpMM are
+# (P/R_A) x R_A tiles (panel rows x column slice).  Reading R35: every
+# redistribution of width f moves (R_A-1)/R_A·N·f elements (inside a panel
+# group, L214), and every SpMM of width f additionally broadcasts its input
+# tiles inside the column group, (P/R_A-1)·N·f elements (L152, L216); the
+# printed R_A rows of Table III, which mix f_{l-1} and f_l and drop the
+# broadcast term of the GEMM-first row, are read by that same rule.
+
+def comm_elements_ra(cfg_id: int, f, n: int, P: int, RA: int) -> float:
+    """Elements moved per epoch by configuration `cfg_id` at R_A = RA (R35)."""
+    assert 1 <= RA <= P and P % RA == 0
+    comm, sparse = simulate(cfg_id, f)
+    return n * ((RA - 1) / RA * comm + (P / RA - 1) * sparse)
+
+
+def layer_comm_ra(f_in: int, n: int, P: int, RA: int) -> float:
+    """Table II "Comm. (R_A < P)" entry for one forward layer whose SpMM and
+    redistribution both have width f_in (as printed, L185-189)."""
+    return (RA - 1) / RA * n * f_in + (P / RA - 1) * n * f_in
+
+
+def max_replication(P: int, mem_bytes: float, h_all_bytes: float, g_bytes: float) -> int:
+    """L160-167: R_A = P·(M − H_all)/G replicas fit, at most P ("when this
+    number is larger than P we are going to use R_A = P").  Reading R36: the
+    grid needs R_A | P, so the largest divisor of P not above that bound; 0 if
+    not even one copy of A fits in the aggregate memory."""
+    bound = P * (mem_bytes - h_all_bytes) / g_bytes if g_bytes > 0 else P
+    cap = min(P, int(bound)) if bound >= 1 else 0
+    for r in range(cap, 0, -1):
+        if P % r == 0:
+            return r
+    return 0
+
+
+def pareto_ra(f, n: int, P: int, RA: int) -> list:
+    """Pareto front in (elements moved at R_A, sparse units)."""
+    L = len(f) - 1
+    costs = {i: (comm_elements_ra(i, f, n, P, RA), simulate(i, f)[1]) for i in range(4 ** L)}
+    return pareto(costs)

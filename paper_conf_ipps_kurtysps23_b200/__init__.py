@@ -38,6 +38,7 @@ _STATUS = {0: "OK", 1: "ERR_ARG", 2: "ERR_CUDA", 3: "ERR_NCCL", 4: "ERR_OOM",
            5: "ERR_UNSUPPORTED", 6: "ERR_STATE"}
 
 TRANSPORTS = {"nccl": 0, "p2p": 1}
+PRECISIONS = {"fp32": 0, "fast": 1}
 
 # C symbols declared in include/rdm.h (checked by tests/test_abi.py)
 EXPORTS = [
@@ -50,6 +51,7 @@ EXPORTS = [
     "rdm_adam_step", "rdm_get_counters", "rdm_reset_counters", "rdm_set_timing",
     "rdm_get_phase_times", "rdm_reset_phase_times", "rdm_redist_plan", "rdm_plan_info",
     "rdm_set_transport", "rdm_get_transport", "rdm_debug_disable_tc",
+    "rdm_set_precision", "rdm_get_precision",
 ]
 
 
@@ -62,7 +64,7 @@ class RdmCounters(ctypes.Structure):
     _fields_ = [(n, ctypes.c_int64) for n in (
         "a2a_calls", "a2a_elems_payload", "a2a_bytes_wire", "a2a_width_units", "spmm_calls",
         "spmm_nnz_cols", "spmm_width_units", "gemm_calls", "gemm_flops", "allreduce_bytes",
-        "kernel_launches")]
+        "kernel_launches", "bcast_elems")]
 
     def as_dict(self):
         return {n: getattr(self, n) for n, _ in self._fields_}
@@ -112,6 +114,7 @@ _sig = {
     "rdm_reset_counters": [_vp],
     "rdm_set_timing": [_vp, _int],
     "rdm_set_transport": [_vp, _int],
+    "rdm_set_precision": [_vp, _int],
     "rdm_get_phase_times": [_vp, ctypes.POINTER(ctypes.c_double), _pi64],
     "rdm_reset_phase_times": [_vp],
     "rdm_redist_plan": [_int, _int, _int, _i64, _i64, _pi64, _pi64, _pi64, _pi64],
@@ -334,6 +337,16 @@ class Context:
         into their producing kernel's epilogue, rdm.h rdm_set_transport);
         applies to GCN instances created afterwards."""
         self._c(_lib.rdm_set_transport(self.h, TRANSPORTS[transport]))
+
+    def set_precision(self, precision):
+        """"fp32" (default; 3xTF32 GEMMs, 1e-4 gate) or "fast" (bf16 SpMM
+        operand, 1xTF32 GEMMs, 2e-2 gate; rdm.h rdm_set_precision); applies to
+        every later call on this context."""
+        self._c(_lib.rdm_set_precision(self.h, PRECISIONS[precision]))
+
+    @property
+    def precision(self):
+        return {v: k for k, v in PRECISIONS.items()}[_lib.rdm_get_precision(self.h)]
 
     @property
     def transport(self):

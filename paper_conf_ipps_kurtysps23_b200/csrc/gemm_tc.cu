@@ -53,6 +53,7 @@ struct TcShape {
   int tiles_m, tiles_n, splits, n_mma;
   int pf;   // issue L2 prefetches of A through tmApf
   int dbg;  // timing experiments only (RDM_TC_DBG): 1 = skip split, 2 = skip MMA
+  int one;  // RDM_PREC_FAST: 1xTF32 (one MMA per k step, no lo operands)
 };
 
 // A operand placement.  For BN ≤ 128 the converter writes A's hi / lo split
@@ -203,7 +204,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
 
   if (warp == 0) {
     if (lane == 0) {
-      const uint32_t bytes = MODE == 0 ? (CF::kABytes + 2 * CF::kBBytes) : (CF::kABytes + CF::kBBytes);
+      const uint32_t bytes = MODE == 0 ? (CF::kABytes + (sh.one ? 1 : 2) * CF::kBBytes) : (CF::kABytes + CF::kBBytes);
       uint32_t kc = 0;
       for (int t = blockIdx.x; t < total; t += gridDim.x) {
         int64_t kbeg;
@@ -228,7 +229,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
             }
             tma_load_2d(A_hi(s), &tmA, &full[s], kk, m0);
             tma_load_2d(B_hi(s), &tmB, &full[s], kk, n0);
-            tma_load_2d(B_lo(s), &tmBlo, &full[s], kk, n0);
+            if (!sh.one) tma_load_2d(B_lo(s), &tmBlo, &full[s], kk, n0);
           } else {
             for (int c = 0; c < BM / 32; ++c) tma_load_2d(A_hi(s) + c * 4096, &tmA, &full[s], m0 + 32 * c, kk);
             for (int c = 0; c < BN / 32; ++c) tma_load_2d(B_hi(s) + c * 4096, &tmB, &full[s], n0 + 32 * c, kk);
@@ -269,6 +270,17 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
             }
             const uint32_t acc0 = (kb > 0 || j > 0) ? 1u : 0u;
             if (sh.dbg & 2) {
+            } else if (sh.one) {
+              // 1xTF32: A_tf32 · B_tf32, rotating over the partial accumulators
+              const uint32_t d = d_tmem + (uint32_t)((j % CF::kNAcc) * CF::kAccCols);
+              if (CF::kTmemA) {
+                tc_mma_ts(d, tmem_base + CF::kACol0 + s * 2 * BK + j * UK, dbh, idesc,
+                          (kb > 0 || j >= CF::kNAcc) ? 1u : 0u);
+              } else {
+                const uint32_t ah = smem_u32(A_hi(s));
+                tc_mma(d, MODE == 0 ? sdesc(ah + j * 32, 16, 1024) : sdesc(ah + j * 1024, 4096, 512, 1), dbh,
+                       idesc, (kb > 0 || j >= CF::kNAcc) ? 1u : 0u);
+              }
             } else if (CF::kTmemA) {
               // A stage s: hi in columns [kACol0 + 64 s, +32), lo in the next 32.
               // Narrow tiles rotate over kNAcc independent accumulators so that
@@ -311,6 +323,17 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         const int s = kc % S;
         mbar_wait(&full[s], (kc / S) & 1);
         if (sh.dbg & 1) {
+        } else if (sh.one) {
+          // 1xTF32: A rounded to tf32 into TMEM; smem operands are read as tf32
+          // by the tensor core as they are (low mantissa bits ignored)
+          if (CF::kTmemA) {
+            float v[32];
+            load_a_row<MODE>(A_hi(s), t128, v);
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] = tf32_rn(v[i]);
+            tmem_st32(tmem_base + ((uint32_t)((warp & 3) * 32) << 16) + CF::kACol0 + s * 2 * BK, v);
+            asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+          }
         } else if (CF::kTmemA) {
           // thread t128 owns A row t128 = TMEM lane (quadrant warp % 4)
           float v[32], h[32];
@@ -327,7 +350,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         } else {
           split_inplace((float4*)A_hi(s), (float4*)A_lo(s), CF::kABytes / 16, t128, 128);
         }
-        if (MODE == 1) split_inplace((float4*)B_hi(s), (float4*)B_lo(s), CF::kBBytes / 16, t128, 128);
+        if (MODE == 1 && !sh.one) split_inplace((float4*)B_hi(s), (float4*)B_lo(s), CF::kBBytes / 16, t128, 128);
         fence_proxy_async();
         tc_fence_before();
         mbar_arrive(&conv[s]);
@@ -514,6 +537,7 @@ void launch_tc_ew(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, cons
   sh.pf = apf != nullptr;
   const char* dbg = getenv("RDM_TC_DBG");
   sh.dbg = dbg ? atoi(dbg) : 0;
+  sh.one = ctx->prec == RDM_PREC_FAST ? 1 : 0;
   const int64_t total = (int64_t)sh.tiles_m * sh.tiles_n * splits;
   const unsigned grid = (unsigned)std::min<int64_t>(total, ctx->num_sms);
   gemm_tc_kernel<BN, MODE, EW><<<grid, CF::kThreads, CF::kSmem, ctx->stream>>>(a, b, blo, apf ? *apf : a, C, ldc,

@@ -117,13 +117,14 @@ struct TileShape {
   int64_t w, ldp;
   int S, SA;          // shared-memory stages, TMEM A slots
   int HS;             // 64-wide k halves per stage (1 or 2)
-  int stage_bytes;    // HS · (3 · n_mma · 128 + 1024)
+  int stage_bytes;    // HS · (NP · n_mma · 128 + 1024)
   int R;              // > 0: concatenated-piece MMAs with R rotating accumulator sets
   int acc_cols;       // TMEM columns per accumulator buffer
   int dbg;            // timing experiments (RDM_TILE_DBG): 1 = skip the MMAs
 };
 
-template <int HS>
+// NP = bf16 pieces of s⊙X: 3 (fp32-class, RDM_PREC_FP32) or 1 (RDM_PREC_FAST).
+template <int HS, int NP>
 __global__ void __launch_bounds__(384, 1)
 hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__ CUtensorMap tmB2d,
                 const uint64_t* __restrict__ bits,
@@ -150,7 +151,7 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__
   // [half][128 rows] u64.  TMEM: two accumulator buffers of acc_cols columns,
   // then SA A slots of 32·HS columns (64·HS bf16 per row, packed in pairs).
   const int bpiece = n_mma * 128;                 // bytes of one piece of one half
-  const int bbytes = HS * 3 * bpiece;
+  const int bbytes = HS * NP * bpiece;
   const uint32_t kAcol = 2 * sh.acc_cols;
   auto B_st = [&](int s) { return smem + s * sh.stage_bytes; };
   auto bits_st = [&](int s) { return smem + s * sh.stage_bytes + bbytes; };
@@ -208,7 +209,7 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__
             if (HS == 2) {
               tma_load_4d(B_st(s), &tmB, &full[s], 0, n0, 0, kb);
             } else {   // three 2-D boxes from the stacked panels (measured faster for one half)
-              for (int pc = 0; pc < 3; ++pc)
+              for (int pc = 0; pc < NP; ++pc)
                 tma_load_2d(B_st(s) + pc * bpiece, &tmB2d, &full[s], (kb + h) * SK, pc * (int)sh.w + n0);
             }
             ++kc;
@@ -219,12 +220,12 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__
     }
   } else if (warp == 1) {
     if (lane == 0) {
-      const uint32_t idesc = idesc_bf16(R ? 3 * n_mma : n_mma);
+      const uint32_t idesc = idesc_bf16(R ? NP * n_mma : n_mma);
       // descriptors advance linearly: +stage_bytes per stage, +3·bpiece per
       // k half, +bpiece per piece, +32 B per k16 step (16-byte units)
       const uint64_t bd0 = sdesc(smem_u32(B_st(0)), 16, 1024);
       const uint32_t st16 = (uint32_t)sh.stage_bytes >> 4, pc16 = (uint32_t)bpiece >> 4;
-      const uint32_t rho_step = 3u * n_mma, rho_end = (uint32_t)R * rho_step;
+      const uint32_t rho_step = (uint32_t)NP * n_mma, rho_end = (uint32_t)R * rho_step;
       int s = 0, a = 0;
       uint32_t ph = 0, aph = 0;
       int it = 0;
@@ -245,7 +246,7 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__
           if (!(sh.dbg & 1)) {
 #pragma unroll
             for (int h = 0; h < HS; ++h) {
-              const uint64_t bh = bd + (uint64_t)(h * 3 * pc16);
+              const uint64_t bh = bd + (uint64_t)(h * NP * pc16);
               const uint32_t th = ta + h * 32;
               if (R) {
 #pragma unroll
@@ -258,8 +259,10 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__
 #pragma unroll
                 for (int j = 0; j < SK / 16; ++j, ++g) {   // 8 packed A columns, 32 B of B rows per k16
                   tc_mma_f16_ts(d_tmem, th + j * 8, bh + 2 * j, idesc, g > 0 ? 1u : 0u);
-                  tc_mma_f16_ts(d_tmem, th + j * 8, bh + pc16 + 2 * j, idesc, 1u);
-                  tc_mma_f16_ts(d_tmem, th + j * 8, bh + 2 * pc16 + 2 * j, idesc, 1u);
+                  if (NP == 3) {
+                    tc_mma_f16_ts(d_tmem, th + j * 8, bh + pc16 + 2 * j, idesc, 1u);
+                    tc_mma_f16_ts(d_tmem, th + j * 8, bh + 2 * pc16 + 2 * j, idesc, 1u);
+                  }
                 }
               }
             }
@@ -325,9 +328,9 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__
           float sum[32];
 #pragma unroll
           for (int i = 0; i < 32; ++i) sum[i] = 0.f;
-          for (int pc = 2; pc >= 0; --pc)
+          for (int pc = NP - 1; pc >= 0; --pc)
             for (int rho = 0; rho < R; ++rho) {
-              tmem_ld32(a0 + (uint32_t)((rho * 3 + pc) * n_mma), rr);
+              tmem_ld32(a0 + (uint32_t)((rho * NP + pc) * n_mma), rr);
 #pragma unroll
               for (int i = 0; i < 32; ++i) sum[i] += __uint_as_float(rr[i]);
             }
@@ -360,7 +363,7 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__
 __global__ void tile_panels_kernel(const float* __restrict__ X, int64_t ldx, const int32_t* __restrict__ hub_ids,
                                    const float* __restrict__ scale, int64_t K2, int64_t w,
                                    __nv_bfloat16* __restrict__ p0, __nv_bfloat16* __restrict__ p1,
-                                   __nv_bfloat16* __restrict__ p2) {
+                                   __nv_bfloat16* __restrict__ p2, int np) {
   __shared__ float t[64][33];
   const int64_t k0 = (int64_t)blockIdx.x * 64, n0 = (int64_t)blockIdx.y * 32;
   for (int i = threadIdx.y; i < 64; i += 8) {
@@ -381,8 +384,10 @@ __global__ void tile_panels_kernel(const float* __restrict__ X, int64_t ldx, con
       const __nv_bfloat16 l = __float2bfloat16_rn(r1 - __bfloat162float(m));
       const int64_t o = n * K2 + k0 + kk;
       p0[o] = h;
-      p1[o] = m;
-      p2[o] = l;
+      if (np == 3) {
+        p1[o] = m;
+        p2[o] = l;
+      }
     }
   }
 }
@@ -403,11 +408,11 @@ PFN_cuTensorMapEncodeTiled_v12000 encode() {
 // p·w·K2): dims {64 (k within a 128-byte swizzle row), n, piece, k / 64}, box
 // {64, n_mma, 3, HS}, so that one TMA lands [half][piece][n_mma][64] in smem
 // with the 128-byte swizzle; rows n ≥ w read as zeros.
-CUtensorMap panel_map(const void* base, int64_t K2, int64_t w, int n_mma, int HS) {
+CUtensorMap panel_map(const void* base, int64_t K2, int64_t w, int n_mma, int HS, int np) {
   CUtensorMap m;
-  cuuint64_t dims[4] = {(cuuint64_t)SK, (cuuint64_t)w, 3, (cuuint64_t)(K2 / SK)};
+  cuuint64_t dims[4] = {(cuuint64_t)SK, (cuuint64_t)w, (cuuint64_t)np, (cuuint64_t)(K2 / SK)};
   cuuint64_t strides[3] = {(cuuint64_t)(K2 * 2), (cuuint64_t)(w * K2 * 2), (cuuint64_t)(SK * 2)};
-  cuuint32_t box[4] = {(cuuint32_t)SK, (cuuint32_t)n_mma, 3, (cuuint32_t)HS};
+  cuuint32_t box[4] = {(cuuint32_t)SK, (cuuint32_t)n_mma, (cuuint32_t)np, (cuuint32_t)HS};
   cuuint32_t es[4] = {1, 1, 1, 1};
   CUresult r = encode()(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 4, const_cast<void*>(base), dims, strides, box, es,
                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
@@ -434,24 +439,25 @@ CUtensorMap stacked_map(const void* base, int64_t K2, int64_t rows, int n_mma) {
 // (L2-gather bound), a tile ≈ ceil(w/128)·(4.5 + 5.2·min(w,128)/128) ns (bit
 // expansion + 3 bf16 MMA pieces per 128-wide chunk), plus ≈ 20 µs per call.
 double csr_entry_s(int64_t w) { return 24e-12 * std::pow((double)w / 128.0, 0.55); }
-double tile_s(int64_t w) {
-  return (double)ceil_div(w, 128) * (4.5e-9 + 5.2e-9 * (double)std::min<int64_t>(w, 128) / 128.0);
+double tile_s(int64_t w, int np = 3) {
+  return (double)ceil_div(w, 128) * (4.5e-9 + 5.2e-9 * np / 3.0 * (double)std::min<int64_t>(w, 128) / 128.0);
 }
 }  // namespace
 
-bool hub_tiles_pay(const Core& c, int64_t w) {
+bool hub_tiles_pay(const Core& c, int64_t w, int np) {
   if (!c.n_tiles) return false;
   if (c.forced) return true;
-  return (double)c.nnz * csr_entry_s(w) > (double)c.n_tiles * tile_s(w) + 20e-6;
+  return (double)c.nnz * csr_entry_s(w) > (double)c.n_tiles * tile_s(w, np) + 20e-6;
 }
 
 void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx, int64_t w, float* part,
-                       int64_t ldp) {
+                       int64_t ldp, int np) {
+  RDM_CHECK_ARG(np == 1 || np == 3, "hub tiles: 1 or 3 bf16 pieces");
   const int64_t K2 = c.K2;
-  __nv_bfloat16* pan = reinterpret_cast<__nv_bfloat16*>(ensure_ws(ctx->ws_core_b, (size_t)3 * w * K2 * 2));
+  __nv_bfloat16* pan = reinterpret_cast<__nv_bfloat16*>(ensure_ws(ctx->ws_core_b, (size_t)np * w * K2 * 2));
   dim3 pg((unsigned)(K2 / 64), (unsigned)ceil_div(w, 32));
   tile_panels_kernel<<<pg, dim3(32, 8), 0, ctx->stream>>>(X, ldx, c.hub_ids->as<int32_t>(), c.scale->as<float>(), K2,
-                                                        w, pan, pan + w * K2, pan + 2 * w * K2);
+                                                        w, pan, pan + w * K2, pan + 2 * w * K2, np);
   RDM_LAUNCHED(ctx);
   TileShape sh;
   sh.n_mma = (int)std::min<int64_t>(128, ((w + 15) / 16) * 16);
@@ -461,25 +467,26 @@ void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx,
   sh.ldp = ldp;
   sh.R = sh.n_mma <= 64 ? (sh.n_mma <= 16 ? 2 : 1) : 0;
   if (const char* e = getenv("RDM_TILE_R")) sh.R = sh.n_mma <= 64 ? std::max(0, std::min(4, atoi(e))) : 0;
-  sh.acc_cols = (int)((sh.R ? sh.R * 3 * sh.n_mma : sh.n_mma) + 31) / 32 * 32;
+  sh.acc_cols = (int)((sh.R ? sh.R * np * sh.n_mma : sh.n_mma) + 31) / 32 * 32;
   // whole tiles per stage when the stage stays small (narrow slices: halves
   // the per-stage fixed cost), else 64-wide k halves
-  sh.HS = 3 * sh.n_mma * 256 + 2048 <= 50 * 1024 ? 2 : 1;
+  sh.HS = np * sh.n_mma * 256 + 2048 <= 50 * 1024 ? 2 : 1;
   if (const char* e = getenv("RDM_TILE_HS")) sh.HS = atoi(e) == 2 ? 2 : 1;
-  sh.stage_bytes = sh.HS * (3 * sh.n_mma * 128 + 1024);
+  sh.stage_bytes = sh.HS * (np * sh.n_mma * 128 + 1024);
   const int avail = kSmemBudget - 1024 - 1024 - 4096;   // align, barriers, LUT
   sh.S = std::min(32, avail / sh.stage_bytes);
   sh.SA = std::min(8, (512 - 2 * sh.acc_cols) / (32 * sh.HS));
   sh.dbg = getenv("RDM_TILE_DBG") ? atoi(getenv("RDM_TILE_DBG")) : 0;
   RDM_CHECK_ARG(sh.S >= 2 && sh.SA >= 2, "hub tiles: TMEM/smem budget");
-  const CUtensorMap tb = panel_map(pan, K2, w, sh.n_mma, sh.HS);
+  const CUtensorMap tb = panel_map(pan, K2, w, sh.n_mma, sh.HS, np);
   // the three panels stacked as one 3w x K2 matrix: rows past a panel's w
   // only feed accumulator columns ≥ w, which are never stored
-  const CUtensorMap tb2 = stacked_map(pan, K2, 3 * w, sh.n_mma);
+  const CUtensorMap tb2 = stacked_map(pan, K2, np * w, sh.n_mma);
   const int smem = sh.S * sh.stage_bytes + 1024 + 1024 + 4096;
   const int64_t total = c.n_items * sh.tiles_n;
   const unsigned grid = (unsigned)std::min<int64_t>(total, ctx->num_sms);
-  auto kern = sh.HS == 2 ? hub_tile_kernel<2> : hub_tile_kernel<1>;
+  auto kern = np == 3 ? (sh.HS == 2 ? hub_tile_kernel<2, 3> : hub_tile_kernel<1, 3>)
+                      : (sh.HS == 2 ? hub_tile_kernel<2, 1> : hub_tile_kernel<1, 1>);
   RDM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
   kern<<<grid, 384, smem, ctx->stream>>>(tb, tb2, c.tiles->as<uint64_t>(), c.tile_cb->as<int32_t>(),
                                          c.item_tb->as<int32_t>(), part, sh);

@@ -102,6 +102,8 @@ struct Core {
 
 struct Csr {
   int64_t n = 0, nnz = 0;
+  int64_t n_in = -1;   // rows of the dense input (columns of A); -1 = n (square)
+  int64_t in_rows() const { return n_in < 0 ? n : n_in; }
   std::unique_ptr<DevBuf> rowptr, col, val;
   Core core;
   // row bins (see spmm.cu): light rows processed warp-per-row, heavy rows
@@ -136,6 +138,7 @@ struct rdm_ctx {
   ncclComm_t comm = nullptr;
   bool poisoned = false;
   int transport = 0;             // RDM_TRANSPORT_NCCL / RDM_TRANSPORT_P2P
+  int prec = 0;                  // RDM_PREC_FP32 / RDM_PREC_FAST
   std::string err;
   rdm::Graph graph;
   bool has_graph = false;
@@ -148,6 +151,13 @@ struct rdm_ctx {
   std::unique_ptr<rdm::DevBuf> ws_stage;                       // host-input staging
   std::unique_ptr<rdm::DevBuf> ws_core_b, ws_core_c;           // hub-core panels / product
   std::unique_ptr<rdm::DevBuf> ws_scratch;
+  // R_A < P (§III-E): row panels of A held by this process (index = panel id;
+  // an NCCL rank holds its own panel only), the panel-group size R_A
+  int panel_RA = 0;
+  int64_t panel_n = 0;
+  std::vector<std::unique_ptr<rdm::Csr>> panels;
+  std::unique_ptr<rdm::DevBuf> ws_panel_in;                    // all-gathered N x w_j input per slot
+  std::unique_ptr<rdm::DevBuf> ws_bf16;                        // RDM_PREC_FAST: bf16 copy of the SpMM input
   // phase timing
   bool timing = false;
   int cur_phase = RDM_PH_OTHER;
@@ -231,9 +241,10 @@ void build_core(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, const int32_t*
 // summed per row block and scaled by s_i in the SpMM epilogue.
 bool build_hub_tiles(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, const int32_t* col_host,
                      const float* val_host);
-bool hub_tiles_pay(const Core& c, int64_t w);
+// np = bf16 pieces of s⊙X: 3 (fp32-class) or 1 (RDM_PREC_FAST).
+bool hub_tiles_pay(const Core& c, int64_t w, int np);
 void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx, int64_t w,
-                       float* part, int64_t ldp);
+                       float* part, int64_t ldp, int np);
 
 // hub-core size rule shared by the host (full graph) and device (subgraph) builders
 int64_t choose_core_K(const int64_t* bucket, int64_t kmax, const char* force, bool* forced);
@@ -274,6 +285,16 @@ void unpack_rows(rdm_ctx* ctx, float* row_slice, int64_t ld_row, int64_t rows, i
 void scatter_slice(rdm_ctx* ctx, const float* src, int64_t lds, int64_t rows, int64_t cols,
                    const Scatter& s);
 
+// panels.cpp — R_A < P (§III-E)
+void set_graph_panels(rdm_ctx* ctx, int RA, int64_t n, int64_t nnz, const int64_t* rowptr,
+                      const int32_t* col, const float* val, int on_host);
+void tile_of(int P, int RA, int64_t n, int64_t f, int p, Range* rows, Range* cols, int64_t* ld);
+void redistribute_panels(rdm_ctx* ctx, rdm_layout from, const float* const* src, float* const* dst,
+                         int64_t n, int64_t f);
+void spmm_panels(rdm_ctx* ctx, const float* const* in, float* const* out, int64_t f, int epi,
+                 const float* bias, const float* const* mask);
+int max_replication(int P, double mem_bytes, double h_all_bytes, double g_bytes);
+
 // misc.cu
 void softmax_xent(rdm_ctx* ctx, const float* Z, int64_t ldz, const int32_t* labels,
                   const uint8_t* mask, int64_t rows, int64_t C, const double* n_train, float* G,
@@ -299,6 +320,10 @@ struct Xfer {
   size_t recv_bytes[BlockTable::kMax];
 };
 void exchange(rdm_ctx* ctx, std::vector<Xfer>& x);   // x[i] for local slot i
+// runtime.cpp — CSR upload / validation (used by rdm_set_graph and the R_A < P panels)
+void upload_csr(rdm_ctx* ctx, Csr& A, int64_t n, int64_t nnz, const int64_t* rowptr, const int32_t* col,
+                const float* val, bool on_host);
+int validate_csr(rdm_ctx* ctx, const int64_t* rowptr, const int32_t* col, int64_t n, int64_t nnz);
 void allreduce(rdm_ctx* ctx, float* const* bufs, int64_t count);
 void allreduce_d(rdm_ctx* ctx, double* const* bufs, int64_t count);
 

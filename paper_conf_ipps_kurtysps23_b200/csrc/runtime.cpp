@@ -302,7 +302,7 @@ std::vector<float*> p2p_open(rdm_ctx* ctx, float* mine, std::vector<void*>& open
 }
 
 // ------------------------------------------------------------------ graph
-static void upload_csr(rdm_ctx* ctx, Csr& A, int64_t n, int64_t nnz, const int64_t* rowptr,
+void upload_csr(rdm_ctx* ctx, Csr& A, int64_t n, int64_t nnz, const int64_t* rowptr,
                        const int32_t* col, const float* val, bool on_host) {
   A.n = n;
   A.nnz = nnz;
@@ -493,6 +493,55 @@ rdm_status rdm_set_transport(rdm_ctx* ctx, int transport) {
 }
 
 int rdm_get_transport(const rdm_ctx* ctx) { return ctx ? ctx->transport : -1; }
+
+rdm_status rdm_set_graph_panels(rdm_ctx* ctx, int R_A, int64_t n, int64_t nnz, const int64_t* rowptr,
+                                const int32_t* col, const float* vals, int on_host) {
+  return guarded(ctx, [&] { set_graph_panels(ctx, R_A, n, nnz, rowptr, col, vals, on_host); });
+}
+
+rdm_status rdm_partition_tile(int world, int R_A, int64_t n, int64_t f, int rank, int64_t* row_lo,
+                              int64_t* row_hi, int64_t* col_lo, int64_t* col_hi, int64_t* ld) {
+  if (world < 1 || R_A < 1 || R_A > world || world % R_A || rank < 0 || rank >= world || n < 0 || f < 0)
+    return RDM_ERR_ARG;
+  Range r, c;
+  int64_t l;
+  tile_of(world, R_A, n, f, rank, &r, &c, &l);
+  if (row_lo) *row_lo = r.lo;
+  if (row_hi) *row_hi = r.hi;
+  if (col_lo) *col_lo = c.lo;
+  if (col_hi) *col_hi = c.hi;
+  if (ld) *ld = l;
+  return RDM_OK;
+}
+
+rdm_status rdm_redistribute_panels(rdm_ctx* ctx, rdm_layout from, const float* const* src,
+                                   float* const* dst, int64_t n, int64_t f) {
+  return guarded(ctx, [&] {
+    RDM_CHECK_ARG(src && dst && f >= 0 && (from == RDM_ROW || from == RDM_COL), "redistribute_panels: bad args");
+    redistribute_panels(ctx, from, src, dst, n, f);
+  });
+}
+
+rdm_status rdm_spmm_panels(rdm_ctx* ctx, const float* const* in_tiles, float* const* out_tiles,
+                           int64_t f, int epilogue, const float* bias, const float* const* mask_tiles) {
+  return guarded(ctx, [&] {
+    RDM_CHECK_ARG(in_tiles && out_tiles && f >= 0, "spmm_panels: bad args");
+    spmm_panels(ctx, in_tiles, out_tiles, f, epilogue, bias, mask_tiles);
+  });
+}
+
+int rdm_max_replication(int world, double mem_bytes_per_gpu, double h_all_bytes_per_gpu, double graph_bytes) {
+  if (world < 1) return -1;
+  return max_replication(world, mem_bytes_per_gpu, h_all_bytes_per_gpu, graph_bytes);
+}
+
+rdm_status rdm_set_precision(rdm_ctx* ctx, int precision) {
+  if (!ctx || (precision != RDM_PREC_FP32 && precision != RDM_PREC_FAST)) return RDM_ERR_ARG;
+  ctx->prec = precision;
+  return RDM_OK;
+}
+
+int rdm_get_precision(const rdm_ctx* ctx) { return ctx ? ctx->prec : -1; }
 
 int rdm_world(const rdm_ctx* ctx) { return ctx ? ctx->world : -1; }
 int rdm_num_local(const rdm_ctx* ctx) { return ctx ? ctx->nlocal() : -1; }

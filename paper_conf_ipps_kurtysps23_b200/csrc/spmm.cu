@@ -23,7 +23,10 @@
 #include <algorithm>
 #include <cmath>
 #include <cstdlib>
+#include <cstring>
 #include <vector>
+
+#include <cuda_bf16.h>
 
 #include "internal.h"
 
@@ -114,13 +117,14 @@ __device__ __forceinline__ float4 apply_epi(float4 a, const Epi& e, int64_t row,
 // every lane issues V independent 128-bit gathers per nnz.  (col, val) of 32
 // nnz are loaded once per batch, coalesced, and broadcast with shuffles (none
 // when G = 1).  Result: lanes of group 0 hold the row-chunk sum.
-template <int G, int V>
+template <int G, int V, int U>
 __device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
                                                const float* __restrict__ val,
                                                const float* __restrict__ xb, int64_t ldx,
                                                int64_t beg, int64_t end, int lane, int c4n,
                                                float4 (&acc)[V]) {
   constexpr int NG = 32 / G;
+  static_assert(G % U == 0, "U must divide G");
   const int g = lane / G, sub = lane % G;
 #pragma unroll
   for (int v = 0; v < V; ++v) acc[v] = make_float4(0.f, 0.f, 0.f, 0.f);
@@ -133,27 +137,59 @@ __device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
       a = __ldcs(val + j);
     }
     const int cnt = (end - base) < 32 ? (int)(end - base) : 32;
+    // U nnz per group are gathered before any of them is consumed (U·V
+    // independent 128-bit loads in flight per lane); an nnz past the row's end
+    // loads nothing and contributes 0·0.
+    if (U == 1) {
+      // one nnz per group at a time, skipped past the row's end
 #pragma unroll
-    for (int t = 0; t < G; ++t) {
-      const int k = t * NG + g;
-      const int cc = (G == 1) ? c : __shfl_sync(kFull, c, k);
-      const float vv = (G == 1) ? a : __shfl_sync(kFull, a, k);
-      if (k < cnt) {
-        const float4* xr = reinterpret_cast<const float4*>(xb + (int64_t)cc * ldx);
-        float4 x[V];
+      for (int t = 0; t < G; ++t) {
+        const int k = t * NG + g;
+        const int cc = (G == 1) ? c : __shfl_sync(kFull, c, k);
+        const float vv = (G == 1) ? a : __shfl_sync(kFull, a, k);
+        if (k < cnt) {
+          const float4* xr = reinterpret_cast<const float4*>(xb + (int64_t)cc * ldx);
+          float4 x[V];
 #pragma unroll
-        for (int v = 0; v < V; ++v)
-          if (v * G + sub < c4n) x[v] = __ldg(xr + v * G + sub);
+          for (int v = 0; v < V; ++v)
+            if (v * G + sub < c4n) x[v] = __ldg(xr + v * G + sub);
 #pragma unroll
-        for (int v = 0; v < V; ++v) {
-          if (v * G + sub < c4n) {
-            acc[v].x = fmaf(vv, x[v].x, acc[v].x);
-            acc[v].y = fmaf(vv, x[v].y, acc[v].y);
-            acc[v].z = fmaf(vv, x[v].z, acc[v].z);
-            acc[v].w = fmaf(vv, x[v].w, acc[v].w);
+          for (int v = 0; v < V; ++v) {
+            if (v * G + sub < c4n) {
+              acc[v].x = fmaf(vv, x[v].x, acc[v].x);
+              acc[v].y = fmaf(vv, x[v].y, acc[v].y);
+              acc[v].z = fmaf(vv, x[v].z, acc[v].z);
+              acc[v].w = fmaf(vv, x[v].w, acc[v].w);
+            }
           }
         }
       }
+      continue;
+    }
+#pragma unroll
+    for (int t0 = 0; t0 < G; t0 += U) {
+      if (t0 * NG >= cnt) break;   // warp-uniform: the rest of the batch is past the row's end
+      float4 x[U][V];
+      float vv[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int k = (t0 + u) * NG + g;
+        const int cc = (G == 1) ? c : __shfl_sync(kFull, c, k);
+        vv[u] = (G == 1) ? a : __shfl_sync(kFull, a, k);
+        const float4* xr = reinterpret_cast<const float4*>(xb + (int64_t)cc * ldx);
+#pragma unroll
+        for (int v = 0; v < V; ++v)
+          x[u][v] = (k < cnt && v * G + sub < c4n) ? __ldg(xr + v * G + sub) : make_float4(0.f, 0.f, 0.f, 0.f);
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          acc[v].x = fmaf(vv[u], x[u][v].x, acc[v].x);
+          acc[v].y = fmaf(vv[u], x[u][v].y, acc[v].y);
+          acc[v].z = fmaf(vv[u], x[u][v].z, acc[v].z);
+          acc[v].w = fmaf(vv[u], x[u][v].w, acc[v].w);
+        }
     }
   }
 #pragma unroll
@@ -174,9 +210,12 @@ __device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
 // Resident CTAs per SM: the gathers are latency-bound, so occupancy is capped
 // by registers only as far as the V accumulators need (measured on the
 // Reddit-shaped residual CSR: V = 4 best at 4 CTAs, V = 3 at 5, V ≤ 2 at 6).
-constexpr int spmm_minb(int V) { return V >= 4 ? 4 : V == 3 ? 5 : 6; }
-template <int G, int V>
-__global__ void __launch_bounds__(kWarps * 32, spmm_minb(V))
+// With U nnz in flight per group the load registers grow by U·V: occupancy
+// by float4-sized register slots (accumulators + loads), s = V + U·V here.
+constexpr int spmm_minb_slots(int s) { return s <= 4 ? 6 : s <= 6 ? 5 : s <= 8 ? 4 : s <= 12 ? 3 : 2; }
+constexpr int spmm_minb(int V, int U) { return U == 1 ? (V >= 4 ? 4 : V == 3 ? 5 : 6) : spmm_minb_slots(V + U * V); }
+template <int G, int V, int U>
+__global__ void __launch_bounds__(kWarps * 32, spmm_minb(V, U))
 spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
             const float* __restrict__ val, const int32_t* __restrict__ light_rows,
             const int64_t* __restrict__ seg_start, const int32_t* __restrict__ seg_row,
@@ -196,7 +235,7 @@ spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
     r = seg_row[item];
     const int64_t beg = seg_start[item];
     const int64_t end = min(beg + kSeg, rowptr[r + 1]);
-    warp_nnz_range<G, V>(col, val, X + cbase, ldx, beg, end, lane, c4n, acc);
+    warp_nnz_range<G, V, U>(col, val, X + cbase, ldx, beg, end, lane, c4n, acc);
     if (lane < G) {
       float* dst = part + item * ld_part + cbase;
 #pragma unroll
@@ -205,7 +244,7 @@ spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
     }
   } else {
     r = light_rows[item - n_seg];
-    warp_nnz_range<G, V>(col, val, X + cbase, ldx, rowptr[r], rowptr[r + 1], lane, c4n, acc);
+    warp_nnz_range<G, V, U>(col, val, X + cbase, ldx, rowptr[r], rowptr[r + 1], lane, c4n, acc);
     if (lane < G) {
       float* dst = out + (int64_t)r * ld_out + cbase;
 #pragma unroll
@@ -218,6 +257,149 @@ spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
         }
       }
     }
+  }
+}
+
+// RDM_PREC_FAST: the same walk over a bf16 copy of the slice.  A lane's
+// 128-bit gather now carries 8 columns; bf16 → fp32 is exact (a shift), the
+// products and sums stay fp32.  acc[v][0..1] = columns 8·ch + 0..3, + 4..7.
+template <int G, int V, int U>
+__device__ __forceinline__ void warp_nnz_range_bf(const int32_t* __restrict__ col,
+                                                  const float* __restrict__ val,
+                                                  const __nv_bfloat16* __restrict__ xb, int64_t ldx,
+                                                  int64_t beg, int64_t end, int lane, int c8n,
+                                                  float4 (&acc)[V][2]) {
+  constexpr int NG = 32 / G;
+  const int g = lane / G, sub = lane % G;
+#pragma unroll
+  for (int v = 0; v < V; ++v) acc[v][0] = acc[v][1] = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int64_t base = beg; base < end; base += 32) {
+    const int64_t j = base + lane;
+    int c = 0;
+    float a = 0.f;
+    if (j < end) {
+      c = __ldcs(col + j);
+      a = __ldcs(val + j);
+    }
+    const int cnt = (end - base) < 32 ? (int)(end - base) : 32;
+#pragma unroll
+    for (int t0 = 0; t0 < G; t0 += U) {
+      if (t0 * NG >= cnt) break;   // warp-uniform: the rest of the batch is past the row's end
+      uint4 x[U][V];
+      float vv[U];
+#pragma unroll
+      for (int u = 0; u < U; ++u) {
+        const int k = (t0 + u) * NG + g;
+        const int cc = (G == 1) ? c : __shfl_sync(kFull, c, k);
+        vv[u] = (G == 1) ? a : __shfl_sync(kFull, a, k);
+        const uint4* xr = reinterpret_cast<const uint4*>(xb + (int64_t)cc * ldx);
+#pragma unroll
+        for (int v = 0; v < V; ++v)
+          x[u][v] = (k < cnt && v * G + sub < c8n) ? __ldg(xr + v * G + sub) : make_uint4(0u, 0u, 0u, 0u);
+      }
+#pragma unroll
+      for (int u = 0; u < U; ++u)
+#pragma unroll
+        for (int v = 0; v < V; ++v) {
+          const uint32_t w4[4] = {x[u][v].x, x[u][v].y, x[u][v].z, x[u][v].w};
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            float4& A = acc[v][h];
+            A.x = fmaf(vv[u], __uint_as_float(w4[2 * h] << 16), A.x);
+            A.y = fmaf(vv[u], __uint_as_float(w4[2 * h] & 0xFFFF0000u), A.y);
+            A.z = fmaf(vv[u], __uint_as_float(w4[2 * h + 1] << 16), A.z);
+            A.w = fmaf(vv[u], __uint_as_float(w4[2 * h + 1] & 0xFFFF0000u), A.w);
+          }
+        }
+    }
+  }
+#pragma unroll
+  for (int off = G; off < 32; off <<= 1) {
+#pragma unroll
+    for (int v = 0; v < V; ++v)
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        acc[v][h].x += __shfl_xor_sync(kFull, acc[v][h].x, off);
+        acc[v][h].y += __shfl_xor_sync(kFull, acc[v][h].y, off);
+        acc[v][h].z += __shfl_xor_sync(kFull, acc[v][h].z, off);
+        acc[v][h].w += __shfl_xor_sync(kFull, acc[v][h].w, off);
+      }
+  }
+}
+
+// bf16 variant of spmm_kernel (same items, bins and epilogue); a vector is 8
+// columns, `w4` is the output's real padded width (stores stop there).
+// twice the accumulators of spmm_kernel: s = 2V + U·V slots
+constexpr int spmm_minb_bf(int V, int U) { return spmm_minb_slots(2 * V + U * V); }
+template <int G, int V, int U>
+__global__ void __launch_bounds__(kWarps * 32, spmm_minb_bf(V, U))
+spmm_kernel_bf(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
+               const float* __restrict__ val, const int32_t* __restrict__ light_rows,
+               const int64_t* __restrict__ seg_start, const int32_t* __restrict__ seg_row,
+               int64_t n_light, int64_t n_seg, const __nv_bfloat16* __restrict__ X, int64_t ldx,
+               float* __restrict__ out, int64_t ld_out, float* __restrict__ part, int64_t ld_part,
+               int64_t w4, int64_t w8, int chunk8, Epi epi) {
+  const int lane = threadIdx.x & 31;
+  const int64_t item = (int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5);
+  if (item >= n_seg + n_light) return;
+  const int64_t cbase = (int64_t)blockIdx.y * chunk8 * 8;
+  const int64_t rem8 = (w8 - cbase) / 8;
+  const int c8n = rem8 < chunk8 ? (int)rem8 : chunk8;
+  const int sub = lane % G;
+  float4 acc[V][2];
+  if (item < n_seg) {
+    const int32_t r = seg_row[item];
+    const int64_t beg = seg_start[item];
+    const int64_t end = min(beg + kSeg, rowptr[r + 1]);
+    warp_nnz_range_bf<G, V, U>(col, val, X + cbase, ldx, beg, end, lane, c8n, acc);
+    if (lane < G) {
+      float* dst = part + item * ld_part + cbase;
+#pragma unroll
+      for (int v = 0; v < V; ++v)
+        if (v * G + sub < c8n) {
+          reinterpret_cast<float4*>(dst)[2 * (v * G + sub)] = acc[v][0];
+          reinterpret_cast<float4*>(dst)[2 * (v * G + sub) + 1] = acc[v][1];
+        }
+    }
+  } else {
+    const int32_t r = light_rows[item - n_seg];
+    warp_nnz_range_bf<G, V, U>(col, val, X + cbase, ldx, rowptr[r], rowptr[r + 1], lane, c8n, acc);
+    if (lane < G) {
+      float* dst = out + (int64_t)r * ld_out;
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        const int ch = v * G + sub;
+        if (ch < c8n) {
+#pragma unroll
+          for (int h = 0; h < 2; ++h) {
+            const int64_t c = cbase + 8 * ch + 4 * h;
+            if (c < w4) {
+              const float4 o = apply_epi(acc[v][h], epi, r, c);
+              *reinterpret_cast<float4*>(dst + c) = o;
+              if (epi.scat.P) scatter_row_store(epi.scat, r, c, o);
+            }
+          }
+        }
+      }
+    }
+  }
+}
+
+// fp32 slice → bf16 copy (round to nearest even), row length ldy = w8, zero
+// pads: one thread per 8 columns.
+__global__ void to_bf16_kernel(const float* __restrict__ X, int64_t ldx, int64_t n, int64_t w4, int64_t w8,
+                               __nv_bfloat16* __restrict__ Y) {
+  const int64_t per = w8 / 8;
+  const int64_t total = n * per;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / per, c = (i - r * per) * 8;
+    const float* xr = X + r * ldx + c;
+    const float4 a = __ldcs(reinterpret_cast<const float4*>(xr));
+    const float4 b = (c + 4 < w4) ? __ldcs(reinterpret_cast<const float4*>(xr + 4)) : make_float4(0.f, 0.f, 0.f, 0.f);
+    __nv_bfloat162 p[4] = {__floats2bfloat162_rn(a.x, a.y), __floats2bfloat162_rn(a.z, a.w),
+                           __floats2bfloat162_rn(b.x, b.y), __floats2bfloat162_rn(b.z, b.w)};
+    *reinterpret_cast<uint4*>(Y + r * w8 + c) = *reinterpret_cast<const uint4*>(p);
   }
 }
 
@@ -241,7 +423,7 @@ __global__ void spmm_heavy_reduce(const int32_t* __restrict__ heavy_rows,
   }
 }
 
-template <int G, int V>
+template <int G, int V, int U>
 void launch_spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out,
                  int64_t ld_out, float* part, int64_t ld_part, int64_t w4, int chunk4,
                  const Epi& epi) {
@@ -249,11 +431,27 @@ void launch_spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, flo
   if (items == 0) return;
   const int64_t chunks = ceil_div(w4, 4 * chunk4);
   dim3 grid((unsigned)ceil_div(items, kWarps), (unsigned)chunks);
-  spmm_kernel<G, V><<<grid, kWarps * 32, 0, ctx->stream>>>(
+  spmm_kernel<G, V, U><<<grid, kWarps * 32, 0, ctx->stream>>>(
       A.rowptr->as<int64_t>(), A.col->as<int32_t>(), A.val->as<float>(),
       A.light_rows->as<int32_t>(), A.seg_start->as<int64_t>(),
       reinterpret_cast<const int32_t*>(A.seg_start->as<int64_t>() + A.n_seg), A.n_light, A.n_seg,
       in, ld_in, out, ld_out, part, ld_part, w4, chunk4, epi);
+  RDM_LAUNCHED(ctx);
+}
+
+template <int G, int V, int U>
+void launch_spmm_bf(rdm_ctx* ctx, const Csr& A, const __nv_bfloat16* in, int64_t ld_in, float* out,
+                    int64_t ld_out, float* part, int64_t ld_part, int64_t w4, int64_t w8, int chunk8,
+                    const Epi& epi) {
+  const int64_t items = A.n_seg + A.n_light;
+  if (items == 0) return;
+  const int64_t chunks = ceil_div(w8, 8 * chunk8);
+  dim3 grid((unsigned)ceil_div(items, kWarps), (unsigned)chunks);
+  spmm_kernel_bf<G, V, U><<<grid, kWarps * 32, 0, ctx->stream>>>(
+      A.rowptr->as<int64_t>(), A.col->as<int32_t>(), A.val->as<float>(),
+      A.light_rows->as<int32_t>(), A.seg_start->as<int64_t>(),
+      reinterpret_cast<const int32_t*>(A.seg_start->as<int64_t>() + A.n_seg), A.n_light, A.n_seg,
+      in, ld_in, out, ld_out, part, ld_part, w4, w8, chunk8, epi);
   RDM_LAUNCHED(ctx);
 }
 
@@ -278,7 +476,22 @@ void pick_gv(int c4, int* G, int* V) {
 }
 
 void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
-             int64_t w4, const Epi& epi);
+             int64_t w4, const Epi& epi, const __nv_bfloat16* inb);
+
+// (G, V, U) for a chunk of c 128-bit vectors per row (4 fp32 or 8 bf16
+// columns each).  Measured on the Reddit- and products-shaped residual CSRs
+// (tools/exp_gvu.py, profiles/r1_spmm_gvu.txt): for bf16 rows several nnz in
+// flight per group (U) pay; fp32 keeps U = 1 (best or tied at every width).
+void pick_gvu(int c, bool bf, int* G, int* V, int* U) {
+  pick_gv(c, G, V);
+  *U = 1;
+  if (bf) {
+    if (c >= 3 && c <= 8) { *G = 8; *V = 1; *U = 4; }
+    else if (c >= 9 && c <= 16) { *G = 8; *V = 2; *U = 2; }
+    else if (c >= 17 && c <= 32) { *G = 16; *V = 2; *U = 2; }
+    else if (c <= 2) *U = std::min(*G, 2);
+  }   // fp32: U = 1 measured best or tied at every width
+}
 
 // Hub-core cost model (B200-calibrated, profiles/r1_core_experiment.md): the
 // CSR SpMM spends ≈ 24 ps · (w/128)^0.55 per nnz (L2-gather bound), the core
@@ -363,18 +576,32 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
                   "spmm: bad scatter descriptor");
     epi.scat = *scat;
   }
-  if (A.core.n_tiles && hub_tiles_pay(A.core, w)) {
+  // RDM_PREC_FAST: one bf16 copy of the input slice per call, gathered by
+  // every row of the residual CSR (rdm.h rdm_set_precision)
+  const __nv_bfloat16* inb = nullptr;
+  if (ctx->prec == RDM_PREC_FAST) {
+    const int64_t w8 = (w4 + 7) & ~int64_t(7);
+    const int64_t nin = A.in_rows();
+    __nv_bfloat16* xb = reinterpret_cast<__nv_bfloat16*>(ensure_ws(ctx->ws_bf16, (size_t)std::max<int64_t>(nin, 1) * w8 * 2));
+    const int64_t total = nin * (w8 / 8);
+    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(total, 256), (int64_t)ctx->num_sms * 16));
+    to_bf16_kernel<<<grid, 256, 0, ctx->stream>>>(in, ld_in, nin, w4, w8, xb);
+    RDM_LAUNCHED(ctx);
+    inb = xb;
+  }
+  const int np = ctx->prec == RDM_PREC_FAST ? 1 : 3;
+  if (A.core.n_tiles && hub_tiles_pay(A.core, w, np)) {
     // binary hub tiles on the kind::f16 tensor cores (hubtiles.cu); the
     // residual CSR's epilogue adds s_i · Σ_items partial for hub rows.
     const int64_t ldp = w4;
     float* part = ensure_ws(ctx->ws_core_c, (size_t)A.core.n_items * 128 * ldp * sizeof(float));
-    hub_tiles_product(ctx, A.core, in, ld_in, w, part, ldp);
+    hub_tiles_product(ctx, A.core, in, ld_in, w, part, ldp, np);
     epi.tpart = part;
     epi.ld_tpart = ldp;
     epi.rb_item = A.core.rb_item->as<int32_t>();
     epi.tscale = A.core.scale->as<float>();
     epi.hub_slot = A.core.hub_slot->as<int32_t>();
-    run_csr(ctx, *A.core.resid, in, ld_in, out, ld_out, w4, epi);
+    run_csr(ctx, *A.core.resid, in, ld_in, out, ld_out, w4, epi, inb);
   } else if (A.core.K && core_pays(A.core, w)) {
     // hub core on the tensor cores: panels Bt[n][k] = split(X[hub_k][n]), then
     // C_core = Acore · X[hubs]; the residual CSR's epilogue adds C_core rows.
@@ -389,9 +616,9 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
     epi.core = cc;
     epi.ld_core = w4;
     epi.hub_slot = A.core.hub_slot->as<int32_t>();
-    run_csr(ctx, *A.core.resid, in, ld_in, out, ld_out, w4, epi);
+    run_csr(ctx, *A.core.resid, in, ld_in, out, ld_out, w4, epi, inb);
   } else {
-    run_csr(ctx, A, in, ld_in, out, ld_out, w4, epi);
+    run_csr(ctx, A, in, ld_in, out, ld_out, w4, epi, inb);
   }
   ctx->counters.spmm_calls++;
   ctx->counters.spmm_nnz_cols += A.nnz * w;
@@ -399,9 +626,11 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
 
 namespace {
 void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
-             int64_t w4, const Epi& epi) {
+             int64_t w4, const Epi& epi, const __nv_bfloat16* inb) {
+  const int64_t w8 = (w4 + 7) & ~int64_t(7);
+  const int64_t ldp = inb ? w8 : w4;
   float* part = nullptr;
-  if (A.n_seg) part = ensure_ws(ctx->ws_seg, (size_t)A.n_seg * w4 * sizeof(float));
+  if (A.n_seg) part = ensure_ws(ctx->ws_seg, (size_t)A.n_seg * ldp * sizeof(float));
   int G, V;
   // Column chunks (blockIdx.y, scheduled chunk after chunk): narrower chunks
   // keep the gathered slice L2-resident at the price of re-streaming the CSR.
@@ -411,20 +640,61 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
   // gain in L2 residency.
   int chunk4 = (w4 > 128 && w4 <= 256) ? 64 : 32;
   if (const char* e = getenv("RDM_SPMM_CHUNK4")) chunk4 = std::max(1, std::min(64, atoi(e)));
-  pick_gv((int)std::min<int64_t>(chunk4, w4 / 4), &G, &V);
-#define RDM_SPMM_CASE(g_, v_) \
-  if (G == g_ && V == v_) launch_spmm<g_, v_>(ctx, A, in, ld_in, out, ld_out, part, w4, w4, chunk4, epi); else
-  RDM_SPMM_CASE(1, 1) RDM_SPMM_CASE(1, 2) RDM_SPMM_CASE(1, 3) RDM_SPMM_CASE(1, 4)
-  RDM_SPMM_CASE(2, 1) RDM_SPMM_CASE(2, 2) RDM_SPMM_CASE(2, 3) RDM_SPMM_CASE(2, 4)
-  RDM_SPMM_CASE(4, 1) RDM_SPMM_CASE(4, 2) RDM_SPMM_CASE(4, 3) RDM_SPMM_CASE(4, 4)
-  RDM_SPMM_CASE(8, 1) RDM_SPMM_CASE(8, 2) RDM_SPMM_CASE(8, 3) RDM_SPMM_CASE(8, 4)
-  RDM_SPMM_CASE(16, 1) RDM_SPMM_CASE(16, 2) RDM_SPMM_CASE(16, 3) RDM_SPMM_CASE(16, 4)
-  RDM_SPMM_CASE(32, 1)
-  throw Error(RDM_ERR_STATE, "spmm: no kernel for G/V");
+  // U = nnz gathered per group before use (loads in flight); the default
+  // keeps ≈ 4 loads of 16 B in flight per lane
+  if (const char* e = getenv("RDM_SPMM_GV")) {   // experiments: "G,V"
+    G = atoi(e);
+    const char* c = strchr(e, ',');
+    V = c ? atoi(c + 1) : 1;
+  }
+  if (inb) {
+    // bf16 rows: the same column chunks, 8 columns per 128-bit gather
+    const int chunk8 = std::max(1, chunk4 / 2);
+    const int c8 = (int)std::min<int64_t>(chunk8, w8 / 8);
+    int U = 1;
+    if (!getenv("RDM_SPMM_GV")) pick_gvu(c8, true, &G, &V, &U);
+    if (const char* e = getenv("RDM_SPMM_U")) U = atoi(e);
+#define RDM_SPMM_CASE(g_, v_, u_) \
+  if (G == g_ && V == v_ && U == u_) launch_spmm_bf<g_, v_, u_>(ctx, A, inb, w8, out, ld_out, part, ldp, w4, w8, chunk8, epi); else
+    RDM_SPMM_CASE(1, 1, 1) RDM_SPMM_CASE(1, 2, 1) RDM_SPMM_CASE(1, 3, 1) RDM_SPMM_CASE(1, 4, 1)
+    RDM_SPMM_CASE(2, 1, 1) RDM_SPMM_CASE(2, 1, 2) RDM_SPMM_CASE(2, 2, 1) RDM_SPMM_CASE(2, 2, 2)
+    RDM_SPMM_CASE(2, 3, 1) RDM_SPMM_CASE(2, 3, 2) RDM_SPMM_CASE(2, 4, 1) RDM_SPMM_CASE(2, 4, 2)
+    RDM_SPMM_CASE(4, 1, 1) RDM_SPMM_CASE(4, 1, 2) RDM_SPMM_CASE(4, 1, 4) RDM_SPMM_CASE(4, 2, 1)
+    RDM_SPMM_CASE(4, 2, 2) RDM_SPMM_CASE(4, 2, 4) RDM_SPMM_CASE(4, 3, 1) RDM_SPMM_CASE(4, 3, 2)
+    RDM_SPMM_CASE(4, 4, 1) RDM_SPMM_CASE(4, 4, 2) RDM_SPMM_CASE(8, 1, 1) RDM_SPMM_CASE(8, 1, 2)
+    RDM_SPMM_CASE(8, 1, 4) RDM_SPMM_CASE(8, 2, 1) RDM_SPMM_CASE(8, 2, 2) RDM_SPMM_CASE(8, 2, 4)
+    RDM_SPMM_CASE(8, 3, 1) RDM_SPMM_CASE(8, 3, 2) RDM_SPMM_CASE(8, 4, 1) RDM_SPMM_CASE(8, 4, 2)
+    RDM_SPMM_CASE(16, 1, 1) RDM_SPMM_CASE(16, 1, 2) RDM_SPMM_CASE(16, 1, 4) RDM_SPMM_CASE(16, 2, 1)
+    RDM_SPMM_CASE(16, 2, 2) RDM_SPMM_CASE(16, 2, 4) RDM_SPMM_CASE(16, 3, 1) RDM_SPMM_CASE(16, 3, 2)
+    RDM_SPMM_CASE(16, 4, 1) RDM_SPMM_CASE(16, 4, 2) RDM_SPMM_CASE(32, 1, 1) RDM_SPMM_CASE(32, 1, 2)
+    RDM_SPMM_CASE(32, 1, 4)
+    throw Error(RDM_ERR_ARG, "spmm: no bf16 kernel for G/V/U");
 #undef RDM_SPMM_CASE
+  } else {
+    const int c4 = (int)std::min<int64_t>(chunk4, w4 / 4);
+    int U = 1;
+    if (!getenv("RDM_SPMM_GV")) pick_gvu(c4, false, &G, &V, &U);
+    if (const char* e = getenv("RDM_SPMM_U")) U = atoi(e);
+#define RDM_SPMM_CASE(g_, v_, u_) \
+  if (G == g_ && V == v_ && U == u_) launch_spmm<g_, v_, u_>(ctx, A, in, ld_in, out, ld_out, part, w4, w4, chunk4, epi); else
+    RDM_SPMM_CASE(1, 1, 1) RDM_SPMM_CASE(1, 2, 1) RDM_SPMM_CASE(1, 3, 1) RDM_SPMM_CASE(1, 4, 1)
+    RDM_SPMM_CASE(2, 1, 1) RDM_SPMM_CASE(2, 1, 2) RDM_SPMM_CASE(2, 2, 1) RDM_SPMM_CASE(2, 2, 2)
+    RDM_SPMM_CASE(2, 3, 1) RDM_SPMM_CASE(2, 3, 2) RDM_SPMM_CASE(2, 4, 1) RDM_SPMM_CASE(2, 4, 2)
+    RDM_SPMM_CASE(4, 1, 1) RDM_SPMM_CASE(4, 1, 2) RDM_SPMM_CASE(4, 1, 4) RDM_SPMM_CASE(4, 2, 1)
+    RDM_SPMM_CASE(4, 2, 2) RDM_SPMM_CASE(4, 2, 4) RDM_SPMM_CASE(4, 3, 1) RDM_SPMM_CASE(4, 3, 2)
+    RDM_SPMM_CASE(4, 4, 1) RDM_SPMM_CASE(4, 4, 2) RDM_SPMM_CASE(8, 1, 1) RDM_SPMM_CASE(8, 1, 2)
+    RDM_SPMM_CASE(8, 1, 4) RDM_SPMM_CASE(8, 2, 1) RDM_SPMM_CASE(8, 2, 2) RDM_SPMM_CASE(8, 2, 4)
+    RDM_SPMM_CASE(8, 3, 1) RDM_SPMM_CASE(8, 3, 2) RDM_SPMM_CASE(8, 4, 1) RDM_SPMM_CASE(8, 4, 2)
+    RDM_SPMM_CASE(16, 1, 1) RDM_SPMM_CASE(16, 1, 2) RDM_SPMM_CASE(16, 1, 4) RDM_SPMM_CASE(16, 2, 1)
+    RDM_SPMM_CASE(16, 2, 2) RDM_SPMM_CASE(16, 2, 4) RDM_SPMM_CASE(16, 3, 1) RDM_SPMM_CASE(16, 3, 2)
+    RDM_SPMM_CASE(16, 4, 1) RDM_SPMM_CASE(16, 4, 2) RDM_SPMM_CASE(32, 1, 1) RDM_SPMM_CASE(32, 1, 2)
+    RDM_SPMM_CASE(32, 1, 4)
+    throw Error(RDM_ERR_ARG, "spmm: no kernel for G/V/U");
+#undef RDM_SPMM_CASE
+  }
   if (A.n_heavy) {
     spmm_heavy_reduce<<<(unsigned)A.n_heavy, 128, 0, ctx->stream>>>(
-        A.heavy_rows->as<int32_t>(), A.heavy_seg->as<int32_t>(), part, w4, out, ld_out, w4, epi);
+        A.heavy_rows->as<int32_t>(), A.heavy_seg->as<int32_t>(), part, ldp, out, ld_out, w4, epi);
     RDM_LAUNCHED(ctx);
   }
 }

@@ -152,3 +152,74 @@ def test_fig7_two_process_roundtrip():
     back = rd.redistribute_col2row(cols, 2)
     for a, b in zip(rows, back):
         assert np.array_equal(a.view(np.uint32), b.view(np.uint32))
+
+
+# ------------------------------------------------- R_A < P (§III-E, NEXT-4)
+import random as _random
+
+
+def test_ra_equals_p_reduces_to_full_replication():
+    """At R_A = P the broadcast term vanishes and every redistribution moves
+    (P−1)/P·N·f (L142): the R_A rows reduce to the plain Table II/III rows."""
+    rng = _random.Random(5)
+    for _ in range(200):
+        f = [rng.randint(1, 700) for _ in range(rng.choice([3, 4]))]
+        n, P = rng.randint(1, 10 ** 6), rng.choice([1, 2, 4, 8])
+        for cid in range(4 ** (len(f) - 1)):
+            c, _ = cm.simulate(cid, f)
+            assert cm.comm_elements_ra(cid, f, n, P, P) == pytest.approx((P - 1) / P * n * c)
+
+
+def test_ra_one_is_cagnet_1d():
+    """R_A = 1 is the 1D scheme of CAGNET [4] (L152-153): no redistribution
+    inside a one-GPU panel group, (P−1)·N·f broadcast per SpMM of width f."""
+    f = [602, 128, 41]
+    for cid in range(16):
+        _, s = cm.simulate(cid, f)
+        assert cm.comm_elements_ra(cid, f, 1000, 8, 1) == pytest.approx(7 * 1000 * s)
+
+
+def test_ra_gt_one_moves_less_than_half_of_ra_one():
+    """L153-154: "when R_A > 1 the data movement will be less than half of the
+    R_A = 1 case" — for the SpMM broadcast, (P/R_A − 1) < (P − 1)/2."""
+    for P in (4, 8, 16, 64):
+        for RA in [r for r in range(2, P + 1) if P % r == 0]:
+            assert (P / RA - 1) < (P - 1) / 2
+            assert cm.layer_comm_ra(128, 1000, P, RA) < 0.5 * cm.layer_comm_ra(128, 1000, P, 1) + \
+                (RA - 1) / RA * 1000 * 128
+
+
+def test_ra_table_ii_row_fig6():
+    """Table II "Comm. (R_A < P)" for Fig. 6 (P = 4, R_A = 2): a forward
+    SpMM-first layer moves (1/2)·N·f (redistribution in the 1x2 group) +
+    1·N·f (broadcast between P0/P2 and P1/P3)."""
+    assert cm.layer_comm_ra(16, 100, 4, 2) == pytest.approx(0.5 * 100 * 16 + 100 * 16)
+    # the simulator agrees for a 1-layer S-first model (SpMM width f0, one redistribution f0, loss free)
+    f = [16, 16]
+    fwd_S_bwd_S = cm.encode({1: 0}, {1: 0}, 1)
+    comm, sparse = cm.simulate(fwd_S_bwd_S, f)
+    assert cm.comm_elements_ra(fwd_S_bwd_S, f, 100, 4, 2) == pytest.approx(
+        100 * (0.5 * comm + 1 * sparse))
+
+
+def test_max_replication_formula():
+    """L160-167: R_A = P·(M − H_all)/G, capped at P, a divisor of P (R36)."""
+    GB = 1e9
+    # papers100M-shaped (13.7 GB CSR) on 8 x 180 GB: full replication fits
+    assert cm.max_replication(8, 180 * GB, 100 * GB, 13.7 * GB) == 8
+    # 40 GB free per GPU, 100 GB graph: 8·40/100 = 3.2 → 2 (largest divisor of 8 ≤ 3)
+    assert cm.max_replication(8, 80 * GB, 40 * GB, 100 * GB) == 2
+    assert cm.max_replication(8, 80 * GB, 40 * GB, 300 * GB) == 1
+    assert cm.max_replication(8, 80 * GB, 79 * GB, 300 * GB) == 0
+    assert cm.max_replication(6, 80 * GB, 40 * GB, 60 * GB) == 3
+
+
+def test_ra_pareto_shifts_to_narrow_spmm():
+    """With R_A < P the SpMM widths are charged communication too, so the
+    front favours configurations with fewer sparse units (Reddit-shaped)."""
+    f, n = [602, 128, 41], 232965
+    front_full = cm.pareto_ra(f, n, 8, 8)
+    assert front_full == cm.pareto_front(f)
+    front_1 = cm.pareto_ra(f, n, 8, 1)
+    best_sparse = min(cm.simulate(i, f)[1] for i in range(16))
+    assert all(cm.simulate(i, f)[1] == best_sparse for i in front_1)

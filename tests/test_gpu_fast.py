@@ -1,0 +1,187 @@
+"""GPU parity of the RDM_PREC_FAST variant (rdm.h
+rdm_set_precision): bf16 SpMM operand with fp32 accumulation, one bf16 piece
+in the binary hub tiles, 1xTF32 GEMMs.
+
+Gates:
+* north star "2e-2 if a bf16 GEMM variant is enabled" for every layer output,
+  gradient and the composed epoch (max relative error per tensor, R26);
+* tighter pins on what the variant computes: without hub tiles the SpMM is
+  exactly A·bf16(X) accumulated in fp32 (compared with the fp64 oracle applied
+  to the bf16-rounded input, fp32 gate 1e-4); the GEMMs are tf32 products
+  (5e-3, a few tf32 unit round-offs 2^-11);
+* redistribution stays bit-exact (pure data movement, unchanged).
+The bf16 rounding below is test-side (round to nearest even on the fp32 bit
+pattern), not library code."""
+import numpy as np
+import pytest
+
+import synth
+from oracle import gcn as og
+
+from test_gpu_gcn import _check, _problem, _run
+
+pytestmark = pytest.mark.gpu
+
+GATE = 2e-2
+
+
+def bf16_rne(x):
+    u = np.ascontiguousarray(x, np.float32).view(np.uint32).astype(np.uint64)
+    r = ((u + 0x7FFF + ((u >> 16) & 1)) >> 16) << 16
+    return r.astype(np.uint32).view(np.float32)
+
+
+@pytest.fixture(scope="module")
+def torch_dev():
+    import torch
+    return torch, torch.device("cuda:0")
+
+
+@pytest.fixture(scope="module")
+def rdm():
+    import paper_conf_ipps_kurtysps23_b200 as r
+    return r
+
+
+def _padded(torch, dev, X):
+    n, w = X.shape
+    t = torch.zeros((n, (w + 3) // 4 * 4), dtype=torch.float32, device=dev)
+    t[:, :w] = torch.from_numpy(np.ascontiguousarray(X, np.float32)).to(dev)
+    return t
+
+
+def test_bf16_rounding_helper():
+    x = np.array([1.0, 1.0 + 2**-8, 1.0 + 2**-7 + 2**-8, 3.0e38, -2.5, 0.0], np.float32)
+    got = bf16_rne(x)
+    assert got[0] == 1.0 and got[1] == 1.0            # tie → even
+    assert got[2] == np.float32(1.0 + 2**-6)          # tie → even (up)
+    assert got[4] == -2.5 and got[5] == 0.0
+
+
+FAST_GRAPHS = {
+    "rmat_cora": lambda: synth.rmat(2708, 5278, seed=1),
+    "directed_empty_rows": lambda: synth.random_directed(3000, 40000, seed=5, empty_rows=50),
+    "star_heavy": lambda: synth.star_graph(9000),
+    "rmat_skewed": lambda: synth.rmat(20000, 400000, seed=3),
+}
+
+
+@pytest.mark.parametrize("gname", list(FAST_GRAPHS))
+@pytest.mark.parametrize("w", [1, 3, 5, 16, 41, 128, 130, 256, 301])
+def test_fast_spmm_is_bf16_input_fp32_accumulate(torch_dev, rdm, gname, w, monkeypatch):
+    torch, dev = torch_dev
+    monkeypatch.setenv("RDM_NO_TILES", "1")
+    monkeypatch.setenv("RDM_NO_CORE", "1")
+    g = FAST_GRAPHS[gname]()
+    sym = gname != "directed_empty_rows"
+    ctx = rdm.Context(device=0)
+    ctx.set_precision("fast")
+    assert ctx.precision == "fast"
+    ctx.set_graph(g.rowptr, g.col, g.val, symmetric=sym)
+    rng = np.random.default_rng(w)
+    X = rng.standard_normal((g.n, w)).astype(np.float32)
+    xd = _padded(torch, dev, X)
+    for transpose in ([0, 1] if not sym else [0]):
+        out = torch.zeros_like(xd)
+        ctx.spmm(transpose, xd, out, w, rdm.EPI_RELU)
+        ctx.sync()
+        f = og.spmm_t if transpose else og.spmm
+        got = out[:, :w].cpu().numpy()
+        exact = np.maximum(f(g, bf16_rne(X)), 0)
+        assert og.max_rel_err(got, exact) < 1e-4               # what the variant computes
+        assert og.max_rel_err(got, np.maximum(f(g, X), 0)) < GATE  # vs the plain product
+        assert np.all(out[:, w:].cpu().numpy() == 0)
+
+
+@pytest.mark.parametrize("w", [4, 16, 41, 128, 256])
+@pytest.mark.parametrize("min_nnz", [1, 40])
+def test_fast_spmm_hub_tiles(torch_dev, rdm, w, min_nnz, monkeypatch):
+    """One bf16 piece of s⊙X on the kind::f16 tensor cores + bf16 residual CSR."""
+    torch, dev = torch_dev
+    monkeypatch.setenv("RDM_TILE_MIN_NNZ", str(min_nnz))
+    g = synth.rmat(6000, 150000, seed=13)
+    ctx = rdm.Context(device=0)
+    ctx.set_precision("fast")
+    ctx.set_graph(g.rowptr, g.col, g.val)
+    assert ctx.graph_info()["n_tiles"] > 0
+    rng = np.random.default_rng(w)
+    X = rng.standard_normal((g.n, w)).astype(np.float32)
+    M = rng.standard_normal((g.n, w)).astype(np.float32)
+    xd, md = _padded(torch, dev, X), _padded(torch, dev, M)
+    out = torch.zeros_like(xd)
+    ctx.spmm(0, xd, out, w, rdm.EPI_RELU | rdm.EPI_MASK, mask=md)
+    ctx.sync()
+    ref = np.maximum(og.spmm(g, X), 0) * (M > 0)
+    err = og.max_rel_err(out[:, :w].cpu().numpy(), ref)
+    assert err < 1e-2, err
+    assert np.all(out[:, w:].cpu().numpy() == 0)
+
+
+GEMM_SHAPES = [(1000, 7, 128), (2049, 41, 128), (777, 128, 41), (3000, 602, 128),
+               (513, 128, 602), (4097, 256, 256), (300, 100, 256), (1, 128, 47), (130, 1433, 128)]
+
+
+@pytest.mark.parametrize("rows,k,m", GEMM_SHAPES)
+def test_fast_gemm_tf32(torch_dev, rdm, rows, k, m):
+    torch, dev = torch_dev
+    ctx = rdm.Context(device=0)
+    ctx.set_precision("fast")
+    rng = np.random.default_rng(rows + k + m)
+    X = rng.standard_normal((rows, k)).astype(np.float32)
+    W = rng.standard_normal((k, m)).astype(np.float32)
+    G = rng.standard_normal((rows, m)).astype(np.float32)
+    Xd, Gd = _padded(torch, dev, X), _padded(torch, dev, G)
+    Wd = torch.from_numpy(W).to(dev)
+    C = torch.zeros((rows, (m + 3) // 4 * 4), device=dev)
+    ctx.gemm(rdm.GEMM_NN, Xd, Wd, C, rows, k, m, rdm.EPI_RELU)
+    D = torch.zeros((rows, (k + 3) // 4 * 4), device=dev)
+    ctx.gemm(rdm.GEMM_NT, Gd, Wd, D, rows, k, m)
+    Y = torch.zeros((k, m), device=dev)
+    ctx.gemm(rdm.GEMM_TN, Xd, Gd, Y, rows, k, m)
+    ctx.sync()
+    X64, W64, G64 = X.astype(np.float64), W.astype(np.float64), G.astype(np.float64)
+    assert og.max_rel_err(C[:, :m].cpu().numpy(), np.maximum(X64 @ W64, 0)) < 5e-3
+    assert og.max_rel_err(D[:, :k].cpu().numpy(), G64 @ W64.T) < 5e-3
+    assert og.max_rel_err(Y.cpu().numpy(), X64.T @ G64) < 5e-3
+    # and it is a different (cheaper) arithmetic than the default 3xTF32
+    ctx.set_precision("fp32")
+    C3 = torch.zeros_like(C)
+    ctx.gemm(rdm.GEMM_NN, Xd, Wd, C3, rows, k, m, rdm.EPI_RELU)
+    ctx.sync()
+    assert og.max_rel_err(C3[:, :m].cpu().numpy(), np.maximum(X64 @ W64, 0)) < 1e-4
+
+
+@pytest.fixture(scope="module")
+def cora():
+    return _problem()
+
+
+@pytest.mark.parametrize("P", [1, 4])
+@pytest.mark.parametrize("cfg", [2, 3, 5, 10, 15])
+def test_fast_epoch_within_gate(rdm, cora, P, cfg):
+    g, H0, Ws, y, m = cora
+    loss, dW, model, ctx, _ = _run(rdm, g, H0, Ws, y, m, cfg, P=P, precision="fast")
+    _check((g, H0, Ws, y, m), loss, dW, model, rdm, P=P, tol=GATE, ltol=1e-3)
+
+
+def test_fast_three_layer_products_shaped(rdm):
+    prob = _problem(n=6000, E=40000, f=(100, 256, 256, 47), seed=2)
+    g, H0, Ws, y, m = prob
+    loss, dW, model, ctx, _ = _run(rdm, g, H0, Ws, y, m, 9, P=2, precision="fast")
+    _check(prob, loss, dW, model, rdm, P=2, tol=GATE, ltol=1e-3)
+
+
+@pytest.mark.parametrize("cfg", [3, 10])
+def test_fast_epoch_hub_tiles(rdm, cfg, monkeypatch):
+    monkeypatch.setenv("RDM_TILE_MIN_NNZ", "20")
+    prob = _problem(n=8000, E=200000, f=(64, 128, 41), seed=5)
+    g, H0, Ws, y, m = prob
+    loss, dW, model, ctx, _ = _run(rdm, g, H0, Ws, y, m, cfg, precision="fast")
+    assert ctx.graph_info()["n_tiles"] > 0
+    _check(prob, loss, dW, model, rdm, tol=GATE, ltol=1e-3)
+
+
+def test_precision_rejects_unknown(rdm):
+    ctx = rdm.Context(device=0)
+    with pytest.raises(rdm.RdmError):
+        ctx._c(rdm._lib.rdm_set_precision(ctx.h, 7))

@@ -22,7 +22,7 @@ def rdm():
     return r
 
 
-def _run(rdm, g, H0, Ws, y, m, cfg, P=1, epochs=1, transport="nccl"):
+def _run(rdm, g, H0, Ws, y, m, cfg, P=1, epochs=1, transport="nccl", precision="fp32"):
     """Run `epochs` epochs (fwd, bwd, Adam) on P ranks (virtual group if P > 1);
     returns loss, dW (of the last epoch), model, ctx and the weights."""
     import torch
@@ -33,6 +33,7 @@ def _run(rdm, g, H0, Ws, y, m, cfg, P=1, epochs=1, transport="nccl"):
     else:
         ctx = rdm.Context(rank=rdm.ALL_RANKS, world=P, device=0)
     ctx.set_transport(transport)
+    ctx.set_precision(precision)
     ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
     model = rdm.GCN(ctx, f, cfg)
     Hs, ys, ms = [], [], []
@@ -94,7 +95,7 @@ def _gather(model, rdm, which, layer, n, width, P):
     raise AssertionError(f"tensor {which}/{layer} not resident")
 
 
-def _check(prob, loss, dW, model, rdm, P=1, check_g0=True):
+def _check(prob, loss, dW, model, rdm, P=1, check_g0=True, tol=1e-4, ltol=1e-5):
     """Compare with the fp64 oracle.  The ReLU decisions 1[Z^l > 0] are taken from
     the kernel's own fp32 forward (reading R30: a float-decided discrete value is
     decided in the kernel's precision on both sides); everything else is fp64.
@@ -107,18 +108,18 @@ def _check(prob, loss, dW, model, rdm, P=1, check_g0=True):
     ref = og.epoch(g, H0, Ws, y, m, relu_masks=[h > 0 for h in Hs])
     # forward parity (independent of the masks)
     for l in range(1, L):
-        assert og.max_rel_err(Hs[l - 1], og.relu(ref.Z[l])) < 1e-4, ("H", l)
+        assert og.max_rel_err(Hs[l - 1], og.relu(ref.Z[l])) < tol, ("H", l)
     flips = sum(int(((h > 0) != (ref.Z[l + 1] > 0)).sum()) for l, h in enumerate(Hs))
-    assert flips <= max(2, 1e-4 * n * max(f)), flips
-    assert abs(loss - ref.loss) <= 1e-5 * abs(ref.loss), (loss, ref.loss)
+    assert flips <= max(2, tol * n * max(f)), flips   # sign decisions within the precision band
+    assert abs(loss - ref.loss) <= ltol * abs(ref.loss), (loss, ref.loss)
     for l in range(L):
         err = og.max_rel_err(dW[l], ref.Y[l + 1])
-        assert err < 1e-4, (l + 1, err)
+        assert err < tol, (l + 1, err)
     Z = _gather(model, rdm, rdm.T_Z, 0, n, f[L], P)
-    assert og.max_rel_err(Z, ref.Z[L]) < 1e-4
+    assert og.max_rel_err(Z, ref.Z[L]) < tol
     if check_g0:
         G0 = _gather(model, rdm, rdm.T_G, 0, n, f[0], P)
-        assert og.max_rel_err(G0, ref.G[0]) < 1e-4
+        assert og.max_rel_err(G0, ref.G[0]) < tol
 
 
 @pytest.mark.parametrize("cfg", list(range(16)))
