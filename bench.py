@@ -49,6 +49,9 @@ def parse():
     ap.add_argument("--precision", default="fp32", choices=["fp32", "fast"],
                     help="operator arithmetic (rdm.h rdm_set_precision): fp32 (1e-4 gate) or fast "
                          "(bf16 SpMM operand + 1xTF32 GEMM, 2e-2 gate)")
+    ap.add_argument("--ra", type=int, default=0,
+                    help="R_A < P partial replication (rdm.h rdm_set_graph_panels): replicas of A; "
+                         "0 = full replication (R_A = P)")
     ap.add_argument("--no-variants", action="store_true",
                     help="skip the extra timing of the fast-precision variant")
     ap.add_argument("--saint", action="store_true",
@@ -422,8 +425,13 @@ def main():
                       unique_id=uid)
     ctx.set_transport(a.transport)
     ctx.set_precision(a.precision)
-    ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
-    pareto, chosen, comm_u, sparse_u = rdm.select_config(list(wl.f), wl.n, wl.nnz, world)
+    panels = 0 < a.ra < world
+    if panels:   # §III-E: R_A copies of A, row panels; tiles + column-group broadcasts
+        ctx.set_graph_panels(a.ra, g.rowptr, g.col, g.val)
+        pareto, chosen, _, _ = rdm.select_config_ra(list(wl.f), wl.n, wl.nnz, world, a.ra)
+    else:
+        ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
+        pareto, chosen, comm_u, sparse_u = rdm.select_config(list(wl.f), wl.n, wl.nnz, world)
     lo, hi, _ = rdm.partition(world, rdm.ROW, wl.n, wl.f[0], rank if world > 1 else 0)
     H0_pin = torch.from_numpy(H0[lo:hi]).pin_memory()
     y_pin = torch.from_numpy(y[lo:hi]).pin_memory()
@@ -440,7 +448,7 @@ def main():
     def build(cfg):
         if "model" in cur:
             cur["model"].close()
-        m = rdm.GCN(ctx, wl.f, cfg)
+        m = rdm.GCN(ctx, wl.f, cfg, panels=panels)
         m.set_input([H0_d], [y_d], [m_d])
         cur["model"] = m
         return m
@@ -618,7 +626,7 @@ def main():
                 "n": n, "nnz": nnz, "graph": "R-MAT (0.57,0.19,0.19,0.05), permuted, symmetric, "
                 "self loops, D^-1/2 (A+I) D^-1/2", "global_batch": n, "seq_len": None,
                 "parallelism": f"rdm{world} (A replicated, H row/col redistributed)",
-                "transport": a.transport,
+                "transport": a.transport, "replicas_of_A": a.ra if panels else world,
                 "config_id": cfg_id, "config_name": rdm.config_name(model.cfg),
                 "pareto": pareto, "pick": a.config,
                 "sweep_ms": ({str(k): round(v, 4) for k, v in sweep.items()} if sweep else None),
@@ -632,6 +640,7 @@ def main():
             "phases_ms_per_step": {k: v / a.steps for k, v in ph_ms.items()},
             "spmm_hbm_gbs": achieved, "a2a_bus_gbs": a2a_bus,
             "a2a_bytes_per_step": cnt["a2a_bytes_wire"] / a.steps,
+            "bcast_elems_per_step": cnt["bcast_elems"] / a.steps,
             "loss": loss_main, "variants": variants,
         }
         print(json.dumps(line), flush=True)

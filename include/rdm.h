@@ -108,7 +108,12 @@ typedef struct {
 enum {
   RDM_GCN_INPUT_GRAD = 1, /* also compute G^0 = A G^1 (W^1)ᵀ (Fig. 4 output; reading R2) —
                              required for costs to match Table IV                       */
-  RDM_GCN_BIAS = 2        /* Z = Â H W + 1 bᵀ (reading R8); not implemented: UNSUPPORTED */
+  RDM_GCN_BIAS = 2,       /* Z = Â H W + 1 bᵀ (reading R8); not implemented: UNSUPPORTED */
+  RDM_GCN_PANELS = 4      /* R_A < P (§III-E): run on the row panels installed by
+                             rdm_set_graph_panels (a symmetric A) instead of the replicated
+                             graph; column-layout tensors are tiles (rdm_partition_tile),
+                             SpMMs broadcast input tiles inside column groups, redistributions
+                             stay inside panel groups; RDM_TRANSPORT_P2P fusion is not used */
 };
 
 /* Tensors exposed by rdm_gcn_tensor (for parity tests / inspection). */
@@ -335,6 +340,15 @@ rdm_status rdm_spmm_panels(rdm_ctx* ctx, const float* const* in_tiles, float* co
                            int64_t f, int epilogue, const float* bias, const float* const* mask_tiles);
 int rdm_max_replication(int world, double mem_bytes_per_gpu, double h_all_bytes_per_gpu,
                         double graph_bytes);
+/* Configuration choice at R_A < P (reading R35): each config's elements moved
+ * per epoch = N·[(R_A−1)/R_A·comm_units + (P/R_A−1)·sparse_units] (Tables
+ * II/III R_A rows); Pareto-optimal configs in (elements, sparse units) into
+ * pareto_ids (*n_pareto: capacity in, count out) and the pick of the same
+ * B200 time model as rdm_select_config.  R_A = P reproduces rdm_select_config's
+ * front.  Pure host function.  Errors: RDM_ERR_ARG (R_A ∤ P, sizes). */
+rdm_status rdm_select_config_ra(int L, const int64_t* f, int64_t n, int64_t nnz, int P, int R_A,
+                                int need_input_grad, int64_t* pareto_ids, int* n_pareto,
+                                int64_t* chosen_id, double* comm_elems, int64_t* sparse_units);
 
 /* In-place sum over all ranks of count floats per local slot (weight-gradient
  * reduction, reading R16).  Virtual group: every slot receives the sum. */

@@ -31,7 +31,7 @@ GEMM_NN, GEMM_NT, GEMM_TN = 0, 1, 2
 ALL_RANKS = -1
 MAX_LAYERS = 8
 UNIQUE_ID_BYTES = 128
-GCN_INPUT_GRAD, GCN_BIAS = 1, 2
+GCN_INPUT_GRAD, GCN_BIAS, GCN_PANELS = 1, 2, 4
 T_H, T_Z, T_G, T_MEMO, T_DWP = range(5)
 PHASES = ["spmm", "gemm", "pack", "a2a", "loss", "allreduce", "adam", "other", "sample"]
 _STATUS = {0: "OK", 1: "ERR_ARG", 2: "ERR_CUDA", 3: "ERR_NCCL", 4: "ERR_OOM",
@@ -51,7 +51,8 @@ EXPORTS = [
     "rdm_adam_step", "rdm_get_counters", "rdm_reset_counters", "rdm_set_timing",
     "rdm_get_phase_times", "rdm_reset_phase_times", "rdm_redist_plan", "rdm_plan_info",
     "rdm_set_transport", "rdm_get_transport", "rdm_debug_disable_tc",
-    "rdm_set_precision", "rdm_get_precision",
+    "rdm_set_precision", "rdm_get_precision", "rdm_set_graph_panels", "rdm_partition_tile",
+    "rdm_redistribute_panels", "rdm_spmm_panels", "rdm_max_replication", "rdm_select_config_ra",
 ]
 
 
@@ -115,6 +116,12 @@ _sig = {
     "rdm_set_timing": [_vp, _int],
     "rdm_set_transport": [_vp, _int],
     "rdm_set_precision": [_vp, _int],
+    "rdm_select_config_ra": [_int, _pi64, _i64, _i64, _int, _int, _int, _pi64, ctypes.POINTER(_int),
+                             _pi64, ctypes.POINTER(ctypes.c_double), _pi64],
+    "rdm_set_graph_panels": [_vp, _int, _i64, _i64, _vp, _vp, _vp, _int],
+    "rdm_partition_tile": [_int, _int, _i64, _i64, _int, _pi64, _pi64, _pi64, _pi64, _pi64],
+    "rdm_redistribute_panels": [_vp, _int, _pp, _pp, _i64, _i64],
+    "rdm_spmm_panels": [_vp, _pp, _pp, _i64, _int, _vp, _pp],
     "rdm_get_phase_times": [_vp, ctypes.POINTER(ctypes.c_double), _pi64],
     "rdm_reset_phase_times": [_vp],
     "rdm_redist_plan": [_int, _int, _int, _i64, _i64, _pi64, _pi64, _pi64, _pi64],
@@ -128,13 +135,15 @@ _lib.rdm_last_error.argtypes = [_vp]
 _lib.rdm_last_error.restype = ctypes.c_char_p
 _lib.rdm_config_to_id.argtypes = [ctypes.POINTER(RdmConfig)]
 _lib.rdm_config_to_id.restype = _i64
-for _n in ("rdm_world", "rdm_num_local", "rdm_get_transport"):
+for _n in ("rdm_world", "rdm_num_local", "rdm_get_transport", "rdm_get_precision"):
     getattr(_lib, _n).argtypes = [_vp]
     getattr(_lib, _n).restype = _int
 _lib.rdm_debug_disable_tc.argtypes = [_int]
 _lib.rdm_debug_disable_tc.restype = _int
 _lib.rdm_local_rank.argtypes = [_vp, _int]
 _lib.rdm_local_rank.restype = _int
+_lib.rdm_max_replication.argtypes = [_int, ctypes.c_double, ctypes.c_double, ctypes.c_double]
+_lib.rdm_max_replication.restype = _int
 
 
 class RdmError(RuntimeError):
@@ -191,6 +200,35 @@ def partition(world, layout, n, f, rank):
     _check(_lib.rdm_partition(world, layout, n, f, rank, ctypes.byref(lo), ctypes.byref(hi),
                               ctypes.byref(ld)), what="rdm_partition")
     return lo.value, hi.value, ld.value
+
+
+def partition_tile(world, r_a, n, f, rank):
+    """Tile of `rank` in the R_A < P grid (rdm.h rdm_partition_tile):
+    (row_lo, row_hi, col_lo, col_hi, ld)."""
+    v = [_i64() for _ in range(5)]
+    _check(_lib.rdm_partition_tile(world, r_a, n, f, rank, *[ctypes.byref(x) for x in v]),
+           what="rdm_partition_tile")
+    return tuple(x.value for x in v)
+
+
+def select_config_ra(f, n, nnz, P, r_a, input_grad=True):
+    """R_A < P configuration choice (rdm.h rdm_select_config_ra):
+    (pareto ids, chosen id, elements moved per epoch, sparse units)."""
+    L = len(f) - 1
+    fa = (ctypes.c_int64 * len(f))(*f)
+    cap = 4 ** L
+    ids = (ctypes.c_int64 * cap)()
+    npar = _int(cap)
+    ch, ce, su = _i64(), ctypes.c_double(), _i64()
+    _check(_lib.rdm_select_config_ra(L, fa, n, nnz, P, r_a, int(input_grad), ids, ctypes.byref(npar),
+                                     ctypes.byref(ch), ctypes.byref(ce), ctypes.byref(su)),
+           what="rdm_select_config_ra")
+    return list(ids[:npar.value]), ch.value, ce.value, su.value
+
+
+def max_replication(world, mem_bytes, h_all_bytes, graph_bytes) -> int:
+    """Largest feasible R_A (rdm.h rdm_max_replication)."""
+    return int(_lib.rdm_max_replication(world, float(mem_bytes), float(h_all_bytes), float(graph_bytes)))
 
 
 def config_from_id(L, cfg_id) -> RdmConfig:
@@ -308,6 +346,24 @@ class Context:
         dp, _b = _parr(dsts)
         self._c(_lib.rdm_redistribute(self.h, from_layout, sp, dp, n, f))
 
+    def set_graph_panels(self, r_a, rowptr, col, val):
+        """Row panels of A for R_A < P (rdm.h rdm_set_graph_panels)."""
+        on_host = not hasattr(rowptr, "data_ptr") or not rowptr.is_cuda
+        n = len(rowptr) - 1
+        self._c(_lib.rdm_set_graph_panels(self.h, r_a, n, int(rowptr[-1]), _ptr(rowptr), _ptr(col),
+                                          _ptr(val), int(on_host)))
+
+    def redistribute_panels(self, from_layout, srcs, dsts, n, f):
+        sp, _a = _parr(srcs)
+        dp, _b = _parr(dsts)
+        self._c(_lib.rdm_redistribute_panels(self.h, from_layout, sp, dp, n, f))
+
+    def spmm_panels(self, ins, outs, f, epilogue=EPI_NONE, bias=None, masks=None):
+        ip, _a = _parr(ins)
+        op, _b = _parr(outs)
+        mp, _c2 = _parr(masks) if masks is not None else (None, None)
+        self._c(_lib.rdm_spmm_panels(self.h, ip, op, f, epilogue, _ptr(bias), mp))
+
     def allreduce_sum(self, bufs):
         bp, _a = _parr(bufs)
         self._c(_lib.rdm_allreduce_sum(self.h, bp, bufs[0].numel()))
@@ -365,14 +421,14 @@ class Context:
 class GCN:
     """A GCN instance (L layers, widths f) running configuration `cfg` (ID or RdmConfig)."""
 
-    def __init__(self, ctx: Context, f, cfg, input_grad=True, saint=None):
+    def __init__(self, ctx: Context, f, cfg, input_grad=True, saint=None, panels=False):
         self.ctx = ctx
         self.f = list(f)
         self.L = len(f) - 1
         self.cfg = config_from_id(self.L, cfg) if isinstance(cfg, int) else cfg
         fa = (ctypes.c_int64 * len(f))(*f)
         h = ctypes.c_void_p()
-        flags = GCN_INPUT_GRAD if input_grad else 0
+        flags = (GCN_INPUT_GRAD if input_grad else 0) | (GCN_PANELS if panels else 0)
         self.saint = saint   # keeps the sampler alive while this instance exists
         if saint is None:
             ctx._c(_lib.rdm_gcn_create(ctx.h, self.L, fa, ctypes.byref(self.cfg), flags,

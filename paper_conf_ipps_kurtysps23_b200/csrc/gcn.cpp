@@ -283,6 +283,10 @@ struct rdm_gcn {
   const rdm::Graph* graph = nullptr;
   rdm_saint* saint = nullptr;
   int64_t n_cap = 0;
+  // R_A < P (RDM_GCN_PANELS, §III-E): column-layout tensors are tiles of the
+  // P/R_A x R_A grid, SpMMs broadcast inside column groups, redistributions
+  // stay inside panel groups (panels.cpp).  0 = full replication.
+  int RA = 0;
   int64_t gver = -1;
 };
 
@@ -291,7 +295,7 @@ namespace {
 
 int norm_lay(const rdm_gcn* g, int l) { return g->ctx->world == 1 ? 0 : l; }
 
-int64_t gn(const rdm_gcn* g) { return g->graph->n; }
+int64_t gn(const rdm_gcn* g) { return g->RA ? g->ctx->panel_n : g->graph->n; }
 
 // rows a row slice of rank p is allocated for: its share of n_cap, or, for a
 // sampler's instance (any n <= n_cap), the largest share ceil(n_cap / P)
@@ -336,6 +340,11 @@ void alloc_buf(rdm_gcn* g, Key k, int l, int64_t width) {
       b.rows = cap_rows(g, p);
       b.cols = width;
       b.ld = roundup4(width);
+    } else if (g->RA) {   // tile: panel rows x column slice over the R_A column groups
+      Range r, c;
+      tile_of(P, g->RA, n, width, p, &r, &c, &b.ld);
+      b.rows = r.size();
+      b.cols = c.size();
     } else {
       b.rows = n;
       b.cols = col_range(width, P, p).size();
@@ -351,7 +360,7 @@ void alloc_buf(rdm_gcn* g, Key k, int l, int64_t width) {
 }
 
 void plan_info(const Planner& pl, const std::vector<Step>& fwd, const std::vector<Step>& bwd,
-               int64_t n, rdm_gcn_info* out) {
+               int64_t n, rdm_gcn_info* out, int RA = 0) {
   rdm_gcn_info in{};
   const int P = pl.P;
   model_costs(pl.L, pl.f.data(), pl.igrad ? 1 : 0, pl.cfg, &in.model_comm_units,
@@ -361,7 +370,8 @@ void plan_info(const Planner& pl, const std::vector<Step>& fwd, const std::vecto
     if (P == 1) return t;
     for (int p = 0; p < P; ++p)
       for (int q = 0; q < P; ++q)
-        if (p != q) t += row_range(n, P, p).size() * col_range(w, P, q).size();
+        if (p != q && (!RA || p / RA == q / RA))   // R_A < P: inside the panel group only
+          t += row_range(n, P, p).size() * (RA ? col_range(w, RA, q % RA) : col_range(w, P, q)).size();
     return t;
   };
   for (auto* v : {&fwd, &bwd})
@@ -509,9 +519,9 @@ void create(rdm_gcn* g) {
     g->scal[s] = reinterpret_cast<double*>(g->mem.back()->ptr);
     RDM_CUDA(cudaMemset(g->scal[s], 0, 4 * sizeof(double)));
   }
-  plan_info(pl, g->fwd, g->bwd, n, &g->info);
+  plan_info(pl, g->fwd, g->bwd, n, &g->info, g->RA);
   g->info.workspace_bytes = g->ws_bytes;
-  if (ctx->transport == RDM_TRANSPORT_P2P && P > 1) setup_fusion(g);
+  if (ctx->transport == RDM_TRANSPORT_P2P && P > 1 && !g->RA) setup_fusion(g);
 }
 
 void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
@@ -523,6 +533,18 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
   if (s.fuse == 1) p2p_barrier(ctx);
   switch (s.op) {
     case S_SPMM: {
+      if (g->RA) {   // Fig. 6: tile broadcast in the column group + row-panel SpMM
+        std::vector<const float*> in(nl), mk(nl);
+        std::vector<float*> out(nl);
+        for (int i = 0; i < nl; ++i) {
+          in[i] = buf(g, i, s.in, s.lin).p;
+          out[i] = buf(g, i, s.out, s.lout).p;
+          mk[i] = (s.epi & RDM_EPI_MASK) ? buf(g, i, s.mask, s.lmask).p : nullptr;
+        }
+        spmm_panels(ctx, in.data(), out.data(), s.width, s.epi, nullptr,
+                    (s.epi & RDM_EPI_MASK) ? mk.data() : nullptr);
+        break;
+      }
       Phase ph(ctx, RDM_PH_SPMM);
       const Csr& A = s.trans ? g->graph->fwd() : g->graph->bwd();
       for (int i = 0; i < nl; ++i) {
@@ -584,7 +606,10 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
         src[i] = buf(g, i, s.in, s.lin).p;
         dst[i] = buf(g, i, s.out, s.lout).p;
       }
-      redistribute(ctx, (rdm_layout)s.lin, src.data(), dst.data(), gn(g), s.width);
+      if (g->RA)
+        redistribute_panels(ctx, (rdm_layout)s.lin, src.data(), dst.data(), gn(g), s.width);
+      else
+        redistribute(ctx, (rdm_layout)s.lin, src.data(), dst.data(), gn(g), s.width);
       break;
     }
     case S_MASK: {
@@ -828,7 +853,10 @@ void apply_input(rdm_gcn* g, const InputArgs* a) {
     src[i] = h.p;
     dst[i] = buf(g, i, {K_H, 0}, RDM_COL).p;
   }
-  if (P > 1) redistribute(ctx, RDM_ROW, src.data(), dst.data(), n, f0);
+  if (P > 1 && g->RA)
+    redistribute_panels(ctx, RDM_ROW, src.data(), dst.data(), n, f0);
+  else if (P > 1)
+    redistribute(ctx, RDM_ROW, src.data(), dst.data(), n, f0);
   std::vector<double*> nt(nl);
   for (int i = 0; i < nl; ++i) {
     const int64_t r = row_range(n, P, ctx->local[i]).size();
@@ -898,14 +926,20 @@ rdm_status rdm_gcn_create(rdm_ctx* ctx, int L, const int64_t* f, const rdm_confi
     ctx->err = "rdm_gcn_create: RDM_GCN_BIAS is not implemented";
     return RDM_ERR_UNSUPPORTED;
   }
-  if (!ctx->has_graph) {
+  const bool panels = (flags & RDM_GCN_PANELS) != 0;
+  if (panels && ctx->panel_RA <= 0) {
+    ctx->err = "rdm_gcn_create: RDM_GCN_PANELS needs rdm_set_graph_panels";
+    return RDM_ERR_STATE;
+  }
+  if (!panels && !ctx->has_graph) {
     ctx->err = "rdm_gcn_create: no graph (call rdm_set_graph)";
     return RDM_ERR_STATE;
   }
   auto* g = new rdm_gcn();
   g->ctx = ctx;
-  g->graph = &ctx->graph;
-  g->n_cap = ctx->graph.n;
+  g->graph = panels ? nullptr : &ctx->graph;
+  g->n_cap = panels ? ctx->panel_n : ctx->graph.n;
+  g->RA = panels ? ctx->panel_RA : 0;
   g->L = L;
   g->flags = flags;
   g->f.assign(f, f + L + 1);

@@ -162,3 +162,51 @@ rdm_status rdm_select_config(int L, const int64_t* f, int64_t n, int64_t nnz, in
 }
 
 }  // extern "C"
+
+// R_A < P (§III-E; reading R35): elements moved per epoch by a configuration
+// = N·[(R_A−1)/R_A·comm_units + (P/R_A−1)·sparse_units]; Pareto in (elements,
+// sparse units); the pick adds the same B200 time model as rdm_select_config
+// with the elements spread over P GPUs.
+extern "C" rdm_status rdm_select_config_ra(int L, const int64_t* f, int64_t n, int64_t nnz, int P,
+                                           int R_A, int need_input_grad, int64_t* pareto_ids,
+                                           int* n_pareto, int64_t* chosen_id, double* comm_elems,
+                                           int64_t* sparse_units) {
+  if (L < 1 || L > 6 || !f || P < 1 || R_A < 1 || R_A > P || P % R_A || n < 0 || nnz < 0)
+    return RDM_ERR_ARG;
+  const int64_t ncfg = int64_t(1) << (2 * L);
+  std::vector<double> ce(ncfg);
+  std::vector<int64_t> ss(ncfg);
+  for (int64_t i = 0; i < ncfg; ++i) {
+    int64_t c, sp;
+    model_costs(L, f, need_input_grad, config_from_id(L, i), &c, &sp);
+    ce[i] = (double)n * ((double)(R_A - 1) / R_A * c + ((double)P / R_A - 1) * sp);
+    ss[i] = sp;
+  }
+  std::vector<int64_t> front;
+  for (int64_t i = 0; i < ncfg; ++i) {
+    bool dom = false;
+    for (int64_t j = 0; j < ncfg && !dom; ++j)
+      dom = ce[j] <= ce[i] && ss[j] <= ss[i] && (ce[j] < ce[i] || ss[j] < ss[i]);
+    if (!dom) front.push_back(i);
+  }
+  if (n_pareto) {
+    const int cap = *n_pareto;
+    for (int k = 0; k < (int)front.size() && k < cap && pareto_ids; ++k) pareto_ids[k] = front[k];
+    *n_pareto = (int)front.size();
+  }
+  const double B_link = 770e9, B_hbm = 6.5e12;
+  int64_t best = -1;
+  double best_t = 0;
+  for (int64_t i : front) {
+    const double t = ce[i] * 4.0 / P / B_link + (double)ss[i] * ((double)nnz * 4.0 / P + 8.0 * n / P) / B_hbm;
+    if (best < 0 || t < best_t * (1 - 1e-12) ||
+        (std::fabs(t - best_t) <= 1e-12 * best_t && (ss[i] < ss[best] || (ss[i] == ss[best] && i < best)))) {
+      best = i;
+      best_t = t;
+    }
+  }
+  if (chosen_id) *chosen_id = best;
+  if (comm_elems) *comm_elems = best >= 0 ? ce[best] : 0.0;
+  if (sparse_units) *sparse_units = best >= 0 ? ss[best] : 0;
+  return RDM_OK;
+}

@@ -163,3 +163,62 @@ def test_error_codes_without_gpu():
     assert e.value.status == rdm.ERR_ARG
     with pytest.raises(rdm.RdmError):
         rdm.config_from_id(2, 16)
+
+
+# ------------------------------------------------- R_A < P host functions (NEXT-4)
+@pytest.mark.parametrize("seed", range(6))
+def test_partition_tile_covers_matrix_once(seed):
+    """Tiles of the P/R_A x R_A grid cover the N x f matrix exactly once, and
+    every rank's row slice lies inside its row panel (so the row ↔ tile
+    redistribution stays inside a panel group, L214)."""
+    rng = random.Random(seed)
+    P = rng.choice([1, 2, 4, 6, 8])
+    RA = rng.choice([r for r in range(1, P + 1) if P % r == 0])
+    n, f = rng.randint(0, 3000), rng.randint(1, 300)
+    cover = np.zeros((n, f), np.int32)
+    for p in range(P):
+        r0, r1, c0, c1, ld = rdm.partition_tile(P, RA, n, f, p)
+        cover[r0:r1, c0:c1] += 1
+        assert ld % 4 == 0 and ld >= c1 - c0
+        lo, hi, _ = rdm.partition(P, rdm.ROW, n, f, p)
+        assert r0 <= lo and hi <= r1
+        # R_A = P: a tile is the plain column slice
+        if RA == P:
+            assert (r0, r1) == (0, n)
+            assert (c0, c1) == rdm.partition(P, rdm.COL, n, f, p)[:2]
+    assert np.all(cover == 1)
+
+
+def test_partition_tile_rejects_bad_grid():
+    with pytest.raises(rdm.RdmError):
+        rdm.partition_tile(8, 3, 100, 10, 0)
+
+
+def test_max_replication_matches_oracle():
+    rng = random.Random(3)
+    for _ in range(500):
+        P = rng.choice([1, 2, 3, 4, 6, 8, 16])
+        M = rng.uniform(1, 200) * 1e9
+        H = rng.uniform(0, 1.2) * M
+        G = rng.uniform(0.1, 400) * 1e9
+        assert rdm.max_replication(P, M, H, G) == ocm.max_replication(P, M, H, G)
+
+
+@pytest.mark.parametrize("seed", range(4))
+def test_select_config_ra_front_matches_oracle(seed):
+    """The library's R_A < P front (elements moved, sparse units) equals the
+    oracle's (reading R35), and R_A = P gives the full-replication front."""
+    rng = random.Random(100 + seed)
+    for _ in range(25):
+        L = rng.choice([2, 3])
+        f = [rng.randint(1, 700) for _ in range(L + 1)]
+        n, nnz = rng.randint(100, 10 ** 7), rng.randint(100, 10 ** 9)
+        P = rng.choice([2, 4, 6, 8])
+        RA = rng.choice([r for r in range(1, P + 1) if P % r == 0])
+        front, chosen, elems, sparse = rdm.select_config_ra(f, n, nnz, P, RA)
+        assert front == ocm.pareto_ra(f, n, P, RA)
+        assert chosen in front
+        assert elems == pytest.approx(ocm.comm_elements_ra(chosen, f, n, P, RA))
+        assert sparse == ocm.simulate(chosen, f)[1]
+        if RA == P:
+            assert front == rdm.select_config(f, n, nnz, P)[0]

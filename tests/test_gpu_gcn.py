@@ -74,7 +74,7 @@ def cora():
     return g, H0, Ws, y, m, ref
 
 
-def _gather(model, rdm, which, layer, n, width, P):
+def _gather(model, rdm, which, layer, n, width, P, ra=0):
     """Full n x width matrix of an internal tensor from whichever layout is resident."""
     full = np.zeros((n, width))
     for layout in (rdm.ROW, rdm.COL):
@@ -88,6 +88,9 @@ def _gather(model, rdm, which, layer, n, width, P):
             elif layout == rdm.ROW:
                 lo, hi, _ = rdm.partition(P, rdm.ROW, n, width, p)
                 full[lo:hi] = t
+            elif ra:   # R_A < P tiles (rdm_partition_tile)
+                r0, r1, c0, c1, _ = rdm.partition_tile(P, ra, n, width, p)
+                full[r0:r1, c0:c1] = t[:r1 - r0, :c1 - c0]
             else:
                 lo, hi, _ = rdm.partition(P, rdm.COL, n, width, p)
                 full[:, lo:hi] = t
@@ -95,7 +98,7 @@ def _gather(model, rdm, which, layer, n, width, P):
     raise AssertionError(f"tensor {which}/{layer} not resident")
 
 
-def _check(prob, loss, dW, model, rdm, P=1, check_g0=True, tol=1e-4, ltol=1e-5):
+def _check(prob, loss, dW, model, rdm, P=1, check_g0=True, tol=1e-4, ltol=1e-5, ra=0):
     """Compare with the fp64 oracle.  The ReLU decisions 1[Z^l > 0] are taken from
     the kernel's own fp32 forward (reading R30: a float-decided discrete value is
     decided in the kernel's precision on both sides); everything else is fp64.
@@ -104,7 +107,7 @@ def _check(prob, loss, dW, model, rdm, P=1, check_g0=True, tol=1e-4, ltol=1e-5):
     L = len(Ws)
     f = [H0.shape[1]] + [w.shape[1] for w in Ws]
     n = g.n
-    Hs = [_gather(model, rdm, rdm.T_H, l, n, f[l], P) for l in range(1, L)]
+    Hs = [_gather(model, rdm, rdm.T_H, l, n, f[l], P, ra) for l in range(1, L)]
     ref = og.epoch(g, H0, Ws, y, m, relu_masks=[h > 0 for h in Hs])
     # forward parity (independent of the masks)
     for l in range(1, L):
@@ -115,10 +118,10 @@ def _check(prob, loss, dW, model, rdm, P=1, check_g0=True, tol=1e-4, ltol=1e-5):
     for l in range(L):
         err = og.max_rel_err(dW[l], ref.Y[l + 1])
         assert err < tol, (l + 1, err)
-    Z = _gather(model, rdm, rdm.T_Z, 0, n, f[L], P)
+    Z = _gather(model, rdm, rdm.T_Z, 0, n, f[L], P, ra)
     assert og.max_rel_err(Z, ref.Z[L]) < tol
     if check_g0:
-        G0 = _gather(model, rdm, rdm.T_G, 0, n, f[0], P)
+        G0 = _gather(model, rdm, rdm.T_G, 0, n, f[0], P, ra)
         assert og.max_rel_err(G0, ref.G[0]) < tol
 
 

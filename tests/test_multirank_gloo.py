@@ -206,3 +206,81 @@ def test_two_rank_plan_matches_oracle(cfg):
     assert all(pr.exitcode == 0 for pr in procs), [pr.exitcode for pr in procs]
     res = [q.get() for _ in range(2)]
     assert sorted(r[0] for r in res) == [0, 1]
+
+
+# ------------------------------------------------------------- R_A < P (NEXT-4)
+def _run_panels(p, P, RA, port, q_out):
+    """One layer's SpMM and redistribution on the P/R_A x R_A grid with real
+    processes: tiles from rdm_partition_tile, the Fig. 6 broadcast of input
+    tiles inside the column group (gloo send/recv), the row-panel product, and
+    the tile → row-slice redistribution inside the panel group; every rank's
+    result equals the oracle's slice."""
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=p, world_size=P)
+    try:
+        g = synth.rmat(700, 4000, seed=4)
+        n, w = g.n, 13
+        X = np.random.default_rng(0).standard_normal((n, w))
+        i, j = p // RA, p % RA
+        r0, r1, c0, c1, _ = rdm.partition_tile(P, RA, n, w, p)
+        mine = torch.from_numpy(np.ascontiguousarray(X[r0:r1, c0:c1]))
+        # broadcast inside column group j: gather In[:, c0:c1] from ranks i2·R_A + j
+        full = np.zeros((n, c1 - c0))
+        full[r0:r1] = mine.numpy()
+        reqs = []
+        bufs = {}
+        for i2 in range(P // RA):
+            qr = i2 * RA + j
+            if qr == p:
+                continue
+            q0, q1, _, _, _ = rdm.partition_tile(P, RA, n, w, qr)
+            bufs[qr] = torch.zeros((q1 - q0, c1 - c0), dtype=torch.float64)
+            reqs.append(dist.isend(mine, qr))
+            reqs.append(dist.irecv(bufs[qr], qr))
+        for rq in reqs:
+            rq.wait()
+        for qr, b in bufs.items():
+            q0, q1, _, _, _ = rdm.partition_tile(P, RA, n, w, qr)
+            full[q0:q1] = b.numpy()
+        # row-panel product: rows r0..r1 of A·In[:, c0:c1]
+        out_tile = og.spmm(g, full)[r0:r1]
+        ref = og.spmm(g, X)
+        assert og.max_rel_err(out_tile, ref[r0:r1, c0:c1]) < 1e-12
+        # tile → row slices inside panel group i
+        lo, hi, _ = rdm.partition(P, ROW, n, w, p)
+        row = np.zeros((hi - lo, w))
+        row[:, c0:c1] = out_tile[lo - r0:hi - r0]
+        reqs, got = [], {}
+        for j2 in range(RA):
+            qr = i * RA + j2
+            if qr == p:
+                continue
+            qlo, qhi, _ = rdm.partition(P, ROW, n, w, qr)
+            _, _, d0, d1, _ = rdm.partition_tile(P, RA, n, w, qr)
+            reqs.append(dist.isend(torch.from_numpy(np.ascontiguousarray(out_tile[qlo - r0:qhi - r0])), qr))
+            got[qr] = torch.zeros((hi - lo, d1 - d0), dtype=torch.float64)
+            reqs.append(dist.irecv(got[qr], qr))
+        for rq in reqs:
+            rq.wait()
+        for qr, b in got.items():
+            _, _, d0, d1, _ = rdm.partition_tile(P, RA, n, w, qr)
+            row[:, d0:d1] = b.numpy()
+        assert og.max_rel_err(row, ref[lo:hi]) < 1e-12
+        q_out.put((p, "ok"))
+    finally:
+        dist.destroy_process_group()
+
+
+@pytest.mark.parametrize("P,RA", [(2, 1), (4, 2)])
+def test_panels_grid_with_processes(P, RA):
+    ctx = mp.get_context("spawn")
+    q = ctx.SimpleQueue()
+    port = _free_port()
+    procs = [ctx.Process(target=_run_panels, args=(p, P, RA, port, q)) for p in range(P)]
+    for pr in procs:
+        pr.start()
+    for pr in procs:
+        pr.join(timeout=180)
+    assert all(pr.exitcode == 0 for pr in procs), [pr.exitcode for pr in procs]
+    assert sorted(q.get()[0] for _ in range(P)) == list(range(P))
