@@ -591,18 +591,18 @@ def main():
     traffic, traffic_src = None, None
     try:
         tj = _json.load(open(os.path.join(ROOT, "profiles", "r1_spmm_traffic.json")))
-        if a.workload == "reddit" and world == 1:
-            ls = tj["spmm_launches"]
+        if a.workload == "reddit" and world == 1 and a.precision == "fp32" and not panels:
+            ls = tj["calls"]   # one w = 128 and one w = 41 call: the epoch has two of each
             traffic = sum(x["dram_bytes"] for x in ls) / len(ls) / 1e9
             traffic_src = tj["source"]
     except Exception:
         pass
     roofline = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
-                "frac": achieved / hbm_peak, "traffic": traffic, "traffic_unit": "GB per launch",
+                "frac": achieved / hbm_peak, "traffic": traffic, "traffic_unit": "GB per SpMM call",
                 "traffic_source": traffic_src,
                 "algorithmic_gb_per_call": alg_bytes / max(1, spmm_calls) / 1e9,
                 "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)",
-                "kernel": "spmm (rdm::spmm_kernel + heavy-row reduce)",
+                "kernel": "spmm call (tile panels + binary hub tiles + residual CSR + heavy-row reduce)",
                 "spmm_share_of_step": ph_ms["spmm"] / max(1e-9, ms_total),
                 "avg_call_ms": ph_ms["spmm"] / max(1, spmm_calls),
                 "gather_gbs": (cnt["spmm_nnz_cols"] * 4) / spmm_s / 1e9 if spmm_s > 0 else 0.0}

@@ -114,6 +114,10 @@ struct Csr {
   std::unique_ptr<DevBuf> heavy_rows;   // int32[n_heavy]
   std::unique_ptr<DevBuf> heavy_seg;    // int32[n_heavy+1]: segment range of heavy row
   int64_t max_deg = 0;
+  // every stored value factors as a_ij = s_i·s_j (GCN normalisation; checked
+  // on the host at rdm_set_graph): fp32 s per row, used by the fast-precision
+  // SpMM (sum of bf16(s_j X_j), s_i in the epilogue); null otherwise
+  std::unique_ptr<DevBuf> fscale;
 };
 
 struct Graph {

@@ -101,6 +101,83 @@ xent_kernel(const float* __restrict__ Z, int64_t ldz, const int32_t* __restrict_
   }
 }
 
+// Narrow rows (C ≤ 128): LPR lanes per row, EPL = 4·V columns per lane as V
+// float4 loads, 32/LPR rows per warp in flight (the one-warp-per-row kernel
+// above serialises two full-warp reductions per row, latency-bound for
+// C = 41 / 47).  Rows are 16-byte aligned with zero pads (executor layout);
+// pads are excluded from the max / sum and written back as zeros.
+template <int LPR, int V>
+__global__ void __launch_bounds__(kLossWarps * 32)
+xent_group_kernel(const float* __restrict__ Z, int64_t ldz, const int32_t* __restrict__ labels,
+                  const uint8_t* __restrict__ mask, int64_t rows, int64_t C,
+                  const double* __restrict__ n_train, float* __restrict__ G, int64_t ldg,
+                  double* __restrict__ partial) {
+  constexpr int RPW = 32 / LPR;
+  __shared__ double red[kLossWarps];
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  const int sub = lane % LPR, grp = lane / LPR;
+  const double nt = *n_train;
+  const float inv_n = nt > 0 ? (float)(1.0 / nt) : 0.f;
+  double local = 0.0;
+  const int64_t stride = (int64_t)gridDim.x * kLossWarps * RPW;
+  for (int64_t base = ((int64_t)blockIdx.x * kLossWarps + wid) * RPW; base < rows; base += stride) {
+    const int64_t i = base + grp;
+    const bool valid = i < rows;
+    float4 v[V];
+    float mx = -FLT_MAX;
+#pragma unroll
+    for (int k = 0; k < V; ++k) {
+      const int64_t c = 4 * (sub + LPR * k);
+      v[k] = (valid && c < C) ? __ldcs(reinterpret_cast<const float4*>(Z + i * ldz + c))
+                              : make_float4(-FLT_MAX, -FLT_MAX, -FLT_MAX, -FLT_MAX);
+      if (c + 1 >= C) v[k].y = -FLT_MAX;
+      if (c + 2 >= C) v[k].z = -FLT_MAX;
+      if (c + 3 >= C) v[k].w = -FLT_MAX;
+      mx = fmaxf(mx, fmaxf(fmaxf(v[k].x, v[k].y), fmaxf(v[k].z, v[k].w)));
+    }
+#pragma unroll
+    for (int o = LPR / 2; o; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
+    float s = 0.f;
+#pragma unroll
+    for (int k = 0; k < V; ++k) {
+      v[k].x = expf(v[k].x - mx);   // exp(-FLT_MAX - mx) = 0 for pads
+      v[k].y = expf(v[k].y - mx);
+      v[k].z = expf(v[k].z - mx);
+      v[k].w = expf(v[k].w - mx);
+      s += (v[k].x + v[k].y) + (v[k].z + v[k].w);
+    }
+#pragma unroll
+    for (int o = LPR / 2; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
+    if (valid) {
+      const int y = labels[i];
+      const bool m = mask ? mask[i] != 0 : true;
+      const float scale = m ? inv_n : 0.f;
+      const float inv_s = 1.f / s;
+#pragma unroll
+      for (int k = 0; k < V; ++k) {
+        const int64_t c = 4 * (sub + LPR * k);
+        if (c < C) {
+          float4 gv;
+          gv.x = (v[k].x * inv_s - (c == y ? 1.f : 0.f)) * scale;
+          gv.y = c + 1 < C ? (v[k].y * inv_s - (c + 1 == y ? 1.f : 0.f)) * scale : 0.f;
+          gv.z = c + 2 < C ? (v[k].z * inv_s - (c + 2 == y ? 1.f : 0.f)) * scale : 0.f;
+          gv.w = c + 3 < C ? (v[k].w * inv_s - (c + 3 == y ? 1.f : 0.f)) * scale : 0.f;
+          *reinterpret_cast<float4*>(G + i * ldg + c) = gv;
+        }
+      }
+      if (sub == 0 && m) local += (double)mx + log((double)s) - (double)Z[i * ldz + y];
+    }
+  }
+  local = warp_sum_d(local);
+  if (lane == 0) red[wid] = local;
+  __syncthreads();
+  if (threadIdx.x == 0) {
+    double t = 0.0;
+    for (int k = 0; k < kLossWarps; ++k) t += red[k];
+    partial[blockIdx.x] = t;
+  }
+}
+
 // Single-block ordered sum of n doubles (fixed tree) → *out.
 __global__ void sum_partials(const double* __restrict__ p, int n, double* __restrict__ out) {
   __shared__ double s[1024];
@@ -221,6 +298,29 @@ void softmax_xent(rdm_ctx* ctx, const float* Z, int64_t ldz, const int32_t* labe
                   int64_t ldg, double* loss_partial) {
   // ≈2 rows per warp; the grid depends only on `rows`, so the partials and
   // their ordered sum are deterministic
+  const bool aligned = ldz % 4 == 0 && ldg % 4 == 0 && ((uintptr_t)Z & 15) == 0 && ((uintptr_t)G & 15) == 0;
+  if (aligned && C <= 128) {
+    // lanes per row: the fewest with ≤ 8 columns each (V ≤ 2 float4), ≥ 2
+    int lpr = 2;
+    while (lpr < 32 && lpr * 8 < C) lpr *= 2;
+    const int V = (int)ceil_div(C, 4 * lpr);
+    const int rpb = kLossWarps * (32 / lpr);
+    const int nb = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(rows, rpb * 2), 16384));
+    double* part = reinterpret_cast<double*>(ensure_ws(ctx->ws_scratch, (size_t)nb * sizeof(double)));
+#define RDM_XENT_CASE(l_, v_)                                                                          \
+  if (lpr == l_ && V == v_)                                                                          \
+    xent_group_kernel<l_, v_><<<nb, kLossWarps * 32, 0, ctx->stream>>>(Z, ldz, labels, mask, rows, C, \
+                                                                       n_train, G, ldg, part);       \
+  else
+    RDM_XENT_CASE(2, 1) RDM_XENT_CASE(2, 2) RDM_XENT_CASE(4, 1) RDM_XENT_CASE(4, 2)
+    RDM_XENT_CASE(8, 1) RDM_XENT_CASE(8, 2) RDM_XENT_CASE(16, 1) RDM_XENT_CASE(16, 2)
+    throw Error(RDM_ERR_STATE, "xent: no kernel for the row shape");
+#undef RDM_XENT_CASE
+    RDM_LAUNCHED(ctx);
+    sum_partials<<<1, 1024, 0, ctx->stream>>>(part, nb, loss_partial);
+    RDM_LAUNCHED(ctx);
+    return;
+  }
   const int nb = (int)std::max<int64_t>(1, std::min<int64_t>(ceil_div(rows, kLossWarps * 2), 16384));
   double* part = reinterpret_cast<double*>(ensure_ws(ctx->ws_scratch, (size_t)nb * sizeof(double)));
   xent_kernel<<<nb, kLossWarps * 32, 0, ctx->stream>>>(Z, ldz, labels, mask, rows, C, n_train, G,

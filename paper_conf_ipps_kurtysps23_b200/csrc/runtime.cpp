@@ -335,12 +335,33 @@ static void set_graph(rdm_ctx* ctx, int64_t n, int64_t nnz, const int64_t* rowpt
   std::vector<int64_t> rp(n + 1);
   RDM_CUDA(cudaMemcpy(rp.data(), g.A.rowptr->ptr, (n + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost));
   build_bins(ctx, g.A, rp.data());
-  if (g.symmetric && n >= 4096 && nnz > 0) {
+  if (g.symmetric && nnz > 0) {
     std::vector<int32_t> hc(nnz);
     std::vector<float> hv(nnz);
     RDM_CUDA(cudaMemcpy(hc.data(), g.A.col->ptr, nnz * sizeof(int32_t), cudaMemcpyDeviceToHost));
     RDM_CUDA(cudaMemcpy(hv.data(), g.A.val->ptr, nnz * sizeof(float), cudaMemcpyDeviceToHost));
-    build_core(ctx, g.A, rp.data(), hc.data(), hv.data());
+    if (n >= 4096) build_core(ctx, g.A, rp.data(), hc.data(), hv.data());
+    // factorisation a_ij = s_i·s_j of every value (s = deg^-1/2, or all ones)
+    // for the fast-precision SpMM's value-free row sums
+    std::vector<float> sc(n);
+    for (int hyp = 0; hyp < 2 && !g.A.fscale; ++hyp) {
+      bool ok = true;
+      std::vector<double> sd(n);
+      for (int64_t i = 0; i < n; ++i)
+        sd[i] = hyp == 0 ? (rp[i + 1] > rp[i] ? 1.0 / std::sqrt((double)(rp[i + 1] - rp[i])) : 0.0) : 1.0;
+      for (int64_t i = 0; i < n && ok; ++i)
+        for (int64_t j = rp[i]; j < rp[i + 1]; ++j) {
+          const double f = sd[i] * sd[hc[j]];
+          if (!(std::fabs((double)hv[j] - f) <= std::ldexp(f, -21))) {
+            ok = false;
+            break;
+          }
+        }
+      if (!ok) continue;
+      for (int64_t i = 0; i < n; ++i) sc[i] = (float)sd[i];
+      g.A.fscale.reset(new DevBuf(std::max<int64_t>(n, 1) * sizeof(float)));
+      RDM_CUDA(cudaMemcpy(g.A.fscale->ptr, sc.data(), n * sizeof(float), cudaMemcpyHostToDevice));
+    }
   }
   if (!g.symmetric) {
     // Aᵀ as CSR: stable counting sort of (col, row) — one-time setup.

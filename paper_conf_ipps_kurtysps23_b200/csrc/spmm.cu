@@ -51,6 +51,7 @@ struct Epi {
   const int32_t* rb_item;   // item range of each 128-row rank block
   const float* tscale;      // s_i of slot i
   Scatter scat;             // fused col→row redistribution (scat.P == 0: off)
+  const float* rscale;      // factored bf16 path: s_i per row (applied first), or null
 };
 
 // Fused col→row redistribution: row r of my column slice (columns c..c+3 of
@@ -70,6 +71,10 @@ __device__ __forceinline__ void scatter_row_store(const Scatter& s, int64_t r, i
 }
 
 __device__ __forceinline__ float4 apply_epi(float4 a, const Epi& e, int64_t row, int64_t c) {
+  if (e.rscale) {   // factored rows: Σ_j bf16(s_j X_j) · s_i
+    const float sc = __ldg(e.rscale + row);
+    a.x *= sc; a.y *= sc; a.z *= sc; a.w *= sc;
+  }
   if (e.core) {  // add the dense hub-core contribution of this row (fixed order: after the CSR sum)
     const int s = __ldg(e.hub_slot + row);
     if (s >= 0) {
@@ -263,7 +268,22 @@ spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
 // RDM_PREC_FAST: the same walk over a bf16 copy of the slice.  A lane's
 // 128-bit gather now carries 8 columns; bf16 → fp32 is exact (a shift), the
 // products and sums stay fp32.  acc[v][0..1] = columns 8·ch + 0..3, + 4..7.
-template <int G, int V, int U>
+// fp32 += bf16 (low or high half of u) · 1.0 in one FHFMA.BF16 (exact
+// product, one rounding = an fp32 add of the widened value).
+__device__ __forceinline__ void acc_bf16_lo(float& a, uint32_t u) {
+  asm("{.reg .b16 l, h;\n\tmov.b32 {l, h}, %1;\n\tfma.rn.f32.bf16 %0, l, %2, %0;\n\t}"
+      : "+f"(a) : "r"(u), "h"((unsigned short)0x3F80));
+}
+__device__ __forceinline__ void acc_bf16_hi(float& a, uint32_t u) {
+  asm("{.reg .b16 l, h;\n\tmov.b32 {l, h}, %1;\n\tfma.rn.f32.bf16 %0, h, %2, %0;\n\t}"
+      : "+f"(a) : "r"(u), "h"((unsigned short)0x3F80));
+}
+
+// FACT: the adjacency factors as â_ij = s_i·s_j (GCN normalisation, checked at
+// rdm_set_graph) and the slice was stored as bf16(s_j·X_j): the row sum needs
+// no values (no val stream, no shuffles of it) and s_i is applied in the
+// epilogue (Epi::rscale).
+template <int G, int V, int U, bool FACT = false>
 __device__ __forceinline__ void warp_nnz_range_bf(const int32_t* __restrict__ col,
                                                   const float* __restrict__ val,
                                                   const __nv_bfloat16* __restrict__ xb, int64_t ldx,
@@ -279,7 +299,7 @@ __device__ __forceinline__ void warp_nnz_range_bf(const int32_t* __restrict__ co
     float a = 0.f;
     if (j < end) {
       c = __ldcs(col + j);
-      a = __ldcs(val + j);
+      if (!FACT) a = __ldcs(val + j);
     }
     const int cnt = (end - base) < 32 ? (int)(end - base) : 32;
 #pragma unroll
@@ -291,7 +311,7 @@ __device__ __forceinline__ void warp_nnz_range_bf(const int32_t* __restrict__ co
       for (int u = 0; u < U; ++u) {
         const int k = (t0 + u) * NG + g;
         const int cc = (G == 1) ? c : __shfl_sync(kFull, c, k);
-        vv[u] = (G == 1) ? a : __shfl_sync(kFull, a, k);
+        vv[u] = FACT ? 1.f : (G == 1) ? a : __shfl_sync(kFull, a, k);
         const uint4* xr = reinterpret_cast<const uint4*>(xb + (int64_t)cc * ldx);
 #pragma unroll
         for (int v = 0; v < V; ++v)
@@ -302,6 +322,16 @@ __device__ __forceinline__ void warp_nnz_range_bf(const int32_t* __restrict__ co
 #pragma unroll
         for (int v = 0; v < V; ++v) {
           const uint32_t w4[4] = {x[u][v].x, x[u][v].y, x[u][v].z, x[u][v].w};
+          if (FACT) {
+#pragma unroll
+            for (int h = 0; h < 2; ++h) {
+              acc_bf16_lo(acc[v][h].x, w4[2 * h]);
+              acc_bf16_hi(acc[v][h].y, w4[2 * h]);
+              acc_bf16_lo(acc[v][h].z, w4[2 * h + 1]);
+              acc_bf16_hi(acc[v][h].w, w4[2 * h + 1]);
+            }
+            continue;
+          }
 #pragma unroll
           for (int h = 0; h < 2; ++h) {
             float4& A = acc[v][h];
@@ -331,7 +361,7 @@ __device__ __forceinline__ void warp_nnz_range_bf(const int32_t* __restrict__ co
 // columns, `w4` is the output's real padded width (stores stop there).
 // twice the accumulators of spmm_kernel: s = 2V + U·V slots
 constexpr int spmm_minb_bf(int V, int U) { return spmm_minb_slots(2 * V + U * V); }
-template <int G, int V, int U>
+template <int G, int V, int U, bool FACT = false>
 __global__ void __launch_bounds__(kWarps * 32, spmm_minb_bf(V, U))
 spmm_kernel_bf(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
                const float* __restrict__ val, const int32_t* __restrict__ light_rows,
@@ -351,7 +381,7 @@ spmm_kernel_bf(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ c
     const int32_t r = seg_row[item];
     const int64_t beg = seg_start[item];
     const int64_t end = min(beg + kSeg, rowptr[r + 1]);
-    warp_nnz_range_bf<G, V, U>(col, val, X + cbase, ldx, beg, end, lane, c8n, acc);
+    warp_nnz_range_bf<G, V, U, FACT>(col, val, X + cbase, ldx, beg, end, lane, c8n, acc);
     if (lane < G) {
       float* dst = part + item * ld_part + cbase;
 #pragma unroll
@@ -363,7 +393,7 @@ spmm_kernel_bf(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ c
     }
   } else {
     const int32_t r = light_rows[item - n_seg];
-    warp_nnz_range_bf<G, V, U>(col, val, X + cbase, ldx, rowptr[r], rowptr[r + 1], lane, c8n, acc);
+    warp_nnz_range_bf<G, V, U, FACT>(col, val, X + cbase, ldx, rowptr[r], rowptr[r + 1], lane, c8n, acc);
     if (lane < G) {
       float* dst = out + (int64_t)r * ld_out;
 #pragma unroll
@@ -385,18 +415,24 @@ spmm_kernel_bf(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ c
   }
 }
 
-// fp32 slice → bf16 copy (round to nearest even), row length ldy = w8, zero
-// pads: one thread per 8 columns.
+// fp32 slice → bf16 copy (round to nearest even) of X (scale == null) or of
+// s_r·X_r (factored adjacency), row length ldy = w8, zero pads: one thread
+// per 8 columns.
 __global__ void to_bf16_kernel(const float* __restrict__ X, int64_t ldx, int64_t n, int64_t w4, int64_t w8,
-                               __nv_bfloat16* __restrict__ Y) {
+                               __nv_bfloat16* __restrict__ Y, const float* __restrict__ scale) {
   const int64_t per = w8 / 8;
   const int64_t total = n * per;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total;
        i += (int64_t)gridDim.x * blockDim.x) {
     const int64_t r = i / per, c = (i - r * per) * 8;
     const float* xr = X + r * ldx + c;
-    const float4 a = __ldcs(reinterpret_cast<const float4*>(xr));
-    const float4 b = (c + 4 < w4) ? __ldcs(reinterpret_cast<const float4*>(xr + 4)) : make_float4(0.f, 0.f, 0.f, 0.f);
+    float4 a = __ldcs(reinterpret_cast<const float4*>(xr));
+    float4 b = (c + 4 < w4) ? __ldcs(reinterpret_cast<const float4*>(xr + 4)) : make_float4(0.f, 0.f, 0.f, 0.f);
+    if (scale) {
+      const float sc = __ldg(scale + r);
+      a.x *= sc; a.y *= sc; a.z *= sc; a.w *= sc;
+      b.x *= sc; b.y *= sc; b.z *= sc; b.w *= sc;
+    }
     __nv_bfloat162 p[4] = {__floats2bfloat162_rn(a.x, a.y), __floats2bfloat162_rn(a.z, a.w),
                            __floats2bfloat162_rn(b.x, b.y), __floats2bfloat162_rn(b.z, b.w)};
     *reinterpret_cast<uint4*>(Y + r * w8 + c) = *reinterpret_cast<const uint4*>(p);
@@ -439,7 +475,7 @@ void launch_spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, flo
   RDM_LAUNCHED(ctx);
 }
 
-template <int G, int V, int U>
+template <int G, int V, int U, bool FACT = false>
 void launch_spmm_bf(rdm_ctx* ctx, const Csr& A, const __nv_bfloat16* in, int64_t ld_in, float* out,
                     int64_t ld_out, float* part, int64_t ld_part, int64_t w4, int64_t w8, int chunk8,
                     const Epi& epi) {
@@ -447,7 +483,7 @@ void launch_spmm_bf(rdm_ctx* ctx, const Csr& A, const __nv_bfloat16* in, int64_t
   if (items == 0) return;
   const int64_t chunks = ceil_div(w8, 8 * chunk8);
   dim3 grid((unsigned)ceil_div(items, kWarps), (unsigned)chunks);
-  spmm_kernel_bf<G, V, U><<<grid, kWarps * 32, 0, ctx->stream>>>(
+  spmm_kernel_bf<G, V, U, FACT><<<grid, kWarps * 32, 0, ctx->stream>>>(
       A.rowptr->as<int64_t>(), A.col->as<int32_t>(), A.val->as<float>(),
       A.light_rows->as<int32_t>(), A.seg_start->as<int64_t>(),
       reinterpret_cast<const int32_t*>(A.seg_start->as<int64_t>() + A.n_seg), A.n_light, A.n_seg,
@@ -476,7 +512,7 @@ void pick_gv(int c4, int* G, int* V) {
 }
 
 void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
-             int64_t w4, const Epi& epi, const __nv_bfloat16* inb);
+             int64_t w4, const Epi& epi, const __nv_bfloat16* inb, bool fact = false);
 
 // (G, V, U) for a chunk of c 128-bit vectors per row (4 fp32 or 8 bf16
 // columns each).  Measured on the Reddit- and products-shaped residual CSRs
@@ -570,7 +606,7 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
                                                 ((uintptr_t)mask & 15) == 0),
                 "spmm: mask requires a 16-byte aligned N x w buffer with ld % 4 == 0");
   RDM_CHECK_ARG(!(epi_flags & RDM_EPI_BIAS) || bias, "spmm: bias pointer missing");
-  Epi epi{epi_flags, bias, mask, ld_mask, w, nullptr, 0, nullptr, nullptr, 0, nullptr, nullptr, Scatter{}};
+  Epi epi{epi_flags, bias, mask, ld_mask, w, nullptr, 0, nullptr, nullptr, 0, nullptr, nullptr, Scatter{}, nullptr};
   if (scat) {
     RDM_CHECK_ARG(scat->mode == 2 && scat->P >= 1 && scat->P <= Scatter::kMax && scat->my_w <= w,
                   "spmm: bad scatter descriptor");
@@ -579,15 +615,19 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
   // RDM_PREC_FAST: one bf16 copy of the input slice per call, gathered by
   // every row of the residual CSR (rdm.h rdm_set_precision)
   const __nv_bfloat16* inb = nullptr;
+  bool fact = false;
   if (ctx->prec == RDM_PREC_FAST) {
     const int64_t w8 = (w4 + 7) & ~int64_t(7);
     const int64_t nin = A.in_rows();
     __nv_bfloat16* xb = reinterpret_cast<__nv_bfloat16*>(ensure_ws(ctx->ws_bf16, (size_t)std::max<int64_t>(nin, 1) * w8 * 2));
     const int64_t total = nin * (w8 / 8);
     const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(total, 256), (int64_t)ctx->num_sms * 16));
-    to_bf16_kernel<<<grid, 256, 0, ctx->stream>>>(in, ld_in, nin, w4, w8, xb);
+    fact = A.fscale != nullptr;
+    to_bf16_kernel<<<grid, 256, 0, ctx->stream>>>(in, ld_in, nin, w4, w8, xb,
+                                                  fact ? A.fscale->as<float>() : nullptr);
     RDM_LAUNCHED(ctx);
     inb = xb;
+    if (fact) epi.rscale = A.fscale->as<float>();
   }
   const int np = ctx->prec == RDM_PREC_FAST ? 1 : 3;
   if (A.core.n_tiles && hub_tiles_pay(A.core, w, np)) {
@@ -601,7 +641,7 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
     epi.rb_item = A.core.rb_item->as<int32_t>();
     epi.tscale = A.core.scale->as<float>();
     epi.hub_slot = A.core.hub_slot->as<int32_t>();
-    run_csr(ctx, *A.core.resid, in, ld_in, out, ld_out, w4, epi, inb);
+    run_csr(ctx, *A.core.resid, in, ld_in, out, ld_out, w4, epi, inb, fact);
   } else if (A.core.K && core_pays(A.core, w)) {
     // hub core on the tensor cores: panels Bt[n][k] = split(X[hub_k][n]), then
     // C_core = Acore · X[hubs]; the residual CSR's epilogue adds C_core rows.
@@ -616,9 +656,9 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
     epi.core = cc;
     epi.ld_core = w4;
     epi.hub_slot = A.core.hub_slot->as<int32_t>();
-    run_csr(ctx, *A.core.resid, in, ld_in, out, ld_out, w4, epi, inb);
+    run_csr(ctx, *A.core.resid, in, ld_in, out, ld_out, w4, epi, inb, fact);
   } else {
-    run_csr(ctx, A, in, ld_in, out, ld_out, w4, epi, inb);
+    run_csr(ctx, A, in, ld_in, out, ld_out, w4, epi, inb, fact);
   }
   ctx->counters.spmm_calls++;
   ctx->counters.spmm_nnz_cols += A.nnz * w;
@@ -626,7 +666,7 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
 
 namespace {
 void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
-             int64_t w4, const Epi& epi, const __nv_bfloat16* inb) {
+             int64_t w4, const Epi& epi, const __nv_bfloat16* inb, bool fact) {
   const int64_t w8 = (w4 + 7) & ~int64_t(7);
   const int64_t ldp = inb ? w8 : w4;
   float* part = nullptr;
@@ -654,6 +694,14 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
     int U = 1;
     if (!getenv("RDM_SPMM_GV")) pick_gvu(c8, true, &G, &V, &U);
     if (const char* e = getenv("RDM_SPMM_U")) U = atoi(e);
+    if (fact) {   // value-free sums of bf16(s_j X_j) for the measured mappings
+#define RDM_SPMM_FCASE(g_, v_, u_) \
+  if (G == g_ && V == v_ && U == u_) { launch_spmm_bf<g_, v_, u_, true>(ctx, A, inb, w8, out, ld_out, part, ldp, w4, w8, chunk8, epi); fact = false; goto heavy; }
+      RDM_SPMM_FCASE(8, 1, 4) RDM_SPMM_FCASE(8, 2, 2) RDM_SPMM_FCASE(16, 2, 2) RDM_SPMM_FCASE(2, 1, 2)
+      RDM_SPMM_FCASE(1, 2, 1) RDM_SPMM_FCASE(1, 1, 1) RDM_SPMM_FCASE(4, 1, 2) RDM_SPMM_FCASE(32, 1, 2)
+#undef RDM_SPMM_FCASE
+      throw Error(RDM_ERR_STATE, "spmm: no factored bf16 kernel for G/V/U");
+    }
 #define RDM_SPMM_CASE(g_, v_, u_) \
   if (G == g_ && V == v_ && U == u_) launch_spmm_bf<g_, v_, u_>(ctx, A, inb, w8, out, ld_out, part, ldp, w4, w8, chunk8, epi); else
     RDM_SPMM_CASE(1, 1, 1) RDM_SPMM_CASE(1, 2, 1) RDM_SPMM_CASE(1, 3, 1) RDM_SPMM_CASE(1, 4, 1)
@@ -692,6 +740,7 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
     throw Error(RDM_ERR_ARG, "spmm: no kernel for G/V/U");
 #undef RDM_SPMM_CASE
   }
+heavy:
   if (A.n_heavy) {
     spmm_heavy_reduce<<<(unsigned)A.n_heavy, 128, 0, ctx->stream>>>(
         A.heavy_rows->as<int32_t>(), A.heavy_seg->as<int32_t>(), part, ldp, out, ld_out, w4, epi);
