@@ -368,6 +368,13 @@ def main():
     local_rank = int(os.environ.get("LOCAL_RANK", "0"))
     import synth
     wl = synth.WORKLOADS[a.workload]
+    if a.workload == "papers" and world < 8:
+        # BASELINE configs[4] is an 8-GPU stress case (≈13.7 GB CSR + ≈70 GB of
+        # dense slices per GPU at P = 8); fewer GPUs do not hold it
+        if rank == 0:
+            print(json.dumps({"metric": METRIC, "impl": a.impl, "unavailable":
+                              "papers100M-shaped workload is defined for 8 GPUs (BASELINE configs[4])"}))
+        return
 
     if a.impl == "reference":
         # Reference arm = the CPU oracle (tier framing): rank 0 only.

@@ -44,6 +44,7 @@
 #include <cuda.h>
 #include <cudaTypedefs.h>
 #include <cuda_bf16.h>
+#include <cuda_fp16.h>
 
 #include <algorithm>
 #include <cmath>
@@ -66,6 +67,10 @@ constexpr int kSmemBudget = 220 * 1024;
 // kind::f16 instruction descriptor: D f32, A/B bf16, K-major both, M = 128.
 __host__ __device__ constexpr uint32_t idesc_bf16(int N) {
   return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+}
+// the same with A/B fp16 (format 0)
+__host__ __device__ constexpr uint32_t idesc_f16(int N) {
+  return (1u << 4) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
 }
 
 __device__ __forceinline__ void bulk_load(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
@@ -110,6 +115,10 @@ __device__ __forceinline__ void tmem_st32u(uint32_t addr, const uint32_t (&v)[32
 __device__ __forceinline__ uint32_t bits2_bf16(uint32_t b) {
   return ((b & 1u) * 0x3F80u) | (((b >> 1) & 1u) * 0x3F800000u);
 }
+// … or two fp16 (1.0 = 0x3C00).
+__device__ __forceinline__ uint32_t bits2_f16(uint32_t b) {
+  return ((b & 1u) * 0x3C00u) | (((b >> 1) & 1u) * 0x3C000000u);
+}
 
 // Launch shape of one product (host-computed).
 struct TileShape {
@@ -121,9 +130,12 @@ struct TileShape {
   int R;              // > 0: concatenated-piece MMAs with R rotating accumulator sets
   int acc_cols;       // TMEM columns per accumulator buffer
   int dbg;            // timing experiments (RDM_TILE_DBG): 1 = skip the MMAs
+  const float* colscale;   // NP == 2: 2^e_n per output column (fp16 pieces are column-scaled)
 };
 
-// NP = bf16 pieces of s⊙X: 3 (fp32-class, RDM_PREC_FP32) or 1 (RDM_PREC_FAST).
+// NP = pieces of s⊙X: 2 fp16 pieces with a per-column power-of-two scale
+// (22 significant bits, fp32-class: RDM_PREC_FP32), 3 bf16 pieces (24 bits,
+// kept for comparison: RDM_TILE_PIECES=3) or 1 bf16 piece (RDM_PREC_FAST).
 template <int HS, int NP>
 __global__ void __launch_bounds__(384, 1)
 hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__ CUtensorMap tmB2d,
@@ -144,7 +156,8 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int total = sh.n_items * sh.tiles_n;
   for (int i = threadIdx.x; i < 256; i += blockDim.x)
-    lut[i] = make_uint4(bits2_bf16(i), bits2_bf16(i >> 2), bits2_bf16(i >> 4), bits2_bf16(i >> 6));
+    lut[i] = NP == 2 ? make_uint4(bits2_f16(i), bits2_f16(i >> 2), bits2_f16(i >> 4), bits2_f16(i >> 6))
+                     : make_uint4(bits2_bf16(i), bits2_bf16(i >> 2), bits2_bf16(i >> 4), bits2_bf16(i >> 6));
   // Two rings.  Shared-memory stage s: the B pieces of HS k-halves as
   // [half][piece][n_mma][64 bf16] (one 4-D TMA; pieces of a half adjacent, so
   // a concatenated MMA of N = 3 n_mma reads all three), then the halves' bits
@@ -220,7 +233,7 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__
     }
   } else if (warp == 1) {
     if (lane == 0) {
-      const uint32_t idesc = idesc_bf16(R ? NP * n_mma : n_mma);
+      const uint32_t idesc = NP == 2 ? idesc_f16(R ? NP * n_mma : n_mma) : idesc_bf16(R ? NP * n_mma : n_mma);
       // descriptors advance linearly: +stage_bytes per stage, +3·bpiece per
       // k half, +bpiece per piece, +32 B per k16 step (16-byte units)
       const uint64_t bd0 = sdesc(smem_u32(B_st(0)), 16, 1024);
@@ -259,10 +272,9 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__
 #pragma unroll
                 for (int j = 0; j < SK / 16; ++j, ++g) {   // 8 packed A columns, 32 B of B rows per k16
                   tc_mma_f16_ts(d_tmem, th + j * 8, bh + 2 * j, idesc, g > 0 ? 1u : 0u);
-                  if (NP == 3) {
-                    tc_mma_f16_ts(d_tmem, th + j * 8, bh + pc16 + 2 * j, idesc, 1u);
-                    tc_mma_f16_ts(d_tmem, th + j * 8, bh + 2 * pc16 + 2 * j, idesc, 1u);
-                  }
+#pragma unroll
+                  for (int pc = 1; pc < NP; ++pc)
+                    tc_mma_f16_ts(d_tmem, th + j * 8, bh + pc * pc16 + 2 * j, idesc, 1u);
                 }
               }
             }
@@ -341,10 +353,15 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__
         }
 #pragma unroll
         for (int i = 0; i < 32; i += 4)
-          if (n0 + c0 + i < sh.w)
-            *reinterpret_cast<float4*>(prow + c0 + i) =
-                make_float4(__uint_as_float(rr[i]), __uint_as_float(rr[i + 1]), __uint_as_float(rr[i + 2]),
-                            __uint_as_float(rr[i + 3]));
+          if (n0 + c0 + i < sh.w) {
+            float4 o = make_float4(__uint_as_float(rr[i]), __uint_as_float(rr[i + 1]), __uint_as_float(rr[i + 2]),
+                                   __uint_as_float(rr[i + 3]));
+            if (NP == 2) {   // undo the column scale of the fp16 pieces (exact: powers of two)
+              const float4 cs = __ldg(reinterpret_cast<const float4*>(sh.colscale + n0 + c0 + i));
+              o.x *= cs.x; o.y *= cs.y; o.z *= cs.z; o.w *= cs.w;
+            }
+            *reinterpret_cast<float4*>(prow + c0 + i) = o;
+          }
       }
       tc_fence_before();
       mbar_arrive(&tempty[acc]);
@@ -388,6 +405,66 @@ __global__ void tile_panels_kernel(const float* __restrict__ X, int64_t ldx, con
         p1[o] = m;
         p2[o] = l;
       }
+    }
+  }
+}
+
+// Column maxima of |s_k · X[hub_k][n]| over the K2 hub slots (bit patterns of
+// non-negative floats order like unsigned ints: atomicMax is exact and
+// order-independent).  Block: 32 columns x 8 k-lanes, 128 k per lane.
+__global__ void tile_colmax_kernel(const float* __restrict__ X, int64_t ldx, const int32_t* __restrict__ hub_ids,
+                                   const float* __restrict__ scale, int64_t K2, int64_t w,
+                                   unsigned int* __restrict__ colmax) {
+  __shared__ float red[8][33];
+  const int64_t n = (int64_t)blockIdx.y * 32 + threadIdx.x;
+  const int64_t k0 = (int64_t)blockIdx.x * 1024;
+  float m = 0.f;
+  if (n < w)
+    for (int64_t k = k0 + threadIdx.y; k < min(K2, k0 + 1024); k += 8)
+      m = fmaxf(m, fabsf(__ldg(scale + k) * __ldg(X + (int64_t)__ldg(hub_ids + k) * ldx + n)));
+  red[threadIdx.y][threadIdx.x] = m;
+  __syncthreads();
+  if (threadIdx.y == 0 && n < w) {
+    for (int i = 1; i < 8; ++i) m = fmaxf(m, red[i][threadIdx.x]);
+    atomicMax(colmax + n, __float_as_uint(m));
+  }
+}
+
+// fp16 pieces: y = s_k · X[hub_k][n] · 2^-e_n with e_n chosen so that the
+// column maximum lands in [2^13, 2^14) (far from fp16 overflow), hi = fp16(y),
+// lo = fp16(y − hi) (the difference is exact in fp32): 22 significant bits.
+// colscale[n] = 2^e_n for the epilogue.
+__global__ void tile_panels_f16_kernel(const float* __restrict__ X, int64_t ldx, const int32_t* __restrict__ hub_ids,
+                                       const float* __restrict__ scale, int64_t K2, int64_t w,
+                                       const unsigned int* __restrict__ colmax, __half* __restrict__ p0,
+                                       __half* __restrict__ p1, float* __restrict__ colscale) {
+  __shared__ float t[64][33];
+  __shared__ float inv[32];
+  const int64_t k0 = (int64_t)blockIdx.x * 64, n0 = (int64_t)blockIdx.y * 32;
+  if (threadIdx.y == 0) {
+    const int64_t n = n0 + threadIdx.x;
+    const float mx = n < w ? __uint_as_float(colmax[n]) : 0.f;
+    const int e = mx > 0.f ? ilogbf(mx) - 13 : 0;
+    inv[threadIdx.x] = ldexpf(1.f, -e);
+    if (blockIdx.x == 0 && n < w) colscale[n] = ldexpf(1.f, e);
+  }
+  for (int i = threadIdx.y; i < 64; i += 8) {
+    const int64_t k = k0 + i, n = n0 + threadIdx.x;
+    t[i][threadIdx.x] = (n < w) ? __ldg(scale + k) * __ldg(X + (int64_t)__ldg(hub_ids + k) * ldx + n) : 0.f;
+  }
+  __syncthreads();
+  for (int i = threadIdx.y; i < 32; i += 8) {
+    const int64_t n = n0 + i;
+    if (n >= w) break;
+#pragma unroll
+    for (int hk = 0; hk < 2; ++hk) {
+      const int kk = hk * 32 + threadIdx.x;
+      const float y = t[kk][i] * inv[i];
+      const __half h = __float2half_rn(y);
+      const __half l = __float2half_rn(y - __half2float(h));
+      const int64_t o = n * K2 + k0 + kk;
+      p0[o] = h;
+      p1[o] = l;
     }
   }
 }
@@ -452,13 +529,32 @@ bool hub_tiles_pay(const Core& c, int64_t w, int np) {
 
 void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx, int64_t w, float* part,
                        int64_t ldp, int np) {
-  RDM_CHECK_ARG(np == 1 || np == 3, "hub tiles: 1 or 3 bf16 pieces");
+  RDM_CHECK_ARG(np >= 1 && np <= 3, "hub tiles: 1, 2 or 3 pieces");
   const int64_t K2 = c.K2;
   __nv_bfloat16* pan = reinterpret_cast<__nv_bfloat16*>(ensure_ws(ctx->ws_core_b, (size_t)np * w * K2 * 2));
   dim3 pg((unsigned)(K2 / 64), (unsigned)ceil_div(w, 32));
-  tile_panels_kernel<<<pg, dim3(32, 8), 0, ctx->stream>>>(X, ldx, c.hub_ids->as<int32_t>(), c.scale->as<float>(), K2,
-                                                        w, pan, pan + w * K2, pan + 2 * w * K2, np);
-  RDM_LAUNCHED(ctx);
+  float* colscale = nullptr;
+  if (np == 2) {
+    // column scales: max |s·X| per column, then fp16 hi / lo pieces
+    const int64_t w4 = (w + 3) / 4 * 4;
+    float* cs = ensure_ws(ctx->ws_tile_cs, (size_t)2 * w4 * sizeof(float));
+    unsigned int* cmax = reinterpret_cast<unsigned int*>(cs + w4);
+    RDM_CUDA(cudaMemsetAsync(cmax, 0, w * sizeof(unsigned int), ctx->stream));
+    RDM_CUDA(cudaMemsetAsync(cs, 0, w4 * sizeof(float), ctx->stream));
+    dim3 mg((unsigned)ceil_div(K2, 1024), (unsigned)ceil_div(w, 32));
+    tile_colmax_kernel<<<mg, dim3(32, 8), 0, ctx->stream>>>(X, ldx, c.hub_ids->as<int32_t>(), c.scale->as<float>(),
+                                                           K2, w, cmax);
+    RDM_LAUNCHED(ctx);
+    tile_panels_f16_kernel<<<pg, dim3(32, 8), 0, ctx->stream>>>(
+        X, ldx, c.hub_ids->as<int32_t>(), c.scale->as<float>(), K2, w, cmax, reinterpret_cast<__half*>(pan),
+        reinterpret_cast<__half*>(pan + w * K2), cs);
+    RDM_LAUNCHED(ctx);
+    colscale = cs;
+  } else {
+    tile_panels_kernel<<<pg, dim3(32, 8), 0, ctx->stream>>>(X, ldx, c.hub_ids->as<int32_t>(), c.scale->as<float>(),
+                                                          K2, w, pan, pan + w * K2, pan + 2 * w * K2, np);
+    RDM_LAUNCHED(ctx);
+  }
   TileShape sh;
   sh.n_mma = (int)std::min<int64_t>(128, ((w + 15) / 16) * 16);
   sh.tiles_n = (int)ceil_div(w, 128);
@@ -477,6 +573,7 @@ void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx,
   sh.S = std::min(32, avail / sh.stage_bytes);
   sh.SA = std::min(8, (512 - 2 * sh.acc_cols) / (32 * sh.HS));
   sh.dbg = getenv("RDM_TILE_DBG") ? atoi(getenv("RDM_TILE_DBG")) : 0;
+  sh.colscale = colscale;
   RDM_CHECK_ARG(sh.S >= 2 && sh.SA >= 2, "hub tiles: TMEM/smem budget");
   const CUtensorMap tb = panel_map(pan, K2, w, sh.n_mma, sh.HS, np);
   // the three panels stacked as one 3w x K2 matrix: rows past a panel's w
@@ -486,7 +583,8 @@ void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx,
   const int64_t total = c.n_items * sh.tiles_n;
   const unsigned grid = (unsigned)std::min<int64_t>(total, ctx->num_sms);
   auto kern = np == 3 ? (sh.HS == 2 ? hub_tile_kernel<2, 3> : hub_tile_kernel<1, 3>)
-                      : (sh.HS == 2 ? hub_tile_kernel<2, 1> : hub_tile_kernel<1, 1>);
+             : np == 2 ? (sh.HS == 2 ? hub_tile_kernel<2, 2> : hub_tile_kernel<1, 2>)
+                       : (sh.HS == 2 ? hub_tile_kernel<2, 1> : hub_tile_kernel<1, 1>);
   RDM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
   kern<<<grid, 384, smem, ctx->stream>>>(tb, tb2, c.tiles->as<uint64_t>(), c.tile_cb->as<int32_t>(),
                                          c.item_tb->as<int32_t>(), part, sh);

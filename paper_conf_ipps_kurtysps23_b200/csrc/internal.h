@@ -161,6 +161,7 @@ struct rdm_ctx {
   int64_t panel_n = 0;
   std::vector<std::unique_ptr<rdm::Csr>> panels;
   std::unique_ptr<rdm::DevBuf> ws_panel_in;                    // all-gathered N x w_j input per slot
+  std::unique_ptr<rdm::DevBuf> ws_tile_cs;                     // fp16 hub tiles: column scales + maxima
   std::unique_ptr<rdm::DevBuf> ws_bf16;                        // RDM_PREC_FAST: bf16 copy of the SpMM input
   // phase timing
   bool timing = false;
@@ -245,7 +246,7 @@ void build_core(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, const int32_t*
 // summed per row block and scaled by s_i in the SpMM epilogue.
 bool build_hub_tiles(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, const int32_t* col_host,
                      const float* val_host);
-// np = bf16 pieces of s⊙X: 3 (fp32-class) or 1 (RDM_PREC_FAST).
+// np = pieces of s⊙X: 2 fp16 (fp32-class default), 3 bf16 (RDM_TILE_PIECES=3) or 1 bf16 (RDM_PREC_FAST).
 bool hub_tiles_pay(const Core& c, int64_t w, int np);
 void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx, int64_t w,
                        float* part, int64_t ldp, int np);

@@ -629,7 +629,14 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
     inb = xb;
     if (fact) epi.rscale = A.fscale->as<float>();
   }
-  const int np = ctx->prec == RDM_PREC_FAST ? 1 : 3;
+  // hub-tile pieces: 2 column-scaled fp16 pieces (fp32-class, default), 3 bf16
+  // pieces (RDM_TILE_PIECES=3, the earlier form) or 1 bf16 piece (fast)
+  // (measured, tools/exp_tiles.py: fp16 pairs pay where the tile is MMA-bound,
+  // w > 64: 1.53 → 1.44 ms at w = 128; narrower tiles are bound by the bit
+  // expansion and the extra column-max pass makes fp16 pairs slower)
+  int np = ctx->prec == RDM_PREC_FAST ? 1 : (w > 64 ? 2 : 3);
+  if (ctx->prec != RDM_PREC_FAST)
+    if (const char* e = getenv("RDM_TILE_PIECES")) np = atoi(e) == 3 ? 3 : 2;
   if (A.core.n_tiles && hub_tiles_pay(A.core, w, np)) {
     // binary hub tiles on the kind::f16 tensor cores (hubtiles.cu); the
     // residual CSR's epilogue adds s_i · Σ_items partial for hub rows.

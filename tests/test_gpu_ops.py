@@ -239,7 +239,8 @@ def test_spmm_hub_core_matches_oracle(torch_dev, w, K, monkeypatch):
 
 @pytest.mark.parametrize("w", [1, 4, 16, 41, 128, 130, 256, 301])
 @pytest.mark.parametrize("min_nnz,k2", [(1, 0), (40, 0), (1, 1024)])
-def test_spmm_hub_tiles_matches_oracle(torch_dev, w, min_nnz, k2, monkeypatch):
+@pytest.mark.parametrize("pieces", ["auto", "2", "3"])
+def test_spmm_hub_tiles_matches_oracle(torch_dev, w, min_nnz, k2, pieces, monkeypatch):
     """Binary hub tiles (kind::f16 tensor cores on 0/1 tiles against the
     3-piece bf16 split of s ⊙ X) + residual CSR == the plain product, with
     epilogues.  min_nnz forces the tile selection (every block with at least
@@ -247,6 +248,8 @@ def test_spmm_hub_tiles_matches_oracle(torch_dev, w, min_nnz, k2, monkeypatch):
     torch, dev = torch_dev
     import paper_conf_ipps_kurtysps23_b200 as rdm
     monkeypatch.setenv("RDM_TILE_MIN_NNZ", str(min_nnz))
+    if pieces != "auto":   # 2 column-scaled fp16 pieces / 3 bf16 pieces at every width
+        monkeypatch.setenv("RDM_TILE_PIECES", pieces)
     if k2:
         monkeypatch.setenv("RDM_TILE_K2", str(k2))
     g = synth.rmat(6000, 150000, seed=13)
@@ -271,12 +274,15 @@ def test_spmm_hub_tiles_matches_oracle(torch_dev, w, min_nnz, k2, monkeypatch):
     assert np.all(out[:, w:].cpu().numpy() == 0)
 
 
-def test_spmm_hub_tiles_wide_range_values(torch_dev, monkeypatch):
-    """Inputs spanning 2^±30 and exact zeros: the three bf16 pieces keep
-    fp32-class relative accuracy per row (no flush of the small pieces)."""
+@pytest.mark.parametrize("pieces", ["2", "3"])
+def test_spmm_hub_tiles_wide_range_values(torch_dev, pieces, monkeypatch):
+    """Inputs spanning 2^±30 per row and exact zeros: the column-scaled fp16
+    pieces and the bf16 pieces keep the fp32 gate (normwise per tensor,
+    reading R26) — no overflow, no lost columns."""
     torch, dev = torch_dev
     import paper_conf_ipps_kurtysps23_b200 as rdm
     monkeypatch.setenv("RDM_TILE_MIN_NNZ", "1")
+    monkeypatch.setenv("RDM_TILE_PIECES", pieces)
     g = synth.rmat(6000, 150000, seed=14)
     ctx = rdm.Context(device=0)
     ctx.set_graph(g.rowptr, g.col, g.val)
