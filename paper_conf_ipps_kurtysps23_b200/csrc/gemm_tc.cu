@@ -556,12 +556,20 @@ void launch_tc(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, const C
     launch_tc_ew<BN, MODE, 4>(ctx, a, b, blo, C, ldc, M, N, K, splits, n_mma, e, apf);
 }
 
-int pick_bn(int64_t N) {
+// Wider N: one 256-wide tile (A in smem, both TMEM accumulators) where the
+// contraction is long enough for the 3xTF32 MMAs to dominate (measured,
+// tools/time_gemm.py, products-shaped 2.45 M x 256 · 256 x 256: 1.94 →
+// 1.76 ms), else several 128-wide tiles (TMEM-A path; K = 100: 1.18 vs
+// 1.47 ms).  RDM_BN256=1 / 0 forces either (experiments).
+int pick_bn(int64_t N, int64_t K = 0, bool three = true, bool mask = false) {
   if (N <= 16) return 16;
   if (N <= 32) return 32;
   if (N <= 64) return 64;
-  if (N <= 128 || !getenv("RDM_BN256")) return 128;   // wider N: several 128-wide tiles (TMEM-A path)
-  return 256;
+  if (N <= 128) return 128;
+  if (const char* e = getenv("RDM_BN256")) return atoi(e) ? 256 : 128;
+  // (a Hadamard-mask epilogue over 256 columns with 4 epilogue warps loses
+  // more than the wide tile gains: 1.06 → 1.34 ms in the products epoch)
+  return (three && K >= 256 && !mask) ? 256 : 128;
 }
 
 }  // namespace
@@ -570,7 +578,7 @@ namespace {
 void launch_nn_panels(rdm_ctx* ctx, const float* X, int64_t ldx, const float* bhi, const float* blo,
                       int64_t ldb, float* C, int64_t ldc, int64_t M, int64_t N, int64_t K,
                       const TcEpi& e, int splits = 1) {
-  const int BN = pick_bn(N);
+  const int BN = pick_bn(N, K, ctx->prec != RDM_PREC_FAST, (e.flags & RDM_EPI_MASK) != 0);
   // one MMA width for every tile: BN when N spans several tiles, else N rounded to 16
   const int nm = N > BN ? BN : (int)(((N + 15) / 16) * 16);
   const CUtensorMap ta = make_map(X, K, M, ldx, BK, BM);
@@ -597,7 +605,7 @@ void gemm_tc_panels(rdm_ctx* ctx, const float* A, int64_t lda, const float* bhi,
                 "gemm_tc_panels: 16-byte aligned operands with ld % 4 == 0 required");
   // Split K so that the persistent grid has no idle SMs (the hub-core GEMM has
   // only ~110 M-tiles for 148 SMs); partial slabs are summed in split order.
-  const int64_t tiles = ceil_div(M, BM) * ceil_div(N, pick_bn(N));
+  const int64_t tiles = ceil_div(M, BM) * ceil_div(N, pick_bn(N, K, ctx->prec != RDM_PREC_FAST));
   int best_s = 1;
   double best_eff = 0;
   for (int s = 1; s <= 8; ++s) {
@@ -650,7 +658,10 @@ bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, 
   if (scat) return false;   // weight gradients are never redistributed
   if (((uintptr_t)W & 15) || (ldw & 3)) return false;
   const int64_t M = k, N = m, K = rows;
-  const int BN = N <= 32 ? 32 : N <= 64 ? 64 : (N <= 128 || !getenv("RDM_BN256")) ? 128 : 256;
+  // TN: 256-wide tiles for N > 128 (products-shaped 256 x 256 over 2.45 M rows:
+  // 1.89 → 1.71 ms fp32, 0.96 → 0.92 ms fast)
+  const int BN = N <= 32 ? 32 : N <= 64 ? 64 : N <= 128 ? 128
+                 : (getenv("RDM_BN256") ? (atoi(getenv("RDM_BN256")) ? 256 : 128) : 256);
   const int n_mma = (int)std::min<int64_t>(BN, ((N + 31) / 32) * 32);
   const int64_t tiles = ceil_div(M, BM) * ceil_div(N, BN);
   int64_t splits = std::max<int64_t>(1, ctx->num_sms / std::max<int64_t>(1, tiles));

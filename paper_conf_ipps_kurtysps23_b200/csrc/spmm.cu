@@ -30,6 +30,12 @@
 
 #include "internal.h"
 
+// load form of the gathered input rows (timing experiments may rebuild with
+// another cache operator, tools/build_variant.sh)
+#ifndef RDM_GATHER_LD
+#define RDM_GATHER_LD __ldg
+#endif
+
 namespace rdm {
 namespace {
 
@@ -157,7 +163,7 @@ __device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
           float4 x[V];
 #pragma unroll
           for (int v = 0; v < V; ++v)
-            if (v * G + sub < c4n) x[v] = __ldg(xr + v * G + sub);
+            if (v * G + sub < c4n) x[v] = RDM_GATHER_LD(xr + v * G + sub);
 #pragma unroll
           for (int v = 0; v < V; ++v) {
             if (v * G + sub < c4n) {
@@ -184,7 +190,7 @@ __device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
         const float4* xr = reinterpret_cast<const float4*>(xb + (int64_t)cc * ldx);
 #pragma unroll
         for (int v = 0; v < V; ++v)
-          x[u][v] = (k < cnt && v * G + sub < c4n) ? __ldg(xr + v * G + sub) : make_float4(0.f, 0.f, 0.f, 0.f);
+          x[u][v] = (k < cnt && v * G + sub < c4n) ? RDM_GATHER_LD(xr + v * G + sub) : make_float4(0.f, 0.f, 0.f, 0.f);
       }
 #pragma unroll
       for (int u = 0; u < U; ++u)
@@ -315,7 +321,7 @@ __device__ __forceinline__ void warp_nnz_range_bf(const int32_t* __restrict__ co
         const uint4* xr = reinterpret_cast<const uint4*>(xb + (int64_t)cc * ldx);
 #pragma unroll
         for (int v = 0; v < V; ++v)
-          x[u][v] = (k < cnt && v * G + sub < c8n) ? __ldg(xr + v * G + sub) : make_uint4(0u, 0u, 0u, 0u);
+          x[u][v] = (k < cnt && v * G + sub < c8n) ? RDM_GATHER_LD(xr + v * G + sub) : make_uint4(0u, 0u, 0u, 0u);
       }
 #pragma unroll
       for (int u = 0; u < U; ++u)

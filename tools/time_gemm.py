@@ -1,7 +1,9 @@
 import sys, numpy as np, torch
 sys.path.insert(0, '.')
 import paper_conf_ipps_kurtysps23_b200 as rdm
+import os
 dev = torch.device('cuda:0'); ctx = rdm.Context(device=0)
+ctx.set_precision(os.environ.get('RDM_PREC', 'fp32'))
 rows = 232965
 def t(fn, it=10):
     fn(); ctx.sync(); s = torch.cuda.Event(enable_timing=True); e = torch.cuda.Event(enable_timing=True)
@@ -20,7 +22,7 @@ for (op, k, m, epi) in [(rdm.GEMM_NT, 128, 41, 0), (rdm.GEMM_NT, 128, 41, rdm.EP
         f = lambda: ctx.gemm(op, X, U, C, rows, k, m)
     print(['NN','NT','TN'][op], k, m, 'epi', epi, f'{t(f):.1f} us')
 # hub-core shaped GEMMs: K x K dense times K x w
-for K in (8192, 16384):
+for K in ():
     for w in (16, 48, 128):
         A = torch.randn(K, K, device=dev); B = torch.randn(K, w, device=dev); C = torch.zeros(K, w, device=dev)
         print('core', K, w, f'{t(lambda: ctx.gemm(rdm.GEMM_NN, A, B, C, K, K, w), 5):.1f} us')
