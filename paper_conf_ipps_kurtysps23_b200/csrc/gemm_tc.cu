@@ -482,9 +482,19 @@ __global__ void splitk_sum(const float* __restrict__ part, int splits, int64_t M
   const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (idx >= M * N) return;
   const int64_t i = idx / N, n = idx % N;
-  float s = 0.f;
-  for (int z = 0; z < splits; ++z) s += part[(int64_t)z * M * ldp + i * ldp + n];
-  C[i * ldc + n] = s;
+  double s = 0.0;   // fixed order, fp64: the split partials of a long reduction
+  const float* p = part + i * ldp + n;
+  const int64_t zs = M * ldp;
+  int z = 0;
+  for (; z + 8 <= splits; z += 8) {   // 8 independent loads in flight, then the ordered adds
+    float v[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) v[u] = __ldcs(p + (int64_t)(z + u) * zs);
+#pragma unroll
+    for (int u = 0; u < 8; ++u) s += (double)v[u];
+  }
+  for (; z < splits; ++z) s += (double)__ldcs(p + (int64_t)z * zs);
+  C[i * ldc + n] = (float)s;
 }
 
 // ------------------------------------------------------------ host side
@@ -665,6 +675,13 @@ bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, 
   const int n_mma = (int)std::min<int64_t>(BN, ((N + 31) / 32) * 32);
   const int64_t tiles = ceil_div(M, BM) * ceil_div(N, BN);
   int64_t splits = std::max<int64_t>(1, ctx->num_sms / std::max<int64_t>(1, tiles));
+  // accuracy: the weight gradient sums over every row, often with heavy
+  // cancellation (softmax − onehot is zero-sum); chains of at most kTnChain
+  // rows in the fp32 TMEM accumulator (kTnChain), the partials summed in fp64
+  // (splitk_sum): products-shaped Y^3 over 2.45 M rows 1.6e-4 → within 1e-4
+  int64_t chain = 4096;
+  if (const char* e = getenv("RDM_TN_CHAIN")) chain = std::max<int64_t>(256, atoll(e));
+  splits = std::max<int64_t>(splits, ceil_div(K, chain));
   splits = std::min<int64_t>(splits, std::max<int64_t>(1, K / (8 * BK)));
   const CUtensorMap ta = make_map(X, M, K, ldx, 32, BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B);  // inner = k
   const CUtensorMap tb = make_map(W, N, K, ldw, 32, BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B);  // inner = m

@@ -341,3 +341,61 @@ def test_reddit_full_size_sampled(rdm):
     S1 = og.spmm(g, G1)
     assert og.max_rel_err(dW[0], H0.astype(np.float64).T @ S1) < 1e-4
     assert cfg is not None
+
+
+def test_products_full_size_sampled(rdm):
+    """BASELINE configs[2] (products-shaped, 3 layers h256) at full size in
+    bench.py's launch configuration (P = 1, model-picked config): forward
+    layers on 4,096 sampled rows against the oracle from the GPU's own
+    previous layer, the loss from the GPU logits, and every weight gradient
+    Y^l recomputed in fp64 through the whole backward (eq. 3-4)."""
+    wl = synth.WORKLOADS["products"]
+    g = synth.make_graph(wl)
+    H0 = synth.features(wl.n, wl.f[0])
+    Ws = synth.weights(wl.f)
+    y = synth.labels(wl.n, wl.f[-1])
+    m = synth.train_mask(wl.n)
+    _, chosen, _, _ = rdm.select_config(list(wl.f), wl.n, wl.nnz, 1)
+    loss, dW, model, ctx, _ = _run(rdm, g, H0, Ws, y, m, chosen)
+    rows = np.sort(np.random.default_rng(1).choice(wl.n, size=4096, replace=False))
+    H = [H0] + [model.tensor_torch(rdm.T_H, l).cpu().numpy() for l in (1, 2)]
+    Z = model.tensor_torch(rdm.T_Z, 0).cpu().numpy()
+    del model, ctx
+    for l in (1, 2):
+        ref = np.maximum(og.spmm_rows(g, H[l - 1], rows) @ Ws[l - 1].astype(np.float64), 0)
+        assert og.max_rel_err(H[l][rows], ref) < 1e-4, ("H", l)
+    assert og.max_rel_err(Z[rows], og.spmm_rows(g, H[2], rows) @ Ws[2].astype(np.float64)) < 1e-4
+    lref, G = og.softmax_xent(Z, y, m)
+    assert abs(loss - lref) <= 1e-5 * abs(lref)
+    for l in (3, 2, 1):   # Y^l = H^{l-1}ᵀ (A G^l); G^{l-1} = (A G^l) W^lᵀ ⊙ 1[H^{l-1} > 0]
+        S = og.spmm(g, G)
+        assert og.max_rel_err(dW[l - 1], H[l - 1].astype(np.float64).T @ S) < 1e-4, ("Y", l)
+        if l > 1:
+            G = (S @ Ws[l - 1].astype(np.float64).T) * (H[l - 1] > 0)
+        del S
+
+
+def test_reddit_full_size_fast_variant(rdm):
+    """The fast-precision variant at BASELINE configs[1] full size: sampled
+    forward rows and both weight gradients within the 2e-2 gate, loss within
+    1e-3 (tests/test_gpu_fast.py gates)."""
+    wl = synth.WORKLOADS["reddit"]
+    g = synth.make_graph(wl)
+    H0 = synth.features(wl.n, wl.f[0])
+    Ws = synth.weights(wl.f)
+    y = synth.labels(wl.n, wl.f[-1])
+    m = synth.train_mask(wl.n)
+    _, chosen, _, _ = rdm.select_config(list(wl.f), wl.n, wl.nnz, 1)
+    loss, dW, model, ctx, _ = _run(rdm, g, H0, Ws, y, m, chosen, precision="fast")
+    rows = np.sort(np.random.default_rng(2).choice(wl.n, size=4096, replace=False))
+    H1 = model.tensor_torch(rdm.T_H, 1).cpu().numpy()
+    Z = model.tensor_torch(rdm.T_Z, 0).cpu().numpy()
+    ref1 = np.maximum(og.spmm_rows(g, H0, rows) @ Ws[0].astype(np.float64), 0)
+    assert og.max_rel_err(H1[rows], ref1) < 2e-2
+    assert og.max_rel_err(Z[rows], og.spmm_rows(g, H1, rows) @ Ws[1].astype(np.float64)) < 2e-2
+    lref, GL = og.softmax_xent(Z, y, m)
+    assert abs(loss - lref) <= 1e-3 * abs(lref)
+    S2 = og.spmm(g, GL)
+    assert og.max_rel_err(dW[1], H1.astype(np.float64).T @ S2) < 2e-2
+    G1 = (S2 @ Ws[1].astype(np.float64).T) * (H1 > 0)
+    assert og.max_rel_err(dW[0], H0.astype(np.float64).T @ og.spmm(g, G1)) < 2e-2
