@@ -52,8 +52,9 @@ struct TcShape {
   int64_t M, N, K, k_per_split;
   int tiles_m, tiles_n, splits, n_mma;
   int pf;   // issue L2 prefetches of A through tmApf
-  int dbg;  // timing experiments only (RDM_TC_DBG): 1 = skip split, 2 = skip MMA
+  int dbg;  // timing experiments only (RDM_TC_DBG): 1 = skip split, 2 = skip MMA, 4 = skip stores
   int one;  // RDM_PREC_FAST: 1xTF32 (one MMA per k step, no lo operands)
+  int tstore;  // epilogue stores through TMA (tmC) — MODE 0, one split, no fused scatter
 };
 
 // A operand placement.  For BN ≤ 128 the converter writes A's hi / lo split
@@ -75,7 +76,9 @@ struct Cfg {
   static constexpr int kABytes = BM * BK * 4;   // 16 KB
   static constexpr int kBBytes = BN * BK * 4;
   static constexpr int kStageBytes = (kTmemA ? 1 : 2) * kABytes + 2 * kBBytes;
-  static constexpr int kEpiBytes = EW * 32 * 33 * 4;  // per-warp 32 x 32 transpose tiles (+1 pad)
+  // per epilogue warp 5 KB (1024-aligned): a 32 x 33 transpose tile, or the
+  // 32 x 32 swizzled box of a TMA store
+  static constexpr int kEpiBytes = EW * 5120;
   static constexpr int kBudget = 224 * 1024 - kEpiBytes - 1024 - 256;
   // deep rings hide TMA latency; with A in TMEM each stage also takes 64 columns
   static constexpr int kMaxStages = kTmemA ? (512 - 2 * kNAcc * kAccCols) / (2 * BK) : 4;
@@ -148,7 +151,7 @@ template <int BN, int MODE, int EW>
 __global__ void __launch_bounds__(256 + 32 * EW, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const __grid_constant__ CUtensorMap tmBlo, const __grid_constant__ CUtensorMap tmApf,
-               float* __restrict__ C, int64_t ldc,
+               const __grid_constant__ CUtensorMap tmC, float* __restrict__ C, int64_t ldc,
                TcShape sh, TcEpi epi) {
   using CF = Cfg<BN, EW>;
   constexpr int S = CF::kStages;
@@ -359,7 +362,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   } else if (warp >= 8) {
     const int q = warp & 3;                    // TMEM lane quadrant of this warp
     const int half = (warp - 8) >> 2;          // column half (chunks 32 apart)
-    float* tb = epi_smem + (warp - 8) * 32 * 33;  // 32 x 32 transpose tile
+    float* tb = epi_smem + (warp - 8) * 1280;   // 32 x 33 transpose tile / 32 x 32 TMA box
     int it = 0;
     for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
       int64_t kbeg;
@@ -392,12 +395,13 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         }
         // lane owns row (row0 + lane): epilogue in registers — the mask row
         // segment is read as 8 independent 128-bit loads per lane — then
-        // transpose through smem and write column-coalesced.
+        // either a TMA store of the 32 x 32 block or a transpose through smem
+        // and column-coalesced stores.
+        float v[32];
+#pragma unroll
+        for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
         if (MODE == 0 && epi.flags) {
           const int64_t row = row0 + lane;
-          float v[32];
-#pragma unroll
-          for (int i = 0; i < 32; ++i) v[i] = __uint_as_float(r[i]);
           if (epi.flags & RDM_EPI_BIAS) {
 #pragma unroll
             for (int i = 0; i < 32; ++i)
@@ -421,15 +425,30 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
               v[4 * j + 3] = mk[j].w > 0.f ? v[4 * j + 3] : 0.f;
             }
           }
-#pragma unroll
-          for (int i = 0; i < 32; ++i) tb[lane * 33 + i] = v[i];
-        } else {
-#pragma unroll
-          for (int i = 0; i < 32; ++i) tb[lane * 33 + i] = __uint_as_float(r[i]);
         }
+        if (sh.tstore) {
+          // the lane's row as 8 float4 chunks of the 128-byte-swizzled box
+          // (chunk j of row r at j ^ (r & 7): conflict-free); the TMA engine
+          // writes the 32 x 32 block, clipping rows ≥ M and columns ≥ N
+          if (lane == 0) bulk_wait_read0();   // the previous box has left shared memory
+          __syncwarp();
+          float4* box = reinterpret_cast<float4*>(tb);
+#pragma unroll
+          for (int j = 0; j < 8; ++j)
+            box[lane * 8 + (j ^ (lane & 7))] = make_float4(v[4 * j], v[4 * j + 1], v[4 * j + 2], v[4 * j + 3]);
+          fence_proxy_async();
+          __syncwarp();
+          if (lane == 0 && !(sh.dbg & 4)) {
+            tma_store_2d(&tmC, tb, (int)(n0 + c0), (int)row0);
+            bulk_commit();
+          }
+          continue;
+        }
+#pragma unroll
+        for (int i = 0; i < 32; ++i) tb[lane * 33 + i] = v[i];
         __syncwarp();
         const int64_t col = n0 + c0 + lane;
-        if (col < sh.N) {
+        if (col < sh.N && !(sh.dbg & 4)) {
           const int nrows = (sh.M - row0) < 32 ? (int)(sh.M - row0) : 32;
 #pragma unroll 8
           for (int rr = 0; rr < nrows; ++rr) Cz[(row0 + rr) * ldc + col] = tb[rr * 33 + lane];
@@ -450,6 +469,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       tc_fence_before();
       mbar_arrive(&tempty[acc]);
     }
+    if (sh.tstore && lane == 0) bulk_wait0();   // every TMA store of this warp has landed
   }
   tc_fence_before();
   __syncthreads();
@@ -548,10 +568,14 @@ void launch_tc_ew(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, cons
   const char* dbg = getenv("RDM_TC_DBG");
   sh.dbg = dbg ? atoi(dbg) : 0;
   sh.one = ctx->prec == RDM_PREC_FAST ? 1 : 0;
+  // TMA-store epilogue: plain row-major output (one split, no fused scatter)
+  sh.tstore = (MODE == 0 && splits == 1 && !e.scat.P && !(getenv("RDM_NO_TSTORE") && atoi(getenv("RDM_NO_TSTORE"))))
+                  ? 1 : 0;
+  const CUtensorMap tc = sh.tstore ? make_map(C, N, M, ldc, 32, 32) : a;
   const int64_t total = (int64_t)sh.tiles_m * sh.tiles_n * splits;
   const unsigned grid = (unsigned)std::min<int64_t>(total, ctx->num_sms);
-  gemm_tc_kernel<BN, MODE, EW><<<grid, CF::kThreads, CF::kSmem, ctx->stream>>>(a, b, blo, apf ? *apf : a, C, ldc,
-                                                                  sh, e);
+  gemm_tc_kernel<BN, MODE, EW><<<grid, CF::kThreads, CF::kSmem, ctx->stream>>>(a, b, blo, apf ? *apf : a, tc, C,
+                                                                  ldc, sh, e);
   RDM_LAUNCHED(ctx);
 }
 
@@ -595,7 +619,10 @@ void launch_nn_panels(rdm_ctx* ctx, const float* X, int64_t ldx, const float* bh
   const CUtensorMap tb = make_map(bhi, K, N, ldb, BK, BN);
   const CUtensorMap tbl = make_map(blo, K, N, ldb, BK, BN);
   // L2-prefetch map: 128 x 128 fp32 boxes (512-byte row segments), no swizzle
-  const bool pf = K > 4 * BK && !getenv("RDM_NO_PF");
+  // (off by default: measured at the end of round 1, tools/time_gemm.py, the
+  // 232,965 x 602 · 602 x 128 NN runs 231 → 225 µs fp32 and 175 → 150 µs fast
+  // without it; RDM_PF=1 re-enables it for experiments)
+  const bool pf = K > 4 * BK && getenv("RDM_PF") && atoi(getenv("RDM_PF"));
   const CUtensorMap tpf = pf ? make_map(X, K, M, ldx, 4 * BK, BM, CU_TENSOR_MAP_SWIZZLE_NONE) : ta;
   const CUtensorMap* p = pf ? &tpf : nullptr;
   switch (BN) {
