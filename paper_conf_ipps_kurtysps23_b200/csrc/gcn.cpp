@@ -287,6 +287,12 @@ struct rdm_gcn {
   // P/R_A x R_A grid, SpMMs broadcast inside column groups, redistributions
   // stay inside panel groups (panels.cpp).  0 = full replication.
   int RA = 0;
+  // weight-gradient GEMMs (S_TN) run on a side stream: they overlap the rest
+  // of the backward pass and are joined before the gradient reduction
+  cudaStream_t side = nullptr;
+  cudaEvent_t ev_fork = nullptr, ev_join = nullptr;
+  bool side_pending = false;
+  std::unique_ptr<rdm::DevBuf> ws_side;   // split-K partials of the side-stream TN
   int64_t gver = -1;
 };
 
@@ -522,6 +528,11 @@ void create(rdm_gcn* g) {
   plan_info(pl, g->fwd, g->bwd, n, &g->info, g->RA);
   g->info.workspace_bytes = g->ws_bytes;
   if (ctx->transport == RDM_TRANSPORT_P2P && P > 1 && !g->RA) setup_fusion(g);
+  if (!(getenv("RDM_NO_SIDE") && atoi(getenv("RDM_NO_SIDE")))) {
+    RDM_CUDA(cudaStreamCreateWithFlags(&g->side, cudaStreamNonBlocking));
+    RDM_CUDA(cudaEventCreateWithFlags(&g->ev_fork, cudaEventDisableTiming));
+    RDM_CUDA(cudaEventCreateWithFlags(&g->ev_join, cudaEventDisableTiming));
+  }
 }
 
 void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
@@ -583,6 +594,21 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
       break;
     }
     case S_TN: {
+      // fork onto the side stream (inputs are ready on the compute stream);
+      // its own split-K workspace, joined in do_backward
+      const bool use_side = g->side != nullptr;
+      cudaStream_t main = ctx->stream;
+      if (use_side) {
+        RDM_CUDA(cudaEventRecord(g->ev_fork, main));
+        RDM_CUDA(cudaStreamWaitEvent(g->side, g->ev_fork, 0));
+        ctx->stream = g->side;
+        std::swap(ctx->ws_gemm, g->ws_side);
+        g->side_pending = true;
+      }
+      struct Restore {
+        rdm_ctx* c; rdm_gcn* g; cudaStream_t m; bool on;
+        ~Restore() { if (on) { c->stream = m; std::swap(c->ws_gemm, g->ws_side); } }
+      } restore{ctx, g, main, use_side};
       Phase ph(ctx, RDM_PH_GEMM);
       const int64_t fin = g->f[s.wl - 1], fout = g->f[s.wl];
       for (int i = 0; i < nl; ++i) {
@@ -720,6 +746,11 @@ void do_backward(void* a_) {
   if (!ctx->virtual_group())
     for (int l = 1; l <= g->L; ++l) g->dwp[0][l] = a->dW[l - 1];
   for (auto& s : g->bwd) run_step(g, s, a->W);
+  if (g->side_pending) {   // every weight gradient is in place before the reduction
+    RDM_CUDA(cudaEventRecord(g->ev_join, g->side));
+    RDM_CUDA(cudaStreamWaitEvent(ctx->stream, g->ev_join, 0));
+    g->side_pending = false;
+  }
   const int nl = ctx->nlocal();
   for (int l = 1; l <= g->L; ++l) {
     const int64_t cnt = g->f[l - 1] * g->f[l];
@@ -997,6 +1028,12 @@ rdm_status rdm_gcn_destroy(rdm_gcn* g) {
     cudaStreamDestroy(g->cs);
     cudaEventDestroy(g->ev_ready);
     cudaEventDestroy(g->ev_free);
+  }
+  if (g->side) {
+    cudaStreamSynchronize(g->side);
+    cudaStreamDestroy(g->side);
+    cudaEventDestroy(g->ev_fork);
+    cudaEventDestroy(g->ev_join);
   }
   if (!g->ipc_opened.empty()) {
     // no rank may free a slice a peer still maps: close, then fence, then free
