@@ -611,8 +611,11 @@ int pick_bn(int64_t N, int64_t K = 0, bool three = true, bool mask = false) {
 namespace {
 void launch_nn_panels(rdm_ctx* ctx, const float* X, int64_t ldx, const float* bhi, const float* blo,
                       int64_t ldb, float* C, int64_t ldc, int64_t M, int64_t N, int64_t K,
-                      const TcEpi& e, int splits = 1) {
-  const int BN = pick_bn(N, K, ctx->prec != RDM_PREC_FAST, (e.flags & RDM_EPI_MASK) != 0);
+                      const TcEpi& e, int splits = 1, bool wide_ok = true) {
+  // (256-wide tiles only for single-split calls: the split-K hub-core GEMM of
+  // the GraphSAINT subgraphs ran slower with them)
+  const int BN = (splits == 1 && wide_ok) ? pick_bn(N, K, ctx->prec != RDM_PREC_FAST, (e.flags & RDM_EPI_MASK) != 0)
+                                         : pick_bn(N, 0, false);
   // one MMA width for every tile: BN when N spans several tiles, else N rounded to 16
   const int nm = N > BN ? BN : (int)(((N + 15) / 16) * 16);
   const CUtensorMap ta = make_map(X, K, M, ldx, BK, BM);
@@ -642,7 +645,7 @@ void gemm_tc_panels(rdm_ctx* ctx, const float* A, int64_t lda, const float* bhi,
                 "gemm_tc_panels: 16-byte aligned operands with ld % 4 == 0 required");
   // Split K so that the persistent grid has no idle SMs (the hub-core GEMM has
   // only ~110 M-tiles for 148 SMs); partial slabs are summed in split order.
-  const int64_t tiles = ceil_div(M, BM) * ceil_div(N, pick_bn(N, K, ctx->prec != RDM_PREC_FAST));
+  const int64_t tiles = ceil_div(M, BM) * ceil_div(N, pick_bn(N, 0, false));
   int best_s = 1;
   double best_eff = 0;
   for (int s = 1; s <= 8; ++s) {
@@ -655,7 +658,7 @@ void gemm_tc_panels(rdm_ctx* ctx, const float* A, int64_t lda, const float* bhi,
     }
   }
   if (best_s == 1) {
-    launch_nn_panels(ctx, A, lda, bhi, blo, ldb, C, ldc, M, N, K, TcEpi{0, nullptr, nullptr, 0});
+    launch_nn_panels(ctx, A, lda, bhi, blo, ldb, C, ldc, M, N, K, TcEpi{0, nullptr, nullptr, 0}, 1, false);
     return;
   }
   const int64_t ldo = roundup4(N);
