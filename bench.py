@@ -252,14 +252,19 @@ def saint_main(a, world, rank, local_rank):
     it = [0]
     sizes = []
 
+    cur = [(n0, nnz0)]
+
     def step():
-        n_s, nnz_s = sam.sample(it[0])
-        sizes.append((n_s, nnz_s))
+        # train on the sampled subgraph (enqueued, asynchronous), then build the
+        # next one on the sampler's stream while the GPU trains (rdm_saint_sample
+        # double-buffers its subgraphs)
+        sizes.append(cur[0])
         model.saint_input(Hd, yd, md)
         model.forward(Wd, loss)
         model.backward(Wd, dW)
         it[0] += 1
         ctx.adam_step(Wd, dW, mo, ve, it[0], lr=0.01)
+        cur[0] = sam.sample(it[0])
 
     for _ in range(max(3, a.warmup)):
         step()
@@ -279,6 +284,7 @@ def saint_main(a, world, rank, local_rank):
     e0.record(stream)
     for _ in range(a.steps):
         step()
+    sam.wait()   # the last step's subgraph build (sampler stream) inside the bracket
     e1.record(stream)
     torch.cuda.synchronize(dev)
     clocks = clk.stop()

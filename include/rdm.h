@@ -477,6 +477,11 @@ rdm_status rdm_saint_destroy(rdm_saint* s);
  * Returns its vertex and entry counts.  Synchronises the ctx stream (the
  * host needs the sizes for the executor's launch shapes). */
 rdm_status rdm_saint_sample(rdm_saint* s, int64_t iteration, int64_t* n_sub, int64_t* nnz_sub);
+/* Make the ctx's stream wait for the sampler's latest subgraph build (which
+ * runs on the sampler's own stream and double-buffers its subgraphs, so a
+ * sample can overlap the training of the previous subgraph).  The executor
+ * does this itself when it switches subgraphs; for timing brackets. */
+rdm_status rdm_saint_wait(rdm_saint* s);
 /* Device pointers to the current subgraph: nodes[n] (int32 original ids,
  * ascending), rowptr[n+1] (int64), col[nnz] (int32 new ids), val[nnz]. */
 rdm_status rdm_saint_subgraph(const rdm_saint* s, const int32_t** nodes, const int64_t** rowptr,

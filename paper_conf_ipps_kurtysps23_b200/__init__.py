@@ -53,6 +53,7 @@ EXPORTS = [
     "rdm_set_transport", "rdm_get_transport", "rdm_debug_disable_tc",
     "rdm_set_precision", "rdm_get_precision", "rdm_set_graph_panels", "rdm_partition_tile",
     "rdm_redistribute_panels", "rdm_spmm_panels", "rdm_max_replication", "rdm_select_config_ra",
+    "rdm_saint_wait",
 ]
 
 
@@ -116,6 +117,7 @@ _sig = {
     "rdm_set_timing": [_vp, _int],
     "rdm_set_transport": [_vp, _int],
     "rdm_set_precision": [_vp, _int],
+    "rdm_saint_wait": [_vp],
     "rdm_select_config_ra": [_int, _pi64, _i64, _i64, _int, _int, _int, _pi64, ctypes.POINTER(_int),
                              _pi64, ctypes.POINTER(ctypes.c_double), _pi64],
     "rdm_set_graph_panels": [_vp, _int, _i64, _i64, _vp, _vp, _vp, _int],
@@ -537,6 +539,10 @@ class Saint:
         n, nnz = _i64(), _i64()
         self.ctx._c(_lib.rdm_saint_sample(self.h, int(iteration), ctypes.byref(n), ctypes.byref(nnz)))
         return n.value, nnz.value
+
+    def wait(self):
+        """The context's stream waits for the latest subgraph build (rdm.h rdm_saint_wait)."""
+        self.ctx._c(_lib.rdm_saint_wait(self.h))
 
     def subgraph(self):
         """Copies of the current subgraph: nodes, rowptr, col, val (torch, on the device)."""

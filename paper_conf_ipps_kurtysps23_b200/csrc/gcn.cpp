@@ -282,6 +282,7 @@ struct rdm_gcn {
   // refreshed whenever the sampler's version changes)
   const rdm::Graph* graph = nullptr;
   rdm_saint* saint = nullptr;
+  int sbuf = 0;           // sampler buffer this instance trains on
   int64_t n_cap = 0;
   // R_A < P (RDM_GCN_PANELS, §III-E): column-layout tensors are tiles of the
   // P/R_A x R_A grid, SpMMs broadcast inside column groups, redistributions
@@ -317,6 +318,10 @@ void sync_graph(rdm_gcn* g) {
   if (!g->saint || g->gver == g->saint->version) return;
   if (g->saint->iteration < 0) throw Error(RDM_ERR_STATE, "GraphSAINT: call rdm_saint_sample first");
   rdm_ctx* ctx = g->ctx;
+  // switch to the latest subgraph buffer once its build has finished
+  g->graph = &g->saint->graph();
+  g->sbuf = g->saint->cur;
+  RDM_CUDA(cudaStreamWaitEvent(ctx->stream, g->saint->ev_done[g->sbuf], 0));
   const int64_t n = gn(g);
   for (int s = 0; s < ctx->nlocal(); ++s)
     for (auto& kv : g->bufs[s])
@@ -731,8 +736,14 @@ void do_forward(void* a_) {
   std::vector<double*> parts(nl);
   for (int i = 0; i < nl; ++i) parts[i] = g->scal[i] + 1;
   allreduce_d(ctx, parts.data(), 1);
-  Phase ph(ctx, RDM_PH_LOSS);
-  finish_loss(ctx, g->scal[0] + 1, g->scal[0] + 0, a->loss);
+  {
+    Phase ph(ctx, RDM_PH_LOSS);
+    finish_loss(ctx, g->scal[0] + 1, g->scal[0] + 0, a->loss);
+  }
+  if (g->saint && g->saint->ev_free[g->sbuf]) {   // forward-only use also releases the buffer
+    RDM_CUDA(cudaEventRecord(g->saint->ev_free[g->sbuf], ctx->stream));
+    g->saint->freed[g->sbuf] = true;
+  }
 }
 
 void do_backward(void* a_) {
@@ -750,6 +761,10 @@ void do_backward(void* a_) {
     RDM_CUDA(cudaEventRecord(g->ev_join, g->side));
     RDM_CUDA(cudaStreamWaitEvent(ctx->stream, g->ev_join, 0));
     g->side_pending = false;
+  }
+  if (g->saint && g->saint->ev_free[g->sbuf]) {   // the sampler may rebuild this buffer now
+    RDM_CUDA(cudaEventRecord(g->saint->ev_free[g->sbuf], ctx->stream));
+    g->saint->freed[g->sbuf] = true;
   }
   const int nl = ctx->nlocal();
   for (int l = 1; l <= g->L; ++l) {
@@ -920,7 +935,7 @@ void do_saint_input(void* a_) {
   Phase ph(ctx, RDM_PH_SAMPLE);
   const int P = ctx->world;
   const int64_t n = gn(g), f0 = g->f[0];
-  const int32_t* nodes = g->saint->nodes->as<int32_t>();
+  const int32_t* nodes = g->saint->nodes_b[g->sbuf]->as<int32_t>();
   for (int i = 0; i < ctx->nlocal(); ++i) {
     const int p = ctx->local[i];
     const Range r = row_range(n, P, p);
@@ -996,7 +1011,7 @@ rdm_status rdm_saint_gcn_create(rdm_saint* s, int L, const int64_t* f, const rdm
   }
   auto* g = new rdm_gcn();
   g->ctx = ctx;
-  g->graph = &s->graph;
+  g->graph = &s->graph();
   g->saint = s;
   g->n_cap = s->n_cap;
   g->L = L;

@@ -186,10 +186,22 @@ struct rdm_saint {
   int walk_len = 0;
   uint64_t seed = 0;
   int64_t n_cap = 0;
-  rdm::Graph graph;       // current subgraph (symmetric: A only)
+  // Double-buffered subgraphs: rdm_saint_sample builds the next subgraph on the
+  // sampler's own stream into the buffer the previous-but-one subgraph used
+  // (after the executor released it, ev_free), while the compute stream still
+  // trains on the current one; the executor waits for ev_done of the buffer it
+  // switches to.
+  rdm::Graph bufs[2];     // subgraphs (symmetric: A only)
+  std::unique_ptr<rdm::DevBuf> nodes_b[2];   // sorted node list of each buffer
+  int cur = 0;            // buffer of the latest sample
+  cudaStream_t sst = nullptr;
+  cudaEvent_t ev_done[2] = {nullptr, nullptr}, ev_free[2] = {nullptr, nullptr};
+  bool freed[2] = {false, false};
+  rdm::Graph& graph() { return bufs[cur]; }
+  const rdm::Graph& graph() const { return bufs[cur]; }
   int64_t version = 0;    // bumped by every rdm_saint_sample
   int64_t iteration = -1;
-  std::unique_ptr<rdm::DevBuf> visits, flag, map, nodes, deg, seg, rps, scal, tmp, mask_s;
+  std::unique_ptr<rdm::DevBuf> visits, flag, map, deg, seg, rps, scal, tmp, mask_s;
   std::unique_ptr<rdm::DevBuf> core_tmp, core_rank, core_seg, core_cnt, core_bucket, tmp2;
 };
 

@@ -475,6 +475,25 @@ void build_core_sub(rdm_saint* s, Csr& S, int64_t kmax, const unsigned long long
 
 void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
   rdm_ctx* ctx = s->ctx;
+  // the whole build runs on the sampler's stream (host round trips wait for
+  // it only), into the buffer not in use by the subgraph being trained
+  if (!s->sst) {
+    RDM_CUDA(cudaStreamCreateWithFlags(&s->sst, cudaStreamNonBlocking));
+    for (int b = 0; b < 2; ++b) {
+      RDM_CUDA(cudaEventCreateWithFlags(&s->ev_done[b], cudaEventDisableTiming));
+      RDM_CUDA(cudaEventCreateWithFlags(&s->ev_free[b], cudaEventDisableTiming));
+    }
+  }
+  const int b = s->iteration < 0 ? 0 : (s->cur ^ 1);
+  struct OnStream {
+    rdm_ctx* c; cudaStream_t m;
+    ~OnStream() { c->stream = m; }
+  } on{ctx, ctx->stream};
+  // the previous sample (same workspaces) was issued on the sampler stream
+  // already; the buffer must have been released by the executor
+  if (s->freed[b]) RDM_CUDA(cudaStreamWaitEvent(s->sst, s->ev_free[b], 0));
+  else RDM_CUDA(cudaStreamSynchronize(ctx->stream));   // never trained on: nothing to wait for but the setup
+  ctx->stream = s->sst;
   Phase ph(ctx, RDM_PH_SAMPLE);
   const Csr& A = ctx->graph.A;
   const int64_t N = A.n, cap = s->n_cap;
@@ -485,7 +504,7 @@ void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
   int32_t* visits = reinterpret_cast<int32_t*>(ensure_ws(s->visits, nv * sizeof(int32_t)));
   int32_t* flag = reinterpret_cast<int32_t*>(ensure_ws(s->flag, N * sizeof(int32_t)));
   int32_t* map = reinterpret_cast<int32_t*>(ensure_ws(s->map, N * sizeof(int32_t)));
-  int32_t* nodes = reinterpret_cast<int32_t*>(ensure_ws(s->nodes, cap * sizeof(int32_t)));
+  int32_t* nodes = reinterpret_cast<int32_t*>(ensure_ws(s->nodes_b[b], cap * sizeof(int32_t)));
   unsigned long long* deg = reinterpret_cast<unsigned long long*>(ensure_ws(s->deg, (cap + 1) * 8));
   // segment tables: nseg[cap+1] | segoff[cap+1] | seg_row[seg_cap] (int32); cnt | pos (int64)
   int32_t* nseg = reinterpret_cast<int32_t*>(ensure_ws(s->seg, (2 * (cap + 1) + seg_cap) * 4 + 16));
@@ -523,7 +542,7 @@ void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
   const int64_t n = (int64_t)hs[0], nnz = (int64_t)hs[1];
   if (n > cap) throw Error(RDM_ERR_STATE, "saint: subgraph larger than its capacity");
 
-  Graph& G = s->graph;
+  Graph& G = s->bufs[b];
   Csr& S = G.A;
   S.core.K = 0;
   S.core.nnz = 0;
@@ -547,6 +566,9 @@ void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
   G.n = n;
   G.nnz = nnz;
   G.symmetric = true;
+  RDM_CUDA(cudaEventRecord(s->ev_done[b], s->sst));
+  s->freed[b] = false;
+  s->cur = b;
   s->iteration = it;
   s->version++;
   *n_out = n;
@@ -606,6 +628,14 @@ rdm_status rdm_saint_destroy(rdm_saint* s) {
   if (!s) return RDM_ERR_ARG;
   cudaSetDevice(s->ctx->device);
   cudaStreamSynchronize(s->ctx->stream);
+  if (s->sst) {
+    cudaStreamSynchronize(s->sst);
+    cudaStreamDestroy(s->sst);
+    for (int b = 0; b < 2; ++b) {
+      cudaEventDestroy(s->ev_done[b]);
+      cudaEventDestroy(s->ev_free[b]);
+    }
+  }
   delete s;
   return RDM_OK;
 }
@@ -635,12 +665,20 @@ rdm_status rdm_saint_sample(rdm_saint* s, int64_t iteration, int64_t* n_sub, int
   return st;
 }
 
+rdm_status rdm_saint_wait(rdm_saint* s) {
+  if (!s) return RDM_ERR_ARG;
+  if (s->sst && s->iteration >= 0 && cudaStreamWaitEvent(s->ctx->stream, s->ev_done[s->cur], 0) != cudaSuccess)
+    return RDM_ERR_CUDA;
+  return RDM_OK;
+}
+
 rdm_status rdm_saint_subgraph(const rdm_saint* s, const int32_t** nodes, const int64_t** rowptr,
                               const int32_t** col, const float** val, int64_t* n, int64_t* nnz) {
   if (!s) return RDM_ERR_ARG;
   if (s->iteration < 0) return RDM_ERR_STATE;
-  const Csr& S = s->graph.A;
-  if (nodes) *nodes = s->nodes->as<int32_t>();
+  if (s->sst) cudaStreamSynchronize(s->sst);   // the build may still be finishing on the sampler stream
+  const Csr& S = s->graph().A;
+  if (nodes) *nodes = s->nodes_b[s->cur]->as<int32_t>();
   if (rowptr) *rowptr = S.rowptr->as<int64_t>();
   if (col) *col = S.col->as<int32_t>();
   if (val) *val = S.val->as<float>();
