@@ -111,6 +111,19 @@ __device__ __forceinline__ void tmem_st32u(uint32_t addr, const uint32_t (&v)[32
       : "memory");
 }
 
+// explicit shared-memory loads (the aligned dynamic-smem pointer is generic to
+// the compiler, which otherwise emits generic LD for the expander's hot loop)
+__device__ __forceinline__ uint4 lds128(uint32_t addr) {
+  uint4 v;
+  asm volatile("ld.shared.v4.u32 {%0, %1, %2, %3}, [%4];" : "=r"(v.x), "=r"(v.y), "=r"(v.z), "=r"(v.w) : "r"(addr));
+  return v;
+}
+__device__ __forceinline__ uint2 lds64(uint32_t addr) {
+  uint2 v;
+  asm volatile("ld.shared.v2.u32 {%0, %1}, [%2];" : "=r"(v.x), "=r"(v.y) : "r"(addr) : "memory");
+  return v;
+}
+
 // Two bits → two bf16 (0 or 1.0 = 0x3F80) packed in one 32-bit word.
 __device__ __forceinline__ uint32_t bits2_bf16(uint32_t b) {
   return ((b & 1u) * 0x3F80u) | (((b >> 1) & 1u) * 0x3F800000u);
@@ -153,6 +166,7 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__
   uint64_t* tempty = tfull + 2;  // [2]
   uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
   uint4* lut = (uint4*)(smem + S * sh.stage_bytes + 1024);   // byte → 8 bf16 (0 / 1)
+  const uint32_t lut_s = smem_u32(lut);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int total = sh.n_items * sh.tiles_n;
   for (int i = threadIdx.x; i < 256; i += blockDim.x)
@@ -306,11 +320,11 @@ hub_tile_kernel(const __grid_constant__ CUtensorMap tmB, const __grid_constant__
         }
 #pragma unroll
         for (int h = 0; h < HS; ++h) {
-          const uint2 b = reinterpret_cast<const uint2*>(bits_st(s) + h * 1024)[r];
+          const uint2 b = lds64(smem_u32(bits_st(s) + h * 1024) + r * 8);
           uint32_t v[32];
 #pragma unroll
           for (int i = 0; i < 8; ++i) {
-            const uint4 e = lut[((i < 4 ? b.x : b.y) >> (8 * (i & 3))) & 0xFFu];
+            const uint4 e = lds128(lut_s + (((i < 4 ? b.x : b.y) >> (8 * (i & 3))) & 0xFFu) * 16);
             v[4 * i] = e.x; v[4 * i + 1] = e.y; v[4 * i + 2] = e.z; v[4 * i + 3] = e.w;
           }
           tmem_st32u(tmem_base + lane_off + kAcol + a * 32 * HS + h * 32, v);
