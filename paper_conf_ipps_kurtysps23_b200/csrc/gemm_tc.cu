@@ -68,7 +68,6 @@ struct TcShape {
 // K, wide outputs) — 8 warps cost one smem stage of transpose buffers.
 template <int BN, int EW>
 struct Cfg {
-  static constexpr int kEpiWarps = EW;
   static constexpr int kThreads = 256 + 32 * EW;
   static constexpr int kAccCols = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
   static constexpr bool kTmemA = BN <= 128;

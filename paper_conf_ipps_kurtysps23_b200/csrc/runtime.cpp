@@ -171,7 +171,7 @@ void redistribute(rdm_ctx* ctx, rdm_layout from, const float* const* src, float*
   const int P = ctx->world;
   const int64_t ld_row = roundup4(f);
   if (P == 1) {
-    if (src[0] != dst[0] && n * ld_row)
+    if (src[0] != dst[0] && n * ld_row != 0)
       RDM_CUDA(cudaMemcpyAsync(dst[0], src[0], n * ld_row * sizeof(float), cudaMemcpyDeviceToDevice,
                                ctx->stream));
     ctx->counters.a2a_calls++;

@@ -151,7 +151,7 @@ __device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
     // U nnz per group are gathered before any of them is consumed (U·V
     // independent 128-bit loads in flight per lane); an nnz past the row's end
     // loads nothing and contributes 0·0.
-    if (U == 1) {
+    if constexpr (U == 1) {
       // one nnz per group at a time, skipped past the row's end
 #pragma unroll
       for (int t = 0; t < G; ++t) {
@@ -175,8 +175,7 @@ __device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
           }
         }
       }
-      continue;
-    }
+    } else {
 #pragma unroll
     for (int t0 = 0; t0 < G; t0 += U) {
       if (t0 * NG >= cnt) break;   // warp-uniform: the rest of the batch is past the row's end
@@ -201,6 +200,7 @@ __device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
           acc[v].z = fmaf(vv[u], x[u][v].z, acc[v].z);
           acc[v].w = fmaf(vv[u], x[u][v].w, acc[v].w);
         }
+    }
     }
   }
 #pragma unroll
@@ -328,7 +328,7 @@ __device__ __forceinline__ void warp_nnz_range_bf(const int32_t* __restrict__ co
 #pragma unroll
         for (int v = 0; v < V; ++v) {
           const uint32_t w4[4] = {x[u][v].x, x[u][v].y, x[u][v].z, x[u][v].w};
-          if (FACT) {
+          if constexpr (FACT) {
 #pragma unroll
             for (int h = 0; h < 2; ++h) {
               acc_bf16_lo(acc[v][h].x, w4[2 * h]);
@@ -336,15 +336,15 @@ __device__ __forceinline__ void warp_nnz_range_bf(const int32_t* __restrict__ co
               acc_bf16_lo(acc[v][h].z, w4[2 * h + 1]);
               acc_bf16_hi(acc[v][h].w, w4[2 * h + 1]);
             }
-            continue;
-          }
+          } else {
 #pragma unroll
-          for (int h = 0; h < 2; ++h) {
-            float4& A = acc[v][h];
-            A.x = fmaf(vv[u], __uint_as_float(w4[2 * h] << 16), A.x);
-            A.y = fmaf(vv[u], __uint_as_float(w4[2 * h] & 0xFFFF0000u), A.y);
-            A.z = fmaf(vv[u], __uint_as_float(w4[2 * h + 1] << 16), A.z);
-            A.w = fmaf(vv[u], __uint_as_float(w4[2 * h + 1] & 0xFFFF0000u), A.w);
+            for (int h = 0; h < 2; ++h) {
+              float4& A = acc[v][h];
+              A.x = fmaf(vv[u], __uint_as_float(w4[2 * h] << 16), A.x);
+              A.y = fmaf(vv[u], __uint_as_float(w4[2 * h] & 0xFFFF0000u), A.y);
+              A.z = fmaf(vv[u], __uint_as_float(w4[2 * h + 1] << 16), A.z);
+              A.w = fmaf(vv[u], __uint_as_float(w4[2 * h + 1] & 0xFFFF0000u), A.w);
+            }
           }
         }
     }
