@@ -44,8 +44,15 @@ for P in (2, 4, 8):
                 m.forward(Ws, loss); m.backward(Ws, dW)
             ph = {k: v / 3 for k, v in ctx.phase_times()[0].items()}
             ctx.set_timing(False)
+            ctx.reset_counters()
+            m.forward(Ws, loss); m.backward(Ws, dW); ctx.sync()
+            c = ctx.counters()
+            info = m.info()
             r = {"P": P, "cfg": cfg, "transport": tr, "ms": round(ms_ep, 3), "loss": float(loss.item()),
-                 "phases": {k: round(v, 3) for k, v in ph.items() if v > 0}}
+                 "phases": {k: round(v, 3) for k, v in ph.items() if v > 0},
+                 "a2a_elems_per_epoch": c["a2a_elems_payload"], "model_comm_units": info["model_comm_units"],
+                 "a2a_elems_over_NxUnits": c["a2a_elems_payload"] / (wl.n * max(1, info["model_comm_units"])),
+                 "per_rank_elems": c["a2a_elems_payload"] / P}
             print(json.dumps(r), flush=True)
             res.append(r)
             m.close(); ctx.close()
