@@ -199,7 +199,7 @@ int rdm_get_transport(const rdm_ctx* ctx);
  *   RDM_PREC_FAST: every rdm_spmm rounds its input column slice to bf16
  *     (round-to-nearest-even) once per call and gathers the bf16 rows
  *     (half the L2/HBM gather bytes), accumulating in fp32; the binary hub
- *     tiles multiply one bf16 piece of s⊙X instead of three; every rdm_gemm
+ *     tiles multiply one bf16 piece of s⊙X (fp32: two column-scaled fp16 or three bf16 pieces); every rdm_gemm
  *     (NN / NT / TN) issues one tf32 MMA per k step instead of 3xTF32 (the
  *     tensor core reads fp32 operands as tf32).  Outputs, gradients and the
  *     loss stay fp32 in the caller's buffers; redistribution stays bit-exact.
