@@ -397,45 +397,70 @@ __global__ void tile_panels_kernel(const float* __restrict__ X, int64_t ldx, con
                                    __nv_bfloat16* __restrict__ p2, int np) {
   __shared__ float t[64][33];
   const int64_t k0 = (int64_t)blockIdx.x * 64, n0 = (int64_t)blockIdx.y * 32;
-  for (int i = threadIdx.y; i < 64; i += 8) {
-    const int64_t k = k0 + i, n = n0 + threadIdx.x;
-    t[i][threadIdx.x] = (n < w) ? __ldg(scale + k) * __ldg(X + (int64_t)__ldg(hub_ids + k) * ldx + n) : 0.f;
+  {
+    // the 8 hub ids first, then 8 independent row gathers per thread
+    const int64_t n = n0 + threadIdx.x;
+    int32_t id[8];
+    float sc[8], x[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      id[u] = __ldg(hub_ids + k0 + threadIdx.y + 8 * u);
+      sc[u] = __ldg(scale + k0 + threadIdx.y + 8 * u);
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) x[u] = (n < w) ? __ldg(X + (int64_t)id[u] * ldx + n) : 0.f;
+#pragma unroll
+    for (int u = 0; u < 8; ++u) t[threadIdx.y + 8 * u][threadIdx.x] = sc[u] * x[u];
   }
   __syncthreads();
   for (int i = threadIdx.y; i < 32; i += 8) {
     const int64_t n = n0 + i;
     if (n >= w) break;
-#pragma unroll
-    for (int hk = 0; hk < 2; ++hk) {
-      const int kk = hk * 32 + threadIdx.x;
-      const float x = t[kk][i];
-      const __nv_bfloat16 h = __float2bfloat16_rn(x);
-      const float r1 = x - __bfloat162float(h);
-      const __nv_bfloat16 m = __float2bfloat16_rn(r1);
-      const __nv_bfloat16 l = __float2bfloat16_rn(r1 - __bfloat162float(m));
-      const int64_t o = n * K2 + k0 + kk;
-      p0[o] = h;
-      if (np == 3) {
-        p1[o] = m;
-        p2[o] = l;
-      }
+    // a pair of consecutive k per thread: 4-byte stores, 128 B per warp and piece
+    const int kk = 2 * threadIdx.x;
+    const float x0 = t[kk][i], x1 = t[kk + 1][i];
+    const __nv_bfloat162 h = __floats2bfloat162_rn(x0, x1);
+    const float r0 = x0 - __low2float(h), r1 = x1 - __high2float(h);
+    const __nv_bfloat162 m = __floats2bfloat162_rn(r0, r1);
+    const __nv_bfloat162 l = __floats2bfloat162_rn(r0 - __low2float(m), r1 - __high2float(m));
+    const int64_t o = n * K2 + k0 + kk;
+    *reinterpret_cast<__nv_bfloat162*>(p0 + o) = h;
+    if (np == 3) {
+      *reinterpret_cast<__nv_bfloat162*>(p1 + o) = m;
+      *reinterpret_cast<__nv_bfloat162*>(p2 + o) = l;
     }
   }
 }
 
 // Column maxima of |s_k · X[hub_k][n]| over the K2 hub slots (bit patterns of
 // non-negative floats order like unsigned ints: atomicMax is exact and
-// order-independent).  Block: 32 columns x 8 k-lanes, 128 k per lane.
+// order-independent).  Block: 32 columns x 8 k-lanes, 32 k per lane (short
+// dependent gather chains: the hub id, then the row).
 __global__ void tile_colmax_kernel(const float* __restrict__ X, int64_t ldx, const int32_t* __restrict__ hub_ids,
                                    const float* __restrict__ scale, int64_t K2, int64_t w,
                                    unsigned int* __restrict__ colmax) {
   __shared__ float red[8][33];
   const int64_t n = (int64_t)blockIdx.y * 32 + threadIdx.x;
-  const int64_t k0 = (int64_t)blockIdx.x * 1024;
+  const int64_t k0 = (int64_t)blockIdx.x * 256;
   float m = 0.f;
-  if (n < w)
-    for (int64_t k = k0 + threadIdx.y; k < min(K2, k0 + 1024); k += 8)
-      m = fmaxf(m, fabsf(__ldg(scale + k) * __ldg(X + (int64_t)__ldg(hub_ids + k) * ldx + n)));
+  if (n < w) {
+    // K2 is a multiple of 128 and blocks start at multiples of 256: a block's
+    // k range is full or half full; batches of 8 independent gathers per thread
+    const int64_t k1 = min(K2, k0 + 256);
+    for (int64_t kb = k0 + threadIdx.y; kb < k1; kb += 64) {
+      int32_t id[8];
+      float sc[8], x[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        id[u] = __ldg(hub_ids + kb + 8 * u);
+        sc[u] = __ldg(scale + kb + 8 * u);
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u) x[u] = __ldg(X + (int64_t)id[u] * ldx + n);
+#pragma unroll
+      for (int u = 0; u < 8; ++u) m = fmaxf(m, fabsf(sc[u] * x[u]));
+    }
+  }
   red[threadIdx.y][threadIdx.x] = m;
   __syncthreads();
   if (threadIdx.y == 0 && n < w) {
@@ -462,24 +487,32 @@ __global__ void tile_panels_f16_kernel(const float* __restrict__ X, int64_t ldx,
     inv[threadIdx.x] = ldexpf(1.f, -e);
     if (blockIdx.x == 0 && n < w) colscale[n] = ldexpf(1.f, e);
   }
-  for (int i = threadIdx.y; i < 64; i += 8) {
-    const int64_t k = k0 + i, n = n0 + threadIdx.x;
-    t[i][threadIdx.x] = (n < w) ? __ldg(scale + k) * __ldg(X + (int64_t)__ldg(hub_ids + k) * ldx + n) : 0.f;
+  {
+    // the 8 hub ids first, then 8 independent row gathers per thread
+    const int64_t n = n0 + threadIdx.x;
+    int32_t id[8];
+    float sc[8], x[8];
+#pragma unroll
+    for (int u = 0; u < 8; ++u) {
+      id[u] = __ldg(hub_ids + k0 + threadIdx.y + 8 * u);
+      sc[u] = __ldg(scale + k0 + threadIdx.y + 8 * u);
+    }
+#pragma unroll
+    for (int u = 0; u < 8; ++u) x[u] = (n < w) ? __ldg(X + (int64_t)id[u] * ldx + n) : 0.f;
+#pragma unroll
+    for (int u = 0; u < 8; ++u) t[threadIdx.y + 8 * u][threadIdx.x] = sc[u] * x[u];
   }
   __syncthreads();
   for (int i = threadIdx.y; i < 32; i += 8) {
     const int64_t n = n0 + i;
     if (n >= w) break;
-#pragma unroll
-    for (int hk = 0; hk < 2; ++hk) {
-      const int kk = hk * 32 + threadIdx.x;
-      const float y = t[kk][i] * inv[i];
-      const __half h = __float2half_rn(y);
-      const __half l = __float2half_rn(y - __half2float(h));
-      const int64_t o = n * K2 + k0 + kk;
-      p0[o] = h;
-      p1[o] = l;
-    }
+    const int kk = 2 * threadIdx.x;   // a pair of consecutive k per thread (4-byte stores)
+    const float y0 = t[kk][i] * inv[i], y1 = t[kk + 1][i] * inv[i];
+    const __half2 h = __floats2half2_rn(y0, y1);
+    const __half2 l = __floats2half2_rn(y0 - __low2float(h), y1 - __high2float(h));
+    const int64_t o = n * K2 + k0 + kk;
+    *reinterpret_cast<__half2*>(p0 + o) = h;
+    *reinterpret_cast<__half2*>(p1 + o) = l;
   }
 }
 
@@ -555,7 +588,7 @@ void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx,
     unsigned int* cmax = reinterpret_cast<unsigned int*>(cs + w4);
     RDM_CUDA(cudaMemsetAsync(cmax, 0, w * sizeof(unsigned int), ctx->stream));
     RDM_CUDA(cudaMemsetAsync(cs, 0, w4 * sizeof(float), ctx->stream));
-    dim3 mg((unsigned)ceil_div(K2, 1024), (unsigned)ceil_div(w, 32));
+    dim3 mg((unsigned)ceil_div(K2, 256), (unsigned)ceil_div(w, 32));
     tile_colmax_kernel<<<mg, dim3(32, 8), 0, ctx->stream>>>(X, ldx, c.hub_ids->as<int32_t>(), c.scale->as<float>(),
                                                            K2, w, cmax);
     RDM_LAUNCHED(ctx);
