@@ -77,10 +77,12 @@ class ClockSampler:
         self.lines = []
 
     def start(self):
+        if os.environ.get("RDM_BENCH_NO_CLOCKS"):   # diagnosis only: no clock record
+            return
         try:
             self.proc = subprocess.Popen(
                 ["nvidia-smi", f"--query-gpu={self.Q}", "--format=csv,noheader,nounits",
-                 "-lms", "100", "-i", str(self.device)],
+                 "-lms", "200", "-i", str(self.device)],
                 stdout=subprocess.PIPE, stderr=subprocess.DEVNULL, text=True)
             self.t = threading.Thread(target=self._read, daemon=True)
             self.t.start()
@@ -266,6 +268,11 @@ def saint_main(a, world, rank, local_rank):
         ctx.adam_step(Wd, dW, mo, ve, it[0], lr=0.01)
         cur[0] = sam.sample(it[0])
 
+    # the clock sampler starts during the warm-up (no idle gap before the timed
+    # steps: after an idle pause the first host-synchronised sampler steps ran
+    # several times slower)
+    clk = ClockSampler(local_rank)
+    clk.start()
     for _ in range(max(3, a.warmup)):
         step()
     ctx.sync()
@@ -273,9 +280,6 @@ def saint_main(a, world, rank, local_rank):
     ctx.reset_counters()
     ctx.reset_phase_times()
     ctx.set_timing(True)
-    clk = ClockSampler(local_rank)
-    clk.start()
-    time.sleep(0.3)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize(dev)

@@ -139,7 +139,15 @@ __global__ void count_kernel(const int64_t* __restrict__ rowptr, const int32_t* 
        sg += ((int64_t)gridDim.x * blockDim.x) >> 5) {
     const Seg q = seg_of(sg, seg_row, segoff, rowptr, nodes);
     int c = 0;
-    for (int64_t k = q.b + lane; k < q.end; k += 32) c += flag[__ldg(col + k)] ? 1 : 0;
+    // 4 chunks of 32 entries per step: the column loads, then the flag
+    // lookups, all independent (memory-level parallelism)
+    for (int64_t k = q.b + lane; k < q.end; k += 128) {
+      int32_t cc[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) cc[u] = (k + 32 * u < q.end) ? __ldg(col + k + 32 * u) : -1;
+#pragma unroll
+      for (int u = 0; u < 4; ++u) c += (cc[u] >= 0 && flag[cc[u]]) ? 1 : 0;
+    }
 #pragma unroll
     for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
     if (lane == 0) {
@@ -177,18 +185,30 @@ __global__ void fill_kernel(const int64_t* __restrict__ rowptr, const int32_t* _
     const Seg q = seg_of(sg, seg_row, segoff, rowptr, nodes);
     int64_t at0 = pos[sg];
     const double di = (double)deg[q.i];
-    for (int64_t k0 = q.b; k0 < q.end; k0 += 32) {
-      const int64_t k = k0 + lane;
-      const int32_t u = k < q.end ? __ldg(col + k) : 0;
-      const bool keep = k < q.end && flag[u];
-      const unsigned m = __ballot_sync(0xffffffffu, keep);
-      if (keep) {
-        const int64_t at = at0 + __popc(m & ((1u << lane) - 1u));
-        const int32_t j = map[u];
-        col_s[at] = j;
-        val_s[at] = (float)(1.0 / sqrt(di * (double)deg[j]));
+    for (int64_t kb = q.b; kb < q.end; kb += 128) {
+      // 4 chunks of 32 entries: loads batched, then compacted chunk by chunk
+      // in the original order
+      int32_t uu[4];
+      bool kp[4];
+#pragma unroll
+      for (int c4 = 0; c4 < 4; ++c4) {
+        const int64_t k = kb + 32 * c4 + lane;
+        uu[c4] = k < q.end ? __ldg(col + k) : 0;
       }
-      at0 += __popc(m);
+#pragma unroll
+      for (int c4 = 0; c4 < 4; ++c4) kp[c4] = (kb + 32 * c4 + lane < q.end) && flag[uu[c4]];
+#pragma unroll
+      for (int c4 = 0; c4 < 4; ++c4) {
+        if (kb + 32 * c4 >= q.end) break;
+        const unsigned m = __ballot_sync(0xffffffffu, kp[c4]);
+        if (kp[c4]) {
+          const int64_t at = at0 + __popc(m & ((1u << lane) - 1u));
+          const int32_t j = map[uu[c4]];
+          col_s[at] = j;
+          val_s[at] = (float)(1.0 / sqrt(di * (double)deg[j]));
+        }
+        at0 += __popc(m);
+      }
     }
   }
 }
@@ -478,7 +498,12 @@ void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
   // the whole build runs on the sampler's stream (host round trips wait for
   // it only), into the buffer not in use by the subgraph being trained
   if (!s->sst) {
-    RDM_CUDA(cudaStreamCreateWithFlags(&s->sst, cudaStreamNonBlocking));
+    // high priority: the host waits on this stream several times per subgraph,
+    // so its short kernels go first whenever SMs free up between the
+    // training kernels of the previous subgraph
+    int lo = 0, hi = 0;
+    RDM_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+    RDM_CUDA(cudaStreamCreateWithPriority(&s->sst, cudaStreamNonBlocking, hi));
     for (int b = 0; b < 2; ++b) {
       RDM_CUDA(cudaEventCreateWithFlags(&s->ev_done[b], cudaEventDisableTiming));
       RDM_CUDA(cudaEventCreateWithFlags(&s->ev_free[b], cudaEventDisableTiming));
