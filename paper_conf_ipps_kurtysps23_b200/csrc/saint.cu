@@ -267,18 +267,35 @@ __global__ void hist_kernel(const int64_t* __restrict__ rp, const int32_t* __res
 }
 
 // CTA per hub (rank r < K): its dense row built in shared memory, then
-// written whole (coalesced; zeros included, so no separate memset).
+// written whole (coalesced; zeros included, so no separate memset).  The
+// col → rank gathers are batched kB per thread (independent loads in flight:
+// hub rows of the dense subgraphs hold thousands of entries, and one
+// dependent gather pair per iteration left the kernel latency-bound).
 __global__ void core_rows_kernel(const int64_t* __restrict__ rp, const int32_t* __restrict__ col,
                                  const float* __restrict__ val, const int32_t* __restrict__ rank,
                                  const int32_t* __restrict__ order, int64_t K, float* __restrict__ dense) {
+  constexpr int kB = 8;
   extern __shared__ float row[];
   for (int64_t r = blockIdx.x; r < K; r += gridDim.x) {
     for (int64_t c = threadIdx.x; c < K; c += blockDim.x) row[c] = 0.f;
     __syncthreads();
     const int32_t i = order[r];
-    for (int64_t k = rp[i] + threadIdx.x; k < rp[i + 1]; k += blockDim.x) {
-      const int32_t rj = rank[__ldg(col + k)];
-      if (rj < K) row[rj] = __ldg(val + k);   // CSR entries are distinct
+    const int64_t e = rp[i + 1];
+    for (int64_t k0 = rp[i] + threadIdx.x; k0 < e; k0 += (int64_t)kB * blockDim.x) {
+      int32_t cj[kB];
+      float vj[kB];
+#pragma unroll
+      for (int u = 0; u < kB; ++u) {
+        const int64_t k = k0 + (int64_t)u * blockDim.x;
+        cj[u] = k < e ? __ldg(col + k) : -1;
+        vj[u] = k < e ? __ldg(val + k) : 0.f;
+      }
+      int32_t rj[kB];
+#pragma unroll
+      for (int u = 0; u < kB; ++u) rj[u] = cj[u] >= 0 ? __ldg(rank + cj[u]) : INT32_MAX;
+#pragma unroll
+      for (int u = 0; u < kB; ++u)
+        if (rj[u] < K) row[rj[u]] = vj[u];   // CSR entries are distinct
     }
     __syncthreads();
     float4* out = reinterpret_cast<float4*>(dense + r * K);
