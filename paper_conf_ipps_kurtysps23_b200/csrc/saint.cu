@@ -253,14 +253,25 @@ __global__ void hist_kernel(const int64_t* __restrict__ rp, const int32_t* __res
     if (i & 7) continue;                       // warp-uniform
     const Seg q = seg_of(sg, seg_row, segoff, rp, nullptr);
     const int32_t ri = rank[i];
-    for (int64_t k0 = q.b; k0 < q.end; k0 += 32) {
-      const int64_t k = k0 + lane;
-      int bk = -1;
-      if (k < q.end) {
-        const int32_t mx = max(ri, rank[__ldg(col + k)]);
-        if (mx < kmax) bk = mx >> 7;
+    for (int64_t k0 = q.b; k0 < q.end; k0 += 128) {
+      // 4 chunks of 32 entries: loads and rank lookups batched
+      int32_t cc[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        const int64_t k = k0 + 32 * u + lane;
+        cc[u] = k < q.end ? __ldg(col + k) : -1;
       }
-      bucket_add(sb, bk, lane);
+      int bk[4];
+#pragma unroll
+      for (int u = 0; u < 4; ++u) {
+        bk[u] = -1;
+        if (cc[u] >= 0) {
+          const int32_t mx = max(ri, rank[cc[u]]);
+          if (mx < kmax) bk[u] = mx >> 7;
+        }
+      }
+#pragma unroll
+      for (int u = 0; u < 4; ++u) bucket_add(sb, bk[u], lane);
     }
   }
   bucket_flush(sb, bucket);
@@ -319,7 +330,13 @@ __global__ void resid_count_kernel(const int64_t* __restrict__ rp, const int32_t
     if (rank[q.i] >= K) {
       c = (int)(q.end - q.b);
     } else {
-      for (int64_t k = q.b + lane; k < q.end; k += 32) c += rank[__ldg(col + k)] >= K ? 1 : 0;
+      for (int64_t k = q.b + lane; k < q.end; k += 128) {
+        int32_t cc[4];
+#pragma unroll
+        for (int u = 0; u < 4; ++u) cc[u] = (k + 32 * u < q.end) ? __ldg(col + k + 32 * u) : -1;
+#pragma unroll
+        for (int u = 0; u < 4; ++u) c += (cc[u] >= 0 && rank[cc[u]] >= K) ? 1 : 0;
+      }
 #pragma unroll
       for (int o = 16; o; o >>= 1) c += __shfl_xor_sync(0xffffffffu, c, o);
     }
@@ -339,18 +356,32 @@ __global__ void resid_kernel(const int64_t* __restrict__ rp, const int32_t* __re
     const Seg q = seg_of(sg, seg_row, segoff, rp, nullptr);
     const bool hub_i = rank[q.i] < K;
     int64_t at0 = pos[sg];
-    for (int64_t k0 = q.b; k0 < q.end; k0 += 32) {
-      const int64_t k = k0 + lane;
-      const bool in = k < q.end;
-      const int32_t c = in ? __ldg(col + k) : 0;
-      const bool keep = in && !(hub_i && rank[c] < K);
-      const unsigned m = __ballot_sync(0xffffffffu, keep);
-      if (keep) {
-        const int64_t at = at0 + __popc(m & ((1u << lane) - 1u));
-        rcol[at] = c;
-        rval[at] = __ldg(val + k);
+    for (int64_t kb = q.b; kb < q.end; kb += 128) {
+      // 4 chunks of 32 entries: column / value loads and rank lookups batched,
+      // then compacted chunk by chunk in the original order (as fill_kernel)
+      int32_t cc[4];
+      float vv[4];
+      bool kp[4];
+#pragma unroll
+      for (int c4 = 0; c4 < 4; ++c4) {
+        const int64_t k = kb + 32 * c4 + lane;
+        cc[c4] = k < q.end ? __ldg(col + k) : 0;
+        vv[c4] = k < q.end ? __ldg(val + k) : 0.f;
       }
-      at0 += __popc(m);
+#pragma unroll
+      for (int c4 = 0; c4 < 4; ++c4)
+        kp[c4] = (kb + 32 * c4 + lane < q.end) && !(hub_i && rank[cc[c4]] < K);
+#pragma unroll
+      for (int c4 = 0; c4 < 4; ++c4) {
+        if (kb + 32 * c4 >= q.end) break;
+        const unsigned m = __ballot_sync(0xffffffffu, kp[c4]);
+        if (kp[c4]) {
+          const int64_t at = at0 + __popc(m & ((1u << lane) - 1u));
+          rcol[at] = cc[c4];
+          rval[at] = vv[c4];
+        }
+        at0 += __popc(m);
+      }
     }
   }
 }
