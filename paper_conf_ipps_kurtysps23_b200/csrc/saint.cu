@@ -197,15 +197,21 @@ __global__ void fill_kernel(const int64_t* __restrict__ rowptr, const int32_t* _
       }
 #pragma unroll
       for (int c4 = 0; c4 < 4; ++c4) kp[c4] = (kb + 32 * c4 + lane < q.end) && flag[uu[c4]];
+      // map / degree gathers of all 4 chunks issued before the compaction
+      int32_t jj[4];
+      unsigned long long dj[4];
+#pragma unroll
+      for (int c4 = 0; c4 < 4; ++c4) jj[c4] = kp[c4] ? map[uu[c4]] : 0;
+#pragma unroll
+      for (int c4 = 0; c4 < 4; ++c4) dj[c4] = kp[c4] ? deg[jj[c4]] : 1ull;
 #pragma unroll
       for (int c4 = 0; c4 < 4; ++c4) {
         if (kb + 32 * c4 >= q.end) break;
         const unsigned m = __ballot_sync(0xffffffffu, kp[c4]);
         if (kp[c4]) {
           const int64_t at = at0 + __popc(m & ((1u << lane) - 1u));
-          const int32_t j = map[uu[c4]];
-          col_s[at] = j;
-          val_s[at] = (float)(1.0 / sqrt(di * (double)deg[j]));
+          col_s[at] = jj[c4];
+          val_s[at] = (float)(1.0 / sqrt(di * (double)dj[c4]));
         }
         at0 += __popc(m);
       }
@@ -502,7 +508,10 @@ void build_core_sub(rdm_saint* s, Csr& S, int64_t kmax, const unsigned long long
   float* dense = ensure_ws(c.A, (size_t)K * K * sizeof(float));
   const int smem = (int)(K * sizeof(float));
   RDM_CUDA(cudaFuncSetAttribute(core_rows_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-  core_rows_kernel<<<(unsigned)std::min<int64_t>(K, (int64_t)ctx->num_sms * 4), 256, smem, ctx->stream>>>(
+  int per_sm = 0;   // as many resident CTAs as the K-float row buffer allows
+  RDM_CUDA(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&per_sm, core_rows_kernel, 256, smem));
+  per_sm = std::max(per_sm, 1);
+  core_rows_kernel<<<(unsigned)std::min<int64_t>(K, (int64_t)ctx->num_sms * per_sm), 256, smem, ctx->stream>>>(
       rp, col, val, rank, order, K, dense);
   RDM_LAUNCHED(ctx);
   // residual CSR: count, scan, fill in the original order
