@@ -180,8 +180,31 @@ struct rdm_ctx {
 
 // GraphSAINT-RDM sampler (saint.cu): the current subgraph and the device
 // workspace that builds it.
+// Pinned host staging buffer (grows, never shrinks): D2H copies into pageable
+// memory block the host at the call, so copies meant to share one sync land here.
+struct rdm_pinned {
+  void* p = nullptr;
+  size_t bytes = 0;
+  rdm_pinned() = default;
+  rdm_pinned(const rdm_pinned&) = delete;
+  rdm_pinned& operator=(const rdm_pinned&) = delete;
+  ~rdm_pinned() { if (p) cudaFreeHost(p); }
+  template <class T> T* get(size_t count) {
+    const size_t want = count * sizeof(T);
+    if (want > bytes) {
+      if (p) cudaFreeHost(p);
+      p = nullptr;
+      bytes = 0;
+      if (cudaMallocHost(&p, want + want / 4) != cudaSuccess) throw ::rdm::Error(RDM_ERR_OOM, "pinned host buffer");
+      bytes = want + want / 4;
+    }
+    return static_cast<T*>(p);
+  }
+};
+
 struct rdm_saint {
   rdm_ctx* ctx = nullptr;
+  rdm_pinned h_scal, h_rp, h_rrp, h_bucket;   // host staging of the sampler's round trips
   int64_t roots = 0;
   int walk_len = 0;
   uint64_t seed = 0;

@@ -394,10 +394,12 @@ __global__ void resid_kernel(const int64_t* __restrict__ rp, const int32_t* __re
 
 // residual rowptr from the segment offsets; hub ids / slots
 __global__ void resid_rp_kernel(const int32_t* __restrict__ segoff, const int64_t* __restrict__ pos,
-                                int64_t n, int64_t rnnz, const int32_t* __restrict__ order,
+                                const int64_t* __restrict__ last_cnt, const int64_t* __restrict__ last_pos,
+                                int64_t n, const int32_t* __restrict__ order,
                                 const int32_t* __restrict__ rank, int64_t K, int64_t* __restrict__ rrp,
                                 int32_t* __restrict__ hub_ids, int32_t* __restrict__ hub_slot) {
   const int64_t nsegs = segoff[n];
+  const int64_t rnnz = *last_pos + *last_cnt;   // residual size: scan's last prefix + count
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i <= n;
        i += (int64_t)gridDim.x * blockDim.x) {
     rrp[i] = segoff[i] < nsegs ? pos[segoff[i]] : rnnz;
@@ -454,15 +456,16 @@ int64_t core_kmax(int64_t n, int64_t nnz) {
   return kmax >= (forced ? 128 : 1024) ? kmax : 0;
 }
 
-// Hub core of the current subgraph S (bins of S already built): ranks,
-// sampled histogram, K, dense rows, residual CSR (+ its bins).
-void build_core_sub(rdm_saint* s, Csr& S, int64_t kmax, const unsigned long long* deg) {
+// Hub core of the current subgraph S, first half (needs S.n, S.nnz and the
+// CSR of S, not its bins): ranks and the sampled histogram, whose copy into
+// the pinned hb is issued here and waited for by the caller together with
+// the rowptr of S (one host sync for both).
+void build_core_sub(rdm_saint* s, Csr& S, int64_t kmax, const unsigned long long* deg,
+                    unsigned long long* hb) {
   rdm_ctx* ctx = s->ctx;
   const int64_t n = S.n, nnz = S.nnz;
-  Core& c = S.core;
   const int64_t* rp = S.rowptr->as<int64_t>();
   const int32_t* col = S.col->as<int32_t>();
-  const float* val = S.val->as<float>();
   // degree order (stable, descending) and ranks
   int32_t* keys = reinterpret_cast<int32_t*>(ensure_ws(s->core_tmp, (size_t)4 * n * sizeof(int32_t) + 256));
   int32_t* iota = keys + n;
@@ -496,9 +499,28 @@ void build_core_sub(rdm_saint* s, Csr& S, int64_t kmax, const unsigned long long
   hist_kernel<<<grid_of(ctx, seg_cap * 32, 256), 256, 0, ctx->stream>>>(rp, col, rank, seg_row, segoff, n, kmax,
                                                                          bucket);
   RDM_LAUNCHED(ctx);
-  std::vector<unsigned long long> hb(kMaxBuckets);
-  RDM_CUDA(cudaMemcpyAsync(hb.data(), bucket, kMaxBuckets * 8, cudaMemcpyDeviceToHost, ctx->stream));
-  RDM_CUDA(cudaStreamSynchronize(ctx->stream));
+  RDM_CUDA(cudaMemcpyAsync(hb, bucket, kMaxBuckets * 8, cudaMemcpyDeviceToHost, ctx->stream));
+}
+
+// Second half, after the host sync that delivered hb (shared with the rowptr
+// of S): K, dense rows, residual CSR (+ its bins).  The workspaces are the
+// ones the first half sized (ensure_ws keeps them).
+void build_core_sub_finish(rdm_saint* s, Csr& S, int64_t kmax, const unsigned long long* hb) {
+  rdm_ctx* ctx = s->ctx;
+  const int64_t n = S.n, nnz = S.nnz;
+  Core& c = S.core;
+  const int64_t* rp = S.rowptr->as<int64_t>();
+  const int32_t* col = S.col->as<int32_t>();
+  const float* val = S.val->as<float>();
+  int32_t* keys = reinterpret_cast<int32_t*>(ensure_ws(s->core_tmp, (size_t)4 * n * sizeof(int32_t) + 256));
+  int32_t* order = keys + 3 * n;
+  int32_t* rank = reinterpret_cast<int32_t*>(ensure_ws(s->core_rank, n * sizeof(int32_t)));
+  const int64_t seg_cap = n + nnz / kSeg + 1;
+  int32_t* nseg = reinterpret_cast<int32_t*>(ensure_ws(s->core_seg, (2 * (n + 1) + seg_cap) * 4 + 16));
+  int32_t* segoff = nseg + (n + 1);
+  int32_t* seg_row = segoff + (n + 1);
+  int64_t* cnt = reinterpret_cast<int64_t*>(ensure_ws(s->core_cnt, 2 * seg_cap * sizeof(int64_t)));
+  int64_t* pos = cnt + seg_cap;
   std::vector<int64_t> b64(kMaxBuckets);
   for (int b = 0; b < kMaxBuckets; ++b) b64[b] = (int64_t)hb[b] * 8;   // 1/8 row sample
   bool forced = false;
@@ -523,28 +545,27 @@ void build_core_sub(rdm_saint* s, Csr& S, int64_t kmax, const unsigned long long
   if (!c.resid) c.resid.reset(new Csr());
   Csr& R = *c.resid;
   int64_t* rrp = reinterpret_cast<int64_t*>(ensure_ws(R.rowptr, (n + 1) * sizeof(int64_t)));
-  // exact residual size: one more small D2H (the scan's last prefix + count)
-  int64_t tail[2];
-  RDM_CUDA(cudaMemcpyAsync(tail, pos + seg_cap - 1, 8, cudaMemcpyDeviceToHost, ctx->stream));
-  RDM_CUDA(cudaMemcpyAsync(tail + 1, cnt + seg_cap - 1, 8, cudaMemcpyDeviceToHost, ctx->stream));
-  RDM_CUDA(cudaStreamSynchronize(ctx->stream));
-  const int64_t rnnz = tail[0] + tail[1];
-  int32_t* rcol = reinterpret_cast<int32_t*>(ensure_ws(R.col, std::max<int64_t>(rnnz, 1) * sizeof(int32_t)));
-  float* rval = ensure_ws(R.val, std::max<int64_t>(rnnz, 1) * sizeof(float));
+  // residual arrays sized by nnz (an upper bound: no host round trip for the
+  // exact size; resid_rp_kernel reads it from the scan's last prefix + count,
+  // and the host learns it with the residual rowptr)
+  int32_t* rcol = reinterpret_cast<int32_t*>(ensure_ws(R.col, std::max<int64_t>(nnz, 1) * sizeof(int32_t)));
+  float* rval = ensure_ws(R.val, std::max<int64_t>(nnz, 1) * sizeof(float));
   resid_kernel<<<grid_of(ctx, seg_cap * 32, 256), 256, 0, ctx->stream>>>(rp, col, val, rank, seg_row, segoff,
                                                                           n, K, pos, rcol, rval);
   RDM_LAUNCHED(ctx);
   int32_t* hub_ids = reinterpret_cast<int32_t*>(ensure_ws(c.hub_ids, K * sizeof(int32_t)));
   int32_t* hub_slot = reinterpret_cast<int32_t*>(ensure_ws(c.hub_slot, n * sizeof(int32_t)));
-  resid_rp_kernel<<<grid_of(ctx, n + 1, 256), 256, 0, ctx->stream>>>(segoff, pos, n, rnnz, order, rank, K,
+  resid_rp_kernel<<<grid_of(ctx, n + 1, 256), 256, 0, ctx->stream>>>(segoff, pos, cnt + seg_cap - 1,
+                                                                       pos + seg_cap - 1, n, order, rank, K,
                                                                        rrp, hub_ids, hub_slot);
   RDM_LAUNCHED(ctx);
-  std::vector<int64_t> rrph(n + 1);
-  RDM_CUDA(cudaMemcpyAsync(rrph.data(), rrp, (n + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, ctx->stream));
+  int64_t* rrph = s->h_rrp.get<int64_t>(n + 1);
+  RDM_CUDA(cudaMemcpyAsync(rrph, rrp, (n + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, ctx->stream));
   RDM_CUDA(cudaStreamSynchronize(ctx->stream));
+  const int64_t rnnz = rrph[n];
   R.n = n;
   R.nnz = rnnz;
-  build_bins(ctx, R, rrph.data());
+  build_bins(ctx, R, rrph);
   c.K = K;
   c.nnz = nnz - rnnz;
   c.forced = forced;
@@ -618,8 +639,8 @@ void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
   count_kernel<<<grid_of(ctx, seg_cap * 32, 256), 256, 0, ctx->stream>>>(
       A.rowptr->as<int64_t>(), A.col->as<int32_t>(), flag, nodes, seg_row, segoff, cap, cnt, deg, scal);
   RDM_LAUNCHED(ctx);
-  unsigned long long hs[2];
-  RDM_CUDA(cudaMemcpyAsync(hs, scal, sizeof(hs), cudaMemcpyDeviceToHost, ctx->stream));
+  unsigned long long* hs = s->h_scal.get<unsigned long long>(2);
+  RDM_CUDA(cudaMemcpyAsync(hs, scal, 2 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, ctx->stream));
   RDM_CUDA(cudaStreamSynchronize(ctx->stream));
   const int64_t n = (int64_t)hs[0], nnz = (int64_t)hs[1];
   if (n > cap) throw Error(RDM_ERR_STATE, "saint: subgraph larger than its capacity");
@@ -638,13 +659,19 @@ void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
       A.rowptr->as<int64_t>(), A.col->as<int32_t>(), flag, map, nodes, seg_row, segoff, cap, deg, pos,
       cs, vs);
   RDM_LAUNCHED(ctx);
-  std::vector<int64_t> rph(n + 1);
-  RDM_CUDA(cudaMemcpyAsync(rph.data(), rp, (n + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, ctx->stream));
-  RDM_CUDA(cudaStreamSynchronize(ctx->stream));
+  int64_t* rph = s->h_rp.get<int64_t>(n + 1);
+  RDM_CUDA(cudaMemcpyAsync(rph, rp, (n + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost, ctx->stream));
   S.n = n;
   S.nnz = nnz;
-  build_bins(ctx, S, rph.data());
-  if (const int64_t kmax = core_kmax(n, nnz)) build_core_sub(s, S, kmax, deg);
+  // the hub core's ranks + histogram need the CSR of S, not its bins: issued
+  // before the host waits, so that one sync brings back rowptr_s and the
+  // histogram together
+  const int64_t kmax = core_kmax(n, nnz);
+  unsigned long long* hb = s->h_bucket.get<unsigned long long>(kMaxBuckets);
+  if (kmax) build_core_sub(s, S, kmax, deg, hb);
+  RDM_CUDA(cudaStreamSynchronize(ctx->stream));
+  build_bins(ctx, S, rph);
+  if (kmax) build_core_sub_finish(s, S, kmax, hb);
   G.n = n;
   G.nnz = nnz;
   G.symmetric = true;
