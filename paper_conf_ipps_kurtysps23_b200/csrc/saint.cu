@@ -17,7 +17,8 @@
 //   cub scans        rowptr_s = prefix of d; segment output offsets
 //   fill_kernel      warp per segment: col_s = map[u] in the original row order,
 //                    val_s = (float)(1 / sqrt((double) d_i d_j))
-// then the host builds the row bins from rowptr_s (one D2H copy).
+// then the host builds the row bins from rowptr_s (one D2H copy, sharing its
+// sync with the hub-core histogram when a core is built).
 #include <cub/cub.cuh>
 
 #include <cmath>
