@@ -286,13 +286,20 @@ def saint_main(a, world, rank, local_rank):
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
     e0.record(stream)
+    # per-step marks on the compute stream (no host sync): the step-time
+    # distribution shows whether a slow run is a few slow steps or all of them
+    marks = []
     for _ in range(a.steps):
         step()
+        ev = torch.cuda.Event(enable_timing=True)
+        ev.record(stream)
+        marks.append(ev)
     sam.wait()   # the last step's subgraph build (sampler stream) inside the bracket
     e1.record(stream)
     torch.cuda.synchronize(dev)
     clocks = clk.stop()
     ms_total = e0.elapsed_time(e1)
+    step_ms = [e0.elapsed_time(marks[0])] + [marks[i - 1].elapsed_time(marks[i]) for i in range(1, len(marks))]
     cnt = ctx.counters()
     ph_ms, _ = ctx.phase_times()
     ctx.set_timing(False)
@@ -346,6 +353,8 @@ def saint_main(a, world, rank, local_rank):
                        "parallelism": f"rdm{world} per subgraph, one Adam step per subgraph (L390)",
                        "l2": "CSR of the full graph streamed by the sampler each step (0.92 GB)"},
             "clocks": clocks,
+            "step_ms": {"median": float(np.median(step_ms)), "min": float(np.min(step_ms)),
+                        "max": float(np.max(step_ms)), "p90": float(np.percentile(step_ms, 90))},
             "e2e": {"value": e_ms, "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 8,
                     "note": "wall clock of the public-API loop; features resident on the device, "
                             "the per-step input is the sampler seed"},
