@@ -285,6 +285,8 @@ def saint_main(a, world, rank, local_rank):
     torch.cuda.synchronize(dev)
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
+    if os.environ.get("RDM_WS_LOG"):
+        print("[bench] timed region start", file=sys.stderr, flush=True)
     e0.record(stream)
     # per-step marks on the compute stream (no host sync): the step-time
     # distribution shows whether a slow run is a few slow steps or all of them

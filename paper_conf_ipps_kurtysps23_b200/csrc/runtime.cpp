@@ -3,6 +3,8 @@
 // executor in gcn.cpp and the cost model in plan.cpp).
 #include <algorithm>
 #include <cmath>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <vector>
 
@@ -54,7 +56,10 @@ float* ensure_ws(std::unique_ptr<DevBuf>& b, size_t bytes) {
   if (!b || b->bytes < bytes) {
     // regrowth (sizes that vary per call, e.g. GraphSAINT subgraphs) gets 25 %
     // headroom so that cudaFree / cudaMalloc — both synchronising — stay rare
-    const size_t want = b ? bytes + bytes / 4 : bytes;
+    static const char* hr = getenv("RDM_WS_HEADROOM");   // percent, diagnosis (default 25)
+    const size_t pct = hr ? (size_t)atoi(hr) : 25;
+    const size_t want = b ? bytes + bytes * pct / 100 : bytes;
+    if (b && getenv("RDM_WS_LOG")) fprintf(stderr, "[rdm ws] regrow %zu -> %zu\n", b->bytes, want);
     b.reset();
     b.reset(new DevBuf(std::max<size_t>(want, 256)));
   }
