@@ -129,14 +129,9 @@ def forward(A, H0, Ws, labels, mask, bs=None, orders=None) -> Result:
     return res
 
 
-def backward(A, res: Result, Ws, relu_masks=None) -> Result:
+def backward(A, res: Result, Ws) -> Result:
     """eqs. (3)(4) with G^l = ∂ℓ/∂Z^l (reading R1), G^0 without Hadamard (R2).
-
-    `relu_masks[l-1]` (optional, l = 1..L-1) replaces the decision 1[Z^l > 0]
-    of σ'(Z^l): where floating point decides a discrete value both sides must
-    take that decision in the same precision (reading R30), so the
-    parity tests pass the fp32 kernel's own sign pattern; the arithmetic stays
-    fp64 and unchanged."""
+    σ'(Z^l) = 1[Z^l > 0] is taken from this oracle's own forward `res.Z`."""
     L = len(Ws)
     G = [None] * (L + 1)
     Y = [None] * (L + 1)
@@ -148,17 +143,16 @@ def backward(A, res: Result, Ws, relu_masks=None) -> Result:
         db[l] = G[l].sum(axis=0)
         D = S @ np.asarray(Ws[l - 1], np.float64).T   # A G^l (W^l)ᵀ
         if l > 1:
-            sig = (res.Z[l - 1] > 0) if relu_masks is None else np.asarray(relu_masks[l - 2], bool)
-            G[l - 1] = D * sig                  # eq. (3), σ'(Z) = 1[Z > 0]
+            G[l - 1] = D * (res.Z[l - 1] > 0)   # eq. (3), σ'(Z) = 1[Z > 0]
         else:
             G[0] = D
     res.G, res.Y, res.db = G, Y, db
     return res
 
 
-def epoch(A, H0, Ws, labels, mask, bs=None, relu_masks=None):
+def epoch(A, H0, Ws, labels, mask, bs=None):
     res = forward(A, H0, Ws, labels, mask, bs)
-    return backward(A, res, Ws, relu_masks)
+    return backward(A, res, Ws)
 
 
 def adam(p, g, m, v, step, lr=0.01, b1=0.9, b2=0.999, eps=1e-8):
@@ -174,11 +168,20 @@ def adam(p, g, m, v, step, lr=0.01, b1=0.9, b2=0.999, eps=1e-8):
 
 
 def max_rel_err(x, ref) -> float:
-    """Normwise max-relative error max|x−r| / max|r| (reading R26)."""
+    """Normwise max-relative error max|x−r| / max|r| (reading R26).
+
+    Shapes must match exactly (no broadcasting); a non-finite entry in x gives
+    inf; an empty pair gives 0; an all-zero reference gives the absolute error."""
     x = np.asarray(x, np.float64)
     ref = np.asarray(ref, np.float64)
-    den = np.abs(ref).max() if ref.size else 0.0
-    num = np.abs(x - ref).max() if ref.size else 0.0
+    if x.shape != ref.shape:
+        raise ValueError(f"max_rel_err: shape {x.shape} vs reference {ref.shape}")
+    if ref.size == 0:
+        return 0.0
+    if not np.all(np.isfinite(x)):
+        return float("inf")
+    den = float(np.abs(ref).max())
+    num = float(np.abs(x - ref).max())
     if den == 0.0:
-        return float(num)
-    return float(num / den)
+        return num
+    return num / den

@@ -11,6 +11,7 @@ import pytest
 import synth
 from oracle import gcn as og
 from oracle import saint as osaint
+from parity import BAND_FP32, relu_tiebreak
 
 pytestmark = pytest.mark.gpu
 
@@ -88,6 +89,26 @@ def _saint_run(rdm, g, H0, Ws, y, m, cfg, P, roots, h, seed, iters):
     s.close()
 
 
+def _full(rdm, model, which, layer, n, width, P):
+    """The full n x width tensor from whichever layout is resident on the P ranks."""
+    for layout in (rdm.ROW, rdm.COL):
+        try:
+            parts = [model.tensor_torch(which, layer, p, layout).cpu().numpy() for p in range(P)]
+        except rdm.RdmError:
+            continue
+        full = np.zeros((n, width))
+        for p, t in enumerate(parts):
+            lo, hi, _ = rdm.partition(P, layout, n, width, p)
+            if P == 1:
+                full[:] = t[:, :width]
+            elif layout == rdm.ROW:
+                full[lo:hi] = t[:, :width]
+            else:
+                full[:, lo:hi] = t[:, :hi - lo]
+        return full
+    raise AssertionError(f"tensor {which}/{layer} not resident")
+
+
 @pytest.mark.parametrize("P,cfg,core", [(1, 3, 0), (1, 10, 0), (2, 3, 0), (4, 10, 0), (4, 2, 0),
                                         (1, 3, 256), (2, 10, 384)])
 def test_saint_gcn_matches_oracle(rdm, P, cfg, core, monkeypatch):
@@ -105,26 +126,15 @@ def test_saint_gcn_matches_oracle(rdm, P, cfg, core, monkeypatch):
     for it, loss, dW, W_now, model in _saint_run(rdm, g, H0, Ws, y, m, cfg, P, roots, h, seed, 3):
         nodes, rp, cs, vs = osaint.sample(g, roots, h, seed, it)
         sub = synth.CSR(len(nodes), rp, cs, vs)
-        # ReLU decisions from the kernel's own forward (reading R30)
-        Hs = []
+        # forward H^l, then the oracle's backward with ReLU ties broken only in the band (R30)
+        Hs = [_full(rdm, model, rdm.T_H, l, len(nodes), f[l], P) for l in range(1, len(Ws))]
+        Zk = _full(rdm, model, rdm.T_Z, 0, len(nodes), f[-1], P)
+        ref = og.forward(sub, H0[nodes], W_now, y[nodes], m[nodes])
         for l in range(1, len(Ws)):
-            full = np.zeros((len(nodes), f[l]))
-            for layout in (rdm.ROW, rdm.COL):
-                try:
-                    parts = [model.tensor_torch(rdm.T_H, l, p, layout).cpu().numpy() for p in range(P)]
-                except rdm.RdmError:
-                    continue
-                for p, t in enumerate(parts):
-                    lo, hi, _ = rdm.partition(P, layout, len(nodes), f[l], p)
-                    if P == 1:
-                        full[:] = t
-                    elif layout == rdm.ROW:
-                        full[lo:hi] = t
-                    else:
-                        full[:, lo:hi] = t
-                break
-            Hs.append(full)
-        ref = og.epoch(sub, H0[nodes], W_now, y[nodes], m[nodes], relu_masks=[x > 0 for x in Hs])
+            assert og.max_rel_err(Hs[l - 1], og.relu(ref.Z[l])) < 1e-4, (it, "H", l)
+        assert og.max_rel_err(Zk, ref.Z[len(Ws)]) < 1e-4, (it, "logits")
+        relu_tiebreak(ref, Hs, BAND_FP32)
+        og.backward(sub, ref, W_now)
         assert abs(loss - ref.loss) <= 1e-5 * abs(ref.loss), (it, loss, ref.loss)
         for l in range(len(Ws)):
             assert og.max_rel_err(dW[l], ref.Y[l + 1]) < 1e-4, (it, l)

@@ -241,8 +241,48 @@ def test_symmetric_rmat_properties():
     assert np.all(np.diff(g.col[g.rowptr[0]:g.rowptr[1]]) > 0)
 
 
-def test_relu_masks_default_equivalence():
-    """Passing the oracle's own decisions 1[Z^l > 0] as relu_masks changes nothing."""
+def test_max_rel_err_catches_perturbations():
+    """Negative pins of the parity comparator (reading R26): a one-element 2e-4
+    perturbation fails the 1e-4 gate; zeros, empty inputs, shape mismatches and
+    non-finite values are handled explicitly."""
+    rng = np.random.default_rng(5)
+    r = rng.standard_normal((300, 17))
+    assert gcn.max_rel_err(r, r) == 0.0
+    x = r.copy()
+    i, j = 123, 7
+    x[i, j] += 2e-4 * np.abs(r).max()
+    e = gcn.max_rel_err(x, r)
+    assert e == pytest.approx(2e-4, rel=1e-9)
+    assert not e < 1e-4
+    x = r.copy()
+    x[0, 0] += 0.9e-4 * np.abs(r).max()
+    assert gcn.max_rel_err(x, r) < 1e-4
+    # the error is normwise: a small element wrong by 100 % of itself passes only if tiny
+    x = r.copy()
+    k = np.unravel_index(np.argmin(np.abs(r)), r.shape)
+    x[k] = 2 * r[k]
+    assert gcn.max_rel_err(x, r) == pytest.approx(abs(r[k]) / np.abs(r).max())
+    # zeros / empty / non-finite / shapes
+    z = np.zeros((4, 3))
+    assert gcn.max_rel_err(z, z) == 0.0
+    assert gcn.max_rel_err(z + 1e-3, z) == pytest.approx(1e-3)
+    assert gcn.max_rel_err(np.zeros((0, 5)), np.zeros((0, 5))) == 0.0
+    bad = r.copy()
+    bad[3, 3] = np.nan
+    assert gcn.max_rel_err(bad, r) == float("inf")
+    bad[3, 3] = np.inf
+    assert not gcn.max_rel_err(bad, r) < 1e-4
+    with pytest.raises(ValueError):
+        gcn.max_rel_err(r[:, :1], r)          # no broadcasting
+    with pytest.raises(ValueError):
+        gcn.max_rel_err(r.T, r)
+
+
+def test_relu_tiebreak_band():
+    """tests/parity.py (reading R30): disagreements inside the band are taken
+    from the kernel, one outside the band fails, and a tie-broken oracle
+    backward equals the plain one when there is nothing to break."""
+    from parity import relu_tiebreak
     n, f = 50, (6, 5, 4, 3)
     g = synth.rmat(n, 150, seed=2)
     H0 = synth.features(n, f[0])
@@ -250,7 +290,28 @@ def test_relu_masks_default_equivalence():
     y = synth.labels(n, f[-1])
     m = synth.train_mask(n)
     a = gcn.epoch(g, H0, Ws, y, m)
-    b = gcn.epoch(g, H0, Ws, y, m, relu_masks=[a.Z[1] > 0, a.Z[2] > 0])
+    ref = gcn.forward(g, H0, Ws, y, m)
+    Hk = [np.maximum(ref.Z[1], 0), np.maximum(ref.Z[2], 0)]
+    assert relu_tiebreak(ref, Hk) == (0, 0.0)
+    gcn.backward(g, ref, Ws)
     for l in (1, 2, 3):
-        assert np.array_equal(a.Y[l], b.Y[l])
-    assert np.array_equal(a.G[0], b.G[0])
+        assert np.array_equal(a.Y[l], ref.Y[l])
+    # in-band flip: the kernel says positive where the oracle's Z is a tiny negative
+    ref = gcn.forward(g, H0, Ws, y, m)
+    Z1 = ref.Z[1]
+    zmax = np.abs(Z1).max()
+    neg = np.argwhere(Z1 < 0)[0]
+    Z1[tuple(neg)] = -0.5 * 2.0 ** -16 * zmax
+    Hk = [np.maximum(Z1, 0), np.maximum(ref.Z[2], 0)]
+    Hk[0][tuple(neg)] = 1e-9
+    nd, worst = relu_tiebreak(ref, Hk)
+    assert nd == 1 and worst == pytest.approx(0.5 * 2.0 ** -16)
+    assert ref.Z[1][tuple(neg)] > 0
+    # out-of-band flip is rejected
+    ref = gcn.forward(g, H0, Ws, y, m)
+    Z1 = ref.Z[1]
+    pos = np.argwhere(Z1 > 1e-3 * np.abs(Z1).max())[0]
+    Hk = [np.maximum(Z1, 0), np.maximum(ref.Z[2], 0)]
+    Hk[0][tuple(pos)] = 0.0
+    with pytest.raises(AssertionError):
+        relu_tiebreak(ref, Hk)
