@@ -54,5 +54,6 @@ def lib():
         L.oracle_spmm_t.argtypes = [i64, vp, vp, vp, vp, i64, vp]
         L.oracle_spmm_rows.argtypes = [vp, vp, vp, vp, i64, i64, vp, i64, vp]
         L.oracle_num_threads.restype = ctypes.c_int
+        L.oracle_set_threads.argtypes = [ctypes.c_int]
         _lib = L
     return _lib

@@ -75,3 +75,6 @@ void oracle_spmm_rows(const int64_t* rowptr, const int32_t* col, const float* va
 }
 
 int oracle_num_threads(void) { return omp_get_max_threads(); }
+
+/* Thread count of the loops above (bench.py times the oracle at nproc and at 1). */
+void oracle_set_threads(int n) { if (n > 0) omp_set_num_threads(n); }
