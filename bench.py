@@ -42,6 +42,10 @@ def parse():
     ap.add_argument("--impl", default="rdm", choices=["rdm", "reference"])
     ap.add_argument("--config", default="auto")
     ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--emulate", type=int, default=0,
+                    help="one-rank emulation of a P-rank job on one GPU (rdm_init_emulated); "
+                         "default workload papers (BASELINE configs[4]) at P = 8")
+    ap.add_argument("--emulate-rank", type=int, default=0)
     ap.add_argument("--threads", type=int, default=0,
                     help="--impl reference: oracle threads (default nproc)")
     ap.add_argument("--ref-budget-s", type=float, default=150.0,
@@ -200,6 +204,8 @@ def saint_main(a, world, rank, local_rank):
     wl = synth.WORKLOADS[a.workload]
     f = [wl.f[0], a.hidden or 256] + [wl.f[-1]] if wl.L == 2 else list(wl.f)
     metric = "GraphSAINT-RDM ms per subgraph step (sample + build + fwd + bwd + Adam)"
+    # BASELINE configs[3]: GraphSAINT on the Reddit-shaped graph, 2 layers, hidden 256
+    saint_name = f"{wl.name.split(' ')[0]} GraphSAINT-RDM {len(f) - 1}L h{f[1]} (BASELINE configs[3])"
     g = synth.make_graph(wl)
     H0 = synth.features(wl.n, f[0])
     y = synth.labels(wl.n, f[-1])
@@ -217,7 +223,7 @@ def saint_main(a, world, rank, local_rank):
                           "n_gpus": a.gpus, "steps": len(times), "warmup": 0, "ms_per_step": v,
                           "higher_is_better": False, "scaling": "strong", "vs_baseline": None,
                           "dtype": "f64", "data": "synthetic",
-                          "config": {"workload": wl.name + "_saint", "f": f, "roots": a.roots,
+                          "config": {"workload": saint_name, "f": f, "roots": a.roots,
                                      "walk_len": a.walk_len},
                           "cpu_baseline": {"value": v, "unit": "ms", "cores": cores, "kind": "oracle",
                                            "sample": desc},
@@ -347,7 +353,7 @@ def saint_main(a, world, rank, local_rank):
             "metric": metric, "value": ms_step, "unit": "ms", "n_gpus": world, "steps": a.steps,
             "warmup": max(3, a.warmup), "ms_per_step": ms_step, "higher_is_better": False,
             "scaling": "strong", "vs_baseline": None, "dtype": "f32", "data": "synthetic",
-            "config": {"workload": wl.name + "_saint", "model": f"GCN 2L f={'/'.join(map(str, f))}",
+            "config": {"workload": saint_name, "model": f"GCN 2L f={'/'.join(map(str, f))}",
                        "sampler": f"random walk, {a.roots} roots, length {a.walk_len} (readings R31-R34)",
                        "n_sub_mean": float(ns[:, 0].mean()), "nnz_sub_mean": float(ns[:, 1].mean()),
                        "config_id": cfg_id, "pareto": pareto, "transport": a.transport,
@@ -366,6 +372,8 @@ def saint_main(a, world, rank, local_rank):
                          "spmm_share_of_step": ph_ms["spmm"] / max(1e-9, ms_total)},
             "cpu_baseline": cpu,
             "phases_ms_per_step": {k: v / a.steps for k, v in ph_ms.items()},
+            "phases_note": "sample = subgraph build on the sampler stream, overlapped with the "
+                           "previous subgraph's training: the phases add up to more than the step",
             "loss": float(loss.item())}), flush=True)
     ctx.sync()
     model.close()
@@ -373,6 +381,132 @@ def saint_main(a, world, rank, local_rank):
     ctx.close()
     if world > 1:
         dist.destroy_process_group()
+
+
+def emulate_main(a):
+    """One-rank emulation of a P-rank job on one GPU (rdm.h rdm_init_emulated):
+    rank `--emulate-rank` of P = --emulate holds exactly its partitions and runs
+    exactly its SpMMs, GEMMs, pack/unpack, loss and Adam at the P-rank shapes;
+    exchanges and all-reduces are skipped (nothing crosses a link).  Default
+    workload: BASELINE configs[4], papers100M-shaped 2L h128 at P = 8, with the
+    liveness-based workspace (RDM_GCN_LOW_MEMORY).  The line reports the rank's
+    compute epoch (device time), its per-phase split, the SpMM roofline, and the
+    exchange volume a real rank would move with the time it would take at the
+    NVLink peer bandwidth B200_PROFILING.md records for this pool (770 GB/s per
+    direction; not measured by this build)."""
+    import numpy as np
+    import torch
+    import paper_conf_ipps_kurtysps23_b200 as rdm
+    import synth
+    P, p = a.emulate, a.emulate_rank
+    wl = synth.WORKLOADS[a.workload]
+    dev = torch.device("cuda", 0)
+    torch.cuda.set_device(dev)
+    stream = torch.cuda.Stream(device=dev)
+    torch.cuda.set_stream(stream)
+    t0 = time.time()
+    g = synth.make_graph(wl)
+    t_gen = time.time() - t0
+    lo, hi, _ = rdm.partition(P, rdm.ROW, wl.n, wl.f[0], p)
+    H0 = torch.from_numpy(synth.features_rows(lo, hi, wl.f[0])).to(dev)
+    y = torch.from_numpy(synth.labels_rows(lo, hi, wl.f[-1])).to(dev)
+    m = torch.ones(hi - lo, dtype=torch.uint8, device=dev)
+    Wd = [torch.from_numpy(w).to(dev) for w in synth.weights(wl.f)]
+    dW = [torch.zeros_like(w) for w in Wd]
+    mom = [torch.zeros_like(w) for w in Wd]
+    vel = [torch.zeros_like(w) for w in Wd]
+    loss = torch.zeros(1, dtype=torch.float64, device=dev)
+    ctx = rdm.Context(rank=p, world=P, device=0, stream=stream, emulate=True)
+    ctx.set_precision(a.precision)
+    t0 = time.time()
+    ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
+    t_set = time.time() - t0
+    ginfo = ctx.graph_info()
+    pareto, chosen, _, _ = rdm.select_config(list(wl.f), wl.n, wl.nnz, P)
+    cfg = chosen if a.config == "auto" else int(a.config)
+    model = rdm.GCN(ctx, wl.f, cfg, low_memory=True)
+    info = model.info()
+    model.set_input([H0], [y], [m])
+    del g
+    step = [0]
+
+    def epoch():
+        model.forward(Wd, loss)
+        model.backward(Wd, dW)
+        step[0] += 1
+        ctx.adam_step(Wd, dW, mom, vel, step[0], lr=0.01)
+
+    for _ in range(max(3, a.warmup)):
+        epoch()
+    ctx.sync()
+    ctx.reset_counters()
+    ctx.reset_phase_times()
+    ctx.set_timing(True)
+    clk = ClockSampler(0)
+    clk.start()
+    time.sleep(0.3)
+    torch.cuda.synchronize(dev)
+    e0 = torch.cuda.Event(enable_timing=True)
+    e1 = torch.cuda.Event(enable_timing=True)
+    e0.record(stream)
+    for _ in range(a.steps):
+        epoch()
+    e1.record(stream)
+    torch.cuda.synchronize(dev)
+    clocks = clk.stop()
+    ms = e0.elapsed_time(e1) / a.steps
+    cnt = ctx.counters()
+    ph_ms, _ = ctx.phase_times()
+    peaks = {}
+    try:
+        peaks = json.load(open(os.path.join(ROOT, "MEASURED_PEAKS.json")))
+    except Exception:
+        pass
+    hbm_peak = float(peaks.get("hbm_gbs", 6650.0))
+    n, nnz = wl.n, wl.nnz
+    calls = cnt["spmm_calls"]
+    sum_w = cnt["spmm_nnz_cols"] / max(1, nnz)          # Σ w_p over the rank's SpMM calls
+    alg = calls * (8 * nnz + 8 * (n + 1)) + 8 * n * sum_w
+    spmm_s = ph_ms["spmm"] / 1e3
+    achieved = alg / spmm_s / 1e9 if spmm_s > 0 else 0.0
+    nvlink = 770.0
+    a2a_ms = cnt["a2a_bytes_wire"] / a.steps / (nvlink * 1e9) * 1e3
+    line = {
+        "metric": METRIC, "impl": "rdm-emulated-rank", "value": ms, "unit": "ms",
+        "n_gpus": 1, "emulated_world": P, "emulated_rank": p, "steps": a.steps,
+        "warmup": max(3, a.warmup), "ms_per_step": ms, "higher_is_better": False,
+        "scaling": "strong", "vs_baseline": None, "dtype": DTYPES[a.precision], "data": "synthetic",
+        "config": {"workload": wl.name + f" (one-rank emulation of P = {P}, BASELINE configs[4])",
+                   "model": f"GCN {wl.L}L f={'/'.join(map(str, wl.f))}", "n": n, "nnz": nnz,
+                   "config_id": cfg, "config_name": rdm.config_name(model.cfg), "pareto": pareto,
+                   "row_slice": [lo, hi], "low_memory": True,
+                   "workspace_gb": info["workspace_bytes"] / 1e9,
+                   "graph_gb": (8 * nnz + 8 * (n + 1)) / 1e9,
+                   "device_mem_peak_gb": torch.cuda.max_memory_allocated(dev) / 1e9,
+                   "device_mem_used_gb": (torch.cuda.mem_get_info(dev)[1] - torch.cuda.mem_get_info(dev)[0]) / 1e9,
+                   "hub_tiles": ginfo.get("n_tiles", 0), "core_K": ginfo.get("core_K", 0),
+                   "gen_s": round(t_gen, 1), "set_graph_s": round(t_set, 1),
+                   "l2": "inputs larger than L2 (13.7 GB CSR streamed per SpMM)"},
+        "what_is_timed": "this rank's compute only: SpMMs, GEMMs, pack/unpack, loss, Adam; no exchange",
+        "clocks": clocks, "gpu_launches": cnt["kernel_launches"],
+        "roofline": {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",
+                     "frac": achieved / hbm_peak, "traffic": None,
+                     "algorithmic_gb_per_call": alg / max(1, calls) / 1e9,
+                     "avg_call_ms": ph_ms["spmm"] / a.steps / max(1, calls / a.steps),
+                     "kernel": "spmm call on the rank's column slice (w = f/P)",
+                     "peak_source": "MEASURED_PEAKS.json hbm_gbs (measured copy)"},
+        "phases_ms_per_step": {k: v / a.steps for k, v in ph_ms.items()},
+        "exchange": {"bytes_per_step": cnt["a2a_bytes_wire"] / a.steps,
+                     "modelled_ms_at_770_gbs": a2a_ms,
+                     "epoch_ms_compute_plus_modelled_exchange": ms + a2a_ms,
+                     "note": "770 GB/s per direction = B200_PROFILING.md's measured peer copy on this "
+                             "pool (not measured by this build); no overlap assumed"},
+        "plan": {"model_comm_units": info["model_comm_units"],
+                 "model_sparse_units": info["model_sparse_units"]},
+    }
+    print(json.dumps(line), flush=True)
+    model.close()
+    ctx.close()
 
 
 def cpu_baseline_full(a, wl, g, H0, Ws, y, msk):
@@ -404,6 +538,10 @@ def cpu_baseline_full(a, wl, g, H0, Ws, y, msk):
 def main():
     a = parse()
     import numpy as np
+    if a.emulate:
+        if a.workload == "reddit" and "--workload" not in sys.argv:
+            a.workload = "papers"
+        return emulate_main(a)
     if a.saint:
         return saint_main(a, int(os.environ.get("WORLD_SIZE", "1")), int(os.environ.get("RANK", "0")),
                           int(os.environ.get("LOCAL_RANK", "0")))
@@ -415,10 +553,12 @@ def main():
     wl = synth.WORKLOADS[a.workload]
     if a.workload == "papers" and world < 8:
         # BASELINE configs[4] is an 8-GPU stress case (≈13.7 GB CSR + ≈70 GB of
-        # dense slices per GPU at P = 8); fewer GPUs do not hold it
+        # dense slices per GPU at P = 8); fewer GPUs do not hold it.  One rank of
+        # it runs on one GPU with --emulate 8.
         if rank == 0:
             print(json.dumps({"metric": METRIC, "impl": a.impl, "unavailable":
-                              "papers100M-shaped workload is defined for 8 GPUs (BASELINE configs[4])"}))
+                              "papers100M-shaped workload is defined for 8 GPUs (BASELINE configs[4]); "
+                              "bench.py --emulate 8 runs one rank of it on one GPU"}))
         return
 
     if a.impl == "reference":

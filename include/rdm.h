@@ -109,11 +109,17 @@ enum {
   RDM_GCN_INPUT_GRAD = 1, /* also compute G^0 = A G^1 (W^1)ᵀ (Fig. 4 output; reading R2) —
                              required for costs to match Table IV                       */
   RDM_GCN_BIAS = 2,       /* Z = Â H W + 1 bᵀ (reading R8); not implemented: UNSUPPORTED */
-  RDM_GCN_PANELS = 4      /* R_A < P (§III-E): run on the row panels installed by
+  RDM_GCN_PANELS = 4,     /* R_A < P (§III-E): run on the row panels installed by
                              rdm_set_graph_panels (a symmetric A) instead of the replicated
                              graph; column-layout tensors are tiles (rdm_partition_tile),
                              SpMMs broadcast input tiles inside column groups, redistributions
                              stay inside panel groups; RDM_TRANSPORT_P2P fusion is not used */
+  RDM_GCN_LOW_MEMORY = 8  /* liveness-based workspace: buffers of the same shape whose lifetimes
+                             within an epoch do not overlap share one allocation (first fit,
+                             largest first).  Results are identical; rdm_gcn_tensor returns
+                             RDM_ERR_STATE for a tensor whose memory a later step reuses.  For
+                             the stress shapes (papers100M-shaped at P = 8, SURVEY App. B:
+                             "~70 GB/GPU of live tensors with liveness-based reuse")      */
 };
 
 /* Tensors exposed by rdm_gcn_tensor (for parity tests / inspection). */
@@ -169,6 +175,19 @@ rdm_status rdm_get_unique_id(void* id);
  * Errors: RDM_ERR_ARG (bad rank/world/device), RDM_ERR_CUDA, RDM_ERR_NCCL. */
 rdm_status rdm_init(rdm_ctx** ctx, int rank, int world, const void* nccl_unique_id, int device,
                     void* cuda_stream);
+/* One-rank emulation of a P-rank job (measurement of the stress shapes, e.g.
+ * BASELINE configs[4], papers100M-shaped at P = 8, on a single GPU): a ctx
+ * that is rank `rank` of `world` ranks with NO peers and no NCCL.  It holds
+ * exactly that rank's partitions (row slice rows_p x f, column slices
+ * N x w_p, its staging buffers) and runs exactly that rank's SpMMs, GEMMs,
+ * pack/unpack, loss and Adam at the P-rank shapes; every exchange and
+ * all-reduce is skipped (nothing crosses a link: the received blocks keep
+ * their previous contents and the counters still count the traffic a real
+ * rank would move).  For timing and memory measurement only — the numerical
+ * results are NOT those of the P-rank job.  RDM_TRANSPORT_P2P is refused
+ * (RDM_ERR_UNSUPPORTED).  Errors: RDM_ERR_ARG (world < 2, rank), RDM_ERR_CUDA. */
+rdm_status rdm_init_emulated(rdm_ctx** ctx, int rank, int world, int device, void* cuda_stream);
+int rdm_is_emulated(const rdm_ctx* ctx);
 rdm_status rdm_finalize(rdm_ctx* ctx);
 const char* rdm_last_error(const rdm_ctx* ctx);
 /* Block until the ctx's stream is idle; surfaces asynchronous CUDA/NCCL faults. */
@@ -429,7 +448,8 @@ typedef struct {
   int64_t plan_comm_units, plan_hidden_comm_units, plan_sparse_units;
   int64_t a2a_elems;
   int n_fwd_steps, n_bwd_steps;
-  int64_t workspace_bytes; /* activation workspace per process */
+  int64_t workspace_bytes; /* activation workspace per process (rdm_plan_info: of rank 0,
+                              honouring RDM_GCN_LOW_MEMORY in flags)                      */
 } rdm_gcn_info;
 rdm_status rdm_gcn_get_info(const rdm_gcn* g, rdm_gcn_info* out);
 /* Human-readable step list (forward then backward) into buf[cap]. */

@@ -31,7 +31,7 @@ GEMM_NN, GEMM_NT, GEMM_TN = 0, 1, 2
 ALL_RANKS = -1
 MAX_LAYERS = 8
 UNIQUE_ID_BYTES = 128
-GCN_INPUT_GRAD, GCN_BIAS, GCN_PANELS = 1, 2, 4
+GCN_INPUT_GRAD, GCN_BIAS, GCN_PANELS, GCN_LOW_MEMORY = 1, 2, 4, 8
 T_H, T_Z, T_G, T_MEMO, T_DWP = range(5)
 PHASES = ["spmm", "gemm", "pack", "a2a", "loss", "allreduce", "adam", "other", "sample"]
 _STATUS = {0: "OK", 1: "ERR_ARG", 2: "ERR_CUDA", 3: "ERR_NCCL", 4: "ERR_OOM",
@@ -53,7 +53,7 @@ EXPORTS = [
     "rdm_set_transport", "rdm_get_transport", "rdm_debug_disable_tc",
     "rdm_set_precision", "rdm_get_precision", "rdm_set_graph_panels", "rdm_partition_tile",
     "rdm_redistribute_panels", "rdm_spmm_panels", "rdm_max_replication", "rdm_select_config_ra",
-    "rdm_saint_wait",
+    "rdm_saint_wait", "rdm_init_emulated", "rdm_is_emulated",
 ]
 
 
@@ -94,6 +94,7 @@ _sig = {
     "rdm_set_stream": [_vp, _vp],
     "rdm_partition": [_int, _int, _i64, _i64, _int, _pi64, _pi64, _pi64],
     "rdm_set_graph": [_vp, _i64, _i64, _vp, _vp, _vp, _int, _int],
+    "rdm_init_emulated": [ctypes.POINTER(_vp), _int, _int, _int, _vp],
     "rdm_spmm": [_vp, _int, _vp, _i64, _vp, _i64, _i64, _int, _vp, _vp, _i64],
     "rdm_gemm": [_vp, _int, _vp, _i64, _vp, _i64, _vp, _i64, _i64, _i64, _i64, _int, _vp, _vp],
     "rdm_redistribute": [_vp, _int, _pp, _pp, _i64, _i64],
@@ -137,7 +138,7 @@ _lib.rdm_last_error.argtypes = [_vp]
 _lib.rdm_last_error.restype = ctypes.c_char_p
 _lib.rdm_config_to_id.argtypes = [ctypes.POINTER(RdmConfig)]
 _lib.rdm_config_to_id.restype = _i64
-for _n in ("rdm_world", "rdm_num_local", "rdm_get_transport", "rdm_get_precision"):
+for _n in ("rdm_world", "rdm_num_local", "rdm_get_transport", "rdm_get_precision", "rdm_is_emulated"):
     getattr(_lib, _n).argtypes = [_vp]
     getattr(_lib, _n).restype = _int
 _lib.rdm_debug_disable_tc.argtypes = [_int]
@@ -265,14 +266,16 @@ def redist_plan(world, rank, from_layout, n, f):
     return {k: list(a) for k, a in zip(keys, arrs)}
 
 
-def plan_info(f, cfg, P, n, input_grad=True):
-    """→ (info dict, step list text) of the executor plan, without a GPU."""
+def plan_info(f, cfg, P, n, input_grad=True, low_memory=False):
+    """→ (info dict, step list text) of the executor plan, without a GPU
+    (workspace_bytes: rank 0's activation workspace)."""
     L = len(f) - 1
     c = config_from_id(L, cfg) if isinstance(cfg, int) else cfg
     fa = (ctypes.c_int64 * len(f))(*f)
     info = RdmGcnInfo()
     buf = ctypes.create_string_buffer(1 << 16)
-    _check(_lib.rdm_plan_info(L, fa, ctypes.byref(c), P, n, GCN_INPUT_GRAD if input_grad else 0,
+    flags = (GCN_INPUT_GRAD if input_grad else 0) | (GCN_LOW_MEMORY if low_memory else 0)
+    _check(_lib.rdm_plan_info(L, fa, ctypes.byref(c), P, n, flags,
                               ctypes.byref(info), buf, len(buf)), what="rdm_plan_info")
     return info.as_dict(), buf.value.decode()
 
@@ -295,15 +298,23 @@ class Context:
     """One rank of a P-process job (NCCL), a single process (world=1), or a
     virtual group of `world` ranks on one GPU (rank=ALL_RANKS)."""
 
-    def __init__(self, rank=0, world=1, device=0, stream=None, unique_id: bytes | None = None):
+    def __init__(self, rank=0, world=1, device=0, stream=None, unique_id: bytes | None = None,
+                 emulate=False):
+        """emulate=True: rank `rank` of `world` with no peers (rdm_init_emulated;
+        timing / memory measurement of one rank of a P-rank job on one GPU)."""
         import torch
         if stream is None:
             stream = torch.cuda.current_stream(device)
         self.stream = stream
         h = ctypes.c_void_p()
-        uid = ctypes.create_string_buffer(unique_id, UNIQUE_ID_BYTES) if unique_id else None
-        _check(_lib.rdm_init(ctypes.byref(h), rank, world, uid, device, stream.cuda_stream),
-               what=f"rdm_init(rank={rank}, world={world}, device={device})")
+        if emulate:
+            _check(_lib.rdm_init_emulated(ctypes.byref(h), rank, world, device, stream.cuda_stream),
+                   what=f"rdm_init_emulated(rank={rank}, world={world}, device={device})")
+        else:
+            uid = ctypes.create_string_buffer(unique_id, UNIQUE_ID_BYTES) if unique_id else None
+            _check(_lib.rdm_init(ctypes.byref(h), rank, world, uid, device, stream.cuda_stream),
+                   what=f"rdm_init(rank={rank}, world={world}, device={device})")
+        self.emulated = bool(emulate)
         self.h = h
         self.world = world
         self.device = device
@@ -423,14 +434,16 @@ class Context:
 class GCN:
     """A GCN instance (L layers, widths f) running configuration `cfg` (ID or RdmConfig)."""
 
-    def __init__(self, ctx: Context, f, cfg, input_grad=True, saint=None, panels=False):
+    def __init__(self, ctx: Context, f, cfg, input_grad=True, saint=None, panels=False,
+                 low_memory=False):
         self.ctx = ctx
         self.f = list(f)
         self.L = len(f) - 1
         self.cfg = config_from_id(self.L, cfg) if isinstance(cfg, int) else cfg
         fa = (ctypes.c_int64 * len(f))(*f)
         h = ctypes.c_void_p()
-        flags = (GCN_INPUT_GRAD if input_grad else 0) | (GCN_PANELS if panels else 0)
+        flags = ((GCN_INPUT_GRAD if input_grad else 0) | (GCN_PANELS if panels else 0)
+                 | (GCN_LOW_MEMORY if low_memory else 0))
         self.saint = saint   # keeps the sampler alive while this instance exists
         if saint is None:
             ctx._c(_lib.rdm_gcn_create(ctx.h, self.L, fa, ctypes.byref(self.cfg), flags,

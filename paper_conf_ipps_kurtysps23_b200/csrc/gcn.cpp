@@ -241,7 +241,141 @@ struct Planner {
 struct Buf {
   float* p = nullptr;
   int64_t rows = 0, cols = 0, ld = 0;
+  bool valid_end = true;   // contents still this tensor's after an epoch (RDM_GCN_LOW_MEMORY)
 };
+
+// ------------------------------------------------------ workspace planning
+// Every (tensor, layout) the plan touches gets a buffer.  Its shape on rank p:
+// a row slice (rows of p x ld(f)), a column slice (N x ld(w_p)) or, at
+// R_A < P, a tile.  Its lifetime is the step interval [first, last] over the
+// epoch's sequence (forward steps, then backward steps; kEnd = the end of the
+// epoch).  H^0 row (the input) lives throughout; the operands of the
+// weight-gradient GEMMs run on a side stream joined at the end of the
+// backward pass, so they live to kEnd; a redistribution's destination may be
+// written by its producer one step earlier (fused P2P transport).
+// RDM_GCN_LOW_MEMORY: buffers of the same shape whose lifetimes do not
+// overlap share one allocation (first-fit, largest first) — same shape, so the
+// zero ld-padding every producer keeps stays zero.
+constexpr int kEnd = 1 << 20;
+
+struct ShapeCtx {
+  int P = 1, p = 0, RA = 0;
+  int64_t n_cap = 0;
+  bool saint = false;
+};
+
+Buf shape_of(const ShapeCtx& sc, int lay, int64_t width) {
+  Buf b;
+  if (lay == RDM_ROW) {
+    b.rows = sc.saint ? ceil_div(sc.n_cap, sc.P) : row_range(sc.n_cap, sc.P, sc.p).size();
+    b.cols = width;
+    b.ld = roundup4(width);
+  } else if (sc.RA) {   // tile: panel rows x column slice over the R_A column groups
+    Range r, c;
+    tile_of(sc.P, sc.RA, sc.n_cap, width, sc.p, &r, &c, &b.ld);
+    b.rows = r.size();
+    b.cols = c.size();
+  } else {
+    b.rows = sc.n_cap;
+    b.cols = col_range(width, sc.P, sc.p).size();
+    b.ld = roundup4(b.cols);
+  }
+  return b;
+}
+
+struct BufPlan {
+  std::pair<int, int> key;   // (tensor id, normalised layout)
+  int64_t width = 0;
+  int first = kEnd, last = -1;
+  Buf shape;
+  int slab = -1;
+};
+struct SlabPlan {
+  size_t bytes = 0;
+  std::vector<int> members;   // indices into the BufPlan list
+};
+
+// Lifetimes of every buffer of the plan (layouts normalised: P = 1 has one).
+std::vector<BufPlan> buffer_lifetimes(const Planner& pl, const std::vector<Step>& fwd,
+                                      const std::vector<Step>& bwd) {
+  std::map<std::pair<int, int>, BufPlan> m;
+  auto lay = [&](int l) { return pl.P == 1 ? 0 : l; };
+  auto use = [&](Key k, int l, int first, int last) {
+    auto key = std::make_pair(k.id(), lay(l));
+    BufPlan& b = m[key];
+    b.key = key;
+    b.width = pl.width.at(k.id());
+    b.first = std::min(b.first, first);
+    b.last = std::max(b.last, last);
+  };
+  use({K_H, 0}, RDM_ROW, -1, kEnd);   // the input, set before the epoch
+  int t = 0;
+  for (auto* v : {&fwd, &bwd})
+    for (const Step& s : *v) {
+      switch (s.op) {
+        case S_SPMM:
+        case S_GEMM:
+          use(s.in, s.lin, t, t);
+          use(s.out, s.lout, t, t);
+          if (s.epi & RDM_EPI_MASK) use(s.mask, s.lmask, t, t);
+          break;
+        case S_TN:
+          use(s.in, s.lin, t, kEnd);
+          use(s.in2, s.lin2, t, kEnd);
+          break;
+        case S_REDIST:
+          use(s.in, s.lin, t, t);
+          use(s.out, s.lout, std::max(0, t - 1), t);
+          break;
+        case S_MASK:
+          use(s.out, s.lout, t, t);
+          use(s.mask, s.lmask, t, t);
+          break;
+        case S_LOSS:
+          use(s.in, s.lin, t, t);
+          use(s.out, s.lout, t, t);
+          break;
+      }
+      ++t;
+    }
+  std::vector<BufPlan> out;
+  for (auto& kv : m) out.push_back(kv.second);
+  return out;
+}
+
+// Shapes + slab assignment for rank sc.p; returns the slabs, fills b.slab.
+std::vector<SlabPlan> plan_slabs(std::vector<BufPlan>& bufs, const ShapeCtx& sc, bool low_memory) {
+  for (auto& b : bufs) b.shape = shape_of(sc, b.key.second, b.width);
+  auto bytes_of = [](const Buf& s) { return (size_t)std::max<int64_t>(1, s.rows * s.ld) * sizeof(float); };
+  std::vector<int> order(bufs.size());
+  for (size_t i = 0; i < bufs.size(); ++i) order[i] = (int)i;
+  std::stable_sort(order.begin(), order.end(), [&](int a, int b) {
+    const size_t ba = bytes_of(bufs[a].shape), bb = bytes_of(bufs[b].shape);
+    return ba != bb ? ba > bb : bufs[a].first < bufs[b].first;
+  });
+  std::vector<SlabPlan> slabs;
+  for (int i : order) {
+    BufPlan& b = bufs[i];
+    int pick = -1;
+    if (low_memory) {
+      for (size_t k = 0; k < slabs.size() && pick < 0; ++k) {
+        const BufPlan& r = bufs[slabs[k].members[0]];
+        if (r.shape.rows != b.shape.rows || r.shape.cols != b.shape.cols || r.shape.ld != b.shape.ld) continue;
+        bool free = true;
+        for (int j : slabs[k].members)
+          if (!(bufs[j].last < b.first || b.last < bufs[j].first)) free = false;
+        if (free) pick = (int)k;
+      }
+    }
+    if (pick < 0) {
+      slabs.push_back({bytes_of(b.shape), {}});
+      pick = (int)slabs.size() - 1;
+    }
+    slabs[pick].members.push_back(i);
+    b.slab = pick;
+  }
+  return slabs;
+}
 
 }  // namespace
 }  // namespace rdm
@@ -336,38 +470,6 @@ Buf& buf(rdm_gcn* g, int slot, Key k, int l) {
     throw Error(RDM_ERR_STATE, std::string("executor: missing buffer ") + kKindName[k.kind] +
                                    std::to_string(k.layer));
   return it->second;
-}
-
-void alloc_buf(rdm_gcn* g, Key k, int l, int64_t width) {
-  rdm_ctx* ctx = g->ctx;
-  const int P = ctx->world;
-  const int64_t n = g->n_cap;
-  for (int s = 0; s < ctx->nlocal(); ++s) {
-    auto key = std::make_pair(k.id(), norm_lay(g, l));
-    if (g->bufs[s].count(key)) continue;
-    const int p = ctx->local[s];
-    Buf b;
-    if (norm_lay(g, l) == RDM_ROW) {
-      b.rows = cap_rows(g, p);
-      b.cols = width;
-      b.ld = roundup4(width);
-    } else if (g->RA) {   // tile: panel rows x column slice over the R_A column groups
-      Range r, c;
-      tile_of(P, g->RA, n, width, p, &r, &c, &b.ld);
-      b.rows = r.size();
-      b.cols = c.size();
-    } else {
-      b.rows = n;
-      b.cols = col_range(width, P, p).size();
-      b.ld = roundup4(b.cols);
-    }
-    const size_t bytes = (size_t)std::max<int64_t>(1, b.rows * b.ld) * sizeof(float);
-    g->mem.emplace_back(new DevBuf(bytes));
-    RDM_CUDA(cudaMemset(g->mem.back()->ptr, 0, bytes));
-    b.p = g->mem.back()->as<float>();
-    g->ws_bytes += bytes;
-    g->bufs[s][key] = b;
-  }
 }
 
 void plan_info(const Planner& pl, const std::vector<Step>& fwd, const std::vector<Step>& bwd,
@@ -476,38 +578,31 @@ void create(rdm_gcn* g) {
   pl.igrad = (g->flags & RDM_GCN_INPUT_GRAD) != 0;
   pl.plan(g->fwd, g->bwd);
   g->bufs.assign(ctx->nlocal(), {});
-  auto touch = [&](const Step& s) {
-    auto w = [&](Key k) { return pl.width.at(k.id()); };
-    switch (s.op) {
-      case S_SPMM:
-      case S_GEMM:
-        alloc_buf(g, s.in, s.lin, w(s.in));
-        alloc_buf(g, s.out, s.lout, w(s.out));
-        if (s.epi & RDM_EPI_MASK) alloc_buf(g, s.mask, s.lmask, w(s.mask));
-        break;
-      case S_TN:
-        alloc_buf(g, s.in, s.lin, w(s.in));
-        alloc_buf(g, s.in2, s.lin2, w(s.in2));
-        break;
-      case S_REDIST:
-        alloc_buf(g, s.in, s.lin, w(s.in));
-        alloc_buf(g, s.out, s.lout, w(s.out));
-        break;
-      case S_MASK:
-        alloc_buf(g, s.out, s.lout, w(s.out));
-        alloc_buf(g, s.mask, s.lmask, w(s.mask));
-        break;
-      case S_LOSS:
-        alloc_buf(g, s.in, s.lin, w(s.in));
-        alloc_buf(g, s.out, s.lout, w(s.out));
-        break;
+  const bool low_memory = (g->flags & RDM_GCN_LOW_MEMORY) != 0;
+  for (int s = 0; s < ctx->nlocal(); ++s) {
+    ShapeCtx sc;
+    sc.P = ctx->world;
+    sc.p = ctx->local[s];
+    sc.RA = g->RA;
+    sc.n_cap = g->n_cap;
+    sc.saint = g->saint != nullptr;
+    std::vector<BufPlan> bp = buffer_lifetimes(pl, g->fwd, g->bwd);
+    std::vector<SlabPlan> slabs = plan_slabs(bp, sc, low_memory);
+    std::vector<float*> base(slabs.size());
+    for (size_t k = 0; k < slabs.size(); ++k) {
+      g->mem.emplace_back(new DevBuf(slabs[k].bytes));
+      RDM_CUDA(cudaMemset(g->mem.back()->ptr, 0, slabs[k].bytes));
+      base[k] = g->mem.back()->as<float>();
+      g->ws_bytes += (int64_t)slabs[k].bytes;
     }
-  };
-  // H^0 lives in both layouts
-  alloc_buf(g, {K_H, 0}, RDM_ROW, g->f[0]);
-  alloc_buf(g, {K_H, 0}, RDM_COL, g->f[0]);
-  for (auto& s : g->fwd) touch(s);
-  for (auto& s : g->bwd) touch(s);
+    for (const BufPlan& b : bp) {
+      Buf x = b.shape;
+      x.p = base[b.slab];
+      for (int j : slabs[b.slab].members)
+        if (bp[j].first > b.first) x.valid_end = false;   // a later tensor reuses this memory
+      g->bufs[s][b.key] = x;
+    }
+  }
   const int P = ctx->world;
   const int64_t n = g->n_cap;
   g->dwp.assign(ctx->nlocal(), std::vector<float*>(g->L + 1, nullptr));
@@ -897,11 +992,14 @@ void apply_input(rdm_gcn* g, const InputArgs* a) {
         RDM_CUDA(cudaMemsetAsync(g->mask[i], 1, r, ctx->stream));
     }
     src[i] = h.p;
-    dst[i] = buf(g, i, {K_H, 0}, RDM_COL).p;
+    auto hc = g->bufs[i].find({Key{K_H, 0}.id(), norm_lay(g, RDM_COL)});
+    dst[i] = hc == g->bufs[i].end() ? nullptr : hc->second.p;
   }
-  if (P > 1 && g->RA)
+  // H^0's column slices only if the plan reads them (reading R12)
+  const bool need_col = P > 1 && dst[0] != nullptr;
+  if (need_col && g->RA)
     redistribute_panels(ctx, RDM_ROW, src.data(), dst.data(), n, f0);
-  else if (P > 1)
+  else if (need_col)
     redistribute(ctx, RDM_ROW, src.data(), dst.data(), n, f0);
   std::vector<double*> nt(nl);
   for (int i = 0; i < nl; ++i) {
@@ -941,10 +1039,10 @@ void do_saint_input(void* a_) {
     const Range r = row_range(n, P, p);
     Buf& hr = buf(g, i, {K_H, 0}, RDM_ROW);
     saint_gather(ctx, a->H, a->ldh, nodes, r.lo, r.size(), 0, f0, hr.p, hr.ld);
-    if (P > 1) {
-      Buf& hc = buf(g, i, {K_H, 0}, RDM_COL);
+    auto hc = g->bufs[i].find({Key{K_H, 0}.id(), norm_lay(g, RDM_COL)});
+    if (P > 1 && hc != g->bufs[i].end()) {
       const Range c = col_range(f0, P, p);
-      saint_gather(ctx, a->H, a->ldh, nodes, 0, n, c.lo, c.size(), hc.p, hc.ld);
+      saint_gather(ctx, a->H, a->ldh, nodes, 0, n, c.lo, c.size(), hc->second.p, hc->second.ld);
     }
     saint_gather_labels(ctx, a->labels, a->mask, nodes, r.lo, r.size(), g->labels[i], g->mask[i]);
   }
@@ -1108,6 +1206,10 @@ rdm_status rdm_gcn_tensor(rdm_gcn* g, int which, int layer, int slot, rdm_layout
     return RDM_ERR_ARG;
   }
   const Buf& b = it->second;
+  if (!b.valid_end) {
+    g->ctx->err = "rdm_gcn_tensor: RDM_GCN_LOW_MEMORY reuses this tensor's memory later in the epoch";
+    return RDM_ERR_STATE;
+  }
   if (ptr) *ptr = b.p;
   if (rows) *rows = b.rows;
   if (cols) *cols = b.cols;
@@ -1142,7 +1244,17 @@ extern "C" rdm_status rdm_plan_info(int L, const int64_t* f, const rdm_config* c
     pl.igrad = (flags & RDM_GCN_INPUT_GRAD) != 0;
     std::vector<Step> fwd, bwd;
     pl.plan(fwd, bwd);
-    if (out) plan_info(pl, fwd, bwd, n, out);
+    if (out) {
+      plan_info(pl, fwd, bwd, n, out);
+      // activation workspace of rank 0 (full replication, no sampler)
+      ShapeCtx sc;
+      sc.P = P;
+      sc.n_cap = n;
+      std::vector<BufPlan> bp = buffer_lifetimes(pl, fwd, bwd);
+      int64_t bytes = 0;
+      for (const SlabPlan& sl : plan_slabs(bp, sc, (flags & RDM_GCN_LOW_MEMORY) != 0)) bytes += (int64_t)sl.bytes;
+      out->workspace_bytes = bytes;
+    }
     if (desc && cap) {
       const std::string s = describe_steps(fwd, bwd);
       std::snprintf(desc, cap, "%s", s.c_str());

@@ -70,6 +70,46 @@ struct DevBuf {
   T* as() const { return static_cast<T*>(ptr); }
 };
 
+// Buffers retired by a regrowth (ensure_ws / Pinned) inside a step: freeing
+// them at once would synchronise the whole device, so they are parked here
+// and released at the next host synchronisation point (rdm_sync, finalize,
+// sampler / executor destruction).
+void retire(void* dev_ptr, void* host_ptr);
+void release_retired();
+
+// Pinned host staging buffer (grows, never shrinks): D2H copies into pageable
+// memory block the host at the call, and H2D copies from pageable memory are
+// synchronous, so copies meant to stay asynchronous go through one of these.
+// A regrowth retires the old buffer (freed at the next rdm_sync / finalize:
+// cudaFreeHost synchronises the device) and is logged under RDM_WS_LOG.
+struct Pinned {
+  void* p = nullptr;
+  size_t bytes = 0;
+  Pinned() = default;
+  Pinned(const Pinned&) = delete;
+  Pinned& operator=(const Pinned&) = delete;
+  Pinned(Pinned&& o) noexcept : p(o.p), bytes(o.bytes) {
+    o.p = nullptr;
+    o.bytes = 0;
+  }
+  Pinned& operator=(Pinned&& o) noexcept {
+    if (this != &o) {
+      if (p) retire(nullptr, p);
+      p = o.p;
+      bytes = o.bytes;
+      o.p = nullptr;
+      o.bytes = 0;
+    }
+    return *this;
+  }
+  ~Pinned();
+  void reserve(size_t want);
+  template <class T> T* get(size_t count) {
+    reserve(count * sizeof(T));
+    return static_cast<T*>(p);
+  }
+};
+
 // ------------------------------------------------------------------- graph
 struct Csr;
 
@@ -113,6 +153,7 @@ struct Csr {
   std::unique_ptr<DevBuf> seg_start;    // int64[n_seg]: first nnz of each segment
   std::unique_ptr<DevBuf> heavy_rows;   // int32[n_heavy]
   std::unique_ptr<DevBuf> heavy_seg;    // int32[n_heavy+1]: segment range of heavy row
+  Pinned bins_stage;                    // pinned staging of the bins' upload (build_bins)
   int64_t max_deg = 0;
   // every stored value factors as a_ij = s_i·s_j (GCN normalisation; checked
   // on the host at rdm_set_graph): fp32 s per row, used by the fast-precision
@@ -141,6 +182,7 @@ struct rdm_ctx {
   cudaStream_t stream = nullptr;
   ncclComm_t comm = nullptr;
   bool poisoned = false;
+  bool emulated = false;         // one rank of a P-rank job with no peers (rdm_init_emulated)
   int transport = 0;             // RDM_TRANSPORT_NCCL / RDM_TRANSPORT_P2P
   int prec = 0;                  // RDM_PREC_FP32 / RDM_PREC_FAST
   std::string err;
@@ -180,35 +222,15 @@ struct rdm_ctx {
 
 // GraphSAINT-RDM sampler (saint.cu): the current subgraph and the device
 // workspace that builds it.
-// Pinned host staging buffer (grows, never shrinks): D2H copies into pageable
-// memory block the host at the call, so copies meant to share one sync land here.
-struct rdm_pinned {
-  void* p = nullptr;
-  size_t bytes = 0;
-  rdm_pinned() = default;
-  rdm_pinned(const rdm_pinned&) = delete;
-  rdm_pinned& operator=(const rdm_pinned&) = delete;
-  ~rdm_pinned() { if (p) cudaFreeHost(p); }
-  template <class T> T* get(size_t count) {
-    const size_t want = count * sizeof(T);
-    if (want > bytes) {
-      if (p) cudaFreeHost(p);
-      p = nullptr;
-      bytes = 0;
-      if (cudaMallocHost(&p, want + want / 4) != cudaSuccess) throw ::rdm::Error(RDM_ERR_OOM, "pinned host buffer");
-      bytes = want + want / 4;
-    }
-    return static_cast<T*>(p);
-  }
-};
-
 struct rdm_saint {
   rdm_ctx* ctx = nullptr;
-  rdm_pinned h_scal, h_rp, h_rrp, h_bucket;   // host staging of the sampler's round trips
+  rdm::Pinned h_scal, h_rp, h_rrp, h_bucket;   // host staging of the sampler's round trips
+  bool reserved = false;  // every workspace sized at its bound (first rdm_saint_sample)
   int64_t roots = 0;
   int walk_len = 0;
   uint64_t seed = 0;
   int64_t n_cap = 0;
+  int64_t nnz_bound = 0;  // entries of any subgraph (reserve_bounds)
   // Double-buffered subgraphs: rdm_saint_sample builds the next subgraph on the
   // sampler's own stream into the buffer the previous-but-one subgraph used
   // (after the executor released it, ev_free), while the compute stream still
@@ -261,7 +283,10 @@ struct Scatter {
 void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
           int64_t w, int epi, const float* bias, const float* mask, int64_t ld_mask,
           const Scatter* scat = nullptr);
-void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host);
+// Row bins from a host copy of the rowptr.  The upload is asynchronous on
+// ctx->stream from A.bins_stage; sync = false leaves the stream unsynchronised
+// (the caller guarantees the staging is not rewritten before the copy ran).
+void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, bool sync = true);
 
 // gemm.cu
 void gemm(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, int64_t ldw, float* C,

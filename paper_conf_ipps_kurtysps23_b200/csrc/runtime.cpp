@@ -6,6 +6,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <mutex>
 #include <vector>
 
 #include "internal.h"
@@ -52,18 +53,75 @@ DevBuf::~DevBuf() {
   if (ptr) cudaFree(ptr);
 }
 
+// Workspace diagnostics, read on every call (tests may set them at any time):
+// RDM_WS_LOG=1 logs every regrowth; RDM_WS_HEADROOM = percent of headroom on a
+// regrowth (default 25, clamped to 0..400).
+static bool ws_log() {
+  const char* v = getenv("RDM_WS_LOG");
+  return v && atoi(v) > 0;
+}
+static size_t ws_headroom_pct() {
+  const char* v = getenv("RDM_WS_HEADROOM");
+  if (!v) return 25;
+  const long x = strtol(v, nullptr, 10);
+  return (size_t)std::min<long>(400, std::max<long>(0, x));
+}
+
+namespace {
+std::mutex g_retired_mu;
+std::vector<void*> g_retired_dev, g_retired_host;
+}  // namespace
+
+void retire(void* dev_ptr, void* host_ptr) {
+  std::lock_guard<std::mutex> lk(g_retired_mu);
+  if (dev_ptr) g_retired_dev.push_back(dev_ptr);
+  if (host_ptr) g_retired_host.push_back(host_ptr);
+}
+
+void release_retired() {
+  std::vector<void*> d, h;
+  {
+    std::lock_guard<std::mutex> lk(g_retired_mu);
+    d.swap(g_retired_dev);
+    h.swap(g_retired_host);
+  }
+  for (void* p : d) cudaFree(p);       // synchronises the device: only at sync points
+  for (void* p : h) cudaFreeHost(p);
+}
+
 float* ensure_ws(std::unique_ptr<DevBuf>& b, size_t bytes) {
   if (!b || b->bytes < bytes) {
-    // regrowth (sizes that vary per call, e.g. GraphSAINT subgraphs) gets 25 %
-    // headroom so that cudaFree / cudaMalloc — both synchronising — stay rare
-    static const char* hr = getenv("RDM_WS_HEADROOM");   // percent, diagnosis (default 25)
-    const size_t pct = hr ? (size_t)atoi(hr) : 25;
-    const size_t want = b ? bytes + bytes * pct / 100 : bytes;
-    if (b && getenv("RDM_WS_LOG")) fprintf(stderr, "[rdm ws] regrow %zu -> %zu\n", b->bytes, want);
-    b.reset();
-    b.reset(new DevBuf(std::max<size_t>(want, 256)));
+    // regrowth (sizes that vary per call, e.g. GraphSAINT subgraphs) gets
+    // headroom so that it stays rare; the old buffer is retired, not freed
+    // (cudaFree would synchronise the device in the middle of a step)
+    const size_t want = b ? bytes + bytes * ws_headroom_pct() / 100 : bytes;
+    if (b && ws_log()) fprintf(stderr, "[rdm ws] regrow %zu -> %zu\n", b->bytes, want);
+    std::unique_ptr<DevBuf> nb(new DevBuf(std::max<size_t>(want, 256)));
+    if (b) {
+      retire(b->ptr, nullptr);
+      b->ptr = nullptr;
+    }
+    b = std::move(nb);
   }
   return b->as<float>();
+}
+
+Pinned::~Pinned() {
+  if (p) cudaFreeHost(p);
+}
+
+void Pinned::reserve(size_t want) {
+  if (want <= bytes) return;
+  const size_t nb = want + want / 4;
+  if (p && ws_log()) fprintf(stderr, "[rdm ws] pinned regrow %zu -> %zu\n", bytes, nb);
+  void* q = nullptr;
+  if (cudaMallocHost(&q, nb) != cudaSuccess) {
+    (void)cudaGetLastError();
+    throw Error(RDM_ERR_OOM, "pinned host buffer of " + std::to_string(nb) + " B");
+  }
+  if (p) retire(nullptr, p);
+  p = q;
+  bytes = nb;
 }
 
 // ------------------------------------------------------------------- timing
@@ -101,6 +159,8 @@ static void drain_events(rdm_ctx* ctx) {
   if (ctx->events.empty()) return;
   RDM_CUDA(cudaStreamSynchronize(ctx->stream));
   for (auto& e : ctx->events) {
+    // phases may have been recorded on another stream (the GraphSAINT sampler's)
+    RDM_CUDA(cudaEventSynchronize(e.b));
     float ms = 0;
     RDM_CUDA(cudaEventElapsedTime(&ms, e.a, e.b));
     ctx->phase_ms[e.phase] += ms;
@@ -126,7 +186,7 @@ void exchange(rdm_ctx* ctx, std::vector<Xfer>& x) {
       }
     return;
   }
-  if (P == 1) return;
+  if (P == 1 || ctx->emulated) return;   // emulated rank: no peers, nothing crosses a link
   const int p = ctx->rank;
   RDM_NCCL(ncclGroupStart());
   for (int q = 0; q < P; ++q) {
@@ -148,7 +208,7 @@ void allreduce(rdm_ctx* ctx, float* const* bufs, int64_t count) {
     for (int i = 1; i < ctx->nlocal(); ++i)
       RDM_CUDA(cudaMemcpyAsync(bufs[i], bufs[0], count * sizeof(float), cudaMemcpyDeviceToDevice,
                                ctx->stream));
-  } else {
+  } else if (!ctx->emulated) {
     RDM_NCCL(ncclAllReduce(bufs[0], bufs[0], count, ncclFloat, ncclSum, ctx->comm, ctx->stream));
   }
   ctx->counters.allreduce_bytes += count * 4;
@@ -164,7 +224,7 @@ void allreduce_d(rdm_ctx* ctx, double* const* bufs, int64_t count) {
     sum_doubles(ctx, tmp, parts.data(), ctx->nlocal());
     for (int i = 0; i < ctx->nlocal(); ++i)
       RDM_CUDA(cudaMemcpyAsync(bufs[i], tmp, sizeof(double), cudaMemcpyDeviceToDevice, ctx->stream));
-  } else {
+  } else if (!ctx->emulated) {
     RDM_NCCL(ncclAllReduce(bufs[0], bufs[0], count, ncclDouble, ncclSum, ctx->comm, ctx->stream));
   }
   ctx->counters.allreduce_bytes += count * 8;
@@ -275,7 +335,7 @@ void count_fused_redist(rdm_ctx* ctx, rdm_layout from, int64_t n, int64_t f) {
 // completes on my stream, every rank's stream has reached the same point.
 // Virtual group / P = 1: stream order already is the barrier.
 void p2p_barrier(rdm_ctx* ctx) {
-  if (ctx->world == 1 || ctx->virtual_group()) return;
+  if (ctx->world == 1 || ctx->virtual_group() || ctx->emulated) return;
   Phase ph(ctx, RDM_PH_A2A);
   float* w = ensure_ws(ctx->ws_scratch, 4096);
   RDM_NCCL(ncclAllReduce(w, w, 1, ncclFloat, ncclSum, ctx->comm, ctx->stream));
@@ -284,6 +344,7 @@ void p2p_barrier(rdm_ctx* ctx) {
 // Peer base addresses of one device allocation per rank (CUDA IPC, handles
 // all-gathered over NCCL).  Virtual group: not used (slots share a process).
 std::vector<float*> p2p_open(rdm_ctx* ctx, float* mine, std::vector<void*>& opened) {
+  if (ctx->emulated) throw Error(RDM_ERR_UNSUPPORTED, "P2P transport on an emulated rank");
   const int P = ctx->world;
   std::vector<float*> out(P, nullptr);
   out[ctx->rank] = mine;
@@ -478,6 +539,34 @@ rdm_status rdm_init(rdm_ctx** out, int rank, int world, const void* uid, int dev
   return RDM_OK;
 }
 
+rdm_status rdm_init_emulated(rdm_ctx** out, int rank, int world, int device, void* stream) {
+  if (!out || world < 2 || world > BlockTable::kMax || rank < 0 || rank >= world) return RDM_ERR_ARG;
+  int ndev = 0;
+  if (cudaGetDeviceCount(&ndev) != cudaSuccess || device < 0 || device >= ndev) {
+    (void)cudaGetLastError();
+    return RDM_ERR_CUDA;
+  }
+  rdm_ctx* ctx = new rdm_ctx();
+  ctx->world = world;
+  ctx->rank = rank;
+  ctx->emulated = true;
+  ctx->device = device;
+  ctx->stream = (cudaStream_t)stream;
+  ctx->local.push_back(rank);
+  rdm_status st = guarded(ctx, [&] {
+    RDM_CUDA(cudaSetDevice(device));
+    RDM_CUDA(cudaDeviceGetAttribute(&ctx->num_sms, cudaDevAttrMultiProcessorCount, device));
+  });
+  if (st != RDM_OK) {
+    delete ctx;
+    return st;
+  }
+  *out = ctx;
+  return RDM_OK;
+}
+
+int rdm_is_emulated(const rdm_ctx* ctx) { return ctx && ctx->emulated ? 1 : 0; }
+
 rdm_status rdm_finalize(rdm_ctx* ctx) {
   if (!ctx) return RDM_ERR_ARG;
   cudaSetDevice(ctx->device);
@@ -490,6 +579,7 @@ rdm_status rdm_finalize(rdm_ctx* ctx) {
   for (auto e : ctx->event_pool) cudaEventDestroy(e);
   if (ctx->comm) ncclCommDestroy(ctx->comm);
   delete ctx;
+  release_retired();
   return RDM_OK;
 }
 
@@ -498,6 +588,7 @@ const char* rdm_last_error(const rdm_ctx* ctx) { return ctx ? ctx->err.c_str() :
 rdm_status rdm_sync(rdm_ctx* ctx) {
   return guarded(ctx, [&] {
     RDM_CUDA(cudaStreamSynchronize(ctx->stream));
+    release_retired();
     if (ctx->comm) {
       ncclResult_t async_err;
       RDM_NCCL(ncclCommGetAsyncError(ctx->comm, &async_err));
@@ -514,6 +605,10 @@ rdm_status rdm_set_stream(rdm_ctx* ctx, void* stream) {
 
 rdm_status rdm_set_transport(rdm_ctx* ctx, int transport) {
   if (!ctx || (transport != RDM_TRANSPORT_NCCL && transport != RDM_TRANSPORT_P2P)) return RDM_ERR_ARG;
+  if (ctx->emulated && transport == RDM_TRANSPORT_P2P) {
+    ctx->err = "rdm_set_transport: an emulated rank has no peer memory";
+    return RDM_ERR_UNSUPPORTED;
+  }
   ctx->transport = transport;
   return RDM_OK;
 }

@@ -21,7 +21,10 @@
 // sync with the hub-core histogram when a core is built).
 #include <cub/cub.cuh>
 
+#include <algorithm>
 #include <cmath>
+#include <functional>
+#include <vector>
 
 #include "internal.h"
 
@@ -566,10 +569,91 @@ void build_core_sub_finish(rdm_saint* s, Csr& S, int64_t kmax, const unsigned lo
   const int64_t rnnz = rrph[n];
   R.n = n;
   R.nnz = rnnz;
-  build_bins(ctx, R, rrph);
+  build_bins(ctx, R, rrph, false);
   c.K = K;
   c.nnz = nnz - rnnz;
   c.forced = forced;
+}
+
+template <class In, class Out>
+size_t scan_temp_bytes(int64_t count) {
+  size_t t = 0;
+  RDM_CUDA(cub::DeviceScan::ExclusiveSum(nullptr, t, (In*)nullptr, (Out*)nullptr, (int)count, (cudaStream_t)0));
+  return t;
+}
+
+// Bins of a CSR with at most `rows` rows and `nnz` entries (spmm.cu: light
+// rows + 2048-entry segments of heavy rows) and their pinned staging.
+void reserve_bins(Csr& C, int64_t rows, int64_t nnz) {
+  const int64_t seg = nnz / 2048 + rows + 1;
+  ensure_ws(C.light_rows, std::max<int64_t>(1, rows) * sizeof(int32_t));
+  ensure_ws(C.seg_start, seg * (sizeof(int64_t) + sizeof(int32_t)));
+  ensure_ws(C.heavy_rows, std::max<int64_t>(1, rows) * sizeof(int32_t));
+  ensure_ws(C.heavy_seg, (rows + 1) * sizeof(int32_t));
+  C.bins_stage.reserve((size_t)seg * 12 + (size_t)(3 * rows + 1) * 4 + 64);
+}
+
+// Every workspace of the sampler sized once at its bound, so that no step
+// allocates (a regrowth inside a step was the cause of the step-time spikes):
+// a subgraph has at most n_cap vertices and at most
+//   nnz_bound = min(nnz(A), Σ of the n_cap largest degrees, n_cap²)
+// entries; its hub core at most core_kmax(n_cap) hubs.
+void reserve_bounds(rdm_saint* s) {
+  rdm_ctx* ctx = s->ctx;
+  const Csr& A = ctx->graph.A;
+  const int64_t N = A.n, cap = s->n_cap;
+  std::vector<int64_t> rp(N + 1);
+  RDM_CUDA(cudaMemcpy(rp.data(), A.rowptr->ptr, (N + 1) * sizeof(int64_t), cudaMemcpyDeviceToHost));
+  std::vector<int64_t> deg(N);
+  for (int64_t i = 0; i < N; ++i) deg[i] = rp[i + 1] - rp[i];
+  if (cap < N) std::nth_element(deg.begin(), deg.begin() + cap, deg.end(), std::greater<int64_t>());
+  int64_t top = 0;
+  for (int64_t i = 0; i < cap; ++i) top += deg[i];
+  const int64_t nnzb = std::max<int64_t>(1, std::min<int64_t>({A.nnz, top, cap * cap}));
+  const int64_t seg_full = cap + A.nnz / kSeg + 1;
+  const int64_t seg_sub = cap + nnzb / kSeg + 1;
+  const int64_t kmax = core_kmax(cap, nnzb);
+  s->nnz_bound = nnzb;
+  for (int b = 0; b < 2; ++b) {
+    Csr& S = s->bufs[b].A;
+    ensure_ws(S.rowptr, (cap + 1) * sizeof(int64_t));
+    ensure_ws(S.col, nnzb * sizeof(int32_t));
+    ensure_ws(S.val, nnzb * sizeof(float));
+    reserve_bins(S, cap, nnzb);
+    ensure_ws(s->nodes_b[b], cap * sizeof(int32_t));
+    if (kmax) {
+      Core& c = S.core;
+      ensure_ws(c.A, (size_t)kmax * kmax * sizeof(float));
+      if (!c.resid) c.resid.reset(new Csr());
+      Csr& R = *c.resid;
+      ensure_ws(R.rowptr, (cap + 1) * sizeof(int64_t));
+      ensure_ws(R.col, nnzb * sizeof(int32_t));
+      ensure_ws(R.val, nnzb * sizeof(float));
+      reserve_bins(R, cap, nnzb);
+      ensure_ws(c.hub_ids, kmax * sizeof(int32_t));
+      ensure_ws(c.hub_slot, cap * sizeof(int32_t));
+    }
+  }
+  ensure_ws(s->core_tmp, (size_t)4 * cap * sizeof(int32_t) + 256);
+  ensure_ws(s->core_rank, cap * sizeof(int32_t));
+  ensure_ws(s->core_seg, (2 * (cap + 1) + seg_sub) * 4 + 16);
+  ensure_ws(s->core_cnt, 2 * seg_sub * sizeof(int64_t));
+  ensure_ws(s->core_bucket, kMaxBuckets * 8);
+  size_t t = 256;
+  t = std::max(t, scan_temp_bytes<int32_t, int32_t>(std::max<int64_t>(N, cap + 1)));
+  t = std::max(t, scan_temp_bytes<unsigned long long, int64_t>(cap + 1));
+  t = std::max(t, scan_temp_bytes<int64_t, int64_t>(std::max(seg_full, seg_sub)));
+  ensure_ws(s->tmp, t);
+  size_t tb = 0;
+  RDM_CUDA(cub::DeviceRadixSort::SortPairsDescending(nullptr, tb, (int32_t*)nullptr, (int32_t*)nullptr,
+                                                      (int32_t*)nullptr, (int32_t*)nullptr, (int)cap, 0, 32,
+                                                      (cudaStream_t)0));
+  ensure_ws(s->tmp2, std::max<size_t>(tb, 256));
+  s->h_rp.reserve((cap + 1) * sizeof(int64_t));
+  s->h_rrp.reserve((cap + 1) * sizeof(int64_t));
+  s->h_scal.reserve(4 * sizeof(unsigned long long));
+  s->h_bucket.reserve(kMaxBuckets * sizeof(unsigned long long));
+  s->reserved = true;
 }
 
 void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
@@ -588,6 +672,7 @@ void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
       RDM_CUDA(cudaEventCreateWithFlags(&s->ev_free[b], cudaEventDisableTiming));
     }
   }
+  if (!s->reserved) reserve_bounds(s);
   const int b = s->iteration < 0 ? 0 : (s->cur ^ 1);
   struct OnStream {
     rdm_ctx* c; cudaStream_t m;
@@ -644,7 +729,7 @@ void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
   RDM_CUDA(cudaMemcpyAsync(hs, scal, 2 * sizeof(unsigned long long), cudaMemcpyDeviceToHost, ctx->stream));
   RDM_CUDA(cudaStreamSynchronize(ctx->stream));
   const int64_t n = (int64_t)hs[0], nnz = (int64_t)hs[1];
-  if (n > cap) throw Error(RDM_ERR_STATE, "saint: subgraph larger than its capacity");
+  if (n > cap || nnz > s->nnz_bound) throw Error(RDM_ERR_STATE, "saint: subgraph larger than its bound");
 
   Graph& G = s->bufs[b];
   Csr& S = G.A;
@@ -671,7 +756,9 @@ void sample(rdm_saint* s, int64_t it, int64_t* n_out, int64_t* nnz_out) {
   unsigned long long* hb = s->h_bucket.get<unsigned long long>(kMaxBuckets);
   if (kmax) build_core_sub(s, S, kmax, deg, hb);
   RDM_CUDA(cudaStreamSynchronize(ctx->stream));
-  build_bins(ctx, S, rph);
+  // bins uploaded asynchronously on the sampler stream: their pinned staging is
+  // rewritten only two samples later, after this stream has been synchronised
+  build_bins(ctx, S, rph, false);
   if (kmax) build_core_sub_finish(s, S, kmax, hb);
   G.n = n;
   G.nnz = nnz;
@@ -747,6 +834,7 @@ rdm_status rdm_saint_destroy(rdm_saint* s) {
     }
   }
   delete s;
+  release_retired();
   return RDM_OK;
 }
 

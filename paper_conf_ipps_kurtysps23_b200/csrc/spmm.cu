@@ -763,8 +763,7 @@ heavy:
 }  // namespace
 
 // Row bins (host, one-time at rdm_set_graph; pure indexing of rowptr).
-void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rp) {
-  (void)ctx;
+void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rp, bool sync) {
   const int64_t n = A.n;
   std::vector<int64_t> cnt(kSeg + 2, 0);
   int64_t n_heavy = 0, n_seg = 0, max_deg = 0;
@@ -781,9 +780,19 @@ void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rp) {
   const int64_t n_light = n - n_heavy;
   std::vector<int64_t> pos(kSeg + 2, 0);
   for (int64_t b = 1; b < kSeg + 2; ++b) pos[b] = pos[b - 1] + cnt[b - 1];
-  std::vector<int32_t> light(n_light);
-  std::vector<int64_t> seg_start(n_seg);
-  std::vector<int32_t> seg_row(n_seg), heavy(n_heavy), heavy_seg(n_heavy + 1);
+  // the bins are written straight into pinned staging, uploaded asynchronously:
+  //   seg_start int64[n_seg] | seg_row int32[n_seg] | light int32[n_light] |
+  //   heavy int32[n_heavy] | heavy_seg int32[n_heavy+1]
+  const size_t b_seg = (size_t)n_seg * (sizeof(int64_t) + sizeof(int32_t));
+  const size_t b_light = (size_t)n_light * sizeof(int32_t);
+  const size_t b_heavy = (size_t)n_heavy * sizeof(int32_t);
+  const size_t b_hseg = (size_t)(n_heavy + 1) * sizeof(int32_t);
+  char* st = A.bins_stage.get<char>(b_seg + b_light + b_heavy + b_hseg + 64);
+  int64_t* seg_start = reinterpret_cast<int64_t*>(st);
+  int32_t* seg_row = reinterpret_cast<int32_t*>(st + (size_t)n_seg * sizeof(int64_t));
+  int32_t* light = reinterpret_cast<int32_t*>(st + b_seg);
+  int32_t* heavy = reinterpret_cast<int32_t*>(st + b_seg + b_light);
+  int32_t* heavy_seg = reinterpret_cast<int32_t*>(st + b_seg + b_light + b_heavy);
   int64_t s = 0, h = 0;
   for (int64_t i = 0; i < n; ++i) {
     const int64_t d = rp[i + 1] - rp[i];
@@ -811,20 +820,12 @@ void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rp) {
   ensure_ws(A.seg_start, std::max<int64_t>(1, n_seg) * (sizeof(int64_t) + sizeof(int32_t)));
   ensure_ws(A.heavy_rows, std::max<int64_t>(1, n_heavy) * sizeof(int32_t));
   ensure_ws(A.heavy_seg, (n_heavy + 1) * sizeof(int32_t));
-  if (n_light)
-    RDM_CUDA(cudaMemcpy(A.light_rows->ptr, light.data(), n_light * sizeof(int32_t),
-                        cudaMemcpyHostToDevice));
-  if (n_seg) {
-    RDM_CUDA(cudaMemcpy(A.seg_start->ptr, seg_start.data(), n_seg * sizeof(int64_t),
-                        cudaMemcpyHostToDevice));
-    RDM_CUDA(cudaMemcpy(A.seg_start->as<int64_t>() + n_seg, seg_row.data(),
-                        n_seg * sizeof(int32_t), cudaMemcpyHostToDevice));
-  }
-  if (n_heavy)
-    RDM_CUDA(cudaMemcpy(A.heavy_rows->ptr, heavy.data(), n_heavy * sizeof(int32_t),
-                        cudaMemcpyHostToDevice));
-  RDM_CUDA(cudaMemcpy(A.heavy_seg->ptr, heavy_seg.data(), (n_heavy + 1) * sizeof(int32_t),
-                      cudaMemcpyHostToDevice));
+  const cudaMemcpyKind h2d = cudaMemcpyHostToDevice;
+  if (n_light) RDM_CUDA(cudaMemcpyAsync(A.light_rows->ptr, light, b_light, h2d, ctx->stream));
+  if (n_seg) RDM_CUDA(cudaMemcpyAsync(A.seg_start->ptr, seg_start, b_seg, h2d, ctx->stream));
+  if (n_heavy) RDM_CUDA(cudaMemcpyAsync(A.heavy_rows->ptr, heavy, b_heavy, h2d, ctx->stream));
+  RDM_CUDA(cudaMemcpyAsync(A.heavy_seg->ptr, heavy_seg, b_hseg, h2d, ctx->stream));
+  if (sync) RDM_CUDA(cudaStreamSynchronize(ctx->stream));
 }
 
 // Dense hub core (one-time, host side, at rdm_set_graph for symmetric A):

@@ -40,6 +40,8 @@ def lib():
         L.synth_rmat_csr.argtypes = [i64, i64, u64, dbl, dbl, dbl, ctypes.c_int, ctypes.c_int, vp, vp, vp]
         L.synth_rmat_csr.restype = ctypes.c_int
         L.synth_features.argtypes = [i64, i64, u64, vp]
+        L.synth_features_rows.argtypes = [i64, i64, i64, u64, vp]
+        L.synth_labels_rows.argtypes = [i64, i64, i64, u64, vp]
         L.synth_glorot.argtypes = [i64, i64, u64, vp]
         L.synth_labels.argtypes = [i64, i64, u64, vp]
         L.synth_mask.argtypes = [i64, dbl, u64, vp]
@@ -93,6 +95,22 @@ def features(n: int, f: int, seed: int = SEED_H) -> np.ndarray:
     out = np.empty((n, f), dtype=np.float32)
     if n * f:
         lib().synth_features(n, f, seed, _p(out))
+    return out
+
+
+def features_rows(lo: int, hi: int, f: int, seed: int = SEED_H) -> np.ndarray:
+    """Rows [lo, hi) of features(n, f, seed) (identical values)."""
+    out = np.empty((hi - lo, f), dtype=np.float32)
+    if (hi - lo) * f:
+        lib().synth_features_rows(lo, hi, f, seed, _p(out))
+    return out
+
+
+def labels_rows(lo: int, hi: int, C: int, seed: int = SEED_LABELS) -> np.ndarray:
+    """Entries [lo, hi) of labels(n, C, seed)."""
+    out = np.empty(hi - lo, dtype=np.int32)
+    if hi > lo:
+        lib().synth_labels_rows(lo, hi, C, seed, _p(out))
     return out
 
 

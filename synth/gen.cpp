@@ -205,6 +205,15 @@ void synth_features(int64_t n, int64_t f, uint64_t seed, float* out) {
       out[i * f + j] = (float)(u24(ctr_hash(seed, 2, (uint64_t)(i * f + j))) * 2.0 - 1.0);
 }
 
+// Rows [lo, hi) of the same features (one rank's row slice of a matrix too
+// large to draw whole on the host).
+void synth_features_rows(int64_t lo, int64_t hi, int64_t f, uint64_t seed, float* out) {
+#pragma omp parallel for schedule(static)
+  for (int64_t i = lo; i < hi; ++i)
+    for (int64_t j = 0; j < f; ++j)
+      out[(i - lo) * f + j] = (float)(u24(ctr_hash(seed, 2, (uint64_t)(i * f + j))) * 2.0 - 1.0);
+}
+
 // Glorot-uniform W (fin x fout, row-major): U[-s, s), s = sqrt(6/(fin+fout)).
 void synth_glorot(int64_t fin, int64_t fout, uint64_t seed, float* out) {
   double s = std::sqrt(6.0 / (double)(fin + fout));
@@ -216,6 +225,12 @@ void synth_glorot(int64_t fin, int64_t fout, uint64_t seed, float* out) {
 void synth_labels(int64_t n, int64_t C, uint64_t seed, int32_t* out) {
 #pragma omp parallel for schedule(static)
   for (int64_t i = 0; i < n; ++i) out[i] = (int32_t)(ctr_hash(seed, 4, (uint64_t)i) % (uint64_t)C);
+}
+
+// Labels of rows [lo, hi).
+void synth_labels_rows(int64_t lo, int64_t hi, int64_t C, uint64_t seed, int32_t* out) {
+#pragma omp parallel for schedule(static)
+  for (int64_t i = lo; i < hi; ++i) out[i - lo] = (int32_t)(ctr_hash(seed, 4, (uint64_t)i) % (uint64_t)C);
 }
 
 // Train mask with a given keep fraction (1.0 -> all ones).

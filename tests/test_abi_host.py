@@ -222,3 +222,45 @@ def test_select_config_ra_front_matches_oracle(seed):
         assert sparse == ocm.simulate(chosen, f)[1]
         if RA == P:
             assert front == rdm.select_config(f, n, nnz, P)[0]
+
+
+def test_low_memory_workspace_papers_p8():
+    """BASELINE configs[4] (papers100M-shaped 2L h128) at P = 8 fits one B200
+    (~70 GB/GPU of live tensors with liveness-based reuse):
+    rank 0's activation workspace under RDM_GCN_LOW_MEMORY, plus the
+    replicated CSR and the redistribution staging, stays below 170 GB."""
+    import synth
+    wl = synth.WORKLOADS["papers"]
+    P = 8
+    pareto, chosen, _, _ = rdm.select_config(list(wl.f), wl.n, wl.nnz, P)
+    assert chosen == 10 and pareto == [10]
+    full, _ = rdm.plan_info(list(wl.f), chosen, P, wl.n)
+    low, _ = rdm.plan_info(list(wl.f), chosen, P, wl.n, low_memory=True)
+    rows0 = wl.n // P + 1
+    staging = 2 * rows0 * max(wl.f) * 4            # pack send + unpack recv staging
+    csr = 8 * wl.nnz + 8 * (wl.n + 1)
+    assert low["workspace_bytes"] < 0.7 * full["workspace_bytes"]
+    assert low["workspace_bytes"] + staging + csr < 170e9, low["workspace_bytes"] / 1e9
+    # identical plan otherwise
+    for k in ("model_comm_units", "model_sparse_units", "plan_comm_units", "a2a_elems"):
+        assert low[k] == full[k]
+
+
+@pytest.mark.parametrize("f,P", [([1433, 128, 7], 1), ([602, 128, 41], 4), ([100, 256, 256, 47], 8)])
+def test_low_memory_never_larger(f, P):
+    """Sharing only ever removes allocations, for every configuration."""
+    L = len(f) - 1
+    for cid in range(4 ** L):
+        a, _ = rdm.plan_info(f, cid, P, 10007)
+        b, _ = rdm.plan_info(f, cid, P, 10007, low_memory=True)
+        assert 0 < b["workspace_bytes"] <= a["workspace_bytes"]
+
+
+def test_feature_row_slices_match_whole_draw():
+    """synth.features_rows / labels_rows (one rank's slice of a matrix too large
+    to draw whole on the host) equal the corresponding rows of the whole draw."""
+    import synth
+    H = synth.features(3001, 17)
+    assert np.array_equal(H[1234:2999], synth.features_rows(1234, 2999, 17))
+    y = synth.labels(3001, 41)
+    assert np.array_equal(y[7:3001], synth.labels_rows(7, 3001, 41))

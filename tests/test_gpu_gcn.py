@@ -401,3 +401,116 @@ def test_reddit_full_size_fast_variant(rdm):
     assert og.max_rel_err(dW[1], H1.astype(np.float64).T @ S2) < 2e-2
     G1 = (S2 @ Ws[1].astype(np.float64).T) * (H1 > 0)
     assert og.max_rel_err(dW[0], H0.astype(np.float64).T @ og.spmm(g, G1)) < 2e-2
+
+
+@pytest.mark.parametrize("P", [1, 4])
+def test_low_memory_epoch_bitwise(rdm, cora, P):
+    """RDM_GCN_LOW_MEMORY (liveness-based buffer sharing) changes no result:
+    loss, every Y^l and G^0 bit-identical to the default workspace, for every
+    configuration; a tensor whose memory a later step reuses is refused."""
+    import torch
+    g, H0, Ws, y, m, _ = cora
+    f = [Ws[0].shape[0]] + [w.shape[1] for w in Ws]
+    dev = torch.device("cuda:0")
+    saw_refusal = False
+    for cfg in range(16):
+        outs = []
+        for low in (False, True):
+            ctx = rdm.Context(device=0) if P == 1 else rdm.Context(rank=rdm.ALL_RANKS, world=P, device=0)
+            ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
+            model = rdm.GCN(ctx, f, cfg, low_memory=low)
+            Hs, ys, ms = [], [], []
+            for p in range(P):
+                lo, hi, _ = rdm.partition(P, rdm.ROW, g.n, f[0], p)
+                Hs.append(torch.from_numpy(np.ascontiguousarray(H0[lo:hi])).to(dev))
+                ys.append(torch.from_numpy(y[lo:hi]).to(dev))
+                ms.append(torch.from_numpy(m[lo:hi]).to(dev))
+            model.set_input(Hs, ys, ms)
+            Wd = [torch.from_numpy(w.copy()).to(dev) for w in Ws]
+            dW = [torch.zeros_like(w) for w in Wd]
+            loss = torch.zeros(1, dtype=torch.float64, device=dev)
+            for _ in range(2):
+                model.forward(Wd, loss)
+                model.backward(Wd, dW)
+            ctx.sync()
+            G0 = _gather(model, rdm, rdm.T_G, 0, g.n, f[0], P)
+            info = model.info()
+            if low:
+                for which, layer in ((rdm.T_H, 1), (rdm.T_Z, 0)):
+                    for lay in (rdm.ROW, rdm.COL):
+                        try:
+                            model.tensor_torch(which, layer, 0, lay)
+                        except rdm.RdmError:
+                            saw_refusal = True
+            outs.append((loss.item(), [d.cpu().numpy() for d in dW], G0, info["workspace_bytes"]))
+            model.close()
+            ctx.close()
+        (l0, d0, g0, w0), (l1, d1, g1, w1) = outs
+        assert l0 == l1, cfg
+        for a, b in zip(d0, d1):
+            assert np.array_equal(a, b), cfg
+        assert np.array_equal(g0, g1), cfg
+        assert w1 <= w0
+    assert saw_refusal
+
+
+def test_emulated_rank(rdm, cora):
+    """rdm_init_emulated: rank p of P with no peers.  Its local operators are
+    the ordinary kernels (rdm_spmm on a column slice of width w_p and rdm_gemm
+    on a row slice equal a plain context's bit for bit); an epoch runs at the
+    P-rank shapes and counts exactly the rank's share of the redistribution
+    traffic (its sends to q != p per rdm_redist_plan); P2P is refused."""
+    import torch
+    g, H0, Ws, y, m, _ = cora
+    f = [Ws[0].shape[0]] + [w.shape[1] for w in Ws]
+    P, p, cfg = 4, 2, 10
+    dev = torch.device("cuda:0")
+    plain = rdm.Context(device=0)
+    plain.set_graph(g.rowptr, g.col, g.val, symmetric=True)
+    em = rdm.Context(rank=p, world=P, device=0, emulate=True)
+    em.set_graph(g.rowptr, g.col, g.val, symmetric=True)
+    with pytest.raises(rdm.RdmError):
+        em.set_transport("p2p")
+    c0, c1, ldc = rdm.partition(P, rdm.COL, g.n, 128, p)
+    X = torch.zeros(g.n, ldc, device=dev)
+    X[:, :c1 - c0] = torch.from_numpy(synth.features(g.n, c1 - c0, seed=9)).to(dev)
+    outs = []
+    for ctx in (plain, em):
+        out = torch.zeros_like(X)
+        ctx.spmm(1, X, out, c1 - c0)
+        ctx.sync()
+        outs.append(out.cpu().numpy())
+    assert np.array_equal(outs[0], outs[1])
+    lo, hi, _ = rdm.partition(P, rdm.ROW, g.n, f[0], p)
+    Hr = torch.from_numpy(np.ascontiguousarray(H0[lo:hi])).to(dev)
+    W1 = torch.from_numpy(Ws[0].copy()).to(dev)
+    outs = []
+    for ctx in (plain, em):
+        C = torch.zeros(hi - lo, f[1], device=dev)
+        ctx.gemm(rdm.GEMM_NN, Hr, W1, C, hi - lo, f[0], f[1])
+        ctx.sync()
+        outs.append(C.cpu().numpy())
+    assert np.array_equal(outs[0], outs[1])
+    # one emulated epoch at the P-rank shapes
+    me = rdm.GCN(em, f, cfg)
+    me.set_input([Hr], [torch.from_numpy(y[lo:hi]).to(dev)], [torch.from_numpy(m[lo:hi]).to(dev)])
+    Wd = [torch.from_numpy(w.copy()).to(dev) for w in Ws]
+    dW = [torch.zeros_like(w) for w in Wd]
+    loss = torch.zeros(1, dtype=torch.float64, device=dev)
+    em.reset_counters()
+    me.forward(Wd, loss)
+    me.backward(Wd, dW)
+    em.sync()
+    cnt = em.counters()
+    _, desc = rdm.plan_info(f, cfg, P, g.n)
+    want = 0
+    for line in desc.splitlines():
+        if line.strip().startswith("A2A"):
+            w = int(line.split("f=")[1].split()[0])
+            fr = rdm.ROW if ".row ->" in line else rdm.COL
+            pl = rdm.redist_plan(P, p, fr, g.n, w)
+            want += 4 * sum(pl["send_elems"][q] for q in range(P) if q != p)
+    assert cnt["a2a_bytes_wire"] == want, (cnt["a2a_bytes_wire"], want)
+    me.close()
+    em.close()
+    plain.close()

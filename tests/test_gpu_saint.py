@@ -190,3 +190,42 @@ def test_saint_core_spmm_matches_oracle(rdm, monkeypatch):
         assert og.max_rel_err(Z, ref.Z[len(Ws)]) < 1e-4
     model.close()
     s.close()
+
+
+@pytest.mark.slow
+def test_saint_config4_full_size_sampled(rdm):
+    """BASELINE configs[3] at full size in bench.py --saint's launch
+    configuration (Reddit-shaped graph, 8,000 roots, walks of 4, 602/256/41,
+    P = 1, model-picked config, hub cores on), against the oracle's own
+    sampler and induced subgraph: forward rows on 4,096 sampled vertices from the
+    GPU's own previous layer, the loss from the GPU's logits, and both weight
+    gradients recomputed in fp64 through the whole backward of the subgraph."""
+    wl = synth.WORKLOADS["reddit"]
+    g = synth.make_graph(wl)
+    f = (wl.f[0], 256, wl.f[-1])
+    H0 = synth.features(wl.n, f[0])
+    Ws = synth.weights(f)
+    y = synth.labels(wl.n, f[-1])
+    m = synth.train_mask(wl.n)
+    roots, h, seed = 8000, 4, 1
+    nodes0, rp0, cs0, _ = osaint.sample(g, roots, h, seed, 0)
+    _, cfg, _, _ = rdm.select_config(list(f), len(nodes0), len(cs0), 1)
+    rng = np.random.default_rng(3)
+    for it, loss, dW, W_now, model in _saint_run(rdm, g, H0, Ws, y, m, cfg, 1, roots, h, seed, 2):
+        nodes, rp, cs, vs = osaint.sample(g, roots, h, seed, it)
+        sub = synth.CSR(len(nodes), rp, cs, vs)
+        n = len(nodes)
+        rows = np.sort(rng.choice(n, size=min(4096, n), replace=False))
+        X0 = H0[nodes]
+        H1 = model.tensor_torch(rdm.T_H, 1).cpu().numpy()
+        Z = model.tensor_torch(rdm.T_Z, 0).cpu().numpy()
+        assert H1.shape == (n, f[1]) and Z.shape == (n, f[2])
+        ref1 = np.maximum(og.spmm_rows(sub, X0, rows) @ W_now[0].astype(np.float64), 0)
+        assert og.max_rel_err(H1[rows], ref1) < 1e-4, (it, "H1")
+        assert og.max_rel_err(Z[rows], og.spmm_rows(sub, H1, rows) @ W_now[1].astype(np.float64)) < 1e-4
+        lref, GL = og.softmax_xent(Z, y[nodes], m[nodes])
+        assert abs(loss - lref) <= 1e-5 * abs(lref), (it, loss, lref)
+        S2 = og.spmm(sub, GL)
+        assert og.max_rel_err(dW[1], H1.astype(np.float64).T @ S2) < 1e-4, (it, "Y2")
+        G1 = (S2 @ W_now[1].astype(np.float64).T) * (H1 > 0)
+        assert og.max_rel_err(dW[0], X0.astype(np.float64).T @ og.spmm(sub, G1)) < 1e-4, (it, "Y1")

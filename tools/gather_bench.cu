@@ -140,11 +140,15 @@ int main(int argc, char** argv) {
           case 64: ms = run<16, 1, 4>(tab, ld4, idx, m, sink, grid); break;
           case 128: ms = run<32, 1, 4>(tab, ld4, idx, m, sink, grid); break;
         }
+        float ms2 = 0;   // the fp32 SpMM's own lane mapping for 512 B rows (G = 8, V = 4)
+        if (rf == 128) ms2 = run<8, 4, 1>(tab, ld4, idx, m, sink, grid);
         const double gbs = m * row_b / (ms * 1e-3) / 1e9;
         printf("{\"row_bytes\": %d, \"table_mb\": %.0f, \"dist\": \"%s\", \"rows\": %lld, "
-               "\"ms\": %.4f, \"delivered_gbs\": %.1f, \"bytes_per_clk\": %.1f, \"index_gbs\": %.1f}\n",
+               "\"ms\": %.4f, \"delivered_gbs\": %.1f, \"bytes_per_clk\": %.1f, \"index_gbs\": %.1f, "
+               "\"spmm_mapping_g8v4_gbs\": %.1f}\n",
                (int)row_b, tmb, dist ? "powerlaw" : "uniform", m, ms, gbs,
-               gbs * 1e9 / (clk * 1e3), m * 4.0 / (ms * 1e-3) / 1e9);
+               gbs * 1e9 / (clk * 1e3), m * 4.0 / (ms * 1e-3) / 1e9,
+               ms2 > 0 ? m * row_b / (ms2 * 1e-3) / 1e9 : 0.0);
         fflush(stdout);
       }
     }
