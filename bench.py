@@ -131,6 +131,15 @@ class ClockSampler:
 
 
 # --------------------------------------------------------------- oracle leg
+def graph_desc(wl):
+    """The input recipe of a workload's graph."""
+    g = "R-MAT (0.57,0.19,0.19,0.05)" if wl.graph == "rmat" else "uniform (Erdos-Renyi)"
+    g += ", permuted" if wl.permute else ", un-permuted (R-MAT order)"
+    v = {"sym": "D^-1/2 (A+I) D^-1/2", "row": "D^-1 (A+I) (not symmetric)",
+         "noise": "D^-1/2 (A+I) D^-1/2 x (1 + u_ij/16), u symmetric (not a rank-1 scaling)"}[wl.values]
+    return g + ", symmetric pattern, self loops, " + v
+
+
 def host_cpu_info():
     """lscpu model / sockets / cores of the host the oracle runs on."""
     info = {"nproc": os.cpu_count()}
@@ -361,7 +370,8 @@ def saint_main(a, world, rank, local_rank):
                        "l2": "CSR of the full graph streamed by the sampler each step (0.92 GB)"},
             "clocks": clocks,
             "step_ms": {"median": float(np.median(step_ms)), "min": float(np.min(step_ms)),
-                        "max": float(np.max(step_ms)), "p90": float(np.percentile(step_ms, 90))},
+                        "max": float(np.max(step_ms)), "p90": float(np.percentile(step_ms, 90)),
+                        "all": [round(float(x), 3) for x in step_ms]},
             "e2e": {"value": e_ms, "unit": "ms", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 8,
                     "note": "wall clock of the public-API loop; features resident on the device, "
                             "the per-step input is the sampler seed"},
@@ -419,7 +429,7 @@ def emulate_main(a):
     ctx = rdm.Context(rank=p, world=P, device=0, stream=stream, emulate=True)
     ctx.set_precision(a.precision)
     t0 = time.time()
-    ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
+    ctx.set_graph(g.rowptr, g.col, g.val, symmetric=synth.symmetric_values(wl))
     t_set = time.time() - t0
     ginfo = ctx.graph_info()
     pareto, chosen, _, _ = rdm.select_config(list(wl.f), wl.n, wl.nnz, P)
@@ -626,12 +636,18 @@ def main():
                       unique_id=uid)
     ctx.set_transport(a.transport)
     ctx.set_precision(a.precision)
+    comm = None
+    if world > 1:
+        comm = ctx.comm_info()
+        print(f"[bench] rank {rank}/{world}: NCCL {comm['nccl_version']} communicator of "
+              f"{comm['ranks']} ranks, user rank {comm['rank']}, CUDA device {comm['device']}",
+              file=sys.stderr, flush=True)
     panels = 0 < a.ra < world
     if panels:   # §III-E: R_A copies of A, row panels; tiles + column-group broadcasts
         ctx.set_graph_panels(a.ra, g.rowptr, g.col, g.val)
         pareto, chosen, _, _ = rdm.select_config_ra(list(wl.f), wl.n, wl.nnz, world, a.ra)
     else:
-        ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
+        ctx.set_graph(g.rowptr, g.col, g.val, symmetric=synth.symmetric_values(wl))
         pareto, chosen, comm_u, sparse_u = rdm.select_config(list(wl.f), wl.n, wl.nnz, world)
     lo, hi, _ = rdm.partition(world, rdm.ROW, wl.n, wl.f[0], rank if world > 1 else 0)
     H0_pin = torch.from_numpy(H0[lo:hi]).pin_memory()
@@ -823,8 +839,7 @@ def main():
             "config": {
                 "workload": wl.name, "model": f"GCN {wl.L}L f={'/'.join(map(str, wl.f))}",
                 "precision": a.precision, "parity_gate": GATES[a.precision],
-                "n": n, "nnz": nnz, "graph": "R-MAT (0.57,0.19,0.19,0.05), permuted, symmetric, "
-                "self loops, D^-1/2 (A+I) D^-1/2", "global_batch": n, "seq_len": None,
+                "n": n, "nnz": nnz, "graph": graph_desc(wl), "global_batch": n, "seq_len": None,
                 "parallelism": f"rdm{world} (A replicated, H row/col redistributed)",
                 "transport": a.transport, "replicas_of_A": a.ra if panels else world,
                 "config_id": cfg_id, "config_name": rdm.config_name(model.cfg),
@@ -841,7 +856,7 @@ def main():
             "spmm_hbm_gbs": achieved, "a2a_bus_gbs": a2a_bus,
             "a2a_bytes_per_step": cnt["a2a_bytes_wire"] / a.steps,
             "bcast_elems_per_step": cnt["bcast_elems"] / a.steps,
-            "loss": loss_main, "variants": variants,
+            "loss": loss_main, "variants": variants, "nccl": comm,
         }
         print(json.dumps(line), flush=True)
     ctx.sync()

@@ -188,6 +188,12 @@ rdm_status rdm_init(rdm_ctx** ctx, int rank, int world, const void* nccl_unique_
  * (RDM_ERR_UNSUPPORTED).  Errors: RDM_ERR_ARG (world < 2, rank), RDM_ERR_CUDA. */
 rdm_status rdm_init_emulated(rdm_ctx** ctx, int rank, int world, int device, void* cuda_stream);
 int rdm_is_emulated(const rdm_ctx* ctx);
+/* The NCCL communicator behind the ctx (one rank of an NCCL job): NCCL
+ * version code, ncclCommCount, ncclCommUserRank, ncclCommCuDevice.  Without a
+ * communicator (world 1, virtual group, emulated rank) comm_ranks = 0 and
+ * comm_rank = comm_device = -1.  Any output pointer may be NULL. */
+rdm_status rdm_comm_info(rdm_ctx* ctx, int* nccl_version, int* comm_ranks, int* comm_rank,
+                         int* comm_device);
 rdm_status rdm_finalize(rdm_ctx* ctx);
 const char* rdm_last_error(const rdm_ctx* ctx);
 /* Block until the ctx's stream is idle; surfaces asynchronous CUDA/NCCL faults. */
@@ -260,12 +266,16 @@ rdm_status rdm_set_graph(rdm_ctx* ctx, int64_t n, int64_t nnz, const int64_t* ro
  * high-degree vertices, the "hub core": the K x K block A[hubs, hubs] (K a
  * multiple of 128, core_nnz entries) held dense and multiplied on the tensor
  * cores, the other entries in a residual CSR (core_K = 0: no core).
- * When every value of the hub region factors as a_ij = s_i s_j (the GCN
- * normalization D^-1/2 (A+I) D^-1/2, or all ones; checked entry by entry to
- * 2^-21 relative) the core is instead a set of "binary hub tiles": the
- * tile_ranks highest-degree vertices' block cut into 128 x 128 rank blocks,
- * the n_tiles blocks dense enough to pay stored as 0/1 and multiplied on the
- * tensor cores against s ⊙ X (core_K = 0, core_nnz = entries moved). */
+ * When every value of the hub region factors as a_ij = r_i c_j (a rank-1
+ * scaling of the 0/1 pattern: the GCN normalization D^-1/2 (A+I) D^-1/2, the
+ * row-normalized D^-1 (A+I), all ones, …; r and c found by a walk over the
+ * moved entries and checked entry by entry to 2^-21 relative) the core is
+ * instead a set of "binary hub tiles": the tile_ranks highest-degree
+ * vertices' block cut into 128 x 128 rank blocks, the n_tiles blocks dense
+ * enough to pay stored as bits and multiplied on the tensor cores against
+ * c ⊙ X (three int8 digits of a per-column 23-bit fixed point on kind::i8 by
+ * default), r applied in the residual SpMM's epilogue (core_K = 0,
+ * core_nnz = entries moved). */
 typedef struct {
   int64_t n, nnz;
   int64_t n_light_rows, n_heavy_rows, n_segments, max_degree;

@@ -53,7 +53,7 @@ EXPORTS = [
     "rdm_set_transport", "rdm_get_transport", "rdm_debug_disable_tc",
     "rdm_set_precision", "rdm_get_precision", "rdm_set_graph_panels", "rdm_partition_tile",
     "rdm_redistribute_panels", "rdm_spmm_panels", "rdm_max_replication", "rdm_select_config_ra",
-    "rdm_saint_wait", "rdm_init_emulated", "rdm_is_emulated",
+    "rdm_saint_wait", "rdm_init_emulated", "rdm_is_emulated", "rdm_comm_info",
 ]
 
 
@@ -95,6 +95,8 @@ _sig = {
     "rdm_partition": [_int, _int, _i64, _i64, _int, _pi64, _pi64, _pi64],
     "rdm_set_graph": [_vp, _i64, _i64, _vp, _vp, _vp, _int, _int],
     "rdm_init_emulated": [ctypes.POINTER(_vp), _int, _int, _int, _vp],
+    "rdm_comm_info": [_vp, ctypes.POINTER(_int), ctypes.POINTER(_int), ctypes.POINTER(_int),
+                      ctypes.POINTER(_int)],
     "rdm_spmm": [_vp, _int, _vp, _i64, _vp, _i64, _i64, _int, _vp, _vp, _i64],
     "rdm_gemm": [_vp, _int, _vp, _i64, _vp, _i64, _vp, _i64, _i64, _i64, _i64, _int, _vp, _vp],
     "rdm_redistribute": [_vp, _int, _pp, _pp, _i64, _i64],
@@ -336,6 +338,13 @@ class Context:
 
     def sync(self):
         self._c(_lib.rdm_sync(self.h))
+
+    def comm_info(self) -> dict:
+        """NCCL version and the communicator's rank count / rank / device (rdm_comm_info)."""
+        v, n, r, d = _int(), _int(), _int(), _int()
+        self._c(_lib.rdm_comm_info(self.h, ctypes.byref(v), ctypes.byref(n), ctypes.byref(r),
+                                   ctypes.byref(d)))
+        return {"nccl_version": v.value, "ranks": n.value, "rank": r.value, "device": d.value}
 
     def set_graph(self, rowptr, col, val, symmetric=True):
         """CSR from numpy (host) or torch (device) arrays: int64 rowptr, int32 col, fp32 val."""

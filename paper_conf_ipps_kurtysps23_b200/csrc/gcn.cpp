@@ -252,7 +252,8 @@ struct Buf {
 // epoch).  H^0 row (the input) lives throughout; the operands of the
 // weight-gradient GEMMs run on a side stream joined at the end of the
 // backward pass, so they live to kEnd; a redistribution's destination may be
-// written by its producer one step earlier (fused P2P transport).
+// written by its producer one step earlier (fused P2P transport).  H^0's
+// column slices, when read, are an input like its row slice: pinned.
 // RDM_GCN_LOW_MEMORY: buffers of the same shape whose lifetimes do not
 // overlap share one allocation (first-fit, largest first) — same shape, so the
 // zero ld-padding every producer keeps stays zero.
@@ -338,6 +339,13 @@ std::vector<BufPlan> buffer_lifetimes(const Planner& pl, const std::vector<Step>
       }
       ++t;
     }
+  // H^0's column slices (when the plan reads them) are an input too: written by
+  // set_input before the epoch and read again by the next epoch
+  auto h0c = m.find(std::make_pair(Key{K_H, 0}.id(), lay(RDM_COL)));
+  if (h0c != m.end()) {
+    h0c->second.first = -1;
+    h0c->second.last = kEnd;
+  }
   std::vector<BufPlan> out;
   for (auto& kv : m) out.push_back(kv.second);
   return out;

@@ -516,6 +516,266 @@ __global__ void tile_panels_f16_kernel(const float* __restrict__ X, int64_t ldx,
   }
 }
 
+// ---------------------------------------------------------------- int8 tiles
+// kind::i8 form (default for fp32).  y = s_k · X[hub_k][n] · 2^-e_n with the
+// column maximum scaled into [2^21, 2^22) is rounded to an integer v
+// (|v| ≤ 2^22: 23 significant bits relative to the column maximum) and split
+// into three signed 8-bit digits v = d2·2^16 + d1·2^8 + d0 (d ∈ [-128, 127]).
+// The 0/1 tile is exact in int8, the MMAs accumulate in s32 exactly, so each
+// output is Σ_j b_ij v_j computed exactly and rounded to fp32 once, ×2^e_n.
+// Against the fp16 pair: the bit expansion is 2 integer ops per 4 elements
+// (the nibble times 0x204081 spreads 4 bits over 4 bytes) instead of a table
+// lookup per 8 bf16, the A operand is half the TMEM bytes, and the int8 MMA
+// rate is twice the fp16 one (3 digits cost 1.5 fp16 MMAs, the pair 2).
+constexpr int I8_NMAX = 64;                 // output columns per pass (3 digits → N ≤ 192)
+
+__host__ __device__ constexpr uint32_t idesc_i8(int N) {
+  // D s32 (2), A / B signed 8-bit (1), K-major both, M = 128
+  return (2u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+}
+
+__device__ __forceinline__ void tc_mma_i8_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t idesc,
+                                             uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::i8 [%0], [%1], %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "r"(tmem_a), "l"(db), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+
+// One stage = one whole tile: B digits [3][n_mma][128 B] (128-byte swizzle,
+// one 3-D TMA), then the tile's bits [half][128 rows] u64.
+__global__ void __launch_bounds__(384, 1)
+hub_tile_i8_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __restrict__ bits,
+                   const int32_t* __restrict__ tile_cb, const int32_t* __restrict__ item_tb,
+                   float* __restrict__ part, const TileShape sh) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  const int S = sh.S, SA = sh.SA, n_mma = sh.n_mma;
+  uint64_t* full = (uint64_t*)(smem + S * sh.stage_bytes);
+  uint64_t* empty = full + S;
+  uint64_t* conv = empty + S;
+  uint64_t* aempty = conv + SA;
+  uint64_t* tfull = aempty + SA;
+  uint64_t* tempty = tfull + 2;
+  uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int total = sh.n_items * sh.tiles_n;
+  const int bbytes = 3 * n_mma * 128;
+  auto B_st = [&](int s) { return smem + s * sh.stage_bytes; };
+  auto bits_st = [&](int s) { return smem + s * sh.stage_bytes + bbytes; };
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&empty[i], 1);
+    }
+    for (int i = 0; i < SA; ++i) {
+      mbar_init(&conv[i], 128);
+      mbar_init(&aempty[i], 1);
+    }
+    for (int b = 0; b < 2; ++b) {
+      mbar_init(&tfull[b], 1);
+      mbar_init(&tempty[b], 128);
+    }
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 2) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(tmem_slot)),
+                 "n"(512));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+  const uint32_t kAcol = 2 * sh.acc_cols;
+
+  if (warp == 0) {
+    if (lane == 0) {
+      int s = 0;
+      uint32_t ph = 0, kc = 0;
+      const uint32_t bytes = (uint32_t)bbytes + 2048;
+      for (int t = blockIdx.x; t < total; t += gridDim.x) {
+        const int item = t / sh.tiles_n;
+        const int n0 = (t % sh.tiles_n) * n_mma;
+        const int tb = item_tb[item], T = item_tb[item + 1] - tb;
+        int ti = (int)(((unsigned)item * 2654435761u) % (unsigned)max(T, 1));
+        for (int i = 0; i < T; ++i) {
+          const int tile = tb + ti;
+          if (++ti == T) ti = 0;
+          if (kc >= (uint32_t)S) mbar_wait(&empty[s], ph ^ 1);
+          mbar_expect_tx(&full[s], bytes);
+          bulk_load(bits_st(s), bits + (int64_t)tile * 2 * TK, 2048, &full[s]);
+          tma_load_4d(B_st(s), &tmB, &full[s], 0, n0, 0, tile_cb[tile]);
+          ++kc;
+          if (++s == S) { s = 0; ph ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      const uint32_t idesc = idesc_i8(3 * n_mma);
+      const uint64_t bd0 = sdesc(smem_u32(B_st(0)), 16, 1024);
+      const uint32_t st16 = (uint32_t)sh.stage_bytes >> 4;
+      int s = 0, a = 0;
+      uint32_t ph = 0, aph = 0;
+      int it = 0;
+      for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
+        const int item = t / sh.tiles_n;
+        const int nst = item_tb[item + 1] - item_tb[item];
+        const int acc = it & 1;
+        if (it >= 2) mbar_wait(&tempty[acc], ((it >> 1) - 1) & 1);
+        tc_fence_after();
+        const uint32_t d_tmem = tmem_base + acc * sh.acc_cols;
+        for (int st = 0; st < nst; ++st) {
+          mbar_wait(&conv[a], aph);
+          tc_fence_after();
+          const uint32_t ta = tmem_base + kAcol + a * 32;
+          const uint64_t bd = bd0 + (uint64_t)(s * st16);
+          if (!(sh.dbg & 1)) {
+#pragma unroll
+            for (int j = 0; j < TK / 32; ++j)   // K = 32 int8 per MMA: 8 A columns, 32 B of B rows
+              tc_mma_i8_ts(d_tmem, ta + j * 8, bd + 2 * j, idesc, (st | j) ? 1u : 0u);
+          }
+          tc_commit(&empty[s]);
+          tc_commit(&aempty[a]);
+          if (++s == S) { s = 0; ph ^= 1; }
+          if (++a == SA) { a = 0; aph ^= 1; }
+        }
+        tc_commit(&tfull[acc]);
+      }
+    }
+  } else if (warp >= 4 && warp < 8) {
+    // expander: row r's 128 bits → 128 int8 0 / 1, four per 32-bit TMEM column
+    const int r = threadIdx.x - 128;
+    const uint32_t lane_off = (uint32_t)((warp & 3) * 32) << 16;
+    int s = 0, a = 0;
+    uint32_t ph = 0, aph = 0, kc = 0;
+    for (int t = blockIdx.x; t < total; t += gridDim.x) {
+      const int item = t / sh.tiles_n;
+      const int nst = item_tb[item + 1] - item_tb[item];
+      for (int st = 0; st < nst; ++st, ++kc) {
+        mbar_wait(&full[s], ph);
+        if (kc >= (uint32_t)SA) {
+          mbar_wait(&aempty[a], aph ^ 1);
+          tc_fence_after();
+        }
+        const uint32_t bs = smem_u32(bits_st(s)) + r * 8;
+        const uint2 h0 = lds64(bs), h1 = lds64(bs + 1024);
+        const uint32_t w4[4] = {h0.x, h0.y, h1.x, h1.y};
+        uint32_t v[32];
+#pragma unroll
+        for (int i = 0; i < 32; ++i) v[i] = (((w4[i >> 3] >> (4 * (i & 7))) & 15u) * 0x204081u) & 0x01010101u;
+        tmem_st32u(tmem_base + lane_off + kAcol + a * 32, v);
+        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+        tc_fence_before();
+        mbar_arrive(&conv[a]);
+        if (++s == S) { s = 0; ph ^= 1; }
+        if (++a == SA) { a = 0; aph ^= 1; }
+      }
+    }
+  } else if (warp >= 8) {
+    const int q = warp & 3;
+    int it = 0;
+    for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
+      const int item = t / sh.tiles_n;
+      const int64_t n0 = (int64_t)(t % sh.tiles_n) * n_mma;
+      const int acc = it & 1;
+      mbar_wait_sleep(&tfull[acc], (it >> 1) & 1);
+      tc_fence_after();
+      float* prow = part + ((int64_t)item * TK + q * 32 + lane) * sh.ldp + n0;
+      for (int c0 = 0; c0 < n_mma; c0 += 32) {
+        if (n0 + c0 >= sh.w) break;
+        uint32_t d2[32], d1[32], d0[32];
+        const uint32_t a0 = tmem_base + acc * sh.acc_cols + ((uint32_t)(q * 32) << 16) + (uint32_t)c0;
+        tmem_ld32(a0, d2);
+        tmem_ld32(a0 + (uint32_t)n_mma, d1);
+        tmem_ld32(a0 + (uint32_t)(2 * n_mma), d0);
+#pragma unroll
+        for (int i = 0; i < 32; i += 4)
+          if (n0 + c0 + i < sh.w) {
+            const float4 cs = __ldg(reinterpret_cast<const float4*>(sh.colscale + n0 + c0 + i));
+            float o[4];
+#pragma unroll
+            for (int u = 0; u < 4; ++u) {
+              const long long v = (long long)(int)d2[i + u] * 65536 + (long long)(int)d1[i + u] * 256 +
+                                  (long long)(int)d0[i + u];
+              o[u] = __ll2float_rn(v);
+            }
+            *reinterpret_cast<float4*>(prow + c0 + i) = make_float4(o[0] * cs.x, o[1] * cs.y, o[2] * cs.z, o[3] * cs.w);
+          }
+      }
+      tc_fence_before();
+      mbar_arrive(&tempty[acc]);
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "n"(512));
+  }
+}
+
+// int8 digit panels P_d[n][k] (row length K2 bytes; d = 0: 2^16 digit, 1: 2^8,
+// 2: 2^0) of y = s_k · X[hub_k][n] · 2^-e_n, e_n = ilogb(colmax_n) − 21;
+// colscale[n] = 2^e_n.  Block: 128 k x 32 n, each thread 4 consecutive k.
+__global__ void tile_panels_i8_kernel(const float* __restrict__ X, int64_t ldx, const int32_t* __restrict__ hub_ids,
+                                      const float* __restrict__ scale, int64_t K2, int64_t w,
+                                      const unsigned int* __restrict__ colmax, int8_t* __restrict__ pan,
+                                      float* __restrict__ colscale) {
+  __shared__ float t[128][33];
+  __shared__ float inv[32];
+  const int64_t k0 = (int64_t)blockIdx.x * 128, n0 = (int64_t)blockIdx.y * 32;
+  if (threadIdx.y == 0) {
+    const int64_t n = n0 + threadIdx.x;
+    const float mx = n < w ? __uint_as_float(colmax[n]) : 0.f;
+    const int e = mx > 0.f ? ilogbf(mx) - 21 : 0;
+    inv[threadIdx.x] = ldexpf(1.f, -e);
+    if (blockIdx.x == 0 && n < w) colscale[n] = ldexpf(1.f, e);
+  }
+  {
+    const int64_t n = n0 + threadIdx.x;
+#pragma unroll
+    for (int h = 0; h < 2; ++h) {
+      int32_t id[8];
+      float sc[8], x[8];
+#pragma unroll
+      for (int u = 0; u < 8; ++u) {
+        const int64_t k = k0 + threadIdx.y + 8 * u + 64 * h;
+        id[u] = __ldg(hub_ids + k);
+        sc[u] = __ldg(scale + k);
+      }
+#pragma unroll
+      for (int u = 0; u < 8; ++u) x[u] = (n < w) ? __ldg(X + (int64_t)id[u] * ldx + n) : 0.f;
+#pragma unroll
+      for (int u = 0; u < 8; ++u) t[threadIdx.y + 8 * u + 64 * h][threadIdx.x] = sc[u] * x[u];
+    }
+  }
+  __syncthreads();
+  for (int i = threadIdx.y; i < 32; i += 8) {
+    const int64_t n = n0 + i;
+    if (n >= w) break;
+    const int kk = 4 * threadIdx.x;
+    uint32_t q[3] = {0u, 0u, 0u};
+#pragma unroll
+    for (int u = 0; u < 4; ++u) {
+      const int v = __float2int_rn(t[kk + u][i] * inv[i]);     // |v| <= 2^22
+      const int e0 = ((v & 255) ^ 128) - 128;
+      const int v1 = (v - e0) >> 8;
+      const int e1 = ((v1 & 255) ^ 128) - 128;
+      const int e2 = (v1 - e1) >> 8;
+      q[0] |= (uint32_t)(e2 & 255) << (8 * u);
+      q[1] |= (uint32_t)(e1 & 255) << (8 * u);
+      q[2] |= (uint32_t)(e0 & 255) << (8 * u);
+    }
+    const int64_t o = n * K2 + k0 + kk;
+#pragma unroll
+    for (int d = 0; d < 3; ++d) *reinterpret_cast<uint32_t*>(pan + (int64_t)d * w * K2 + o) = q[d];
+  }
+}
+
 PFN_cuTensorMapEncodeTiled_v12000 encode() {
   static PFN_cuTensorMapEncodeTiled_v12000 fn = nullptr;
   if (!fn) {
@@ -545,6 +805,22 @@ CUtensorMap panel_map(const void* base, int64_t K2, int64_t w, int n_mma, int HS
   return m;
 }
 
+// 4-D int8 map over the three digit panels P_d[n][k] (row length K2 bytes,
+// panel d at d·w·K2): dims {128 (k within a tile = one 128-byte swizzle row),
+// n, digit, k / 128}, box {128, n_mma, 3, 1}: one TMA lands [digit][n_mma][128].
+CUtensorMap panel_map_i8(const void* base, int64_t K2, int64_t w, int n_mma) {
+  CUtensorMap m;
+  cuuint64_t dims[4] = {(cuuint64_t)TK, (cuuint64_t)w, 3, (cuuint64_t)(K2 / TK)};
+  cuuint64_t strides[3] = {(cuuint64_t)K2, (cuuint64_t)(w * K2), (cuuint64_t)TK};
+  cuuint32_t box[4] = {(cuuint32_t)TK, (cuuint32_t)n_mma, 3, 1};
+  cuuint32_t es[4] = {1, 1, 1, 1};
+  CUresult r = encode()(&m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 4, const_cast<void*>(base), dims, strides, box, es,
+                        CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
+                        CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS) throw Error(RDM_ERR_CUDA, "cuTensorMapEncodeTiled (int8 panels) failed (" + std::to_string((int)r) + ")");
+  return m;
+}
+
 CUtensorMap stacked_map(const void* base, int64_t K2, int64_t rows, int n_mma) {
   CUtensorMap m;
   cuuint64_t dims[2] = {(cuuint64_t)K2, (cuuint64_t)rows};
@@ -564,6 +840,8 @@ CUtensorMap stacked_map(const void* base, int64_t K2, int64_t rows, int n_mma) {
 // expansion + 3 bf16 MMA pieces per 128-wide chunk), plus ≈ 20 µs per call.
 double csr_entry_s(int64_t w) { return 24e-12 * std::pow((double)w / 128.0, 0.55); }
 double tile_s(int64_t w, int np = 3) {
+  if (np == kPiecesI8)   // int8 digits: 64-wide passes, cheap expansion (first estimate)
+    return (double)ceil_div(w, I8_NMAX) * (1.2e-9 + 2.0e-9 * (double)std::min<int64_t>(w, I8_NMAX) / I8_NMAX);
   return (double)ceil_div(w, 128) * (4.5e-9 + 5.2e-9 * np / 3.0 * (double)std::min<int64_t>(w, 128) / 128.0);
 }
 }  // namespace
@@ -574,8 +852,53 @@ bool hub_tiles_pay(const Core& c, int64_t w, int np) {
   return (double)c.nnz * csr_entry_s(w) > (double)c.n_tiles * tile_s(w, np) + 20e-6;
 }
 
+// int8 digits (np == kPiecesI8): column maxima, digit panels, hub_tile_i8_kernel.
+void hub_tiles_product_i8(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx, int64_t w, float* part,
+                          int64_t ldp) {
+  const int64_t K2 = c.K2;
+  int8_t* pan = reinterpret_cast<int8_t*>(ensure_ws(ctx->ws_core_b, (size_t)3 * w * K2));
+  const int64_t w4 = (w + 3) / 4 * 4;
+  float* cs = ensure_ws(ctx->ws_tile_cs, (size_t)2 * w4 * sizeof(float));
+  unsigned int* cmax = reinterpret_cast<unsigned int*>(cs + w4);
+  RDM_CUDA(cudaMemsetAsync(cmax, 0, w * sizeof(unsigned int), ctx->stream));
+  RDM_CUDA(cudaMemsetAsync(cs, 0, w4 * sizeof(float), ctx->stream));
+  dim3 mg((unsigned)ceil_div(K2, 256), (unsigned)ceil_div(w, 32));
+  tile_colmax_kernel<<<mg, dim3(32, 8), 0, ctx->stream>>>(X, ldx, c.hub_ids->as<int32_t>(), c.scale->as<float>(),
+                                                         K2, w, cmax);
+  RDM_LAUNCHED(ctx);
+  dim3 pg((unsigned)(K2 / TK), (unsigned)ceil_div(w, 32));
+  tile_panels_i8_kernel<<<pg, dim3(32, 8), 0, ctx->stream>>>(X, ldx, c.hub_ids->as<int32_t>(), c.scale->as<float>(),
+                                                           K2, w, cmax, pan, cs);
+  RDM_LAUNCHED(ctx);
+  TileShape sh{};
+  sh.n_mma = (int)std::min<int64_t>(I8_NMAX, ((w + 15) / 16) * 16);
+  sh.tiles_n = (int)ceil_div(w, sh.n_mma);
+  sh.n_items = (int)c.n_items;
+  sh.w = w;
+  sh.ldp = ldp;
+  sh.R = 1;
+  sh.HS = 1;
+  sh.acc_cols = (3 * sh.n_mma + 31) / 32 * 32;
+  sh.stage_bytes = (3 * sh.n_mma * 128 + 2048 + 1023) / 1024 * 1024;
+  const int avail = kSmemBudget - 1024 - 1024;
+  sh.S = std::min(32, avail / sh.stage_bytes);
+  sh.SA = std::min(8, (512 - 2 * sh.acc_cols) / 32);
+  sh.dbg = getenv("RDM_TILE_DBG") ? atoi(getenv("RDM_TILE_DBG")) : 0;
+  sh.colscale = cs;
+  RDM_CHECK_ARG(sh.S >= 2 && sh.SA >= 2, "hub tiles (int8): TMEM/smem budget");
+  const CUtensorMap tb = panel_map_i8(pan, K2, w, sh.n_mma);
+  const int smem = sh.S * sh.stage_bytes + 1024 + 1024;
+  const int64_t total = c.n_items * sh.tiles_n;
+  const unsigned grid = (unsigned)std::min<int64_t>(total, ctx->num_sms);
+  RDM_CUDA(cudaFuncSetAttribute(hub_tile_i8_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  hub_tile_i8_kernel<<<grid, 384, smem, ctx->stream>>>(tb, c.tiles->as<uint64_t>(), c.tile_cb->as<int32_t>(),
+                                                       c.item_tb->as<int32_t>(), part, sh);
+  RDM_LAUNCHED(ctx);
+}
+
 void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx, int64_t w, float* part,
                        int64_t ldp, int np) {
+  if (np == kPiecesI8) return hub_tiles_product_i8(ctx, c, X, ldx, w, part, ldp);
   RDM_CHECK_ARG(np >= 1 && np <= 3, "hub tiles: 1, 2 or 3 pieces");
   const int64_t K2 = c.K2;
   __nv_bfloat16* pan = reinterpret_cast<__nv_bfloat16*>(ensure_ws(ctx->ws_core_b, (size_t)np * w * K2 * 2));
@@ -691,25 +1014,118 @@ bool build_hub_tiles(rdm_ctx* ctx, Csr& A, const int64_t* rp, const int32_t* col
   const int64_t n_tiles = (int64_t)tile_cb.size();
   if (n_tiles == 0 || n_tiles > (int64_t)INT32_MAX / (TK * TK)) return false;
   if (!forced && (double)moved * csr_entry_s(128) < (double)n_tiles * tile_s(128) + 100e-6) return false;
-  // factorisation â_ij = s_i s_j on every moved entry: s = deg^-1/2 (GCN), else s = 1
-  std::vector<double> s(n);
-  bool ok = false;
-  for (int hyp = 0; hyp < 2 && !ok; ++hyp) {
-    for (int64_t i = 0; i < n; ++i) s[i] = hyp == 0 ? 1.0 / std::sqrt((double)(rp[i + 1] - rp[i])) : 1.0;
-    ok = true;
-    for (int64_t i = 0; i < n && ok; ++i) {
+  // factorisation â_ij = r_i · c_j on every moved entry (any rank-1 scaling of
+  // a 0/1 block: the symmetric GCN normalisation s_i s_j, the row-normalised
+  // D^-1 (A+I) (r = 1/deg, c = 1), unit values, …).  r and c are found by a
+  // walk over the moved entries (a row fixes the columns it reaches, a column
+  // fixes the rows that reach it; the pattern is symmetric), every component
+  // anchored at r = 1, then every moved entry is checked to 2^-21 relative.
+  std::vector<double> rs(K2, 0.0), cs(K2, 0.0);   // by rank
+  auto in_tile = [&](int64_t ri, int64_t rj) {
+    return rj < K2 && tile_id[(size_t)(ri / TK) * nrb + rj / TK] >= 0;
+  };
+  auto verify = [&]() {
+    for (int64_t i = 0; i < n; ++i) {
       const int64_t ri = rank[i];
       if (ri >= K2) continue;
       for (int64_t j = rp[i]; j < rp[i + 1]; ++j) {
         const int64_t rj = rank[col[j]];
-        if (rj >= K2 || tile_id[(size_t)(ri / TK) * nrb + rj / TK] < 0) continue;
-        const double f = s[i] * s[col[j]];
-        if (!(std::fabs((double)val[j] - f) <= std::ldexp(f, -21))) {
-          ok = false;
-          break;
+        if (!in_tile(ri, rj)) continue;
+        const double f = rs[ri] * cs[rj];
+        if (f == 0.0 || !(std::fabs((double)val[j] - f) <= std::ldexp(std::fabs(f), -21))) return false;
+      }
+    }
+    return true;
+  };
+  // closed forms first (exact factors): s s (GCN), 1/deg · 1 (row-normalised),
+  // 1 · 1/deg (column-normalised), 1 · 1
+  bool ok = false;
+  for (int hyp = 0; hyp < 4 && !ok; ++hyp) {
+    for (int64_t k = 0; k < K2; ++k) {
+      const double d = (double)(rp[order[k] + 1] - rp[order[k]]);
+      const double s = 1.0 / std::sqrt(d);
+      rs[k] = hyp == 0 ? s : hyp == 1 ? 1.0 / d : 1.0;
+      cs[k] = hyp == 0 ? s : hyp == 2 ? 1.0 / d : 1.0;
+    }
+    ok = verify();
+  }
+  if (!ok) {
+    // any other rank-1 scaling: a walk over the moved entries (a row fixes the
+    // columns it reaches, a column fixes the rows that reach it; the pattern is
+    // symmetric), each component anchored at r = 1, then two refinement sweeps
+    // (geometric means of the ratios: the walk's rounding errors grow with the
+    // path length) before the check
+    auto value = [&](int64_t i, int64_t j) -> double {   // a_ij (vertex ids), found in row i
+      const int32_t* b = col + rp[i];
+      const int32_t* e = col + rp[i + 1];
+      const int32_t* f = std::lower_bound(b, e, (int32_t)j);
+      return (f != e && *f == (int32_t)j) ? (double)val[f - col] : std::nan("");
+    };
+    std::fill(rs.begin(), rs.end(), 0.0);
+    std::fill(cs.begin(), cs.end(), 0.0);
+    std::vector<char> rset(K2, 0), cset(K2, 0);
+    std::vector<int64_t> queue;   // >= 0: row rank, < 0: -(column rank) - 1
+    ok = true;
+    for (int64_t root = 0; root < K2 && ok; ++root) {
+      if (rset[root]) continue;
+      rs[root] = 1.0;
+      rset[root] = 1;
+      queue.assign(1, root);
+      while (!queue.empty() && ok) {
+        const int64_t q = queue.back();
+        queue.pop_back();
+        if (q >= 0) {
+          const int64_t i = order[q];
+          for (int64_t j = rp[i]; j < rp[i + 1]; ++j) {
+            const int64_t rj = rank[col[j]];
+            if (!in_tile(q, rj) || cset[rj]) continue;
+            cs[rj] = (double)val[j] / rs[q];
+            cset[rj] = 1;
+            queue.push_back(-rj - 1);
+          }
+        } else {
+          const int64_t cj = -q - 1, v = order[cj];
+          for (int64_t k = rp[v]; k < rp[v + 1]; ++k) {
+            const int64_t rk = rank[col[k]];
+            if (rk >= K2 || rset[rk] || !in_tile(rk, cj)) continue;
+            const double a = value(col[k], v);
+            if (!(a == a) || a == 0.0 || cs[cj] == 0.0) { ok = false; break; }
+            rs[rk] = a / cs[cj];
+            rset[rk] = 1;
+            queue.push_back(rk);
+          }
         }
       }
     }
+    for (int sweep = 0; sweep < 2 && ok; ++sweep) {
+      std::vector<double> lr(K2, 0.0), lc(K2, 0.0);
+      std::vector<int64_t> nr(K2, 0), nc(K2, 0);
+      for (int64_t i = 0; i < n; ++i) {   // rows from the columns
+        const int64_t ri = rank[i];
+        if (ri >= K2) continue;
+        for (int64_t j = rp[i]; j < rp[i + 1]; ++j) {
+          const int64_t rj = rank[col[j]];
+          if (!in_tile(ri, rj) || val[j] <= 0.f || cs[rj] <= 0.0) continue;
+          lr[ri] += std::log((double)val[j] / cs[rj]);
+          nr[ri]++;
+        }
+      }
+      for (int64_t k = 0; k < K2; ++k)
+        if (nr[k]) rs[k] = std::exp(lr[k] / nr[k]);
+      for (int64_t i = 0; i < n; ++i) {   // columns from the rows
+        const int64_t ri = rank[i];
+        if (ri >= K2) continue;
+        for (int64_t j = rp[i]; j < rp[i + 1]; ++j) {
+          const int64_t rj = rank[col[j]];
+          if (!in_tile(ri, rj) || val[j] <= 0.f || rs[ri] <= 0.0) continue;
+          lc[rj] += std::log((double)val[j] / rs[ri]);
+          nc[rj]++;
+        }
+      }
+      for (int64_t k = 0; k < K2; ++k)
+        if (nc[k]) cs[k] = std::exp(lc[k] / nc[k]);
+    }
+    ok = ok && verify();
   }
   if (!ok) return false;
   Core& c = A.core;
@@ -777,8 +1193,11 @@ bool build_hub_tiles(rdm_ctx* ctx, Csr& A, const int64_t* rp, const int32_t* col
         ++o;
       }
   }
-  std::vector<float> sc(c.K2);
-  for (int64_t k = 0; k < c.K2; ++k) sc[k] = (float)s[order[k]];
+  std::vector<float> sc(c.K2), sr(c.K2);
+  for (int64_t k = 0; k < c.K2; ++k) {
+    sc[k] = (float)cs[k];   // column scale of hub slot k (panels)
+    sr[k] = (float)rs[k];   // row scale (the SpMM epilogue)
+  }
   std::vector<int32_t> slot(n);
   for (int64_t v = 0; v < n; ++v) slot[v] = rank[v] < c.K2 ? rank[v] : -1;
   auto up = [&](std::unique_ptr<DevBuf>& b, const void* p, size_t bytes) {
@@ -789,6 +1208,7 @@ bool build_hub_tiles(rdm_ctx* ctx, Csr& A, const int64_t* rp, const int32_t* col
   up(c.item_tb, item_tb.data(), item_tb.size() * 4);
   up(c.rb_item, rb_item.data(), rb_item.size() * 4);
   up(c.scale, sc.data(), sc.size() * 4);
+  up(c.rscale, sr.data(), sr.size() * 4);
   up(c.hub_ids, order.data(), c.K2 * 4);
   up(c.hub_slot, slot.data(), n * 4);
   c.resid.reset(new Csr());

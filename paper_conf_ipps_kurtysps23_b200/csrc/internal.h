@@ -137,7 +137,8 @@ struct Core {
   std::unique_ptr<DevBuf> tile_cb;     // int32[n_tiles]: column block of each tile
   std::unique_ptr<DevBuf> item_tb;     // int32[n_items+1]: tile range of each work item
   std::unique_ptr<DevBuf> rb_item;     // int32[n_rb+1]: item range of each row block
-  std::unique_ptr<DevBuf> scale;       // fp32[K2]: s of the vertex of slot k
+  std::unique_ptr<DevBuf> scale;       // fp32[K2]: column scale c of the vertex of slot k (a_ij = r_i c_j)
+  std::unique_ptr<DevBuf> rscale;      // fp32[K2]: row scale r of the vertex of slot k
 };
 
 struct Csr {
@@ -154,6 +155,10 @@ struct Csr {
   std::unique_ptr<DevBuf> heavy_rows;   // int32[n_heavy]
   std::unique_ptr<DevBuf> heavy_seg;    // int32[n_heavy+1]: segment range of heavy row
   Pinned bins_stage;                    // pinned staging of the bins' upload (build_bins)
+  // hot-row panel (spmm.cu build_hot): the hot_max most referenced columns
+  // encoded as -(rank+1) in a second column stream; hot_ids[rank] = vertex
+  int64_t hot_max = 0;
+  std::unique_ptr<DevBuf> col_hot, hot_ids;
   int64_t max_deg = 0;
   // every stored value factors as a_ij = s_i·s_j (GCN normalisation; checked
   // on the host at rdm_set_graph): fp32 s per row, used by the fast-precision
@@ -205,6 +210,7 @@ struct rdm_ctx {
   std::unique_ptr<rdm::DevBuf> ws_panel_in;                    // all-gathered N x w_j input per slot
   std::unique_ptr<rdm::DevBuf> ws_tile_cs;                     // fp16 hub tiles: column scales + maxima
   std::unique_ptr<rdm::DevBuf> ws_bf16;                        // RDM_PREC_FAST: bf16 copy of the SpMM input
+  std::unique_ptr<rdm::DevBuf> ws_hot;                         // hot-row panel of the SpMM input
   // phase timing
   bool timing = false;
   int cur_phase = RDM_PH_OTHER;
@@ -287,6 +293,9 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
 // ctx->stream from A.bins_stage; sync = false leaves the stream unsynchronised
 // (the caller guarantees the staging is not rewritten before the copy ran).
 void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, bool sync = true);
+// Hot-row panel of the CSR the SpMM streams (A itself, or its hub-core residual):
+// device-built reference counts, stable descending order, encoded column stream.
+void build_hot(rdm_ctx* ctx, Csr& A);
 
 // gemm.cu
 void gemm(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, int64_t ldw, float* C,
@@ -306,7 +315,9 @@ void build_core(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, const int32_t*
 // summed per row block and scaled by s_i in the SpMM epilogue.
 bool build_hub_tiles(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, const int32_t* col_host,
                      const float* val_host);
-// np = pieces of s⊙X: 2 fp16 (fp32-class default), 3 bf16 (RDM_TILE_PIECES=3) or 1 bf16 (RDM_PREC_FAST).
+// np = pieces of s⊙X: kPiecesI8 = three int8 digits on kind::i8 (fp32-class default), 2 fp16
+// (RDM_TILE_PIECES=2), 3 bf16 (RDM_TILE_PIECES=3) or 1 bf16 (RDM_PREC_FAST).
+constexpr int kPiecesI8 = 8;
 bool hub_tiles_pay(const Core& c, int64_t w, int np);
 void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx, int64_t w,
                        float* part, int64_t ldp, int np);

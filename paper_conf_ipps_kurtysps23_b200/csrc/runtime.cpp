@@ -449,6 +449,17 @@ static void set_graph(rdm_ctx* ctx, int64_t n, int64_t nnz, const int64_t* rowpt
       }
     upload_csr(ctx, g.AT, n, nnz, trp.data(), tc.data(), tv.data(), true);
     build_bins(ctx, g.AT, trp.data());
+    // hub tiles / dense core for both operators (any square CSR; the tiles
+    // need a rank-1 value scaling a_ij = r_i c_j, e.g. a row-normalised graph)
+    if (n >= 4096 && nnz > 0) {
+      build_core(ctx, g.A, rp.data(), c.data(), v.data());
+      build_core(ctx, g.AT, trp.data(), tc.data(), tv.data());
+    }
+  }
+  // hot-row panels of the CSRs the SpMM streams (the hub-core residual if any)
+  for (Csr* S : {&g.A, &g.AT}) {
+    if (!S->col) continue;
+    build_hot(ctx, S->core.resid ? *S->core.resid : *S);
   }
   RDM_CUDA(cudaDeviceSynchronize());
   ctx->has_graph = true;
@@ -566,6 +577,24 @@ rdm_status rdm_init_emulated(rdm_ctx** out, int rank, int world, int device, voi
 }
 
 int rdm_is_emulated(const rdm_ctx* ctx) { return ctx && ctx->emulated ? 1 : 0; }
+
+rdm_status rdm_comm_info(rdm_ctx* ctx, int* nccl_version, int* comm_ranks, int* comm_rank,
+                         int* comm_device) {
+  if (!ctx) return RDM_ERR_ARG;
+  return guarded(ctx, [&] {
+    int v = 0, n = 0, r = -1, d = -1;
+    RDM_NCCL(ncclGetVersion(&v));
+    if (ctx->comm) {
+      RDM_NCCL(ncclCommCount(ctx->comm, &n));
+      RDM_NCCL(ncclCommUserRank(ctx->comm, &r));
+      RDM_NCCL(ncclCommCuDevice(ctx->comm, &d));
+    }
+    if (nccl_version) *nccl_version = v;
+    if (comm_ranks) *comm_ranks = n;
+    if (comm_rank) *comm_rank = r;
+    if (comm_device) *comm_device = d;
+  });
+}
 
 rdm_status rdm_finalize(rdm_ctx* ctx) {
   if (!ctx) return RDM_ERR_ARG;

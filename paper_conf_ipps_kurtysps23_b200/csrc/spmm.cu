@@ -27,6 +27,7 @@
 #include <vector>
 
 #include <cuda_bf16.h>
+#include <cub/cub.cuh>
 
 #include "internal.h"
 
@@ -55,7 +56,7 @@ struct Epi {
   const float* tpart;       // binary hub tiles: per-item partials (n_items x 128 x ld_tpart) or null
   int64_t ld_tpart;
   const int32_t* rb_item;   // item range of each 128-row rank block
-  const float* tscale;      // s_i of slot i
+  const float* tscale;      // row scale r_i of hub slot i (a_ij = r_i c_j)
   Scatter scat;             // fused col→row redistribution (scat.P == 0: off)
   const float* rscale;      // factored bf16 path: s_i per row (applied first), or null
 };
@@ -121,6 +122,25 @@ __device__ __forceinline__ float4 apply_epi(float4 a, const Epi& e, int64_t row,
   return a;
 }
 
+// Hot-row panel (DRAM-resident slices): the residual CSR's column stream
+// `col_hot` encodes the columns of the hot_max most referenced vertices as
+// -(rank+1); per call the rows of the hw hottest are copied into a compact
+// panel xh (contiguous, full 128-byte lines, kept in L2 by an access-policy
+// window), ranks in [hw, hot_max) read X at ids[rank].  hw == 0: off.
+struct Hot {
+  const float* xh;        // hw x ldh (chunk offset applied by the kernel)
+  const int32_t* ids;     // vertex of each hot rank
+  int64_t ldh;
+  int hw;
+};
+
+__device__ __forceinline__ const float* row_ptr(const float* xb, int64_t ldx, int cc, const Hot& h,
+                                                int64_t cbase) {
+  if (cc >= 0) return xb + (int64_t)cc * ldx;
+  const int r = -cc - 1;
+  return r < h.hw ? h.xh + cbase + (int64_t)r * h.ldh : xb + (int64_t)__ldg(h.ids + r) * ldx;
+}
+
 // Warp computes Σ_{j in [beg,end)} val[j] · X[col[j], chunk columns].  A group
 // of G lanes owns one nnz at a time; lane `sub` of the group loads float4
 // chunks sub, sub+G, …, sub+(V-1)G of the row chunk (each warp-level load is a
@@ -133,7 +153,7 @@ __device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
                                                const float* __restrict__ val,
                                                const float* __restrict__ xb, int64_t ldx,
                                                int64_t beg, int64_t end, int lane, int c4n,
-                                               float4 (&acc)[V]) {
+                                               float4 (&acc)[V], const Hot& hot, int64_t cbase) {
   constexpr int NG = 32 / G;
   static_assert(G % U == 0, "U must divide G");
   const int g = lane / G, sub = lane % G;
@@ -159,7 +179,7 @@ __device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
         const int cc = (G == 1) ? c : __shfl_sync(kFull, c, k);
         const float vv = (G == 1) ? a : __shfl_sync(kFull, a, k);
         if (k < cnt) {
-          const float4* xr = reinterpret_cast<const float4*>(xb + (int64_t)cc * ldx);
+          const float4* xr = reinterpret_cast<const float4*>(row_ptr(xb, ldx, cc, hot, cbase));
           float4 x[V];
 #pragma unroll
           for (int v = 0; v < V; ++v)
@@ -186,7 +206,8 @@ __device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
         const int k = (t0 + u) * NG + g;
         const int cc = (G == 1) ? c : __shfl_sync(kFull, c, k);
         vv[u] = (G == 1) ? a : __shfl_sync(kFull, a, k);
-        const float4* xr = reinterpret_cast<const float4*>(xb + (int64_t)cc * ldx);
+        const float4* xr = reinterpret_cast<const float4*>(
+            k < cnt ? row_ptr(xb, ldx, cc, hot, cbase) : xb);
 #pragma unroll
         for (int v = 0; v < V; ++v)
           x[u][v] = (k < cnt && v * G + sub < c4n) ? RDM_GATHER_LD(xr + v * G + sub) : make_float4(0.f, 0.f, 0.f, 0.f);
@@ -232,7 +253,7 @@ spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
             const int64_t* __restrict__ seg_start, const int32_t* __restrict__ seg_row,
             int64_t n_light, int64_t n_seg, const float* __restrict__ X, int64_t ldx,
             float* __restrict__ out, int64_t ld_out, float* __restrict__ part, int64_t ld_part,
-            int64_t w4, int chunk4, Epi epi) {
+            int64_t w4, int chunk4, Epi epi, Hot hot) {
   const int lane = threadIdx.x & 31;
   const int64_t item = (int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5);
   if (item >= n_seg + n_light) return;
@@ -246,7 +267,7 @@ spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
     r = seg_row[item];
     const int64_t beg = seg_start[item];
     const int64_t end = min(beg + kSeg, rowptr[r + 1]);
-    warp_nnz_range<G, V, U>(col, val, X + cbase, ldx, beg, end, lane, c4n, acc);
+    warp_nnz_range<G, V, U>(col, val, X + cbase, ldx, beg, end, lane, c4n, acc, hot, cbase);
     if (lane < G) {
       float* dst = part + item * ld_part + cbase;
 #pragma unroll
@@ -255,7 +276,7 @@ spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
     }
   } else {
     r = light_rows[item - n_seg];
-    warp_nnz_range<G, V, U>(col, val, X + cbase, ldx, rowptr[r], rowptr[r + 1], lane, c4n, acc);
+    warp_nnz_range<G, V, U>(col, val, X + cbase, ldx, rowptr[r], rowptr[r + 1], lane, c4n, acc, hot, cbase);
     if (lane < G) {
       float* dst = out + (int64_t)r * ld_out + cbase;
 #pragma unroll
@@ -468,16 +489,16 @@ __global__ void spmm_heavy_reduce(const int32_t* __restrict__ heavy_rows,
 template <int G, int V, int U>
 void launch_spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out,
                  int64_t ld_out, float* part, int64_t ld_part, int64_t w4, int chunk4,
-                 const Epi& epi) {
+                 const Epi& epi, const Hot& hot) {
   const int64_t items = A.n_seg + A.n_light;
   if (items == 0) return;
   const int64_t chunks = ceil_div(w4, 4 * chunk4);
   dim3 grid((unsigned)ceil_div(items, kWarps), (unsigned)chunks);
   spmm_kernel<G, V, U><<<grid, kWarps * 32, 0, ctx->stream>>>(
-      A.rowptr->as<int64_t>(), A.col->as<int32_t>(), A.val->as<float>(),
+      A.rowptr->as<int64_t>(), hot.hw ? A.col_hot->as<int32_t>() : A.col->as<int32_t>(), A.val->as<float>(),
       A.light_rows->as<int32_t>(), A.seg_start->as<int64_t>(),
       reinterpret_cast<const int32_t*>(A.seg_start->as<int64_t>() + A.n_seg), A.n_light, A.n_seg,
-      in, ld_in, out, ld_out, part, ld_part, w4, chunk4, epi);
+      in, ld_in, out, ld_out, part, ld_part, w4, chunk4, epi, hot);
   RDM_LAUNCHED(ctx);
 }
 
@@ -524,9 +545,16 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
 // columns each).  Measured on the Reddit- and products-shaped residual CSRs
 // (tools/exp_gvu.py, profiles/r1_spmm_gvu.txt): for bf16 rows several nnz in
 // flight per group (U) pay; fp32 keeps U = 1 (best or tied at every width).
-void pick_gvu(int c, bool bf, int* G, int* V, int* U) {
+void pick_gvu(int c, bool bf, int* G, int* V, int* U, bool dram_slice = false) {
   pick_gv(c, G, V);
   *U = 1;
+  if (!bf) {
+    // 9-12 vectors (w = 33..48): 8 lanes x 2 (profiles/r2_spmm_gvu.txt: w = 41 0.82 → 0.79 ms)
+    if (c >= 9 && c <= 12) { *G = 8; *V = 2; }
+    // DRAM-resident slices (larger than L2): the gathers wait on DRAM, so narrow
+    // rows keep 4 nnz in flight per group (papers100M-shaped w = 16)
+    if (dram_slice && c <= 8) { *V = 1; *G = c <= 4 ? 4 : 8; *U = 4; }
+  }
   if (bf) {
     if (c >= 3 && c <= 8) { *G = 8; *V = 1; *U = 4; }
     else if (c >= 9 && c <= 16) { *G = 8; *V = 2; *U = 2; }
@@ -640,9 +668,9 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
   // (measured, tools/exp_tiles.py: fp16 pairs pay where the tile is MMA-bound,
   // w > 64: 1.53 → 1.44 ms at w = 128; narrower tiles are bound by the bit
   // expansion and the extra column-max pass makes fp16 pairs slower)
-  int np = ctx->prec == RDM_PREC_FAST ? 1 : (w > 64 ? 2 : 3);
+  int np = ctx->prec == RDM_PREC_FAST ? 1 : kPiecesI8;
   if (ctx->prec != RDM_PREC_FAST)
-    if (const char* e = getenv("RDM_TILE_PIECES")) np = atoi(e) == 3 ? 3 : 2;
+    if (const char* e = getenv("RDM_TILE_PIECES")) np = atoi(e) == 3 ? 3 : atoi(e) == 2 ? 2 : kPiecesI8;
   if (A.core.n_tiles && hub_tiles_pay(A.core, w, np)) {
     // binary hub tiles on the kind::f16 tensor cores (hubtiles.cu); the
     // residual CSR's epilogue adds s_i · Σ_items partial for hub rows.
@@ -652,7 +680,7 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
     epi.tpart = part;
     epi.ld_tpart = ldp;
     epi.rb_item = A.core.rb_item->as<int32_t>();
-    epi.tscale = A.core.scale->as<float>();
+    epi.tscale = A.core.rscale->as<float>();
     epi.hub_slot = A.core.hub_slot->as<int32_t>();
     run_csr(ctx, *A.core.resid, in, ld_in, out, ld_out, w4, epi, inb, fact);
   } else if (A.core.K && core_pays(A.core, w)) {
@@ -678,6 +706,71 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
 }
 
 namespace {
+// xh[r] = X[ids[r]] for the hw hottest rows (float4 copies, full leading dim).
+__global__ void hot_gather_kernel(const float* __restrict__ X, int64_t ldx, const int32_t* __restrict__ ids,
+                                  int64_t hw, int64_t ld4, float* __restrict__ xh) {
+  const int64_t total = hw * ld4;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t r = i / ld4, c = i - r * ld4;
+    reinterpret_cast<float4*>(xh)[i] = __ldg(reinterpret_cast<const float4*>(X + (int64_t)__ldg(ids + r) * ldx) + c);
+  }
+}
+
+// L2 access-policy window on the hot panel for the duration of one SpMM
+// (persisting hits; cleared on scope exit).  RDM_HOT_PERSIST=0 disables.
+struct HotWindow {
+  rdm_ctx* ctx;
+  bool on = false;
+  explicit HotWindow(rdm_ctx* c) : ctx(c) {}
+  void set(void* base, size_t bytes) {
+    const char* e = getenv("RDM_HOT_PERSIST");
+    if (e && !atoi(e)) return;
+    static size_t limit = 0;
+    if (!limit) {
+      int dev = 0, maxp = 0;
+      cudaGetDevice(&dev);
+      cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev);
+      limit = (size_t)maxp;
+      if (limit) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, limit);
+      (void)cudaGetLastError();
+    }
+    if (!limit) return;
+    cudaStreamAttrValue v{};
+    v.accessPolicyWindow.base_ptr = base;
+    v.accessPolicyWindow.num_bytes = std::min(bytes, limit);
+    v.accessPolicyWindow.hitRatio = 1.0f;
+    v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
+    v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
+    on = cudaStreamSetAttribute(ctx->stream, cudaStreamAttributeAccessPolicyWindow, &v) == cudaSuccess;
+    (void)cudaGetLastError();
+  }
+  ~HotWindow() {
+    if (!on) return;
+    cudaStreamAttrValue v{};
+    v.accessPolicyWindow.num_bytes = 0;
+    cudaStreamSetAttribute(ctx->stream, cudaStreamAttributeAccessPolicyWindow, &v);
+    cudaCtxResetPersistingL2Cache();
+    (void)cudaGetLastError();
+  }
+};
+
+// Per call: how many hot rows fit the panel budget (RDM_HOT_MB, default 64 MB)
+// at this leading dim, their copy, and the window.
+Hot hot_panel(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, int64_t w4, HotWindow& win) {
+  (void)w4;
+  double mb = 64.0;
+  if (const char* e = getenv("RDM_HOT_MB")) mb = atof(e);
+  const int64_t hw = std::min<int64_t>(A.hot_max, (int64_t)(mb * 1048576.0 / (ld_in * 4.0)));
+  if (hw <= 0) return Hot{nullptr, nullptr, 0, 0};
+  float* xh = ensure_ws(ctx->ws_hot, (size_t)hw * ld_in * sizeof(float));
+  const int64_t total = hw * (ld_in / 4);
+  const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(total, 256), (int64_t)ctx->num_sms * 16));
+  hot_gather_kernel<<<grid, 256, 0, ctx->stream>>>(in, ld_in, A.hot_ids->as<int32_t>(), hw, ld_in / 4, xh);
+  RDM_LAUNCHED(ctx);
+  win.set(xh, (size_t)hw * ld_in * sizeof(float));
+  return Hot{xh, A.hot_ids->as<int32_t>(), ld_in, (int)hw};
+}
+
 void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
              int64_t w4, const Epi& epi, const __nv_bfloat16* inb, bool fact) {
   const int64_t w8 = (w4 + 7) & ~int64_t(7);
@@ -734,10 +827,14 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
   } else {
     const int c4 = (int)std::min<int64_t>(chunk4, w4 / 4);
     int U = 1;
-    if (!getenv("RDM_SPMM_GV")) pick_gvu(c4, false, &G, &V, &U);
+    const bool dram_slice = (double)A.in_rows() * (double)ld_in * 4.0 > 96e6;
+    if (!getenv("RDM_SPMM_GV")) pick_gvu(c4, false, &G, &V, &U, dram_slice);
+    Hot hot{nullptr, nullptr, 0, 0};
+    HotWindow window(ctx);
+    if (dram_slice && A.col_hot) hot = hot_panel(ctx, A, in, ld_in, w4, window);
     if (const char* e = getenv("RDM_SPMM_U")) U = atoi(e);
 #define RDM_SPMM_CASE(g_, v_, u_) \
-  if (G == g_ && V == v_ && U == u_) launch_spmm<g_, v_, u_>(ctx, A, in, ld_in, out, ld_out, part, w4, w4, chunk4, epi); else
+  if (G == g_ && V == v_ && U == u_) launch_spmm<g_, v_, u_>(ctx, A, in, ld_in, out, ld_out, part, w4, w4, chunk4, epi, hot); else
     RDM_SPMM_CASE(1, 1, 1) RDM_SPMM_CASE(1, 2, 1) RDM_SPMM_CASE(1, 3, 1) RDM_SPMM_CASE(1, 4, 1)
     RDM_SPMM_CASE(2, 1, 1) RDM_SPMM_CASE(2, 1, 2) RDM_SPMM_CASE(2, 2, 1) RDM_SPMM_CASE(2, 2, 2)
     RDM_SPMM_CASE(2, 3, 1) RDM_SPMM_CASE(2, 3, 2) RDM_SPMM_CASE(2, 4, 1) RDM_SPMM_CASE(2, 4, 2)
@@ -749,7 +846,7 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
     RDM_SPMM_CASE(16, 1, 1) RDM_SPMM_CASE(16, 1, 2) RDM_SPMM_CASE(16, 1, 4) RDM_SPMM_CASE(16, 2, 1)
     RDM_SPMM_CASE(16, 2, 2) RDM_SPMM_CASE(16, 2, 4) RDM_SPMM_CASE(16, 3, 1) RDM_SPMM_CASE(16, 3, 2)
     RDM_SPMM_CASE(16, 4, 1) RDM_SPMM_CASE(16, 4, 2) RDM_SPMM_CASE(32, 1, 1) RDM_SPMM_CASE(32, 1, 2)
-    RDM_SPMM_CASE(32, 1, 4)
+    RDM_SPMM_CASE(32, 1, 4) RDM_SPMM_CASE(8, 1, 8)
     throw Error(RDM_ERR_ARG, "spmm: no kernel for G/V/U");
 #undef RDM_SPMM_CASE
   }
@@ -761,6 +858,65 @@ heavy:
   }
 }
 }  // namespace
+
+namespace {
+__global__ void ref_count_kernel(const int32_t* __restrict__ col, int64_t nnz, int32_t* __restrict__ cnt) {
+  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nnz; j += (int64_t)gridDim.x * blockDim.x)
+    atomicAdd(cnt + col[j], 1);
+}
+__global__ void iota_kernel(int32_t* __restrict__ v, int64_t n) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < n; i += (int64_t)gridDim.x * blockDim.x)
+    v[i] = (int32_t)i;
+}
+__global__ void hot_rank_kernel(const int32_t* __restrict__ order, int64_t hmax, int32_t* __restrict__ rank) {
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < hmax; i += (int64_t)gridDim.x * blockDim.x)
+    rank[order[i]] = (int32_t)i;
+}
+__global__ void hot_encode_kernel(const int32_t* __restrict__ col, int64_t nnz, const int32_t* __restrict__ rank,
+                                  int32_t* __restrict__ out) {
+  for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nnz; j += (int64_t)gridDim.x * blockDim.x) {
+    const int32_t c = col[j];
+    const int32_t r = rank[c];
+    out[j] = r >= 0 ? -r - 1 : c;
+  }
+}
+}  // namespace
+
+// Hot-row panel (see Hot): built for CSRs whose input slice can exceed L2
+// (>= 1 M input rows) — RDM_NO_HOT=1 disables.  hot_max = min(rows, 8 M):
+// the per-call panel takes the hottest rows that fit its byte budget.
+void build_hot(rdm_ctx* ctx, Csr& A) {
+  const char* off = getenv("RDM_NO_HOT");
+  const int64_t nin = A.in_rows();
+  if ((off && atoi(off)) || A.nnz == 0 || nin < (1 << 20) || nin >= INT32_MAX) return;
+  const int64_t hmax = std::min<int64_t>(nin, 1 << 23);
+  DevBuf cnt(nin * 4), iota(nin * 4), keys(nin * 4), order(nin * 4), rank(nin * 4);
+  const unsigned g = (unsigned)(ctx->num_sms * 8);
+  RDM_CUDA(cudaMemsetAsync(cnt.ptr, 0, nin * 4, ctx->stream));
+  ref_count_kernel<<<g, 256, 0, ctx->stream>>>(A.col->as<int32_t>(), A.nnz, cnt.as<int32_t>());
+  RDM_LAUNCHED(ctx);
+  iota_kernel<<<g, 256, 0, ctx->stream>>>(iota.as<int32_t>(), nin);
+  RDM_LAUNCHED(ctx);
+  size_t tb = 0;
+  RDM_CUDA(cub::DeviceRadixSort::SortPairsDescending(nullptr, tb, cnt.as<int32_t>(), keys.as<int32_t>(),
+                                                      iota.as<int32_t>(), order.as<int32_t>(), (int)nin, 0, 32,
+                                                      ctx->stream));
+  DevBuf tmp(std::max<size_t>(tb, 256));
+  RDM_CUDA(cub::DeviceRadixSort::SortPairsDescending(tmp.ptr, tb, cnt.as<int32_t>(), keys.as<int32_t>(),
+                                                      iota.as<int32_t>(), order.as<int32_t>(), (int)nin, 0, 32,
+                                                      ctx->stream));
+  RDM_CUDA(cudaMemsetAsync(rank.ptr, 0xFF, nin * 4, ctx->stream));   // -1 = cold
+  hot_rank_kernel<<<g, 256, 0, ctx->stream>>>(order.as<int32_t>(), hmax, rank.as<int32_t>());
+  RDM_LAUNCHED(ctx);
+  A.col_hot.reset(new DevBuf(A.nnz * 4));
+  hot_encode_kernel<<<g, 256, 0, ctx->stream>>>(A.col->as<int32_t>(), A.nnz, rank.as<int32_t>(),
+                                                A.col_hot->as<int32_t>());
+  RDM_LAUNCHED(ctx);
+  A.hot_ids.reset(new DevBuf(hmax * 4));
+  RDM_CUDA(cudaMemcpyAsync(A.hot_ids->ptr, order.ptr, hmax * 4, cudaMemcpyDeviceToDevice, ctx->stream));
+  RDM_CUDA(cudaStreamSynchronize(ctx->stream));
+  A.hot_max = hmax;
+}
 
 // Row bins (host, one-time at rdm_set_graph; pure indexing of rowptr).
 void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rp, bool sync) {

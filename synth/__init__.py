@@ -200,7 +200,10 @@ class Workload:
     n: int
     n_edges: int          # undirected edges before self loops: nnz = 2*n_edges + n
     f: tuple              # (f_0, ..., f_L)
-    graph: str = "rmat"
+    graph: str = "rmat"   # "rmat" (Graph500 a,b,c,d) or "er" (uniform)
+    permute: bool = True  # seeded vertex permutation (Graph500: worst-case locality)
+    values: str = "sym"   # "sym": D^-1/2 (A+I) D^-1/2; "noise": sym x (1 + 2^-4 u_ij), u_ij = u_ji
+                          # (symmetric, not a rank-1 scaling); "row": D^-1 (A+I) (not symmetric)
 
     @property
     def nnz(self) -> int:
@@ -217,10 +220,42 @@ WORKLOADS = {
     "reddit": Workload("reddit-shaped 2L h128", 232965, 57307946, (602, 128, 41)),
     "products": Workload("products-shaped 3L h256", 2449029, 61859140, (100, 256, 256, 47)),
     "papers": Workload("papers100M-shaped 2L h128", 111059956, 799470022, (128, 128, 172)),
+    # controls for the input specialisations: uniform graph, values
+    # that are not a rank-1 scaling of the pattern, row-normalised values, and
+    # the un-permuted (locality-preserving) R-MAT order
+    "reddit-er": Workload("reddit-shaped ER 2L h128", 232965, 57307946, (602, 128, 41), graph="er"),
+    "reddit-noise": Workload("reddit-shaped, non-factorable values 2L h128", 232965, 57307946, (602, 128, 41),
+                             values="noise"),
+    "reddit-row": Workload("reddit-shaped, row-normalised 2L h128", 232965, 57307946, (602, 128, 41),
+                           values="row"),
+    "products-er": Workload("products-shaped ER 3L h256", 2449029, 61859140, (100, 256, 256, 47), graph="er"),
+    "papers-local": Workload("papers100M-shaped, un-permuted 2L h128", 111059956, 799470022, (128, 128, 172),
+                             permute=False),
 }
 
 
 def make_graph(w: Workload, seed: int = SEED_GRAPH) -> CSR:
     if w.graph == "er":
-        return erdos_renyi(w.n, w.n_edges, seed)
-    return rmat(w.n, w.n_edges, seed)
+        g = erdos_renyi(w.n, w.n_edges, seed)
+    else:
+        g = rmat(w.n, w.n_edges, seed, permute=w.permute)
+    if w.values == "noise":
+        rows = np.repeat(np.arange(g.n, dtype=np.int64), np.diff(g.rowptr))
+        lo = np.minimum(rows, g.col).astype(np.uint64)
+        hi = np.maximum(rows, g.col).astype(np.uint64)
+        h = (lo * np.uint64(0x9E3779B97F4A7C15)) ^ (hi * np.uint64(0xBF58476D1CE4E5B9))
+        h ^= h >> np.uint64(29)
+        h *= np.uint64(0x94D049BB133111EB)
+        h ^= h >> np.uint64(32)
+        u = (h >> np.uint64(40)).astype(np.float64) / 16777216.0
+        g = CSR(g.n, g.rowptr, g.col, (g.val.astype(np.float64) * (1.0 + u / 16.0)).astype(np.float32))
+    elif w.values == "row":
+        deg = np.diff(g.rowptr).astype(np.float64)
+        rows = np.repeat(np.arange(g.n), np.diff(g.rowptr))
+        g = CSR(g.n, g.rowptr, g.col, (1.0 / deg[rows]).astype(np.float32))
+    return g
+
+
+def symmetric_values(w: Workload) -> bool:
+    """Whether make_graph(w)'s values satisfy A = Aᵀ (rdm_set_graph's `symmetric`)."""
+    return w.values != "row"

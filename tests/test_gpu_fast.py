@@ -24,6 +24,8 @@ from test_gpu_gcn import _check, _problem, _run
 pytestmark = pytest.mark.gpu
 
 GATE = 2e-2
+# loss: the north star states 1e-5 relative for the loss with no variant exception
+LOSS_GATE = 1e-5
 
 
 def bf16_rne(x):
@@ -194,14 +196,14 @@ def cora():
 def test_fast_epoch_within_gate(rdm, cora, P, cfg):
     g, H0, Ws, y, m = cora
     loss, dW, model, ctx, _ = _run(rdm, g, H0, Ws, y, m, cfg, P=P, precision="fast")
-    _check((g, H0, Ws, y, m), loss, dW, model, rdm, P=P, tol=GATE, ltol=1e-3)
+    _check((g, H0, Ws, y, m), loss, dW, model, rdm, P=P, tol=GATE, ltol=LOSS_GATE)
 
 
 def test_fast_three_layer_products_shaped(rdm):
     prob = _problem(n=6000, E=40000, f=(100, 256, 256, 47), seed=2)
     g, H0, Ws, y, m = prob
     loss, dW, model, ctx, _ = _run(rdm, g, H0, Ws, y, m, 9, P=2, precision="fast")
-    _check(prob, loss, dW, model, rdm, P=2, tol=GATE, ltol=1e-3)
+    _check(prob, loss, dW, model, rdm, P=2, tol=GATE, ltol=LOSS_GATE)
 
 
 @pytest.mark.parametrize("cfg", [3, 10])
@@ -211,7 +213,7 @@ def test_fast_epoch_hub_tiles(rdm, cfg, monkeypatch):
     g, H0, Ws, y, m = prob
     loss, dW, model, ctx, _ = _run(rdm, g, H0, Ws, y, m, cfg, precision="fast")
     assert ctx.graph_info()["n_tiles"] > 0
-    _check(prob, loss, dW, model, rdm, tol=GATE, ltol=1e-3)
+    _check(prob, loss, dW, model, rdm, tol=GATE, ltol=LOSS_GATE)
 
 
 def test_precision_rejects_unknown(rdm):

@@ -241,9 +241,9 @@ def test_spmm_hub_core_matches_oracle(torch_dev, w, K, monkeypatch):
 @pytest.mark.parametrize("min_nnz,k2", [(1, 0), (40, 0), (1, 1024)])
 @pytest.mark.parametrize("pieces", ["auto", "2", "3"])
 def test_spmm_hub_tiles_matches_oracle(torch_dev, w, min_nnz, k2, pieces, monkeypatch):
-    """Binary hub tiles (kind::f16 tensor cores on 0/1 tiles against the
-    3-piece bf16 split of s ⊙ X) + residual CSR == the plain product, with
-    epilogues.  min_nnz forces the tile selection (every block with at least
+    """Binary hub tiles (tensor cores on 0/1 tiles against s ⊙ X as three int8
+    digits on kind::i8 (auto), two column-scaled fp16 or three bf16 pieces on
+    kind::f16) + residual CSR == the plain product, with epilogues.  min_nnz forces the tile selection (every block with at least
     that many entries), k2 limits the rank range (0 = all)."""
     torch, dev = torch_dev
     import paper_conf_ipps_kurtysps23_b200 as rdm
@@ -274,11 +274,12 @@ def test_spmm_hub_tiles_matches_oracle(torch_dev, w, min_nnz, k2, pieces, monkey
     assert np.all(out[:, w:].cpu().numpy() == 0)
 
 
-@pytest.mark.parametrize("pieces", ["2", "3"])
+@pytest.mark.parametrize("pieces", ["auto", "2", "3"])
 def test_spmm_hub_tiles_wide_range_values(torch_dev, pieces, monkeypatch):
-    """Inputs spanning 2^±30 per row and exact zeros: the column-scaled fp16
-    pieces and the bf16 pieces keep the fp32 gate (normwise per tensor,
-    reading R26) — no overflow, no lost columns."""
+    """Inputs spanning 2^±30 per row and exact zeros: the int8 digits (auto:
+    23-bit fixed point per column), the column-scaled fp16 pieces and the bf16
+    pieces keep the fp32 gate (normwise per tensor, reading R26) — no
+    overflow, no lost columns."""
     torch, dev = torch_dev
     import paper_conf_ipps_kurtysps23_b200 as rdm
     monkeypatch.setenv("RDM_TILE_MIN_NNZ", "1")
@@ -320,3 +321,39 @@ def test_spmm_hub_tiles_need_factorised_values(torch_dev, monkeypatch):
         ctx.sync()
         g2 = synth.CSR(g.n, g.rowptr, g.col, vals)
         assert og.max_rel_err(out[:, :w].cpu().numpy(), og.spmm(g2, X)) < TOL
+
+
+@pytest.mark.parametrize("norm", ["row", "col", "weighted"])
+def test_spmm_hub_tiles_general_rank1_values(torch_dev, norm, monkeypatch):
+    """Tiles factor any rank-1 scaling a_ij = r_i c_j of the 0/1 pattern, not only
+    the symmetric s_i s_j: the row-normalised D^-1 (A+I), the column-normalised
+    (A+I) D^-1 and random positive r, c all build tiles and match the oracle."""
+    torch, dev = torch_dev
+    import paper_conf_ipps_kurtysps23_b200 as rdm
+    monkeypatch.setenv("RDM_TILE_MIN_NNZ", "1")
+    g = synth.rmat(6000, 150000, seed=16)
+    deg = np.diff(g.rowptr).astype(np.float64)
+    rows = np.repeat(np.arange(g.n), np.diff(g.rowptr))
+    rng = np.random.default_rng(4)
+    if norm == "row":
+        v = 1.0 / deg[rows]
+    elif norm == "col":
+        v = 1.0 / deg[g.col]
+    else:
+        r, c = rng.uniform(0.1, 10, g.n), rng.uniform(0.1, 10, g.n)
+        v = r[rows] * c[g.col]
+    g2 = synth.CSR(g.n, g.rowptr, g.col, v.astype(np.float32))
+    ctx = rdm.Context(device=0)
+    ctx.set_graph(g2.rowptr, g2.col, g2.val, symmetric=False)   # values are not symmetric
+    assert ctx.graph_info()["n_tiles"] > 0
+    for w in (41, 128):
+        X = rng.standard_normal((g.n, w)).astype(np.float32)
+        xd = _padded(torch, dev, X)
+        out = torch.zeros_like(xd)
+        ctx.spmm(0, xd, out, w)
+        ctx.sync()
+        assert og.max_rel_err(out[:, :w].cpu().numpy(), og.spmm(g2, X)) < TOL
+        out.zero_()
+        ctx.spmm(1, xd, out, w)          # Aᵀ·X from the transpose's own tiles
+        ctx.sync()
+        assert og.max_rel_err(out[:, :w].cpu().numpy(), og.spmm_t(g2, X)) < TOL
