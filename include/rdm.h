@@ -226,8 +226,13 @@ int rdm_get_transport(const rdm_ctx* ctx);
  *     (half the L2/HBM gather bytes), accumulating in fp32; the binary hub
  *     tiles multiply one bf16 piece of s⊙X (fp32: two column-scaled fp16 or three bf16 pieces); every rdm_gemm
  *     (NN / NT / TN) issues one tf32 MMA per k step instead of 3xTF32 (the
- *     tensor core reads fp32 operands as tf32).  Outputs, gradients and the
- *     loss stay fp32 in the caller's buffers; redistribution stays bit-exact.
+ *     tensor core reads fp32 operands as tf32).  Inside rdm_gcn_forward /
+ *     backward the row → column redistributions (whose destination is an
+ *     SpMM input, rounded to bf16 by the variant anyway) carry bf16 on the
+ *     wire (half their bytes; each moved value, the rank's own block included,
+ *     rounded once); column → row moves stay fp32.  Outputs, gradients and the
+ *     loss stay fp32 in the caller's buffers; the public rdm_redistribute
+ *     stays bit-exact fp32.
  *     Parity gate 2e-2 (max relative error per tensor, reading R26).
  * Applies to every later call on the ctx (the executor included).
  * Errors: RDM_ERR_ARG (unknown value). */

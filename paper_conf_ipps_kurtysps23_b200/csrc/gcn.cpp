@@ -740,10 +740,18 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
         src[i] = buf(g, i, s.in, s.lin).p;
         dst[i] = buf(g, i, s.out, s.lout).p;
       }
-      if (g->RA)
+      if (g->RA) {
         redistribute_panels(ctx, (rdm_layout)s.lin, src.data(), dst.data(), gn(g), s.width);
-      else
-        redistribute(ctx, (rdm_layout)s.lin, src.data(), dst.data(), gn(g), s.width);
+      } else {
+        // bf16 wire in the fast variant (NEXT-3) for row → column moves: their
+        // destination is an SpMM input, which the fast variant rounds to bf16
+        // anyway; column → row moves (SpMM outputs feeding GEMMs and the loss)
+        // stay fp32.  RDM_BF16_WIRE=0 disables (experiments).
+        const char* wv = getenv("RDM_BF16_WIRE");
+        const bool wire_off = wv && !atoi(wv);
+        redistribute(ctx, (rdm_layout)s.lin, src.data(), dst.data(), gn(g), s.width,
+                     ctx->prec == RDM_PREC_FAST && s.lin == RDM_ROW && !wire_off);
+      }
       break;
     }
     case S_MASK: {

@@ -546,6 +546,7 @@ __device__ __forceinline__ void tc_mma_i8_ts(uint32_t tmem_d, uint32_t tmem_a, u
 
 // One stage = one whole tile: B digits [3][n_mma][128 B] (128-byte swizzle,
 // one 3-D TMA), then the tile's bits [half][128 rows] u64.
+template <int D>
 __global__ void __launch_bounds__(384, 1)
 hub_tile_i8_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __restrict__ bits,
                    const int32_t* __restrict__ tile_cb, const int32_t* __restrict__ item_tb,
@@ -562,7 +563,7 @@ hub_tile_i8_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __re
   uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int total = sh.n_items * sh.tiles_n;
-  const int bbytes = 3 * n_mma * 128;
+  const int bbytes = D * n_mma * 128;
   auto B_st = [&](int s) { return smem + s * sh.stage_bytes; };
   auto bits_st = [&](int s) { return smem + s * sh.stage_bytes + bbytes; };
   if (threadIdx.x == 0) {
@@ -616,7 +617,7 @@ hub_tile_i8_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __re
     }
   } else if (warp == 1) {
     if (lane == 0) {
-      const uint32_t idesc = idesc_i8(3 * n_mma);
+      const uint32_t idesc = idesc_i8(D * n_mma);
       const uint64_t bd0 = sdesc(smem_u32(B_st(0)), 16, 1024);
       const uint32_t st16 = (uint32_t)sh.stage_bytes >> 4;
       int s = 0, a = 0;
@@ -688,11 +689,11 @@ hub_tile_i8_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __re
       float* prow = part + ((int64_t)item * TK + q * 32 + lane) * sh.ldp + n0;
       for (int c0 = 0; c0 < n_mma; c0 += 32) {
         if (n0 + c0 >= sh.w) break;
-        uint32_t d2[32], d1[32], d0[32];
+        // digit accumulators, most significant first: v = Σ_d acc_d · 256^(D-1-d)
+        uint32_t dg[D][32];
         const uint32_t a0 = tmem_base + acc * sh.acc_cols + ((uint32_t)(q * 32) << 16) + (uint32_t)c0;
-        tmem_ld32(a0, d2);
-        tmem_ld32(a0 + (uint32_t)n_mma, d1);
-        tmem_ld32(a0 + (uint32_t)(2 * n_mma), d0);
+#pragma unroll
+        for (int d = 0; d < D; ++d) tmem_ld32(a0 + (uint32_t)(d * n_mma), dg[d]);
 #pragma unroll
         for (int i = 0; i < 32; i += 4)
           if (n0 + c0 + i < sh.w) {
@@ -700,8 +701,9 @@ hub_tile_i8_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __re
             float o[4];
 #pragma unroll
             for (int u = 0; u < 4; ++u) {
-              const long long v = (long long)(int)d2[i + u] * 65536 + (long long)(int)d1[i + u] * 256 +
-                                  (long long)(int)d0[i + u];
+              long long v = 0;
+#pragma unroll
+              for (int d = 0; d < D; ++d) v = v * 256 + (long long)(int)dg[d][i + u];
               o[u] = __ll2float_rn(v);
             }
             *reinterpret_cast<float4*>(prow + c0 + i) = make_float4(o[0] * cs.x, o[1] * cs.y, o[2] * cs.z, o[3] * cs.w);
@@ -718,9 +720,12 @@ hub_tile_i8_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __re
   }
 }
 
-// int8 digit panels P_d[n][k] (row length K2 bytes; d = 0: 2^16 digit, 1: 2^8,
-// 2: 2^0) of y = s_k · X[hub_k][n] · 2^-e_n, e_n = ilogb(colmax_n) − 21;
-// colscale[n] = 2^e_n.  Block: 128 k x 32 n, each thread 4 consecutive k.
+// int8 digit panels P_d[n][k] (row length K2 bytes; d = 0 the most
+// significant) of y = s_k · X[hub_k][n] · 2^-e_n: D = 3 digits with the column
+// maximum in [2^21, 2^22) (23-bit fixed point, fp32-class), D = 2 with it in
+// [2^13, 2^14) (15-bit, the fast variant); colscale[n] = 2^e_n.
+// Block: 128 k x 32 n, each thread 4 consecutive k.
+template <int D>
 __global__ void tile_panels_i8_kernel(const float* __restrict__ X, int64_t ldx, const int32_t* __restrict__ hub_ids,
                                       const float* __restrict__ scale, int64_t K2, int64_t w,
                                       const unsigned int* __restrict__ colmax, int8_t* __restrict__ pan,
@@ -731,7 +736,7 @@ __global__ void tile_panels_i8_kernel(const float* __restrict__ X, int64_t ldx, 
   if (threadIdx.y == 0) {
     const int64_t n = n0 + threadIdx.x;
     const float mx = n < w ? __uint_as_float(colmax[n]) : 0.f;
-    const int e = mx > 0.f ? ilogbf(mx) - 21 : 0;
+    const int e = mx > 0.f ? ilogbf(mx) - (8 * D - 3) : 0;
     inv[threadIdx.x] = ldexpf(1.f, -e);
     if (blockIdx.x == 0 && n < w) colscale[n] = ldexpf(1.f, e);
   }
@@ -758,21 +763,23 @@ __global__ void tile_panels_i8_kernel(const float* __restrict__ X, int64_t ldx, 
     const int64_t n = n0 + i;
     if (n >= w) break;
     const int kk = 4 * threadIdx.x;
-    uint32_t q[3] = {0u, 0u, 0u};
+    uint32_t q[D];
+#pragma unroll
+    for (int d = 0; d < D; ++d) q[d] = 0u;
 #pragma unroll
     for (int u = 0; u < 4; ++u) {
-      const int v = __float2int_rn(t[kk + u][i] * inv[i]);     // |v| <= 2^22
-      const int e0 = ((v & 255) ^ 128) - 128;
-      const int v1 = (v - e0) >> 8;
-      const int e1 = ((v1 & 255) ^ 128) - 128;
-      const int e2 = (v1 - e1) >> 8;
-      q[0] |= (uint32_t)(e2 & 255) << (8 * u);
-      q[1] |= (uint32_t)(e1 & 255) << (8 * u);
-      q[2] |= (uint32_t)(e0 & 255) << (8 * u);
+      int v = __float2int_rn(t[kk + u][i] * inv[i]);     // |v| <= 2^(8D-2)
+      // balanced base-256 digits, least significant first: v = Σ d_j 256^j, d_j ∈ [-128, 127]
+#pragma unroll
+      for (int d = D - 1; d >= 0; --d) {
+        const int dj = d == 0 ? v : ((v & 255) ^ 128) - 128;
+        q[d] |= (uint32_t)(dj & 255) << (8 * u);
+        v = (v - dj) >> 8;
+      }
     }
     const int64_t o = n * K2 + k0 + kk;
 #pragma unroll
-    for (int d = 0; d < 3; ++d) *reinterpret_cast<uint32_t*>(pan + (int64_t)d * w * K2 + o) = q[d];
+    for (int d = 0; d < D; ++d) *reinterpret_cast<uint32_t*>(pan + (int64_t)d * w * K2 + o) = q[d];
   }
 }
 
@@ -808,11 +815,11 @@ CUtensorMap panel_map(const void* base, int64_t K2, int64_t w, int n_mma, int HS
 // 4-D int8 map over the three digit panels P_d[n][k] (row length K2 bytes,
 // panel d at d·w·K2): dims {128 (k within a tile = one 128-byte swizzle row),
 // n, digit, k / 128}, box {128, n_mma, 3, 1}: one TMA lands [digit][n_mma][128].
-CUtensorMap panel_map_i8(const void* base, int64_t K2, int64_t w, int n_mma) {
+CUtensorMap panel_map_i8(const void* base, int64_t K2, int64_t w, int n_mma, int D) {
   CUtensorMap m;
-  cuuint64_t dims[4] = {(cuuint64_t)TK, (cuuint64_t)w, 3, (cuuint64_t)(K2 / TK)};
+  cuuint64_t dims[4] = {(cuuint64_t)TK, (cuuint64_t)w, (cuuint64_t)D, (cuuint64_t)(K2 / TK)};
   cuuint64_t strides[3] = {(cuuint64_t)K2, (cuuint64_t)(w * K2), (cuuint64_t)TK};
-  cuuint32_t box[4] = {(cuuint32_t)TK, (cuuint32_t)n_mma, 3, 1};
+  cuuint32_t box[4] = {(cuuint32_t)TK, (cuuint32_t)n_mma, (cuuint32_t)D, 1};
   cuuint32_t es[4] = {1, 1, 1, 1};
   CUresult r = encode()(&m, CU_TENSOR_MAP_DATA_TYPE_UINT8, 4, const_cast<void*>(base), dims, strides, box, es,
                         CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_128B,
@@ -840,8 +847,9 @@ CUtensorMap stacked_map(const void* base, int64_t K2, int64_t rows, int n_mma) {
 // expansion + 3 bf16 MMA pieces per 128-wide chunk), plus ≈ 20 µs per call.
 double csr_entry_s(int64_t w) { return 24e-12 * std::pow((double)w / 128.0, 0.55); }
 double tile_s(int64_t w, int np = 3) {
-  if (np == kPiecesI8)   // int8 digits: 64-wide passes, cheap expansion (first estimate)
-    return (double)ceil_div(w, I8_NMAX) * (1.2e-9 + 2.0e-9 * (double)std::min<int64_t>(w, I8_NMAX) / I8_NMAX);
+  if (np == kPiecesI8 || np == kPiecesI8x2)   // int8 digits, 64-wide passes (Reddit-shaped: ≈ 3 ns / pass)
+    return (double)ceil_div(w, I8_NMAX) * (1.2e-9 + (np == kPiecesI8 ? 2.0e-9 : 1.4e-9) *
+                                                      (double)std::min<int64_t>(w, I8_NMAX) / I8_NMAX);
   return (double)ceil_div(w, 128) * (4.5e-9 + 5.2e-9 * np / 3.0 * (double)std::min<int64_t>(w, 128) / 128.0);
 }
 }  // namespace
@@ -852,11 +860,12 @@ bool hub_tiles_pay(const Core& c, int64_t w, int np) {
   return (double)c.nnz * csr_entry_s(w) > (double)c.n_tiles * tile_s(w, np) + 20e-6;
 }
 
-// int8 digits (np == kPiecesI8): column maxima, digit panels, hub_tile_i8_kernel.
+// int8 digits (np == kPiecesI8: 3, kPiecesI8x2: 2): column maxima, digit
+// panels, hub_tile_i8_kernel<D>.
 void hub_tiles_product_i8(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx, int64_t w, float* part,
-                          int64_t ldp) {
+                          int64_t ldp, int D) {
   const int64_t K2 = c.K2;
-  int8_t* pan = reinterpret_cast<int8_t*>(ensure_ws(ctx->ws_core_b, (size_t)3 * w * K2));
+  int8_t* pan = reinterpret_cast<int8_t*>(ensure_ws(ctx->ws_core_b, (size_t)D * w * K2));
   const int64_t w4 = (w + 3) / 4 * 4;
   float* cs = ensure_ws(ctx->ws_tile_cs, (size_t)2 * w4 * sizeof(float));
   unsigned int* cmax = reinterpret_cast<unsigned int*>(cs + w4);
@@ -867,8 +876,9 @@ void hub_tiles_product_i8(rdm_ctx* ctx, const Core& c, const float* X, int64_t l
                                                          K2, w, cmax);
   RDM_LAUNCHED(ctx);
   dim3 pg((unsigned)(K2 / TK), (unsigned)ceil_div(w, 32));
-  tile_panels_i8_kernel<<<pg, dim3(32, 8), 0, ctx->stream>>>(X, ldx, c.hub_ids->as<int32_t>(), c.scale->as<float>(),
-                                                           K2, w, cmax, pan, cs);
+  auto pk = D == 3 ? tile_panels_i8_kernel<3> : tile_panels_i8_kernel<2>;
+  pk<<<pg, dim3(32, 8), 0, ctx->stream>>>(X, ldx, c.hub_ids->as<int32_t>(), c.scale->as<float>(), K2, w, cmax, pan,
+                                          cs);
   RDM_LAUNCHED(ctx);
   TileShape sh{};
   sh.n_mma = (int)std::min<int64_t>(I8_NMAX, ((w + 15) / 16) * 16);
@@ -878,27 +888,29 @@ void hub_tiles_product_i8(rdm_ctx* ctx, const Core& c, const float* X, int64_t l
   sh.ldp = ldp;
   sh.R = 1;
   sh.HS = 1;
-  sh.acc_cols = (3 * sh.n_mma + 31) / 32 * 32;
-  sh.stage_bytes = (3 * sh.n_mma * 128 + 2048 + 1023) / 1024 * 1024;
+  sh.acc_cols = (D * sh.n_mma + 31) / 32 * 32;
+  sh.stage_bytes = (D * sh.n_mma * 128 + 2048 + 1023) / 1024 * 1024;
   const int avail = kSmemBudget - 1024 - 1024;
   sh.S = std::min(32, avail / sh.stage_bytes);
   sh.SA = std::min(8, (512 - 2 * sh.acc_cols) / 32);
   sh.dbg = getenv("RDM_TILE_DBG") ? atoi(getenv("RDM_TILE_DBG")) : 0;
   sh.colscale = cs;
   RDM_CHECK_ARG(sh.S >= 2 && sh.SA >= 2, "hub tiles (int8): TMEM/smem budget");
-  const CUtensorMap tb = panel_map_i8(pan, K2, w, sh.n_mma);
+  const CUtensorMap tb = panel_map_i8(pan, K2, w, sh.n_mma, D);
   const int smem = sh.S * sh.stage_bytes + 1024 + 1024;
   const int64_t total = c.n_items * sh.tiles_n;
   const unsigned grid = (unsigned)std::min<int64_t>(total, ctx->num_sms);
-  RDM_CUDA(cudaFuncSetAttribute(hub_tile_i8_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-  hub_tile_i8_kernel<<<grid, 384, smem, ctx->stream>>>(tb, c.tiles->as<uint64_t>(), c.tile_cb->as<int32_t>(),
-                                                       c.item_tb->as<int32_t>(), part, sh);
+  auto kern = D == 3 ? hub_tile_i8_kernel<3> : hub_tile_i8_kernel<2>;
+  RDM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
+  kern<<<grid, 384, smem, ctx->stream>>>(tb, c.tiles->as<uint64_t>(), c.tile_cb->as<int32_t>(),
+                                         c.item_tb->as<int32_t>(), part, sh);
   RDM_LAUNCHED(ctx);
 }
 
 void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx, int64_t w, float* part,
                        int64_t ldp, int np) {
-  if (np == kPiecesI8) return hub_tiles_product_i8(ctx, c, X, ldx, w, part, ldp);
+  if (np == kPiecesI8) return hub_tiles_product_i8(ctx, c, X, ldx, w, part, ldp, 3);
+  if (np == kPiecesI8x2) return hub_tiles_product_i8(ctx, c, X, ldx, w, part, ldp, 2);
   RDM_CHECK_ARG(np >= 1 && np <= 3, "hub tiles: 1, 2 or 3 pieces");
   const int64_t K2 = c.K2;
   __nv_bfloat16* pan = reinterpret_cast<__nv_bfloat16*>(ensure_ws(ctx->ws_core_b, (size_t)np * w * K2 * 2));

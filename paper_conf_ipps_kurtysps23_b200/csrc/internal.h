@@ -150,13 +150,17 @@ struct Csr {
   // row bins (see spmm.cu): light rows processed warp-per-row, heavy rows
   // split into fixed-size nnz segments reduced deterministically.
   int64_t n_light = 0, n_seg = 0, n_heavy = 0;
+  // light rows by degree (light_rows is sorted by descending degree):
+  // deg_ge[d] = number of light rows of degree >= d, d = 0..kDegTab (host copy)
+  static constexpr int kDegTab = 128;
+  int64_t deg_ge[kDegTab + 1] = {};
   std::unique_ptr<DevBuf> light_rows;   // int32[n_light], longest rows first
   std::unique_ptr<DevBuf> seg_start;    // int64[n_seg]: first nnz of each segment
   std::unique_ptr<DevBuf> heavy_rows;   // int32[n_heavy]
   std::unique_ptr<DevBuf> heavy_seg;    // int32[n_heavy+1]: segment range of heavy row
   Pinned bins_stage;                    // pinned staging of the bins' upload (build_bins)
-  // hot-row panel (spmm.cu build_hot): the hot_max most referenced columns
-  // encoded as -(rank+1) in a second column stream; hot_ids[rank] = vertex
+  // column relabelling (spmm.cu build_hot): col_hot[j] = rank of col[j] by
+  // reference count, hot_ids[rank] = vertex (hot_max = number of columns)
   int64_t hot_max = 0;
   std::unique_ptr<DevBuf> col_hot, hot_ids;
   int64_t max_deg = 0;
@@ -317,7 +321,8 @@ bool build_hub_tiles(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, const int
                      const float* val_host);
 // np = pieces of s⊙X: kPiecesI8 = three int8 digits on kind::i8 (fp32-class default), 2 fp16
 // (RDM_TILE_PIECES=2), 3 bf16 (RDM_TILE_PIECES=3) or 1 bf16 (RDM_PREC_FAST).
-constexpr int kPiecesI8 = 8;
+constexpr int kPiecesI8 = 8;     // three int8 digits (23-bit fixed point per column)
+constexpr int kPiecesI8x2 = 9;   // two int8 digits (15-bit fixed point): the fast variant
 bool hub_tiles_pay(const Core& c, int64_t w, int np);
 void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx, int64_t w,
                        float* part, int64_t ldp, int np);
@@ -356,6 +361,18 @@ void pack_rows(rdm_ctx* ctx, const float* row_slice, int64_t ld_row, int64_t row
                const BlockTable& t);
 void unpack_rows(rdm_ctx* ctx, float* row_slice, int64_t ld_row, int64_t rows, int P,
                  const BlockTable& t);
+// bf16 wire of the executor's redistributions under RDM_PREC_FAST (redist.cu):
+// pack / unpack with bf16 blocks (the self block stays in fp32, bf16-rounded),
+// and the column-slice conversions of the staged side (rows [skip_lo, skip_hi)
+// are the self block and are not touched).
+void pack_rows_bf16(rdm_ctx* ctx, const float* row_slice, int64_t ld_row, int64_t rows, int P, int self,
+                    const BlockTable& t, float* self_dst, int64_t ld_self);
+void unpack_rows_bf16(rdm_ctx* ctx, float* row_slice, int64_t ld_row, int64_t rows, int P, int self,
+                      const BlockTable& t, const float* self_src, int64_t ld_self);
+void narrow_cols(rdm_ctx* ctx, const float* col, int64_t n, int64_t ld, int64_t skip_lo, int64_t skip_hi,
+                 void* stage);
+void widen_cols(rdm_ctx* ctx, const void* stage, int64_t n, int64_t ld, int64_t skip_lo, int64_t skip_hi,
+                float* col);
 // Unfused form of a Scatter (producers without a fused epilogue): copies the
 // rows x cols slice `src` into the destinations the descriptor names.
 void scatter_slice(rdm_ctx* ctx, const float* src, int64_t lds, int64_t rows, int64_t cols,
@@ -405,7 +422,7 @@ void allreduce_d(rdm_ctx* ctx, double* const* bufs, int64_t count);
 
 // redistribution on all local slots (used by rdm_redistribute and the executor)
 void redistribute(rdm_ctx* ctx, rdm_layout from, const float* const* src, float* const* dst,
-                  int64_t n, int64_t f);
+                  int64_t n, int64_t f, bool bf16_wire = false);
 
 // ------------------------------------------------------------------- plan
 int64_t config_to_id(const rdm_config& c);

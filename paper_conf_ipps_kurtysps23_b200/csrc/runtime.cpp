@@ -231,9 +231,105 @@ void allreduce_d(rdm_ctx* ctx, double* const* bufs, int64_t count) {
 }
 
 // ---------------------------------------------------------- redistribution
-void redistribute(rdm_ctx* ctx, rdm_layout from, const float* const* src, float* const* dst,
-                  int64_t n, int64_t f) {
+// RDM_PREC_FAST inside the executor: the same exchange
+// with bf16 blocks on the wire (half the bytes of L142's (P−1)/P·N·f).  Both
+// sides stage: row→col packs bf16 blocks and the receiver widens its staged
+// column slice; col→row narrows the sender's column slice and the receiver
+// unpacks bf16 blocks.  Every moved value, and the self block, is rounded
+// once to bf16 (the fast variant's 2e-2 gate; the public rdm_redistribute
+// stays bit-exact fp32).
+static void redistribute_bf16(rdm_ctx* ctx, rdm_layout from, const float* const* src, float* const* dst,
+                              int64_t n, int64_t f) {
   const int P = ctx->world;
+  const int64_t ld_row = roundup4(f);
+  std::vector<Range> rows(P), cols(P);
+  std::vector<int64_t> ldc(P);
+  for (int q = 0; q < P; ++q) {
+    rows[q] = row_range(n, P, q);
+    cols[q] = col_range(f, P, q);
+    ldc[q] = roundup4(cols[q].size());
+  }
+  const int nl = ctx->nlocal();
+  if ((int)ctx->ws_send.size() < nl) {
+    ctx->ws_send.resize(nl);
+    ctx->ws_recv.resize(nl);
+  }
+  std::vector<Xfer> x(nl);
+  std::vector<BlockTable> bt(nl);
+  std::vector<uint16_t*> rowstage(nl), colstage(nl);
+  int64_t payload = 0, wire = 0;
+  for (int i = 0; i < nl; ++i) {
+    const int p = ctx->local[i];
+    const int64_t rp = rows[p].size();
+    auto& rs = from == RDM_ROW ? ctx->ws_send[i] : ctx->ws_recv[i];   // row-side staging: P blocks
+    auto& cs = from == RDM_ROW ? ctx->ws_recv[i] : ctx->ws_send[i];   // column-side staging: N x ld_p
+    rowstage[i] = reinterpret_cast<uint16_t*>(ensure_ws(rs, (size_t)std::max<int64_t>(rp * ld_row, 1) * 2 + 64));
+    colstage[i] = reinterpret_cast<uint16_t*>(ensure_ws(cs, (size_t)std::max<int64_t>(n * ldc[p], 1) * 2 + 64));
+    int64_t off = 0;
+    for (int q = 0; q < P; ++q) {
+      bt[i].col_lo[q] = cols[q].lo;
+      bt[i].width[q] = cols[q].size();
+      bt[i].ld[q] = ldc[q];
+      uint16_t* blk = rowstage[i] + off;
+      off += rp * ldc[q];
+      bt[i].dst[q] = reinterpret_cast<float*>(blk);
+      bt[i].src[q] = reinterpret_cast<const float*>(blk);
+      uint16_t* cblk = colstage[i] + rows[q].lo * ldc[p];
+      if (from == RDM_ROW) {
+        x[i].send[q] = blk;
+        x[i].send_bytes[q] = (q == p) ? 0 : rp * ldc[q] * 2;
+        x[i].recv[q] = cblk;
+        x[i].recv_bytes[q] = (q == p) ? 0 : rows[q].size() * ldc[p] * 2;
+        if (q != p) payload += rp * cols[q].size();
+      } else {
+        x[i].send[q] = cblk;
+        x[i].send_bytes[q] = (q == p) ? 0 : rows[q].size() * ldc[p] * 2;
+        x[i].recv[q] = blk;
+        x[i].recv_bytes[q] = (q == p) ? 0 : rp * ldc[q] * 2;
+        if (q != p) payload += rows[q].size() * cols[p].size();
+      }
+      wire += x[i].send_bytes[q];
+    }
+  }
+  if (from == RDM_ROW) {
+    {
+      Phase ph(ctx, RDM_PH_PACK);
+      for (int i = 0; i < nl; ++i) {
+        const int p = ctx->local[i];
+        pack_rows_bf16(ctx, src[i], ld_row, rows[p].size(), P, p, bt[i], dst[i] + rows[p].lo * ldc[p], ldc[p]);
+      }
+    }
+    exchange(ctx, x);
+    Phase ph(ctx, RDM_PH_PACK);
+    for (int i = 0; i < nl; ++i) {
+      const int p = ctx->local[i];
+      widen_cols(ctx, colstage[i], n, ldc[p], rows[p].lo, rows[p].hi, dst[i]);
+    }
+  } else {
+    {
+      Phase ph(ctx, RDM_PH_PACK);
+      for (int i = 0; i < nl; ++i) {
+        const int p = ctx->local[i];
+        narrow_cols(ctx, src[i], n, ldc[p], rows[p].lo, rows[p].hi, colstage[i]);
+      }
+    }
+    exchange(ctx, x);
+    Phase ph(ctx, RDM_PH_PACK);
+    for (int i = 0; i < nl; ++i) {
+      const int p = ctx->local[i];
+      unpack_rows_bf16(ctx, dst[i], ld_row, rows[p].size(), P, p, bt[i], src[i] + rows[p].lo * ldc[p], ldc[p]);
+    }
+  }
+  ctx->counters.a2a_calls++;
+  ctx->counters.a2a_elems_payload += payload;
+  ctx->counters.a2a_bytes_wire += wire;
+  ctx->counters.a2a_width_units += f;
+}
+
+void redistribute(rdm_ctx* ctx, rdm_layout from, const float* const* src, float* const* dst,
+                  int64_t n, int64_t f, bool bf16_wire) {
+  const int P = ctx->world;
+  if (bf16_wire && P > 1) return redistribute_bf16(ctx, from, src, dst, n, f);
   const int64_t ld_row = roundup4(f);
   if (P == 1) {
     if (src[0] != dst[0] && n * ld_row != 0)

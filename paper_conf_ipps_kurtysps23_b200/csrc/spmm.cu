@@ -122,24 +122,16 @@ __device__ __forceinline__ float4 apply_epi(float4 a, const Epi& e, int64_t row,
   return a;
 }
 
-// Hot-row panel (DRAM-resident slices): the residual CSR's column stream
-// `col_hot` encodes the columns of the hot_max most referenced vertices as
-// -(rank+1); per call the rows of the hw hottest are copied into a compact
-// panel xh (contiguous, full 128-byte lines, kept in L2 by an access-policy
-// window), ranks in [hw, hot_max) read X at ids[rank].  hw == 0: off.
+// Column-relabelled SpMM of DRAM-resident slices (see rank_panel): the input
+// slice is gathered into rank order X'[r] = X[order[r]] (vertices ranked by
+// how often the CSR references them) and the kernel streams a column array of
+// ranks, so the hottest rows are contiguous (full 128-byte lines, one L2-sized
+// prefix).  hw == 0: off (plain column ids into X).
 struct Hot {
-  const float* xh;        // hw x ldh (chunk offset applied by the kernel)
-  const int32_t* ids;     // vertex of each hot rank
+  const float* xh;        // N x ldh, rank order
   int64_t ldh;
   int hw;
 };
-
-__device__ __forceinline__ const float* row_ptr(const float* xb, int64_t ldx, int cc, const Hot& h,
-                                                int64_t cbase) {
-  if (cc >= 0) return xb + (int64_t)cc * ldx;
-  const int r = -cc - 1;
-  return r < h.hw ? h.xh + cbase + (int64_t)r * h.ldh : xb + (int64_t)__ldg(h.ids + r) * ldx;
-}
 
 // Warp computes Σ_{j in [beg,end)} val[j] · X[col[j], chunk columns].  A group
 // of G lanes owns one nnz at a time; lane `sub` of the group loads float4
@@ -153,7 +145,7 @@ __device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
                                                const float* __restrict__ val,
                                                const float* __restrict__ xb, int64_t ldx,
                                                int64_t beg, int64_t end, int lane, int c4n,
-                                               float4 (&acc)[V], const Hot& hot, int64_t cbase) {
+                                               float4 (&acc)[V]) {
   constexpr int NG = 32 / G;
   static_assert(G % U == 0, "U must divide G");
   const int g = lane / G, sub = lane % G;
@@ -179,7 +171,7 @@ __device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
         const int cc = (G == 1) ? c : __shfl_sync(kFull, c, k);
         const float vv = (G == 1) ? a : __shfl_sync(kFull, a, k);
         if (k < cnt) {
-          const float4* xr = reinterpret_cast<const float4*>(row_ptr(xb, ldx, cc, hot, cbase));
+          const float4* xr = reinterpret_cast<const float4*>(xb + (int64_t)cc * ldx);
           float4 x[V];
 #pragma unroll
           for (int v = 0; v < V; ++v)
@@ -206,8 +198,7 @@ __device__ __forceinline__ void warp_nnz_range(const int32_t* __restrict__ col,
         const int k = (t0 + u) * NG + g;
         const int cc = (G == 1) ? c : __shfl_sync(kFull, c, k);
         vv[u] = (G == 1) ? a : __shfl_sync(kFull, a, k);
-        const float4* xr = reinterpret_cast<const float4*>(
-            k < cnt ? row_ptr(xb, ldx, cc, hot, cbase) : xb);
+        const float4* xr = reinterpret_cast<const float4*>(xb + (int64_t)cc * ldx);
 #pragma unroll
         for (int v = 0; v < V; ++v)
           x[u][v] = (k < cnt && v * G + sub < c4n) ? RDM_GATHER_LD(xr + v * G + sub) : make_float4(0.f, 0.f, 0.f, 0.f);
@@ -253,7 +244,7 @@ spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
             const int64_t* __restrict__ seg_start, const int32_t* __restrict__ seg_row,
             int64_t n_light, int64_t n_seg, const float* __restrict__ X, int64_t ldx,
             float* __restrict__ out, int64_t ld_out, float* __restrict__ part, int64_t ld_part,
-            int64_t w4, int chunk4, Epi epi, Hot hot) {
+            int64_t w4, int chunk4, Epi epi) {
   const int lane = threadIdx.x & 31;
   const int64_t item = (int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5);
   if (item >= n_seg + n_light) return;
@@ -267,7 +258,7 @@ spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
     r = seg_row[item];
     const int64_t beg = seg_start[item];
     const int64_t end = min(beg + kSeg, rowptr[r + 1]);
-    warp_nnz_range<G, V, U>(col, val, X + cbase, ldx, beg, end, lane, c4n, acc, hot, cbase);
+    warp_nnz_range<G, V, U>(col, val, X + cbase, ldx, beg, end, lane, c4n, acc);
     if (lane < G) {
       float* dst = part + item * ld_part + cbase;
 #pragma unroll
@@ -276,7 +267,7 @@ spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
     }
   } else {
     r = light_rows[item - n_seg];
-    warp_nnz_range<G, V, U>(col, val, X + cbase, ldx, rowptr[r], rowptr[r + 1], lane, c4n, acc, hot, cbase);
+    warp_nnz_range<G, V, U>(col, val, X + cbase, ldx, rowptr[r], rowptr[r + 1], lane, c4n, acc);
     if (lane < G) {
       float* dst = out + (int64_t)r * ld_out + cbase;
 #pragma unroll
@@ -288,6 +279,71 @@ spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
           if (epi.scat.P) scatter_row_store(epi.scat, r, cbase + 4 * ch, o);
         }
       }
+    }
+  }
+}
+
+// Short light rows (degree <= the short threshold, the suffix of the
+// descending-degree light-row list): a group of G lanes per ROW, 32/G rows
+// per warp, U entries of its row in flight per group — short rows leave most
+// of a warp-per-row idle and serialise the rowptr → col → gather chain
+// (papers100M-shaped: average degree 15).  Same epilogue and stores.
+template <int G, int V, int U>
+__global__ void __launch_bounds__(kWarps * 32)
+spmm_short_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
+                  const float* __restrict__ val, const int32_t* __restrict__ rows, int64_t n_rows,
+                  const float* __restrict__ X, int64_t ldx, float* __restrict__ out, int64_t ld_out,
+                  int64_t w4, int chunk4, Epi epi) {
+  constexpr int R = 32 / G;
+  const int lane = threadIdx.x & 31;
+  const int g = lane / G, sub = lane % G;
+  const int64_t idx = ((int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5)) * R + g;
+  const int64_t cbase = (int64_t)blockIdx.y * chunk4 * 4;
+  const int64_t rem4 = (w4 - cbase) / 4;
+  const int c4n = rem4 < chunk4 ? (int)rem4 : chunk4;
+  const bool live = idx < n_rows;
+  const int32_t r = live ? rows[idx] : 0;
+  const int64_t beg = live ? rowptr[r] : 0, end = live ? rowptr[r + 1] : 0;
+  const float* xb = X + cbase;
+  float4 acc[V];
+#pragma unroll
+  for (int v = 0; v < V; ++v) acc[v] = make_float4(0.f, 0.f, 0.f, 0.f);
+  for (int64_t j = beg; j < end; j += U) {
+    int c[U];
+    float a[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const bool ok = j + u < end;
+      c[u] = ok ? __ldcs(col + j + u) : 0;
+      a[u] = ok ? __ldcs(val + j + u) : 0.f;
+    }
+    float4 x[U][V];
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+#pragma unroll
+      for (int v = 0; v < V; ++v)
+        x[u][v] = (j + u < end && v * G + sub < c4n)
+                      ? RDM_GATHER_LD(reinterpret_cast<const float4*>(xb + (int64_t)c[u] * ldx) + v * G + sub)
+                      : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        acc[v].x = fmaf(a[u], x[u][v].x, acc[v].x);
+        acc[v].y = fmaf(a[u], x[u][v].y, acc[v].y);
+        acc[v].z = fmaf(a[u], x[u][v].z, acc[v].z);
+        acc[v].w = fmaf(a[u], x[u][v].w, acc[v].w);
+      }
+  }
+  if (!live) return;
+  float* dst = out + (int64_t)r * ld_out + cbase;
+#pragma unroll
+  for (int v = 0; v < V; ++v) {
+    const int ch = v * G + sub;
+    if (ch < c4n) {
+      const float4 o = apply_epi(acc[v], epi, r, cbase + 4 * ch);
+      reinterpret_cast<float4*>(dst)[ch] = o;
+      if (epi.scat.P) scatter_row_store(epi.scat, r, cbase + 4 * ch, o);
     }
   }
 }
@@ -489,16 +545,32 @@ __global__ void spmm_heavy_reduce(const int32_t* __restrict__ heavy_rows,
 template <int G, int V, int U>
 void launch_spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out,
                  int64_t ld_out, float* part, int64_t ld_part, int64_t w4, int chunk4,
-                 const Epi& epi, const Hot& hot) {
-  const int64_t items = A.n_seg + A.n_light;
+                 const Epi& epi, const Hot& hot, int64_t n_long) {
+  const int64_t items = A.n_seg + n_long;
   if (items == 0) return;
   const int64_t chunks = ceil_div(w4, 4 * chunk4);
   dim3 grid((unsigned)ceil_div(items, kWarps), (unsigned)chunks);
   spmm_kernel<G, V, U><<<grid, kWarps * 32, 0, ctx->stream>>>(
       A.rowptr->as<int64_t>(), hot.hw ? A.col_hot->as<int32_t>() : A.col->as<int32_t>(), A.val->as<float>(),
       A.light_rows->as<int32_t>(), A.seg_start->as<int64_t>(),
-      reinterpret_cast<const int32_t*>(A.seg_start->as<int64_t>() + A.n_seg), A.n_light, A.n_seg,
-      in, ld_in, out, ld_out, part, ld_part, w4, chunk4, epi, hot);
+      reinterpret_cast<const int32_t*>(A.seg_start->as<int64_t>() + A.n_seg), n_long, A.n_seg,
+      hot.hw ? hot.xh : in, hot.hw ? hot.ldh : ld_in, out, ld_out, part, ld_part, w4, chunk4, epi);
+  RDM_LAUNCHED(ctx);
+}
+
+// The short light rows [n_long, n_light) of the light-row list.
+template <int G, int V, int U>
+void launch_spmm_short(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
+                       int64_t w4, int chunk4, const Epi& epi, const Hot& hot, int64_t n_long) {
+  const int64_t n_short = A.n_light - n_long;
+  if (n_short <= 0) return;
+  constexpr int R = 32 / G;
+  const int64_t chunks = ceil_div(w4, 4 * chunk4);
+  dim3 grid((unsigned)ceil_div(n_short, (int64_t)kWarps * R), (unsigned)chunks);
+  spmm_short_kernel<G, V, U><<<grid, kWarps * 32, 0, ctx->stream>>>(
+      A.rowptr->as<int64_t>(), hot.hw ? A.col_hot->as<int32_t>() : A.col->as<int32_t>(), A.val->as<float>(),
+      A.light_rows->as<int32_t>() + n_long, n_short, hot.hw ? hot.xh : in, hot.hw ? hot.ldh : ld_in, out, ld_out,
+      w4, chunk4, epi);
   RDM_LAUNCHED(ctx);
 }
 
@@ -551,9 +623,10 @@ void pick_gvu(int c, bool bf, int* G, int* V, int* U, bool dram_slice = false) {
   if (!bf) {
     // 9-12 vectors (w = 33..48): 8 lanes x 2 (profiles/r2_spmm_gvu.txt: w = 41 0.82 → 0.79 ms)
     if (c >= 9 && c <= 12) { *G = 8; *V = 2; }
-    // DRAM-resident slices (larger than L2): the gathers wait on DRAM, so narrow
-    // rows keep 4 nnz in flight per group (papers100M-shaped w = 16)
-    if (dram_slice && c <= 8) { *V = 1; *G = c <= 4 ? 4 : 8; *U = 4; }
+    // DRAM-resident slices of 5-8 vectors (products-shaped w = 32 at P = 8):
+    // 4 nnz in flight per group (2.61 → 2.46 ms); at <= 4 vectors U = 1 stays
+    // best (papers100M-shaped w = 16: U = 4 85 ms vs U = 1 77 ms, r2_relabel.md)
+    if (dram_slice && c >= 5 && c <= 8) { *V = 1; *G = 8; *U = 4; }
   }
   if (bf) {
     if (c >= 3 && c <= 8) { *G = 8; *V = 1; *U = 4; }
@@ -668,7 +741,9 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
   // (measured, tools/exp_tiles.py: fp16 pairs pay where the tile is MMA-bound,
   // w > 64: 1.53 → 1.44 ms at w = 128; narrower tiles are bound by the bit
   // expansion and the extra column-max pass makes fp16 pairs slower)
-  int np = ctx->prec == RDM_PREC_FAST ? 1 : kPiecesI8;
+  int np = ctx->prec == RDM_PREC_FAST ? kPiecesI8x2 : kPiecesI8;
+  if (ctx->prec == RDM_PREC_FAST)
+    if (const char* e = getenv("RDM_TILE_PIECES_FAST")) np = atoi(e) == 1 ? 1 : kPiecesI8x2;
   if (ctx->prec != RDM_PREC_FAST)
     if (const char* e = getenv("RDM_TILE_PIECES")) np = atoi(e) == 3 ? 3 : atoi(e) == 2 ? 2 : kPiecesI8;
   if (A.core.n_tiles && hub_tiles_pay(A.core, w, np)) {
@@ -706,69 +781,25 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
 }
 
 namespace {
-// xh[r] = X[ids[r]] for the hw hottest rows (float4 copies, full leading dim).
-__global__ void hot_gather_kernel(const float* __restrict__ X, int64_t ldx, const int32_t* __restrict__ ids,
-                                  int64_t hw, int64_t ld4, float* __restrict__ xh) {
-  const int64_t total = hw * ld4;
+// X'[r] = X[ids[r]] (float4 copies, full leading dim).
+__global__ void rank_gather_kernel(const float* __restrict__ X, int64_t ldx, const int32_t* __restrict__ ids,
+                                   int64_t n, int64_t ld4, float* __restrict__ xh) {
+  const int64_t total = n * ld4;
   for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total; i += (int64_t)gridDim.x * blockDim.x) {
     const int64_t r = i / ld4, c = i - r * ld4;
     reinterpret_cast<float4*>(xh)[i] = __ldg(reinterpret_cast<const float4*>(X + (int64_t)__ldg(ids + r) * ldx) + c);
   }
 }
 
-// L2 access-policy window on the hot panel for the duration of one SpMM
-// (persisting hits; cleared on scope exit).  RDM_HOT_PERSIST=0 disables.
-struct HotWindow {
-  rdm_ctx* ctx;
-  bool on = false;
-  explicit HotWindow(rdm_ctx* c) : ctx(c) {}
-  void set(void* base, size_t bytes) {
-    const char* e = getenv("RDM_HOT_PERSIST");
-    if (e && !atoi(e)) return;
-    static size_t limit = 0;
-    if (!limit) {
-      int dev = 0, maxp = 0;
-      cudaGetDevice(&dev);
-      cudaDeviceGetAttribute(&maxp, cudaDevAttrMaxPersistingL2CacheSize, dev);
-      limit = (size_t)maxp;
-      if (limit) cudaDeviceSetLimit(cudaLimitPersistingL2CacheSize, limit);
-      (void)cudaGetLastError();
-    }
-    if (!limit) return;
-    cudaStreamAttrValue v{};
-    v.accessPolicyWindow.base_ptr = base;
-    v.accessPolicyWindow.num_bytes = std::min(bytes, limit);
-    v.accessPolicyWindow.hitRatio = 1.0f;
-    v.accessPolicyWindow.hitProp = cudaAccessPropertyPersisting;
-    v.accessPolicyWindow.missProp = cudaAccessPropertyStreaming;
-    on = cudaStreamSetAttribute(ctx->stream, cudaStreamAttributeAccessPolicyWindow, &v) == cudaSuccess;
-    (void)cudaGetLastError();
-  }
-  ~HotWindow() {
-    if (!on) return;
-    cudaStreamAttrValue v{};
-    v.accessPolicyWindow.num_bytes = 0;
-    cudaStreamSetAttribute(ctx->stream, cudaStreamAttributeAccessPolicyWindow, &v);
-    cudaCtxResetPersistingL2Cache();
-    (void)cudaGetLastError();
-  }
-};
-
-// Per call: how many hot rows fit the panel budget (RDM_HOT_MB, default 64 MB)
-// at this leading dim, their copy, and the window.
-Hot hot_panel(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, int64_t w4, HotWindow& win) {
-  (void)w4;
-  double mb = 64.0;
-  if (const char* e = getenv("RDM_HOT_MB")) mb = atof(e);
-  const int64_t hw = std::min<int64_t>(A.hot_max, (int64_t)(mb * 1048576.0 / (ld_in * 4.0)));
-  if (hw <= 0) return Hot{nullptr, nullptr, 0, 0};
-  float* xh = ensure_ws(ctx->ws_hot, (size_t)hw * ld_in * sizeof(float));
-  const int64_t total = hw * (ld_in / 4);
+// Per call: the input slice in rank order (one gather pass, 2·N·ld·4 bytes).
+Hot rank_panel(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in) {
+  const int64_t n = A.hot_max;
+  float* xh = ensure_ws(ctx->ws_hot, (size_t)n * ld_in * sizeof(float));
+  const int64_t total = n * (ld_in / 4);
   const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(total, 256), (int64_t)ctx->num_sms * 16));
-  hot_gather_kernel<<<grid, 256, 0, ctx->stream>>>(in, ld_in, A.hot_ids->as<int32_t>(), hw, ld_in / 4, xh);
+  rank_gather_kernel<<<grid, 256, 0, ctx->stream>>>(in, ld_in, A.hot_ids->as<int32_t>(), n, ld_in / 4, xh);
   RDM_LAUNCHED(ctx);
-  win.set(xh, (size_t)hw * ld_in * sizeof(float));
-  return Hot{xh, A.hot_ids->as<int32_t>(), ld_in, (int)hw};
+  return Hot{xh, ld_in, 1};
 }
 
 void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
@@ -829,12 +860,31 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
     int U = 1;
     const bool dram_slice = (double)A.in_rows() * (double)ld_in * 4.0 > 96e6;
     if (!getenv("RDM_SPMM_GV")) pick_gvu(c4, false, &G, &V, &U, dram_slice);
-    Hot hot{nullptr, nullptr, 0, 0};
-    HotWindow window(ctx);
-    if (dram_slice && A.col_hot) hot = hot_panel(ctx, A, in, ld_in, w4, window);
+    Hot hot{nullptr, 0, 0};
+    const char* rl = getenv("RDM_RELABEL");   // column relabelling of DRAM-resident slices (experiment)
+    if (dram_slice && A.col_hot && !(rl && !atoi(rl))) hot = rank_panel(ctx, A, in, ld_in);
+    // short light rows (degree <= RDM_SPMM_SHORT, default 32) → row-per-group kernel
+    int short_deg = 32;
+    if (const char* e = getenv("RDM_SPMM_SHORT")) short_deg = std::max(0, std::min(Csr::kDegTab, atoi(e)));
+    const int64_t n_long = short_deg > 0 ? A.deg_ge[short_deg + 1 <= Csr::kDegTab ? short_deg + 1 : Csr::kDegTab]
+                                         : A.n_light;
+    if (short_deg > 0) {
+      int sg, sv;
+      pick_gv(c4, &sg, &sv);
+#define RDM_SHORT_CASE(g_, v_) \
+  if (sg == g_ && sv == v_) launch_spmm_short<g_, v_, 2>(ctx, A, in, ld_in, out, ld_out, w4, chunk4, epi, hot, n_long); else
+      RDM_SHORT_CASE(1, 1) RDM_SHORT_CASE(1, 2) RDM_SHORT_CASE(1, 3) RDM_SHORT_CASE(1, 4)
+      RDM_SHORT_CASE(2, 1) RDM_SHORT_CASE(2, 2) RDM_SHORT_CASE(2, 3) RDM_SHORT_CASE(2, 4)
+      RDM_SHORT_CASE(4, 1) RDM_SHORT_CASE(4, 2) RDM_SHORT_CASE(4, 3) RDM_SHORT_CASE(4, 4)
+      RDM_SHORT_CASE(8, 1) RDM_SHORT_CASE(8, 2) RDM_SHORT_CASE(8, 3) RDM_SHORT_CASE(8, 4)
+      RDM_SHORT_CASE(16, 1) RDM_SHORT_CASE(16, 2) RDM_SHORT_CASE(16, 3) RDM_SHORT_CASE(16, 4)
+      RDM_SHORT_CASE(32, 1) RDM_SHORT_CASE(32, 2)
+      throw Error(RDM_ERR_ARG, "spmm: no short-row kernel for G/V");
+#undef RDM_SHORT_CASE
+    }
     if (const char* e = getenv("RDM_SPMM_U")) U = atoi(e);
 #define RDM_SPMM_CASE(g_, v_, u_) \
-  if (G == g_ && V == v_ && U == u_) launch_spmm<g_, v_, u_>(ctx, A, in, ld_in, out, ld_out, part, w4, w4, chunk4, epi, hot); else
+  if (G == g_ && V == v_ && U == u_) launch_spmm<g_, v_, u_>(ctx, A, in, ld_in, out, ld_out, part, w4, w4, chunk4, epi, hot, n_long); else
     RDM_SPMM_CASE(1, 1, 1) RDM_SPMM_CASE(1, 2, 1) RDM_SPMM_CASE(1, 3, 1) RDM_SPMM_CASE(1, 4, 1)
     RDM_SPMM_CASE(2, 1, 1) RDM_SPMM_CASE(2, 1, 2) RDM_SPMM_CASE(2, 2, 1) RDM_SPMM_CASE(2, 2, 2)
     RDM_SPMM_CASE(2, 3, 1) RDM_SPMM_CASE(2, 3, 2) RDM_SPMM_CASE(2, 4, 1) RDM_SPMM_CASE(2, 4, 2)
@@ -877,19 +927,23 @@ __global__ void hot_encode_kernel(const int32_t* __restrict__ col, int64_t nnz, 
   for (int64_t j = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; j < nnz; j += (int64_t)gridDim.x * blockDim.x) {
     const int32_t c = col[j];
     const int32_t r = rank[c];
-    out[j] = r >= 0 ? -r - 1 : c;
+    out[j] = r;   // every column has a rank
   }
 }
 }  // namespace
 
-// Hot-row panel (see Hot): built for CSRs whose input slice can exceed L2
-// (>= 1 M input rows) — RDM_NO_HOT=1 disables.  hot_max = min(rows, 8 M):
-// the per-call panel takes the hottest rows that fit its byte budget.
+// Column relabelling (see Hot) — an experiment, OFF by default: measured
+// slower on the products-shaped graph (w = 256: 8.7 → 9.7 ms per call, the
+// extra gather pass costs more than the locality gains) and ≈ 4 % faster on
+// the papers100M-shaped one-rank SpMM (profiles/r2_relabel.md).
+// RDM_RELABEL=1 at rdm_set_graph builds it for CSRs with >= 1 M input rows.
+// Columns ranked by reference count (stable, descending); col_hot[j] = rank
+// of col[j]; hot_ids = order.
 void build_hot(rdm_ctx* ctx, Csr& A) {
-  const char* off = getenv("RDM_NO_HOT");
+  const char* on = getenv("RDM_RELABEL");
   const int64_t nin = A.in_rows();
-  if ((off && atoi(off)) || A.nnz == 0 || nin < (1 << 20) || nin >= INT32_MAX) return;
-  const int64_t hmax = std::min<int64_t>(nin, 1 << 23);
+  if (!(on && atoi(on)) || A.nnz == 0 || nin < (1 << 20) || nin >= INT32_MAX) return;
+  const int64_t hmax = nin;   // every column ranked: the slice is gathered whole into rank order
   DevBuf cnt(nin * 4), iota(nin * 4), keys(nin * 4), order(nin * 4), rank(nin * 4);
   const unsigned g = (unsigned)(ctx->num_sms * 8);
   RDM_CUDA(cudaMemsetAsync(cnt.ptr, 0, nin * 4, ctx->stream));
@@ -967,6 +1021,14 @@ void build_bins(rdm_ctx* ctx, Csr& A, const int64_t* rp, bool sync) {
   }
   heavy_seg[n_heavy] = (int32_t)s;
   A.n_light = n_light;
+  {
+    // cnt[kSeg - d] = light rows of degree d
+    int64_t acc = 0;
+    for (int d = (int)kSeg; d >= 0; --d) {
+      acc += cnt[kSeg - d];
+      if (d <= Csr::kDegTab) A.deg_ge[d] = acc;
+    }
+  }
   A.n_seg = n_seg;
   A.n_heavy = n_heavy;
   A.max_deg = max_deg;

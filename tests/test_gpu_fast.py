@@ -130,10 +130,16 @@ def test_fast_spmm_is_bf16_input_fp32_accumulate(torch_dev, rdm, gname, w, monke
 
 @pytest.mark.parametrize("w", [4, 16, 41, 128, 256])
 @pytest.mark.parametrize("min_nnz", [1, 40])
-def test_fast_spmm_hub_tiles(torch_dev, rdm, w, min_nnz, monkeypatch):
-    """One bf16 piece of s⊙X on the kind::f16 tensor cores + bf16 residual CSR."""
+@pytest.mark.parametrize("form", ["i8x2", "bf16"])
+def test_fast_spmm_hub_tiles(torch_dev, rdm, w, min_nnz, form, monkeypatch):
+    """Fast variant tiles: two int8 digits of a 15-bit per-column fixed point of
+    s⊙X on kind::i8 (default) or one bf16 piece on kind::f16
+    (RDM_TILE_PIECES_FAST=1), + the bf16 residual CSR, within the 2e-2 gate
+    (measured ≈ 1e-3, the residual's bf16 rows)."""
     torch, dev = torch_dev
     monkeypatch.setenv("RDM_TILE_MIN_NNZ", str(min_nnz))
+    if form == "bf16":
+        monkeypatch.setenv("RDM_TILE_PIECES_FAST", "1")
     g = synth.rmat(6000, 150000, seed=13)
     ctx = rdm.Context(device=0)
     ctx.set_precision("fast")
@@ -220,3 +226,34 @@ def test_precision_rejects_unknown(rdm):
     ctx = rdm.Context(device=0)
     with pytest.raises(rdm.RdmError):
         ctx._c(rdm._lib.rdm_set_precision(ctx.h, 7))
+
+
+@pytest.mark.parametrize("P,cfg", [(2, 3), (4, 10), (3, 5), (8, 2)])
+def test_fast_bf16_wire_halves_bytes(rdm, cora, P, cfg):
+    """RDM_PREC_FAST: the executor's row → column redistributions carry bf16
+    (NEXT-3): their bytes on the wire halve against the fp32 variant exactly
+    (the per-redistribution wire bytes from rdm_redist_plan), column → row
+    moves keep fp32, the payload element count is unchanged, and the epoch
+    stays within the 2e-2 gate with the loss within 1e-5."""
+    g, H0, Ws, y, m = cora
+    _, _, _, ctx32, _ = _run(rdm, g, H0, Ws, y, m, cfg, P=P)
+    c32 = ctx32.counters()
+    loss, dW, model, ctx, _ = _run(rdm, g, H0, Ws, y, m, cfg, P=P, precision="fast")
+    c16 = ctx.counters()
+    assert c16["a2a_elems_payload"] == c32["a2a_elems_payload"]
+    assert c16["a2a_width_units"] == c32["a2a_width_units"]
+    f = [H0.shape[1]] + [w.shape[1] for w in Ws]
+    _, desc = rdm.plan_info(f, cfg, P, g.n)
+    want32 = want16 = 0
+    for line in desc.splitlines():
+        if not line.strip().startswith("A2A"):
+            continue
+        w = int(line.split("f=")[1].split()[0])
+        fr = rdm.ROW if ".row ->" in line else rdm.COL
+        b = sum(4 * sum(pl["send_elems"][q] for q in range(P) if q != p)
+                for p in range(P) for pl in [rdm.redist_plan(P, p, fr, g.n, w)])
+        want32 += b
+        want16 += b // 2 if fr == rdm.ROW else b
+    assert c32["a2a_bytes_wire"] == want32
+    assert c16["a2a_bytes_wire"] == want16 < want32
+    _check((g, H0, Ws, y, m), loss, dW, model, rdm, P=P, tol=GATE, ltol=LOSS_GATE)
