@@ -804,14 +804,19 @@ def main():
     alg_bytes = spmm_calls * (8 * nnz + 8 * (n + 1)) + 8 * n * sum_w
     spmm_s = ph_ms["spmm"] / 1e3
     achieved = alg_bytes / spmm_s / 1e9 if spmm_s > 0 else 0.0
-    # traffic: DRAM bytes per SpMM launch from the committed ncu --set full capture
+    # traffic: DRAM bytes per SpMM call from the committed ncu --set full capture
+    # (profiles/r2_spmm_traffic.json, per width), averaged over this epoch's calls
     traffic, traffic_src = None, None
     try:
-        tj = _json.load(open(os.path.join(ROOT, "profiles", "r1_spmm_traffic.json")))
-        if a.workload == "reddit" and world == 1 and a.precision == "fp32" and not panels:
-            ls = tj["calls"]   # one w = 128 and one w = 41 call: the epoch has two of each
-            traffic = sum(x["dram_bytes"] for x in ls) / len(ls) / 1e9
-            traffic_src = tj["source"]
+        tj = _json.load(open(os.path.join(ROOT, "profiles", "r2_spmm_traffic.json")))
+        rec = tj.get(wl.name)
+        if rec and world == 1 and a.precision == "fp32" and not panels:
+            _, desc = rdm.plan_info(list(wl.f), cfg_id, 1, n)
+            ws = [int(l.split("w=")[1].split()[0]) for l in desc.splitlines() if l.strip().startswith("SPMM")]
+            per = rec["per_width_gb"]
+            if ws and all(f"w{w}" in per for w in ws):
+                traffic = sum(per[f"w{w}"] for w in ws) / len(ws)
+                traffic_src = rec["source"]
     except Exception:
         pass
     roofline = {"bound": "hbm", "achieved": achieved, "peak": hbm_peak, "unit": "GB/s",

@@ -437,6 +437,10 @@ struct rdm_gcn {
   bool side_pending = false;
   std::unique_ptr<rdm::DevBuf> ws_side;   // split-K partials of the side-stream TN
   int64_t gver = -1;
+  // (tensor, layout) whose current contents arrived over the bf16 wire (fast
+  // variant): an SpMM reading them uses them as the bf16 values they are
+  // (no second rounding of s_j·x_j, rdm_ctx::spmm_in_bf16)
+  std::set<std::pair<int, int>> wire_bf16;
 };
 
 namespace rdm {
@@ -645,6 +649,10 @@ void create(rdm_gcn* g) {
 
 void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
   rdm_ctx* ctx = g->ctx;
+  // any producer but the bf16-wire redistribution (and the in-place mask,
+  // which keeps bf16 values bf16) leaves fp32 values in its output
+  if (s.op == S_SPMM || s.op == S_GEMM || s.op == S_LOSS || s.op == S_REDIST)
+    g->wire_bf16.erase({s.out.id(), norm_lay(g, s.lout)});
   const int nl = ctx->nlocal();
   const int P = ctx->world;
   // a fused producer overwrites peers' destination slices: every rank must be
@@ -677,12 +685,14 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
           ldm = m.ld;
         }
         const int64_t w = P == 1 ? s.width : col_range(s.width, P, ctx->local[i]).size();
+        ctx->spmm_in_bf16 = g->wire_bf16.count({s.in.id(), norm_lay(g, s.lin)}) > 0;
         if (s.fuse == 1) {
           const Scatter sc = make_scatter(g, s, i);
           spmm(ctx, A, in.p, in.ld, out.p, out.ld, w, s.epi, nullptr, mk, ldm, &sc);
         } else {
           spmm(ctx, A, in.p, in.ld, out.p, out.ld, w, s.epi, nullptr, mk, ldm);
         }
+        ctx->spmm_in_bf16 = false;
       }
       ctx->counters.spmm_width_units += s.width;
       break;
@@ -748,9 +758,9 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
         // anyway; column → row moves (SpMM outputs feeding GEMMs and the loss)
         // stay fp32.  RDM_BF16_WIRE=0 disables (experiments).
         const char* wv = getenv("RDM_BF16_WIRE");
-        const bool wire_off = wv && !atoi(wv);
-        redistribute(ctx, (rdm_layout)s.lin, src.data(), dst.data(), gn(g), s.width,
-                     ctx->prec == RDM_PREC_FAST && s.lin == RDM_ROW && !wire_off);
+        const bool wire = ctx->prec == RDM_PREC_FAST && s.lin == RDM_ROW && P > 1 && !(wv && !atoi(wv));
+        redistribute(ctx, (rdm_layout)s.lin, src.data(), dst.data(), gn(g), s.width, wire);
+        if (wire) g->wire_bf16.insert({s.out.id(), norm_lay(g, s.lout)});
       }
       break;
     }

@@ -568,7 +568,10 @@ void launch_tc_ew(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, cons
   sh.dbg = dbg ? atoi(dbg) : 0;
   sh.one = ctx->prec == RDM_PREC_FAST ? 1 : 0;
   // TMA-store epilogue: plain row-major output (one split, no fused scatter)
-  sh.tstore = (MODE == 0 && splits == 1 && !e.scat.P && !(getenv("RDM_NO_TSTORE") && atoi(getenv("RDM_NO_TSTORE"))))
+  // (TMA needs a 16-byte aligned base and a row pitch that is a multiple of
+  // 16 bytes; other outputs take the transpose-and-store path)
+  sh.tstore = (MODE == 0 && splits == 1 && !e.scat.P && ((uintptr_t)C & 15) == 0 && (ldc & 3) == 0 &&
+               !(getenv("RDM_NO_TSTORE") && atoi(getenv("RDM_NO_TSTORE"))))
                   ? 1 : 0;
   const CUtensorMap tc = sh.tstore ? make_map(C, N, M, ldc, 32, 32) : a;
   const int64_t total = (int64_t)sh.tiles_m * sh.tiles_n * splits;

@@ -194,6 +194,7 @@ struct rdm_ctx {
   bool emulated = false;         // one rank of a P-rank job with no peers (rdm_init_emulated)
   int transport = 0;             // RDM_TRANSPORT_NCCL / RDM_TRANSPORT_P2P
   int prec = 0;                  // RDM_PREC_FP32 / RDM_PREC_FAST
+  bool spmm_in_bf16 = false;     // executor → spmm: the input holds bf16 values (bf16 wire)
   std::string err;
   rdm::Graph graph;
   bool has_graph = false;

@@ -33,7 +33,7 @@ ctx.set_graph(g.rowptr, g.col, g.val, symmetric=True)
 for (r, k, m) in ((1000, 64, 128), (1000, 128, 41), (700, 256, 256)):
     X = torch.randn(r, k, device=dev)
     W = torch.randn(k, m, device=dev)
-    C = torch.zeros(r, m, device=dev)
+    C = torch.zeros(r, (m + 3) // 4 * 4, device=dev)[:, :m]
     ctx.gemm(rdm.GEMM_NN, X, W, C, r, k, m)
     Ct = torch.zeros(r, k, device=dev)
     ctx.gemm(rdm.GEMM_NT, C, W, Ct, r, k, m)
