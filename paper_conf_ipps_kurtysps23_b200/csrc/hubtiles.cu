@@ -720,6 +720,193 @@ hub_tile_i8_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __re
   }
 }
 
+// Pair form of hub_tile_i8_kernel: a work unit is a run of merged entries
+// of a row-block PAIR (2p, 2p+1); each stage carries ONE digit-panel load for
+// the column block and both tiles' bits (a zero tile where a row block has
+// none), and the MMA issuer multiplies both A tiles against it into two
+// accumulators — half the panel ingress per tile.  TMEM: the two accumulators
+// (single-buffered: 2·D·n_mma columns) then SA slots of 64 columns (the two
+// expanded A tiles).  part holds 256 rows per item (rows 0-127: block 2p).
+template <int D>
+__global__ void __launch_bounds__(384, 1)
+hub_tile_i8_pair_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __restrict__ bits,
+                        const uint64_t* __restrict__ zero_bits, const int32_t* __restrict__ pm_cb,
+                        const int32_t* __restrict__ pm_t1, const int32_t* __restrict__ pm_t2,
+                        const int32_t* __restrict__ pitem_pm, float* __restrict__ part, const TileShape sh) {
+  extern __shared__ uint8_t smem_raw[];
+  uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
+  const int S = sh.S, SA = sh.SA, n_mma = sh.n_mma;
+  uint64_t* full = (uint64_t*)(smem + S * sh.stage_bytes);
+  uint64_t* empty = full + S;
+  uint64_t* conv = empty + S;
+  uint64_t* aempty = conv + SA;
+  uint64_t* tfull = aempty + SA;
+  uint64_t* tempty = tfull + 1;
+  uint32_t* tmem_slot = (uint32_t*)(tempty + 1);
+  const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
+  const int total = sh.n_items * sh.tiles_n;
+  const int bbytes = D * n_mma * 128;
+  const int accw = D * n_mma;                      // columns of one accumulator
+  auto B_st = [&](int s) { return smem + s * sh.stage_bytes; };
+  auto bits_st = [&](int s) { return smem + s * sh.stage_bytes + bbytes; };   // [tile 2][half 2][128] u64
+  if (threadIdx.x == 0) {
+    for (int i = 0; i < S; ++i) {
+      mbar_init(&full[i], 1);
+      mbar_init(&empty[i], 1);
+    }
+    for (int i = 0; i < SA; ++i) {
+      mbar_init(&conv[i], 128);
+      mbar_init(&aempty[i], 1);
+    }
+    mbar_init(&tfull[0], 1);
+    mbar_init(&tempty[0], 128);
+    asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
+  }
+  if (warp == 2) {
+    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                     smem_u32(tmem_slot)),
+                 "n"(512));
+    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+  }
+  tc_fence_before();
+  __syncthreads();
+  tc_fence_after();
+  const uint32_t tmem_base = *tmem_slot;
+  const uint32_t kAcol = (uint32_t)sh.acc_cols;     // both accumulators, rounded up
+
+  if (warp == 0) {
+    if (lane == 0) {
+      int s = 0;
+      uint32_t ph = 0, kc = 0;
+      const uint32_t bytes = (uint32_t)bbytes + 4096;
+      for (int t = blockIdx.x; t < total; t += gridDim.x) {
+        const int item = t / sh.tiles_n;
+        const int n0 = (t % sh.tiles_n) * n_mma;
+        const int mb = pitem_pm[item], M = pitem_pm[item + 1] - mb;
+        int mi = (int)(((unsigned)item * 2654435761u) % (unsigned)max(M, 1));
+        for (int i = 0; i < M; ++i) {
+          const int m = mb + mi;
+          if (++mi == M) mi = 0;
+          if (kc >= (uint32_t)S) mbar_wait(&empty[s], ph ^ 1);
+          mbar_expect_tx(&full[s], bytes);
+          const int t1 = pm_t1[m], t2 = pm_t2[m];
+          bulk_load(bits_st(s), t1 >= 0 ? bits + (int64_t)t1 * 2 * TK : zero_bits, 2048, &full[s]);
+          bulk_load(bits_st(s) + 2048, t2 >= 0 ? bits + (int64_t)t2 * 2 * TK : zero_bits, 2048, &full[s]);
+          tma_load_4d(B_st(s), &tmB, &full[s], 0, n0, 0, pm_cb[m]);
+          ++kc;
+          if (++s == S) { s = 0; ph ^= 1; }
+        }
+      }
+    }
+  } else if (warp == 1) {
+    if (lane == 0) {
+      const uint32_t idesc = idesc_i8(D * n_mma);
+      const uint64_t bd0 = sdesc(smem_u32(B_st(0)), 16, 1024);
+      const uint32_t st16 = (uint32_t)sh.stage_bytes >> 4;
+      int s = 0, a = 0;
+      uint32_t ph = 0, aph = 0;
+      int it = 0;
+      for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
+        const int item = t / sh.tiles_n;
+        const int nst = pitem_pm[item + 1] - pitem_pm[item];
+        if (it >= 1) mbar_wait(&tempty[0], (it - 1) & 1);   // single-buffered accumulators
+        tc_fence_after();
+        for (int st = 0; st < nst; ++st) {
+          mbar_wait(&conv[a], aph);
+          tc_fence_after();
+          const uint32_t ta = tmem_base + kAcol + a * 64;
+          const uint64_t bd = bd0 + (uint64_t)(s * st16);
+          if (!(sh.dbg & 1)) {
+#pragma unroll
+            for (int j = 0; j < TK / 32; ++j) {
+              const uint32_t acc = (st | j) ? 1u : 0u;
+              tc_mma_i8_ts(tmem_base, ta + j * 8, bd + 2 * j, idesc, acc);
+              tc_mma_i8_ts(tmem_base + (uint32_t)accw, ta + 32 + j * 8, bd + 2 * j, idesc, acc);
+            }
+          }
+          tc_commit(&empty[s]);
+          tc_commit(&aempty[a]);
+          if (++s == S) { s = 0; ph ^= 1; }
+          if (++a == SA) { a = 0; aph ^= 1; }
+        }
+        tc_commit(&tfull[0]);
+      }
+    }
+  } else if (warp >= 4 && warp < 8) {
+    const int r = threadIdx.x - 128;
+    const uint32_t lane_off = (uint32_t)((warp & 3) * 32) << 16;
+    int s = 0, a = 0;
+    uint32_t ph = 0, aph = 0, kc = 0;
+    for (int t = blockIdx.x; t < total; t += gridDim.x) {
+      const int item = t / sh.tiles_n;
+      const int nst = pitem_pm[item + 1] - pitem_pm[item];
+      for (int st = 0; st < nst; ++st, ++kc) {
+        mbar_wait(&full[s], ph);
+        if (kc >= (uint32_t)SA) {
+          mbar_wait(&aempty[a], aph ^ 1);
+          tc_fence_after();
+        }
+#pragma unroll
+        for (int tt = 0; tt < 2; ++tt) {
+          const uint32_t bs = smem_u32(bits_st(s)) + tt * 2048 + r * 8;
+          const uint2 h0 = lds64(bs), h1 = lds64(bs + 1024);
+          const uint32_t w4[4] = {h0.x, h0.y, h1.x, h1.y};
+          uint32_t v[32];
+#pragma unroll
+          for (int i = 0; i < 32; ++i) v[i] = (((w4[i >> 3] >> (4 * (i & 7))) & 15u) * 0x204081u) & 0x01010101u;
+          tmem_st32u(tmem_base + lane_off + kAcol + a * 64 + tt * 32, v);
+        }
+        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+        tc_fence_before();
+        mbar_arrive(&conv[a]);
+        if (++s == S) { s = 0; ph ^= 1; }
+        if (++a == SA) { a = 0; aph ^= 1; }
+      }
+    }
+  } else if (warp >= 8) {
+    const int q = warp & 3;
+    int it = 0;
+    for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
+      const int item = t / sh.tiles_n;
+      const int64_t n0 = (int64_t)(t % sh.tiles_n) * n_mma;
+      mbar_wait_sleep(&tfull[0], it & 1);
+      tc_fence_after();
+#pragma unroll 1
+      for (int tt = 0; tt < 2; ++tt) {
+        float* prow = part + ((int64_t)item * 2 * TK + tt * TK + q * 32 + lane) * sh.ldp + n0;
+        for (int c0 = 0; c0 < n_mma; c0 += 32) {
+          if (n0 + c0 >= sh.w) break;
+          uint32_t dg[D][32];
+          const uint32_t a0 = tmem_base + (uint32_t)(tt * accw) + ((uint32_t)(q * 32) << 16) + (uint32_t)c0;
+#pragma unroll
+          for (int d = 0; d < D; ++d) tmem_ld32(a0 + (uint32_t)(d * n_mma), dg[d]);
+#pragma unroll
+          for (int i = 0; i < 32; i += 4)
+            if (n0 + c0 + i < sh.w) {
+              const float4 cs = __ldg(reinterpret_cast<const float4*>(sh.colscale + n0 + c0 + i));
+              float o[4];
+#pragma unroll
+              for (int u = 0; u < 4; ++u) {
+                long long v = 0;
+#pragma unroll
+                for (int d = 0; d < D; ++d) v = v * 256 + (long long)(int)dg[d][i + u];
+                o[u] = __ll2float_rn(v);
+              }
+              *reinterpret_cast<float4*>(prow + c0 + i) = make_float4(o[0] * cs.x, o[1] * cs.y, o[2] * cs.z, o[3] * cs.w);
+            }
+        }
+      }
+      tc_fence_before();
+      mbar_arrive(&tempty[0]);
+    }
+  }
+  tc_fence_before();
+  __syncthreads();
+  if (warp == 2) {
+    asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base), "n"(512));
+  }
+}
+
 // int8 digit panels P_d[n][k] (row length K2 bytes; d = 0 the most
 // significant) of y = s_k · X[hub_k][n] · 2^-e_n: D = 3 digits with the column
 // maximum in [2^21, 2^22) (23-bit fixed point, fp32-class), D = 2 with it in
@@ -854,6 +1041,12 @@ double tile_s(int64_t w, int np = 3) {
 }
 }  // namespace
 
+// The int8 tiles run in row-block pairs unless RDM_TILE_PAIRS=0.
+bool tiles_paired() {
+  const char* e = getenv("RDM_TILE_PAIRS");
+  return !(e && !atoi(e));
+}
+
 bool hub_tiles_pay(const Core& c, int64_t w, int np) {
   if (!c.n_tiles) return false;
   if (c.forced) return true;
@@ -897,6 +1090,26 @@ void hub_tiles_product_i8(rdm_ctx* ctx, const Core& c, const float* X, int64_t l
   sh.colscale = cs;
   RDM_CHECK_ARG(sh.S >= 2 && sh.SA >= 2, "hub tiles (int8): TMEM/smem budget");
   const CUtensorMap tb = panel_map_i8(pan, K2, w, sh.n_mma, D);
+  if (tiles_paired()) {
+    // two row blocks per panel load (hub_tile_i8_pair_kernel)
+    TileShape ps = sh;
+    ps.n_items = (int)c.n_pitems;
+    ps.acc_cols = (2 * D * sh.n_mma + 31) / 32 * 32;
+    ps.stage_bytes = (D * sh.n_mma * 128 + 4096 + 1023) / 1024 * 1024;
+    ps.S = std::min(32, (kSmemBudget - 1024 - 1024) / ps.stage_bytes);
+    ps.SA = std::min(8, (512 - ps.acc_cols) / 64);
+    RDM_CHECK_ARG(ps.S >= 2 && ps.SA >= 2, "hub tiles (int8 pairs): TMEM/smem budget");
+    const int psmem = ps.S * ps.stage_bytes + 1024 + 1024;
+    const int64_t ptotal = c.n_pitems * ps.tiles_n;
+    const unsigned pgrid = (unsigned)std::min<int64_t>(ptotal, ctx->num_sms);
+    auto pk = D == 3 ? hub_tile_i8_pair_kernel<3> : hub_tile_i8_pair_kernel<2>;
+    RDM_CUDA(cudaFuncSetAttribute(pk, cudaFuncAttributeMaxDynamicSharedMemorySize, psmem));
+    pk<<<pgrid, 384, psmem, ctx->stream>>>(tb, c.tiles->as<uint64_t>(), c.zero_bits->as<uint64_t>(),
+                                           c.pm_cb->as<int32_t>(), c.pm_t1->as<int32_t>(),
+                                           c.pm_t2->as<int32_t>(), c.pitem_pm->as<int32_t>(), part, ps);
+    RDM_LAUNCHED(ctx);
+    return;
+  }
   const int smem = sh.S * sh.stage_bytes + 1024 + 1024;
   const int64_t total = c.n_items * sh.tiles_n;
   const unsigned grid = (unsigned)std::min<int64_t>(total, ctx->num_sms);
@@ -1205,6 +1418,41 @@ bool build_hub_tiles(rdm_ctx* ctx, Csr& A, const int64_t* rp, const int32_t* col
         ++o;
       }
   }
+  // pair items (int8 kernel): row blocks 2p and 2p+1 against ONE panel load
+  // per column block in the union of their tiles (merged in column order; a
+  // row block without a tile there multiplies a zero tile); runs of at most
+  // `chunk` merged entries, ≈ 4 items per SM
+  std::vector<int32_t> pm_cb, pm_t1, pm_t2, pitem_pm, pair_item;
+  {
+    const int64_t n_pairs = (c.n_rb + 1) / 2;
+    std::vector<int64_t> pm_first(n_pairs + 1, 0);
+    for (int64_t p = 0; p < n_pairs; ++p) {
+      pm_first[p] = (int64_t)pm_cb.size();
+      const int64_t r1 = 2 * p, r2 = 2 * p + 1;
+      int64_t i = rb_first[r1], ie = rb_first[r1 + 1];
+      int64_t j = r2 < c.n_rb ? rb_first[r2] : 0, je = r2 < c.n_rb ? rb_first[r2 + 1] : 0;
+      while (i < ie || j < je) {
+        const int32_t ci = i < ie ? tile_cb[i] : INT32_MAX, cj = j < je ? tile_cb[j] : INT32_MAX;
+        const int32_t cb = std::min(ci, cj);
+        pm_cb.push_back(cb);
+        pm_t1.push_back(ci == cb ? (int32_t)i++ : -1);
+        pm_t2.push_back(cj == cb ? (int32_t)j++ : -1);
+      }
+    }
+    pm_first[n_pairs] = (int64_t)pm_cb.size();
+    const int64_t pchunk = std::max<int64_t>(4, ceil_div((int64_t)pm_cb.size(), (int64_t)ctx->num_sms * 4));
+    pair_item.assign(n_pairs + 1, 0);
+    for (int64_t p = 0; p < n_pairs; ++p) {
+      pair_item[p] = (int32_t)pitem_pm.size();
+      const int64_t m0 = pm_first[p], M = pm_first[p + 1] - m0;
+      const int64_t nit = ceil_div(M, pchunk);
+      for (int64_t k = 0; k < nit; ++k) pitem_pm.push_back((int32_t)(m0 + M * k / nit));
+    }
+    pair_item[n_pairs] = (int32_t)pitem_pm.size();
+    c.n_pairs = n_pairs;
+    c.n_pitems = (int64_t)pitem_pm.size();
+    pitem_pm.push_back((int32_t)pm_cb.size());
+  }
   std::vector<float> sc(c.K2), sr(c.K2);
   for (int64_t k = 0; k < c.K2; ++k) {
     sc[k] = (float)cs[k];   // column scale of hub slot k (panels)
@@ -1221,6 +1469,15 @@ bool build_hub_tiles(rdm_ctx* ctx, Csr& A, const int64_t* rp, const int32_t* col
   up(c.rb_item, rb_item.data(), rb_item.size() * 4);
   up(c.scale, sc.data(), sc.size() * 4);
   up(c.rscale, sr.data(), sr.size() * 4);
+  up(c.pm_cb, pm_cb.data(), pm_cb.size() * 4);
+  up(c.pm_t1, pm_t1.data(), pm_t1.size() * 4);
+  up(c.pm_t2, pm_t2.data(), pm_t2.size() * 4);
+  up(c.pitem_pm, pitem_pm.data(), pitem_pm.size() * 4);
+  up(c.pair_item, pair_item.data(), pair_item.size() * 4);
+  {
+    std::vector<uint64_t> z(2 * TK, 0);
+    up(c.zero_bits, z.data(), z.size() * 8);
+  }
   up(c.hub_ids, order.data(), c.K2 * 4);
   up(c.hub_slot, slot.data(), n * 4);
   c.resid.reset(new Csr());

@@ -139,6 +139,12 @@ struct Core {
   std::unique_ptr<DevBuf> rb_item;     // int32[n_rb+1]: item range of each row block
   std::unique_ptr<DevBuf> scale;       // fp32[K2]: column scale c of the vertex of slot k (a_ij = r_i c_j)
   std::unique_ptr<DevBuf> rscale;      // fp32[K2]: row scale r of the vertex of slot k
+  // pair items (int8 kernel): row blocks 2p, 2p+1 merged by column block
+  int64_t n_pairs = 0, n_pitems = 0;
+  std::unique_ptr<DevBuf> pm_cb, pm_t1, pm_t2;   // int32[merged]: column block, tile of 2p / 2p+1 (-1 none)
+  std::unique_ptr<DevBuf> pitem_pm;              // int32[n_pitems+1]: merged range of each item
+  std::unique_ptr<DevBuf> pair_item;             // int32[n_pairs+1]: item range of each pair
+  std::unique_ptr<DevBuf> zero_bits;             // one all-zero tile (2 KB)
 };
 
 struct Csr {
@@ -325,6 +331,8 @@ bool build_hub_tiles(rdm_ctx* ctx, Csr& A, const int64_t* rowptr_host, const int
 constexpr int kPiecesI8 = 8;     // three int8 digits (23-bit fixed point per column)
 constexpr int kPiecesI8x2 = 9;   // two int8 digits (15-bit fixed point): the fast variant
 bool hub_tiles_pay(const Core& c, int64_t w, int np);
+// int8 tiles in row-block pairs (partials of 256 rows per item, items per pair)
+bool tiles_paired();
 void hub_tiles_product(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx, int64_t w,
                        float* part, int64_t ldp, int np);
 

@@ -53,9 +53,10 @@ struct Epi {
   const float* core;        // hub-core product (K x ld_core) or null
   int64_t ld_core;
   const int32_t* hub_slot;  // int32[N], -1 for non-hubs
-  const float* tpart;       // binary hub tiles: per-item partials (n_items x 128 x ld_tpart) or null
+  const float* tpart;       // binary hub tiles: per-item partials (n_items x 2^item_shift x ld_tpart) or null
   int64_t ld_tpart;
-  const int32_t* rb_item;   // item range of each 128-row rank block
+  const int32_t* rb_item;   // item range of each block of 2^item_shift ranks
+  int item_shift;           // 7: items of one row block; 8: of a row-block pair
   const float* tscale;      // row scale r_i of hub slot i (a_ij = r_i c_j)
   Scatter scat;             // fused col→row redistribution (scat.P == 0: off)
   const float* rscale;      // factored bf16 path: s_i per row (applied first), or null
@@ -92,11 +93,12 @@ __device__ __forceinline__ float4 apply_epi(float4 a, const Epi& e, int64_t row,
   if (e.tpart) {  // binary hub tiles: s_i · Σ_items partial (item order; after the CSR sum)
     const int s = __ldg(e.hub_slot + row);
     if (s >= 0) {
-      const int i0 = __ldg(e.rb_item + (s >> 7)), i1 = __ldg(e.rb_item + (s >> 7) + 1);
+      const int blk = s >> e.item_shift, rr = s & ((1 << e.item_shift) - 1);
+      const int i0 = __ldg(e.rb_item + blk), i1 = __ldg(e.rb_item + blk + 1);
       float4 t = make_float4(0.f, 0.f, 0.f, 0.f);
       for (int it = i0; it < i1; ++it) {
-        const float4 k =
-            __ldg(reinterpret_cast<const float4*>(e.tpart + ((int64_t)it * 128 + (s & 127)) * e.ld_tpart + c));
+        const float4 k = __ldg(reinterpret_cast<const float4*>(
+            e.tpart + (((int64_t)it << e.item_shift) + rr) * e.ld_tpart + c));
         t.x += k.x; t.y += k.y; t.z += k.z; t.w += k.w;
       }
       const float sc = __ldg(e.tscale + s);
@@ -713,7 +715,7 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
                                                 ((uintptr_t)mask & 15) == 0),
                 "spmm: mask requires a 16-byte aligned N x w buffer with ld % 4 == 0");
   RDM_CHECK_ARG(!(epi_flags & RDM_EPI_BIAS) || bias, "spmm: bias pointer missing");
-  Epi epi{epi_flags, bias, mask, ld_mask, w, nullptr, 0, nullptr, nullptr, 0, nullptr, nullptr, Scatter{}, nullptr};
+  Epi epi{epi_flags, bias, mask, ld_mask, w, nullptr, 0, nullptr, nullptr, 0, nullptr, 7, nullptr, Scatter{}, nullptr};
   if (scat) {
     RDM_CHECK_ARG(scat->mode == 2 && scat->P >= 1 && scat->P <= Scatter::kMax && scat->my_w <= w,
                   "spmm: bad scatter descriptor");
@@ -752,11 +754,14 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
     // binary hub tiles on the kind::f16 tensor cores (hubtiles.cu); the
     // residual CSR's epilogue adds s_i · Σ_items partial for hub rows.
     const int64_t ldp = w4;
-    float* part = ensure_ws(ctx->ws_core_c, (size_t)A.core.n_items * 128 * ldp * sizeof(float));
+    const bool pairs = (np == kPiecesI8 || np == kPiecesI8x2) && tiles_paired();
+    const size_t prow = pairs ? (size_t)A.core.n_pitems * 256 : (size_t)A.core.n_items * 128;
+    float* part = ensure_ws(ctx->ws_core_c, prow * ldp * sizeof(float));
     hub_tiles_product(ctx, A.core, in, ld_in, w, part, ldp, np);
     epi.tpart = part;
     epi.ld_tpart = ldp;
-    epi.rb_item = A.core.rb_item->as<int32_t>();
+    epi.rb_item = pairs ? A.core.pair_item->as<int32_t>() : A.core.rb_item->as<int32_t>();
+    epi.item_shift = pairs ? 8 : 7;
     epi.tscale = A.core.rscale->as<float>();
     epi.hub_slot = A.core.hub_slot->as<int32_t>();
     run_csr(ctx, *A.core.resid, in, ld_in, out, ld_out, w4, epi, inb, fact);
