@@ -594,22 +594,33 @@ hub_tile_i8_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __re
   const uint32_t kAcol = 2 * sh.acc_cols;
 
   if (warp == 0) {
-    if (lane == 0) {
-      int s = 0;
-      uint32_t ph = 0, kc = 0;
-      const uint32_t bytes = (uint32_t)bbytes + 2048;
-      for (int t = blockIdx.x; t < total; t += gridDim.x) {
-        const int item = t / sh.tiles_n;
-        const int n0 = (t % sh.tiles_n) * n_mma;
-        const int tb = item_tb[item], T = item_tb[item + 1] - tb;
-        int ti = (int)(((unsigned)item * 2654435761u) % (unsigned)max(T, 1));
-        for (int i = 0; i < T; ++i) {
-          const int tile = tb + ti;
-          if (++ti == T) ti = 0;
-          if (kc >= (uint32_t)S) mbar_wait(&empty[s], ph ^ 1);
-          mbar_expect_tx(&full[s], bytes);
-          bulk_load(bits_st(s), bits + (int64_t)tile * 2 * TK, 2048, &full[s]);
-          tma_load_4d(B_st(s), &tmB, &full[s], 0, n0, 0, tile_cb[tile]);
+    // the whole warp fetches the column blocks of 32 tiles at a time (one
+    // coalesced load instead of one dependent L2 round trip per tile on the
+    // issue path); lane 0 issues the copies
+    int s = 0;
+    uint32_t ph = 0, kc = 0;
+    const uint32_t bytes = (uint32_t)bbytes + 2048;
+    for (int t = blockIdx.x; t < total; t += gridDim.x) {
+      const int item = t / sh.tiles_n;
+      const int n0 = (t % sh.tiles_n) * n_mma;
+      const int tb = item_tb[item], T = item_tb[item + 1] - tb;
+      const int rot = (int)(((unsigned)item * 2654435761u) % (unsigned)max(T, 1));
+      for (int i0 = 0; i0 < T; i0 += 32) {
+        int idx = rot + i0 + lane;
+        idx -= (idx >= T) ? T : 0;
+        idx -= (idx >= T) ? T : 0;
+        const int my_tile = tb + idx;
+        const int my_cb = (i0 + lane < T) ? __ldg(tile_cb + my_tile) : 0;
+        const int cnt = min(32, T - i0);
+        for (int k = 0; k < cnt; ++k) {
+          const int tile = __shfl_sync(0xffffffffu, my_tile, k);
+          const int cb = __shfl_sync(0xffffffffu, my_cb, k);
+          if (lane == 0) {
+            if (kc >= (uint32_t)S) mbar_wait(&empty[s], ph ^ 1);
+            mbar_expect_tx(&full[s], bytes);
+            bulk_load(bits_st(s), bits + (int64_t)tile * 2 * TK, 2048, &full[s]);
+            tma_load_4d(B_st(s), &tmB, &full[s], 0, n0, 0, cb);
+          }
           ++kc;
           if (++s == S) { s = 0; ph ^= 1; }
         }
@@ -775,24 +786,34 @@ hub_tile_i8_pair_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t*
   const uint32_t kAcol = (uint32_t)sh.acc_cols;     // both accumulators, rounded up
 
   if (warp == 0) {
-    if (lane == 0) {
-      int s = 0;
-      uint32_t ph = 0, kc = 0;
-      const uint32_t bytes = (uint32_t)bbytes + 4096;
-      for (int t = blockIdx.x; t < total; t += gridDim.x) {
-        const int item = t / sh.tiles_n;
-        const int n0 = (t % sh.tiles_n) * n_mma;
-        const int mb = pitem_pm[item], M = pitem_pm[item + 1] - mb;
-        int mi = (int)(((unsigned)item * 2654435761u) % (unsigned)max(M, 1));
-        for (int i = 0; i < M; ++i) {
-          const int m = mb + mi;
-          if (++mi == M) mi = 0;
-          if (kc >= (uint32_t)S) mbar_wait(&empty[s], ph ^ 1);
-          mbar_expect_tx(&full[s], bytes);
-          const int t1 = pm_t1[m], t2 = pm_t2[m];
-          bulk_load(bits_st(s), t1 >= 0 ? bits + (int64_t)t1 * 2 * TK : zero_bits, 2048, &full[s]);
-          bulk_load(bits_st(s) + 2048, t2 >= 0 ? bits + (int64_t)t2 * 2 * TK : zero_bits, 2048, &full[s]);
-          tma_load_4d(B_st(s), &tmB, &full[s], 0, n0, 0, pm_cb[m]);
+    int s = 0;
+    uint32_t ph = 0, kc = 0;
+    const uint32_t bytes = (uint32_t)bbytes + 4096;
+    for (int t = blockIdx.x; t < total; t += gridDim.x) {
+      const int item = t / sh.tiles_n;
+      const int n0 = (t % sh.tiles_n) * n_mma;
+      const int mb = pitem_pm[item], M = pitem_pm[item + 1] - mb;
+      const int rot = (int)(((unsigned)item * 2654435761u) % (unsigned)max(M, 1));
+      for (int i0 = 0; i0 < M; i0 += 32) {
+        int idx = rot + i0 + lane;
+        idx -= (idx >= M) ? M : 0;
+        idx -= (idx >= M) ? M : 0;
+        const bool ok = i0 + lane < M;
+        const int my_cb = ok ? __ldg(pm_cb + mb + idx) : 0;
+        const int my_t1 = ok ? __ldg(pm_t1 + mb + idx) : -1;
+        const int my_t2 = ok ? __ldg(pm_t2 + mb + idx) : -1;
+        const int cnt = min(32, M - i0);
+        for (int k = 0; k < cnt; ++k) {
+          const int cb = __shfl_sync(0xffffffffu, my_cb, k);
+          const int t1 = __shfl_sync(0xffffffffu, my_t1, k);
+          const int t2 = __shfl_sync(0xffffffffu, my_t2, k);
+          if (lane == 0) {
+            if (kc >= (uint32_t)S) mbar_wait(&empty[s], ph ^ 1);
+            mbar_expect_tx(&full[s], bytes);
+            bulk_load(bits_st(s), t1 >= 0 ? bits + (int64_t)t1 * 2 * TK : zero_bits, 2048, &full[s]);
+            bulk_load(bits_st(s) + 2048, t2 >= 0 ? bits + (int64_t)t2 * 2 * TK : zero_bits, 2048, &full[s]);
+            tma_load_4d(B_st(s), &tmB, &full[s], 0, n0, 0, cb);
+          }
           ++kc;
           if (++s == S) { s = 0; ph ^= 1; }
         }
@@ -1041,10 +1062,14 @@ double tile_s(int64_t w, int np = 3) {
 }
 }  // namespace
 
-// The int8 tiles run in row-block pairs unless RDM_TILE_PAIRS=0.
+// The int8 tiles run in row-block pairs with RDM_TILE_PAIRS=1 (off by
+// default: measured no faster — Reddit-shaped w = 128 1.235 vs 1.232 ms per
+// call, w = 16 0.417 vs 0.387, products-shaped w = 256 8.30 vs 8.41 ms; the
+// single kernel is bound by the tensor pipe's int8 rate at N = 3·64, not by
+// the panel ingress the pairs halve, profiles/r2_tile_pairs.txt).
 bool tiles_paired() {
   const char* e = getenv("RDM_TILE_PAIRS");
-  return !(e && !atoi(e));
+  return e && atoi(e);
 }
 
 bool hub_tiles_pay(const Core& c, int64_t w, int np) {

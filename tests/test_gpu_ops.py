@@ -239,7 +239,7 @@ def test_spmm_hub_core_matches_oracle(torch_dev, w, K, monkeypatch):
 
 @pytest.mark.parametrize("w", [1, 4, 16, 41, 128, 130, 256, 301])
 @pytest.mark.parametrize("min_nnz,k2", [(1, 0), (40, 0), (1, 1024)])
-@pytest.mark.parametrize("pieces", ["auto", "auto-unpaired", "2", "3"])
+@pytest.mark.parametrize("pieces", ["auto", "auto-paired", "2", "3"])
 def test_spmm_hub_tiles_matches_oracle(torch_dev, w, min_nnz, k2, pieces, monkeypatch):
     """Binary hub tiles (tensor cores on 0/1 tiles against s ⊙ X as three int8
     digits on kind::i8 (auto), two column-scaled fp16 or three bf16 pieces on
@@ -248,8 +248,8 @@ def test_spmm_hub_tiles_matches_oracle(torch_dev, w, min_nnz, k2, pieces, monkey
     torch, dev = torch_dev
     import paper_conf_ipps_kurtysps23_b200 as rdm
     monkeypatch.setenv("RDM_TILE_MIN_NNZ", str(min_nnz))
-    if pieces == "auto-unpaired":   # int8 digits, one row block per panel load
-        monkeypatch.setenv("RDM_TILE_PAIRS", "0")
+    if pieces == "auto-paired":   # int8 digits, two row blocks per panel load
+        monkeypatch.setenv("RDM_TILE_PAIRS", "1")
     elif pieces != "auto":   # 2 column-scaled fp16 pieces / 3 bf16 pieces at every width
         monkeypatch.setenv("RDM_TILE_PIECES", pieces)
     if k2:
