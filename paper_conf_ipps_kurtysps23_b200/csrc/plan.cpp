@@ -138,7 +138,9 @@ rdm_status rdm_select_config(int L, const int64_t* f, int64_t n, int64_t nnz, in
   }
   // Pick (reading R23): modelled B200 time.  Redistribution: each unit of
   // width moves (P−1)/P·N·4 bytes total, i.e. (P−1)/P²·N·4 per GPU, over
-  // NVLink (~770 GB/s measured per direction).  SpMM: each call streams the
+  // NVLink at 770 GB/s per direction (the peer-copy bandwidth
+  // B200_PROFILING.md reports for this pool; not measured by this build —
+  // every box it ran on had one GPU).  SpMM: each call streams the
   // replicated CSR (≈8 B/nnz + 8 B/row) and its N x w/P slice twice
   // (≈6.5 TB/s HBM).  The number of SpMM calls is not in the model; the
   // width term is what the paper's sparse units measure.
