@@ -46,6 +46,8 @@ def parse():
                     help="one-rank emulation of a P-rank job on one GPU (rdm_init_emulated); "
                          "default workload papers (BASELINE configs[4]) at P = 8")
     ap.add_argument("--emulate-rank", type=int, default=0)
+    ap.add_argument("--emulate-check", type=int, default=1,
+                    help="--emulate: per-op parity on 4,096 sampled rows against the fp64 oracle")
     ap.add_argument("--threads", type=int, default=0,
                     help="--impl reference: oracle threads (default nproc)")
     ap.add_argument("--ref-budget-s", type=float, default=150.0,
@@ -434,6 +436,36 @@ def emulate_main(a):
     ginfo = ctx.graph_info()
     pareto, chosen, _, _ = rdm.select_config(list(wl.f), wl.n, wl.nnz, P)
     cfg = chosen if a.config == "auto" else int(a.config)
+    # per-op parity at these full sizes, in this launch configuration (SURVEY
+    # §8(c) "per-op on sampled rows"): the rank's SpMM on a seeded column
+    # slice of width w_p and its NN GEMM on its row slice, against the fp64
+    # oracle on 4,096 sampled output rows
+    parity = None
+    if a.emulate_check:
+        from oracle import gcn as og
+        rng = np.random.default_rng(11)
+        n_all = wl.n
+        c0, c1, ldc = rdm.partition(P, rdm.COL, n_all, wl.f[1], p)
+        wp = c1 - c0
+        Xc = torch.zeros(n_all, ldc, device=dev)
+        Xc[:, :wp] = torch.from_numpy(synth.features(n_all, wp, seed=12)).to(dev)
+        Oc = torch.zeros_like(Xc)
+        ctx.spmm(1, Xc, Oc, wp)
+        ctx.sync()
+        rows = np.sort(rng.choice(n_all, size=4096, replace=False))
+        ref = og.spmm_rows(g, Xc[:, :wp].cpu().numpy(), rows)
+        e_sp = og.max_rel_err(Oc[rows][:, :wp].cpu().numpy(), ref)
+        del Xc, Oc
+        Tr = torch.zeros(hi - lo, wl.f[1], device=dev)
+        ctx.gemm(rdm.GEMM_NN, H0, Wd[0], Tr, hi - lo, wl.f[0], wl.f[1])
+        ctx.sync()
+        rr = np.sort(rng.choice(hi - lo, size=4096, replace=False))
+        e_gm = og.max_rel_err(Tr[rr].cpu().numpy(),
+                              H0[rr].cpu().numpy().astype(np.float64) @ Wd[0].cpu().numpy().astype(np.float64))
+        del Tr
+        parity = {"spmm_w": wp, "spmm_rows_checked": 4096, "spmm_max_rel_err": e_sp,
+                  "gemm_nn_rows_checked": 4096, "gemm_nn_max_rel_err": e_gm, "gate": 1e-4,
+                  "pass": bool(e_sp < 1e-4 and e_gm < 1e-4)}
     model = rdm.GCN(ctx, wl.f, cfg, low_memory=True)
     info = model.info()
     model.set_input([H0], [y], [m])
@@ -513,6 +545,7 @@ def emulate_main(a):
                              "pool (not measured by this build); no overlap assumed"},
         "plan": {"model_comm_units": info["model_comm_units"],
                  "model_sparse_units": info["model_sparse_units"]},
+        "parity": parity,
     }
     print(json.dumps(line), flush=True)
     model.close()
