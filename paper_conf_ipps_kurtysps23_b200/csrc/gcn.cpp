@@ -647,6 +647,14 @@ void create(rdm_gcn* g) {
   }
 }
 
+// The step after `s` in its pass (nullptr at the end).
+const Step* next_step(const rdm_gcn* g, const Step* s) {
+  for (auto* v : {&g->fwd, &g->bwd})
+    if (!v->empty() && s >= &v->front() && s <= &v->back())
+      return s == &v->back() ? nullptr : s + 1;
+  return nullptr;
+}
+
 void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
   rdm_ctx* ctx = g->ctx;
   // any producer but the bf16-wire redistribution (and the in-place mask,
@@ -700,14 +708,37 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
     case S_GEMM: {
       Phase ph(ctx, RDM_PH_GEMM);
       const int64_t fin = g->f[s.wl - 1], fout = g->f[s.wl];
+      // fast variant at P = 1 (row and column layouts coincide): when the next
+      // step is an SpMM reading this output, the GEMM's epilogue also writes
+      // the SpMM's bf16 input (× s_i for factored values) — the cast folded
+      // into the producer (NEXT-3)
+      const Step* nxt = next_step(g, &s);
+      const bool fold = ctx->prec == RDM_PREC_FAST && P == 1 && nl == 1 && !g->RA && nxt &&
+                        nxt->op == S_SPMM && nxt->in.id() == s.out.id() &&
+                        !(getenv("RDM_FOLD_CAST") && !atoi(getenv("RDM_FOLD_CAST")));
       for (int i = 0; i < nl; ++i) {
         Buf& in = buf(g, i, s.in, s.lin);
         Buf& out = buf(g, i, s.out, s.lout);
         const float* mk = (s.epi & RDM_EPI_MASK) ? buf(g, i, s.mask, s.lmask).p : nullptr;
         Scatter sc;
         if (s.fuse == 1) sc = make_scatter(g, s, i);
+        const int64_t ncol = s.gop == RDM_GEMM_NN ? fout : fin;
+        if (fold) {
+          const Csr& An = nxt->trans ? g->graph->fwd() : g->graph->bwd();
+          const int64_t w8 = (roundup4(ncol) + 7) & ~int64_t(7);
+          ctx->gemm_twin = ensure_ws(ctx->ws_bf16, (size_t)std::max<int64_t>(An.in_rows(), 1) * w8 * 2);
+          ctx->gemm_twin_ld = w8;
+          ctx->gemm_twin_scale = An.fscale ? An.fscale->as<float>() : nullptr;
+          ctx->gemm_twin_written = false;
+        }
         gemm(ctx, s.gop, in.p, in.ld, W[s.wl - 1], fout, out.p, out.ld, in.rows, fin, fout, s.epi,
              nullptr, mk, s.fuse == 1 ? &sc : nullptr);
+        if (fold) {
+          ctx->bf16_twin_src = ctx->gemm_twin_written ? out.p : nullptr;
+          ctx->bf16_twin_fact = ctx->gemm_twin_scale != nullptr;
+          ctx->gemm_twin = nullptr;
+          ctx->gemm_twin_scale = nullptr;
+        }
       }
       break;
     }

@@ -25,6 +25,7 @@
 //            split-K over rows with an ordered (deterministic) reduction.
 #include <cuda.h>
 #include <cudaTypedefs.h>
+#include <cuda_bf16.h>
 
 #include <algorithm>
 #include <cstdlib>
@@ -46,6 +47,12 @@ struct TcEpi {
   const float* mask;
   int64_t ld_mask;
   Scatter scat;   // fused row→column redistribution (MODE 0, no split-K); scat.P == 0: off
+  // RDM_PREC_FAST: a bf16 copy of the output (× twin_scale[row] when not null),
+  // row length ld_twin, columns [N, ld_twin) zero — the next SpMM's input
+  // (the cast folded into this epilogue); null: off
+  uint16_t* twin = nullptr;
+  int64_t ld_twin = 0;
+  const float* twin_scale = nullptr;
 };
 
 struct TcShape {
@@ -425,6 +432,28 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
             }
           }
         }
+        if (MODE == 0 && epi.twin) {
+          const int64_t row = row0 + lane;
+          if (row < sh.M) {
+            const float sc = epi.twin_scale ? __ldg(epi.twin_scale + row) : 1.f;
+            uint4* dst = reinterpret_cast<uint4*>(epi.twin + row * epi.ld_twin + n0 + c0);
+            const int64_t cmax = epi.ld_twin - (n0 + c0);   // columns of this chunk inside the copy
+#pragma unroll
+            for (int j = 0; j < 4; ++j) {
+              if (8 * j >= cmax) break;
+              uint32_t w[4];
+#pragma unroll
+              for (int h = 0; h < 4; ++h) {
+                const int i = 8 * j + 2 * h;
+                const float a = (n0 + c0 + i < sh.N) ? v[i] * sc : 0.f;
+                const float b = (n0 + c0 + i + 1 < sh.N) ? v[i + 1] * sc : 0.f;
+                __nv_bfloat162 pr = __floats2bfloat162_rn(a, b);
+                w[h] = *reinterpret_cast<uint32_t*>(&pr);
+              }
+              dst[j] = make_uint4(w[0], w[1], w[2], w[3]);
+            }
+          }
+        }
         if (sh.tstore) {
           // the lane's row as 8 float4 chunks of the 128-byte-swizzled box
           // (chunk j of row r at j ^ (r & 7): conflict-free); the TMA engine
@@ -683,6 +712,12 @@ bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, 
   TcEpi e{epi, bias, mask, ldc, Scatter{}};
   if (op == RDM_GEMM_NN || op == RDM_GEMM_NT) {
     if (scat) e.scat = *scat;
+    if (ctx->gemm_twin) {
+      e.twin = static_cast<uint16_t*>(ctx->gemm_twin);
+      e.ld_twin = ctx->gemm_twin_ld;
+      e.twin_scale = ctx->gemm_twin_scale;
+      ctx->gemm_twin_written = true;
+    }
     const int64_t M = rows;
     const int64_t N = op == RDM_GEMM_NN ? m : k;   // output columns
     const int64_t K = op == RDM_GEMM_NN ? k : m;   // contraction

@@ -201,6 +201,15 @@ struct rdm_ctx {
   int transport = 0;             // RDM_TRANSPORT_NCCL / RDM_TRANSPORT_P2P
   int prec = 0;                  // RDM_PREC_FP32 / RDM_PREC_FAST
   bool spmm_in_bf16 = false;     // executor → spmm: the input holds bf16 values (bf16 wire)
+  // fast variant, cast folded into the producing GEMM (executor → gemm_tc):
+  // the GEMM also writes a bf16 copy (row length gemm_twin_ld, rows × scale)
+  void* gemm_twin = nullptr;
+  int64_t gemm_twin_ld = 0;
+  const float* gemm_twin_scale = nullptr;
+  bool gemm_twin_written = false;
+  // … and the SpMM that reads `bf16_twin_src` takes the copy instead of casting
+  const float* bf16_twin_src = nullptr;
+  bool bf16_twin_fact = false;
   std::string err;
   rdm::Graph graph;
   bool has_graph = false;

@@ -729,14 +729,20 @@ void spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out
     const int64_t w8 = (w4 + 7) & ~int64_t(7);
     const int64_t nin = A.in_rows();
     __nv_bfloat16* xb = reinterpret_cast<__nv_bfloat16*>(ensure_ws(ctx->ws_bf16, (size_t)std::max<int64_t>(nin, 1) * w8 * 2));
-    const int64_t total = nin * (w8 / 8);
-    const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(total, 256), (int64_t)ctx->num_sms * 16));
-    // the value-free factored rows need bf16(s_j·X_j); an input that already
-    // holds bf16 values (bf16 wire) is used as is, with the values (no second rounding)
-    fact = A.fscale != nullptr && !ctx->spmm_in_bf16;
-    to_bf16_kernel<<<grid, 256, 0, ctx->stream>>>(in, ld_in, nin, w4, w8, xb,
-                                                  fact ? A.fscale->as<float>() : nullptr);
-    RDM_LAUNCHED(ctx);
+    if (ctx->bf16_twin_src == in) {
+      // the producing GEMM already wrote this bf16 input (cast folded into its epilogue)
+      fact = ctx->bf16_twin_fact;
+    } else {
+      const int64_t total = nin * (w8 / 8);
+      const unsigned grid = (unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(total, 256), (int64_t)ctx->num_sms * 16));
+      // the value-free factored rows need bf16(s_j·X_j); an input that already
+      // holds bf16 values (bf16 wire) is used as is, with the values (no second rounding)
+      fact = A.fscale != nullptr && !ctx->spmm_in_bf16;
+      to_bf16_kernel<<<grid, 256, 0, ctx->stream>>>(in, ld_in, nin, w4, w8, xb,
+                                                    fact ? A.fscale->as<float>() : nullptr);
+      RDM_LAUNCHED(ctx);
+    }
+    ctx->bf16_twin_src = nullptr;
     inb = xb;
     if (fact) epi.rscale = A.fscale->as<float>();
   }

@@ -261,3 +261,33 @@ def test_fast_bf16_wire_halves_bytes(rdm, cora, P, cfg):
     assert c32["a2a_bytes_wire"] == want32
     assert c16["a2a_bytes_wire"] == want16 < want32
     _check((g, H0, Ws, y, m), loss, dW, model, rdm, P=P, tol=GATE, ltol=LOSS_GATE)
+
+
+@pytest.mark.parametrize("cfg", [3, 10, 15])
+def test_fast_cast_folded_into_gemm(rdm, cora, cfg, monkeypatch):
+    """NEXT-3: at P = 1 the fast variant's GEMM epilogue writes the next SpMM's
+    bf16 input itself (× s_i for factored values) instead of a separate cast
+    pass — bit-identical results, fewer launches."""
+    g, H0, Ws, y, m = cora
+    out = {}
+    for fold in ("0", "1"):
+        monkeypatch.setenv("RDM_FOLD_CAST", fold)
+        loss, dW, model, ctx, _ = _run(rdm, g, H0, Ws, y, m, cfg, P=1, precision="fast")
+        out[fold] = (loss, dW, ctx.counters()["kernel_launches"])
+        model.close()
+        ctx.close()
+    assert out["0"][0] == out["1"][0]
+    for a, b in zip(out["0"][1], out["1"][1]):
+        assert np.array_equal(a, b)
+    f = [H0.shape[1]] + [w.shape[1] for w in Ws]
+    _, desc = rdm.plan_info(f, cfg, 1, g.n)
+    steps = [l.split() for l in desc.splitlines() if l.startswith("  ")]
+
+    def gemm_out(t):   # "GEMM NN X W -> Y.row ..." (not TN)
+        return t[t.index("->") + 1].split(".")[0] if t[0] == "GEMM" and t[1] in ("NN", "NT") else None
+
+    def spmm_in(t):    # "SPMM A^T X.col -> ..."
+        return t[2].split(".")[0] if t[0] == "SPMM" else None
+
+    folds = sum(1 for a, b in zip(steps, steps[1:]) if gemm_out(a) and gemm_out(a) == spmm_in(b))
+    assert out["1"][2] == out["0"][2] - folds, (out, folds)
