@@ -441,6 +441,12 @@ struct rdm_gcn {
   // variant): an SpMM reading them uses them as the bf16 values they are
   // (no second rounding of s_j·x_j, rdm_ctx::spmm_in_bf16)
   std::set<std::pair<int, int>> wire_bf16;
+  // ReLU sign bits (1/32 of the fp32 Hadamard operand): a row-layout H^l that a
+  // GEMM NN produces with ReLU and a later GEMM reads as its mask; per slot
+  // one u32 per 32 columns, `mb_valid` once the producer wrote them this epoch
+  std::map<std::pair<int, int>, std::vector<uint32_t*>> mbits;
+  std::map<std::pair<int, int>, int64_t> mbits_ld;
+  std::set<std::pair<int, int>> mb_valid;
 };
 
 namespace rdm {
@@ -615,6 +621,32 @@ void create(rdm_gcn* g) {
       g->bufs[s][b.key] = x;
     }
   }
+  // ReLU sign bits for GEMM → GEMM Hadamards in the row layout (RDM_MASK_BITS=0: off)
+  if (!g->RA && !(getenv("RDM_MASK_BITS") && !atoi(getenv("RDM_MASK_BITS")))) {
+    std::set<std::pair<int, int>> relu_rows;
+    for (auto* v : {&g->fwd, &g->bwd})
+      for (const Step& st : *v)
+        if (st.op == S_GEMM && (st.epi & RDM_EPI_RELU) && st.lout == RDM_ROW)
+          relu_rows.insert({st.out.id(), norm_lay(g, st.lout)});
+    for (auto* v : {&g->fwd, &g->bwd})
+      for (const Step& st : *v) {
+        if (st.op != S_GEMM || !(st.epi & RDM_EPI_MASK) || st.lmask != RDM_ROW) continue;
+        const auto key = std::make_pair(st.mask.id(), norm_lay(g, st.lmask));
+        if (!relu_rows.count(key) || g->mbits.count(key)) continue;
+        std::vector<uint32_t*> per(ctx->nlocal());
+        int64_t ldw = 0;
+        for (int sl = 0; sl < ctx->nlocal(); ++sl) {
+          const Buf& b = g->bufs[sl].at(key);
+          ldw = (b.cols + 31) / 32;
+          const size_t bytes = (size_t)std::max<int64_t>(1, b.rows * ldw) * 4;
+          g->mem.emplace_back(new DevBuf(bytes));
+          per[sl] = g->mem.back()->as<uint32_t>();
+          g->ws_bytes += (int64_t)bytes;
+        }
+        g->mbits[key] = per;
+        g->mbits_ld[key] = ldw;
+      }
+  }
   const int P = ctx->world;
   const int64_t n = g->n_cap;
   g->dwp.assign(ctx->nlocal(), std::vector<float*>(g->L + 1, nullptr));
@@ -659,8 +691,10 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
   rdm_ctx* ctx = g->ctx;
   // any producer but the bf16-wire redistribution (and the in-place mask,
   // which keeps bf16 values bf16) leaves fp32 values in its output
-  if (s.op == S_SPMM || s.op == S_GEMM || s.op == S_LOSS || s.op == S_REDIST)
+  if (s.op == S_SPMM || s.op == S_GEMM || s.op == S_LOSS || s.op == S_REDIST) {
     g->wire_bf16.erase({s.out.id(), norm_lay(g, s.lout)});
+    g->mb_valid.erase({s.out.id(), norm_lay(g, s.lout)});   // (re)set by the GEMM that writes bits
+  }
   const int nl = ctx->nlocal();
   const int P = ctx->world;
   // a fused producer overwrites peers' destination slices: every rank must be
@@ -731,8 +765,27 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
           ctx->gemm_twin_scale = An.fscale ? An.fscale->as<float>() : nullptr;
           ctx->gemm_twin_written = false;
         }
+        const auto okey = std::make_pair(s.out.id(), norm_lay(g, s.lout));
+        const auto mkey = std::make_pair(s.mask.id(), norm_lay(g, s.lmask));
+        auto ob = g->mbits.find(okey);
+        if ((s.epi & RDM_EPI_RELU) && ob != g->mbits.end()) {
+          ctx->gemm_bits_out = ob->second[i];
+          ctx->gemm_bits_ld = g->mbits_ld[okey];
+          ctx->gemm_bits_written = false;
+        }
+        auto mbit = g->mbits.find(mkey);
+        if ((s.epi & RDM_EPI_MASK) && mbit != g->mbits.end() && g->mb_valid.count(mkey)) {
+          ctx->gemm_mask_bits = mbit->second[i];
+          ctx->gemm_mask_bits_ld = g->mbits_ld[mkey];
+        }
         gemm(ctx, s.gop, in.p, in.ld, W[s.wl - 1], fout, out.p, out.ld, in.rows, fin, fout, s.epi,
              nullptr, mk, s.fuse == 1 ? &sc : nullptr);
+        if (ctx->gemm_bits_out) {
+          if (ctx->gemm_bits_written) g->mb_valid.insert(okey);
+          else g->mb_valid.erase(okey);
+        }
+        ctx->gemm_bits_out = nullptr;
+        ctx->gemm_mask_bits = nullptr;
         if (fold) {
           ctx->bf16_twin_src = ctx->gemm_twin_written ? out.p : nullptr;
           ctx->bf16_twin_fact = ctx->gemm_twin_scale != nullptr;

@@ -53,6 +53,13 @@ struct TcEpi {
   uint16_t* twin = nullptr;
   int64_t ld_twin = 0;
   const float* twin_scale = nullptr;
+  // ReLU sign bits of the output (1[v > 0], one u32 per 32 columns, row length
+  // ld_bits_out words) for a later Hadamard; and the Hadamard read from such
+  // bits instead of the fp32 mask (1/32 of its bytes)
+  uint32_t* bits_out = nullptr;
+  int64_t ld_bits_out = 0;
+  const uint32_t* mask_bits = nullptr;
+  int64_t ld_mask_bits = 0;
 };
 
 struct TcShape {
@@ -417,7 +424,11 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
 #pragma unroll
             for (int i = 0; i < 32; ++i) v[i] = fmaxf(v[i], 0.f);
           }
-          if ((epi.flags & RDM_EPI_MASK) && row < sh.M) {
+          if ((epi.flags & RDM_EPI_MASK) && row < sh.M && epi.mask_bits) {
+            const uint32_t mb = __ldg(epi.mask_bits + row * epi.ld_mask_bits + ((n0 + c0) >> 5));
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] = (mb >> i) & 1u ? v[i] : 0.f;
+          } else if ((epi.flags & RDM_EPI_MASK) && row < sh.M) {
             const float4* mrow = reinterpret_cast<const float4*>(epi.mask + row * epi.ld_mask + n0 + c0);
             float4 mk[8];
 #pragma unroll
@@ -431,6 +442,12 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
               v[4 * j + 3] = mk[j].w > 0.f ? v[4 * j + 3] : 0.f;
             }
           }
+        }
+        if (MODE == 0 && epi.bits_out && row0 + lane < sh.M) {
+          uint32_t mb = 0;
+#pragma unroll
+          for (int i = 0; i < 32; ++i) mb |= (n0 + c0 + i < sh.N && v[i] > 0.f) ? (1u << i) : 0u;
+          epi.bits_out[(row0 + lane) * epi.ld_bits_out + ((n0 + c0) >> 5)] = mb;
         }
         if (MODE == 0 && epi.twin) {
           const int64_t row = row0 + lane;
@@ -712,6 +729,11 @@ bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, 
   TcEpi e{epi, bias, mask, ldc, Scatter{}};
   if (op == RDM_GEMM_NN || op == RDM_GEMM_NT) {
     if (scat) e.scat = *scat;
+    e.bits_out = ctx->gemm_bits_out;
+    e.ld_bits_out = ctx->gemm_bits_ld;
+    e.mask_bits = ctx->gemm_mask_bits;
+    e.ld_mask_bits = ctx->gemm_mask_bits_ld;
+    if (ctx->gemm_bits_out) ctx->gemm_bits_written = true;
     if (ctx->gemm_twin) {
       e.twin = static_cast<uint16_t*>(ctx->gemm_twin);
       e.ld_twin = ctx->gemm_twin_ld;

@@ -210,6 +210,14 @@ struct rdm_ctx {
   // … and the SpMM that reads `bf16_twin_src` takes the copy instead of casting
   const float* bf16_twin_src = nullptr;
   bool bf16_twin_fact = false;
+  // ReLU sign bits (executor → gemm_tc, NN/NT): write them for the output /
+  // read the Hadamard from them; gemm_bits_written reports that the tensor-core
+  // path (not the SIMT fallback) ran
+  uint32_t* gemm_bits_out = nullptr;
+  int64_t gemm_bits_ld = 0;
+  const uint32_t* gemm_mask_bits = nullptr;
+  int64_t gemm_mask_bits_ld = 0;
+  bool gemm_bits_written = false;
   std::string err;
   rdm::Graph graph;
   bool has_graph = false;

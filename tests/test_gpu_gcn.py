@@ -514,3 +514,27 @@ def test_emulated_rank(rdm, cora):
     me.close()
     em.close()
     plain.close()
+
+
+@pytest.mark.parametrize("f,cfgs", [((64, 48, 41), [0, 2, 5, 8, 10, 15]), ((60, 40, 32, 9), [0, 9, 25, 37, 63])])
+def test_relu_bits_hadamard_bitwise(rdm, f, cfgs, monkeypatch):
+    """A row-layout H^l produced by a GEMM with ReLU and used as the Hadamard
+    mask of a later GEMM is passed as sign bits (1/32 of the fp32 operand's
+    bytes): every result bit-identical to reading the fp32 mask."""
+    import torch
+    prob = _problem(n=3000, E=30000, f=f, seed=21)
+    g, H0, Ws, y, m = prob
+    for cfg in cfgs:
+        out = {}
+        for bits in ("0", "1"):
+            monkeypatch.setenv("RDM_MASK_BITS", bits)
+            loss, dW, model, ctx, _ = _run(rdm, g, H0, Ws, y, m, cfg)
+            G0 = model.tensor_torch(rdm.T_G, 0).cpu().numpy()
+            out[bits] = (loss, dW, G0)
+            model.close()
+            ctx.close()
+        assert out["0"][0] == out["1"][0], cfg
+        for a, b in zip(out["0"][1], out["1"][1]):
+            assert np.array_equal(a, b), cfg
+        assert np.array_equal(out["0"][2], out["1"][2]), cfg
+    _check(prob, *_run(rdm, g, H0, Ws, y, m, cfgs[-1])[:3], rdm)
