@@ -315,3 +315,73 @@ def test_relu_tiebreak_band():
     Hk[0][tuple(pos)] = 0.0
     with pytest.raises(AssertionError):
         relu_tiebreak(ref, Hk)
+
+
+def _biases(f, seed=21):
+    rng = np.random.default_rng(seed)
+    return [rng.standard_normal(f[l]) * 0.3 for l in range(1, len(f))]
+
+
+def test_bias_identity_graph_is_mlp_with_bias():
+    """Â = I with biases (reading R8): torch.nn.Linear(bias=True) layers give
+    the logits, and autograd gives dW and db (pin P4-i with bias)."""
+    n, f = 30, (5, 4, 3)
+    g = synth.identity_graph(n)
+    H0 = synth.features(n, f[0])
+    Ws = synth.weights(f)
+    bs = _biases(f)
+    y = synth.labels(n, f[-1])
+    m = synth.train_mask(n)
+    res = gcn.epoch(g, H0, Ws, y, m, bs)
+    lin = [torch.nn.Linear(f[i], f[i + 1], bias=True).double() for i in range(2)]
+    with torch.no_grad():
+        for i in range(2):
+            lin[i].weight.copy_(torch.tensor(Ws[i].astype(np.float64).T))
+            lin[i].bias.copy_(torch.tensor(bs[i]))
+    out = lin[1](torch.relu(lin[0](torch.tensor(H0.astype(np.float64)))))
+    mt = torch.tensor(m.astype(bool))
+    loss = torch.nn.functional.cross_entropy(out[mt], torch.tensor(y, dtype=torch.long)[mt])
+    loss.backward()
+    np.testing.assert_allclose(res.Z[2], out.detach().numpy(), atol=1e-13)
+    assert abs(res.loss - float(loss)) <= 1e-12 * abs(float(loss))
+    for l in (1, 2):
+        np.testing.assert_allclose(res.db[l], lin[l - 1].bias.grad.numpy(), atol=1e-13)
+        np.testing.assert_allclose(res.Y[l], lin[l - 1].weight.grad.numpy().T, atol=1e-13)
+
+
+def test_bias_finite_differences_three_layers():
+    """Central differences on b^l entries of a 3-layer GCN on an R-MAT graph
+    (pin P3 for db^l = 1ᵀ G^l); also checks dW with biases present."""
+    n, f = 40, (6, 5, 4, 3)
+    g = synth.rmat(n, 120, seed=12)
+    H0 = synth.features(n, f[0]).astype(np.float64)
+    Ws = [w.astype(np.float64) for w in synth.weights(f)]
+    bs = _biases(f)
+    y = synth.labels(n, f[-1])
+    m = synth.train_mask(n)
+    res = gcn.epoch(g, H0, Ws, y, m, bs)
+    rng = np.random.default_rng(9)
+    checked = 0
+    for l in range(1, len(f)):
+        for j in range(f[l]):
+            h = 1e-6
+            bp = [b.copy() for b in bs]
+            bm = [b.copy() for b in bs]
+            bp[l - 1][j] += h
+            bm[l - 1][j] -= h
+            rp, rm = gcn.forward(g, H0, Ws, y, m, bp), gcn.forward(g, H0, Ws, y, m, bm)
+            if any(np.any(np.sign(rp.Z[k]) != np.sign(rm.Z[k])) for k in range(1, len(f) - 1)):
+                continue
+            fd = (rp.loss - rm.loss) / (2 * h)
+            assert abs(fd - res.db[l][j]) <= 1e-6 * max(1e-3, abs(fd)), (l, j, fd, res.db[l][j])
+            checked += 1
+        i, j = rng.integers(0, f[l - 1]), rng.integers(0, f[l])
+        h = 1e-6 * max(1.0, abs(Ws[l - 1][i, j]))
+        Wp = [w.copy() for w in Ws]
+        Wm = [w.copy() for w in Ws]
+        Wp[l - 1][i, j] += h
+        Wm[l - 1][i, j] -= h
+        rp, rm = gcn.forward(g, H0, Wp, y, m, bs), gcn.forward(g, H0, Wm, y, m, bs)
+        fd = (rp.loss - rm.loss) / (2 * h)
+        assert abs(fd - res.Y[l][i, j]) <= 1e-6 * max(1e-3, abs(fd))
+    assert checked >= 8
