@@ -108,7 +108,12 @@ typedef struct {
 enum {
   RDM_GCN_INPUT_GRAD = 1, /* also compute G^0 = A G^1 (W^1)ᵀ (Fig. 4 output; reading R2) —
                              required for costs to match Table IV                       */
-  RDM_GCN_BIAS = 2,       /* Z = Â H W + 1 bᵀ (reading R8); not implemented: UNSUPPORTED */
+  RDM_GCN_BIAS = 2,       /* Z^l = Â H^{l-1} W^l + 1 (b^l)ᵀ before σ (reading R8): the bias
+                             is fused into the epilogue of Z^l's producer (the SpMM or the
+                             GEMM, whichever runs last for the layer's config); the backward
+                             pass adds db^l = 1ᵀ G^l (deterministic fp64 column sums of the
+                             masked G^l in whatever layout it is resident, all-reduced with
+                             Y^l).  rdm_gcn_forward/backward then require b / db.          */
   RDM_GCN_PANELS = 4,     /* R_A < P (§III-E): run on the row panels installed by
                              rdm_set_graph_panels (a symmetric A) instead of the replicated
                              graph; column-layout tensors are tiles (rdm_partition_tile),
@@ -440,14 +445,18 @@ rdm_status rdm_gcn_set_input(rdm_gcn* g, const float* const* H0_row,
 
 /* Forward pass of all layers + loss (eq. 1-2; loss L206, reading R5).  W[l]
  * (l = 0..L-1) = W^{l+1}, f_l x f_{l+1} row-major, replicated (one copy per
- * process).  loss_dev: device double, receives the global mean loss.
+ * process).  b: with RDM_GCN_BIAS, b[l] = b^{l+1} (f_{l+1} floats, device,
+ * replicated), RDM_ERR_ARG if b or any b[l] is null; ignored otherwise (may
+ * be null).  loss_dev: device double, receives the global mean loss.
  * Collective. */
 rdm_status rdm_gcn_forward(rdm_gcn* g, const float* const* W, const float* const* b,
                            double* loss_dev);
 
 /* Backward pass (eq. 3-4) with fwd→bwd memo reuse (§III-C):
  * dW[l] receives Y^{l+1}, all-reduced over ranks (one copy per process);
- * db ignored (bias unsupported).  Collective. */
+ * with RDM_GCN_BIAS, db[l] (f_{l+1} floats, device) receives db^{l+1} =
+ * 1ᵀ G^{l+1}, all-reduced likewise (RDM_ERR_ARG if null); db is ignored
+ * otherwise.  Collective. */
 rdm_status rdm_gcn_backward(rdm_gcn* g, const float* const* W, float* const* dW, float* const* db);
 
 /* What the executor will run for this instance (per epoch, per rank):

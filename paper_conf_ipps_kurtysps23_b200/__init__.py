@@ -268,7 +268,7 @@ def redist_plan(world, rank, from_layout, n, f):
     return {k: list(a) for k, a in zip(keys, arrs)}
 
 
-def plan_info(f, cfg, P, n, input_grad=True, low_memory=False):
+def plan_info(f, cfg, P, n, input_grad=True, low_memory=False, bias=False):
     """→ (info dict, step list text) of the executor plan, without a GPU
     (workspace_bytes: rank 0's activation workspace)."""
     L = len(f) - 1
@@ -276,7 +276,8 @@ def plan_info(f, cfg, P, n, input_grad=True, low_memory=False):
     fa = (ctypes.c_int64 * len(f))(*f)
     info = RdmGcnInfo()
     buf = ctypes.create_string_buffer(1 << 16)
-    flags = (GCN_INPUT_GRAD if input_grad else 0) | (GCN_LOW_MEMORY if low_memory else 0)
+    flags = ((GCN_INPUT_GRAD if input_grad else 0) | (GCN_LOW_MEMORY if low_memory else 0)
+             | (GCN_BIAS if bias else 0))
     _check(_lib.rdm_plan_info(L, fa, ctypes.byref(c), P, n, flags,
                               ctypes.byref(info), buf, len(buf)), what="rdm_plan_info")
     return info.as_dict(), buf.value.decode()
@@ -444,7 +445,7 @@ class GCN:
     """A GCN instance (L layers, widths f) running configuration `cfg` (ID or RdmConfig)."""
 
     def __init__(self, ctx: Context, f, cfg, input_grad=True, saint=None, panels=False,
-                 low_memory=False):
+                 low_memory=False, bias=False):
         self.ctx = ctx
         self.f = list(f)
         self.L = len(f) - 1
@@ -452,7 +453,8 @@ class GCN:
         fa = (ctypes.c_int64 * len(f))(*f)
         h = ctypes.c_void_p()
         flags = ((GCN_INPUT_GRAD if input_grad else 0) | (GCN_PANELS if panels else 0)
-                 | (GCN_LOW_MEMORY if low_memory else 0))
+                 | (GCN_LOW_MEMORY if low_memory else 0) | (GCN_BIAS if bias else 0))
+        self.bias = bool(bias)
         self.saint = saint   # keeps the sampler alive while this instance exists
         if saint is None:
             ctx._c(_lib.rdm_gcn_create(ctx.h, self.L, fa, ctypes.byref(self.cfg), flags,
@@ -493,14 +495,18 @@ class GCN:
                                              _ptr(labels_full),
                                              None if mask_full is None else _ptr(mask_full)))
 
-    def forward(self, Ws, loss_dev):
+    def forward(self, Ws, loss_dev, bs=None):
+        """bs: the L bias vectors b^l (f_l floats each, device) of a bias=True model."""
         wp, _a = _parr(Ws)
-        self.ctx._c(_lib.rdm_gcn_forward(self.h, wp, None, _ptr(loss_dev)))
+        bp, _b = _parr(bs) if bs is not None else (None, None)
+        self.ctx._c(_lib.rdm_gcn_forward(self.h, wp, bp, _ptr(loss_dev)))
 
-    def backward(self, Ws, dWs):
+    def backward(self, Ws, dWs, dbs=None):
+        """dbs: the L bias gradients db^l (f_l floats each, device) of a bias=True model."""
         wp, _a = _parr(Ws)
         dp, _b = _parr(dWs)
-        self.ctx._c(_lib.rdm_gcn_backward(self.h, wp, dp, None))
+        bp, _c2 = _parr(dbs) if dbs is not None else (None, None)
+        self.ctx._c(_lib.rdm_gcn_backward(self.h, wp, dp, bp))
 
     def info(self) -> dict:
         i = RdmGcnInfo()
@@ -582,8 +588,8 @@ class Saint:
                      torch.zeros(s, dtype=tt[t], device=dev)
                      for p, s, t in zip(ps, shapes, types))
 
-    def gcn(self, f, cfg, input_grad=True):
-        return GCN(self.ctx, f, cfg, input_grad=input_grad, saint=self)
+    def gcn(self, f, cfg, input_grad=True, bias=False):
+        return GCN(self.ctx, f, cfg, input_grad=input_grad, saint=self, bias=bias)
 
     def close(self):
         if getattr(self, "h", None):

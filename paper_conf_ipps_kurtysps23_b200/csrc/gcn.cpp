@@ -38,7 +38,7 @@ struct Key {
   int kind = 0, layer = 0;
   int id() const { return kind * 64 + layer; }
 };
-enum Op { S_SPMM = 0, S_GEMM, S_TN, S_REDIST, S_MASK, S_LOSS };
+enum Op { S_SPMM = 0, S_GEMM, S_TN, S_REDIST, S_MASK, S_LOSS, S_COLSUM };
 
 struct Step {
   int op = 0;
@@ -48,6 +48,7 @@ struct Step {
   int64_t width = 0;
   bool hidden = false;
   int fuse = 0;   // RDM_TRANSPORT_P2P: 1 = producer also scatters (next step), 2 = redist done by producer
+  int bl = 0;     // RDM_GCN_BIAS: layer whose bias b^bl this step adds (0 = none) / sums (S_COLSUM)
 };
 
 struct Planner {
@@ -55,6 +56,7 @@ struct Planner {
   std::vector<int64_t> f;
   rdm_config cfg{};
   bool igrad = true;
+  bool bias = false;   // RDM_GCN_BIAS (reading R8): Z^l = Â H W + 1 b^lᵀ, db^l = 1ᵀ G^l
   std::set<std::pair<int, int>> res, masked;
   std::map<int, int64_t> width;
   std::set<int> pending;
@@ -135,6 +137,15 @@ struct Planner {
     produce(out, RDM_ROW, w);
     if (epi & RDM_EPI_MASK) masked.insert({out.id(), lay(RDM_ROW)});
   }
+  void colsum(Key gk, int ly, int l) {   // db^l = 1ᵀ G^l from its resident (masked) layout
+    Step s;
+    s.op = S_COLSUM;
+    s.in = gk;
+    s.lin = ly;
+    s.bl = l;
+    s.width = f[l];
+    cur->push_back(s);
+  }
   void tn(Key x, Key u, int wl) {
     Step s;
     s.op = S_TN;
@@ -154,17 +165,20 @@ struct Planner {
     for (int l = 1; l <= L; ++l) {
       Key hin{K_H, l - 1}, hout = l < L ? Key{K_H, l} : Key{K_Z, 0}, t{K_T, l};
       const int epi = l < L ? RDM_EPI_RELU : 0;
+      const int be = bias ? RDM_EPI_BIAS : 0;   // bias before ReLU, after both products (R8)
       if (!cfg.fwd_D[l - 1]) {
         need(hin, RDM_COL, false);
         spmm(1, hin, t, f[l - 1]);
         need(t, RDM_ROW, false);
-        gemm(RDM_GEMM_NN, t, l, hout, f[l], epi);
+        gemm(RDM_GEMM_NN, t, l, hout, f[l], epi | be);
+        cur->back().bl = bias ? l : 0;
         memo[l] = true;
       } else {
         need(hin, RDM_ROW, false);
         gemm(RDM_GEMM_NN, hin, l, t, f[l]);
         need(t, RDM_COL, false);
-        spmm(1, t, hout, f[l], epi);
+        spmm(1, t, hout, f[l], epi | be);
+        cur->back().bl = bias ? l : 0;
       }
     }
     need({K_Z, 0}, RDM_ROW, false);
@@ -185,6 +199,7 @@ struct Planner {
       const bool out = l > 1 || igrad;
       if (!cfg.bwd_D[l - 1]) {
         needG(l, RDM_COL);
+        if (bias) colsum(g, RDM_COL, l);
         Key u{K_U, l};
         spmm(0, g, u, f[l]);
         need(u, RDM_ROW, false);
@@ -206,6 +221,7 @@ struct Planner {
         }
       } else {
         needG(l, RDM_ROW);
+        if (bias) colsum(g, RDM_ROW, l);
         Key v{K_V, l};
         gemm(RDM_GEMM_NT, g, l, v, f[l - 1]);
         if (memo[l]) tn(t, g, l);
@@ -336,6 +352,9 @@ std::vector<BufPlan> buffer_lifetimes(const Planner& pl, const std::vector<Step>
           use(s.in, s.lin, t, t);
           use(s.out, s.lout, t, t);
           break;
+        case S_COLSUM:
+          use(s.in, s.lin, t, t);
+          break;
       }
       ++t;
     }
@@ -401,6 +420,8 @@ struct rdm_gcn {
   // per slot: (key id, layout) → buffer
   std::vector<std::map<std::pair<int, int>, Buf>> bufs;
   std::vector<std::vector<float*>> dwp;     // per slot per layer partial Y (virtual group)
+  std::vector<std::vector<float*>> dbp;     // RDM_GCN_BIAS: per slot per layer partial db (virtual group)
+  const float* const* bcur = nullptr;       // RDM_GCN_BIAS: the forward pass's b^l (device, f_l floats)
   std::vector<int32_t*> labels;
   std::vector<uint8_t*> mask;
   std::vector<double*> scal;                // per slot: [0] n_train, [1] loss partial
@@ -594,6 +615,7 @@ void create(rdm_gcn* g) {
   pl.f = g->f;
   pl.cfg = g->cfg;
   pl.igrad = (g->flags & RDM_GCN_INPUT_GRAD) != 0;
+  pl.bias = (g->flags & RDM_GCN_BIAS) != 0;
   pl.plan(g->fwd, g->bwd);
   g->bufs.assign(ctx->nlocal(), {});
   const bool low_memory = (g->flags & RDM_GCN_LOW_MEMORY) != 0;
@@ -650,6 +672,7 @@ void create(rdm_gcn* g) {
   const int P = ctx->world;
   const int64_t n = g->n_cap;
   g->dwp.assign(ctx->nlocal(), std::vector<float*>(g->L + 1, nullptr));
+  g->dbp.assign(ctx->nlocal(), std::vector<float*>(g->L + 1, nullptr));
   g->labels.assign(ctx->nlocal(), nullptr);
   g->mask.assign(ctx->nlocal(), nullptr);
   g->scal.assign(ctx->nlocal(), nullptr);
@@ -659,6 +682,10 @@ void create(rdm_gcn* g) {
       for (int l = 1; l <= g->L; ++l) {
         g->mem.emplace_back(new DevBuf((size_t)g->f[l - 1] * g->f[l] * sizeof(float)));
         g->dwp[s][l] = g->mem.back()->as<float>();
+        if (g->flags & RDM_GCN_BIAS) {
+          g->mem.emplace_back(new DevBuf((size_t)g->f[l] * sizeof(float)));
+          g->dbp[s][l] = g->mem.back()->as<float>();
+        }
       }
     }
     g->mem.emplace_back(new DevBuf(std::max<int64_t>(r, 1) * sizeof(int32_t)));
@@ -710,7 +737,7 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
           out[i] = buf(g, i, s.out, s.lout).p;
           mk[i] = (s.epi & RDM_EPI_MASK) ? buf(g, i, s.mask, s.lmask).p : nullptr;
         }
-        spmm_panels(ctx, in.data(), out.data(), s.width, s.epi, nullptr,
+        spmm_panels(ctx, in.data(), out.data(), s.width, s.epi, s.bl ? g->bcur[s.bl - 1] : nullptr,
                     (s.epi & RDM_EPI_MASK) ? mk.data() : nullptr);
         break;
       }
@@ -726,13 +753,16 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
           mk = m.p;
           ldm = m.ld;
         }
-        const int64_t w = P == 1 ? s.width : col_range(s.width, P, ctx->local[i]).size();
+        const Range cr = P == 1 ? Range{0, s.width} : col_range(s.width, P, ctx->local[i]);
+        const int64_t w = cr.size();
+        // bias of the column slice (reading R8: added after both products, before σ)
+        const float* bias = s.bl ? g->bcur[s.bl - 1] + cr.lo : nullptr;
         ctx->spmm_in_bf16 = g->wire_bf16.count({s.in.id(), norm_lay(g, s.lin)}) > 0;
         if (s.fuse == 1) {
           const Scatter sc = make_scatter(g, s, i);
-          spmm(ctx, A, in.p, in.ld, out.p, out.ld, w, s.epi, nullptr, mk, ldm, &sc);
+          spmm(ctx, A, in.p, in.ld, out.p, out.ld, w, s.epi, bias, mk, ldm, &sc);
         } else {
-          spmm(ctx, A, in.p, in.ld, out.p, out.ld, w, s.epi, nullptr, mk, ldm);
+          spmm(ctx, A, in.p, in.ld, out.p, out.ld, w, s.epi, bias, mk, ldm);
         }
         ctx->spmm_in_bf16 = false;
       }
@@ -779,7 +809,7 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
           ctx->gemm_mask_bits_ld = g->mbits_ld[mkey];
         }
         gemm(ctx, s.gop, in.p, in.ld, W[s.wl - 1], fout, out.p, out.ld, in.rows, fin, fout, s.epi,
-             nullptr, mk, s.fuse == 1 ? &sc : nullptr);
+             s.bl ? g->bcur[s.bl - 1] : nullptr, mk, s.fuse == 1 ? &sc : nullptr);
         if (ctx->gemm_bits_out) {
           if (ctx->gemm_bits_written) g->mb_valid.insert(okey);
           else g->mb_valid.erase(okey);
@@ -857,6 +887,27 @@ void run_step(rdm_gcn* g, const Step& s, const float* const* W) {
       }
       break;
     }
+    case S_COLSUM: {   // db^l partial of this slot: 1ᵀ G^l over its rows, at its column offset
+      Phase ph(ctx, RDM_PH_OTHER);
+      for (int i = 0; i < nl; ++i) {
+        Buf& x = buf(g, i, s.in, s.lin);
+        float* dst = g->dbp[i][s.bl];
+        int64_t lo = 0;
+        if (s.lin == RDM_COL && P > 1) {
+          if (g->RA) {
+            Range r, c;
+            int64_t ld;
+            tile_of(P, g->RA, gn(g), s.width, ctx->local[i], &r, &c, &ld);
+            lo = c.lo;
+          } else {
+            lo = col_range(s.width, P, ctx->local[i]).lo;
+          }
+        }
+        if (x.cols < s.width) RDM_CUDA(cudaMemsetAsync(dst, 0, s.width * sizeof(float), ctx->stream));
+        colsum(ctx, x.p, x.ld, x.rows, x.cols, dst + lo);
+      }
+      break;
+    }
     case S_LOSS: {
       Phase ph(ctx, RDM_PH_LOSS);
       for (int i = 0; i < nl; ++i) {
@@ -899,7 +950,11 @@ std::string step_str(const Step& s) {
     case S_LOSS:
       o << "LOSS  " << k(s.in, s.lin) << " -> " << k(s.out, s.lout);
       break;
+    case S_COLSUM:
+      o << "BSUM  1^T " << k(s.in, s.lin) << " -> db" << s.bl;
+      break;
   }
+  if ((s.op == S_SPMM || s.op == S_GEMM) && s.bl) o << " +b" << s.bl;
   return o.str();
 }
 
@@ -914,12 +969,14 @@ std::string describe_steps(const std::vector<Step>& fwd, const std::vector<Step>
 struct FwdArgs {
   rdm_gcn* g;
   const float* const* W;
+  const float* const* b;
   double* loss;
 };
 struct BwdArgs {
   rdm_gcn* g;
   const float* const* W;
   float* const* dW;
+  float* const* db;
 };
 
 void consume_staged(rdm_gcn* g);
@@ -932,11 +989,17 @@ void do_forward(void* a_) {
   if (!g->input_set) throw Error(RDM_ERR_STATE, "rdm_gcn_forward: call rdm_gcn_set_input first");
   RDM_CHECK_ARG(a->W && a->loss, "rdm_gcn_forward: W and loss_dev required");
   for (int l = 0; l < g->L; ++l) RDM_CHECK_ARG(a->W[l], "rdm_gcn_forward: null W");
+  const bool bias = (g->flags & RDM_GCN_BIAS) != 0;
+  RDM_CHECK_ARG(!bias || a->b, "rdm_gcn_forward: the model has biases (RDM_GCN_BIAS): b required");
+  if (bias)
+    for (int l = 0; l < g->L; ++l) RDM_CHECK_ARG(a->b[l], "rdm_gcn_forward: null b");
+  g->bcur = bias ? a->b : nullptr;
   if (g->staged) {
     Phase ph(ctx, RDM_PH_OTHER);
     consume_staged(g);
   }
   for (auto& s : g->fwd) run_step(g, s, a->W);
+  g->bcur = nullptr;
   const int nl = ctx->nlocal();
   std::vector<double*> parts(nl);
   for (int i = 0; i < nl; ++i) parts[i] = g->scal[i] + 1;
@@ -959,8 +1022,15 @@ void do_backward(void* a_) {
   if (g->saint && g->gver != g->saint->version)
     throw Error(RDM_ERR_STATE, "rdm_gcn_backward: the subgraph changed since the forward pass");
   for (int l = 0; l < g->L; ++l) RDM_CHECK_ARG(a->W[l] && a->dW[l], "rdm_gcn_backward: null W/dW");
+  const bool bias = (g->flags & RDM_GCN_BIAS) != 0;
+  RDM_CHECK_ARG(!bias || a->db, "rdm_gcn_backward: the model has biases (RDM_GCN_BIAS): db required");
+  if (bias)
+    for (int l = 0; l < g->L; ++l) RDM_CHECK_ARG(a->db[l], "rdm_gcn_backward: null db");
   if (!ctx->virtual_group())
-    for (int l = 1; l <= g->L; ++l) g->dwp[0][l] = a->dW[l - 1];
+    for (int l = 1; l <= g->L; ++l) {
+      g->dwp[0][l] = a->dW[l - 1];
+      if (bias) g->dbp[0][l] = a->db[l - 1];
+    }
   for (auto& s : g->bwd) run_step(g, s, a->W);
   if (g->side_pending) {   // every weight gradient is in place before the reduction
     RDM_CUDA(cudaEventRecord(g->ev_join, g->side));
@@ -983,6 +1053,18 @@ void do_backward(void* a_) {
     } else {
       float* b = a->dW[l - 1];
       allreduce(ctx, &b, cnt);
+    }
+    if (bias) {   // db^l: the slots' partials (row slices / column ranges) summed like Y^l
+      if (ctx->virtual_group()) {
+        Phase ph(ctx, RDM_PH_ALLREDUCE);
+        std::vector<const float*> parts(nl);
+        for (int i = 0; i < nl; ++i) parts[i] = g->dbp[i][l];
+        sum_slots(ctx, a->db[l - 1], parts.data(), nl, g->f[l]);
+        ctx->counters.allreduce_bytes += g->f[l] * 4;
+      } else {
+        float* b = a->db[l - 1];
+        allreduce(ctx, &b, g->f[l]);
+      }
     }
   }
 }
@@ -1176,10 +1258,6 @@ rdm_status rdm_gcn_create(rdm_ctx* ctx, int L, const int64_t* f, const rdm_confi
   if (!ctx || !out || !f || !cfg || L < 1 || L > RDM_MAX_LAYERS || cfg->L != L) return RDM_ERR_ARG;
   for (int l = 0; l <= L; ++l)
     if (f[l] < 1) return RDM_ERR_ARG;
-  if (flags & RDM_GCN_BIAS) {
-    ctx->err = "rdm_gcn_create: RDM_GCN_BIAS is not implemented";
-    return RDM_ERR_UNSUPPORTED;
-  }
   const bool panels = (flags & RDM_GCN_PANELS) != 0;
   if (panels && ctx->panel_RA <= 0) {
     ctx->err = "rdm_gcn_create: RDM_GCN_PANELS needs rdm_set_graph_panels";
@@ -1213,10 +1291,6 @@ rdm_status rdm_saint_gcn_create(rdm_saint* s, int L, const int64_t* f, const rdm
   rdm_ctx* ctx = s->ctx;
   for (int l = 0; l <= L; ++l)
     if (f[l] < 1) return RDM_ERR_ARG;
-  if (flags & RDM_GCN_BIAS) {
-    ctx->err = "rdm_saint_gcn_create: RDM_GCN_BIAS is not implemented";
-    return RDM_ERR_UNSUPPORTED;
-  }
   auto* g = new rdm_gcn();
   g->ctx = ctx;
   g->graph = &s->graph();
@@ -1277,16 +1351,14 @@ rdm_status rdm_gcn_set_input(rdm_gcn* g, const float* const* H0_row, const int32
 
 rdm_status rdm_gcn_forward(rdm_gcn* g, const float* const* W, const float* const* b,
                            double* loss_dev) {
-  (void)b;
   if (!g) return RDM_ERR_ARG;
-  FwdArgs a{g, W, loss_dev};
+  FwdArgs a{g, W, b, loss_dev};
   return rdm_guarded_call(g->ctx, do_forward, &a);
 }
 
 rdm_status rdm_gcn_backward(rdm_gcn* g, const float* const* W, float* const* dW, float* const* db) {
-  (void)db;
   if (!g) return RDM_ERR_ARG;
-  BwdArgs a{g, W, dW};
+  BwdArgs a{g, W, dW, db};
   return rdm_guarded_call(g->ctx, do_backward, &a);
 }
 
@@ -1352,6 +1424,7 @@ extern "C" rdm_status rdm_plan_info(int L, const int64_t* f, const rdm_config* c
     pl.f.assign(f, f + L + 1);
     pl.cfg = *cfg;
     pl.igrad = (flags & RDM_GCN_INPUT_GRAD) != 0;
+    pl.bias = (flags & RDM_GCN_BIAS) != 0;
     std::vector<Step> fwd, bwd;
     pl.plan(fwd, bwd);
     if (out) {

@@ -419,6 +419,8 @@ void softmax_xent(rdm_ctx* ctx, const float* Z, int64_t ldz, const int32_t* labe
                   const uint8_t* mask, int64_t rows, int64_t C, const double* n_train, float* G,
                   int64_t ldg, double* loss_partial);
 void count_mask(rdm_ctx* ctx, const uint8_t* mask, int64_t rows, double* out);
+// out[c] = Σ_r G[r, c] (fp64 accumulation, fixed order), c < cols
+void colsum(rdm_ctx* ctx, const float* G, int64_t ldg, int64_t rows, int64_t cols, float* out);
 void apply_mask(rdm_ctx* ctx, float* X, int64_t ldx, const float* H, int64_t ldh, int64_t rows,
                 int64_t cols);
 void sum_slots(rdm_ctx* ctx, float* out, const float* const* parts, int nparts, int64_t count);

@@ -225,6 +225,40 @@ __global__ void apply_mask_kernel(float* __restrict__ X, int64_t ldx, const floa
   }
 }
 
+// db^l = 1ᵀ G^l (reading R8), deterministic: CTA (column tile of 32, row
+// chunk) — lane = column, warp w sums rows chunk_lo + w, + 8, … in fp64 (each
+// warp load is one 128-byte row segment); the 8 warp sums are added in warp
+// order and the chunk partials in chunk order by colsum_finish_kernel.
+constexpr int kColsumRows = 512;   // rows per chunk
+__global__ void __launch_bounds__(256) colsum_kernel(const float* __restrict__ G, int64_t ldg,
+                                                     int64_t rows, int64_t cols, int64_t rows_per,
+                                                     double* __restrict__ part) {
+  __shared__ double red[8][33];
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  const int64_t c = (int64_t)blockIdx.x * 32 + lane;
+  const int64_t r0 = (int64_t)blockIdx.y * rows_per, r1 = min(rows, r0 + rows_per);
+  double s = 0.0;
+  if (c < cols)
+    for (int64_t r = r0 + warp; r < r1; r += 8) s += (double)__ldg(G + r * ldg + c);
+  red[warp][lane] = s;
+  __syncthreads();
+  if (warp == 0) {
+    double t = 0.0;
+#pragma unroll
+    for (int w = 0; w < 8; ++w) t += red[w][lane];
+    if (c < cols) part[(int64_t)blockIdx.y * cols + c] = t;
+  }
+}
+
+__global__ void colsum_finish_kernel(const double* __restrict__ part, int nchunks, int64_t cols,
+                                     float* __restrict__ out) {
+  const int64_t c = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (c >= cols) return;
+  double t = 0.0;
+  for (int k = 0; k < nchunks; ++k) t += part[(int64_t)k * cols + c];
+  out[c] = (float)t;
+}
+
 struct PtrTab {
   const float* p[BlockTable::kMax];
 };
@@ -343,6 +377,20 @@ void apply_mask(rdm_ctx* ctx, float* X, int64_t ldx, const float* H, int64_t ldh
   const int64_t c4 = roundup4(cols) / 4;
   if (rows * c4 == 0) return;
   apply_mask_kernel<<<grid_for(ctx, rows * c4), 256, 0, ctx->stream>>>(X, ldx, H, ldh, rows, c4);
+  RDM_LAUNCHED(ctx);
+}
+
+void colsum(rdm_ctx* ctx, const float* G, int64_t ldg, int64_t rows, int64_t cols, float* out) {
+  if (cols <= 0) return;
+  const int64_t ct = (cols + 31) / 32;
+  // ~4 CTAs per SM over the whole grid, chunks of at least kColsumRows rows
+  const int64_t want = std::max<int64_t>(1, (int64_t)4 * ctx->num_sms / ct);
+  const int64_t nchunks = std::max<int64_t>(1, std::min(want, ceil_div(rows, kColsumRows)));
+  const int64_t rows_per = std::max<int64_t>(1, ceil_div(rows, nchunks));
+  double* part = reinterpret_cast<double*>(ensure_ws(ctx->ws_scratch, (size_t)nchunks * cols * sizeof(double)));
+  colsum_kernel<<<dim3((unsigned)ct, (unsigned)nchunks), 256, 0, ctx->stream>>>(G, ldg, rows, cols, rows_per, part);
+  RDM_LAUNCHED(ctx);
+  colsum_finish_kernel<<<(unsigned)ceil_div(cols, 128), 128, 0, ctx->stream>>>(part, (int)nchunks, cols, out);
   RDM_LAUNCHED(ctx);
 }
 

@@ -491,8 +491,7 @@ void build_core_sub(rdm_saint* s, Csr& S, int64_t kmax, const unsigned long long
   int32_t* nseg = reinterpret_cast<int32_t*>(ensure_ws(s->core_seg, (2 * (n + 1) + seg_cap) * 4 + 16));
   int32_t* segoff = nseg + (n + 1);
   int32_t* seg_row = segoff + (n + 1);
-  int64_t* cnt = reinterpret_cast<int64_t*>(ensure_ws(s->core_cnt, 2 * seg_cap * sizeof(int64_t)));
-  int64_t* pos = cnt + seg_cap;
+  ensure_ws(s->core_cnt, 2 * seg_cap * sizeof(int64_t));   // sized here: the residual pass reuses it
   unsigned long long* bucket = reinterpret_cast<unsigned long long*>(ensure_ws(s->core_bucket, kMaxBuckets * 8));
   rowseg_kernel<<<grid_of(ctx, n + 1, 256), 256, 0, ctx->stream>>>(rp, nullptr, n, nullptr, n, nseg);
   RDM_LAUNCHED(ctx);

@@ -264,3 +264,32 @@ def test_feature_row_slices_match_whole_draw():
     assert np.array_equal(H[1234:2999], synth.features_rows(1234, 2999, 17))
     y = synth.labels(3001, 41)
     assert np.array_equal(y[7:3001], synth.labels_rows(7, 3001, 41))
+
+
+@pytest.mark.parametrize("f,P", [([1433, 128, 7], 1), ([602, 128, 41], 4), ([100, 256, 256, 47], 8)])
+def test_bias_plan(f, P):
+    """RDM_GCN_BIAS (reading R8): in every configuration each layer's bias is
+    fused into exactly one producer of Z^l — the last product of the layer
+    (GEMM for order S, SpMM for order D) — and db^l is summed exactly once from
+    G^l after its Hadamard mask; nothing else in the plan changes."""
+    L = len(f) - 1
+    for cid in range(4 ** L):
+        a, da = rdm.plan_info(f, cid, P, 10007)
+        b, db = rdm.plan_info(f, cid, P, 10007, bias=True)
+        for k in ("plan_comm_units", "plan_sparse_units", "a2a_elems", "workspace_bytes"):
+            assert a[k] == b[k], (cid, k)
+        cfg = rdm.config_from_id(L, cid)
+        fwd, bwd = db.split("backward:")
+        for l in range(1, L + 1):
+            adds = [s for s in fwd.splitlines() if s.endswith(f" +b{l}")]
+            assert len(adds) == 1, (cid, l, fwd)
+            kind = "SPMM" if cfg.fwd_D[l - 1] else "GEMM"
+            assert adds[0].strip().startswith(kind), (cid, l, adds)
+            assert f"-> {'Z0' if l == L else f'H{l}'}." in adds[0], adds   # Z^L is stored as Z0
+            sums = [i for i, s in enumerate(bwd.splitlines()) if s.strip().endswith(f"-> db{l}")]
+            assert len(sums) == 1, (cid, l, bwd)
+        # with the bias lines removed the plan is the bias-free plan
+        clean = "\n".join(s for s in db.splitlines() if "BSUM" not in s)
+        for l in range(1, L + 1):
+            clean = clean.replace(f" +b{l}", "")
+        assert clean == da.rstrip("\n") or clean + "\n" == da, cid
