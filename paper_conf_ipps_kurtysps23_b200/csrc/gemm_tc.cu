@@ -28,6 +28,7 @@
 #include <cuda_bf16.h>
 
 #include <algorithm>
+#include <cstdio>
 #include <cstdlib>
 #include <cstring>
 
@@ -80,26 +81,37 @@ struct TcShape {
 // EW = epilogue warps: 4 (one per TMEM lane quadrant) for mainloop-bound
 // calls, 8 (two per quadrant, column halves) for epilogue-bound ones (short
 // K, wide outputs) — 8 warps cost one smem stage of transpose buffers.
-template <int BN, int EW>
+// PAIR = 2: a CTA pair (cluster of 2, tcgen05 cta_group::2) computes a
+// 256 x BN tile: each CTA holds its own 128 rows of A and HALF of the B panel
+// (BN/2 rows), the leader's MMAs (M = 256) read both halves, so every SM loads
+// half the W panel bytes per row it computes.
+// ASM = 1 (pairs, BN <= 128): A split in shared memory instead of TMEM, which
+// leaves TMEM to two partial accumulators per buffer (the three MMAs of a k
+// step alternate between them instead of serialising on one).
+template <int BN, int EW, int PAIR = 1, int ASM = 0>
 struct Cfg {
   static constexpr int kThreads = 256 + 32 * EW;
   static constexpr int kAccCols = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
-  static constexpr bool kTmemA = BN <= 128;
-  static constexpr int kNAcc = !kTmemA ? 1 : BN <= 32 ? 4 : BN <= 64 ? 2 : 1;  // partial accumulators
+  static constexpr bool kTmemA = BN <= 128 && !ASM;
+  static constexpr int kNAcc = !kTmemA ? (BN <= 128 ? 2 : 1) : BN <= 32 ? 4 : BN <= 64 ? 2 : 1;  // partial accumulators
   static constexpr int kABytes = BM * BK * 4;   // 16 KB
-  static constexpr int kBBytes = BN * BK * 4;
+  static constexpr int kBBytes = (BN / PAIR) * BK * 4;
   static constexpr int kStageBytes = (kTmemA ? 1 : 2) * kABytes + 2 * kBBytes;
   // per epilogue warp 5 KB (1024-aligned): a 32 x 33 transpose tile, or the
   // 32 x 32 swizzled box of a TMA store
   static constexpr int kEpiBytes = EW * 5120;
-  static constexpr int kBudget = 224 * 1024 - kEpiBytes - 1024 - 256;
-  // deep rings hide TMA latency; with A in TMEM each stage also takes 64 columns
-  static constexpr int kMaxStages = kTmemA ? (512 - 2 * kNAcc * kAccCols) / (2 * BK) : 4;
+  static constexpr int kBudget = 224 * 1024 - kEpiBytes - 1024 - 512;
+  // deep rings hide TMA latency.  With A in TMEM the converted A stages form
+  // a second ring (64 TMEM columns each, whatever the accumulators leave),
+  // decoupled from the smem ring of raw A + B tiles, which can run deeper.
+  static constexpr int kStagesT0 = kTmemA ? (512 - 2 * kNAcc * kAccCols) / (2 * BK) : 0;
+  static constexpr int kStagesT = kStagesT0 < 8 ? kStagesT0 : 8;
+  static constexpr int kMaxStages = kTmemA ? 8 : 4;
   static constexpr int kFitStages = kBudget / kStageBytes < 8 ? kBudget / kStageBytes : 8;
   static constexpr int kStages = kFitStages < kMaxStages ? kFitStages : kMaxStages;
-  static constexpr int kSmem = kStages * kStageBytes + kEpiBytes + 1024 /*align*/ + 256 /*barriers*/;
+  static constexpr int kSmem = kStages * kStageBytes + kEpiBytes + 1024 /*align*/ + 512 /*barriers*/;
   static constexpr int kACol0 = 2 * kNAcc * kAccCols;  // first TMEM column of the A stages
-  static constexpr int kUsedCols = kACol0 + (kTmemA ? kStages * 2 * BK : 0);
+  static constexpr int kUsedCols = kACol0 + kStagesT * 2 * BK;
   static constexpr int kTmemCols = kUsedCols <= 32 ? 32 : kUsedCols <= 64 ? 64 : kUsedCols <= 128 ? 128
                                    : kUsedCols <= 256 ? 256 : 512;
   static_assert(kUsedCols <= 512, "TMEM overflow");
@@ -113,6 +125,40 @@ __device__ __forceinline__ void tc_mma_ts(uint32_t tmem_d, uint32_t tmem_a, uint
       "tcgen05.mma.cta_group::1.kind::tf32 [%0], [%1], %2, %3, p;\n\t}" ::"r"(tmem_d),
       "r"(tmem_a), "l"(db), "r"(idesc), "r"(accumulate)
       : "memory");
+}
+
+template <int PAIR>
+__device__ __forceinline__ void tc_mma_ts_g(uint32_t tmem_d, uint32_t tmem_a, uint64_t db,
+                                            uint32_t idesc, uint32_t accumulate) {
+  if (PAIR == 1) {
+    tc_mma_ts(tmem_d, tmem_a, db, idesc, accumulate);
+  } else {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::2.kind::tf32 [%0], [%1], %2, %3, p;\n\t}" ::"r"(tmem_d),
+        "r"(tmem_a), "l"(db), "r"(idesc), "r"(accumulate)
+        : "memory");
+  }
+}
+template <int PAIR>
+__device__ __forceinline__ void tc_mma_g(uint32_t tmem_d, uint64_t da, uint64_t db, uint32_t idesc,
+                                         uint32_t accumulate) {
+  if (PAIR == 1) {
+    tc_mma(tmem_d, da, db, idesc, accumulate);
+  } else {
+    asm volatile(
+        "{\n\t.reg .pred p;\n\t"
+        "setp.ne.b32 p, %4, 0;\n\t"
+        "tcgen05.mma.cta_group::2.kind::tf32 [%0], %1, %2, %3, p;\n\t}" ::"r"(tmem_d),
+        "l"(da), "l"(db), "r"(idesc), "r"(accumulate)
+        : "memory");
+  }
+}
+template <int PAIR>
+__device__ __forceinline__ void tc_commit_g(uint64_t* b) {
+  if (PAIR == 1) tc_commit(b);
+  else tc_commit_pair(b);
 }
 
 __device__ __forceinline__ void tmem_st32(uint32_t addr, const float (&v)[32]) {
@@ -160,28 +206,39 @@ __device__ __forceinline__ void load_a_row(const uint8_t* tile, int m, float (&v
 // overlaps the mainloop of tile i + 1.
 // MODE 0: NN/NT (A K-major + converter, B pre-split K-major).
 // MODE 1: TN (A, B MN-major, both split in smem), split-K slabs.
-template <int BN, int MODE, int EW>
+template <int BN, int MODE, int EW, int PAIR, int ASM>
 __global__ void __launch_bounds__(256 + 32 * EW, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const __grid_constant__ CUtensorMap tmBlo, const __grid_constant__ CUtensorMap tmApf,
                const __grid_constant__ CUtensorMap tmC, float* __restrict__ C, int64_t ldc,
                TcShape sh, TcEpi epi) {
-  using CF = Cfg<BN, EW>;
-  constexpr int S = CF::kStages;
+  static_assert(PAIR == 1 || MODE == 0, "CTA pairs: NN / NT only");
+  using CF = Cfg<BN, EW, PAIR, ASM>;
+  constexpr int S = CF::kStages;      // smem ring (raw A + B panels)
+  constexpr int ST = CF::kStagesT;    // TMEM ring of converted A (kTmemA)
+  constexpr int SC = CF::kTmemA ? ST : S;   // ring the converter hands to the MMA
   extern __shared__ uint8_t smem_raw[];
   uint8_t* smem = (uint8_t*)(((uintptr_t)smem_raw + 1023) & ~(uintptr_t)1023);
   uint8_t* stage_base = smem;
   float* epi_smem = (float*)(smem + S * CF::kStageBytes);
   uint64_t* full = (uint64_t*)(smem + S * CF::kStageBytes + CF::kEpiBytes);
-  uint64_t* conv = full + S;
-  uint64_t* empty = conv + S;
+  uint64_t* conv = full + S;     // [SC]
+  uint64_t* empty = conv + SC;
   uint64_t* tfull = empty + S;   // [2]
   uint64_t* tempty = tfull + 2;  // [2]
-  uint32_t* tmem_slot = (uint32_t*)(tempty + 2);
+  uint64_t* aempty = tempty + 2;  // [ST] TMEM A stage consumed by the MMAs
+  uint32_t* tmem_slot = (uint32_t*)(aempty + (ST > 0 ? ST : 1));
 
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int tiles_mn = sh.tiles_m * sh.tiles_n;
   const int total = tiles_mn * sh.splits;
+  // tiles are strided over CTAs (PAIR = 1) or CTA pairs (PAIR = 2: the two
+  // CTAs of a cluster take the same tile, rows rank·128 … of its 256)
+  const uint32_t rank = PAIR == 2 ? cluster_ctarank() : 0u;
+  const int cta0 = PAIR == 2 ? (int)(blockIdx.x >> 1) : (int)blockIdx.x;
+  const int ncta = PAIR == 2 ? (int)(gridDim.x >> 1) : (int)gridDim.x;
+  // pair: the B half of this CTA (rows of the MMA's N) and its size in bytes
+  const int b_rows = PAIR == 2 ? sh.n_mma / 2 : BN;
 
   constexpr int kAB = (CF::kTmemA ? 1 : 2) * CF::kABytes;   // A bytes per stage in smem
   auto A_hi = [&](int s) { return stage_base + s * CF::kStageBytes; };
@@ -198,35 +255,47 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   if (threadIdx.x == 0) {
     for (int s = 0; s < S; ++s) {
       mbar_init(&full[s], 1);
-      mbar_init(&conv[s], 128);
       mbar_init(&empty[s], 1);
     }
+    // pair: one arrival per converter warp of both CTAs, on the leader's barrier
+    for (int s = 0; s < SC; ++s) mbar_init(&conv[s], PAIR == 2 ? 8 : 128);
+    for (int s = 0; s < ST; ++s) mbar_init(&aempty[s], 1);
     for (int b = 0; b < 2; ++b) {
       mbar_init(&tfull[b], 1);
-      mbar_init(&tempty[b], 32 * EW);
+      mbar_init(&tempty[b], PAIR == 2 ? 2 * EW : 32 * EW);
     }
     asm volatile("fence.mbarrier_init.release.cluster;" ::: "memory");
   }
   if (warp == 2) {
-    asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
-                     smem_u32(tmem_slot)),
-                 "n"(CF::kTmemCols));
-    asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    if (PAIR == 2) {
+      asm volatile("tcgen05.alloc.cta_group::2.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                       smem_u32(tmem_slot)),
+                   "n"(CF::kTmemCols));
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::2.sync.aligned;");
+    } else {
+      asm volatile("tcgen05.alloc.cta_group::1.sync.aligned.shared::cta.b32 [%0], %1;" ::"r"(
+                       smem_u32(tmem_slot)),
+                   "n"(CF::kTmemCols));
+      asm volatile("tcgen05.relinquish_alloc_permit.cta_group::1.sync.aligned;");
+    }
   }
   tc_fence_before();
   __syncthreads();
+  if (PAIR == 2) cluster_sync_all();   // both CTAs' barriers initialised before any remote arrival
   tc_fence_after();
   const uint32_t tmem_base = *tmem_slot;
 
   if (warp == 0) {
     if (lane == 0) {
-      const uint32_t bytes = MODE == 0 ? (CF::kABytes + (sh.one ? 1 : 2) * CF::kBBytes) : (CF::kABytes + CF::kBBytes);
+      const uint32_t bbytes = (uint32_t)b_rows * BK * 4;
+      const uint32_t bytes = MODE == 0 ? (CF::kABytes + (sh.one ? 1 : 2) * bbytes) : (CF::kABytes + CF::kBBytes);
       uint32_t kc = 0;
-      for (int t = blockIdx.x; t < total; t += gridDim.x) {
+      for (int t = cta0; t < total; t += ncta) {
         int64_t kbeg;
         const int nkb = tile_kb(t, kbeg);
         const int rem = t % tiles_mn;
-        const int m0 = (rem / sh.tiles_n) * BM, n0 = (rem % sh.tiles_n) * BN;
+        const int m0 = (rem / sh.tiles_n) * (BM * PAIR) + (int)rank * BM;
+        const int n0 = (rem % sh.tiles_n) * BN + (int)rank * b_rows;
         for (int kb = 0; kb < nkb; ++kb, ++kc) {
           const int s = kc % S;
           if (kc >= (uint32_t)S) mbar_wait(&empty[s], ((kc / S) - 1) & 1);
@@ -254,21 +323,27 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       }
     }
   } else if (warp == 1) {
-    if (lane == 0) {
+    if (lane == 0 && rank == 0) {   // pair: the leader CTA issues the pair's MMAs
       // A read from TMEM is K-major by construction (the converter writes rows)
-      const uint32_t idesc = idesc_tf32(sh.n_mma, CF::kTmemA ? 0 : MODE, MODE);
+      const uint32_t idesc = idesc_tf32(sh.n_mma, CF::kTmemA ? 0 : MODE, MODE, BM * PAIR);
       uint32_t kc = 0;
       int it = 0;
-      for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
+      for (int t = cta0; t < total; t += ncta, ++it) {
         int64_t kbeg;
         const int nkb = tile_kb(t, kbeg);
         const int acc = it & 1;
-        if (it >= 2) mbar_wait(&tempty[acc], ((it >> 1) - 1) & 1);
+        if (it >= 2) {
+          if (PAIR == 2) mbar_wait_cluster(&tempty[acc], ((it >> 1) - 1) & 1);
+          else mbar_wait(&tempty[acc], ((it >> 1) - 1) & 1);
+        }
         tc_fence_after();
         const uint32_t d_tmem = tmem_base + acc * (CF::kNAcc * CF::kAccCols);
         for (int kb = 0; kb < nkb; ++kb, ++kc) {
           const int s = kc % S;
-          mbar_wait(&conv[s], (kc / S) & 1);
+          const int st = CF::kTmemA ? (int)(kc % ST) : 0;
+          const int cs = kc % SC;
+          if (PAIR == 2) mbar_wait_cluster(&conv[cs], (kc / SC) & 1);
+          else mbar_wait(&conv[cs], (kc / SC) & 1);
           tc_fence_after();
           const uint32_t bh = smem_u32(B_hi(s)), bl = smem_u32(B_lo(s));
 #pragma unroll
@@ -290,24 +365,24 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
               // 1xTF32: A_tf32 · B_tf32, rotating over the partial accumulators
               const uint32_t d = d_tmem + (uint32_t)((j % CF::kNAcc) * CF::kAccCols);
               if (CF::kTmemA) {
-                tc_mma_ts(d, tmem_base + CF::kACol0 + s * 2 * BK + j * UK, dbh, idesc,
-                          (kb > 0 || j >= CF::kNAcc) ? 1u : 0u);
+                tc_mma_ts_g<PAIR>(d, tmem_base + CF::kACol0 + st * 2 * BK + j * UK, dbh, idesc,
+                                  (kb > 0 || j >= CF::kNAcc) ? 1u : 0u);
               } else {
                 const uint32_t ah = smem_u32(A_hi(s));
-                tc_mma(d, MODE == 0 ? sdesc(ah + j * 32, 16, 1024) : sdesc(ah + j * 1024, 4096, 512, 1), dbh,
-                       idesc, (kb > 0 || j >= CF::kNAcc) ? 1u : 0u);
+                tc_mma_g<PAIR>(d, MODE == 0 ? sdesc(ah + j * 32, 16, 1024) : sdesc(ah + j * 1024, 4096, 512, 1),
+                               dbh, idesc, (kb > 0 || j >= CF::kNAcc) ? 1u : 0u);
               }
             } else if (CF::kTmemA) {
-              // A stage s: hi in columns [kACol0 + 64 s, +32), lo in the next 32.
+              // A stage st: hi in columns [kACol0 + 64 st, +32), lo in the next 32.
               // Narrow tiles rotate over kNAcc independent accumulators so that
               // consecutive MMAs do not serialise on one accumulator.
-              const uint32_t ta = tmem_base + CF::kACol0 + s * 2 * BK + j * UK;
+              const uint32_t ta = tmem_base + CF::kACol0 + st * 2 * BK + j * UK;
               const uint32_t tab[3] = {ta, ta, ta + BK};
 #pragma unroll
               for (int p = 0; p < 3; ++p) {
                 const int i = j * 3 + p;
                 const uint32_t d = d_tmem + (uint32_t)((i % CF::kNAcc) * CF::kAccCols);
-                tc_mma_ts(d, tab[p], p == 1 ? dbl : dbh, idesc, (kb > 0 || i >= CF::kNAcc) ? 1u : 0u);
+                tc_mma_ts_g<PAIR>(d, tab[p], p == 1 ? dbl : dbh, idesc, (kb > 0 || i >= CF::kNAcc) ? 1u : 0u);
               }
             } else {
               const uint32_t ah = smem_u32(A_hi(s)), al = smem_u32(A_lo(s));
@@ -319,24 +394,42 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
                 dah = sdesc(ah + j * 1024, 4096, 512, 1);
                 dal = sdesc(al + j * 1024, 4096, 512, 1);
               }
-              tc_mma(d_tmem, dah, dbh, idesc, acc0);
-              tc_mma(d_tmem, dah, dbl, idesc, 1u);
-              tc_mma(d_tmem, dal, dbh, idesc, 1u);
+              if (CF::kNAcc == 1) {
+                tc_mma_g<PAIR>(d_tmem, dah, dbh, idesc, acc0);
+                tc_mma_g<PAIR>(d_tmem, dah, dbl, idesc, 1u);
+                tc_mma_g<PAIR>(d_tmem, dal, dbh, idesc, 1u);
+              } else {
+                const uint64_t da3[3] = {dah, dah, dal}, db3[3] = {dbh, dbl, dbh};
+#pragma unroll
+                for (int p = 0; p < 3; ++p) {
+                  const int i = j * 3 + p;
+                  const uint32_t d = d_tmem + (uint32_t)((i % CF::kNAcc) * CF::kAccCols);
+                  tc_mma_g<PAIR>(d, da3[p], db3[p], idesc, (kb > 0 || i >= CF::kNAcc) ? 1u : 0u);
+                }
+              }
             }
           }
-          tc_commit(&empty[s]);
+          tc_commit_g<PAIR>(&empty[s]);   // pair: frees the stage in both CTAs
+          if (CF::kTmemA) tc_commit_g<PAIR>(&aempty[st]);
         }
-        tc_commit(&tfull[acc]);   // fires when this tile's MMAs (if any) are done
+        tc_commit_g<PAIR>(&tfull[acc]);   // fires when this tile's MMAs (if any) are done
       }
     }
   } else if (warp >= 4 && warp < 8) {
     const int t128 = threadIdx.x - 128;
+    const uint32_t conv_leader = PAIR == 2 ? mapa_u32(smem_u32(conv), 0) : 0u;
     uint32_t kc = 0;
-    for (int t = blockIdx.x; t < total; t += gridDim.x) {
+    for (int t = cta0; t < total; t += ncta) {
       int64_t kbeg;
       const int nkb = tile_kb(t, kbeg);
       for (int kb = 0; kb < nkb; ++kb, ++kc) {
         const int s = kc % S;
+        const int st = CF::kTmemA ? (int)(kc % ST) : 0;
+        const int cs = kc % SC;
+        if (CF::kTmemA && kc >= (uint32_t)ST) {   // the MMAs have read TMEM stage st
+          mbar_wait(&aempty[st], ((kc / ST) - 1) & 1);
+          tc_fence_after();
+        }
         mbar_wait(&full[s], (kc / S) & 1);
         if (sh.dbg & 1) {
         } else if (sh.one) {
@@ -347,7 +440,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
             load_a_row<MODE>(A_hi(s), t128, v);
 #pragma unroll
             for (int i = 0; i < 32; ++i) v[i] = tf32_rn(v[i]);
-            tmem_st32(tmem_base + ((uint32_t)((warp & 3) * 32) << 16) + CF::kACol0 + s * 2 * BK, v);
+            tmem_st32(tmem_base + ((uint32_t)((warp & 3) * 32) << 16) + CF::kACol0 + st * 2 * BK, v);
             asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
           }
         } else if (CF::kTmemA) {
@@ -359,7 +452,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
             h[i] = tf32_rn(v[i]);
             v[i] = tf32_rn(v[i] - h[i]);
           }
-          const uint32_t ta = tmem_base + ((uint32_t)((warp & 3) * 32) << 16) + CF::kACol0 + s * 2 * BK;
+          const uint32_t ta = tmem_base + ((uint32_t)((warp & 3) * 32) << 16) + CF::kACol0 + st * 2 * BK;
           tmem_st32(ta, h);
           tmem_st32(ta + BK, v);
           asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
@@ -369,19 +462,28 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         if (MODE == 1 && !sh.one) split_inplace((float4*)B_hi(s), (float4*)B_lo(s), CF::kBBytes / 16, t128, 128);
         fence_proxy_async();
         tc_fence_before();
-        mbar_arrive(&conv[s]);
+        if (PAIR == 2) {
+          // this CTA's A half (TMEM / smem) and B half (landed: full[s]) are
+          // ready: one release arrival per warp on the leader's barrier
+          __syncwarp();
+          if (lane == 0) mbar_arrive_cluster(conv_leader + (uint32_t)(cs * sizeof(uint64_t)));
+        } else {
+          mbar_arrive(&conv[cs]);
+        }
       }
     }
   } else if (warp >= 8) {
     const int q = warp & 3;                    // TMEM lane quadrant of this warp
     const int half = (warp - 8) >> 2;          // column half (chunks 32 apart)
     float* tb = epi_smem + (warp - 8) * 1280;   // 32 x 33 transpose tile / 32 x 32 TMA box
+    const uint32_t tempty_leader = PAIR == 2 ? mapa_u32(smem_u32(tempty), 0) : 0u;
     int it = 0;
-    for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
+    for (int t = cta0; t < total; t += ncta, ++it) {
       int64_t kbeg;
       const int nkb = tile_kb(t, kbeg);
       const int z = t / tiles_mn, rem = t % tiles_mn;
-      const int64_t m0 = (int64_t)(rem / sh.tiles_n) * BM, n0 = (int64_t)(rem % sh.tiles_n) * BN;
+      const int64_t m0 = (int64_t)(rem / sh.tiles_n) * (BM * PAIR) + (int64_t)rank * BM;
+      const int64_t n0 = (int64_t)(rem % sh.tiles_n) * BN;
       const int acc = it & 1;
       mbar_wait_sleep(&tfull[acc], (it >> 1) & 1);
       tc_fence_after();
@@ -512,13 +614,23 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         __syncwarp();
       }
       tc_fence_before();
-      mbar_arrive(&tempty[acc]);
+      if (PAIR == 2) {
+        __syncwarp();
+        if (lane == 0) mbar_arrive_cluster(tempty_leader + (uint32_t)(acc * sizeof(uint64_t)));
+      } else {
+        mbar_arrive(&tempty[acc]);
+      }
     }
     if (sh.tstore && lane == 0) bulk_wait0();   // every TMA store of this warp has landed
   }
   tc_fence_before();
   __syncthreads();
-  if (warp == 2) {
+  if (PAIR == 2) {
+    cluster_sync_all();   // the peer's MMAs (reading this CTA's smem / TMEM) are done
+    if (warp == 2)
+      asm volatile("tcgen05.dealloc.cta_group::2.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
+                   "n"(CF::kTmemCols));
+  } else if (warp == 2) {
     asm volatile("tcgen05.dealloc.cta_group::1.sync.aligned.b32 %0, %1;" ::"r"(tmem_base),
                  "n"(CF::kTmemCols));
   }
@@ -593,19 +705,19 @@ CUtensorMap make_map(const float* base, int64_t inner, int64_t outer, int64_t ld
   return m;
 }
 
-template <int BN, int MODE, int EW>
+template <int BN, int MODE, int EW, int PAIR, int ASM>
 void launch_tc_ew(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& blo,
                float* C, int64_t ldc, int64_t M, int64_t N, int64_t K, int splits, int n_mma,
                const TcEpi& e, const CUtensorMap* apf = nullptr) {
-  using CF = Cfg<BN, EW>;
-  RDM_CUDA(cudaFuncSetAttribute(gemm_tc_kernel<BN, MODE, EW>, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                CF::kSmem));
+  using CF = Cfg<BN, EW, PAIR, ASM>;
+  auto kern = gemm_tc_kernel<BN, MODE, EW, PAIR, ASM>;
+  RDM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, CF::kSmem));
   TcShape sh;
   sh.M = M;
   sh.N = N;
   sh.K = K;
   sh.k_per_split = ceil_div(ceil_div(K, splits), BK) * BK;
-  sh.tiles_m = (int)ceil_div(M, BM);
+  sh.tiles_m = (int)ceil_div(M, BM * PAIR);
   sh.tiles_n = (int)ceil_div(N, BN);
   sh.splits = splits;
   sh.n_mma = n_mma;
@@ -621,21 +733,74 @@ void launch_tc_ew(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, cons
                   ? 1 : 0;
   const CUtensorMap tc = sh.tstore ? make_map(C, N, M, ldc, 32, 32) : a;
   const int64_t total = (int64_t)sh.tiles_m * sh.tiles_n * splits;
-  const unsigned grid = (unsigned)std::min<int64_t>(total, ctx->num_sms);
-  gemm_tc_kernel<BN, MODE, EW><<<grid, CF::kThreads, CF::kSmem, ctx->stream>>>(a, b, blo, apf ? *apf : a, tc, C,
-                                                                  ldc, sh, e);
+  if (PAIR == 1) {
+    const unsigned grid = (unsigned)std::min<int64_t>(total, ctx->num_sms);
+    kern<<<grid, CF::kThreads, CF::kSmem, ctx->stream>>>(a, b, blo, apf ? *apf : a, tc, C, ldc, sh, e);
+  } else {
+    // clusters of 2 CTAs (one CTA pair per TPC); the persistent grid is the
+    // number of pairs that are co-resident (a GPC with an odd number of free
+    // SMs leaves one idle: a grid of num_sms / 2 pairs would run a second wave)
+    cudaLaunchConfig_t cfg{};
+    cfg.blockDim = dim3(CF::kThreads);
+    cfg.dynamicSmemBytes = CF::kSmem;
+    cfg.stream = ctx->stream;
+    cudaLaunchAttribute attr[1];
+    attr[0].id = cudaLaunchAttributeClusterDimension;
+    attr[0].val.clusterDim.x = 2;
+    attr[0].val.clusterDim.y = 1;
+    attr[0].val.clusterDim.z = 1;
+    cfg.attrs = attr;
+    cfg.numAttrs = 1;
+    static int max_pairs = 0;   // per instantiation
+    if (max_pairs == 0) {
+      cfg.gridDim = dim3((unsigned)ctx->num_sms);
+      int n = 0;
+      RDM_CUDA(cudaOccupancyMaxActiveClusters(&n, kern, &cfg));
+      max_pairs = std::max(1, std::min(n, ctx->num_sms / 2));
+      if (getenv("RDM_PAIR_LOG")) fprintf(stderr, "rdm: gemm pair BN=%d EW=%d: %d co-resident pairs\n", BN, EW, n);
+    }
+    cfg.gridDim = dim3((unsigned)(2 * std::min<int64_t>(total, max_pairs)));
+    const CUtensorMap apm = apf ? *apf : a;
+    RDM_CUDA(cudaLaunchKernelEx(&cfg, kern, a, b, blo, apm, tc, C, ldc, sh, e));
+  }
   RDM_LAUNCHED(ctx);
 }
 
-template <int BN, int MODE>
+template <int BN, int MODE, int PAIR = 1, int ASM = 0>
 void launch_tc(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& blo,
                float* C, int64_t ldc, int64_t M, int64_t N, int64_t K, int splits, int n_mma,
                const TcEpi& e, const CUtensorMap* apf = nullptr) {
   // short contractions produce a wide output per k-block: epilogue-bound
   if (BN <= 128 && K <= 256)
-    launch_tc_ew<BN, MODE, 8>(ctx, a, b, blo, C, ldc, M, N, K, splits, n_mma, e, apf);
+    launch_tc_ew<BN, MODE, 8, PAIR, ASM>(ctx, a, b, blo, C, ldc, M, N, K, splits, n_mma, e, apf);
   else
-    launch_tc_ew<BN, MODE, 4>(ctx, a, b, blo, C, ldc, M, N, K, splits, n_mma, e, apf);
+    launch_tc_ew<BN, MODE, 4, PAIR, ASM>(ctx, a, b, blo, C, ldc, M, N, K, splits, n_mma, e, apf);
+}
+
+// CTA pairs for the row-sliced NN / NT products: every SM loads half of the W
+// panel per row it computes (the 602-wide contractions are bound by each SM's
+// ingress of A plus the re-read W panel).  Off for narrow outputs (BN < 32:
+// the pair's N must be a multiple of 32) and for grids that would not fill the
+// GPU's pairs.  RDM_PAIR=0 / 1 forces either (experiments).
+// Measured per call (tools/time_gemm.py, profiles/r2_gemm_pair.md): BN = 256
+// pairs (A in smem) 1.61 → 1.32 ms for the products-shaped 2.45 M x 256 · 256
+// x 256; BN ≤ 128 with A in TMEM gains where K is short and N ≤ 256 (K = 100,
+// N = 256: 1.10 → 1.02 ms), with A split in smem and two partial accumulators
+// where K is long or the tile narrow (K = 602: 229 → 208 µs; N = 41: 68 → 52
+// µs); the 602-wide NT (K = 128, five 128-wide tiles) stays single.
+// Returns 0 (single CTA), 1 (pair, A in TMEM / smem for BN = 256), 2 (pair, A
+// split in smem, BN ≤ 128).
+int use_pair(rdm_ctx* ctx, int64_t M, int64_t N, int64_t K, int BN, int splits) {
+  if (BN < 32 || splits > 1) return 0;
+  const char* fp = getenv("RDM_PAIR");
+  const char* fa = getenv("RDM_PAIR_ASMEM");
+  if (fp && !atoi(fp)) return 0;
+  if (!fp && M < (int64_t)ctx->num_sms * BM) return 0;
+  if (BN == 256) return 1;
+  if (fa) return atoi(fa) ? 2 : 1;
+  if (K >= 256 || BN <= 64) return 2;
+  if (N <= 256 || fp) return 1;
+  return 0;
 }
 
 // Wider N: one 256-wide tile (A in smem, both TMEM accumulators) where the
@@ -664,11 +829,14 @@ void launch_nn_panels(rdm_ctx* ctx, const float* X, int64_t ldx, const float* bh
   // the GraphSAINT subgraphs ran slower with them)
   const int BN = (splits == 1 && wide_ok) ? pick_bn(N, K, ctx->prec != RDM_PREC_FAST, (e.flags & RDM_EPI_MASK) != 0)
                                          : pick_bn(N, 0, false);
-  // one MMA width for every tile: BN when N spans several tiles, else N rounded to 16
-  const int nm = N > BN ? BN : (int)(((N + 15) / 16) * 16);
+  const int pmode = use_pair(ctx, M, N, K, BN, splits);
+  const bool pair = pmode != 0;
+  // one MMA width for every tile: BN when N spans several tiles, else N rounded
+  // to 16 (to 32 for a pair, whose CTAs load nm/2 rows of B each)
+  const int nm = N > BN ? BN : pair ? (int)(((N + 31) / 32) * 32) : (int)(((N + 15) / 16) * 16);
   const CUtensorMap ta = make_map(X, K, M, ldx, BK, BM);
-  const CUtensorMap tb = make_map(bhi, K, N, ldb, BK, BN);
-  const CUtensorMap tbl = make_map(blo, K, N, ldb, BK, BN);
+  const CUtensorMap tb = make_map(bhi, K, N, ldb, BK, pair ? nm / 2 : BN);
+  const CUtensorMap tbl = make_map(blo, K, N, ldb, BK, pair ? nm / 2 : BN);
   // L2-prefetch map: 128 x 128 fp32 boxes (512-byte row segments), no swizzle
   // (off by default: measured at the end of round 1, tools/time_gemm.py, the
   // 232,965 x 602 · 602 x 128 NN runs 231 → 225 µs fp32 and 175 → 150 µs fast
@@ -676,6 +844,22 @@ void launch_nn_panels(rdm_ctx* ctx, const float* X, int64_t ldx, const float* bh
   const bool pf = K > 4 * BK && getenv("RDM_PF") && atoi(getenv("RDM_PF"));
   const CUtensorMap tpf = pf ? make_map(X, K, M, ldx, 4 * BK, BM, CU_TENSOR_MAP_SWIZZLE_NONE) : ta;
   const CUtensorMap* p = pf ? &tpf : nullptr;
+  if (pmode == 2) {
+    switch (BN) {
+      case 64: launch_tc<64, 0, 2, 1>(ctx, ta, tb, tbl, C, ldc, M, N, K, splits, nm, e, p); return;
+      case 128: launch_tc<128, 0, 2, 1>(ctx, ta, tb, tbl, C, ldc, M, N, K, splits, nm, e, p); return;
+      default: break;
+    }
+  }
+  if (pair) {
+    switch (BN) {
+      case 32: launch_tc<32, 0, 2>(ctx, ta, tb, tbl, C, ldc, M, N, K, splits, nm, e, p); break;
+      case 64: launch_tc<64, 0, 2>(ctx, ta, tb, tbl, C, ldc, M, N, K, splits, nm, e, p); break;
+      case 128: launch_tc<128, 0, 2>(ctx, ta, tb, tbl, C, ldc, M, N, K, splits, nm, e, p); break;
+      default: launch_tc<256, 0, 2>(ctx, ta, tb, tbl, C, ldc, M, N, K, splits, nm, e, p); break;
+    }
+    return;
+  }
   switch (BN) {
     case 16: launch_tc<16, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, splits, nm, e, p); break;
     case 32: launch_tc<32, 0>(ctx, ta, tb, tbl, C, ldc, M, N, K, splits, nm, e, p); break;
