@@ -29,7 +29,7 @@ ROOT = os.path.dirname(os.path.abspath(__file__))
 sys.path.insert(0, ROOT)
 
 METRIC = "full-batch GCN epoch ms at 1/2/4/8 B200; SpMM HBM GB/s; all-to-all bus GB/s"
-DTYPES = {"fp32": "f32", "fast": "bf16 SpMM operand + tf32 GEMM, f32 accumulate"}
+DTYPES = {"fp32": "f32", "fast": "bf16 SpMM operand + bf16 (kind::f16) NN/NT GEMM, tf32 TN, f32 accumulate"}
 GATES = {"fp32": 1e-4, "fast": 2e-2}
 
 
@@ -764,13 +764,20 @@ def main():
     torch.cuda.synchronize(dev)
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
+    marks = [torch.cuda.Event(enable_timing=True) for _ in range(a.steps)]
     e0.record(stream)
-    for _ in range(a.steps):
+    for i in range(a.steps):
         epoch()
+        marks[i].record(stream)   # per-epoch mark (mean, median, p95)
     e1.record(stream)
     torch.cuda.synchronize(dev)
     clocks = clk.stop()
     ms_total = e0.elapsed_time(e1)
+    ep_ms = [e0.elapsed_time(marks[0])] + [marks[i - 1].elapsed_time(marks[i]) for i in range(1, a.steps)]
+    if world > 1:
+        t = torch.tensor(ep_ms, device=dev)
+        dist.all_reduce(t, op=dist.ReduceOp.MAX)
+        ep_ms = t.tolist()
     cnt = ctx.counters()
     ph_ms, ph_launch = ctx.phase_times()
     ctx.set_timing(False)
@@ -891,6 +898,10 @@ def main():
             "clocks": clocks, "e2e": e2e, "gpu_launches": cnt["kernel_launches"],
             "roofline": roofline, "cpu_baseline": cpu,
             "phases_ms_per_step": {k: v / a.steps for k, v in ph_ms.items()},
+            "step_ms": {"mean": float(np.mean(ep_ms)), "median": float(np.median(ep_ms)),
+                        "p95": float(np.percentile(ep_ms, 95)), "min": float(np.min(ep_ms)),
+                        "max": float(np.max(ep_ms)),
+                        "note": "per-epoch CUDA-event intervals on the library stream, max over ranks"},
             "spmm_hbm_gbs": achieved, "a2a_bus_gbs": a2a_bus,
             "a2a_bytes_per_step": cnt["a2a_bytes_wire"] / a.steps,
             "bcast_elems_per_step": cnt["bcast_elems"] / a.steps,

@@ -230,8 +230,10 @@ int rdm_get_transport(const rdm_ctx* ctx);
  *     (round-to-nearest-even) once per call and gathers the bf16 rows
  *     (half the L2/HBM gather bytes), accumulating in fp32; the binary hub
  *     tiles multiply one bf16 piece of s⊙X (fp32: two column-scaled fp16 or three bf16 pieces); every rdm_gemm
- *     (NN / NT / TN) issues one tf32 MMA per k step instead of 3xTF32 (the
- *     tensor core reads fp32 operands as tf32).  Inside rdm_gcn_forward /
+ *     NN / NT runs on kind::f16 with bf16 operands (X rounded to nearest even
+ *     as it is staged, W as bf16 panels; fp32 accumulation; RDM_F16_GEMM=0
+ *     keeps one tf32 MMA per k step), TN issues one tf32 MMA per k step
+ *     instead of 3xTF32.  Inside rdm_gcn_forward /
  *     backward the row → column redistributions (whose destination is an
  *     SpMM input, rounded to bf16 by the variant anyway) carry bf16 on the
  *     wire (half their bytes; each moved value, the rank's own block included,

@@ -88,14 +88,18 @@ struct TcShape {
 // ASM = 1 (pairs, BN <= 128): A split in shared memory instead of TMEM, which
 // leaves TMEM to two partial accumulators per buffer (the three MMAs of a k
 // step alternate between them instead of serialising on one).
-template <int BN, int EW, int PAIR = 1, int ASM = 0>
+// F16 = 1 (fast variant, A in TMEM): kind::f16 MMAs on bf16 operands — A
+// rounded to bf16 pairs by the converter (16 TMEM columns per 32-wide k-block),
+// W as bf16 K-major panels with the 64-byte swizzle (64 B per row per k-block).
+template <int BN, int EW, int PAIR = 1, int ASM = 0, int F16 = 0>
 struct Cfg {
   static constexpr int kThreads = 256 + 32 * EW;
   static constexpr int kAccCols = BN <= 32 ? 32 : BN <= 64 ? 64 : BN <= 128 ? 128 : 256;
   static constexpr bool kTmemA = BN <= 128 && !ASM;
-  static constexpr int kNAcc = !kTmemA ? (BN <= 128 ? 2 : 1) : BN <= 32 ? 4 : BN <= 64 ? 2 : 1;  // partial accumulators
+  // partial accumulators (the bf16 path issues 2 MMAs per k-block: at most 2)
+  static constexpr int kNAcc = !kTmemA ? (BN <= 128 ? 2 : 1) : BN <= 32 ? (F16 ? 2 : 4) : BN <= 64 ? 2 : 1;
   static constexpr int kABytes = BM * BK * 4;   // 16 KB
-  static constexpr int kBBytes = (BN / PAIR) * BK * 4;
+  static constexpr int kBBytes = (BN / PAIR) * BK * (F16 ? 2 : 4);
   static constexpr int kStageBytes = (kTmemA ? 1 : 2) * kABytes + 2 * kBBytes;
   // per epilogue warp 5 KB (1024-aligned): a 32 x 33 transpose tile, or the
   // 32 x 32 swizzled box of a TMA store
@@ -104,14 +108,15 @@ struct Cfg {
   // deep rings hide TMA latency.  With A in TMEM the converted A stages form
   // a second ring (64 TMEM columns each, whatever the accumulators leave),
   // decoupled from the smem ring of raw A + B tiles, which can run deeper.
-  static constexpr int kStagesT0 = kTmemA ? (512 - 2 * kNAcc * kAccCols) / (2 * BK) : 0;
+  static constexpr int kAStride = F16 ? BK / 2 : 2 * BK;   // TMEM columns per A stage
+  static constexpr int kStagesT0 = kTmemA ? (512 - 2 * kNAcc * kAccCols) / kAStride : 0;
   static constexpr int kStagesT = kStagesT0 < 8 ? kStagesT0 : 8;
   static constexpr int kMaxStages = kTmemA ? 8 : 4;
   static constexpr int kFitStages = kBudget / kStageBytes < 8 ? kBudget / kStageBytes : 8;
   static constexpr int kStages = kFitStages < kMaxStages ? kFitStages : kMaxStages;
   static constexpr int kSmem = kStages * kStageBytes + kEpiBytes + 1024 /*align*/ + 512 /*barriers*/;
   static constexpr int kACol0 = 2 * kNAcc * kAccCols;  // first TMEM column of the A stages
-  static constexpr int kUsedCols = kACol0 + kStagesT * 2 * BK;
+  static constexpr int kUsedCols = kACol0 + kStagesT * kAStride;
   static constexpr int kTmemCols = kUsedCols <= 32 ? 32 : kUsedCols <= 64 ? 64 : kUsedCols <= 128 ? 128
                                    : kUsedCols <= 256 ? 256 : 512;
   static_assert(kUsedCols <= 512, "TMEM overflow");
@@ -155,6 +160,29 @@ __device__ __forceinline__ void tc_mma_g(uint32_t tmem_d, uint64_t da, uint64_t 
         : "memory");
   }
 }
+// kind::f16 (bf16) MMA with A from TMEM (bf16 pairs packed in 32-bit columns)
+__device__ __forceinline__ void tc_mma_bf16_ts(uint32_t tmem_d, uint32_t tmem_a, uint64_t db, uint32_t idesc,
+                                               uint32_t accumulate) {
+  asm volatile(
+      "{\n\t.reg .pred p;\n\t"
+      "setp.ne.b32 p, %4, 0;\n\t"
+      "tcgen05.mma.cta_group::1.kind::f16 [%0], [%1], %2, %3, p;\n\t}" ::"r"(tmem_d),
+      "r"(tmem_a), "l"(db), "r"(idesc), "r"(accumulate)
+      : "memory");
+}
+// kind::f16 instruction descriptor: D f32, A/B bf16, both K-major, M = 128, N.
+__host__ __device__ constexpr uint32_t idesc_bf16k(int N) {
+  return (1u << 4) | (1u << 7) | (1u << 10) | ((uint32_t)(N >> 3) << 17) | ((uint32_t)(BM >> 4) << 24);
+}
+__device__ __forceinline__ void tmem_st16u(uint32_t addr, const uint32_t (&v)[16]) {
+  asm volatile(
+      "tcgen05.st.sync.aligned.32x32b.x16.b32 [%0], {%1,%2,%3,%4,%5,%6,%7,%8,%9,%10,%11,%12,%13,%14,%15,%16};" ::"r"(
+          addr),
+      "r"(v[0]), "r"(v[1]), "r"(v[2]), "r"(v[3]), "r"(v[4]), "r"(v[5]), "r"(v[6]), "r"(v[7]), "r"(v[8]),
+      "r"(v[9]), "r"(v[10]), "r"(v[11]), "r"(v[12]), "r"(v[13]), "r"(v[14]), "r"(v[15])
+      : "memory");
+}
+
 template <int PAIR>
 __device__ __forceinline__ void tc_commit_g(uint64_t* b) {
   if (PAIR == 1) tc_commit(b);
@@ -206,14 +234,15 @@ __device__ __forceinline__ void load_a_row(const uint8_t* tile, int m, float (&v
 // overlaps the mainloop of tile i + 1.
 // MODE 0: NN/NT (A K-major + converter, B pre-split K-major).
 // MODE 1: TN (A, B MN-major, both split in smem), split-K slabs.
-template <int BN, int MODE, int EW, int PAIR, int ASM>
+template <int BN, int MODE, int EW, int PAIR, int ASM, int F16>
 __global__ void __launch_bounds__(256 + 32 * EW, 1)
 gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ CUtensorMap tmB,
                const __grid_constant__ CUtensorMap tmBlo, const __grid_constant__ CUtensorMap tmApf,
                const __grid_constant__ CUtensorMap tmC, float* __restrict__ C, int64_t ldc,
                TcShape sh, TcEpi epi) {
   static_assert(PAIR == 1 || MODE == 0, "CTA pairs: NN / NT only");
-  using CF = Cfg<BN, EW, PAIR, ASM>;
+  static_assert(!F16 || (MODE == 0 && PAIR == 1 && BN <= 128 && !ASM), "bf16 GEMM: NN / NT, A in TMEM");
+  using CF = Cfg<BN, EW, PAIR, ASM, F16>;
   constexpr int S = CF::kStages;      // smem ring (raw A + B panels)
   constexpr int ST = CF::kStagesT;    // TMEM ring of converted A (kTmemA)
   constexpr int SC = CF::kTmemA ? ST : S;   // ring the converter hands to the MMA
@@ -287,7 +316,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
 
   if (warp == 0) {
     if (lane == 0) {
-      const uint32_t bbytes = (uint32_t)b_rows * BK * 4;
+      const uint32_t bbytes = (uint32_t)b_rows * BK * (F16 ? 2 : 4);
       const uint32_t bytes = MODE == 0 ? (CF::kABytes + (sh.one ? 1 : 2) * bbytes) : (CF::kABytes + CF::kBBytes);
       uint32_t kc = 0;
       for (int t = cta0; t < total; t += ncta) {
@@ -325,7 +354,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   } else if (warp == 1) {
     if (lane == 0 && rank == 0) {   // pair: the leader CTA issues the pair's MMAs
       // A read from TMEM is K-major by construction (the converter writes rows)
-      const uint32_t idesc = idesc_tf32(sh.n_mma, CF::kTmemA ? 0 : MODE, MODE, BM * PAIR);
+      const uint32_t idesc = F16 ? idesc_bf16k(sh.n_mma) : idesc_tf32(sh.n_mma, CF::kTmemA ? 0 : MODE, MODE, BM * PAIR);
       uint32_t kc = 0;
       int it = 0;
       for (int t = cta0; t < total; t += ncta, ++it) {
@@ -346,8 +375,19 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           else mbar_wait(&conv[cs], (kc / SC) & 1);
           tc_fence_after();
           const uint32_t bh = smem_u32(B_hi(s)), bl = smem_u32(B_lo(s));
+          if (F16) {
+            // two K = 16 steps per 32-wide k-block: 8 packed A columns and 32 B
+            // of each 64-byte-swizzled B row per step
 #pragma unroll
-          for (int j = 0; j < BK / UK; ++j) {
+            for (int j = 0; j < 2; ++j) {
+              const uint32_t d = d_tmem + (uint32_t)((j % CF::kNAcc) * CF::kAccCols);
+              if (!(sh.dbg & 2))
+                tc_mma_bf16_ts(d, tmem_base + CF::kACol0 + st * CF::kAStride + j * 8, sdesc(bh + j * 32, 16, 512, 4),
+                               idesc, (kb > 0 || j >= CF::kNAcc) ? 1u : 0u);
+            }
+          }
+#pragma unroll
+          for (int j = 0; j < (F16 ? 0 : BK / UK); ++j) {
             uint64_t dbh, dbl;
             if (MODE == 0) {  // K-major: advance 32 B along the swizzled row
               dbh = sdesc(bh + j * 32, 16, 1024);
@@ -365,7 +405,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
               // 1xTF32: A_tf32 · B_tf32, rotating over the partial accumulators
               const uint32_t d = d_tmem + (uint32_t)((j % CF::kNAcc) * CF::kAccCols);
               if (CF::kTmemA) {
-                tc_mma_ts_g<PAIR>(d, tmem_base + CF::kACol0 + st * 2 * BK + j * UK, dbh, idesc,
+                tc_mma_ts_g<PAIR>(d, tmem_base + CF::kACol0 + st * CF::kAStride + j * UK, dbh, idesc,
                                   (kb > 0 || j >= CF::kNAcc) ? 1u : 0u);
               } else {
                 const uint32_t ah = smem_u32(A_hi(s));
@@ -376,7 +416,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
               // A stage st: hi in columns [kACol0 + 64 st, +32), lo in the next 32.
               // Narrow tiles rotate over kNAcc independent accumulators so that
               // consecutive MMAs do not serialise on one accumulator.
-              const uint32_t ta = tmem_base + CF::kACol0 + st * 2 * BK + j * UK;
+              const uint32_t ta = tmem_base + CF::kACol0 + st * CF::kAStride + j * UK;
               const uint32_t tab[3] = {ta, ta, ta + BK};
 #pragma unroll
               for (int p = 0; p < 3; ++p) {
@@ -435,12 +475,24 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         } else if (sh.one) {
           // 1xTF32: A rounded to tf32 into TMEM; smem operands are read as tf32
           // by the tensor core as they are (low mantissa bits ignored)
-          if (CF::kTmemA) {
+          if (CF::kTmemA && F16) {
+            // bf16 pairs (lower k in the low half), round to nearest even
+            float v[32];
+            load_a_row<MODE>(A_hi(s), t128, v);
+            uint32_t pk[16];
+#pragma unroll
+            for (int i = 0; i < 16; ++i) {
+              __nv_bfloat162 pr = __floats2bfloat162_rn(v[2 * i], v[2 * i + 1]);
+              pk[i] = *reinterpret_cast<uint32_t*>(&pr);
+            }
+            tmem_st16u(tmem_base + ((uint32_t)((warp & 3) * 32) << 16) + CF::kACol0 + st * CF::kAStride, pk);
+            asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+          } else if (CF::kTmemA) {
             float v[32];
             load_a_row<MODE>(A_hi(s), t128, v);
 #pragma unroll
             for (int i = 0; i < 32; ++i) v[i] = tf32_rn(v[i]);
-            tmem_st32(tmem_base + ((uint32_t)((warp & 3) * 32) << 16) + CF::kACol0 + st * 2 * BK, v);
+            tmem_st32(tmem_base + ((uint32_t)((warp & 3) * 32) << 16) + CF::kACol0 + st * CF::kAStride, v);
             asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
           }
         } else if (CF::kTmemA) {
@@ -452,7 +504,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
             h[i] = tf32_rn(v[i]);
             v[i] = tf32_rn(v[i] - h[i]);
           }
-          const uint32_t ta = tmem_base + ((uint32_t)((warp & 3) * 32) << 16) + CF::kACol0 + st * 2 * BK;
+          const uint32_t ta = tmem_base + ((uint32_t)((warp & 3) * 32) << 16) + CF::kACol0 + st * CF::kAStride;
           tmem_st32(ta, h);
           tmem_st32(ta + BK, v);
           asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
@@ -654,6 +706,20 @@ __global__ void prep_b_kernel(const float* __restrict__ W, int64_t ldw, int64_t 
   }
 }
 
+// bf16 B panels for the fast variant's kind::f16 GEMM: Bt[n][kk] (K-major, row
+// length ldb, columns [K, ldb) zero), rounded to nearest even.
+__global__ void prep_b_bf16_kernel(const float* __restrict__ W, int64_t ldw, int64_t K, int64_t N, int transpose,
+                                   __nv_bfloat16* __restrict__ bt, int64_t ldb) {
+  const int64_t total = N * ldb;
+  for (int64_t i = (int64_t)blockIdx.x * blockDim.x + threadIdx.x; i < total;
+       i += (int64_t)gridDim.x * blockDim.x) {
+    const int64_t n = i / ldb, kk = i % ldb;
+    float x = 0.f;
+    if (kk < K) x = transpose ? W[kk * ldw + n] : W[n * ldw + kk];
+    bt[i] = __float2bfloat16_rn(x);
+  }
+}
+
 __global__ void splitk_sum(const float* __restrict__ part, int splits, int64_t M, int64_t N,
                            int64_t ldp, float* __restrict__ C, int64_t ldc) {
   const int64_t idx = (int64_t)blockIdx.x * blockDim.x + threadIdx.x;
@@ -705,12 +771,12 @@ CUtensorMap make_map(const float* base, int64_t inner, int64_t outer, int64_t ld
   return m;
 }
 
-template <int BN, int MODE, int EW, int PAIR, int ASM>
+template <int BN, int MODE, int EW, int PAIR, int ASM, int F16 = 0>
 void launch_tc_ew(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, const CUtensorMap& blo,
                float* C, int64_t ldc, int64_t M, int64_t N, int64_t K, int splits, int n_mma,
                const TcEpi& e, const CUtensorMap* apf = nullptr) {
-  using CF = Cfg<BN, EW, PAIR, ASM>;
-  auto kern = gemm_tc_kernel<BN, MODE, EW, PAIR, ASM>;
+  using CF = Cfg<BN, EW, PAIR, ASM, F16>;
+  auto kern = gemm_tc_kernel<BN, MODE, EW, PAIR, ASM, F16>;
   RDM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, CF::kSmem));
   TcShape sh;
   sh.M = M;
@@ -764,6 +830,23 @@ void launch_tc_ew(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, cons
     RDM_CUDA(cudaLaunchKernelEx(&cfg, kern, a, b, blo, apm, tc, C, ldc, sh, e));
   }
   RDM_LAUNCHED(ctx);
+}
+
+// 2-D bf16 tensor map with the 64-byte swizzle (the fast GEMM's B panels: one
+// 32-wide k-block is 64 bytes per row)
+CUtensorMap make_map_bf16(const __nv_bfloat16* base, int64_t inner, int64_t outer, int64_t ld, int box_inner,
+                          int box_outer) {
+  CUtensorMap m;
+  cuuint64_t dims[2] = {(cuuint64_t)inner, (cuuint64_t)outer};
+  cuuint64_t strides[1] = {(cuuint64_t)(ld * 2)};
+  cuuint32_t box[2] = {(cuuint32_t)box_inner, (cuuint32_t)box_outer};
+  cuuint32_t es[2] = {1, 1};
+  CUresult r = encode_fn()(&m, CU_TENSOR_MAP_DATA_TYPE_BFLOAT16, 2, (void*)base, dims, strides, box, es,
+                           CU_TENSOR_MAP_INTERLEAVE_NONE, CU_TENSOR_MAP_SWIZZLE_64B,
+                           CU_TENSOR_MAP_L2_PROMOTION_L2_256B, CU_TENSOR_MAP_FLOAT_OOB_FILL_NONE);
+  if (r != CUDA_SUCCESS)
+    throw Error(RDM_ERR_CUDA, "cuTensorMapEncodeTiled (bf16) failed (" + std::to_string((int)r) + ")");
+  return m;
 }
 
 template <int BN, int MODE, int PAIR = 1, int ASM = 0>
@@ -822,6 +905,35 @@ int pick_bn(int64_t N, int64_t K = 0, bool three = true, bool mask = false) {
 }  // namespace
 
 namespace {
+// Fast variant, NN / NT: bf16 operands on kind::f16 (twice the tf32 MMA rate,
+// half the W panel bytes); A stays fp32 in HBM and is rounded by the converter.
+// RDM_F16_GEMM=0 keeps the 1xTF32 kernel (experiments).
+bool use_f16_gemm(rdm_ctx* ctx) {
+  if (ctx->prec != RDM_PREC_FAST) return false;
+  const char* e = getenv("RDM_F16_GEMM");
+  return !e || atoi(e) != 0;
+}
+
+void launch_nn_bf16(rdm_ctx* ctx, const float* X, int64_t ldx, const __nv_bfloat16* bt, int64_t ldb, float* C,
+                    int64_t ldc, int64_t M, int64_t N, int64_t K, const TcEpi& e) {
+  const int BN = pick_bn(N, 0, false);
+  const int nm = N > BN ? BN : (int)(((N + 15) / 16) * 16);
+  const CUtensorMap ta = make_map(X, K, M, ldx, BK, BM);
+  const CUtensorMap tb = make_map_bf16(bt, K, N, ldb, BK, BN);
+  switch (BN) {
+#define RDM_F16_CASE(B)                                                                        \
+  case B:                                                                                      \
+    if (K <= 256) launch_tc_ew<B, 0, 8, 1, 0, 1>(ctx, ta, tb, tb, C, ldc, M, N, K, 1, nm, e); \
+    else launch_tc_ew<B, 0, 4, 1, 0, 1>(ctx, ta, tb, tb, C, ldc, M, N, K, 1, nm, e);          \
+    break;
+    RDM_F16_CASE(16)
+    RDM_F16_CASE(32)
+    RDM_F16_CASE(64)
+    default: RDM_F16_CASE(128)
+#undef RDM_F16_CASE
+  }
+}
+
 void launch_nn_panels(rdm_ctx* ctx, const float* X, int64_t ldx, const float* bhi, const float* blo,
                       int64_t ldb, float* C, int64_t ldc, int64_t M, int64_t N, int64_t K,
                       const TcEpi& e, int splits = 1, bool wide_ok = true) {
@@ -927,6 +1039,19 @@ bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, 
     const int64_t M = rows;
     const int64_t N = op == RDM_GEMM_NN ? m : k;   // output columns
     const int64_t K = op == RDM_GEMM_NN ? k : m;   // contraction
+    if (use_f16_gemm(ctx)) {
+      // rows padded to 128 bytes (zeros past K): an unaligned panel pitch (K = 100:
+      // 208 B) made every 64-byte box row straddle sectors — 0.69 → 1.0 ms
+      const int64_t ldb16 = (K + 63) / 64 * 64;
+      __nv_bfloat16* bt =
+          reinterpret_cast<__nv_bfloat16*>(ensure_ws(ctx->ws_tcb, (size_t)N * ldb16 * sizeof(__nv_bfloat16)));
+      prep_b_bf16_kernel<<<(unsigned)std::max<int64_t>(1, std::min<int64_t>(ceil_div(N * ldb16, 256), 4096)), 256,
+                           0, ctx->stream>>>(W, ldw, K, N, op == RDM_GEMM_NN ? 1 : 0, bt, ldb16);
+      RDM_LAUNCHED(ctx);
+      launch_nn_bf16(ctx, X, ldx, bt, ldb16, C, ldc, M, N, K, e);
+      return true;
+    }
+    // (128-byte panel rows, as the bf16 path uses, measured within noise here)
     const int64_t ldb = roundup4(K);
     float* bws = ensure_ws(ctx->ws_tcb, (size_t)2 * N * ldb * sizeof(float));
     float* bhi = bws;
