@@ -142,7 +142,7 @@ struct TileShape {
   int stage_bytes;    // HS · (NP · n_mma · 128 + 1024)
   int R;              // > 0: concatenated-piece MMAs with R rotating accumulator sets
   int acc_cols;       // TMEM columns per accumulator buffer
-  int dbg;            // timing experiments (RDM_TILE_DBG): 1 = skip the MMAs
+  int dbg;            // timing experiments (RDM_TILE_DBG): 1 = skip the MMAs, 2 = the i8 expansion, 4 = the i8 stores
   const float* colscale;   // NP == 2: 2^e_n per output column (fp16 pieces are column-scaled)
 };
 
@@ -544,11 +544,16 @@ __device__ __forceinline__ void tc_mma_i8_ts(uint32_t tmem_d, uint32_t tmem_a, u
       : "memory");
 }
 
-// One stage = one whole tile: B digits [3][n_mma][128 B] (128-byte swizzle,
-// one 3-D TMA), then the tile's bits [half][128 rows] u64.
-template <int D>
+// One stage = TP whole tiles of one item: TP digit panels [D][n_mma][128 B]
+// (128-byte swizzle, one 4-D TMA each), then the TP tiles' bits [half][128
+// rows] u64; an item's last stage is padded with the all-zero tile.  TP = 2
+// halves the per-stage handshakes (expander → MMA issuer → commits → ring
+// slots): 355 → 318 µs per Reddit-shaped w = 128 call, 174 → 159 µs at w = 41
+// (profiles/r2_tile_stages.md — halving the panel bytes alone changed nothing).
+template <int D, int TP>
 __global__ void __launch_bounds__(384, 1)
 hub_tile_i8_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __restrict__ bits,
+                   const uint64_t* __restrict__ zero_bits,
                    const int32_t* __restrict__ tile_cb, const int32_t* __restrict__ item_tb,
                    float* __restrict__ part, const TileShape sh) {
   extern __shared__ uint8_t smem_raw[];
@@ -564,8 +569,8 @@ hub_tile_i8_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __re
   const int warp = threadIdx.x >> 5, lane = threadIdx.x & 31;
   const int total = sh.n_items * sh.tiles_n;
   const int bbytes = D * n_mma * 128;
-  auto B_st = [&](int s) { return smem + s * sh.stage_bytes; };
-  auto bits_st = [&](int s) { return smem + s * sh.stage_bytes + bbytes; };
+  auto B_st = [&](int s, int u) { return smem + s * sh.stage_bytes + u * bbytes; };
+  auto bits_st = [&](int s, int u) { return smem + s * sh.stage_bytes + TP * bbytes + u * 2048; };
   if (threadIdx.x == 0) {
     for (int i = 0; i < S; ++i) {
       mbar_init(&full[i], 1);
@@ -599,44 +604,59 @@ hub_tile_i8_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __re
     // issue path); lane 0 issues the copies
     int s = 0;
     uint32_t ph = 0, kc = 0;
-    const uint32_t bytes = (uint32_t)bbytes + 2048;
+    // (timing experiments: 8 = load half of each digit panel, as one CTA of a
+    // pair would; 16 = skip the bits copies)
+    const uint32_t bytes =
+        (uint32_t)TP * ((uint32_t)((sh.dbg & 8) ? bbytes / 2 : bbytes) + ((sh.dbg & 16) ? 0 : 2048));
+    int u = 0;   // tile slot within the current stage
     for (int t = blockIdx.x; t < total; t += gridDim.x) {
       const int item = t / sh.tiles_n;
       const int n0 = (t % sh.tiles_n) * n_mma;
       const int tb = item_tb[item], T = item_tb[item + 1] - tb;
       const int rot = (int)(((unsigned)item * 2654435761u) % (unsigned)max(T, 1));
-      for (int i0 = 0; i0 < T; i0 += 32) {
+      const int Tp = (T + TP - 1) / TP * TP;   // padded with zero tiles
+      for (int i0 = 0; i0 < Tp; i0 += 32) {
         int idx = rot + i0 + lane;
         idx -= (idx >= T) ? T : 0;
         idx -= (idx >= T) ? T : 0;
-        const int my_tile = tb + idx;
-        const int my_cb = (i0 + lane < T) ? __ldg(tile_cb + my_tile) : 0;
-        const int cnt = min(32, T - i0);
+        const bool real = i0 + lane < T;
+        const int my_tile = real ? tb + idx : -1;
+        const int my_cb = real ? __ldg(tile_cb + tb + idx) : 0;
+        const int cnt = min(32, Tp - i0);
+        int last_cb = __shfl_sync(0xffffffffu, my_cb, 0);
         for (int k = 0; k < cnt; ++k) {
           const int tile = __shfl_sync(0xffffffffu, my_tile, k);
-          const int cb = __shfl_sync(0xffffffffu, my_cb, k);
+          int cb = __shfl_sync(0xffffffffu, my_cb, k);
+          if (tile < 0) cb = last_cb;   // zero tile: any panel
+          last_cb = cb;
           if (lane == 0) {
-            if (kc >= (uint32_t)S) mbar_wait(&empty[s], ph ^ 1);
-            mbar_expect_tx(&full[s], bytes);
-            bulk_load(bits_st(s), bits + (int64_t)tile * 2 * TK, 2048, &full[s]);
-            tma_load_4d(B_st(s), &tmB, &full[s], 0, n0, 0, cb);
+            if (u == 0) {
+              if (kc >= (uint32_t)S) mbar_wait(&empty[s], ph ^ 1);
+              mbar_expect_tx(&full[s], bytes);
+            }
+            if (!(sh.dbg & 16))
+              bulk_load(bits_st(s, u), tile >= 0 ? bits + (int64_t)tile * 2 * TK : zero_bits, 2048, &full[s]);
+            tma_load_4d(B_st(s, u), &tmB, &full[s], 0, n0, 0, cb);
           }
-          ++kc;
-          if (++s == S) { s = 0; ph ^= 1; }
+          if (++u == TP) {
+            u = 0;
+            ++kc;
+            if (++s == S) { s = 0; ph ^= 1; }
+          }
         }
       }
     }
   } else if (warp == 1) {
     if (lane == 0) {
       const uint32_t idesc = idesc_i8(D * n_mma);
-      const uint64_t bd0 = sdesc(smem_u32(B_st(0)), 16, 1024);
-      const uint32_t st16 = (uint32_t)sh.stage_bytes >> 4;
+      const uint64_t bd0 = sdesc(smem_u32(B_st(0, 0)), 16, 1024);
+      const uint32_t st16 = (uint32_t)sh.stage_bytes >> 4, bb16 = (uint32_t)bbytes >> 4;
       int s = 0, a = 0;
       uint32_t ph = 0, aph = 0;
       int it = 0;
       for (int t = blockIdx.x; t < total; t += gridDim.x, ++it) {
         const int item = t / sh.tiles_n;
-        const int nst = item_tb[item + 1] - item_tb[item];
+        const int nst = (item_tb[item + 1] - item_tb[item] + TP - 1) / TP;
         const int acc = it & 1;
         if (it >= 2) mbar_wait(&tempty[acc], ((it >> 1) - 1) & 1);
         tc_fence_after();
@@ -644,12 +664,15 @@ hub_tile_i8_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __re
         for (int st = 0; st < nst; ++st) {
           mbar_wait(&conv[a], aph);
           tc_fence_after();
-          const uint32_t ta = tmem_base + kAcol + a * 32;
-          const uint64_t bd = bd0 + (uint64_t)(s * st16);
           if (!(sh.dbg & 1)) {
 #pragma unroll
-            for (int j = 0; j < TK / 32; ++j)   // K = 32 int8 per MMA: 8 A columns, 32 B of B rows
-              tc_mma_i8_ts(d_tmem, ta + j * 8, bd + 2 * j, idesc, (st | j) ? 1u : 0u);
+            for (int uu = 0; uu < TP; ++uu) {
+              const uint32_t ta = tmem_base + kAcol + (a * TP + uu) * 32;
+              const uint64_t bd = bd0 + (uint64_t)(s * st16 + uu * bb16);
+#pragma unroll
+              for (int j = 0; j < TK / 32; ++j)   // K = 32 int8 per MMA: 8 A columns, 32 B of B rows
+                tc_mma_i8_ts(d_tmem, ta + j * 8, bd + 2 * j, idesc, (st | uu | j) ? 1u : 0u);
+            }
           }
           tc_commit(&empty[s]);
           tc_commit(&aempty[a]);
@@ -667,21 +690,26 @@ hub_tile_i8_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __re
     uint32_t ph = 0, aph = 0, kc = 0;
     for (int t = blockIdx.x; t < total; t += gridDim.x) {
       const int item = t / sh.tiles_n;
-      const int nst = item_tb[item + 1] - item_tb[item];
+      const int nst = (item_tb[item + 1] - item_tb[item] + TP - 1) / TP;
       for (int st = 0; st < nst; ++st, ++kc) {
         mbar_wait(&full[s], ph);
         if (kc >= (uint32_t)SA) {
           mbar_wait(&aempty[a], aph ^ 1);
           tc_fence_after();
         }
-        const uint32_t bs = smem_u32(bits_st(s)) + r * 8;
-        const uint2 h0 = lds64(bs), h1 = lds64(bs + 1024);
-        const uint32_t w4[4] = {h0.x, h0.y, h1.x, h1.y};
-        uint32_t v[32];
+        if (!(sh.dbg & 2)) {   // (timing experiments: 2 = skip the expansion)
 #pragma unroll
-        for (int i = 0; i < 32; ++i) v[i] = (((w4[i >> 3] >> (4 * (i & 7))) & 15u) * 0x204081u) & 0x01010101u;
-        tmem_st32u(tmem_base + lane_off + kAcol + a * 32, v);
-        asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+          for (int uu = 0; uu < TP; ++uu) {
+            const uint32_t bs = smem_u32(bits_st(s, uu)) + r * 8;
+            const uint2 h0 = lds64(bs), h1 = lds64(bs + 1024);
+            const uint32_t w4[4] = {h0.x, h0.y, h1.x, h1.y};
+            uint32_t v[32];
+#pragma unroll
+            for (int i = 0; i < 32; ++i) v[i] = (((w4[i >> 3] >> (4 * (i & 7))) & 15u) * 0x204081u) & 0x01010101u;
+            tmem_st32u(tmem_base + lane_off + kAcol + (a * TP + uu) * 32, v);
+          }
+          asm volatile("tcgen05.wait::st.sync.aligned;" ::: "memory");
+        }
         tc_fence_before();
         mbar_arrive(&conv[a]);
         if (++s == S) { s = 0; ph ^= 1; }
@@ -707,7 +735,7 @@ hub_tile_i8_kernel(const __grid_constant__ CUtensorMap tmB, const uint64_t* __re
         for (int d = 0; d < D; ++d) tmem_ld32(a0 + (uint32_t)(d * n_mma), dg[d]);
 #pragma unroll
         for (int i = 0; i < 32; i += 4)
-          if (n0 + c0 + i < sh.w) {
+          if (n0 + c0 + i < sh.w && !(sh.dbg & 4)) {   // (4 = skip the stores)
             const float4 cs = __ldg(reinterpret_cast<const float4*>(sh.colscale + n0 + c0 + i));
             float o[4];
 #pragma unroll
@@ -1080,6 +1108,12 @@ bool hub_tiles_pay(const Core& c, int64_t w, int np) {
 
 // int8 digits (np == kPiecesI8: 3, kPiecesI8x2: 2): column maxima, digit
 // panels, hub_tile_i8_kernel<D>.
+// tiles per stage of hub_tile_i8_kernel (RDM_TILE_TPS=1 / 2 for experiments)
+int tile_tps() {
+  const char* e = getenv("RDM_TILE_TPS");
+  return e && atoi(e) == 1 ? 1 : 2;
+}
+
 void hub_tiles_product_i8(rdm_ctx* ctx, const Core& c, const float* X, int64_t ldx, int64_t w, float* part,
                           int64_t ldp, int D) {
   const int64_t K2 = c.K2;
@@ -1107,14 +1141,15 @@ void hub_tiles_product_i8(rdm_ctx* ctx, const Core& c, const float* X, int64_t l
   sh.R = 1;
   sh.HS = 1;
   sh.acc_cols = (D * sh.n_mma + 31) / 32 * 32;
-  sh.stage_bytes = (D * sh.n_mma * 128 + 2048 + 1023) / 1024 * 1024;
+  const int TP = tile_tps();
+  sh.stage_bytes = (TP * (D * sh.n_mma * 128 + 2048) + 1023) / 1024 * 1024;
   const int avail = kSmemBudget - 1024 - 1024;
   sh.S = std::min(32, avail / sh.stage_bytes);
-  sh.SA = std::min(8, (512 - 2 * sh.acc_cols) / 32);
+  sh.SA = std::min(8, (512 - 2 * sh.acc_cols) / (32 * TP));
   sh.dbg = getenv("RDM_TILE_DBG") ? atoi(getenv("RDM_TILE_DBG")) : 0;
   sh.colscale = cs;
   RDM_CHECK_ARG(sh.S >= 2 && sh.SA >= 2, "hub tiles (int8): TMEM/smem budget");
-  const CUtensorMap tb = panel_map_i8(pan, K2, w, sh.n_mma, D);
+  const CUtensorMap tb = panel_map_i8(pan, K2, w, (sh.dbg & 8) ? sh.n_mma / 2 : sh.n_mma, D);
   if (tiles_paired()) {
     // two row blocks per panel load (hub_tile_i8_pair_kernel)
     TileShape ps = sh;
@@ -1138,10 +1173,11 @@ void hub_tiles_product_i8(rdm_ctx* ctx, const Core& c, const float* X, int64_t l
   const int smem = sh.S * sh.stage_bytes + 1024 + 1024;
   const int64_t total = c.n_items * sh.tiles_n;
   const unsigned grid = (unsigned)std::min<int64_t>(total, ctx->num_sms);
-  auto kern = D == 3 ? hub_tile_i8_kernel<3> : hub_tile_i8_kernel<2>;
+  auto kern = D == 3 ? (TP == 2 ? hub_tile_i8_kernel<3, 2> : hub_tile_i8_kernel<3, 1>)
+                     : (TP == 2 ? hub_tile_i8_kernel<2, 2> : hub_tile_i8_kernel<2, 1>);
   RDM_CUDA(cudaFuncSetAttribute(kern, cudaFuncAttributeMaxDynamicSharedMemorySize, smem));
-  kern<<<grid, 384, smem, ctx->stream>>>(tb, c.tiles->as<uint64_t>(), c.tile_cb->as<int32_t>(),
-                                         c.item_tb->as<int32_t>(), part, sh);
+  kern<<<grid, 384, smem, ctx->stream>>>(tb, c.tiles->as<uint64_t>(), c.zero_bits->as<uint64_t>(),
+                                         c.tile_cb->as<int32_t>(), c.item_tb->as<int32_t>(), part, sh);
   RDM_LAUNCHED(ctx);
 }
 

@@ -1,0 +1,4 @@
+# round 2, call aj: hub_tile_i8_kernel decomposition (RDM_TILE_DBG) under an ncu launch list
+mkdir -p gpurun_out
+timeout 900 ncu --metrics gpu__time_duration.sum,sm__pipe_tc_cycles_active.avg.pct_of_peak_sustained_elapsed --clock-control none -k regex:hub_tile_i8 --csv --log-file gpurun_out/r2aj_tile_dbg.csv python tools/exp_tile_dbg.py > gpurun_out/r2aj_tile_dbg.log 2>&1
+echo done
