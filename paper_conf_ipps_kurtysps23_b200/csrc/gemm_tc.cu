@@ -870,7 +870,8 @@ void launch_tc(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, const C
 // x 256; BN ≤ 128 with A in TMEM gains where K is short and N ≤ 256 (K = 100,
 // N = 256: 1.10 → 1.02 ms), with A split in smem and two partial accumulators
 // where K is long or the tile narrow (K = 602: 229 → 208 µs; N = 41: 68 → 52
-// µs); the 602-wide NT (K = 128, five 128-wide tiles) stays single.
+// µs); the 602-wide NT (K = 128, five 128-wide tiles) and single-tile short
+// contractions stay single.
 // Returns 0 (single CTA), 1 (pair, A in TMEM / smem for BN = 256), 2 (pair, A
 // split in smem, BN ≤ 128).
 int use_pair(rdm_ctx* ctx, int64_t M, int64_t N, int64_t K, int BN, int splits) {
@@ -882,7 +883,10 @@ int use_pair(rdm_ctx* ctx, int64_t M, int64_t N, int64_t K, int BN, int splits) 
   if (BN == 256) return 1;
   if (fa) return atoi(fa) ? 2 : 1;
   if (K >= 256 || BN <= 64) return 2;
-  if (N <= 256 || fp) return 1;
+  // two 128-wide tiles (products-shaped 100 → 256): A in TMEM; one tile of a
+  // short contraction (the Reddit-shaped NT 41 → 128 with its mask: 75 vs 82
+  // µs in the epoch's launch list) and the five tiles of the 602-wide NT stay single
+  if ((N > BN && N <= 256) || fp) return 1;
   return 0;
 }
 
