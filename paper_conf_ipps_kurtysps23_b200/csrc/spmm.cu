@@ -625,6 +625,10 @@ void pick_gvu(int c, bool bf, int* G, int* V, int* U, bool dram_slice = false) {
   if (!bf) {
     // 9-12 vectors (w = 33..48): 8 lanes x 2 (profiles/r2_spmm_gvu.txt: w = 41 0.82 → 0.79 ms)
     if (c >= 9 && c <= 12) { *G = 8; *V = 2; }
+    // L2-resident slices of 17-32 vectors (Reddit-shaped w = 128): 16 lanes x 2
+    // — fewer registers, 6 CTAs per SM instead of 4 (1.207 → 1.168 ms per call,
+    // profiles/r2_spmm_u.txt)
+    if (!dram_slice && c >= 17 && c <= 32) { *G = 16; *V = 2; }
     // DRAM-resident slices of 5-8 vectors (products-shaped w = 32 at P = 8):
     // 4 nnz in flight per group (2.61 → 2.46 ms); at <= 4 vectors U = 1 stays
     // best (papers100M-shaped w = 16: U = 4 85 ms vs U = 1 77 ms, r2_relabel.md)
