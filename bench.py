@@ -102,6 +102,12 @@ class ClockSampler:
         for line in self.proc.stdout:
             self.lines.append(line.strip())
 
+    def ready(self):
+        """True once nvidia-smi has produced its first sample (its start-up
+        NVML initialisation stalls host-side CUDA calls for up to ~100 ms:
+        it must not land inside the timed region)."""
+        return self.proc is None or len(self.lines) > 0
+
     def stop(self):
         if not self.proc:
             return None
@@ -290,6 +296,12 @@ def saint_main(a, world, rank, local_rank):
     clk = ClockSampler(local_rank)
     clk.start()
     for _ in range(max(3, a.warmup)):
+        step()
+    # keep warming up until the clock sampler is past its start-up (a one-off
+    # 10-100 ms stall of the host-synchronised sampler steps otherwise hit the
+    # 4th timed step)
+    t_w = time.time()
+    while not clk.ready() and time.time() - t_w < 5.0:
         step()
     ctx.sync()
     sizes.clear()
@@ -487,6 +499,9 @@ def emulate_main(a):
     clk = ClockSampler(0)
     clk.start()
     time.sleep(0.3)
+    t_w = time.time()
+    while not clk.ready() and time.time() - t_w < 5.0:
+        time.sleep(0.05)
     torch.cuda.synchronize(dev)
     e0 = torch.cuda.Event(enable_timing=True)
     e1 = torch.cuda.Event(enable_timing=True)
@@ -759,6 +774,9 @@ def main():
     clk = ClockSampler(local_rank)
     clk.start()
     time.sleep(0.3)
+    t_w = time.time()
+    while not clk.ready() and time.time() - t_w < 5.0:
+        time.sleep(0.05)
     if world > 1:
         dist.barrier()
     torch.cuda.synchronize(dev)

@@ -873,13 +873,16 @@ void launch_tc(rdm_ctx* ctx, const CUtensorMap& a, const CUtensorMap& b, const C
 // µs); the 602-wide NT (K = 128, five 128-wide tiles) and single-tile short
 // contractions stay single.
 // Returns 0 (single CTA), 1 (pair, A in TMEM / smem for BN = 256), 2 (pair, A
-// split in smem, BN ≤ 128).
+// split in smem, BN ≤ 128); pairs only from 148·256 rows on.
 int use_pair(rdm_ctx* ctx, int64_t M, int64_t N, int64_t K, int BN, int splits) {
   if (BN < 32 || splits > 1) return 0;
   const char* fp = getenv("RDM_PAIR");
   const char* fa = getenv("RDM_PAIR_ASMEM");
   if (fp && !atoi(fp)) return 0;
-  if (!fp && M < (int64_t)ctx->num_sms * BM) return 0;
+  // at least two 256-row pair tiles per SM pair: the GraphSAINT subgraphs
+  // (≈ 25 k rows, GEMMs running beside the sampler's kernels on its own
+  // stream) ran 3.74 → 3.85 ms per step with pairs, which need whole TPCs free
+  if (!fp && M < (int64_t)ctx->num_sms * 2 * BM) return 0;
   if (BN == 256) return 1;
   if (fa) return atoi(fa) ? 2 : 1;
   if (K >= 256 || BN <= 64) return 2;

@@ -619,16 +619,16 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
 // columns each).  Measured on the Reddit- and products-shaped residual CSRs
 // (tools/exp_gvu.py, profiles/r1_spmm_gvu.txt): for bf16 rows several nnz in
 // flight per group (U) pay; fp32 keeps U = 1 (best or tied at every width).
-void pick_gvu(int c, bool bf, int* G, int* V, int* U, bool dram_slice = false) {
+void pick_gvu(int c, bool bf, int* G, int* V, int* U, bool dram_slice = false, bool near_l2 = false) {
   pick_gv(c, G, V);
   *U = 1;
   if (!bf) {
     // 9-12 vectors (w = 33..48): 8 lanes x 2 (profiles/r2_spmm_gvu.txt: w = 41 0.82 → 0.79 ms)
     if (c >= 9 && c <= 12) { *G = 8; *V = 2; }
-    // L2-resident slices of 17-32 vectors (Reddit-shaped w = 128): 16 lanes x 2
-    // — fewer registers, 6 CTAs per SM instead of 4 (1.207 → 1.168 ms per call,
-    // profiles/r2_spmm_u.txt)
-    if (!dram_slice && c >= 17 && c <= 32) { *G = 16; *V = 2; }
+    // slices of 17-32 vectors up to ≈ 2 L2s (Reddit-shaped w = 128, 119 MB):
+    // 16 lanes x 2 — fewer registers, 6 CTAs per SM instead of 4 (1.207 →
+    // 1.168 ms per call, profiles/r2_spmm_u.txt)
+    if (near_l2 && c >= 17 && c <= 32) { *G = 16; *V = 2; }
     // DRAM-resident slices of 5-8 vectors (products-shaped w = 32 at P = 8):
     // 4 nnz in flight per group (2.61 → 2.46 ms); at <= 4 vectors U = 1 stays
     // best (papers100M-shaped w = 16: U = 4 85 ms vs U = 1 77 ms, r2_relabel.md)
@@ -875,8 +875,9 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
   } else {
     const int c4 = (int)std::min<int64_t>(chunk4, w4 / 4);
     int U = 1;
-    const bool dram_slice = (double)A.in_rows() * (double)ld_in * 4.0 > 96e6;
-    if (!getenv("RDM_SPMM_GV")) pick_gvu(c4, false, &G, &V, &U, dram_slice);
+    const double slice_bytes = (double)A.in_rows() * (double)ld_in * 4.0;
+    const bool dram_slice = slice_bytes > 96e6;
+    if (!getenv("RDM_SPMM_GV")) pick_gvu(c4, false, &G, &V, &U, dram_slice, slice_bytes <= 256e6);
     Hot hot{nullptr, 0, 0};
     const char* rl = getenv("RDM_RELABEL");   // column relabelling of DRAM-resident slices (experiment)
     if (dram_slice && A.col_hot && !(rl && !atoi(rl))) hot = rank_panel(ctx, A, in, ld_in);
