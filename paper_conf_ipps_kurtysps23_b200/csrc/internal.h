@@ -248,6 +248,10 @@ struct rdm_ctx {
   };
   std::vector<Ev> events;
   std::vector<cudaEvent_t> event_pool;
+  // auxiliary stream: the SpMM's short-row kernel runs on it beside the
+  // long-row kernel (disjoint rows), forked / joined with these events
+  cudaStream_t aux = nullptr;
+  cudaEvent_t aux_fork = nullptr, aux_join = nullptr;
   double phase_ms[RDM_PH_COUNT] = {};
   int64_t phase_launches[RDM_PH_COUNT] = {};
   bool virtual_group() const { return rank == RDM_ALL_RANKS && world > 1; }

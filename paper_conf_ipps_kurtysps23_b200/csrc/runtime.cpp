@@ -702,6 +702,12 @@ rdm_status rdm_finalize(rdm_ctx* ctx) {
     cudaEventDestroy(e.b);
   }
   for (auto e : ctx->event_pool) cudaEventDestroy(e);
+  if (ctx->aux) {
+    cudaStreamSynchronize(ctx->aux);
+    cudaStreamDestroy(ctx->aux);
+    cudaEventDestroy(ctx->aux_fork);
+    cudaEventDestroy(ctx->aux_join);
+  }
   if (ctx->comm) ncclCommDestroy(ctx->comm);
   delete ctx;
   release_retired();

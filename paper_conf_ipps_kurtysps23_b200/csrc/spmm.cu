@@ -563,13 +563,14 @@ void launch_spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, flo
 // The short light rows [n_long, n_light) of the light-row list.
 template <int G, int V, int U>
 void launch_spmm_short(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
-                       int64_t w4, int chunk4, const Epi& epi, const Hot& hot, int64_t n_long) {
+                       int64_t w4, int chunk4, const Epi& epi, const Hot& hot, int64_t n_long,
+                       cudaStream_t st) {
   const int64_t n_short = A.n_light - n_long;
   if (n_short <= 0) return;
   constexpr int R = 32 / G;
   const int64_t chunks = ceil_div(w4, 4 * chunk4);
   dim3 grid((unsigned)ceil_div(n_short, (int64_t)kWarps * R), (unsigned)chunks);
-  spmm_short_kernel<G, V, U><<<grid, kWarps * 32, 0, ctx->stream>>>(
+  spmm_short_kernel<G, V, U><<<grid, kWarps * 32, 0, st>>>(
       A.rowptr->as<int64_t>(), hot.hw ? A.col_hot->as<int32_t>() : A.col->as<int32_t>(), A.val->as<float>(),
       A.light_rows->as<int32_t>() + n_long, n_short, hot.hw ? hot.xh : in, hot.hw ? hot.ldh : ld_in, out, ld_out,
       w4, chunk4, epi);
@@ -886,11 +887,30 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
     if (const char* e = getenv("RDM_SPMM_SHORT")) short_deg = std::max(0, std::min(Csr::kDegTab, atoi(e)));
     const int64_t n_long = short_deg > 0 ? A.deg_ge[short_deg + 1 <= Csr::kDegTab ? short_deg + 1 : Csr::kDegTab]
                                          : A.n_light;
+    // The short rows run on the auxiliary stream beside the long-row kernel
+    // (disjoint output rows, both read only the tile partials finished
+    // before): its CTAs fill the long kernel's register-limited occupancy and
+    // its tail.  RDM_SPMM_CONC=0: one stream (experiments).
+    const char* conc_e = getenv("RDM_SPMM_CONC");
+    const bool conc = short_deg > 0 && A.n_light > n_long && (A.n_seg + n_long) > 0 && !(conc_e && !atoi(conc_e));
+    cudaStream_t sst = ctx->stream;
+    if (conc) {
+      if (!ctx->aux) {
+        int lo = 0, hi = 0;
+        RDM_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+        RDM_CUDA(cudaStreamCreateWithPriority(&ctx->aux, cudaStreamNonBlocking, lo));
+        RDM_CUDA(cudaEventCreateWithFlags(&ctx->aux_fork, cudaEventDisableTiming));
+        RDM_CUDA(cudaEventCreateWithFlags(&ctx->aux_join, cudaEventDisableTiming));
+      }
+      RDM_CUDA(cudaEventRecord(ctx->aux_fork, ctx->stream));
+      RDM_CUDA(cudaStreamWaitEvent(ctx->aux, ctx->aux_fork, 0));
+      sst = ctx->aux;
+    }
     if (short_deg > 0) {
       int sg, sv;
       pick_gv(c4, &sg, &sv);
 #define RDM_SHORT_CASE(g_, v_) \
-  if (sg == g_ && sv == v_) launch_spmm_short<g_, v_, 2>(ctx, A, in, ld_in, out, ld_out, w4, chunk4, epi, hot, n_long); else
+  if (sg == g_ && sv == v_) launch_spmm_short<g_, v_, 2>(ctx, A, in, ld_in, out, ld_out, w4, chunk4, epi, hot, n_long, sst); else
       RDM_SHORT_CASE(1, 1) RDM_SHORT_CASE(1, 2) RDM_SHORT_CASE(1, 3) RDM_SHORT_CASE(1, 4)
       RDM_SHORT_CASE(2, 1) RDM_SHORT_CASE(2, 2) RDM_SHORT_CASE(2, 3) RDM_SHORT_CASE(2, 4)
       RDM_SHORT_CASE(4, 1) RDM_SHORT_CASE(4, 2) RDM_SHORT_CASE(4, 3) RDM_SHORT_CASE(4, 4)
@@ -917,6 +937,10 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
     RDM_SPMM_CASE(32, 1, 4) RDM_SPMM_CASE(8, 1, 8)
     throw Error(RDM_ERR_ARG, "spmm: no kernel for G/V/U");
 #undef RDM_SPMM_CASE
+    if (conc) {
+      RDM_CUDA(cudaEventRecord(ctx->aux_join, ctx->aux));
+      RDM_CUDA(cudaStreamWaitEvent(ctx->stream, ctx->aux_join, 0));
+    }
   }
 heavy:
   if (A.n_heavy) {
