@@ -40,6 +40,20 @@ namespace {
 using namespace tc;
 
 constexpr int BK = 32;         // fp32 elements per 128-byte swizzle row
+
+// Timeline trace of CTA 0 (build with -DRDM_TC_TRACE, tools/build_variant.sh;
+// read with rdm_debug_tc_trace, tools/tc_trace.py): clock64 per role and
+// k-block / tile.
+#ifdef RDM_TC_TRACE
+constexpr int kTrN = 4096;
+__device__ long long g_tc_trace[8][kTrN];
+#define TCTRACE(ev, idx)                                                        \
+  do {                                                                          \
+    if (blockIdx.x == 0 && (idx) < kTrN) g_tc_trace[ev][idx] = clock64();      \
+  } while (0)
+#else
+#define TCTRACE(ev, idx) do { } while (0)
+#endif
 constexpr int UK = 8;          // UMMA K for kind::tf32
 
 struct TcEpi {
@@ -328,6 +342,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         for (int kb = 0; kb < nkb; ++kb, ++kc) {
           const int s = kc % S;
           if (kc >= (uint32_t)S) mbar_wait(&empty[s], ((kc / S) - 1) & 1);
+          TCTRACE(0, kc);
           mbar_expect_tx(&full[s], bytes);
           const int kk = (int)(kbeg + (int64_t)kb * BK);
           if (MODE == 0) {
@@ -373,6 +388,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           const int cs = kc % SC;
           if (PAIR == 2) mbar_wait_cluster(&conv[cs], (kc / SC) & 1);
           else mbar_wait(&conv[cs], (kc / SC) & 1);
+          TCTRACE(3, kc);
           tc_fence_after();
           const uint32_t bh = smem_u32(B_hi(s)), bl = smem_u32(B_lo(s));
           if (F16) {
@@ -453,6 +469,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           if (CF::kTmemA) tc_commit_g<PAIR>(&aempty[st]);
         }
         tc_commit_g<PAIR>(&tfull[acc]);   // fires when this tile's MMAs (if any) are done
+        TCTRACE(4, it);
       }
     }
   } else if (warp >= 4 && warp < 8) {
@@ -471,6 +488,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           tc_fence_after();
         }
         mbar_wait(&full[s], (kc / S) & 1);
+        if (threadIdx.x == 128) TCTRACE(1, kc);
         if (sh.dbg & 1) {
         } else if (sh.one) {
           // 1xTF32: A rounded to tf32 into TMEM; smem operands are read as tf32
@@ -521,6 +539,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
           if (lane == 0) mbar_arrive_cluster(conv_leader + (uint32_t)(cs * sizeof(uint64_t)));
         } else {
           mbar_arrive(&conv[cs]);
+          if (threadIdx.x == 128) TCTRACE(2, kc);
         }
       }
     }
@@ -538,6 +557,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
       const int64_t n0 = (int64_t)(rem % sh.tiles_n) * BN;
       const int acc = it & 1;
       mbar_wait_sleep(&tfull[acc], (it >> 1) & 1);
+      if (threadIdx.x == 256) TCTRACE(5, it);
       tc_fence_after();
       float* Cz = C + (int64_t)z * sh.M * ldc;
       const int64_t row0 = m0 + q * 32;
@@ -671,6 +691,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
         if (lane == 0) mbar_arrive_cluster(tempty_leader + (uint32_t)(acc * sizeof(uint64_t)));
       } else {
         mbar_arrive(&tempty[acc]);
+        if (threadIdx.x == 256) TCTRACE(6, it);
       }
     }
     if (sh.tstore && lane == 0) bulk_wait0();   // every TMA store of this warp has landed
@@ -1112,6 +1133,17 @@ bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, 
 }
 
 }  // namespace rdm
+
+extern "C" int rdm_debug_tc_trace(long long* out, int n) {
+#ifdef RDM_TC_TRACE
+  const int m = n < 8 * rdm::kTrN ? n : 8 * rdm::kTrN;
+  return cudaMemcpyFromSymbol(out, rdm::g_tc_trace, (size_t)m * sizeof(long long)) == cudaSuccess ? m : -1;
+#else
+  (void)out;
+  (void)n;
+  return 0;
+#endif
+}
 
 extern "C" int rdm_debug_disable_tc(int disable) {
   rdm::g_tc_disabled = disable != 0;
