@@ -919,7 +919,7 @@ int use_pair(rdm_ctx* ctx, int64_t M, int64_t N, int64_t K, int BN, int splits) 
 // tools/time_gemm.py, products-shaped 2.45 M x 256 · 256 x 256: 1.94 →
 // 1.76 ms), else several 128-wide tiles (TMEM-A path; K = 100: 1.18 vs
 // 1.47 ms).  RDM_BN256=1 / 0 forces either (experiments).
-int pick_bn(int64_t N, int64_t K = 0, bool three = true, bool mask = false) {
+int pick_bn(int64_t N, int64_t K = 0, bool three = true, bool mask = false, bool pairs = false) {
   if (N <= 16) return 16;
   if (N <= 32) return 32;
   if (N <= 64) return 64;
@@ -927,7 +927,12 @@ int pick_bn(int64_t N, int64_t K = 0, bool three = true, bool mask = false) {
   if (const char* e = getenv("RDM_BN256")) return atoi(e) ? 256 : 128;
   // (a Hadamard-mask epilogue over 256 columns with 4 epilogue warps loses
   // more than the wide tile gains: 1.06 → 1.34 ms in the products epoch)
-  return (three && K >= 256 && !mask) ? 256 : 128;
+  if (!three || mask) return 128;
+  // 256-wide tiles on CTA pairs pay at short K too (tools/time_gemm.py,
+  // profiles/r2_gemm_pair.md: the Reddit-shaped 602-wide NT, K = 128, 243 →
+  // 205 µs; products-shaped NN 100 → 256, 1.12 → 0.83 ms); single CTAs only
+  // from K = 256 on
+  return (K >= 256 || pairs) ? 256 : 128;
 }
 
 }  // namespace
@@ -967,7 +972,10 @@ void launch_nn_panels(rdm_ctx* ctx, const float* X, int64_t ldx, const float* bh
                       const TcEpi& e, int splits = 1, bool wide_ok = true) {
   // (256-wide tiles only for single-split calls: the split-K hub-core GEMM of
   // the GraphSAINT subgraphs ran slower with them)
-  const int BN = (splits == 1 && wide_ok) ? pick_bn(N, K, ctx->prec != RDM_PREC_FAST, (e.flags & RDM_EPI_MASK) != 0)
+  // would a 256-wide tile run on CTA pairs (use_pair's row threshold)?
+  const bool pairs_ok = splits == 1 && use_pair(ctx, M, N, K, 256, 1) != 0;
+  const int BN = (splits == 1 && wide_ok) ? pick_bn(N, K, ctx->prec != RDM_PREC_FAST, (e.flags & RDM_EPI_MASK) != 0,
+                                                    pairs_ok)
                                          : pick_bn(N, 0, false);
   const int pmode = use_pair(ctx, M, N, K, BN, splits);
   const bool pair = pmode != 0;
