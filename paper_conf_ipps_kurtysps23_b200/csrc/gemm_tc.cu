@@ -927,12 +927,14 @@ int pick_bn(int64_t N, int64_t K = 0, bool three = true, bool mask = false, bool
   if (const char* e = getenv("RDM_BN256")) return atoi(e) ? 256 : 128;
   // (a Hadamard-mask epilogue over 256 columns with 4 epilogue warps loses
   // more than the wide tile gains: 1.06 → 1.34 ms in the products epoch)
-  if (!three || mask) return 128;
-  // 256-wide tiles on CTA pairs pay at short K too (tools/time_gemm.py,
-  // profiles/r2_gemm_pair.md: the Reddit-shaped 602-wide NT, K = 128, 243 →
-  // 205 µs; products-shaped NN 100 → 256, 1.12 → 0.83 ms); single CTAs only
-  // from K = 256 on
-  return (K >= 256 || pairs) ? 256 : 128;
+  if (!three) return 128;
+  // 256-wide tiles on CTA pairs pay at short K and with the Hadamard mask too
+  // (profiles/r2_gemm_pair.md: the Reddit-shaped 602-wide NT, K = 128, 243 →
+  // 205 µs; products-shaped NN 100 → 256 1.12 → 0.83 ms; the products epoch
+  // with its masked NT 256 → 256 on 256-wide pair tiles 41.44 → 40.82 ms);
+  // single CTAs only from K = 256 on and without a mask
+  if (pairs) return 256;
+  return (K >= 256 && !mask) ? 256 : 128;
 }
 
 }  // namespace
