@@ -310,7 +310,53 @@ spmm_short_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict_
   float4 acc[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) acc[v] = make_float4(0.f, 0.f, 0.f, 0.f);
-  for (int64_t j = beg; j < end; j += U) {
+  // The row's first 32 (col, val) in one coalesced load up front (32/G per
+  // lane of the group), handed out by shuffles: the loop below then exposes
+  // one gather latency per step instead of a (col, val) load followed by the
+  // gather.  Same entry order, same sums.
+  constexpr int SL = 32 / G;
+  int pc[SL];
+  float pv[SL];
+#pragma unroll
+  for (int s = 0; s < SL; ++s) {
+    const int64_t j = beg + s * G + sub;
+    const bool ok = j < end;
+    pc[s] = ok ? __ldcs(col + j) : 0;
+    pv[s] = ok ? __ldcs(val + j) : 0.f;
+  }
+  const int deg = (int)(end - beg);
+  const int dmax = __reduce_max_sync(kFull, deg < 32 ? deg : 32);
+#pragma unroll
+  for (int e0 = 0; e0 < 32; e0 += U) {
+    if (e0 >= dmax) break;   // warp-uniform
+    int c[U];
+    float a[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int e = e0 + u;
+      c[u] = __shfl_sync(kFull, pc[e / G], g * G + (e % G));
+      a[u] = __shfl_sync(kFull, pv[e / G], g * G + (e % G));
+    }
+    float4 x[U][V];
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+#pragma unroll
+      for (int v = 0; v < V; ++v)
+        x[u][v] = (e0 + u < deg && v * G + sub < c4n)
+                      ? RDM_GATHER_LD(reinterpret_cast<const float4*>(xb + (int64_t)c[u] * ldx) + v * G + sub)
+                      : make_float4(0.f, 0.f, 0.f, 0.f);
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        acc[v].x = fmaf(a[u], x[u][v].x, acc[v].x);
+        acc[v].y = fmaf(a[u], x[u][v].y, acc[v].y);
+        acc[v].z = fmaf(a[u], x[u][v].z, acc[v].z);
+        acc[v].w = fmaf(a[u], x[u][v].w, acc[v].w);
+      }
+  }
+  // rows longer than 32 (RDM_SPMM_SHORT > 32, experiments): the rest entry by entry
+  for (int64_t j = beg + 32; j < end; j += U) {
     int c[U];
     float a[U];
 #pragma unroll
