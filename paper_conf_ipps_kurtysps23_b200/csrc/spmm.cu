@@ -290,7 +290,7 @@ spmm_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
 // per warp, U entries of its row in flight per group — short rows leave most
 // of a warp-per-row idle and serialise the rowptr → col → gather chain
 // (papers100M-shaped: average degree 15).  Same epilogue and stores.
-template <int G, int V, int U>
+template <int G, int V, int U, int NB = 32>
 __global__ void __launch_bounds__(kWarps * 32)
 spmm_short_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
                   const float* __restrict__ val, const int32_t* __restrict__ rows, int64_t n_rows,
@@ -310,11 +310,11 @@ spmm_short_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict_
   float4 acc[V];
 #pragma unroll
   for (int v = 0; v < V; ++v) acc[v] = make_float4(0.f, 0.f, 0.f, 0.f);
-  // The row's first 32 (col, val) in one coalesced load up front (32/G per
+  // The row's first NB (col, val) in one coalesced load up front (NB/G per
   // lane of the group), handed out by shuffles: the loop below then exposes
   // one gather latency per step instead of a (col, val) load followed by the
   // gather.  Same entry order, same sums.
-  constexpr int SL = 32 / G;
+  constexpr int SL = NB / G;
   int pc[SL];
   float pv[SL];
 #pragma unroll
@@ -325,9 +325,9 @@ spmm_short_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict_
     pv[s] = ok ? __ldcs(val + j) : 0.f;
   }
   const int deg = (int)(end - beg);
-  const int dmax = __reduce_max_sync(kFull, deg < 32 ? deg : 32);
+  const int dmax = __reduce_max_sync(kFull, deg < NB ? deg : NB);
 #pragma unroll
-  for (int e0 = 0; e0 < 32; e0 += U) {
+  for (int e0 = 0; e0 < NB; e0 += U) {
     if (e0 >= dmax) break;   // warp-uniform
     int c[U];
     float a[U];
@@ -355,8 +355,8 @@ spmm_short_kernel(const int64_t* __restrict__ rowptr, const int32_t* __restrict_
         acc[v].w = fmaf(a[u], x[u][v].w, acc[v].w);
       }
   }
-  // rows longer than 32 (RDM_SPMM_SHORT > 32, experiments): the rest entry by entry
-  for (int64_t j = beg + 32; j < end; j += U) {
+  // rows longer than NB (RDM_SPMM_SHORT > 64, experiments): the rest entry by entry
+  for (int64_t j = beg + NB; j < end; j += U) {
     int c[U];
     float a[U];
 #pragma unroll
@@ -610,13 +610,14 @@ void launch_spmm(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, flo
 template <int G, int V, int U>
 void launch_spmm_short(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* out, int64_t ld_out,
                        int64_t w4, int chunk4, const Epi& epi, const Hot& hot, int64_t n_long,
-                       cudaStream_t st) {
+                       cudaStream_t st, int short_deg) {
   const int64_t n_short = A.n_light - n_long;
   if (n_short <= 0) return;
   constexpr int R = 32 / G;
   const int64_t chunks = ceil_div(w4, 4 * chunk4);
   dim3 grid((unsigned)ceil_div(n_short, (int64_t)kWarps * R), (unsigned)chunks);
-  spmm_short_kernel<G, V, U><<<grid, kWarps * 32, 0, st>>>(
+  auto kern = short_deg > 32 ? spmm_short_kernel<G, V, U, 64> : spmm_short_kernel<G, V, U, 32>;
+  kern<<<grid, kWarps * 32, 0, st>>>(
       A.rowptr->as<int64_t>(), hot.hw ? A.col_hot->as<int32_t>() : A.col->as<int32_t>(), A.val->as<float>(),
       A.light_rows->as<int32_t>() + n_long, n_short, hot.hw ? hot.xh : in, hot.hw ? hot.ldh : ld_in, out, ld_out,
       w4, chunk4, epi);
@@ -929,7 +930,11 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
     const char* rl = getenv("RDM_RELABEL");   // column relabelling of DRAM-resident slices (experiment)
     if (dram_slice && A.col_hot && !(rl && !atoi(rl))) hot = rank_panel(ctx, A, in, ld_in);
     // short light rows (degree <= RDM_SPMM_SHORT, default 32) → row-per-group kernel
-    int short_deg = 32;
+    // degree threshold of the short-row kernel: 64 for slices up to 25 vectors
+    // (w ≤ 100: w = 41 0.625 → 0.608, w = 47 2.50 → 2.41, w = 100 4.82 → 4.73
+    // ms per call), 32 for wider ones (w = 256: 8.15 vs 8.72 at 64),
+    // profiles/r2_spmm_short_thr.txt
+    int short_deg = c4 <= 25 ? 64 : 32;
     if (const char* e = getenv("RDM_SPMM_SHORT")) short_deg = std::max(0, std::min(Csr::kDegTab, atoi(e)));
     const int64_t n_long = short_deg > 0 ? A.deg_ge[short_deg + 1 <= Csr::kDegTab ? short_deg + 1 : Csr::kDegTab]
                                          : A.n_light;
@@ -956,7 +961,7 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
       int sg, sv;
       pick_gv(c4, &sg, &sv);
 #define RDM_SHORT_CASE(g_, v_) \
-  if (sg == g_ && sv == v_) launch_spmm_short<g_, v_, 2>(ctx, A, in, ld_in, out, ld_out, w4, chunk4, epi, hot, n_long, sst); else
+  if (sg == g_ && sv == v_) launch_spmm_short<g_, v_, 2>(ctx, A, in, ld_in, out, ld_out, w4, chunk4, epi, hot, n_long, sst, short_deg); else
       RDM_SHORT_CASE(1, 1) RDM_SHORT_CASE(1, 2) RDM_SHORT_CASE(1, 3) RDM_SHORT_CASE(1, 4)
       RDM_SHORT_CASE(2, 1) RDM_SHORT_CASE(2, 2) RDM_SHORT_CASE(2, 3) RDM_SHORT_CASE(2, 4)
       RDM_SHORT_CASE(4, 1) RDM_SHORT_CASE(4, 2) RDM_SHORT_CASE(4, 3) RDM_SHORT_CASE(4, 4)
