@@ -254,7 +254,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
                const __grid_constant__ CUtensorMap tmBlo, const __grid_constant__ CUtensorMap tmApf,
                const __grid_constant__ CUtensorMap tmC, float* __restrict__ C, int64_t ldc,
                TcShape sh, TcEpi epi) {
-  static_assert(PAIR == 1 || MODE == 0, "CTA pairs: NN / NT only");
+  // (CTA pairs: NN / NT, and TN with MN-major B halves of 32-wide chunks)
   static_assert(!F16 || (MODE == 0 && PAIR == 1 && BN <= 128 && !ASM), "bf16 GEMM: NN / NT, A in TMEM");
   using CF = Cfg<BN, EW, PAIR, ASM, F16>;
   constexpr int S = CF::kStages;      // smem ring (raw A + B panels)
@@ -331,7 +331,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
   if (warp == 0) {
     if (lane == 0) {
       const uint32_t bbytes = (uint32_t)b_rows * BK * (F16 ? 2 : 4);
-      const uint32_t bytes = MODE == 0 ? (CF::kABytes + (sh.one ? 1 : 2) * bbytes) : (CF::kABytes + CF::kBBytes);
+      const uint32_t bytes = MODE == 0 ? (CF::kABytes + (sh.one ? 1 : 2) * bbytes) : (CF::kABytes + bbytes);
       uint32_t kc = 0;
       for (int t = cta0; t < total; t += ncta) {
         int64_t kbeg;
@@ -361,7 +361,7 @@ gemm_tc_kernel(const __grid_constant__ CUtensorMap tmA, const __grid_constant__ 
             if (!sh.one) tma_load_2d(B_lo(s), &tmBlo, &full[s], kk, n0);
           } else {
             for (int c = 0; c < BM / 32; ++c) tma_load_2d(A_hi(s) + c * 4096, &tmA, &full[s], m0 + 32 * c, kk);
-            for (int c = 0; c < BN / 32; ++c) tma_load_2d(B_hi(s) + c * 4096, &tmB, &full[s], n0 + 32 * c, kk);
+            for (int c = 0; c < b_rows / 32; ++c) tma_load_2d(B_hi(s) + c * 4096, &tmB, &full[s], n0 + 32 * c, kk);
           }
         }
       }
@@ -1109,8 +1109,19 @@ bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, 
   const int BN = N <= 32 ? 32 : N <= 64 ? 64 : N <= 128 ? 128
                  : (getenv("RDM_BN256") ? (atoi(getenv("RDM_BN256")) ? 256 : 128) : 256);
   const int n_mma = (int)std::min<int64_t>(BN, ((N + 31) / 32) * 32);
-  const int64_t tiles = ceil_div(M, BM) * ceil_div(N, BN);
-  int64_t splits = std::max<int64_t>(1, ctx->num_sms / std::max<int64_t>(1, tiles));
+  // CTA pairs (M = 256 per pair, each CTA loading half of U's 32-wide chunks):
+  // every SM loads half the U bytes per row chunk and the MMAs read half of B
+  // from its smem.  Needs M ≥ 256 and halves of whole 32-wide chunks.
+  const char* tp = getenv("RDM_TN_PAIR");
+  // Only where the 256-row pair tiles cover M with little padding: products-
+  // shaped 256 x 256 1.91 → 1.29 ms, while the 602-wide Reddit-shaped one (a
+  // third pair tile of 90 rows) went 236 → 276 µs (profiles/r2_gemm_pair.md).
+  const bool tile_fit = ceil_div(M, 2 * BM) * 2 * BM - M <= M / 10;
+  const bool pair = !(tp && !atoi(tp)) && M >= 2 * BM && BN >= 64 && n_mma % 64 == 0 &&
+                    ((K >= (int64_t)ctx->num_sms * 2 * BM && tile_fit) || (tp && atoi(tp)));   // RDM_TN_PAIR=1: forced (tests)
+  const int64_t tiles = ceil_div(M, BM * (pair ? 2 : 1)) * ceil_div(N, BN);
+  const int64_t slots = pair ? ctx->num_sms / 2 : ctx->num_sms;
+  int64_t splits = std::max<int64_t>(1, slots / std::max<int64_t>(1, tiles));
   // accuracy: the weight gradient sums over every row, often with heavy
   // cancellation (softmax − onehot is zero-sum); chains of at most kTnChain
   // rows in the fp32 TMEM accumulator (kTnChain), the partials summed in fp64
@@ -1118,6 +1129,9 @@ bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, 
   int64_t chain = 4096;
   if (const char* e = getenv("RDM_TN_CHAIN")) chain = std::max<int64_t>(256, atoll(e));
   splits = std::max<int64_t>(splits, ceil_div(K, chain));
+  // as many splits as the rounds of the persistent grid hold anyway (shorter
+  // chains, no idle slots in the last round)
+  splits = std::max<int64_t>(splits, ceil_div(tiles * splits, slots) * slots / tiles);
   splits = std::min<int64_t>(splits, std::max<int64_t>(1, K / (8 * BK)));
   const CUtensorMap ta = make_map(X, M, K, ldx, 32, BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B);  // inner = k
   const CUtensorMap tb = make_map(W, N, K, ldw, 32, BK, CU_TENSOR_MAP_SWIZZLE_128B_ATOM_32B);  // inner = m
@@ -1128,7 +1142,14 @@ bool gemm_tc(rdm_ctx* ctx, int op, const float* X, int64_t ldx, const float* W, 
     out = ensure_ws(ctx->ws_gemm, (size_t)splits * M * ldo * sizeof(float));
   }
   TcEpi none{0, nullptr, nullptr, 0};
-  switch (BN) {
+  if (pair) {
+    const CUtensorMap tbh = tb;   // the same 32 x 32 chunk boxes; each CTA loads its half of the chunks
+    switch (BN) {
+      case 64: launch_tc<64, 1, 2>(ctx, ta, tbh, tbh, out, ldo, M, N, K, (int)splits, n_mma, none); break;
+      case 128: launch_tc<128, 1, 2>(ctx, ta, tbh, tbh, out, ldo, M, N, K, (int)splits, n_mma, none); break;
+      default: launch_tc<256, 1, 2>(ctx, ta, tbh, tbh, out, ldo, M, N, K, (int)splits, n_mma, none); break;
+    }
+  } else switch (BN) {
     case 32: launch_tc<32, 1>(ctx, ta, tb, tb, out, ldo, M, N, K, (int)splits, n_mma, none); break;
     case 64: launch_tc<64, 1>(ctx, ta, tb, tb, out, ldo, M, N, K, (int)splits, n_mma, none); break;
     case 128: launch_tc<128, 1>(ctx, ta, tb, tb, out, ldo, M, N, K, (int)splits, n_mma, none); break;
