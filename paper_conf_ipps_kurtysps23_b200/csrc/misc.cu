@@ -123,8 +123,12 @@ xent_group_kernel(const float* __restrict__ Z, int64_t ldz, const int32_t* __res
   for (int64_t base = ((int64_t)blockIdx.x * kLossWarps + wid) * RPW; base < rows; base += stride) {
     const int64_t i = base + grp;
     const bool valid = i < rows;
+    // label and mask issued with the logits (no dependent load after the
+    // reductions); the label's logit is picked from registers below
+    const int y = valid ? __ldg(labels + i) : -1;
+    const bool m = valid && (mask ? __ldg(mask + i) != 0 : true);
     float4 v[V];
-    float mx = -FLT_MAX;
+    float mx = -FLT_MAX, zy = 0.f;
 #pragma unroll
     for (int k = 0; k < V; ++k) {
       const int64_t c = 4 * (sub + LPR * k);
@@ -134,7 +138,14 @@ xent_group_kernel(const float* __restrict__ Z, int64_t ldz, const int32_t* __res
       if (c + 2 >= C) v[k].z = -FLT_MAX;
       if (c + 3 >= C) v[k].w = -FLT_MAX;
       mx = fmaxf(mx, fmaxf(fmaxf(v[k].x, v[k].y), fmaxf(v[k].z, v[k].w)));
+      if (y == c) zy = v[k].x;
+      if (y == c + 1) zy = v[k].y;
+      if (y == c + 2) zy = v[k].z;
+      if (y == c + 3) zy = v[k].w;
     }
+    // exactly one lane of the group holds z_y: a sum of it and zeros is exact
+#pragma unroll
+    for (int o = LPR / 2; o; o >>= 1) zy += __shfl_xor_sync(0xffffffffu, zy, o);
 #pragma unroll
     for (int o = LPR / 2; o; o >>= 1) mx = fmaxf(mx, __shfl_xor_sync(0xffffffffu, mx, o));
     float s = 0.f;
@@ -149,8 +160,6 @@ xent_group_kernel(const float* __restrict__ Z, int64_t ldz, const int32_t* __res
 #pragma unroll
     for (int o = LPR / 2; o; o >>= 1) s += __shfl_xor_sync(0xffffffffu, s, o);
     if (valid) {
-      const int y = labels[i];
-      const bool m = mask ? mask[i] != 0 : true;
       const float scale = m ? inv_n : 0.f;
       const float inv_s = 1.f / s;
 #pragma unroll
@@ -165,7 +174,7 @@ xent_group_kernel(const float* __restrict__ Z, int64_t ldz, const int32_t* __res
           *reinterpret_cast<float4*>(G + i * ldg + c) = gv;
         }
       }
-      if (sub == 0 && m) local += (double)mx + log((double)s) - (double)Z[i * ldz + y];
+      if (sub == 0 && m) local += (double)mx + log((double)s) - (double)zy;
     }
   }
   local = warp_sum_d(local);
