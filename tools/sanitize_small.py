@@ -41,6 +41,35 @@ for (r, k, m) in ((1000, 64, 128), (1000, 128, 41), (700, 256, 256)):
     ctx.gemm(rdm.GEMM_TN, X, C, Y, r, k, m)
 ctx.sync()
 print("gemm ok", flush=True)
+# round-2 kernels: CTA-pair GEMMs (A in TMEM / smem, 256-wide), TN on pairs,
+# the fast variant's kind::f16 GEMMs
+for env in ({"RDM_PAIR": "1", "RDM_PAIR_ASMEM": "0"}, {"RDM_PAIR": "1", "RDM_PAIR_ASMEM": "1"},
+            {"RDM_TN_PAIR": "1"}):
+    os.environ.update(env)
+    for (r, k, m) in ((1000, 64, 128), (1000, 128, 41), (700, 256, 256), (600, 128, 602)):
+        X = torch.randn(r, k, device=dev)
+        W = torch.randn(k, m, device=dev)
+        C = torch.zeros(r, (m + 3) // 4 * 4, device=dev)
+        ctx.gemm(rdm.GEMM_NN, X, W, C, r, k, m)
+        Ct = torch.zeros(r, k, device=dev)
+        ctx.gemm(rdm.GEMM_NT, C, W, Ct, r, k, m)
+        Y = torch.zeros(k, m, device=dev)
+        ctx.gemm(rdm.GEMM_TN, X, C, Y, r, k, m)
+    ctx.sync()
+    for key in env:
+        os.environ.pop(key)
+    print("gemm", env, "ok", flush=True)
+ctx.set_precision("fast")
+for (r, k, m) in ((1000, 64, 128), (1000, 128, 41), (700, 100, 256)):
+    X = torch.randn(r, k + (-k) % 4, device=dev)
+    W = torch.randn(k, m, device=dev)
+    C = torch.zeros(r, (m + 3) // 4 * 4, device=dev)
+    ctx.gemm(rdm.GEMM_NN, X, W, C, r, k, m)
+    Ct = torch.zeros(r, (k + 3) // 4 * 4, device=dev)
+    ctx.gemm(rdm.GEMM_NT, C, W, Ct, r, k, m)
+ctx.sync()
+ctx.set_precision("fp32")
+print("gemm f16 ok", flush=True)
 f = [70, 32, 7]
 vg = rdm.Context(rank=rdm.ALL_RANKS, world=2, device=0)
 vg.set_graph(g.rowptr, g.col, g.val, symmetric=True)
