@@ -886,6 +886,19 @@ def main():
                 "spmm_share_of_step": ph_ms["spmm"] / max(1e-9, ms_total),
                 "avg_call_ms": ph_ms["spmm"] / max(1, spmm_calls),
                 "gather_gbs": (cnt["spmm_nnz_cols"] * 4) / spmm_s / 1e9 if spmm_s > 0 else 0.0}
+    # the unit that actually paces the residual CSR kernels (committed ncu
+    # capture of the same build, profiles/r2_spmm_units.json): L1/TEX, not HBM
+    try:
+        uj = _json.load(open(os.path.join(ROOT, "profiles", "r2_spmm_units.json"))).get(wl.name)
+        if uj and world == 1 and a.precision == "fp32" and not panels:
+            roofline["residual_kernels_pct_of_peak"] = {
+                k: {"l1tex": round(v[0]["l1tex__throughput.avg.pct_of_peak_sustained_elapsed"], 1),
+                    "l2": round(v[0]["lts__throughput.avg.pct_of_peak_sustained_elapsed"], 1),
+                    "dram_read": round(v[0]["dram__bytes_read.sum.pct_of_peak_sustained_elapsed"], 1)}
+                for k, v in uj["kernels"].items()}
+            roofline["residual_kernels_source"] = uj["source"]
+    except Exception:
+        pass
     a2a_s = ph_ms["a2a"] / 1e3
     a2a_bus = (cnt["a2a_bytes_wire"] / a2a_s / 1e9) if a2a_s > 0 and cnt["a2a_bytes_wire"] else None
 
