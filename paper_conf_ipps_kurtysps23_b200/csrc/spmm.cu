@@ -546,6 +546,118 @@ spmm_kernel_bf(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ c
   }
 }
 
+// bf16 variant of spmm_short_kernel (RDM_PREC_FAST): a group of G lanes per
+// short row, the row's first 32 (col, val) loaded up front and shuffled, U
+// entries in flight, each lane V 128-bit gathers of 8 bf16 columns; the same
+// epilogue and stores as spmm_kernel_bf.
+template <int G, int V, int U, bool FACT>
+__global__ void __launch_bounds__(kWarps * 32)
+spmm_short_kernel_bf(const int64_t* __restrict__ rowptr, const int32_t* __restrict__ col,
+                     const float* __restrict__ val, const int32_t* __restrict__ rows, int64_t n_rows,
+                     const __nv_bfloat16* __restrict__ X, int64_t ldx, float* __restrict__ out, int64_t ld_out,
+                     int64_t w4, int64_t w8, int chunk8, Epi epi) {
+  constexpr int R = 32 / G, NB = 32, SL = NB / G;
+  const int lane = threadIdx.x & 31;
+  const int g = lane / G, sub = lane % G;
+  const int64_t idx = ((int64_t)blockIdx.x * kWarps + (threadIdx.x >> 5)) * R + g;
+  const int64_t cbase = (int64_t)blockIdx.y * chunk8 * 8;
+  const int64_t rem8 = (w8 - cbase) / 8;
+  const int c8n = rem8 < chunk8 ? (int)rem8 : chunk8;
+  const bool live = idx < n_rows;
+  const int32_t r = live ? rows[idx] : 0;
+  const int64_t beg = live ? rowptr[r] : 0, end = live ? rowptr[r + 1] : 0;
+  const __nv_bfloat16* xb = X + cbase;
+  float4 acc[V][2];
+#pragma unroll
+  for (int v = 0; v < V; ++v) acc[v][0] = acc[v][1] = make_float4(0.f, 0.f, 0.f, 0.f);
+  int pc[SL];
+  float pv[SL];
+#pragma unroll
+  for (int s = 0; s < SL; ++s) {
+    const int64_t j = beg + s * G + sub;
+    const bool ok = j < end;
+    pc[s] = ok ? __ldcs(col + j) : 0;
+    pv[s] = (ok && !FACT) ? __ldcs(val + j) : 0.f;
+  }
+  const int deg = (int)(end - beg);
+  const int dmax = __reduce_max_sync(kFull, deg < NB ? deg : NB);
+  auto step = [&](const int (&c)[U], const float (&a)[U], const bool (&ok)[U]) {
+    uint4 x[U][V];
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+#pragma unroll
+      for (int v = 0; v < V; ++v)
+        x[u][v] = (ok[u] && v * G + sub < c8n)
+                      ? RDM_GATHER_LD(reinterpret_cast<const uint4*>(xb + (int64_t)c[u] * ldx) + v * G + sub)
+                      : make_uint4(0u, 0u, 0u, 0u);
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+#pragma unroll
+      for (int v = 0; v < V; ++v) {
+        const uint32_t w4r[4] = {x[u][v].x, x[u][v].y, x[u][v].z, x[u][v].w};
+#pragma unroll
+        for (int h = 0; h < 2; ++h) {
+          float4& A = acc[v][h];
+          if constexpr (FACT) {
+            acc_bf16_lo(A.x, w4r[2 * h]);
+            acc_bf16_hi(A.y, w4r[2 * h]);
+            acc_bf16_lo(A.z, w4r[2 * h + 1]);
+            acc_bf16_hi(A.w, w4r[2 * h + 1]);
+          } else {
+            A.x = fmaf(a[u], __uint_as_float(w4r[2 * h] << 16), A.x);
+            A.y = fmaf(a[u], __uint_as_float(w4r[2 * h] & 0xFFFF0000u), A.y);
+            A.z = fmaf(a[u], __uint_as_float(w4r[2 * h + 1] << 16), A.z);
+            A.w = fmaf(a[u], __uint_as_float(w4r[2 * h + 1] & 0xFFFF0000u), A.w);
+          }
+        }
+      }
+  };
+#pragma unroll
+  for (int e0 = 0; e0 < NB; e0 += U) {
+    if (e0 >= dmax) break;   // warp-uniform
+    int c[U];
+    float a[U];
+    bool ok[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const int e = e0 + u;
+      c[u] = __shfl_sync(kFull, pc[e / G], g * G + (e % G));
+      a[u] = FACT ? 1.f : __shfl_sync(kFull, pv[e / G], g * G + (e % G));
+      ok[u] = e < deg;
+    }
+    step(c, a, ok);
+  }
+  for (int64_t j = beg + NB; j < end; j += U) {   // rows above the batch (RDM_SPMM_SHORT > 32)
+    int c[U];
+    float a[U];
+    bool ok[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      ok[u] = j + u < end;
+      c[u] = ok[u] ? __ldcs(col + j + u) : 0;
+      a[u] = (ok[u] && !FACT) ? __ldcs(val + j + u) : 0.f;
+    }
+    step(c, a, ok);
+  }
+  if (!live) return;
+  float* dst = out + (int64_t)r * ld_out;
+#pragma unroll
+  for (int v = 0; v < V; ++v) {
+    const int ch = v * G + sub;
+    if (ch < c8n) {
+#pragma unroll
+      for (int h = 0; h < 2; ++h) {
+        const int64_t cc = cbase + 8 * ch + 4 * h;
+        if (cc < w4) {
+          const float4 o = apply_epi(acc[v][h], epi, r, cc);
+          *reinterpret_cast<float4*>(dst + cc) = o;
+          if (epi.scat.P) scatter_row_store(epi.scat, r, cc, o);
+        }
+      }
+    }
+  }
+}
+
 // fp32 slice → bf16 copy (round to nearest even) of X (scale == null) or of
 // s_r·X_r (factored adjacency), row length ldy = w8, zero pads: one thread
 // per 8 columns.
@@ -627,16 +739,33 @@ void launch_spmm_short(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_i
 template <int G, int V, int U, bool FACT = false>
 void launch_spmm_bf(rdm_ctx* ctx, const Csr& A, const __nv_bfloat16* in, int64_t ld_in, float* out,
                     int64_t ld_out, float* part, int64_t ld_part, int64_t w4, int64_t w8, int chunk8,
-                    const Epi& epi) {
-  const int64_t items = A.n_seg + A.n_light;
+                    const Epi& epi, int64_t n_long = -1) {
+  if (n_long < 0) n_long = A.n_light;
+  const int64_t items = A.n_seg + n_long;
   if (items == 0) return;
   const int64_t chunks = ceil_div(w8, 8 * chunk8);
   dim3 grid((unsigned)ceil_div(items, kWarps), (unsigned)chunks);
   spmm_kernel_bf<G, V, U, FACT><<<grid, kWarps * 32, 0, ctx->stream>>>(
       A.rowptr->as<int64_t>(), A.col->as<int32_t>(), A.val->as<float>(),
       A.light_rows->as<int32_t>(), A.seg_start->as<int64_t>(),
-      reinterpret_cast<const int32_t*>(A.seg_start->as<int64_t>() + A.n_seg), A.n_light, A.n_seg,
+      reinterpret_cast<const int32_t*>(A.seg_start->as<int64_t>() + A.n_seg), n_long, A.n_seg,
       in, ld_in, out, ld_out, part, ld_part, w4, w8, chunk8, epi);
+  RDM_LAUNCHED(ctx);
+}
+
+// The short light rows [n_long, n_light) of the bf16 path (2 entries in flight).
+template <int G, int V, bool FACT>
+void launch_spmm_short_bf(rdm_ctx* ctx, const Csr& A, const __nv_bfloat16* in, int64_t ld_in, float* out,
+                          int64_t ld_out, int64_t w4, int64_t w8, int chunk8, const Epi& epi, int64_t n_long,
+                          cudaStream_t st) {
+  const int64_t n_short = A.n_light - n_long;
+  if (n_short <= 0) return;
+  constexpr int R = 32 / G;
+  const int64_t chunks = ceil_div(w8, 8 * chunk8);
+  dim3 grid((unsigned)ceil_div(n_short, (int64_t)kWarps * R), (unsigned)chunks);
+  spmm_short_kernel_bf<G, V, 2, FACT><<<grid, kWarps * 32, 0, st>>>(
+      A.rowptr->as<int64_t>(), A.col->as<int32_t>(), A.val->as<float>(), A.light_rows->as<int32_t>() + n_long,
+      n_short, in, ld_in, out, ld_out, w4, w8, chunk8, epi);
   RDM_LAUNCHED(ctx);
 }
 
@@ -896,16 +1025,58 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
     int U = 1;
     if (!getenv("RDM_SPMM_GV")) pick_gvu(c8, true, &G, &V, &U);
     if (const char* e = getenv("RDM_SPMM_U")) U = atoi(e);
+    // short light rows (degree ≤ 32) on the auxiliary stream, as in the fp32 path
+    // (RDM_SPMM_SHORT_BF=0: warp-per-row for every light row)
+    const char* sbf = getenv("RDM_SPMM_SHORT_BF");
+    int64_t n_long = A.n_light;
+    bool fork = false;
+    if (!(sbf && !atoi(sbf))) {
+      int sg, sv;
+      pick_gv(c8, &sg, &sv);
+      const int64_t nl = A.deg_ge[33 <= Csr::kDegTab ? 33 : Csr::kDegTab];
+      if (A.n_light > nl) {
+        if (!ctx->aux) {
+          int lo = 0, hi = 0;
+          RDM_CUDA(cudaDeviceGetStreamPriorityRange(&lo, &hi));
+          RDM_CUDA(cudaStreamCreateWithPriority(&ctx->aux, cudaStreamNonBlocking, lo));
+          RDM_CUDA(cudaEventCreateWithFlags(&ctx->aux_fork, cudaEventDisableTiming));
+          RDM_CUDA(cudaEventCreateWithFlags(&ctx->aux_join, cudaEventDisableTiming));
+        }
+        RDM_CUDA(cudaEventRecord(ctx->aux_fork, ctx->stream));
+        RDM_CUDA(cudaStreamWaitEvent(ctx->aux, ctx->aux_fork, 0));
+        bool done = true;
+#define RDM_SHORT_BF_CASE(g_, v_)                                                                       \
+  if (sg == g_ && sv == v_) {                                                                           \
+    if (fact) launch_spmm_short_bf<g_, v_, true>(ctx, A, inb, w8, out, ld_out, w4, w8, chunk8, epi, nl, ctx->aux); \
+    else launch_spmm_short_bf<g_, v_, false>(ctx, A, inb, w8, out, ld_out, w4, w8, chunk8, epi, nl, ctx->aux);     \
+  } else
+        RDM_SHORT_BF_CASE(1, 1) RDM_SHORT_BF_CASE(2, 1) RDM_SHORT_BF_CASE(2, 2) RDM_SHORT_BF_CASE(2, 3)
+        RDM_SHORT_BF_CASE(4, 1) RDM_SHORT_BF_CASE(4, 2) RDM_SHORT_BF_CASE(4, 3) RDM_SHORT_BF_CASE(4, 4)
+        RDM_SHORT_BF_CASE(8, 1) RDM_SHORT_BF_CASE(8, 2) RDM_SHORT_BF_CASE(8, 3) RDM_SHORT_BF_CASE(8, 4)
+        RDM_SHORT_BF_CASE(16, 1) RDM_SHORT_BF_CASE(16, 2) RDM_SHORT_BF_CASE(16, 3) RDM_SHORT_BF_CASE(16, 4)
+        RDM_SHORT_BF_CASE(32, 1) { done = false; }
+#undef RDM_SHORT_BF_CASE
+        if (done) {
+          n_long = nl;
+          fork = true;
+        }
+        RDM_CUDA(cudaEventRecord(ctx->aux_join, ctx->aux));
+        if (!done) RDM_CUDA(cudaStreamWaitEvent(ctx->stream, ctx->aux_join, 0));
+      }
+    }
+    auto join = [&]() {
+      if (fork) RDM_CUDA(cudaStreamWaitEvent(ctx->stream, ctx->aux_join, 0));
+    };
     if (fact) {   // value-free sums of bf16(s_j X_j) for the measured mappings
 #define RDM_SPMM_FCASE(g_, v_, u_) \
-  if (G == g_ && V == v_ && U == u_) { launch_spmm_bf<g_, v_, u_, true>(ctx, A, inb, w8, out, ld_out, part, ldp, w4, w8, chunk8, epi); fact = false; goto heavy; }
+  if (G == g_ && V == v_ && U == u_) { launch_spmm_bf<g_, v_, u_, true>(ctx, A, inb, w8, out, ld_out, part, ldp, w4, w8, chunk8, epi, n_long); join(); fact = false; goto heavy; }
       RDM_SPMM_FCASE(8, 1, 4) RDM_SPMM_FCASE(8, 2, 2) RDM_SPMM_FCASE(16, 2, 2) RDM_SPMM_FCASE(2, 1, 2)
       RDM_SPMM_FCASE(1, 2, 1) RDM_SPMM_FCASE(1, 1, 1) RDM_SPMM_FCASE(4, 1, 2) RDM_SPMM_FCASE(32, 1, 2)
 #undef RDM_SPMM_FCASE
       throw Error(RDM_ERR_STATE, "spmm: no factored bf16 kernel for G/V/U");
     }
 #define RDM_SPMM_CASE(g_, v_, u_) \
-  if (G == g_ && V == v_ && U == u_) launch_spmm_bf<g_, v_, u_>(ctx, A, inb, w8, out, ld_out, part, ldp, w4, w8, chunk8, epi); else
+  if (G == g_ && V == v_ && U == u_) launch_spmm_bf<g_, v_, u_>(ctx, A, inb, w8, out, ld_out, part, ldp, w4, w8, chunk8, epi, n_long); else
     RDM_SPMM_CASE(1, 1, 1) RDM_SPMM_CASE(1, 2, 1) RDM_SPMM_CASE(1, 3, 1) RDM_SPMM_CASE(1, 4, 1)
     RDM_SPMM_CASE(2, 1, 1) RDM_SPMM_CASE(2, 1, 2) RDM_SPMM_CASE(2, 2, 1) RDM_SPMM_CASE(2, 2, 2)
     RDM_SPMM_CASE(2, 3, 1) RDM_SPMM_CASE(2, 3, 2) RDM_SPMM_CASE(2, 4, 1) RDM_SPMM_CASE(2, 4, 2)
@@ -920,6 +1091,7 @@ void run_csr(rdm_ctx* ctx, const Csr& A, const float* in, int64_t ld_in, float* 
     RDM_SPMM_CASE(32, 1, 4)
     throw Error(RDM_ERR_ARG, "spmm: no bf16 kernel for G/V/U");
 #undef RDM_SPMM_CASE
+    join();
   } else {
     const int c4 = (int)std::min<int64_t>(chunk4, w4 / 4);
     int U = 1;
